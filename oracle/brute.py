@@ -1,0 +1,181 @@
+"""Independent big-int / Fraction brute force of the Sieve back-end -- TEST INFRASTRUCTURE ONLY.
+
+A second, deliberately naive implementation of SURVEY.md 8(c), written from
+the paper's definitions without looking at oracle/sieve_oracle.c's structure:
+
+* moments and every comparison with Python integers (no overflow possible);
+* CoV < theta as the exact rational comparison sigma^2 < theta^2 mu^2 with Fractions;
+* fma emulated exactly: float(Fraction(a) * Fraction(b) + Fraction(c)) is correctly rounded
+  (Python's int/int true division rounds to nearest-even), since Python 3.12 has no math.fma;
+* the prediction C_pred = sum_s W_s y_rep / x_rep evaluated exactly as a Fraction.
+
+Only for tiny traces (a few hundred invocations, small G).
+"""
+import math
+from fractions import Fraction
+
+LOG2E = 1.4426950408889634074
+LN2_HI = 6.93147180369123816490e-01
+LN2_LO = 1.90821492927058770002e-10
+TWO52 = 2.0 ** 52
+
+
+def fma(a, b, c):
+    return float(Fraction(a) * Fraction(b) + Fraction(c))
+
+
+def inv_fact(i):
+    return float(Fraction(1, math.factorial(i)))
+
+
+def det_exp(t):
+    k = float(round(t * LOG2E))          # Python round() on floats is round-half-even == rint
+    r = fma(-k, LN2_HI, t)
+    r = fma(-k, LN2_LO, r)
+    p = inv_fact(13)
+    for i in range(12, -1, -1):
+        p = fma(p, -r, inv_fact(i))
+    return math.ldexp(p, -int(k))
+
+
+def q_term(g, x, inv_h):
+    z = (g - float(x)) * inv_h
+    t = (z * z) * 0.5
+    if t > 37.0:
+        return 0
+    return int(round(det_exp(t) * TWO52))
+
+
+def cov_below(vals, theta):
+    """population CoV < theta, exactly (sigma = sqrt of the mean squared deviation)"""
+    n = len(vals)
+    mu = Fraction(sum(vals), n)
+    var = sum((Fraction(v) - mu) ** 2 for v in vals) / n
+    return var < theta * theta * mu * mu
+
+
+def bandwidth(vals, bw_scale):
+    n = len(vals)
+    s1 = sum(vals)
+    s2 = sum(v * v for v in vals)
+    num = n * s2 - s1 * s1                # exact integer
+    var = float(num) / (float(n) * float(n))   # float(int) is correctly rounded
+    h_raw = (bw_scale * math.sqrt(var)) * math.pow(float(n), -0.2)
+    e = math.frexp(h_raw)[1] - 1 - 15    # ilogb(h_raw) - 15
+    return math.ldexp(float(round(math.ldexp(h_raw, -e))), e)
+
+
+def grid(lo, hi, G):
+    return [float(lo) + float((hi - lo) * j) / float(G - 1) for j in range(G)]
+
+
+def kde(vals, lo, hi, h, G):
+    inv_h = 1.0 / h
+    return [sum(q_term(g, x, inv_h) for x in vals) for g in grid(lo, hi, G)]
+
+
+def valley_cuts(D, shift):
+    """indices m of the valleys: hysteresis delta = max(1, max D >> shift), run midpoints"""
+    delta = max(1, max(D) >> shift)
+    cuts = []
+    mode = "up"
+    top = D[0]
+    for j in range(1, len(D)):
+        d = D[j]
+        if mode == "up":
+            top = max(top, d)
+            if d + delta <= top:
+                mode, low, a, b = "down", d, j, j
+        else:
+            if d < low:
+                low, a, b = d, j, j
+            elif d == low and b == j - 1:
+                b = j
+            elif d >= low + delta:
+                cuts.append((a + b) // 2)
+                mode, top = "up", d
+    return cuts
+
+
+def stratify(kid, x, K, cta=None, cycles=None, theta=Fraction(2, 5), G=64, shift=10,
+             bw_scale=1.06, max_rounds=64):
+    n = len(kid)
+    kid = [int(k) for k in kid]
+    x = [int(v) for v in x]
+    cta = [0] * n if cta is None else [int(c) for c in cta]
+    strata = []  # dicts
+    for k in range(K):
+        rows = [i for i in range(n) if kid[i] == k]
+        if not rows:
+            continue
+        vals = [x[i] for i in rows]
+        if min(vals) == max(vals):
+            strata.append(dict(kid=k, tier=1, lo=min(vals), hi=max(vals), h=0.0, rnd=0))
+            continue
+        if cov_below(vals, theta):
+            strata.append(dict(kid=k, tier=2, lo=min(vals), hi=max(vals), h=0.0, rnd=0))
+            continue
+        open_ = [vals]
+        rnd = 0
+        while open_:
+            rnd += 1
+            if rnd > max_rounds:
+                raise RuntimeError("ELIMIT")
+            nxt = []
+            for seg in open_:
+                lo, hi = min(seg), max(seg)
+                h = bandwidth(seg, bw_scale)
+                D = kde(seg, lo, hi, h, G)
+                gs = grid(lo, hi, G)
+                T = sorted({math.ceil(gs[m]) for m in valley_cuts(D, shift)})
+                T = [t for t in T if lo < t <= hi]
+                if not T:
+                    T = [(lo + hi + 1) // 2]
+                bounds = [0] + T + [1 << 64]
+                for a, b in zip(bounds[:-1], bounds[1:]):
+                    part = [v for v in seg if a <= v < b]
+                    if not part:
+                        continue
+                    if min(part) == max(part) or cov_below(part, theta):
+                        strata.append(dict(kid=k, tier=3, lo=min(part), hi=max(part), h=h, rnd=rnd))
+                    else:
+                        nxt.append(part)
+            open_ = nxt
+    strata.sort(key=lambda s: (s["kid"], s["lo"]))
+    sid = [None] * n
+    for s_i, s in enumerate(strata):
+        for i in range(n):
+            if kid[i] == s["kid"] and s["lo"] <= x[i] <= s["hi"]:
+                sid[i] = s_i
+    for s_i, s in enumerate(strata):
+        mem = [i for i in range(n) if sid[i] == s_i]
+        s["count"] = len(mem)
+        s["W"] = sum(x[i] for i in mem)
+        if s["tier"] == 1:
+            rep = min(mem)
+        else:
+            by_cta = {}
+            for i in mem:
+                by_cta.setdefault(cta[i], []).append(i)
+            best = max(by_cta.values(), key=lambda l: (len(l), -min(l)))
+            rep = min(best)
+        s["rep"] = rep
+        s["rep_instr"] = x[rep]
+        s["rep_cycles"] = None if cycles is None else int(cycles[rep])
+        s["rep_cta"] = cta[rep]
+    return strata, sid
+
+
+def predict(strata, cycles=None, rep_cycles=None):
+    """C_pred exactly; IPC = 1 / sum_s w_s / IPC_s; error; speedup"""
+    I = sum(s["W"] for s in strata)
+    ys = rep_cycles if rep_cycles is not None else [s["rep_cycles"] for s in strata]
+    c_pred = sum(Fraction(s["W"] * y, s["rep_instr"]) for s, y in zip(strata, ys))
+    out = {"predicted_cycles_exact": c_pred, "predicted_cycles": float(c_pred),
+           "predicted_ipc": float(Fraction(I) / c_pred) if c_pred else math.inf}
+    if cycles is not None:
+        cm = sum(int(c) for c in cycles)
+        out["measured_cycles"] = float(cm)
+        out["error"] = float(abs(c_pred - cm) / cm) if cm else math.nan
+        out["speedup"] = float(Fraction(cm, sum(ys)))
+    return out

@@ -1,0 +1,641 @@
+/*
+ * oracle/sieve_oracle.c -- plain, slow, single-threaded CPU oracle for the Sieve
+ * stratification back-end (Naderan-Tahan, SeyyedAghaei, Eeckhout, ISPASS'23).
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load this library.  It shares no code,
+ * header, table or constant with the CUDA product path (paper_conf_ispass_naderantahanse23_b200/),
+ * and neither side includes the other.
+ *
+ * Citation form: P:NN = /root/reference/PAPER.md line NN.  Readings A1..A24 and the
+ * step names O1..O9 are those of SURVEY.md section 8(c), restated in DESIGN.md section 3.
+ *
+ * Every function below is written in the order of the paper / the 8(c) reading, with
+ * no blocking, fusion or reordering:
+ *   O1 group invocations by kernel
+ *   O2 exact moments n, S1, S2, lo, hi (u128)
+ *   O3 tier: Tier-1 iff lo==hi, Tier-2 iff CoV < theta    P:75-85 (A1-A5)
+ *   O4 Tier-1/2: one stratum per kernel
+ *   O5 Tier-3 refinement: Gaussian KDE on a grid, valleys, split until CoV < theta
+ *                                                         P:89, [8] P:317, [36] P:349 (A6-A15)
+ *   O6 stratum numbering by (kernel, lo)                  A23
+ *   O7 representative: first-chronological (Tier-1) / first-chronological with the most
+ *      dominant CTA size (Tier-2/3)                       P:93, P:103 (A16-A19)
+ *   O8 weights W_s = sum of instruction counts
+ *   O9 prediction: weighted harmonic-mean IPC, C_pred = I / IPC, error, speedup
+ *                                                         P:99-101, P:200-208 (A22)
+ *
+ * Pins (tests/test_oracle_*.py): tier closed forms and exact-boundary multisets, big-int
+ * moments, det_exp vs libm exp (<= 1 ulp), KDE vs scikit-learn / scipy / direct sums,
+ * hand-built valley sequences, symmetric two-point masses, strata invariants,
+ * representative brute force, prediction identities (homogeneous cycles => error 0,
+ * CPI arithmetic-mean form), and an independent Python big-int brute force (oracle/brute.py).
+ *
+ * Build: gcc -O2 -std=c11 -ffp-contract=off -fPIC -shared (no -ffast-math: every
+ * floating-point step must be the IEEE basic operation written here).
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+typedef unsigned __int128 u128;
+
+/* ------------------------------------------------------------------------------------------
+ * Status codes (the oracle's own; same numeric meaning as the product's API, re-declared)
+ * ------------------------------------------------------------------------------------------ */
+#define OR_OK 0
+#define OR_EINVAL (-1)
+#define OR_ERANGE (-2)
+#define OR_ENOMEM (-3)
+#define OR_EDOM (-6)
+#define OR_ELIMIT (-7)
+
+/* ------------------------------------------------------------------------------------------
+ * 256-bit unsigned integers (little-endian 64-bit limbs) for the exact CoV comparison (A5).
+ * ------------------------------------------------------------------------------------------ */
+typedef struct { uint64_t w[4]; } u256;
+
+static u256 u256_from128(u128 a) {
+  u256 r = {{(uint64_t)a, (uint64_t)(a >> 64), 0, 0}};
+  return r;
+}
+
+/* schoolbook product of two values that each fit in 128 bits; the result fits in 256 */
+static u256 u256_mul128(u128 a, u128 b) {
+  uint64_t x[2] = {(uint64_t)a, (uint64_t)(a >> 64)};
+  uint64_t y[2] = {(uint64_t)b, (uint64_t)(b >> 64)};
+  uint64_t r[4] = {0, 0, 0, 0};
+  for (int i = 0; i < 2; i++) {
+    u128 carry = 0;
+    for (int j = 0; j < 2; j++) {
+      u128 t = (u128)x[i] * y[j] + r[i + j] + carry;
+      r[i + j] = (uint64_t)t;
+      carry = t >> 64;
+    }
+    int k = i + 2;
+    while (carry) {
+      u128 t = (u128)r[k] + carry;
+      r[k] = (uint64_t)t;
+      carry = t >> 64;
+      k++;
+    }
+  }
+  u256 out = {{r[0], r[1], r[2], r[3]}};
+  return out;
+}
+
+/* (a * small) where a < 2^256 / small; used for q^2 * (...) and p^2 * (...) */
+static u256 u256_mul_u64(u256 a, uint64_t m) {
+  u256 r;
+  u128 carry = 0;
+  for (int i = 0; i < 4; i++) {
+    u128 t = (u128)a.w[i] * m + carry;
+    r.w[i] = (uint64_t)t;
+    carry = t >> 64;
+  }
+  return r;
+}
+
+static u256 u256_sub(u256 a, u256 b) { /* requires a >= b */
+  u256 r;
+  uint64_t borrow = 0;
+  for (int i = 0; i < 4; i++) {
+    uint64_t bi = b.w[i] + borrow;
+    uint64_t nb = (bi < borrow) || (a.w[i] < bi);
+    r.w[i] = a.w[i] - bi;
+    borrow = nb;
+  }
+  return r;
+}
+
+static int u256_cmp(u256 a, u256 b) {
+  for (int i = 3; i >= 0; i--) {
+    if (a.w[i] < b.w[i]) return -1;
+    if (a.w[i] > b.w[i]) return 1;
+  }
+  return 0;
+}
+
+/* correctly rounded (round-to-nearest-even) conversion of a 256-bit integer to double */
+static double u256_to_double(u256 a) {
+  if (a.w[3] == 0 && a.w[2] == 0) {
+    u128 v = ((u128)a.w[1] << 64) | a.w[0];
+    return (double)v; /* libgcc __floatuntidf: correctly rounded */
+  }
+  int top = a.w[3] ? 3 : 2;
+  int bits = 64 * top + (64 - __builtin_clzll(a.w[top]));
+  int s = bits - 64; /* keep the top 64 bits, OR the rest into a sticky LSB */
+  uint64_t t = 0, sticky = 0;
+  for (int b = 0; b < 64; b++) {
+    int src = s + b;
+    if ((a.w[src / 64] >> (src % 64)) & 1u) t |= (uint64_t)1 << b;
+  }
+  for (int b = 0; b < s; b++)
+    if ((a.w[b / 64] >> (b % 64)) & 1u) { sticky = 1; break; }
+  return ldexp((double)(t | sticky), s); /* >= 11 dropped bits, so the sticky LSB is exact */
+}
+
+/* ------------------------------------------------------------------------------------------
+ * O3 tier rule.  CoV = sigma/mu with population sigma (A1: "the average
+ * squared differences with the mean").  CoV < p/q  <=>  q^2 (n S2 - S1^2) < p^2 S1^2 (A3, A5).
+ * Tier-1 iff lo == hi (A4).  CoV exactly theta is Tier-3 (A2, "otherwise").
+ * ------------------------------------------------------------------------------------------ */
+static int cov_below(uint64_t n, u128 S1, u128 S2, uint32_t p, uint32_t q) {
+  u256 nS2 = u256_mul128((u128)n, S2);
+  u256 S1sq = u256_mul128(S1, S1);
+  u256 diff = u256_sub(nS2, S1sq); /* n S2 - S1^2 >= 0 by Cauchy-Schwarz */
+  u256 lhs = u256_mul_u64(diff, (uint64_t)q * q);
+  u256 rhs = u256_mul_u64(S1sq, (uint64_t)p * p);
+  return u256_cmp(lhs, rhs) < 0;
+}
+
+int oracle_tier(uint64_t n, uint64_t s1_lo, uint64_t s1_hi, uint64_t s2_lo, uint64_t s2_hi,
+                uint64_t lo, uint64_t hi, uint32_t p, uint32_t q) {
+  u128 S1 = ((u128)s1_hi << 64) | s1_lo, S2 = ((u128)s2_hi << 64) | s2_lo;
+  if (lo == hi) return 1;
+  return cov_below(n, S1, S2, p, q) ? 2 : 3;
+}
+
+/* ------------------------------------------------------------------------------------------
+ * O5a bandwidth: Scott's normal-reference rule [36] P:349 (A8):
+ *   var = rn(n S2 - S1^2) / (rn(n) * rn(n)),  sigma = sqrt(var),
+ *   h_raw = (bw_scale * sigma) * pow(n, -0.2),  h = h_raw rounded to 16 significant bits.
+ * ------------------------------------------------------------------------------------------ */
+double oracle_bandwidth(uint64_t n, uint64_t s1_lo, uint64_t s1_hi, uint64_t s2_lo,
+                        uint64_t s2_hi, double bw_scale) {
+  u128 S1 = ((u128)s1_hi << 64) | s1_lo, S2 = ((u128)s2_hi << 64) | s2_lo;
+  u256 diff = u256_sub(u256_mul128((u128)n, S2), u256_mul128(S1, S1));
+  double dn = (double)n;
+  double var = u256_to_double(diff) / (dn * dn);
+  double sigma = sqrt(var);
+  double h_raw = (bw_scale * sigma) * pow(dn, -0.2);
+  int e = ilogb(h_raw) - 15;
+  return ldexp(rint(ldexp(h_raw, -e)), e);
+}
+
+/* O5b grid point j on [lo, hi] inclusive (A9): g_j = rn(lo) + rn((hi-lo)*j) / rn(G-1) */
+static double grid_point(uint64_t lo, uint64_t hi, uint32_t j, uint32_t G) {
+  double a = (double)lo;
+  double b = (double)((hi - lo) * (uint64_t)j);
+  double c = (double)(G - 1);
+  return a + b / c;
+}
+
+double oracle_grid_point(uint64_t lo, uint64_t hi, uint32_t j, uint32_t G) {
+  return grid_point(lo, hi, j, G);
+}
+
+/* ------------------------------------------------------------------------------------------
+ * O5c det_exp(t) = e^{-t} for t in [0, 37] (A10), built only from IEEE basic operations:
+ *   k = rint(t * LOG2E); r = fma(-k, LN2_HI, t); r = fma(-k, LN2_LO, r);
+ *   P(r) = sum_{i=0}^{13} (-r)^i / i!  by Horner with fma, starting from 1/13!;
+ *   det_exp = ldexp(P, -k).
+ * ------------------------------------------------------------------------------------------ */
+static const double OR_LOG2E = 1.4426950408889634074;
+static const double OR_LN2_HI = 6.93147180369123816490e-01;
+static const double OR_LN2_LO = 1.90821492927058770002e-10;
+static const double OR_INV_FACT[14] = {
+    1.0,         1.0,          1.0 / 2.0,          1.0 / 6.0,          1.0 / 24.0,
+    1.0 / 120.0, 1.0 / 720.0,  1.0 / 5040.0,       1.0 / 40320.0,      1.0 / 362880.0,
+    1.0 / 3628800.0, 1.0 / 39916800.0, 1.0 / 479001600.0, 1.0 / 6227020800.0};
+
+double oracle_det_exp(double t) {
+  double k = rint(t * OR_LOG2E);
+  double r = fma(-k, OR_LN2_HI, t);
+  r = fma(-k, OR_LN2_LO, r);
+  double mr = -r;
+  double p = OR_INV_FACT[13];
+  for (int i = 12; i >= 0; i--) p = fma(p, mr, OR_INV_FACT[i]);
+  return ldexp(p, -(int)k);
+}
+
+/* fixed-point kernel value Q(x, g) = rint(det_exp(t) * 2^52), 0 if t > 37 (A10) */
+static uint64_t kernel_q(double g, double xd, double inv_h) {
+  double z = (g - xd) * inv_h;
+  double t = (z * z) * 0.5;
+  if (t > 37.0) return 0;
+  return (uint64_t)rint(oracle_det_exp(t) * 4503599627370496.0 /* 2^52 */);
+}
+
+uint64_t oracle_q(double t) {
+  if (t > 37.0) return 0;
+  return (uint64_t)rint(oracle_det_exp(t) * 4503599627370496.0);
+}
+
+/* O5c density on the grid: D_j = sum over the segment's values of Q(x, g_j), u128 */
+static void kde_grid(const uint64_t* v, uint64_t m, uint64_t lo, uint64_t hi, double h,
+                     uint32_t G, u128* D) {
+  double inv_h = 1.0 / h;
+  for (uint32_t j = 0; j < G; j++) {
+    double g = grid_point(lo, hi, j, G);
+    u128 acc = 0;
+    for (uint64_t i = 0; i < m; i++) acc += kernel_q(g, (double)v[i], inv_h);
+    D[j] = acc;
+  }
+}
+
+void oracle_kde(const uint64_t* v, uint64_t m, uint64_t lo, uint64_t hi, double h, uint32_t G,
+                uint64_t* d_lo, uint64_t* d_hi) {
+  u128* D = (u128*)malloc(sizeof(u128) * G);
+  kde_grid(v, m, lo, hi, h, G, D);
+  for (uint32_t j = 0; j < G; j++) { d_lo[j] = (uint64_t)D[j]; d_hi[j] = (uint64_t)(D[j] >> 64); }
+  free(D);
+}
+
+/* ------------------------------------------------------------------------------------------
+ * O5d valleys (A11): hysteresis two-state scan with delta = max(1, Dmax >> shift); a cut at
+ * the midpoint of the minimum's run; the edges are never valleys.  Returns #cut indices.
+ * ------------------------------------------------------------------------------------------ */
+static uint32_t valleys(const u128* D, uint32_t G, uint32_t shift, uint32_t* cut_idx) {
+  u128 dmax = 0;
+  for (uint32_t j = 0; j < G; j++) if (D[j] > dmax) dmax = D[j];
+  u128 delta = dmax >> shift;
+  if (delta < 1) delta = 1;
+  int seek_min = 0;
+  u128 mx = D[0], mn = 0;
+  uint32_t a = 0, b = 0, nc = 0;
+  for (uint32_t j = 1; j < G; j++) {
+    u128 d = D[j];
+    if (!seek_min) {
+      if (d > mx) mx = d;
+      if (d + delta <= mx) { seek_min = 1; mn = d; a = b = j; }
+    } else {
+      if (d < mn) { mn = d; a = b = j; }
+      else if (d == mn && b == j - 1) { b = j; }
+      else if (d >= mn + delta) { cut_idx[nc++] = (a + b) / 2; seek_min = 0; mx = d; }
+    }
+  }
+  return nc;
+}
+
+uint32_t oracle_valleys(const uint64_t* d_lo, const uint64_t* d_hi, uint32_t G, uint32_t shift,
+                        uint32_t* cut_idx) {
+  u128* D = (u128*)malloc(sizeof(u128) * G);
+  for (uint32_t j = 0; j < G; j++) D[j] = ((u128)d_hi[j] << 64) | d_lo[j];
+  uint32_t nc = valleys(D, G, shift, cut_idx);
+  free(D);
+  return nc;
+}
+
+/* ------------------------------------------------------------------------------------------
+ * Result object
+ * ------------------------------------------------------------------------------------------ */
+typedef struct {
+  uint32_t kernel_id, tier, index_in_kernel, rep_cta;
+  uint64_t lo, hi, count, instr_sum_lo, instr_sum_hi;
+  uint64_t rep_id, rep_instr, rep_cycles;
+  double bandwidth;
+  uint32_t split_round, pad;
+} oracle_stratum;
+
+typedef struct {
+  uint32_t kernel_id, round, split_kind, n_cuts;
+  uint64_t lo, hi, count;
+  double bandwidth;
+  uint64_t *d_lo, *d_hi, *cuts;
+} oracle_segment;
+
+typedef struct {
+  double predicted_cycles, predicted_ipc, measured_cycles, error, speedup;
+  uint64_t total_instr_lo, total_instr_hi;
+} oracle_prediction;
+
+typedef struct {
+  uint64_t n;
+  uint32_t G;
+  oracle_stratum* strata;
+  uint64_t n_strata;
+  uint32_t* sid; /* per input row */
+  oracle_segment* segs;
+  uint64_t n_segs, cap_segs;
+  int has_cycles;
+  u128 c_meas;
+  u128 total_instr;
+  uint32_t rounds;
+  uint64_t kde_terms_nonzero;
+} oracle_result;
+
+/* a candidate part / open segment of one Tier-3 kernel */
+typedef struct {
+  uint32_t kid;
+  uint64_t* v; /* its instruction counts (owned) */
+  uint64_t n;
+  u128 S1, S2;
+  uint64_t lo, hi;
+  double h_from; /* bandwidth of the segment whose split created it */
+  uint32_t round_from;
+} part_t;
+
+static void moments(const uint64_t* v, uint64_t m, u128* S1, u128* S2, uint64_t* lo,
+                    uint64_t* hi) {
+  u128 s1 = 0, s2 = 0;
+  uint64_t l = UINT64_MAX, h = 0;
+  for (uint64_t i = 0; i < m; i++) {
+    s1 += v[i];
+    s2 += (u128)v[i] * v[i];
+    if (v[i] < l) l = v[i];
+    if (v[i] > h) h = v[i];
+  }
+  *S1 = s1; *S2 = s2; *lo = l; *hi = h;
+}
+
+typedef struct { uint32_t kid; uint64_t lo, hi, n; u128 S1; uint32_t tier; double h; uint32_t round; } fin_t;
+
+static int push_seg(oracle_result* R, oracle_segment s) {
+  if (R->n_segs == R->cap_segs) {
+    uint64_t nc = R->cap_segs ? 2 * R->cap_segs : 64;
+    oracle_segment* ns = (oracle_segment*)realloc(R->segs, nc * sizeof(oracle_segment));
+    if (!ns) return OR_ENOMEM;
+    R->segs = ns; R->cap_segs = nc;
+  }
+  R->segs[R->n_segs++] = s;
+  return OR_OK;
+}
+
+static int cmp_fin(const void* a, const void* b) {
+  const fin_t* x = (const fin_t*)a; const fin_t* y = (const fin_t*)b;
+  if (x->kid != y->kid) return x->kid < y->kid ? -1 : 1;
+  if (x->lo != y->lo) return x->lo < y->lo ? -1 : 1;
+  return 0;
+}
+
+void oracle_free(oracle_result* R) {
+  if (!R) return;
+  for (uint64_t i = 0; i < R->n_segs; i++) {
+    free(R->segs[i].d_lo); free(R->segs[i].d_hi); free(R->segs[i].cuts);
+  }
+  free(R->segs); free(R->strata); free(R->sid); free(R);
+}
+
+/* ------------------------------------------------------------------------------------------
+ * The whole back-end, O1..O8.
+ * ids: global invocation id per row (nullable: row index), used for "first-chronological"
+ * (A18) so that a subset of kernels can be stratified with their original ids.
+ * ------------------------------------------------------------------------------------------ */
+int oracle_stratify(uint64_t n, uint32_t K, const uint32_t* kid, const uint64_t* x,
+                    const uint32_t* cta, const uint64_t* cycles, const uint64_t* ids,
+                    uint32_t theta_num, uint32_t theta_den, uint32_t G, uint32_t valley_shift,
+                    uint32_t max_rounds, double bw_scale, int keep_debug, oracle_result** out) {
+  *out = NULL;
+  if (theta_num == 0 || theta_den == 0 || G < 3 || G > 65536 || K == 0 || valley_shift > 120)
+    return OR_EINVAL;
+  for (uint64_t i = 0; i < n; i++) {
+    if (kid[i] >= K) return OR_EINVAL;
+    if (x[i] == 0 || x[i] >= ((uint64_t)1 << 44)) return OR_ERANGE; /* A21 */
+  }
+  oracle_result* R = (oracle_result*)calloc(1, sizeof(oracle_result));
+  if (!R) return OR_ENOMEM;
+  R->n = n; R->G = G; R->has_cycles = cycles != NULL;
+  R->sid = (uint32_t*)malloc(sizeof(uint32_t) * (n ? n : 1));
+
+  /* O1 group by kernel id (counting sort, stable in row order) */
+  uint64_t* cnt = (uint64_t*)calloc(K + 1, sizeof(uint64_t));
+  for (uint64_t i = 0; i < n; i++) cnt[kid[i] + 1]++;
+  for (uint32_t k = 0; k < K; k++) cnt[k + 1] += cnt[k];
+  uint64_t* rows = (uint64_t*)malloc(sizeof(uint64_t) * (n ? n : 1));
+  uint64_t* pos = (uint64_t*)malloc(sizeof(uint64_t) * (K + 1));
+  memcpy(pos, cnt, sizeof(uint64_t) * (K + 1));
+  for (uint64_t i = 0; i < n; i++) rows[pos[kid[i]]++] = i;
+  free(pos);
+
+  fin_t* fin = NULL;
+  uint64_t n_fin = 0, cap_fin = 0;
+#define PUSH_FIN(F) do { if (n_fin == cap_fin) { cap_fin = cap_fin ? 2 * cap_fin : 256; \
+      fin = (fin_t*)realloc(fin, cap_fin * sizeof(fin_t)); } fin[n_fin++] = (F); } while (0)
+
+  int status = OR_OK;
+  uint32_t max_round_seen = 0;
+  u128* D = (u128*)malloc(sizeof(u128) * G);
+  uint32_t* cut_idx = (uint32_t*)malloc(sizeof(uint32_t) * G);
+  uint64_t* T = (uint64_t*)malloc(sizeof(uint64_t) * (G + 1));
+
+  for (uint32_t k = 0; k < K && status == OR_OK; k++) {
+    uint64_t m = cnt[k + 1] - cnt[k];
+    if (m == 0) continue;
+    uint64_t* v = (uint64_t*)malloc(sizeof(uint64_t) * m);
+    for (uint64_t j = 0; j < m; j++) v[j] = x[rows[cnt[k] + j]];
+    /* O2 exact moments */
+    u128 S1, S2; uint64_t lo, hi;
+    moments(v, m, &S1, &S2, &lo, &hi);
+    R->total_instr += S1;
+    /* O3 tier */
+    uint32_t tier = lo == hi ? 1 : (cov_below(m, S1, S2, theta_num, theta_den) ? 2 : 3);
+    if (tier != 3) { /* O4 */
+      fin_t f = {k, lo, hi, m, S1, tier, 0.0, 0};
+      PUSH_FIN(f);
+      free(v);
+      continue;
+    }
+    /* O5 Tier-3 refinement: open <- [(k, all invocations of k)] */
+    part_t* open = (part_t*)malloc(sizeof(part_t));
+    uint64_t n_open = 1;
+    open[0].kid = k; open[0].v = v; open[0].n = m; open[0].S1 = S1; open[0].S2 = S2;
+    open[0].lo = lo; open[0].hi = hi;
+    uint32_t round = 0;
+    while (n_open > 0) {
+      round++;
+      if (round > max_rounds) { status = OR_ELIMIT; break; }
+      if (round > max_round_seen) max_round_seen = round;
+      part_t* next = NULL;
+      uint64_t n_next = 0, cap_next = 0;
+      for (uint64_t s = 0; s < n_open; s++) { /* open segments in (k, lo) order */
+        part_t* P = &open[s];
+        /* a. bandwidth */
+        double h = oracle_bandwidth(P->n, (uint64_t)P->S1, (uint64_t)(P->S1 >> 64),
+                                    (uint64_t)P->S2, (uint64_t)(P->S2 >> 64), bw_scale);
+        /* b, c. grid and fixed-point density */
+        kde_grid(P->v, P->n, P->lo, P->hi, h, G, D);
+        /* d. valleys -> thresholds T = ceil(g_m), deduplicated, lo < T <= hi */
+        uint32_t nc = valleys(D, G, valley_shift, cut_idx);
+        uint32_t nt = 0;
+        for (uint32_t c = 0; c < nc; c++) {
+          double gm = grid_point(P->lo, P->hi, cut_idx[c], G);
+          uint64_t t = (uint64_t)ceil(gm);
+          if (t <= P->lo || t > P->hi) continue;
+          if (nt > 0 && T[nt - 1] == t) continue;
+          T[nt++] = t;
+        }
+        uint32_t kind = 1;
+        /* e. fallback: value-range bisection */
+        if (nt == 0) { T[nt++] = (P->lo + P->hi + 1) >> 1; kind = 2; }
+        if (keep_debug) {
+          oracle_segment sg;
+          sg.kernel_id = k; sg.round = round; sg.split_kind = kind; sg.n_cuts = nt;
+          sg.lo = P->lo; sg.hi = P->hi; sg.count = P->n; sg.bandwidth = h;
+          sg.d_lo = (uint64_t*)malloc(8 * G); sg.d_hi = (uint64_t*)malloc(8 * G);
+          sg.cuts = (uint64_t*)malloc(8 * nt);
+          for (uint32_t j = 0; j < G; j++) { sg.d_lo[j] = (uint64_t)D[j]; sg.d_hi[j] = (uint64_t)(D[j] >> 64); }
+          for (uint32_t c = 0; c < nt; c++) sg.cuts[c] = T[c];
+          push_seg(R, sg);
+        }
+        /* f. parts: x < T1 | T1 <= x < T2 | ... ; empty parts dropped */
+        for (uint32_t q = 0; q <= nt; q++) {
+          uint64_t a = q == 0 ? 0 : T[q - 1];
+          uint64_t b = q == nt ? UINT64_MAX : T[q];
+          uint64_t pm = 0;
+          for (uint64_t i = 0; i < P->n; i++) if (P->v[i] >= a && P->v[i] < b) pm++;
+          if (pm == 0) continue;
+          uint64_t* pv = (uint64_t*)malloc(sizeof(uint64_t) * pm);
+          uint64_t w = 0;
+          for (uint64_t i = 0; i < P->n; i++) if (P->v[i] >= a && P->v[i] < b) pv[w++] = P->v[i];
+          part_t np;
+          np.kid = k; np.v = pv; np.n = pm;
+          moments(pv, pm, &np.S1, &np.S2, &np.lo, &np.hi);
+          np.h_from = h; np.round_from = round;
+          if (np.lo == np.hi || cov_below(np.n, np.S1, np.S2, theta_num, theta_den)) {
+            fin_t f = {k, np.lo, np.hi, np.n, np.S1, 3, h, round};
+            PUSH_FIN(f);
+            free(pv);
+          } else {
+            if (n_next == cap_next) { cap_next = cap_next ? 2 * cap_next : 8;
+              next = (part_t*)realloc(next, cap_next * sizeof(part_t)); }
+            next[n_next++] = np;
+          }
+        }
+      }
+      for (uint64_t s = 0; s < n_open; s++) free(open[s].v);
+      free(open);
+      open = next; n_open = n_next;
+      /* next round's open set stays in (k, lo) order: parts were appended by ascending value */
+    }
+    for (uint64_t s = 0; s < n_open; s++) free(open[s].v);
+    free(open);
+  }
+  free(D); free(cut_idx); free(T);
+  R->rounds = max_round_seen;
+  if (status != OR_OK) { free(fin); free(rows); free(cnt); oracle_free(R); return status; }
+
+  /* O6 global stratum order by (kid, lo) */
+  qsort(fin, n_fin, sizeof(fin_t), cmp_fin);
+  R->n_strata = n_fin;
+  R->strata = (oracle_stratum*)calloc(n_fin ? n_fin : 1, sizeof(oracle_stratum));
+  uint64_t* kbase = (uint64_t*)malloc(sizeof(uint64_t) * (K + 1));
+  for (uint32_t k = 0; k <= K; k++) kbase[k] = UINT64_MAX;
+  for (uint64_t s = 0; s < n_fin; s++) {
+    oracle_stratum* o = &R->strata[s];
+    if (kbase[fin[s].kid] == UINT64_MAX) kbase[fin[s].kid] = s;
+    o->kernel_id = fin[s].kid; o->tier = fin[s].tier;
+    o->index_in_kernel = (uint32_t)(s - kbase[fin[s].kid]);
+    o->lo = fin[s].lo; o->hi = fin[s].hi; o->count = fin[s].n;
+    o->instr_sum_lo = (uint64_t)fin[s].S1; o->instr_sum_hi = (uint64_t)(fin[s].S1 >> 64);
+    o->bandwidth = fin[s].h; o->split_round = fin[s].round;
+  }
+
+  /* assignment: each invocation goes to the stratum of its kernel whose [lo, hi] holds x */
+  for (uint64_t i = 0; i < n; i++) {
+    uint32_t k = kid[i];
+    uint64_t s = kbase[k];
+    while (!(x[i] >= R->strata[s].lo && x[i] <= R->strata[s].hi)) s++;
+    R->sid[i] = (uint32_t)s;
+  }
+
+  /* O7 representatives.  Tier-1: first-chronological invocation.  Tier-2/3: per CTA value,
+   * (count, first id); dominant = max count, ties to the smaller first id; rep = its first. */
+  for (uint64_t s = 0; s < n_fin; s++) {
+    oracle_stratum* o = &R->strata[s];
+    uint32_t k = o->kernel_id;
+    uint64_t m = cnt[k + 1] - cnt[k];
+    /* the stratum's members, in row order */
+    uint64_t nm = 0;
+    uint64_t* mem = (uint64_t*)malloc(sizeof(uint64_t) * m);
+    for (uint64_t j = 0; j < m; j++) { uint64_t r = rows[cnt[k] + j]; if (R->sid[r] == s) mem[nm++] = r; }
+    uint64_t best_row = mem[0], best_id = ids ? ids[mem[0]] : mem[0];
+    for (uint64_t j = 1; j < nm; j++) {
+      uint64_t id = ids ? ids[mem[j]] : mem[j];
+      if (id < best_id) { best_id = id; best_row = mem[j]; }
+    }
+    if (o->tier != 1) {
+      /* distinct CTA values with count and first id (quadratic, plain) */
+      uint32_t* cv = (uint32_t*)malloc(sizeof(uint32_t) * nm);
+      uint64_t* cc = (uint64_t*)malloc(sizeof(uint64_t) * nm);
+      uint64_t* cf = (uint64_t*)malloc(sizeof(uint64_t) * nm);
+      uint64_t* cr = (uint64_t*)malloc(sizeof(uint64_t) * nm);
+      uint64_t nd = 0;
+      for (uint64_t j = 0; j < nm; j++) {
+        uint32_t c = cta ? cta[mem[j]] : 0;
+        uint64_t id = ids ? ids[mem[j]] : mem[j];
+        uint64_t d = 0;
+        while (d < nd && cv[d] != c) d++;
+        if (d == nd) { cv[nd] = c; cc[nd] = 0; cf[nd] = id; cr[nd] = mem[j]; nd++; }
+        cc[d]++;
+        if (id < cf[d]) { cf[d] = id; cr[d] = mem[j]; }
+      }
+      uint64_t b = 0;
+      for (uint64_t d = 1; d < nd; d++)
+        if (cc[d] > cc[b] || (cc[d] == cc[b] && cf[d] < cf[b])) b = d;
+      best_id = cf[b]; best_row = cr[b];
+      free(cv); free(cc); free(cf); free(cr);
+    }
+    o->rep_id = best_id;
+    o->rep_cta = cta ? cta[best_row] : 0;
+    o->rep_instr = x[best_row];
+    o->rep_cycles = cycles ? cycles[best_row] : 0;
+    free(mem);
+  }
+
+  /* totals: I = sum of W_s (O8), C_meas = sum of y (O9) */
+  if (cycles) { u128 c = 0; for (uint64_t i = 0; i < n; i++) c += cycles[i]; R->c_meas = c; }
+  free(kbase); free(fin); free(rows); free(cnt);
+  *out = R;
+  return OR_OK;
+}
+
+/* ------------------------------------------------------------------------------------------
+ * O8/O9 prediction:
+ *   w_s = W_s / I;  IPC_s = x_rep / y_rep;  IPC = 1 / sum_s w_s / IPC_s;
+ *   C_pred = I / IPC = sum_s W_s * y_rep / x_rep  (accumulated in __float128, then rounded);
+ *   error = |C_pred - C_meas| / C_meas;  speedup = C_meas / sum_s y_rep.
+ * rep_cycles: nullable; else per-stratum cycles of the representatives (e.g. simulated).
+ * ------------------------------------------------------------------------------------------ */
+int oracle_predict(const oracle_result* R, const uint64_t* rep_cycles, oracle_prediction* out) {
+  if (!R->has_cycles && !rep_cycles) return OR_EDOM;
+  __float128 cp = 0, yrep = 0, I = 0;
+  for (uint64_t s = 0; s < R->n_strata; s++) {
+    const oracle_stratum* o = &R->strata[s];
+    u128 W = ((u128)o->instr_sum_hi << 64) | o->instr_sum_lo;
+    uint64_t y = rep_cycles ? rep_cycles[s] : o->rep_cycles;
+    cp += ((__float128)W * (__float128)y) / (__float128)o->rep_instr;
+    yrep += (__float128)y;
+    I += (__float128)W;
+  }
+  out->predicted_cycles = (double)cp;
+  out->predicted_ipc = (double)(I / cp);
+  out->total_instr_lo = (uint64_t)R->total_instr;
+  out->total_instr_hi = (uint64_t)(R->total_instr >> 64);
+  if (R->has_cycles) {
+    __float128 cm = (__float128)R->c_meas;
+    out->measured_cycles = (double)cm;
+    out->error = R->c_meas == 0 ? NAN : (double)((cp > cm ? cp - cm : cm - cp) / cm);
+    out->speedup = (double)(cm / yrep);
+  } else {
+    out->measured_cycles = NAN; out->error = NAN; out->speedup = NAN;
+  }
+  return OR_OK;
+}
+
+/* accessors */
+uint64_t oracle_strata_count(const oracle_result* R) { return R->n_strata; }
+void oracle_strata_copy(const oracle_result* R, oracle_stratum* dst) {
+  memcpy(dst, R->strata, sizeof(oracle_stratum) * R->n_strata);
+}
+void oracle_sid_copy(const oracle_result* R, uint32_t* dst) { memcpy(dst, R->sid, 4 * R->n); }
+uint64_t oracle_segment_count(const oracle_result* R) { return R->n_segs; }
+int oracle_segment_get(const oracle_result* R, uint64_t i, uint32_t* meta4, uint64_t* meta3,
+                       double* h, uint64_t* d_lo, uint64_t* d_hi, uint64_t* cuts) {
+  if (i >= R->n_segs) return OR_EINVAL;
+  const oracle_segment* s = &R->segs[i];
+  meta4[0] = s->kernel_id; meta4[1] = s->round; meta4[2] = s->split_kind; meta4[3] = s->n_cuts;
+  meta3[0] = s->lo; meta3[1] = s->hi; meta3[2] = s->count;
+  *h = s->bandwidth;
+  if (d_lo) memcpy(d_lo, s->d_lo, 8 * R->G);
+  if (d_hi) memcpy(d_hi, s->d_hi, 8 * R->G);
+  if (cuts) memcpy(cuts, s->cuts, 8 * s->n_cuts);
+  return OR_OK;
+}
+uint32_t oracle_rounds(const oracle_result* R) { return R->rounds; }
+void oracle_totals(const oracle_result* R, uint64_t* out4) {
+  out4[0] = (uint64_t)R->total_instr; out4[1] = (uint64_t)(R->total_instr >> 64);
+  out4[2] = (uint64_t)R->c_meas; out4[3] = (uint64_t)(R->c_meas >> 64);
+}
+int oracle_sizeof_stratum(void) { return (int)sizeof(oracle_stratum); }

@@ -1,0 +1,207 @@
+"""Pins of the CPU oracle against things other than itself (closed forms, libm, scikit-learn,
+scipy, hand-built sequences, symmetry).  Each test names the PAPER.md passage (P:NN) or the
+DESIGN.md reading (A*) it checks."""
+import math
+import random
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle import brute
+
+TWO52 = 2.0 ** 52
+
+
+# ---------------------------------------------------------------- O3 tiers
+@pytest.mark.parametrize("vals,expect", [
+    ([5, 5, 5], 1),                      # identical counts -> Tier-1
+    ([4, 6], 2),                         # CoV = 1/5 < 2/5 -> Tier-2
+    ([3, 7], 3),                         # CoV = 2/5 exactly -> Tier-3 ("otherwise"; A2)
+    ([5, 17, 17, 21], 3),                # CoV = 6/15 = 2/5 exactly -> Tier-3
+    ([11, 23, 27, 39], 3),               # CoV = 2/5 exactly (mu 25, sigma 10)
+    ([1, 9], 3),                         # CoV = 4/5
+    ([2 ** 40, 2 ** 40 + 1] * 3, 2),     # tiny variance that fp64 one-pass loses (A4)
+    ([123456789], 1),                    # n = 1
+    ([10, 10, 10, 11], 2),
+])
+def test_tier_closed_forms(vals, expect):
+    assert oracle.tier(vals) == expect
+
+
+def test_tier_boundary_multisets_exact():
+    # every multiset of 2..4 values < 40 whose population CoV is exactly 2/5 must be Tier-3,
+    # and nudging theta up by 1/1000 must make it Tier-2 (the boundary is exact, A3)
+    found = 0
+    for a in range(1, 40):
+        for b in range(a + 1, 40):
+            v = [a, b]
+            mu = Fraction(a + b, 2)
+            var = (Fraction(a) - mu) ** 2 / 2 + (Fraction(b) - mu) ** 2 / 2
+            if var == Fraction(4, 25) * mu * mu:
+                found += 1
+                assert oracle.tier(v, (2, 5)) == 3
+                assert oracle.tier(v, (401, 1000)) == 2
+                assert oracle.tier(v, (399, 1000)) == 3
+    assert found >= 5
+
+
+def test_tier_matches_numpy_away_from_boundary():
+    rng = np.random.default_rng(1)
+    for _ in range(300):
+        n = int(rng.integers(2, 50))
+        v = rng.integers(1, 10 ** 6, n)
+        cov = v.std() / v.mean()          # numpy: population std (ddof=0)
+        if abs(cov - 0.4) < 1e-6 or v.min() == v.max():
+            continue
+        assert oracle.tier([int(a) for a in v]) == (2 if cov < 0.4 else 3)
+
+
+def test_tier_theta_variants():
+    assert oracle.tier([4, 6], (1, 5)) == 3      # CoV = 1/5 exactly at theta = 0.2
+    assert oracle.tier([4, 6], (1, 10)) == 3
+    assert oracle.tier([4, 6], (1, 1)) == 2
+
+
+# ---------------------------------------------------------------- det_exp, Q (A10)
+def test_det_exp_within_one_ulp_of_libm():
+    rng = random.Random(7)
+    ts = [0.0, 1e-300, 0.5, 1.0, math.log(2), 36.99, 37.0] + [rng.uniform(0, 37) for _ in range(20000)]
+    for t in ts:
+        e = math.exp(-t)
+        d = oracle.det_exp(t)
+        assert abs(d - e) <= math.ulp(e), (t, d, e)
+
+
+def test_det_exp_matches_exact_fma_emulation():
+    # brute.det_exp emulates fma with exact rationals; any dropped/added rounding step differs
+    rng = random.Random(11)
+    for _ in range(400):
+        t = rng.uniform(0, 37)
+        assert oracle.det_exp(t) == brute.det_exp(t)
+
+
+def test_q_cutoff_and_peak():
+    assert oracle.q_of_t(0.0) == 2 ** 52
+    assert oracle.q_of_t(37.0) == round(math.exp(-37) * TWO52)   # 0.38 -> 0
+    assert oracle.q_of_t(37.0000001) == 0
+    assert oracle.q_of_t(36.0) == round(math.exp(-36.0) * TWO52)
+    # exp(-37) * 2^52 < 0.5: the cutoff drops nothing the rounding would keep
+    assert math.exp(-37) * TWO52 < 0.5
+
+
+# ---------------------------------------------------------------- bandwidth ([36]; A8)
+def test_bandwidth_scott_normal_reference():
+    rng = np.random.default_rng(3)
+    for _ in range(50):
+        v = rng.integers(1, 10 ** 9, int(rng.integers(2, 3000)))
+        h = oracle.bandwidth([int(a) for a in v])
+        ref = 1.06 * v.std() * len(v) ** -0.2          # population sigma, Scott's 1.06 n^-1/5
+        assert abs(h - ref) <= ref * 2.0 ** -15
+        m, e = math.frexp(h)                             # 16 significant bits
+        assert (m * 2 ** 16) == int(m * 2 ** 16)
+
+
+def test_bandwidth_matches_brute():
+    rng = random.Random(5)
+    for _ in range(100):
+        v = [rng.randrange(1, 1 << 44) for _ in range(rng.randrange(2, 40))]
+        if min(v) == max(v):
+            continue
+        assert oracle.bandwidth(v) == brute.bandwidth(v, 1.06)
+
+
+# ---------------------------------------------------------------- grid (A9)
+def test_grid_endpoints_exact():
+    for lo, hi, G in [(1, 2, 3), (100, 1000, 1024), (12345, (1 << 44) - 1, 1024), (7, 8, 1000)]:
+        assert oracle.grid_point(lo, hi, 0, G) == float(lo)
+        assert oracle.grid_point(lo, hi, G - 1, G) == float(hi)
+
+
+# ---------------------------------------------------------------- KDE ([8] P:317)
+def _direct_gauss_sum(vals, grid, h):
+    z = (grid[:, None] - vals[None, :].astype(np.float64)) / h
+    return np.exp(-0.5 * z * z).sum(axis=1)
+
+
+def test_kde_against_sklearn_and_scipy():
+    from scipy.stats import gaussian_kde
+    from sklearn.neighbors import KernelDensity
+    rng = np.random.default_rng(12)
+    vals = np.concatenate([rng.normal(10_000, 300, 400), rng.normal(14_000, 500, 600)])
+    vals = np.clip(np.round(vals), 1, None).astype(np.uint64)
+    lo, hi, G = int(vals.min()), int(vals.max()), 256
+    h = oracle.bandwidth([int(v) for v in vals])
+    D = np.array([float(d) for d in oracle.kde(vals, lo, hi, h, G)]) / TWO52
+    grid = np.array([oracle.grid_point(lo, hi, j, G) for j in range(G)])
+    n = len(vals)
+    kd = KernelDensity(kernel="gaussian", bandwidth=h).fit(vals.astype(np.float64)[:, None])
+    sk = np.exp(kd.score_samples(grid[:, None])) * n * h * math.sqrt(2 * math.pi)
+    assert np.max(np.abs(D - sk)) <= 1e-12 * sk.max() + 1e-9
+    sig1 = vals.astype(np.float64).std(ddof=1)
+    sp = gaussian_kde(vals.astype(np.float64), bw_method=h / sig1)(grid) * n * h * math.sqrt(2 * math.pi)
+    assert np.max(np.abs(D - sp)) <= 1e-9 * sp.max()
+    direct = _direct_gauss_sum(vals, grid, h)
+    assert np.max(np.abs(D - direct)) <= 1e-12 * direct.max() + 1e-9
+
+
+def test_kde_matches_brute_bit_exact():
+    rng = random.Random(21)
+    vals = [rng.choice([1000, 5000]) + rng.randrange(-50, 50) for _ in range(40)]
+    lo, hi, G = min(vals), max(vals), 32
+    h = brute.bandwidth(vals, 1.06)
+    assert oracle.kde(np.array(vals, np.uint64), lo, hi, h, G) == brute.kde(vals, lo, hi, h, G)
+
+
+# ---------------------------------------------------------------- valleys (A11)
+def test_valleys_hand_built():
+    s = 10
+    big = 1 << 20
+    # zero plateau between two peaks -> one cut at the plateau midpoint
+    D = [big, big // 2, 0, 0, 0, 0, 0, big // 2, big]
+    assert oracle.valleys(D, s) == [4]
+    # ripple below delta -> no cut
+    D = [big, big - 3, big - 1, big - 2, big]
+    assert oracle.valleys(D, s) == []
+    # monotone -> no cut; edges are never valleys
+    assert oracle.valleys(list(range(100, 0, -1)), 0) == []
+    assert oracle.valleys(list(range(1, 101)), 0) == []
+    # k separated peaks -> k-1 cuts
+    peak = [0, 50, 100, 50, 0]
+    D = peak * 4
+    assert oracle.valleys(D, 3) == [4, 9, 14]
+    # the minimum's run: the first run of the minimum value wins
+    D = [100, 10, 10, 10, 20, 10, 100]
+    assert oracle.valleys(D, 2) == [2]
+    # agree with the brute force on random sequences
+    rng = random.Random(3)
+    for _ in range(500):
+        D = [rng.randrange(0, 1 << rng.randrange(1, 60)) for _ in range(rng.randrange(3, 64))]
+        sh = rng.randrange(0, 12)
+        assert oracle.valleys(D, sh) == brute.valley_cuts(D, sh)
+
+
+# ---------------------------------------------------------------- symmetry pins (O5)
+def test_two_point_masses_split_at_midpoint():
+    a, b, m = 1000, 10_000, 500
+    x = np.array([a] * m + [b] * m, np.uint64)
+    kid = np.zeros(2 * m, np.uint32)
+    r = oracle.stratify(kid, x, 1, keep_debug=True)
+    assert len(r.strata) == 2
+    assert list(r.strata["lo"]) == [a, b] and list(r.strata["hi"]) == [a, b]
+    seg = r.segments()[0]
+    assert seg["split_kind"] == 1 and seg["n_cuts"] == 1
+    spacing = (b - a) / 1023
+    assert abs(int(seg["cuts"][0]) - math.ceil((a + b) / 2)) <= spacing + 1
+
+
+def test_bimodal_mixture_one_cut_near_midpoint():
+    rng = np.random.default_rng(4)
+    mu1, mu2, s = 100_000, 300_000, 4_000       # separation >> 2h (bimodal, textbook)
+    x = np.concatenate([rng.normal(mu1, s, 3000), rng.normal(mu2, s, 3000)]).round().astype(np.uint64)
+    r = oracle.stratify(np.zeros(len(x), np.uint32), x, 1, keep_debug=True)
+    seg = r.segments()[0]
+    assert seg["n_cuts"] == 1 and seg["split_kind"] == 1
+    assert abs(int(seg["cuts"][0]) - 200_000) < 10_000
+    assert len(r.strata) == 2
