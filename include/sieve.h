@@ -1,0 +1,200 @@
+/*
+ * include/sieve.h -- C-ABI of the B200-native Sieve stratification library (libsieve.so).
+ *
+ * Sieve (Naderan-Tahan, SeyyedAghaei, Eeckhout, ISPASS'23; /root/reference/PAPER.md, cited
+ * P:NN) samples a GPU workload from its profile: "a big table with as many rows as there are
+ * kernel invocations ... (kernel name, kernel invocation ID, and instruction count)" (P:59,
+ * P:65).  The back-end groups invocations per kernel, tiers kernels by the
+ * coefficient of variation of their instruction counts, splits high-CoV kernels
+ * into strata with a kernel density estimate, picks one representative invocation per
+ * stratum with an instruction-count weight, and predicts application cycles from
+ * the representatives' IPC by a weighted harmonic mean.
+ *
+ * Every fully specified reading of an under-specified step is listed in DESIGN.md section 3
+ * (A1..A24, same numbering as SURVEY.md 8(c)); the CPU oracle (oracle/) implements the same
+ * readings independently, and integer outputs of this library are bit-identical to it.
+ *
+ * Conventions
+ *   - Every call returns an int status: SIEVE_OK (0) or a negative SIEVE_E* code.  No C++
+ *     exception crosses the ABI.  sieve_last_error() returns thread-local detail text.
+ *   - Pointers are plain host or device pointers as documented per argument; sizes are
+ *     element counts unless named *_bytes.  No framework types appear in any signature.
+ *   - All device work runs on the stream given to sieve_ctx_create; every call is
+ *     synchronous on return (results are complete and host outputs written).
+ *   - With world > 1, sieve_stratify and sieve_predict are COLLECTIVE: every rank calls them
+ *     in the same order; all ranks return identical strata (replicated decisions over exact,
+ *     order-independent integer reductions, so results are byte-identical for any world size).
+ */
+#ifndef SIEVE_H
+#define SIEVE_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* ---- status codes ---------------------------------------------------------------------- */
+enum {
+  SIEVE_OK = 0,
+  SIEVE_EINVAL = -1, /* null / foreign handle, theta_num or theta_den = 0, G < 3 or > 65536,
+                        kernel id >= num_kernels, bad flag combination */
+  SIEVE_ERANGE = -2, /* instruction count 0 or >= 2^44 (A21), n_local >= 2^32,
+                        num_kernels == 0 or > 65536 */
+  SIEVE_ENOMEM = -3, /* device or host allocation failed */
+  SIEVE_ECUDA = -4,  /* CUDA runtime error (detail in sieve_last_error) */
+  SIEVE_ENCCL = -5,  /* NCCL error or NCCL library not loadable */
+  SIEVE_EDOM = -6,   /* sieve_predict without any cycle source for the representatives */
+  SIEVE_ELIMIT = -7, /* the Tier-3 refinement needed more than max_rounds rounds (A15) */
+  SIEVE_ESTATE = -8  /* call not valid in this state (e.g. debug data not kept) */
+};
+
+/* memory-kind flags for sieve_load_trace */
+#define SIEVE_MEM_HOST 0u   /* columns are host pointers: copied to the device (H2D) */
+#define SIEVE_MEM_DEVICE 1u /* columns are device pointers on the ctx's device: copied D2D */
+#define SIEVE_ADOPT 2u      /* with SIEVE_MEM_DEVICE: borrow the caller's buffers, no copy; the
+                               caller keeps them alive and unchanged until sieve_trace_free */
+
+typedef struct sieve_ctx_s* sieve_ctx;       /* device, stream, communicator, allocator */
+typedef struct sieve_trace_s* sieve_trace;   /* this rank's slice of the profile, on the device */
+typedef struct sieve_strata_s* sieve_strata; /* the result; replicated on every rank */
+typedef struct sieve_group_s* sieve_group;   /* in-process rank group (several ranks, one GPU) */
+
+/* optional device allocator hook (e.g. a framework's caching allocator); stream is a
+   cudaStream_t passed as void* */
+typedef void* (*sieve_alloc_fn)(size_t bytes, void* stream, void* user);
+typedef void (*sieve_free_fn)(void* p, void* stream, void* user);
+
+/* ---- contexts and communicators -------------------------------------------------------- */
+
+/* NCCL unique id for a multi-process communicator (128 bytes).  Call on rank 0 and
+   broadcast the bytes to every rank by any means (e.g. torch.distributed). */
+int sieve_get_unique_id(uint8_t out[128]);
+
+/* Create a context on CUDA device `cuda_device` using stream `cuda_stream` (a cudaStream_t,
+   NULL = the legacy default stream).  world == 1: no communicator (nccl_id must be NULL).
+   world > 1: ncclCommInitRank(world, *nccl_id, rank) -- one process (or thread) per GPU. */
+int sieve_ctx_create(int cuda_device, void* cuda_stream, int rank, int world,
+                     const uint8_t* nccl_id, sieve_ctx* out);
+
+/* In-process rank group for parity tests on ONE GPU (NCCL cannot place two ranks of one
+   communicator on one device): `world` host threads each create a context with
+   sieve_ctx_create_in_group and call the collective entry points concurrently; partials are
+   combined by the same exact limb reductions that the NCCL path uses, through device
+   memory of the shared GPU and a host barrier. */
+int sieve_group_create(int world, sieve_group* out);
+void sieve_group_destroy(sieve_group g);
+int sieve_ctx_create_in_group(int cuda_device, void* cuda_stream, sieve_group g, int rank,
+                              sieve_ctx* out);
+
+int sieve_ctx_set_allocator(sieve_ctx ctx, sieve_alloc_fn alloc, sieve_free_fn free_fn, void* user);
+void sieve_ctx_destroy(sieve_ctx ctx);
+
+/* ---- the profile (extended with CTA size P:93 and cycles P:125, A20) -------- */
+
+/* Load this rank's contiguous, chronological slice of the profile.
+     n_local      rows in this slice (< 2^32); may be 0
+     first_id     global invocation id of row 0 (exclusive prefix of the slice sizes); the
+                  invocation ID of row j is first_id + j ("first-chronological" = the
+                  smallest id, A18)
+     num_kernels  K: kernel ids are dense in [0, K), 1 <= K <= 65536 ("kernel name",
+                  interned by the caller); must be the same on every rank
+     kernel_id    [n_local] u32
+     instr        [n_local] u64 dynamic instruction count, 1 <= x < 2^44 (A21)
+     cta          [n_local] u32 CTA (thread-block) size, opaque key (A16); NULL = all equal
+     cycles       [n_local] u64 measured cycles; NULL = no measured cycles
+     mem          SIEVE_MEM_HOST | SIEVE_MEM_DEVICE [| SIEVE_ADOPT]
+   Value validation (kernel id < K, 1 <= x < 2^44) happens on the device in the first pass of
+   sieve_stratify, which returns SIEVE_EINVAL / SIEVE_ERANGE on a bad row. */
+int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_id, uint32_t num_kernels,
+                     const uint32_t* kernel_id, const uint64_t* instr, const uint32_t* cta,
+                     const uint64_t* cycles, uint32_t mem, sieve_trace* out);
+void sieve_trace_free(sieve_trace t);
+
+/* ---- stratification ------------------------------------------------------------ */
+typedef struct {
+  uint32_t theta_num, theta_den; /* theta = num/den, exact rational (P:85 default 0.4 = 2/5; A3) */
+  uint32_t grid_points;          /* G, KDE grid points on [lo, hi] (A9), 3 <= G <= 65536; 1024 */
+  uint32_t valley_shift;         /* hysteresis delta = max(1, Dmax >> shift) (A11); 10 */
+  uint32_t max_rounds;           /* refinement round bound (A15); 64 */
+  uint32_t keep_debug;           /* 1: keep every KDE segment for sieve_segment_get */
+  double bw_scale;               /* Scott's normal-reference factor (A8); 1.06 */
+} sieve_params;
+
+void sieve_params_default(sieve_params* p);
+
+/* Stratify the loaded profile (collective if world > 1).
+     stratum_of_invocation  nullable DEVICE pointer [n_local] u32: receives the global stratum
+                            index of every row of this rank's slice
+     out                    the stratum table, replicated on every rank
+   Strata are ordered by (kernel id, lowest instruction count) (A23). */
+int sieve_stratify(sieve_trace t, const sieve_params* p, uint32_t* stratum_of_invocation,
+                   sieve_strata* out);
+
+typedef struct {
+  uint32_t kernel_id;
+  uint32_t tier;            /* 1, 2, 3 */
+  uint32_t index_in_kernel; /* 0.. by ascending instruction counts */
+  uint32_t rep_cta;         /* CTA size of the representative */
+  uint64_t lo, hi;          /* smallest / largest instruction count in the stratum */
+  uint64_t count;           /* invocations in the stratum */
+  uint64_t instr_sum_lo, instr_sum_hi; /* W_s = sum of instruction counts, u128 */
+  uint64_t rep_id;          /* global invocation id of the representative */
+  uint64_t rep_instr, rep_cycles; /* x and y of the representative (y = 0 without cycles) */
+  double bandwidth;         /* KDE bandwidth h of the segment whose split created this stratum;
+                               0 for Tier-1/2 */
+  uint32_t split_round;     /* refinement round that created it; 0 for Tier-1/2 */
+  uint32_t pad;
+} sieve_stratum;
+
+int sieve_strata_count(sieve_strata s, uint64_t* n);
+/* copy min(cap, count) strata to a HOST array */
+int sieve_strata_copy(sieve_strata s, sieve_stratum* host_out, uint64_t cap);
+/* refinement rounds used, KDE terms evaluated (diagnostics) */
+int sieve_strata_stats(sieve_strata s, uint32_t* rounds, uint64_t* kde_terms);
+void sieve_strata_free(sieve_strata s);
+
+/* ---- debug: every KDE segment of every round (requires keep_debug = 1, else ESTATE) ---- */
+typedef struct {
+  uint32_t kernel_id, round, split_kind /* 1 = valley, 2 = bisect */, n_cuts;
+  uint64_t lo, hi, count;
+  double bandwidth;
+} sieve_segment;
+
+int sieve_segment_count(sieve_strata s, uint64_t* n);
+/* density_lo/hi: nullable HOST arrays [G]: D_j as u128 = hi:lo (fixed point 2^-52);
+   cuts: nullable HOST array [n_cuts]: integer thresholds (x < T left, x >= T right; A12) */
+int sieve_segment_get(sieve_strata s, uint64_t idx, sieve_segment* out, uint64_t* density_lo,
+                      uint64_t* density_hi, uint64_t* cuts);
+
+/* ---- prediction --------------------------------------------- */
+typedef struct {
+  double predicted_cycles; /* C_pred = I / IPC = sum_s W_s * y_rep / x_rep (A22) */
+  double predicted_ipc;    /* IPC = 1 / sum_s w_s / IPC_s */
+  double measured_cycles;  /* C_meas = sum of the trace's cycles; NaN without a cycles column */
+  double error;            /* |C_pred - C_meas| / C_meas; NaN if unknown or C_meas = 0 */
+  double speedup;          /* C_meas / sum_s y_rep; NaN without a cycles column */
+  uint64_t total_instr_lo, total_instr_hi; /* I = sum of all instruction counts, u128 */
+} sieve_prediction;
+
+/* Predict application cycles (collective if world > 1).
+     rep_cycles  nullable HOST array [n_strata]: cycles of each representative (e.g. from
+                 detailed simulation); NULL = take y of the representatives from the
+                 trace's cycles column (SIEVE_EDOM if the trace has none). */
+int sieve_predict(sieve_strata s, sieve_trace t, const uint64_t* rep_cycles, sieve_prediction* out);
+
+/* ---- misc ----------------------------------------------------------------------------------- */
+const char* sieve_last_error(void); /* thread-local; valid until the next call on this thread */
+const char* sieve_version(void);
+
+/* exact limb encoding used by every cross-rank reduction (host utility, no GPU needed):
+   a u128 value is split into 32-bit limbs carried in u64 lanes so that a lane-wise u64 sum
+   over up to 2^32 ranks cannot overflow; normalisation propagates the carries. */
+void sieve_u128_to_limbs(uint64_t lo, uint64_t hi, uint64_t limbs[4]);
+void sieve_limbs_to_u128(const uint64_t limbs[4], uint64_t* lo, uint64_t* hi);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SIEVE_H */

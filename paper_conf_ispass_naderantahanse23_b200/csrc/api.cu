@@ -1,0 +1,903 @@
+// api.cu -- the C-ABI (include/sieve.h) and the host orchestrator of the stratification path.
+//
+// The orchestrator sequences the device passes and takes the few replicated, exact host
+// decisions the paper's method needs between them:
+//   pass A moments -> [AR-1] -> tiers (exact u256 CoV test) -> Tier-3 compaction ->
+//   radix sort -> prefix sums -> rounds { bandwidth h (host fp64, Scott [36]) -> KDE ->
+//   [AR-2] -> valleys -> part moments -> [AR-3] -> exact CoV test per part } ->
+//   stratum table (kernel, lo) -> pass B assignment + (stratum, CTA) statistics -> [AR-4] ->
+//   representatives -> representatives' (x, y) -> [AR-5].
+// Every [AR-*] is an exact u64-lane all-reduce (limbs for u128), so each rank takes identical
+// decisions and the strata are byte-identical for any number of ranks.
+#include <math.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <string>
+#include <vector>
+
+#include "comm.h"
+#include "kernels.cuh"
+
+// ------------------------------------------------------------------------------------------
+// errors
+// ------------------------------------------------------------------------------------------
+static thread_local std::string t_err;
+void sv_set_error(const std::string& msg) { t_err = msg; }
+int sv_fail(int code, const std::string& msg) { t_err = msg; return code; }
+int sv_cuda(cudaError_t e, const char* what, int line) {
+  char buf[512];
+  snprintf(buf, sizeof buf, "CUDA error %s (%s) at api line %d: %s", cudaGetErrorName(e),
+           cudaGetErrorString(e), line, what);
+  t_err = buf;
+  return e == cudaErrorMemoryAllocation ? SIEVE_ENOMEM : SIEVE_ECUDA;
+}
+extern "C" const char* sieve_last_error(void) { return t_err.c_str(); }
+extern "C" const char* sieve_version(void) { return "sieve-b200 0.1 (sm_100a)"; }
+
+int sv_num_sms() {
+  static int cache[64] = {0};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  if (!cache[dev]) {
+    int v = 0;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+    cache[dev] = v > 0 ? v : 148;
+  }
+  return cache[dev];
+}
+
+extern "C" void sieve_u128_to_limbs(uint64_t lo, uint64_t hi, uint64_t limbs[4]) {
+  limbs_from_u128(lo, hi, (u64*)limbs);
+}
+extern "C" void sieve_limbs_to_u128(const uint64_t limbs[4], uint64_t* lo, uint64_t* hi) {
+  limbs_to_u128((const u64*)limbs, (u64*)lo, (u64*)hi);
+}
+
+// ------------------------------------------------------------------------------------------
+// handles
+// ------------------------------------------------------------------------------------------
+#define CTX_MAGIC 0x51E7C7A0u
+#define TRACE_MAGIC 0x51E7C7A1u
+#define STRATA_MAGIC 0x51E7C7A2u
+
+struct sieve_ctx_s {
+  uint32_t magic = CTX_MAGIC;
+  int device = 0;
+  cudaStream_t stream = 0;
+  int rank = 0, world = 1;
+  Comm* comm = nullptr;
+  sieve_alloc_fn af = nullptr;
+  sieve_free_fn ff = nullptr;
+  void* user = nullptr;
+};
+
+struct sieve_trace_s {
+  uint32_t magic = TRACE_MAGIC;
+  sieve_ctx ctx = nullptr;
+  u64 n = 0, first_id = 0;
+  u32 K = 0;
+  u32* kid = nullptr;
+  u64* x = nullptr;
+  u32* cta = nullptr;
+  u64* y = nullptr;
+  bool owned = true;
+};
+
+struct SegDebug {
+  sieve_segment meta;
+  std::vector<u64> dlo, dhi, cuts;
+};
+
+struct sieve_strata_s {
+  uint32_t magic = STRATA_MAGIC;
+  sieve_ctx ctx = nullptr;
+  std::vector<sieve_stratum> st;
+  std::vector<SegDebug> segs;
+  bool keep_debug = false;
+  u32 G = 0;
+  u32 rounds = 0;
+  u64 kde_terms = 0;
+  u128 total_instr = 0, c_meas = 0;
+  bool has_cycles = false;
+};
+
+static bool ctx_ok(sieve_ctx c) { return c && c->magic == CTX_MAGIC; }
+static bool trace_ok(sieve_trace t) { return t && t->magic == TRACE_MAGIC && ctx_ok(t->ctx); }
+static bool strata_ok(sieve_strata s) { return s && s->magic == STRATA_MAGIC; }
+
+// device memory through the ctx allocator (default: stream-ordered cudaMallocAsync)
+static int dalloc(sieve_ctx c, void** p, size_t bytes) {
+  *p = nullptr;
+  if (bytes == 0) bytes = 16;
+  if (c->af) {
+    *p = c->af(bytes, (void*)c->stream, c->user);
+    if (!*p) return sv_fail(SIEVE_ENOMEM, "allocator hook returned NULL");
+    return SIEVE_OK;
+  }
+  SV_CUDA(cudaMallocAsync(p, bytes, c->stream));
+  return SIEVE_OK;
+}
+static void dfree(sieve_ctx c, void* p) {
+  if (!p) return;
+  if (c->ff) c->ff(p, (void*)c->stream, c->user);
+  else cudaFreeAsync(p, c->stream);
+}
+
+template <typename T>
+struct DBuf {
+  sieve_ctx c = nullptr;
+  T* p = nullptr;
+  size_t n = 0;
+  DBuf() {}
+  explicit DBuf(sieve_ctx cc) : c(cc) {}
+  DBuf(const DBuf&) = delete;
+  DBuf& operator=(const DBuf&) = delete;
+  ~DBuf() { release(); }
+  void release() { if (p) dfree(c, p); p = nullptr; n = 0; }
+  int alloc(size_t count) {
+    release();
+    n = count;
+    void* q;
+    int st = dalloc(c, &q, count * sizeof(T));
+    p = (T*)q;
+    return st;
+  }
+  T* get() const { return p; }
+};
+
+// ------------------------------------------------------------------------------------------
+// contexts
+// ------------------------------------------------------------------------------------------
+extern "C" int sieve_get_unique_id(uint8_t out[128]) {
+  if (!out) return sv_fail(SIEVE_EINVAL, "out is NULL");
+  return nccl_unique_id(out);
+}
+
+static int ctx_common(int dev, void* stream, sieve_ctx* out, sieve_ctx_s** c) {
+  if (!out) return sv_fail(SIEVE_EINVAL, "out is NULL");
+  *out = nullptr;
+  int ndev = 0;
+  SV_CUDA(cudaGetDeviceCount(&ndev));
+  if (dev < 0 || dev >= ndev) return sv_fail(SIEVE_EINVAL, "bad cuda_device");
+  SV_CUDA(cudaSetDevice(dev));
+  // keep freed pool memory for the next call (repeated stratify calls do not re-map)
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  *c = new sieve_ctx_s();
+  (*c)->device = dev;
+  (*c)->stream = (cudaStream_t)stream;
+  return SIEVE_OK;
+}
+
+extern "C" int sieve_ctx_create(int cuda_device, void* cuda_stream, int rank, int world,
+                                const uint8_t* nccl_id, sieve_ctx* out) {
+  if (world < 1 || rank < 0 || rank >= world) return sv_fail(SIEVE_EINVAL, "bad rank/world");
+  if ((world == 1) != (nccl_id == nullptr)) return sv_fail(SIEVE_EINVAL, "nccl_id must be NULL iff world == 1");
+  sieve_ctx_s* c;
+  SV_TRY(ctx_common(cuda_device, cuda_stream, out, &c));
+  c->rank = rank;
+  c->world = world;
+  if (world > 1) {
+    int st = nccl_comm_create(rank, world, nccl_id, &c->comm);
+    if (st != SIEVE_OK) { delete c; return st; }
+  }
+  *out = c;
+  return SIEVE_OK;
+}
+
+extern "C" int sieve_ctx_create_in_group(int cuda_device, void* cuda_stream, sieve_group g, int rank,
+                                         sieve_ctx* out) {
+  sieve_ctx_s* c;
+  SV_TRY(ctx_common(cuda_device, cuda_stream, out, &c));
+  int st = group_comm_create(g, rank, &c->comm);
+  if (st != SIEVE_OK) { delete c; return st; }
+  c->rank = c->comm->rank;
+  c->world = c->comm->world;
+  *out = c;
+  return SIEVE_OK;
+}
+
+extern "C" int sieve_ctx_set_allocator(sieve_ctx ctx, sieve_alloc_fn a, sieve_free_fn f, void* user) {
+  if (!ctx_ok(ctx) || (!a) != (!f)) return sv_fail(SIEVE_EINVAL, "bad ctx or allocator pair");
+  ctx->af = a; ctx->ff = f; ctx->user = user;
+  return SIEVE_OK;
+}
+
+extern "C" void sieve_ctx_destroy(sieve_ctx ctx) {
+  if (!ctx_ok(ctx)) return;
+  delete ctx->comm;
+  ctx->magic = 0;
+  delete ctx;
+}
+
+extern "C" void sieve_params_default(sieve_params* p) {
+  if (!p) return;
+  p->theta_num = 2;
+  p->theta_den = 5;
+  p->grid_points = 1024;
+  p->valley_shift = 10;
+  p->max_rounds = 64;
+  p->keep_debug = 0;
+  p->bw_scale = 1.06;
+}
+
+// ------------------------------------------------------------------------------------------
+// trace
+// ------------------------------------------------------------------------------------------
+extern "C" int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_id, uint32_t K,
+                                const uint32_t* kernel_id, const uint64_t* instr, const uint32_t* cta,
+                                const uint64_t* cycles, uint32_t mem, sieve_trace* out) {
+  if (!out) return sv_fail(SIEVE_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!ctx_ok(ctx)) return sv_fail(SIEVE_EINVAL, "bad ctx");
+  if (K == 0 || K > SIEVE_MAX_K) return sv_fail(SIEVE_ERANGE, "num_kernels must be in [1, 65536]");
+  if (n_local >= (1ull << 32)) return sv_fail(SIEVE_ERANGE, "n_local must be < 2^32");
+  if (n_local && (!kernel_id || !instr)) return sv_fail(SIEVE_EINVAL, "kernel_id and instr are required");
+  if (mem & ~3u) return sv_fail(SIEVE_EINVAL, "bad mem flags");
+  bool dev = mem & SIEVE_MEM_DEVICE, adopt = mem & SIEVE_ADOPT;
+  if (adopt && !dev) return sv_fail(SIEVE_EINVAL, "SIEVE_ADOPT needs SIEVE_MEM_DEVICE");
+  SV_CUDA(cudaSetDevice(ctx->device));
+  sieve_trace_s* t = new sieve_trace_s();
+  t->ctx = ctx; t->n = n_local; t->first_id = first_id; t->K = K; t->owned = !adopt;
+  if (adopt) {
+    t->kid = (u32*)kernel_id; t->x = (u64*)instr; t->cta = (u32*)cta; t->y = (u64*)cycles;
+  } else {
+    cudaMemcpyKind kind = dev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+    auto cp = [&](void** dst, const void* src, size_t bytes) -> int {
+      if (!src) { *dst = nullptr; return SIEVE_OK; }
+      SV_TRY(dalloc(ctx, dst, bytes));
+      if (bytes) SV_CUDA(cudaMemcpyAsync(*dst, src, bytes, kind, ctx->stream));
+      return SIEVE_OK;
+    };
+    int st = SIEVE_OK;
+    if (st == SIEVE_OK) st = cp((void**)&t->kid, kernel_id ? kernel_id : (const uint32_t*)&t->n, n_local * 4);
+    if (st == SIEVE_OK) st = cp((void**)&t->x, instr ? instr : (const uint64_t*)&t->n, n_local * 8);
+    if (st == SIEVE_OK) st = cp((void**)&t->cta, cta, n_local * 4);
+    if (st == SIEVE_OK) st = cp((void**)&t->y, cycles, n_local * 8);
+    if (st == SIEVE_OK) { cudaError_t e = cudaStreamSynchronize(ctx->stream); if (e) st = sv_cuda(e, "load sync", __LINE__); }
+    if (st != SIEVE_OK) { t->magic = TRACE_MAGIC; sieve_trace_free(t); return st; }
+  }
+  *out = t;
+  return SIEVE_OK;
+}
+
+extern "C" void sieve_trace_free(sieve_trace t) {
+  if (!t || t->magic != TRACE_MAGIC) return;
+  if (t->owned && ctx_ok(t->ctx)) {
+    cudaSetDevice(t->ctx->device);
+    dfree(t->ctx, t->kid); dfree(t->ctx, t->x); dfree(t->ctx, t->cta); dfree(t->ctx, t->y);
+    cudaStreamSynchronize(t->ctx->stream);
+  }
+  t->magic = 0;
+  delete t;
+}
+
+// ------------------------------------------------------------------------------------------
+// exact host arithmetic for the replicated decisions
+// ------------------------------------------------------------------------------------------
+struct W256 { u64 w[4]; };  // little-endian words
+
+static W256 w256_mul(u128 a, u128 b) {
+  u64 A[2] = {(u64)a, (u64)(a >> 64)}, B[2] = {(u64)b, (u64)(b >> 64)};
+  W256 r = {{0, 0, 0, 0}};
+  for (int i = 0; i < 2; i++)
+    for (int j = 0; j < 2; j++) {
+      u128 p = (u128)A[i] * B[j];
+      // add p at word i+j with carry propagation
+      int k = i + j;
+      u128 add = p;
+      while (add && k < 4) {
+        u128 s = (u128)r.w[k] + (u64)add;
+        r.w[k] = (u64)s;
+        add = (add >> 64) + (s >> 64);
+        k++;
+      }
+    }
+  return r;
+}
+static W256 w256_mul_small(W256 a, u64 m) {
+  W256 r;
+  u128 c = 0;
+  for (int i = 0; i < 4; i++) { u128 p = (u128)a.w[i] * m + c; r.w[i] = (u64)p; c = p >> 64; }
+  return r;
+}
+static W256 w256_sub(W256 a, W256 b) {
+  W256 r;
+  u64 br = 0;
+  for (int i = 0; i < 4; i++) {
+    u128 d = (u128)a.w[i] - b.w[i] - br;
+    r.w[i] = (u64)d;
+    br = (u64)(d >> 127);  // borrow if negative
+  }
+  return r;
+}
+static bool w256_lt(W256 a, W256 b) {
+  for (int i = 3; i >= 0; i--) if (a.w[i] != b.w[i]) return a.w[i] < b.w[i];
+  return false;
+}
+// correctly rounded conversion to double (round to nearest even)
+static double w256_to_double(W256 a) {
+  int top = 3;
+  while (top > 0 && a.w[top] == 0) top--;
+  if (top <= 1) return (double)(((u128)a.w[1] << 64) | a.w[0]);
+  int lz = __builtin_clzll(a.w[top]);
+  int nbits = 64 * top + 64 - lz;
+  int sh = nbits - 64;                         // >= 65 here
+  // extract the 64 bits [sh, sh+64) and a sticky of the bits below
+  int wq = sh / 64, bq = sh % 64;
+  u64 hi64 = bq ? ((a.w[wq] >> bq) | (a.w[wq + 1] << (64 - bq))) : a.w[wq];
+  bool sticky = bq ? (a.w[wq] & ((1ull << bq) - 1)) != 0 : false;
+  for (int i = 0; i < wq && !sticky; i++) sticky = a.w[i] != 0;
+  return ldexp((double)(hi64 | (sticky ? 1ull : 0ull)), sh);
+}
+
+// CoV < p/q  <=>  q^2 (n S2 - S1^2) < p^2 S1^2   (A1-A5)
+static bool cov_lt(u64 n, u128 s1, u128 s2, u32 p, u32 q) {
+  W256 var_n2 = w256_sub(w256_mul(n, s2), w256_mul(s1, s1));
+  return w256_lt(w256_mul_small(var_n2, (u64)q * q), w256_mul_small(w256_mul(s1, s1), (u64)p * p));
+}
+
+// Scott's normal-reference bandwidth ([36]; A8), rounded to 16 significant bits
+static double scott_h(u64 n, u128 s1, u128 s2, double bw_scale) {
+  W256 v = w256_sub(w256_mul(n, s2), w256_mul(s1, s1));
+  double dn = (double)n;
+  double var = w256_to_double(v) / (dn * dn);
+  double h_raw = (bw_scale * sqrt(var)) * pow(dn, -0.2);
+  int e = ilogb(h_raw) - 15;
+  return ldexp(rint(ldexp(h_raw, -e)), e);
+}
+
+static inline u128 u128_of(u64 lo, u64 hi) { return ((u128)hi << 64) | lo; }
+static inline u128 limbs_u128(const u64* l) { u64 lo, hi; limbs_to_u128(l, &lo, &hi); return u128_of(lo, hi); }
+static inline u32 bitlen(u64 v) { return v ? 64 - __builtin_clzll(v) : 0; }
+
+static int allreduce(sieve_ctx c, u64* buf, size_t n, ReduceOp op) {
+  if (!c->comm) return SIEVE_OK;
+  return c->comm->allreduce(buf, n, op, c->stream);
+}
+
+template <typename T>
+static int d2h(sieve_ctx c, std::vector<T>& h, const T* d, size_t n) {
+  h.resize(n);
+  if (n) SV_CUDA(cudaMemcpyAsync(h.data(), d, n * sizeof(T), cudaMemcpyDeviceToHost, c->stream));
+  return SIEVE_OK;
+}
+template <typename T>
+static int h2d(sieve_ctx c, T* d, const std::vector<T>& h) {
+  if (!h.empty()) SV_CUDA(cudaMemcpyAsync(d, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice, c->stream));
+  return SIEVE_OK;
+}
+static int sync(sieve_ctx c) { SV_CUDA(cudaStreamSynchronize(c->stream)); return SIEVE_OK; }
+
+// ------------------------------------------------------------------------------------------
+// sieve_stratify
+// ------------------------------------------------------------------------------------------
+struct OpenSeg { u32 kid, t3rank; u64 lo, hi, n; u128 s1, s2; };
+struct Fin { u32 kid, tier; u64 lo, hi, n; u128 s1; double h; u32 round; };
+
+static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out, sieve_strata_s* R) {
+  sieve_ctx c = t->ctx;
+  cudaStream_t S = c->stream;
+  const u32 K = t->K, G = P->grid_points;
+  const u64 n = t->n;
+
+  // ---------------- pass A: per-kernel moments + totals --------------------------------------
+  const int gridA = moments_grid();
+  const u32 kt = (u32)moments_kt(K);
+  DBuf<KMomPartial> part(c);
+  DBuf<u64> blk_tot(c), lanes(c), mm(c), local_n(c), tot(c);
+  SV_TRY(part.alloc((size_t)gridA * kt));
+  SV_TRY(blk_tot.alloc((size_t)gridA * 3));
+  SV_TRY(lanes.alloc((size_t)K * MOM_LANES));
+  SV_TRY(mm.alloc((size_t)K * 2));
+  SV_TRY(local_n.alloc(K));
+  // tot: [0..4) C_meas limbs (SUM), [4] max x (MAX), [5..8) error lanes (MAX)
+  SV_TRY(tot.alloc(8));
+  SV_CUDA(cudaMemsetAsync(tot.get(), 0, 8 * 8, S));
+  for (u32 k0 = 0; k0 < K; k0 += kt) {
+    u32 kk = std::min(kt, K - k0);
+    if (n) {
+      launch_moments(t->kid, t->x, t->y, n, K, k0, kk, part.get(), blk_tot.get(), tot.get() + 5,
+                     gridA, S);
+      launch_moments_reduce(part.get(), blk_tot.get(), gridA, k0, kk, K, lanes.get(), mm.get(),
+                            local_n.get(), tot.get(), tot.get() + 4, k0 == 0, S);
+    }
+  }
+  if (!n) {
+    SV_CUDA(cudaMemsetAsync(lanes.get(), 0, (size_t)K * MOM_LANES * 8, S));
+    SV_CUDA(cudaMemsetAsync(local_n.get(), 0, (size_t)K * 8, S));
+    std::vector<u64> mmh(2 * (size_t)K);
+    for (u32 k = 0; k < K; k++) { mmh[2 * k] = ~0ull; mmh[2 * k + 1] = 0; }
+    SV_TRY(h2d(c, mm.get(), mmh));
+  }
+  SV_CUDA(cudaGetLastError());
+  // AR-1: sums, then min/max (mm is interleaved min,max per kernel: reduce via a [2][K] copy)
+  std::vector<u64> h_lanes, h_mm, h_tot, h_localn;
+  if (c->comm) {
+    DBuf<u64> mn(c), mx(c);
+    SV_TRY(mn.alloc(K + 1));
+    SV_TRY(mx.alloc(K + 4));
+    SV_CUDA(cudaMemcpy2DAsync(mn.get(), 8, mm.get(), 16, 8, K, cudaMemcpyDeviceToDevice, S));
+    SV_CUDA(cudaMemcpy2DAsync(mx.get(), 8, mm.get() + 1, 16, 8, K, cudaMemcpyDeviceToDevice, S));
+    SV_CUDA(cudaMemcpyAsync(mx.get() + K, tot.get() + 4, 4 * 8, cudaMemcpyDeviceToDevice, S));
+    SV_TRY(allreduce(c, lanes.get(), (size_t)K * MOM_LANES, RED_SUM));
+    SV_TRY(allreduce(c, tot.get(), 4, RED_SUM));
+    SV_TRY(allreduce(c, mn.get(), K, RED_MIN));
+    SV_TRY(allreduce(c, mx.get(), K + 4, RED_MAX));
+    SV_CUDA(cudaMemcpy2DAsync(mm.get(), 16, mn.get(), 8, 8, K, cudaMemcpyDeviceToDevice, S));
+    SV_CUDA(cudaMemcpy2DAsync(mm.get() + 1, 16, mx.get(), 8, 8, K, cudaMemcpyDeviceToDevice, S));
+    SV_CUDA(cudaMemcpyAsync(tot.get() + 4, mx.get() + K, 4 * 8, cudaMemcpyDeviceToDevice, S));
+    SV_TRY(d2h(c, h_lanes, lanes.get(), (size_t)K * MOM_LANES));
+    SV_TRY(d2h(c, h_mm, mm.get(), (size_t)K * 2));
+    SV_TRY(d2h(c, h_tot, tot.get(), 8));
+    SV_TRY(d2h(c, h_localn, local_n.get(), K));
+    SV_TRY(sync(c));
+  } else {
+    SV_TRY(d2h(c, h_lanes, lanes.get(), (size_t)K * MOM_LANES));
+    SV_TRY(d2h(c, h_mm, mm.get(), (size_t)K * 2));
+    SV_TRY(d2h(c, h_tot, tot.get(), 8));
+    SV_TRY(d2h(c, h_localn, local_n.get(), K));
+    SV_TRY(sync(c));
+  }
+  part.release(); blk_tot.release();
+  if (h_tot[5]) return sv_fail(SIEVE_EINVAL, "kernel id >= num_kernels in the trace");
+  if (h_tot[6]) return sv_fail(SIEVE_ERANGE, "instruction count 0 or >= 2^44 in the trace (A21)");
+  R->c_meas = limbs_u128(&h_tot[0]);
+  const u64 max_x = h_tot[4];
+
+  // ---------------- tiers ---------------------------------------------------------
+  std::vector<Fin> fin;
+  std::vector<OpenSeg> open;
+  std::vector<u32> t3rank(K, 0xFFFFFFFFu);
+  u32 n_t3 = 0;
+  u64 n3_local = 0;
+  u128 I = 0;
+  for (u32 k = 0; k < K; k++) {
+    const u64* L = &h_lanes[(size_t)k * MOM_LANES];
+    u64 nk = L[0];
+    if (!nk) continue;
+    u128 s1 = limbs_u128(L + 1), s2 = limbs_u128(L + 5);
+    u64 lo = h_mm[2 * k], hi = h_mm[2 * k + 1];
+    I += s1;
+    if (lo == hi) {                                              // Tier-1 (A4)
+      fin.push_back({k, 1, lo, hi, nk, s1, 0.0, 0});
+    } else if (cov_lt(nk, s1, s2, P->theta_num, P->theta_den)) { // Tier-2
+      fin.push_back({k, 2, lo, hi, nk, s1, 0.0, 0});
+    } else {                                                     // Tier-3 -> refinement
+      t3rank[k] = n_t3++;
+      n3_local += h_localn[k];
+      open.push_back({k, t3rank[k], lo, hi, nk, s1, s2});
+    }
+  }
+  R->total_instr = I;
+
+  // ---------------- Tier-3 keys: compact, sort, prefix sums ----------------------------------
+  const u32 bx = std::max<u32>(1, bitlen(max_x));
+  const u64 xmask = (bx >= 64) ? ~0ull : ((1ull << bx) - 1);
+  const int nbits = (int)(bx + bitlen(n_t3 ? n_t3 - 1 : 0));
+  DBuf<u64> keys(c), P1(c), P2(c);
+  DBuf<u32> d_t3rank(c);
+  DBuf<unsigned long long> counter(c);
+  SV_TRY(counter.alloc(4));
+  if (n_t3 && n3_local) {
+    SV_TRY(d_t3rank.alloc(K));
+    SV_TRY(h2d(c, d_t3rank.get(), t3rank));
+    SV_TRY(keys.alloc(n3_local));
+    SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
+    launch_t3_compact(t->kid, t->x, n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
+    {
+      DBuf<char> tmp(c);
+      SV_TRY(tmp.alloc(radix_sort_temp_bytes(n3_local, false)));
+      SV_TRY(radix_sort(keys.get(), nullptr, n3_local, nbits, tmp.get(), S));
+    }
+    SV_TRY(P1.alloc(2 * (n3_local + 1)));
+    SV_TRY(P2.alloc(2 * (n3_local + 1)));
+    {
+      DBuf<char> tmp(c);
+      SV_TRY(tmp.alloc(prefix128_temp_bytes(n3_local)));
+      launch_prefix128(keys.get(), n3_local, xmask, P1.get(), P2.get(), tmp.get(), S);
+    }
+    SV_CUDA(cudaGetLastError());
+  }
+  const u64 nkeys = (n_t3 && n3_local) ? n3_local : 0;
+
+  // ---------------- refinement rounds (A6-A15) ------------------------------------------
+  DBuf<unsigned long long> terms(c);
+  SV_TRY(terms.alloc(2));
+  SV_CUDA(cudaMemsetAsync(terms.get(), 0, 16, S));
+  u32 round = 0;
+  const u32 tstride = G / 2 + 1;
+  const u32 tps = div_up(G, KDE_TJ);
+  while (!open.empty()) {
+    round++;
+    if (round > P->max_rounds) return sv_fail(SIEVE_ELIMIT, "Tier-3 refinement exceeded max_rounds");
+    const u32 nseg = (u32)open.size();
+    std::vector<SegDev> hs(nseg);
+    std::vector<double> hh(nseg);
+    for (u32 s = 0; s < nseg; s++) {
+      const OpenSeg& o = open[s];
+      double h = scott_h(o.n, o.s1, o.s2, P->bw_scale);
+      hh[s] = h;
+      u64 base = (u64)o.t3rank << bx;
+      hs[s].key_lo = base + o.lo;
+      hs[s].key_hi = base + o.hi;
+      hs[s].lo = o.lo;
+      hs[s].hi = o.hi;
+      hs[s].h = h;
+      hs[s].inv_h = 1.0 / h;
+      hs[s].begin = hs[s].end = 0;
+    }
+    DBuf<SegDev> segs(c);
+    SV_TRY(segs.alloc(nseg));
+    SV_TRY(h2d(c, segs.get(), hs));
+    DBuf<u64> D(c);
+    SV_TRY(D.alloc((size_t)nseg * G * 2));
+    SV_CUDA(cudaMemsetAsync(D.get(), 0, (size_t)nseg * G * 16, S));
+    if (nkeys) {
+      launch_seg_ranges(segs.get(), nseg, keys.get(), nkeys, S);
+      DBuf<u64> tile_range(c);
+      DBuf<u32> tile_items(c);
+      DBuf<char> stemp(c);
+      SV_TRY(tile_range.alloc((size_t)nseg * tps * 2));
+      SV_TRY(tile_items.alloc((size_t)nseg * tps + 1));
+      SV_TRY(stemp.alloc(((size_t)nseg * tps / 4096 + 4) * 4));
+      u32 items = 0;
+      SV_TRY(kde_plan(segs.get(), nseg, G, keys.get(), nkeys, xmask, tile_range.get(),
+                      tile_items.get(), stemp.get(), &items, S));
+      launch_kde(segs.get(), nseg, G, keys.get(), xmask, tile_range.get(), tile_items.get(), items,
+                 D.get(), counter.get() + 1, terms.get(), S);
+      SV_CUDA(cudaGetLastError());
+    }
+    if (c->comm) {  // AR-2: densities as 32-bit limbs
+      DBuf<u64> lim(c);
+      SV_TRY(lim.alloc((size_t)nseg * G * 4));
+      launch_u128_to_limbs(D.get(), (u64)nseg * G, lim.get(), S);
+      SV_TRY(allreduce(c, lim.get(), (size_t)nseg * G * 4, RED_SUM));
+      launch_limbs_to_u128(lim.get(), (u64)nseg * G, D.get(), S);
+    }
+    DBuf<u64> T(c);
+    DBuf<u32> ntk(c);
+    SV_TRY(T.alloc((size_t)nseg * tstride));
+    SV_TRY(ntk.alloc((size_t)nseg * 2));
+    launch_valleys(segs.get(), nseg, G, P->valley_shift, D.get(), T.get(), tstride, ntk.get(),
+                   ntk.get() + nseg, S);
+    std::vector<u32> h_ntk;
+    SV_TRY(d2h(c, h_ntk, ntk.get(), (size_t)nseg * 2));
+    SV_TRY(sync(c));
+    std::vector<u32> part_off(nseg + 1);
+    u32 nparts = 0;
+    for (u32 s = 0; s < nseg; s++) { part_off[s] = nparts; nparts += h_ntk[s] + 1; }
+    part_off[nseg] = nparts;
+    DBuf<u32> d_off(c);
+    SV_TRY(d_off.alloc(nseg + 1));
+    SV_TRY(h2d(c, d_off.get(), part_off));
+    DBuf<u64> pl(c), pm(c), pab(c);
+    SV_TRY(pl.alloc((size_t)nparts * MOM_LANES));
+    SV_TRY(pm.alloc((size_t)nparts * 2));
+    SV_TRY(pab.alloc((size_t)nparts * 2));
+    launch_part_stats(segs.get(), nseg, T.get(), tstride, ntk.get(), d_off.get(), nparts,
+                      nkeys ? keys.get() : nullptr, nkeys, bx, P1.get(), P2.get(), pl.get(),
+                      pm.get(), pab.get(), S);
+    SV_CUDA(cudaGetLastError());
+    SV_TRY(allreduce(c, pl.get(), (size_t)nparts * MOM_LANES, RED_SUM));   // AR-3
+    SV_TRY(allreduce(c, pm.get(), nparts, RED_MIN));
+    SV_TRY(allreduce(c, pm.get() + nparts, nparts, RED_MAX));
+    std::vector<u64> h_pl, h_pm, h_ab;
+    SV_TRY(d2h(c, h_pl, pl.get(), (size_t)nparts * MOM_LANES));
+    SV_TRY(d2h(c, h_pm, pm.get(), (size_t)nparts * 2));
+    SV_TRY(d2h(c, h_ab, pab.get(), (size_t)nparts * 2));
+    std::vector<u64> h_D, h_T;
+    if (R->keep_debug) {
+      SV_TRY(d2h(c, h_D, D.get(), (size_t)nseg * G * 2));
+      SV_TRY(d2h(c, h_T, T.get(), (size_t)nseg * tstride));
+    }
+    SV_TRY(sync(c));
+    std::vector<OpenSeg> next;
+    for (u32 s = 0; s < nseg; s++) {
+      if (R->keep_debug) {
+        SegDebug sd;
+        sd.meta.kernel_id = open[s].kid;
+        sd.meta.round = round;
+        sd.meta.split_kind = h_ntk[nseg + s];
+        sd.meta.n_cuts = h_ntk[s];
+        sd.meta.lo = open[s].lo;
+        sd.meta.hi = open[s].hi;
+        sd.meta.count = open[s].n;
+        sd.meta.bandwidth = hh[s];
+        sd.dlo.resize(G); sd.dhi.resize(G);
+        for (u32 j = 0; j < G; j++) {
+          sd.dlo[j] = h_D[2 * ((size_t)s * G + j)];
+          sd.dhi[j] = h_D[2 * ((size_t)s * G + j) + 1];
+        }
+        sd.cuts.assign(h_T.begin() + (size_t)s * tstride, h_T.begin() + (size_t)s * tstride + h_ntk[s]);
+        R->segs.push_back(std::move(sd));
+      }
+      for (u32 p = part_off[s]; p < part_off[s + 1]; p++) {
+        const u64* L = &h_pl[(size_t)p * MOM_LANES];
+        u64 pn = L[0];
+        if (!pn) continue;  // empty part: dropped (A13 f)
+        u128 s1 = limbs_u128(L + 1), s2 = limbs_u128(L + 5);
+        u64 lo = h_pm[p], hi = h_pm[nparts + p];
+        if (lo == hi || cov_lt(pn, s1, s2, P->theta_num, P->theta_den))
+          fin.push_back({open[s].kid, 3, lo, hi, pn, s1, hh[s], round});
+        else
+          next.push_back({open[s].kid, open[s].t3rank, lo, hi, pn, s1, s2});
+      }
+    }
+    open.swap(next);
+  }
+  R->rounds = round;
+  {
+    std::vector<unsigned long long> ht;
+    SV_TRY(d2h(c, ht, terms.get(), 1));
+    SV_TRY(sync(c));
+    R->kde_terms = ht[0];
+  }
+  P1.release(); P2.release(); keys.release();
+
+  // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
+  std::sort(fin.begin(), fin.end(), [](const Fin& a, const Fin& b) {
+    return a.kid != b.kid ? a.kid < b.kid : a.lo < b.lo;
+  });
+  const u32 ns = (u32)fin.size();
+  std::vector<KTab> ktab(K, KTab{0, 0, 0, 0});
+  std::vector<u64> lows;
+  std::vector<u32> tiers(ns);
+  for (u32 s = 0; s < ns; s++) {
+    const Fin& f = fin[s];
+    tiers[s] = f.tier;
+    KTab& e = ktab[f.kid];
+    if (e.m == 0) { e.base = s; e.lows_off = (u32)lows.size(); }
+    else lows.push_back(f.lo);
+    e.m++;
+  }
+  // lows for a kernel with m strata are its strata 1..m-1 lower bounds, contiguous per kernel
+  // (pushed in order above because fin is sorted by (kid, lo))
+  if (lows.empty()) lows.push_back(0);
+
+  // ---------------- pass B: assignment + (stratum, CTA) statistics ---------------------
+  DBuf<KTab> d_ktab(c);
+  DBuf<u64> d_lows(c), errf(c);
+  SV_TRY(d_ktab.alloc(K));
+  SV_TRY(d_lows.alloc(lows.size()));
+  SV_TRY(errf.alloc(4));
+  SV_TRY(h2d(c, d_ktab.get(), ktab));
+  SV_TRY(h2d(c, d_lows.get(), lows));
+  u64 cap = 1;
+  while (cap < std::max<u64>(1u << 16, 8ull * ns)) cap <<= 1;
+  DBuf<u64> gkeys(c), gcnt(c), gfirst(c);
+  u64 E = 0;
+  DBuf<u64> ekey(c), ecnt(c), efirst(c);
+  for (int attempt = 0;; attempt++) {
+    SV_TRY(gkeys.alloc(cap)); SV_TRY(gcnt.alloc(cap)); SV_TRY(gfirst.alloc(cap));
+    launch_fill_u64(gkeys.get(), cap, HASH_EMPTY, S);
+    SV_CUDA(cudaMemsetAsync(gcnt.get(), 0, cap * 8, S));
+    launch_fill_u64(gfirst.get(), cap, ~0ull, S);
+    SV_CUDA(cudaMemsetAsync(errf.get(), 0, 32, S));
+    GHash gh{gkeys.get(), gcnt.get(), gfirst.get(), cap};
+    launch_assign(t->kid, t->x, t->cta, n, t->first_id, d_ktab.get(), d_lows.get(), sid_out, gh,
+                  errf.get(), assign_grid(), S);
+    SV_CUDA(cudaGetLastError());
+    SV_TRY(ekey.alloc(cap)); SV_TRY(ecnt.alloc(cap)); SV_TRY(efirst.alloc(cap));
+    SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
+    launch_hash_compact(gh, ekey.get(), ecnt.get(), efirst.get(), counter.get(), S);
+    std::vector<u64> hflag;
+    std::vector<unsigned long long> hcnt;
+    SV_TRY(d2h(c, hflag, errf.get(), 4));
+    SV_TRY(d2h(c, hcnt, counter.get(), 1));
+    SV_TRY(sync(c));
+    // the retry decision must be identical on every rank
+    DBuf<u64> fl(c);
+    SV_TRY(fl.alloc(1));
+    SV_TRY(h2d(c, fl.get(), std::vector<u64>{hflag[2]}));
+    SV_TRY(allreduce(c, fl.get(), 1, RED_MAX));
+    std::vector<u64> gfl;
+    SV_TRY(d2h(c, gfl, fl.get(), 1));
+    SV_TRY(sync(c));
+    if (!gfl[0]) { E = hcnt[0]; break; }
+    if (attempt > 6) return sv_fail(SIEVE_ENOMEM, "(stratum, CTA) table kept overflowing");
+    cap <<= 2;
+  }
+  gkeys.release(); gcnt.release(); gfirst.release();
+  // gather every rank's entries (AR-4: all-gather expressed as a SUM over zero-padded slots)
+  u64 Etot = E, Eoff = 0;
+  DBuf<u64> ak(c), ac(c), af(c);
+  if (c->comm) {
+    DBuf<u64> cnts(c);
+    SV_TRY(cnts.alloc(c->world));
+    std::vector<u64> mine(c->world, 0);
+    mine[c->rank] = E;
+    SV_TRY(h2d(c, cnts.get(), mine));
+    SV_TRY(allreduce(c, cnts.get(), c->world, RED_SUM));
+    std::vector<u64> all;
+    SV_TRY(d2h(c, all, cnts.get(), c->world));
+    SV_TRY(sync(c));
+    Etot = 0;
+    for (int r = 0; r < c->world; r++) { if (r == c->rank) Eoff = Etot; Etot += all[r]; }
+    SV_TRY(ak.alloc(Etot * 3));
+    SV_CUDA(cudaMemsetAsync(ak.get(), 0, Etot * 3 * 8, S));
+    SV_CUDA(cudaMemcpyAsync(ak.get() + Eoff, ekey.get(), E * 8, cudaMemcpyDeviceToDevice, S));
+    SV_CUDA(cudaMemcpyAsync(ak.get() + Etot + Eoff, ecnt.get(), E * 8, cudaMemcpyDeviceToDevice, S));
+    SV_CUDA(cudaMemcpyAsync(ak.get() + 2 * Etot + Eoff, efirst.get(), E * 8, cudaMemcpyDeviceToDevice, S));
+    SV_TRY(allreduce(c, ak.get(), Etot * 3, RED_SUM));
+  } else {
+    SV_TRY(ak.alloc(Etot * 3));
+    SV_CUDA(cudaMemcpyAsync(ak.get(), ekey.get(), E * 8, cudaMemcpyDeviceToDevice, S));
+    SV_CUDA(cudaMemcpyAsync(ak.get() + Etot, ecnt.get(), E * 8, cudaMemcpyDeviceToDevice, S));
+    SV_CUDA(cudaMemcpyAsync(ak.get() + 2 * Etot, efirst.get(), E * 8, cudaMemcpyDeviceToDevice, S));
+  }
+  ekey.release(); ecnt.release(); efirst.release();
+  // sort entries by (stratum, CTA) with their index as payload, then gather count / first
+  DBuf<u32> idx(c);
+  DBuf<u64> sk(c), scnt(c), sfirst(c);
+  SV_TRY(idx.alloc(Etot));
+  SV_TRY(sk.alloc(Etot)); SV_TRY(scnt.alloc(Etot)); SV_TRY(sfirst.alloc(Etot));
+  {
+    std::vector<u32> iota(Etot);
+    for (u64 i = 0; i < Etot; i++) iota[i] = (u32)i;
+    SV_TRY(h2d(c, idx.get(), iota));
+  }
+  SV_CUDA(cudaMemcpyAsync(sk.get(), ak.get(), Etot * 8, cudaMemcpyDeviceToDevice, S));
+  {
+    DBuf<char> tmp(c);
+    SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
+    SV_TRY(radix_sort(sk.get(), idx.get(), Etot, 32 + (int)bitlen(ns ? ns - 1 : 0), tmp.get(), S));
+  }
+  launch_gather_u64(ak.get() + Etot, idx.get(), Etot, scnt.get(), S);
+  launch_gather_u64(ak.get() + 2 * Etot, idx.get(), Etot, sfirst.get(), S);
+  DBuf<u32> d_tier(c);
+  DBuf<u64> rep(c), repxy(c);
+  SV_TRY(d_tier.alloc(ns));
+  SV_TRY(rep.alloc(2 * (size_t)ns));
+  SV_TRY(repxy.alloc(2 * (size_t)ns));
+  SV_TRY(h2d(c, d_tier.get(), tiers));
+  launch_reps(sk.get(), scnt.get(), sfirst.get(), Etot, d_tier.get(), ns, rep.get(), rep.get() + ns, S);
+  launch_rep_xy(rep.get(), ns, t->first_id, n, t->x, t->y, repxy.get(), S);
+  SV_CUDA(cudaGetLastError());
+  SV_TRY(allreduce(c, repxy.get(), 2 * (size_t)ns, RED_SUM));   // AR-5: owner contributes
+  std::vector<u64> h_rep, h_xy;
+  SV_TRY(d2h(c, h_rep, rep.get(), 2 * (size_t)ns));
+  SV_TRY(d2h(c, h_xy, repxy.get(), 2 * (size_t)ns));
+  SV_TRY(sync(c));
+
+  // ---------------- assemble --------------------------------------------------------------------
+  R->st.resize(ns);
+  std::vector<u32> first_of(K, 0xFFFFFFFFu);
+  for (u32 s = 0; s < ns; s++) {
+    const Fin& f = fin[s];
+    sieve_stratum& o = R->st[s];
+    memset(&o, 0, sizeof o);
+    if (first_of[f.kid] == 0xFFFFFFFFu) first_of[f.kid] = s;
+    o.kernel_id = f.kid;
+    o.tier = f.tier;
+    o.index_in_kernel = s - first_of[f.kid];
+    o.rep_cta = (u32)h_rep[ns + s];
+    o.lo = f.lo; o.hi = f.hi; o.count = f.n;
+    o.instr_sum_lo = (u64)f.s1; o.instr_sum_hi = (u64)(f.s1 >> 64);
+    o.rep_id = h_rep[s];
+    o.rep_instr = h_xy[2 * (size_t)s];
+    o.rep_cycles = h_xy[2 * (size_t)s + 1];
+    o.bandwidth = f.h;
+    o.split_round = f.round;
+  }
+  return SIEVE_OK;
+}
+
+extern "C" int sieve_stratify(sieve_trace t, const sieve_params* p, uint32_t* sid_out, sieve_strata* out) {
+  if (!out) return sv_fail(SIEVE_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!trace_ok(t)) return sv_fail(SIEVE_EINVAL, "bad trace handle");
+  sieve_params P;
+  if (p) P = *p; else sieve_params_default(&P);
+  if (P.theta_num == 0 || P.theta_den == 0) return sv_fail(SIEVE_EINVAL, "theta must be a positive fraction");
+  if (P.grid_points < 3 || P.grid_points > 65536) return sv_fail(SIEVE_EINVAL, "grid_points must be in [3, 65536]");
+  if (P.valley_shift > 120) return sv_fail(SIEVE_EINVAL, "valley_shift must be <= 120");
+  if (!(P.bw_scale > 0)) return sv_fail(SIEVE_EINVAL, "bw_scale must be > 0");
+  if (P.max_rounds == 0) P.max_rounds = 1;
+  sieve_ctx c = t->ctx;
+  SV_CUDA(cudaSetDevice(c->device));
+  sieve_strata_s* R = new sieve_strata_s();
+  R->ctx = c;
+  R->G = P.grid_points;
+  R->keep_debug = P.keep_debug != 0;
+  R->has_cycles = t->y != nullptr;
+  int st = stratify_impl(t, &P, sid_out, R);
+  if (st != SIEVE_OK) {
+    cudaStreamSynchronize(c->stream);
+    delete R;
+    return st;
+  }
+  *out = R;
+  return SIEVE_OK;
+}
+
+extern "C" int sieve_strata_count(sieve_strata s, uint64_t* n) {
+  if (!strata_ok(s) || !n) return sv_fail(SIEVE_EINVAL, "bad strata handle");
+  *n = s->st.size();
+  return SIEVE_OK;
+}
+extern "C" int sieve_strata_copy(sieve_strata s, sieve_stratum* host_out, uint64_t cap) {
+  if (!strata_ok(s) || (!host_out && cap)) return sv_fail(SIEVE_EINVAL, "bad strata handle");
+  u64 m = std::min<u64>(cap, s->st.size());
+  if (m) memcpy(host_out, s->st.data(), m * sizeof(sieve_stratum));
+  return SIEVE_OK;
+}
+extern "C" int sieve_strata_stats(sieve_strata s, uint32_t* rounds, uint64_t* terms) {
+  if (!strata_ok(s)) return sv_fail(SIEVE_EINVAL, "bad strata handle");
+  if (rounds) *rounds = s->rounds;
+  if (terms) *terms = s->kde_terms;
+  return SIEVE_OK;
+}
+extern "C" void sieve_strata_free(sieve_strata s) {
+  if (!strata_ok(s)) return;
+  s->magic = 0;
+  delete s;
+}
+extern "C" int sieve_segment_count(sieve_strata s, uint64_t* n) {
+  if (!strata_ok(s) || !n) return sv_fail(SIEVE_EINVAL, "bad strata handle");
+  if (!s->keep_debug) return sv_fail(SIEVE_ESTATE, "stratify was called without keep_debug");
+  *n = s->segs.size();
+  return SIEVE_OK;
+}
+extern "C" int sieve_segment_get(sieve_strata s, uint64_t idx, sieve_segment* out, uint64_t* dlo,
+                                 uint64_t* dhi, uint64_t* cuts) {
+  if (!strata_ok(s)) return sv_fail(SIEVE_EINVAL, "bad strata handle");
+  if (!s->keep_debug) return sv_fail(SIEVE_ESTATE, "stratify was called without keep_debug");
+  if (idx >= s->segs.size()) return sv_fail(SIEVE_EINVAL, "segment index out of range");
+  const SegDebug& d = s->segs[idx];
+  if (out) *out = d.meta;
+  if (dlo) memcpy(dlo, d.dlo.data(), d.dlo.size() * 8);
+  if (dhi) memcpy(dhi, d.dhi.data(), d.dhi.size() * 8);
+  if (cuts) memcpy(cuts, d.cuts.data(), d.cuts.size() * 8);
+  return SIEVE_OK;
+}
+
+// ------------------------------------------------------------------------------------------
+// sieve_predict
+// ------------------------------------------------------------------------------------------
+static double u128_to_double_host(u128 v) { return (double)v; }  // libgcc: correctly rounded
+
+extern "C" int sieve_predict(sieve_strata s, sieve_trace t, const uint64_t* rep_cycles, sieve_prediction* out) {
+  if (!strata_ok(s) || !trace_ok(t) || !out) return sv_fail(SIEVE_EINVAL, "bad handle");
+  if (!rep_cycles && !s->has_cycles) return sv_fail(SIEVE_EDOM, "no cycle source for the representatives");
+  sieve_ctx c = t->ctx;
+  SV_CUDA(cudaSetDevice(c->device));
+  const u32 ns = (u32)s->st.size();
+  std::vector<u64> hW(2 * (size_t)ns), hx(ns), hy(ns);
+  for (u32 i = 0; i < ns; i++) {
+    hW[2 * i] = s->st[i].instr_sum_lo;
+    hW[2 * i + 1] = s->st[i].instr_sum_hi;
+    hx[i] = s->st[i].rep_instr;
+    hy[i] = rep_cycles ? rep_cycles[i] : s->st[i].rep_cycles;
+  }
+  DBuf<u64> dW(c), dx(c), dy(c);
+  DBuf<double> dout(c);
+  SV_TRY(dW.alloc(hW.size())); SV_TRY(dx.alloc(ns)); SV_TRY(dy.alloc(ns)); SV_TRY(dout.alloc(4));
+  SV_TRY(h2d(c, dW.get(), hW)); SV_TRY(h2d(c, dx.get(), hx)); SV_TRY(h2d(c, dy.get(), hy));
+  launch_predict(dW.get(), dx.get(), dy.get(), ns, dout.get(), c->stream);
+  SV_CUDA(cudaGetLastError());
+  std::vector<double> r;
+  SV_TRY(d2h(c, r, dout.get(), 4));
+  SV_TRY(sync(c));
+  out->predicted_cycles = r[0];
+  out->predicted_ipc = r[3];
+  out->total_instr_lo = (u64)s->total_instr;
+  out->total_instr_hi = (u64)(s->total_instr >> 64);
+  if (s->has_cycles) {
+    double cm = u128_to_double_host(s->c_meas);
+    out->measured_cycles = cm;
+    out->error = s->c_meas == 0 ? NAN : fabs(r[0] - cm) / cm;
+    out->speedup = cm / r[1];
+  } else {
+    out->measured_cycles = NAN;
+    out->error = NAN;
+    out->speedup = NAN;
+  }
+  return SIEVE_OK;
+}

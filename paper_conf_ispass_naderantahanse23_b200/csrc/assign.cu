@@ -1,0 +1,222 @@
+// assign.cu -- pass B: assign every invocation to its stratum and gather, per (stratum, CTA
+// size), the count and the first-chronological invocation id; then pick each stratum's
+// representative (footnote P:103):
+//   Tier-1: the first-chronological invocation;
+//   Tier-2/3: the first-chronological invocation with the most dominant CTA size
+//             (max count; a tie goes to the CTA size seen first, A17).
+//
+// B200 design: one coalesced pass (kernel id, x, CTA in; stratum id out).  Stratum lookup is a
+// per-kernel table plus a branch-free binary search over the kernel's stratum lower bounds.
+// (stratum, CTA) statistics use a block-private open-addressing hash table in shared memory
+// (native 32-bit atomics for counts and first offsets; 64-bit CAS only on first insertion),
+// flushed into an L2-resident global table when half full and at the end of the block's range.
+// The global table's contents (not its slot order) are deterministic; entries are compacted,
+// gathered across ranks, radix-sorted by key and reduced, so the result is identical for any
+// number of ranks or blocks.
+#include "kernels.cuh"
+
+#define AS_THREADS 512
+#define AS_IPT 4
+#define AS_HC 4096          // shared hash capacity (entries)
+#define AS_MAXP 32          // probes before falling back to the global table
+
+int assign_grid() { return 2 * sv_num_sms(); }
+
+__device__ __forceinline__ u32 hash_key(u64 k) {
+  return (u32)((k * 0x9E3779B97F4A7C15ull) >> 32);
+}
+
+__device__ void ghash_update(GHash gh, u64 key, u64 cnt, u64 first, u64* errflags) {
+  u64 h = (u64)hash_key(key) & (gh.cap - 1);
+  for (u64 probe = 0; probe < gh.cap; probe++) {
+    u64 cur = gh.keys[h];
+    if (cur == HASH_EMPTY) {
+      cur = atomicCAS((unsigned long long*)&gh.keys[h], HASH_EMPTY, key);
+      if (cur == HASH_EMPTY) cur = key;
+    }
+    if (cur == key) {
+      atomicAdd((unsigned long long*)&gh.cnt[h], (unsigned long long)cnt);
+      atomicMin((unsigned long long*)&gh.first[h], (unsigned long long)first);
+      return;
+    }
+    h = (h + 1) & (gh.cap - 1);
+  }
+  atomicMax((unsigned long long*)&errflags[2], 1ull);  // global table full: caller retries bigger
+}
+
+__global__ void __launch_bounds__(AS_THREADS)
+k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __restrict__ cta,
+         u64 n, u64 first_id, const KTab* __restrict__ ktab, const u64* __restrict__ lows,
+         u32* __restrict__ sid_out, GHash gh, u64* errflags) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  u64* hk = (u64*)smem;              // [AS_HC]
+  u32* hc = (u32*)(hk + AS_HC);      // [AS_HC]
+  u32* hf = hc + AS_HC;              // [AS_HC]
+  __shared__ u32 s_fill;
+  for (u32 i = threadIdx.x; i < AS_HC; i += AS_THREADS) { hk[i] = HASH_EMPTY; hc[i] = 0; hf[i] = 0xFFFFFFFFu; }
+  if (threadIdx.x == 0) s_fill = 0;
+  __syncthreads();
+  u64 chunk = (n + gridDim.x - 1) / gridDim.x;
+  u64 b0 = (u64)blockIdx.x * chunk;
+  u64 b1 = b0 + chunk < n ? b0 + chunk : n;
+  const u64 tile = (u64)AS_THREADS * AS_IPT;
+  for (u64 base = b0; base < b1; base += tile) {
+#pragma unroll
+    for (int j = 0; j < AS_IPT; j++) {
+      u64 i = base + (u64)j * AS_THREADS + threadIdx.x;
+      if (i >= b1) continue;
+      u32 k = __ldcs(kid + i);
+      u64 v = __ldcs(x + i);
+      KTab kt = ktab[k];
+      u32 sid = kt.base;
+      if (kt.m > 1) {  // number of lower bounds lows[1..m) that are <= v
+        const u64* L = lows + kt.lows_off;
+        u32 lo = 0, cnt = kt.m - 1;
+        while (cnt > 0) {
+          u32 half = cnt >> 1;
+          if (L[lo + half] <= v) { lo += half + 1; cnt -= half + 1; } else cnt = half;
+        }
+        sid += lo;
+      }
+      if (sid_out) sid_out[i] = sid;
+      u32 c = cta ? __ldcs(cta + i) : 0u;
+      u64 key = ((u64)sid << 32) | c;
+      u32 rel = (u32)(i - b0);
+      u32 h = hash_key(key) & (AS_HC - 1);
+      bool done = false;
+      for (int p = 0; p < AS_MAXP; p++) {
+        u64 cur = hk[h];
+        if (cur == HASH_EMPTY) {
+          cur = atomicCAS((unsigned long long*)&hk[h], HASH_EMPTY, key);
+          if (cur == HASH_EMPTY) { atomicAdd(&s_fill, 1u); cur = key; }
+        }
+        if (cur == key) {
+          atomicAdd(&hc[h], 1u);
+          atomicMin(&hf[h], rel);
+          done = true;
+          break;
+        }
+        h = (h + 1) & (AS_HC - 1);
+      }
+      if (!done) ghash_update(gh, key, 1, first_id + i, errflags);
+    }
+    __syncthreads();
+    bool last = base + tile >= b1;
+    if (s_fill > AS_HC / 2 || last) {
+      for (u32 e = threadIdx.x; e < AS_HC; e += AS_THREADS) {
+        u64 key = hk[e];
+        if (key != HASH_EMPTY) {
+          ghash_update(gh, key, hc[e], first_id + b0 + hf[e], errflags);
+          hk[e] = HASH_EMPTY; hc[e] = 0; hf[e] = 0xFFFFFFFFu;
+        }
+      }
+      __syncthreads();
+      if (threadIdx.x == 0) s_fill = 0;
+      __syncthreads();
+    }
+  }
+}
+
+void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 first_id,
+                   const KTab* ktab, const u64* lows, u32* sid_out, GHash gh, u64* errflags,
+                   int grid, cudaStream_t s) {
+  if (n == 0) return;
+  size_t smem = (size_t)AS_HC * (8 + 4 + 4);
+  cudaFuncSetAttribute(k_assign, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  u64 maxgrid = (n + (u64)AS_THREADS * AS_IPT - 1) / ((u64)AS_THREADS * AS_IPT);
+  if ((u64)grid > maxgrid) grid = (int)maxgrid;
+  k_assign<<<grid, AS_THREADS, smem, s>>>(kid, x, cta, n, first_id, ktab, lows, sid_out, gh, errflags);
+}
+
+__global__ void k_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst,
+                               unsigned long long* count) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  bool occ = i < gh.cap && gh.keys[i] != HASH_EMPTY;
+  u32 m = __ballot_sync(0xffffffffu, occ);
+  unsigned long long base = 0;
+  if (lane_id() == 0 && m) base = atomicAdd(count, (unsigned long long)__popc(m));
+  base = __shfl_sync(0xffffffffu, base, 0);
+  if (occ) {
+    u64 o = base + __popc(m & ((1u << lane_id()) - 1u));
+    okey[o] = gh.keys[i];
+    ocnt[o] = gh.cnt[i];
+    ofirst[o] = gh.first[i];
+  }
+}
+
+void launch_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst, unsigned long long* count,
+                         cudaStream_t s) {
+  k_hash_compact<<<div_up(gh.cap, 256), 256, 0, s>>>(gh, okey, ocnt, ofirst, count);
+}
+
+__global__ void k_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) dst[i] = src[idx[i]];
+}
+void launch_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst, cudaStream_t s) {
+  if (n) k_gather_u64<<<div_up(n, 256), 256, 0, s>>>(src, idx, n, dst);
+}
+
+// one thread per stratum over its (sorted) entries; equal keys (from different ranks) merge
+__global__ void k_reps(const u64* key, const u64* cnt, const u64* first, u64 E, const u32* tier,
+                       u32 nstrata, u64* rep_id, u64* rep_cta) {
+  u32 s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= nstrata) return;
+  u64 lo = 0, hi = E;
+  u64 kv = (u64)s << 32;
+  while (lo < hi) { u64 m = (lo + hi) >> 1; if (key[m] < kv) lo = m + 1; else hi = m; }
+  u64 best_c = 0, best_f = ~0ull, best_k = 0;   // dominant CTA (count desc, first asc)
+  u64 min_f = ~0ull, min_k = 0;                 // first-chronological overall
+  u64 i = lo;
+  while (i < E && (key[i] >> 32) == s) {
+    u64 k = key[i], c = 0, f = ~0ull;
+    while (i < E && key[i] == k) { c += cnt[i]; f = first[i] < f ? first[i] : f; i++; }
+    if (c > best_c || (c == best_c && f < best_f)) { best_c = c; best_f = f; best_k = k; }
+    if (f < min_f) { min_f = f; min_k = k; }
+  }
+  if (tier[s] == 1) { rep_id[s] = min_f; rep_cta[s] = min_k & 0xFFFFFFFFull; }
+  else { rep_id[s] = best_f; rep_cta[s] = best_k & 0xFFFFFFFFull; }
+}
+
+void launch_reps(const u64* key, const u64* cnt, const u64* first, u64 E, const u32* tier,
+                 u32 nstrata, u64* rep_id, u64* rep_cta, cudaStream_t s) {
+  if (nstrata) k_reps<<<div_up(nstrata, 128), 128, 0, s>>>(key, cnt, first, E, tier, nstrata, rep_id, rep_cta);
+}
+
+__global__ void k_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, const u64* x,
+                         const u64* y, u64* out) {
+  u32 s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= nstrata) return;
+  u64 r = rep_id[s];
+  bool mine = r >= first_id && r - first_id < n_local;
+  out[2 * (u64)s] = mine ? x[r - first_id] : 0;
+  out[2 * (u64)s + 1] = (mine && y) ? y[r - first_id] : 0;
+}
+
+void launch_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, const u64* x,
+                   const u64* y, u64* out, cudaStream_t s) {
+  if (nstrata) k_rep_xy<<<div_up(nstrata, 128), 128, 0, s>>>(rep_id, nstrata, first_id, n_local, x, y, out);
+}
+
+// ------------------------------------------------------------------------------------------
+__global__ void k_fill_u64(u64* p, u64 n, u64 v) {
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) p[i] = v;
+}
+void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s) {
+  if (n) k_fill_u64<<<min(div_up(n, 256), 4096u), 256, 0, s>>>(p, n, v);
+}
+
+__global__ void k_u128_to_limbs(const u64* src, u64 n, u64* limbs) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) limbs_from_u128(src[2 * i], src[2 * i + 1], limbs + 4 * i);
+}
+__global__ void k_limbs_to_u128(const u64* limbs, u64 n, u64* dst) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) limbs_to_u128(limbs + 4 * i, dst + 2 * i, dst + 2 * i + 1);
+}
+void launch_u128_to_limbs(const u64* src, u64 n, u64* limbs, cudaStream_t s) {
+  if (n) k_u128_to_limbs<<<div_up(n, 256), 256, 0, s>>>(src, n, limbs);
+}
+void launch_limbs_to_u128(const u64* limbs, u64 n, u64* dst, cudaStream_t s) {
+  if (n) k_limbs_to_u128<<<div_up(n, 256), 256, 0, s>>>(limbs, n, dst);
+}

@@ -1,0 +1,23 @@
+// comm.h -- cross-rank reductions on u64 lanes (SUM / MIN / MAX), the only collective the path
+// needs: every cross-rank quantity is additive (counts, 32-bit limbs of u128 sums, fixed-point
+// densities, per-(stratum, CTA) counts, owner-contributed representative values) or a min /
+// max (smallest / largest instruction count, first invocation id).  See DESIGN.md section 6.
+#pragma once
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include <stdint.h>
+
+#include "common.cuh"
+
+struct Comm {
+  int rank = 0, world = 1;
+  virtual ~Comm() {}
+  // in-place all-reduce of n u64 lanes on `s`; returns SIEVE_OK or an error status
+  virtual int allreduce(u64* buf, size_t n, ReduceOp op, cudaStream_t s) = 0;
+};
+
+int nccl_unique_id(uint8_t out[128]);
+int nccl_comm_create(int rank, int world, const uint8_t id[128], Comm** out);
+
+struct sieve_group_s;
+int group_comm_create(sieve_group_s* g, int rank, Comm** out);

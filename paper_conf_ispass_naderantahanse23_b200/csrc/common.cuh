@@ -1,0 +1,74 @@
+// common.cuh -- shared device/host helpers of libsieve (the product).  Nothing here is shared
+// with oracle/ (the CPU oracle is a separate, independent implementation).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "sieve.h"
+
+typedef unsigned long long u64;
+typedef unsigned int u32;
+typedef unsigned __int128 u128;
+
+#define SIEVE_MAX_K 65536u
+#define SIEVE_X_LIMIT (1ull << 44)
+
+// ------------------------------------------------------------------------------------------
+// error plumbing (host)
+// ------------------------------------------------------------------------------------------
+void sv_set_error(const std::string& msg);
+int sv_fail(int code, const std::string& msg);
+int sv_cuda(cudaError_t e, const char* what, int line);
+#define SV_CUDA(x)                                         \
+  do {                                                     \
+    cudaError_t _e = (x);                                  \
+    if (_e != cudaSuccess) return sv_cuda(_e, #x, __LINE__); \
+  } while (0)
+#define SV_TRY(x)            \
+  do {                       \
+    int _s = (x);            \
+    if (_s != SIEVE_OK) return _s; \
+  } while (0)
+
+// ------------------------------------------------------------------------------------------
+// reductions across ranks operate on u64 lanes; u128 values travel as 4 x 32-bit limbs
+// ------------------------------------------------------------------------------------------
+enum ReduceOp { RED_SUM = 0, RED_MIN = 1, RED_MAX = 2 };
+
+__host__ __device__ inline void limbs_from_u128(u64 lo, u64 hi, u64* l) {
+  l[0] = lo & 0xFFFFFFFFull;
+  l[1] = lo >> 32;
+  l[2] = hi & 0xFFFFFFFFull;
+  l[3] = hi >> 32;
+}
+
+// normalise 4 lanes that each hold a sum of 32-bit limbs (< 2^64) back to a u128
+__host__ __device__ inline void limbs_to_u128(const u64* l, u64* lo, u64* hi) {
+  u64 c = 0;
+  u64 w[4];
+  for (int i = 0; i < 4; i++) {
+    // l[i] + c can exceed 2^64 only if the true value overflowed u128 (never, by the bounds)
+    u64 s = l[i] + c;
+    w[i] = s & 0xFFFFFFFFull;
+    c = (s >> 32) + ((s < l[i]) ? (1ull << 32) : 0ull);
+  }
+  *lo = w[0] | (w[1] << 32);
+  *hi = w[2] | (w[3] << 32);
+}
+
+// device u128 accumulate into (lo, hi) words without __int128 on device paths
+__device__ __forceinline__ void add128(u64& lo, u64& hi, u64 alo, u64 ahi) {
+  u64 s = lo + alo;
+  hi += ahi + (s < lo ? 1ull : 0ull);
+  lo = s;
+}
+
+__device__ __forceinline__ u32 lane_id() { return threadIdx.x & 31u; }
+
+// ------------------------------------------------------------------------------------------
+// launch helpers
+// ------------------------------------------------------------------------------------------
+static inline unsigned div_up(u64 a, u64 b) { return (unsigned)((a + b - 1) / b); }
+int sv_num_sms();

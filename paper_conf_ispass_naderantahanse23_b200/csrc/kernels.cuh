@@ -1,0 +1,129 @@
+// kernels.cuh -- launchers of every sm_100a kernel on the stratification path, and the small
+// device-side tables they share.  See DESIGN.md section 5 for each kernel's roofline.
+#pragma once
+#include "common.cuh"
+
+// ---------------- pass A: per-kernel exact moments ----------------------------------
+// Per-block partial record per kernel (48 B): n, S1 (96-bit: lo + 32-bit hi), S2 (u128),
+// min and max instruction count.
+struct KMomPartial {
+  u32 n;
+  u32 s1hi;
+  u64 s1lo;
+  u64 s2lo, s2hi;
+  u64 mn, mx;
+};
+// Per-kernel result of pass A (before / after the cross-rank reduction):
+//   lanes[k*9 + 0] = n,  lanes[k*9 + 1..4] = S1 limbs,  lanes[k*9 + 5..8] = S2 limbs   (SUM)
+//   mm[k*2 + 0] = min x (MIN), mm[k*2 + 1] = max x (MAX)
+// totals: tot_lanes[0..3] = C_meas limbs (SUM); tot_max[0] = max x, tot_max[1] = error flags
+#define MOM_LANES 9
+#define ERRF_KID 1ull
+#define ERRF_RANGE 2ull
+
+struct MomentsScratch {
+  KMomPartial* part;   // [grid][kt]
+  u64* blk_tot;        // [grid][3]: C_meas lo, hi, max x
+  int grid;
+  u32 kt;
+};
+int moments_kt(u32 K);  // kernels per smem pass
+int moments_grid();
+void launch_moments(const u32* kid, const u64* x, const u64* y, u64 n, u32 K, u32 k0, u32 kt,
+                    KMomPartial* part, u64* blk_tot, u64* errflags, int grid, cudaStream_t s);
+void launch_moments_reduce(const KMomPartial* part, const u64* blk_tot, int grid, u32 k0, u32 kt,
+                           u32 K, u64* lanes, u64* mm, u64* local_n, u64* tot_lanes, u64* tot_max,
+                           bool do_totals, cudaStream_t s);
+
+// ---------------- Tier-3 key compaction ------------------------------------------------------
+// key = (t3rank(kid) << bx) + x ; t3rank = 0xFFFFFFFF for kernels not in Tier-3
+void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u32 bx,
+                       u64* keys_out, unsigned long long* counter, cudaStream_t s);
+
+// ---------------- LSD radix sort (u64 keys, optional u32 payload) ----------------------------
+size_t radix_sort_temp_bytes(u64 n, bool with_vals);
+// sorts keys[0..n) on bits [0, nbits); result in keys/vals (in place via internal ping-pong)
+int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s);
+
+// ---------------- prefix sums of x and x^2 over sorted Tier-3 keys -----------------------------
+// P1[i] = sum_{j<i} x_j, P2[i] = sum_{j<i} x_j^2, as u128 pairs (lo, hi), i in [0, n]
+size_t prefix128_temp_bytes(u64 n);
+void launch_prefix128(const u64* keys, u64 n, u64 xmask, u64* P1, u64* P2, void* temp,
+                      cudaStream_t s);
+
+// ---------------- KDE over open segments ([8], [36]; A6-A10) -----------------------------
+struct SegDev {
+  u64 key_lo;   // (t3rank << bx) + lo   -- first key of the segment's value range
+  u64 key_hi;   // (t3rank << bx) + hi   -- last key (inclusive)
+  u64 lo, hi;   // value range [lo, hi] (global, replicated)
+  double h, inv_h;
+  u64 begin, end; // local index range in the sorted keys (filled on device)
+};
+#define KDE_TJ 128      // grid points per tile (one thread each)
+#define KDE_CH 1024     // values per work item chunk (staged in shared memory)
+struct KdeScratch {
+  u64* tile_range;     // [nseg*tiles][2]
+  u32* tile_items;     // [nseg*tiles + 1] exclusive scan of chunks per tile
+  void* scan_temp;
+  unsigned long long* work_counter;
+};
+void launch_seg_ranges(SegDev* segs, u32 nseg, const u64* keys, u64 nkeys, cudaStream_t s);
+// returns total work items through *items_host (synchronises the stream once)
+int kde_plan(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 nkeys, u64 xmask,
+             u64* tile_range, u32* tile_items, void* scan_temp, u32* items_host, cudaStream_t s);
+void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
+                const u64* tile_range, const u32* tile_items, u32 items, u64* D /* [nseg][G][2] */,
+                unsigned long long* work_counter, unsigned long long* terms, cudaStream_t s);
+
+// ---------------- valleys and thresholds (A11-A13) ---------------------------------------------
+// T[s*tstride + q], nt[s], kind[s] (1 = valley, 2 = bisect)
+void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T,
+                    u32 tstride, u32* nt, u32* kind, cudaStream_t s);
+
+// ---------------- part moments (A13 f) ----------------------------------------------------------
+// parts of segment s: q = 0..nt[s]; part_off[s] = first part index (exclusive scan of nt+1)
+// out: lanes[p*9..] (n, S1 limbs, S2 limbs), mm[p*2..] (min, max), ab[p*2..] value interval
+void launch_part_stats(const SegDev* segs, u32 nseg, const u64* T, u32 tstride, const u32* nt,
+                       const u32* part_off, u32 nparts, const u64* keys, u64 nkeys, u32 bx,
+                       const u64* P1, const u64* P2, u64* lanes, u64* mm, u64* ab, cudaStream_t s);
+
+// ---------------- pass B: assignment + per-(stratum, CTA) statistics -------------------
+struct KTab {      // per kernel
+  u32 base;        // global id of its first stratum
+  u32 m;           // number of strata
+  u32 lows_off;    // offset of its strata lower bounds in `lows` (Tier-3 only)
+  u32 pad;
+};
+struct GHash {     // global (sid, cta) table
+  u64* keys;       // EMPTY = ~0
+  u64* cnt;
+  u64* first;
+  u64 cap;         // power of two
+};
+#define HASH_EMPTY 0xFFFFFFFFFFFFFFFFull
+int assign_grid();
+void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 first_id,
+                   const KTab* ktab, const u64* lows, u32* sid_out, GHash gh, u64* errflags,
+                   int grid, cudaStream_t s);
+// compact occupied entries into (key, cnt, first) arrays; *count (device) += entries
+void launch_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst, unsigned long long* count,
+                         cudaStream_t s);
+void launch_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst, cudaStream_t s);
+// reduce duplicates of equal keys (sorted) and pick each stratum's representative
+void launch_reps(const u64* key, const u64* cnt, const u64* first, u64 E, const u32* tier,
+                 u32 nstrata, u64* rep_id, u64* rep_cta, cudaStream_t s);
+// representative (x, y) from the owner rank: out[s*2] = x, out[s*2+1] = y (0 if not local)
+void launch_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, const u64* x,
+                   const u64* y, u64* out, cudaStream_t s);
+
+// ---------------- prediction ----------------------------------------------
+// strata: W (lo,hi), rep x, rep y ; out[0] = C_pred, out[1] = sum y_rep, out[2] = I (double),
+// out[3] = IPC
+void launch_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, double* out,
+                    cudaStream_t s);
+
+// ---------------- misc -------------------------------------------------------------------------
+void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s);
+// cross-rank encoding of u128 pairs [n][2] <-> 4 limbs [n][4]
+void launch_u128_to_limbs(const u64* src, u64 n, u64* limbs, cudaStream_t s);
+void launch_limbs_to_u128(const u64* limbs, u64 n, u64* dst, cudaStream_t s);

@@ -1,0 +1,310 @@
+"""Thin Python binding of libsieve.so (include/sieve.h): argument marshalling only.
+
+Every step of the stratification path runs in the library's sm_100a kernels.  PyTorch is used
+only for device memory (tensors), streams and process groups (the NCCL unique-id exchange).
+There is no CPU fallback: if libsieve.so is missing or cannot load, importing this module raises.
+
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    ctx = sieve.Ctx(device=0)
+    tr = sieve.load_trace(ctx, kid, x, num_kernels=K, cta=cta, cycles=y)   # numpy or CUDA tensors
+    st = sieve.stratify(tr)                 # -> Strata; st.table is a numpy structured array
+    pred = sieve.predict(st, tr)            # dict: predicted_cycles, predicted_ipc, error, ...
+"""
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsieve.so")
+
+SIEVE_OK, SIEVE_EINVAL, SIEVE_ERANGE, SIEVE_ENOMEM = 0, -1, -2, -3
+SIEVE_ECUDA, SIEVE_ENCCL, SIEVE_EDOM, SIEVE_ELIMIT, SIEVE_ESTATE = -4, -5, -6, -7, -8
+MEM_HOST, MEM_DEVICE, ADOPT = 0, 1, 2
+
+STRATUM_DTYPE = np.dtype([
+    ("kernel_id", "<u4"), ("tier", "<u4"), ("index_in_kernel", "<u4"), ("rep_cta", "<u4"),
+    ("lo", "<u8"), ("hi", "<u8"), ("count", "<u8"), ("instr_sum_lo", "<u8"), ("instr_sum_hi", "<u8"),
+    ("rep_id", "<u8"), ("rep_instr", "<u8"), ("rep_cycles", "<u8"), ("bandwidth", "<f8"),
+    ("split_round", "<u4"), ("pad", "<u4")])
+
+EXPORTED = [
+    "sieve_get_unique_id", "sieve_ctx_create", "sieve_group_create", "sieve_group_destroy",
+    "sieve_ctx_create_in_group", "sieve_ctx_set_allocator", "sieve_ctx_destroy",
+    "sieve_load_trace", "sieve_trace_free", "sieve_params_default", "sieve_stratify",
+    "sieve_strata_count", "sieve_strata_copy", "sieve_strata_stats", "sieve_strata_free",
+    "sieve_segment_count", "sieve_segment_get", "sieve_predict", "sieve_last_error",
+    "sieve_version", "sieve_u128_to_limbs", "sieve_limbs_to_u128",
+]
+
+
+class Params(ctypes.Structure):
+    _fields_ = [("theta_num", ctypes.c_uint32), ("theta_den", ctypes.c_uint32),
+                ("grid_points", ctypes.c_uint32), ("valley_shift", ctypes.c_uint32),
+                ("max_rounds", ctypes.c_uint32), ("keep_debug", ctypes.c_uint32),
+                ("bw_scale", ctypes.c_double)]
+
+
+class _Segment(ctypes.Structure):
+    _fields_ = [("kernel_id", ctypes.c_uint32), ("round", ctypes.c_uint32),
+                ("split_kind", ctypes.c_uint32), ("n_cuts", ctypes.c_uint32),
+                ("lo", ctypes.c_uint64), ("hi", ctypes.c_uint64), ("count", ctypes.c_uint64),
+                ("bandwidth", ctypes.c_double)]
+
+
+class _Prediction(ctypes.Structure):
+    _fields_ = [("predicted_cycles", ctypes.c_double), ("predicted_ipc", ctypes.c_double),
+                ("measured_cycles", ctypes.c_double), ("error", ctypes.c_double),
+                ("speedup", ctypes.c_double), ("total_instr_lo", ctypes.c_uint64),
+                ("total_instr_hi", ctypes.c_uint64)]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build it with `python -c 'import __graft_entry__ as g; "
+                          "g.build()'` (no CPU fallback exists)")
+    L = ctypes.CDLL(LIB_PATH, mode=ctypes.RTLD_GLOBAL)
+    vp, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+    P = ctypes.POINTER
+    sig = {
+        "sieve_get_unique_id": ([vp], i32),
+        "sieve_ctx_create": ([i32, vp, i32, i32, vp, P(vp)], i32),
+        "sieve_group_create": ([i32, P(vp)], i32),
+        "sieve_group_destroy": ([vp], None),
+        "sieve_ctx_create_in_group": ([i32, vp, vp, i32, P(vp)], i32),
+        "sieve_ctx_set_allocator": ([vp, vp, vp, vp], i32),
+        "sieve_ctx_destroy": ([vp], None),
+        "sieve_load_trace": ([vp, u64, u64, u32, vp, vp, vp, vp, u32, P(vp)], i32),
+        "sieve_trace_free": ([vp], None),
+        "sieve_params_default": ([P(Params)], None),
+        "sieve_stratify": ([vp, P(Params), vp, P(vp)], i32),
+        "sieve_strata_count": ([vp, P(u64)], i32),
+        "sieve_strata_copy": ([vp, vp, u64], i32),
+        "sieve_strata_stats": ([vp, P(u32), P(u64)], i32),
+        "sieve_strata_free": ([vp], None),
+        "sieve_segment_count": ([vp, P(u64)], i32),
+        "sieve_segment_get": ([vp, u64, P(_Segment), vp, vp, vp], i32),
+        "sieve_predict": ([vp, vp, vp, P(_Prediction)], i32),
+        "sieve_last_error": ([], ctypes.c_char_p),
+        "sieve_version": ([], ctypes.c_char_p),
+        "sieve_u128_to_limbs": ([u64, u64, vp], None),
+        "sieve_limbs_to_u128": ([vp, P(u64), P(u64)], None),
+    }
+    for name, (args, res) in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = res
+    return L
+
+
+_L = _load()
+
+
+class SieveError(RuntimeError):
+    def __init__(self, code, where):
+        msg = _L.sieve_last_error().decode(errors="replace")
+        super().__init__(f"{where} failed with status {code}: {msg}")
+        self.code = code
+
+
+def _check(code, where):
+    if code != SIEVE_OK:
+        raise SieveError(code, where)
+
+
+def version():
+    return _L.sieve_version().decode()
+
+
+def u128_to_limbs(v):
+    out = (ctypes.c_uint64 * 4)()
+    _L.sieve_u128_to_limbs(v & ((1 << 64) - 1), v >> 64, out)
+    return list(out)
+
+
+def limbs_to_u128(limbs):
+    arr = (ctypes.c_uint64 * 4)(*[int(l) for l in limbs])
+    lo, hi = ctypes.c_uint64(), ctypes.c_uint64()
+    _L.sieve_limbs_to_u128(arr, ctypes.byref(lo), ctypes.byref(hi))
+    return (hi.value << 64) | lo.value
+
+
+def get_unique_id():
+    buf = (ctypes.c_uint8 * 128)()
+    _check(_L.sieve_get_unique_id(buf), "sieve_get_unique_id")
+    return bytes(buf)
+
+
+def _stream_handle(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+class Group:
+    """In-process rank group: `world` threads share one GPU (multi-rank parity tests)."""
+
+    def __init__(self, world):
+        h = ctypes.c_void_p()
+        _check(_L.sieve_group_create(world, ctypes.byref(h)), "sieve_group_create")
+        self._h = h
+        self.world = world
+
+    def __del__(self):
+        if getattr(self, "_h", None):
+            _L.sieve_group_destroy(self._h)
+            self._h = None
+
+
+class Ctx:
+    """sieve_ctx: device, stream and (world > 1) an NCCL communicator."""
+
+    def __init__(self, device=0, stream=None, rank=0, world=1, nccl_id=None, group=None):
+        h = ctypes.c_void_p()
+        sh = _stream_handle(stream)
+        if group is not None:
+            _check(_L.sieve_ctx_create_in_group(device, sh, group._h, rank, ctypes.byref(h)),
+                   "sieve_ctx_create_in_group")
+        else:
+            idbuf = None if nccl_id is None else (ctypes.c_uint8 * 128)(*nccl_id)
+            _check(_L.sieve_ctx_create(device, sh, rank, world, idbuf, ctypes.byref(h)),
+                   "sieve_ctx_create")
+        self._h = h
+        self.device, self.rank, self.world = device, rank, world if group is None else group.world
+        self._group = group
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _L.sieve_ctx_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        self.close()
+
+
+def _col(a, dtype, device_ok=True):
+    """(pointer, is_device, keepalive) for a numpy array or a CUDA tensor."""
+    if a is None:
+        return None, None, None
+    if isinstance(a, np.ndarray):
+        a = np.ascontiguousarray(a, dtype)
+        return a.ctypes.data_as(ctypes.c_void_p), False, a
+    import torch
+    if isinstance(a, torch.Tensor):
+        want = {np.uint32: (torch.uint32, torch.int32), np.uint64: (torch.uint64, torch.int64)}[dtype]
+        if a.dtype not in want:
+            raise TypeError(f"tensor dtype {a.dtype} does not match {np.dtype(dtype)}")
+        if not a.is_contiguous():
+            raise ValueError("tensor must be contiguous")
+        if a.is_cuda:
+            return ctypes.c_void_p(a.data_ptr()), True, a
+        return ctypes.c_void_p(a.data_ptr()), False, a
+    raise TypeError(f"unsupported column type {type(a)}")
+
+
+class Trace:
+    def __init__(self, h, ctx, n, keep):
+        self._h, self.ctx, self.n, self._keep = h, ctx, n, keep
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _L.sieve_trace_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        self.close()
+
+
+def load_trace(ctx, kernel_id, instr, num_kernels, cta=None, cycles=None, first_id=0, adopt=False):
+    """sieve_load_trace: columns as numpy arrays (host, copied H2D) or CUDA tensors (device)."""
+    cols = [_col(kernel_id, np.uint32), _col(instr, np.uint64), _col(cta, np.uint32),
+            _col(cycles, np.uint64)]
+    kinds = {c[1] for c in cols if c[1] is not None}
+    if len(kinds) > 1:
+        raise ValueError("all columns must be on the same side (host or device)")
+    on_dev = kinds == {True}
+    mem = (MEM_DEVICE if on_dev else MEM_HOST) | (ADOPT if adopt else 0)
+    n = len(kernel_id)
+    h = ctypes.c_void_p()
+    _check(_L.sieve_load_trace(ctx._h, n, first_id, num_kernels, cols[0][0], cols[1][0], cols[2][0],
+                               cols[3][0], mem, ctypes.byref(h)), "sieve_load_trace")
+    return Trace(h, ctx, n, [c[2] for c in cols] if adopt else None)
+
+
+def default_params(**kw):
+    p = Params()
+    _L.sieve_params_default(ctypes.byref(p))
+    if "theta" in kw:
+        p.theta_num, p.theta_den = kw.pop("theta")
+    for k, v in kw.items():
+        setattr(p, k, v)
+    return p
+
+
+class Strata:
+    def __init__(self, h):
+        self._h = h
+        n = ctypes.c_uint64()
+        _check(_L.sieve_strata_count(h, ctypes.byref(n)), "sieve_strata_count")
+        self.table = np.zeros(n.value, STRATUM_DTYPE)
+        if n.value:
+            _check(_L.sieve_strata_copy(h, self.table.ctypes.data_as(ctypes.c_void_p), n.value),
+                   "sieve_strata_copy")
+        r, t = ctypes.c_uint32(), ctypes.c_uint64()
+        _check(_L.sieve_strata_stats(h, ctypes.byref(r), ctypes.byref(t)), "sieve_strata_stats")
+        self.rounds, self.kde_terms = r.value, t.value
+
+    def __len__(self):
+        return len(self.table)
+
+    def segments(self, G):
+        n = ctypes.c_uint64()
+        _check(_L.sieve_segment_count(self._h, ctypes.byref(n)), "sieve_segment_count")
+        out = []
+        for i in range(n.value):
+            m = _Segment()
+            _check(_L.sieve_segment_get(self._h, i, ctypes.byref(m), None, None, None), "sieve_segment_get")
+            dlo = np.zeros(G, np.uint64)
+            dhi = np.zeros(G, np.uint64)
+            cuts = np.zeros(m.n_cuts, np.uint64)
+            _check(_L.sieve_segment_get(self._h, i, ctypes.byref(m), dlo.ctypes.data_as(ctypes.c_void_p),
+                                        dhi.ctypes.data_as(ctypes.c_void_p),
+                                        cuts.ctypes.data_as(ctypes.c_void_p)), "sieve_segment_get")
+            out.append({"kernel_id": m.kernel_id, "round": m.round, "split_kind": m.split_kind,
+                        "n_cuts": m.n_cuts, "lo": m.lo, "hi": m.hi, "count": m.count,
+                        "bandwidth": m.bandwidth, "d_lo": dlo, "d_hi": dhi, "cuts": cuts})
+        return out
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _L.sieve_strata_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        self.close()
+
+
+def stratify(trace, params=None, stratum_of_invocation=None, **kw):
+    """sieve_stratify; stratum_of_invocation: optional CUDA int32/uint32 tensor [n_local]."""
+    p = params if params is not None else default_params(**kw)
+    sid_ptr = None
+    if stratum_of_invocation is not None:
+        sid_ptr = ctypes.c_void_p(stratum_of_invocation.data_ptr())
+    h = ctypes.c_void_p()
+    _check(_L.sieve_stratify(trace._h, ctypes.byref(p), sid_ptr, ctypes.byref(h)), "sieve_stratify")
+    return Strata(h)
+
+
+def predict(strata, trace, rep_cycles=None):
+    out = _Prediction()
+    rc = None
+    if rep_cycles is not None:
+        rc = np.ascontiguousarray(rep_cycles, np.uint64)
+    _check(_L.sieve_predict(strata._h, trace._h, None if rc is None else rc.ctypes.data_as(ctypes.c_void_p),
+                            ctypes.byref(out)), "sieve_predict")
+    return {"predicted_cycles": out.predicted_cycles, "predicted_ipc": out.predicted_ipc,
+            "measured_cycles": out.measured_cycles, "error": out.error, "speedup": out.speedup,
+            "total_instr": (out.total_instr_hi << 64) | out.total_instr_lo}

@@ -1,0 +1,75 @@
+"""The multi-rank path on ONE GPU: R ranks as host threads in an in-process group (the same
+exact limb reductions the NCCL path uses), each holding a contiguous slice of the trace.  The
+strata must be byte-identical to R = 1 and to the oracle; per-rank stratum ids must
+concatenate to the single-rank ids (byte-identical across R)."""
+import threading
+
+import numpy as np
+import pytest
+
+import gen
+from paper_conf_ispass_naderantahanse23_b200.distributed import shard_bounds
+from tests.gpu_helpers import assert_tables_equal, run_gpu, run_oracle
+
+pytestmark = pytest.mark.gpu
+
+
+def _run_group(tr, world, G=1024):
+    import torch
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    grp = sieve.Group(world)
+    n = len(tr["kid"])
+    res = [None] * world
+    errs = []
+
+    def rank_main(r):
+        try:
+            torch.cuda.set_device(0)
+            s = torch.cuda.Stream()
+            ctx = sieve.Ctx(device=0, stream=s, rank=r, group=grp)
+            first, cnt = shard_bounds(n, world, r)
+            sl = slice(first, first + cnt)
+            trace = sieve.load_trace(ctx, tr["kid"][sl], tr["x"][sl], num_kernels=tr["K"],
+                                     cta=tr["cta"][sl], cycles=tr["y"][sl], first_id=first)
+            with torch.cuda.stream(s):
+                sid = torch.empty(max(cnt, 1), dtype=torch.int32, device="cuda")
+            st = sieve.stratify(trace, stratum_of_invocation=sid, grid_points=G)
+            pred = sieve.predict(st, trace)
+            s.synchronize()
+            res[r] = (st.table.copy(), sid[:cnt].cpu().numpy().view(np.uint32), pred)
+            del st, trace, ctx
+        except Exception as e:  # pragma: no cover - reported below
+            errs.append((r, repr(e)))
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=600)
+    assert not errs, errs
+    return res
+
+
+@pytest.mark.parametrize("name,world", [("C1", 2), ("C2", 2), ("C2", 3), ("C2", 4)])
+def test_group_ranks_identical(name, world):
+    tr = gen.make_trace(name)
+    one = run_gpu(tr)
+    o = run_oracle(tr)
+    res = _run_group(tr, world)
+    for table, _, _ in res:
+        assert table.tobytes() == one["table"].tobytes()
+    assert_tables_equal(res[0][0], o.strata)
+    sid = np.concatenate([r[1] for r in res])
+    assert np.array_equal(sid, one["sid"])
+    assert np.array_equal(sid, o.sid)
+    preds = [r[2] for r in res]
+    assert all(p == preds[0] for p in preds)
+
+
+def test_group_rank_with_empty_slice():
+    tr = gen.make_trace("C1")
+    tr = {k: (v[:3] if isinstance(v, np.ndarray) else v) for k, v in tr.items()}
+    res = _run_group(tr, 4)   # rank 3 holds no invocation
+    o = run_oracle(tr)
+    for table, _, _ in res:
+        assert_tables_equal(table, o.strata)

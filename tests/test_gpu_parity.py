@@ -1,0 +1,169 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the CPU oracle on identical seeded
+inputs.  Integer outputs bit-exact (tiers, strata, per-invocation stratum ids, representatives,
+weights, fixed-point densities, cut thresholds); bandwidths bitwise; predictions within 1e-9
+relative (north_star tolerance)."""
+import random
+
+import numpy as np
+import pytest
+
+import gen
+from tests.gpu_helpers import (assert_predictions_close, assert_segments_equal,
+                               assert_tables_equal, run_gpu, run_oracle)
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no GPU")
+
+
+@pytest.mark.parametrize("name", ["C1", "C2"])
+def test_config_parity_full(name):
+    tr = gen.make_trace(name)
+    g = run_gpu(tr, keep_debug=True)
+    o = run_oracle(tr, keep_debug=True)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+    assert g["rounds"] == o.rounds
+    assert_segments_equal(g["segments"], o.segments())
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    assert_predictions_close(sieve.predict(g["strata"], g["trace"]), o.predict())
+
+
+def test_c3_parity():
+    tr = gen.make_trace("C3")
+    g = run_gpu(tr)
+    o = run_oracle(tr)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    assert_predictions_close(sieve.predict(g["strata"], g["trace"]), o.predict())
+
+
+@pytest.mark.parametrize("G", [3, 64, 1000, 4096])
+def test_grid_sizes(G):
+    tr = gen.make_trace("C2", n=120_000)
+    g = run_gpu(tr, G=G, keep_debug=True)
+    o = run_oracle(tr, G=G, keep_debug=True)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+    assert_segments_equal(g["segments"], o.segments())
+
+
+@pytest.mark.parametrize("theta", [(1, 10), (1, 2), (1, 1), (3, 7)])
+def test_theta_values(theta):
+    tr = gen.make_trace("C2", n=100_000)
+    g = run_gpu(tr, theta=theta)
+    o = run_oracle(tr, theta=theta)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+
+
+def test_device_columns_and_nullable_columns():
+    tr = gen.make_trace("C1")
+    o = run_oracle(tr, cta=False, cycles=False)
+    g = run_gpu(tr, cta=False, cycles=False, device_cols=True)
+    assert_tables_equal(g["table"], o.strata)
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    with pytest.raises(sieve.SieveError) as e:
+        sieve.predict(g["strata"], g["trace"])
+    assert e.value.code == -6
+    rc = np.arange(1, len(g["table"]) + 1, dtype=np.uint64) * 1000
+    assert_predictions_close(sieve.predict(g["strata"], g["trace"], rc), o.predict(rc))
+
+
+def _micro(seed):
+    rng = random.Random(seed)
+    n = rng.randrange(1, 3000)
+    K = rng.randrange(1, 40)
+    kid = np.array([rng.randrange(K) for _ in range(n)], np.uint32)
+    modes = {k: [rng.randrange(1, 1 << rng.choice([8, 20, 43])) for _ in range(rng.randrange(1, 5))]
+             for k in range(K)}
+    x = []
+    for k in kid:
+        m = rng.choice(modes[int(k)])
+        x.append(max(1, min((1 << 44) - 1, m + rng.randrange(-(m // 10) - 1, m // 10 + 2))))
+    return {"kid": kid, "x": np.array(x, np.uint64),
+            "cta": np.array([rng.choice([32, 64, 1024, 7]) for _ in range(n)], np.uint32),
+            "y": np.array([rng.randrange(0, 1 << 40) for _ in range(n)], np.uint64), "K": K}
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_micro_traces(seed):
+    tr = _micro(seed)
+    G = [3, 17, 128, 1024][seed % 4]
+    g = run_gpu(tr, G=G, keep_debug=True)
+    o = run_oracle(tr, G=G, keep_debug=True)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+    assert_segments_equal(g["segments"], o.segments())
+
+
+def test_edge_cases():
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    # empty trace
+    tr = {"kid": np.zeros(0, np.uint32), "x": np.zeros(0, np.uint64), "cta": np.zeros(0, np.uint32),
+          "y": np.zeros(0, np.uint64), "K": 5}
+    g = run_gpu(tr, with_sid=False)
+    assert len(g["table"]) == 0
+    # single invocation, single kernel
+    tr = {"kid": np.zeros(1, np.uint32), "x": np.array([(1 << 44) - 1], np.uint64),
+          "cta": np.array([128], np.uint32), "y": np.array([5], np.uint64), "K": 1}
+    assert_tables_equal(run_gpu(tr)["table"], run_oracle(tr).strata)
+    # every kernel invoked once, values at the edges of the range
+    n = 5000
+    tr = {"kid": np.arange(n, dtype=np.uint32), "x": np.array([1 + (i * 7919) % ((1 << 44) - 1) for i in range(n)], np.uint64),
+          "cta": np.full(n, 256, np.uint32), "y": np.arange(1, n + 1, dtype=np.uint64), "K": n}
+    assert_tables_equal(run_gpu(tr)["table"], run_oracle(tr).strata)
+    # two equal point masses (symmetric density)
+    x = np.array([1000] * 400 + [10_000] * 400, np.uint64)
+    tr = {"kid": np.zeros(800, np.uint32), "x": x, "cta": np.full(800, 64, np.uint32),
+          "y": x * 3, "K": 1}
+    assert_tables_equal(run_gpu(tr)["table"], run_oracle(tr).strata)
+    # invalid rows are rejected on the device
+    bad = dict(tr)
+    bad["x"] = x.copy()
+    bad["x"][17] = 0
+    with pytest.raises(sieve.SieveError) as e:
+        run_gpu(bad)
+    assert e.value.code == -2
+    bad["x"] = x.copy()
+    bad["kid"] = np.zeros(800, np.uint32)
+    bad["kid"][5] = 3
+    with pytest.raises(sieve.SieveError) as e:
+        run_gpu(bad)
+    assert e.value.code == -1
+    # max_rounds exceeded
+    xx = np.array([1, 2, 4, 8, 16, 32, 64, 128, 256, 512, 1024, 2048] * 3, np.uint64)
+    tr = {"kid": np.zeros(len(xx), np.uint32), "x": xx, "cta": np.zeros(len(xx), np.uint32),
+          "y": xx, "K": 1}
+    with pytest.raises(sieve.SieveError) as e:
+        run_gpu(tr, max_rounds=1)
+    assert e.value.code == -7
+
+
+def test_many_kernels_multiple_smem_passes():
+    # K > 2048 makes pass A run several kernel-id ranges
+    rng = np.random.default_rng(3)
+    n, K = 200_000, 9000
+    kid = rng.integers(0, K, n).astype(np.uint32)
+    base = rng.integers(1, 1 << 30, K).astype(np.uint64)
+    x = base[kid] + rng.integers(0, 3, n).astype(np.uint64) * (base[kid] // 2)
+    tr = {"kid": kid, "x": x, "cta": rng.choice([64, 128], n).astype(np.uint32),
+          "y": rng.integers(1, 1 << 30, n).astype(np.uint64), "K": K}
+    g = run_gpu(tr)
+    o = run_oracle(tr)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+
+
+def test_homogeneous_prediction_exact():
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr = gen.make_trace("C2", homogeneous=1)
+    g = run_gpu(tr)
+    p = sieve.predict(g["strata"], g["trace"])
+    assert p["error"] < 1e-12
