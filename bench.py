@@ -1,0 +1,328 @@
+#!/usr/bin/env python
+"""bench.py -- throughput of the Sieve stratification hot path on B200.
+
+metric: kernel invocations stratified per second (BASELINE.json), one "step" = the whole hot
+path (sieve_stratify + sieve_predict: moments, tiering, Tier-3 sort, KDE rounds, valleys,
+parts, assignment, representatives, prediction) over one synthetic trace.  Workload at N=1:
+C4 (100M invocations, 2,000 kernels, MLPerf-shaped), the BASELINE.json config the
+"1/2/4/8 B200" metric is quoted on; with N GPUs the same 100M-invocation trace is sharded
+contiguously over the ranks (strong scaling; NCCL all-reduces of moments, KDE grids, parts).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C4] [--impl reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...
+
+Prints ONE JSON line on rank 0.  `value` is device-timed (CUDA events on the library's stream,
+barrier + synchronize on both sides, max over ranks) with the trace resident in HBM; `e2e` is
+the same metric through the C-ABI from pinned HOST buffers (H2D of the columns inside the timed
+region, the stratum table and prediction read back).  `roofline` is the dominant kernel
+(fixed-point KDE, FP64-pipe bound) with its time measured by CUDA events around its launches
+inside the timed steps.  `cpu_baseline` is the CPU oracle timed on a bounded sample.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+KDE_FP64_OPS_PER_TERM = 24   # FP64-pipe instructions per in-window KDE term
+FP64_LANES_PER_SM = 64       # B200: 64 FP64 FMA lanes / SM / clk (microbenchmark: 62.9)
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C4")
+    ap.add_argument("--impl", default="sieve", choices=["sieve", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample", type=int, default=1_000_000)
+    return ap.parse_args()
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            return json.load(f), "measured"
+    return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 100 ms while running."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.samples = []
+        self.proc = None
+        self.marks = {}
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits", "-lms", "100",
+                 "-i", str(self.device)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except OSError:
+            self.proc = None
+            return
+        self.th = threading.Thread(target=self._read, daemon=True)
+        self.th.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.samples.append((time.time(), line.strip()))
+
+    def mark(self, name):
+        self.marks[name] = time.time()
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self, t0_key="t0", t1_key="t1"):
+        t0, t1 = self.marks.get(t0_key, 0), self.marks.get(t1_key, 1e30)
+        rows = [s for ts, s in self.samples if t0 - 0.15 <= ts <= t1 + 0.15]
+        if len(rows) < 3:
+            rows = [s for _, s in self.samples]
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            f = [x.strip() for x in r.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def cpu_oracle_rate(cfg, sample):
+    """The CPU oracle (as it stands, single-threaded) on the first `sample` invocations."""
+    import gen
+    import oracle
+    g = gen.Generator(cfg)
+    tr = g.fill(0, sample)
+    t = time.perf_counter()
+    r = oracle.stratify(tr["kid"], tr["x"], cfg.K, tr["cta"], tr["y"])
+    r.predict()
+    dt = time.perf_counter() - t
+    return sample / dt, dt
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle on bounded samples of the same workload (rank 0)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import gen
+    cfg = gen.get_config(args.config)
+    per_step = 250_000
+    rates = []
+    for i in range(args.warmup + args.steps):
+        rate, dt = cpu_oracle_rate(cfg, per_step)
+        if i >= args.warmup:
+            rates.append((per_step, dt))
+    tot_n = sum(n for n, _ in rates)
+    tot_t = sum(t for _, t in rates)
+    value = tot_n / tot_t
+    sample = f"first {per_step} invocations of {cfg.name} per step (same generator), oracle single-threaded"
+    line = {"impl": "reference", "metric": "kernel invocations stratified/sec", "value": value,
+            "unit": "invocations/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1000 * tot_t / len(rates), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u64/u128 + f64", "data": "synthetic",
+            "config": {"workload": cfg.name, "invocations": cfg.n, "kernels": cfg.K, "sample": per_step},
+            "cpu_baseline": {"value": value, "unit": "invocations/s", "cores": 1, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": "invocations/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+    import gen
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    from paper_conf_ispass_naderantahanse23_b200.distributed import make_ctx, shard_bounds
+
+    rank, world = int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    cfg = gen.get_config(args.config)
+    first, n_local = shard_bounds(cfg.n, world, rank)
+
+    # ---- synthetic input: this rank's slice, generated on the host into pinned memory ----
+    g = gen.Generator(cfg)
+    pin = lambda n, dt: torch.empty(n, dtype=dt, pin_memory=True)
+    h = {"kid": pin(n_local, torch.int32), "x": pin(n_local, torch.int64),
+         "cta": pin(n_local, torch.int32), "y": pin(n_local, torch.int64)}
+    hn = {"kid": h["kid"].numpy().view(np.uint32), "x": h["x"].numpy().view(np.uint64),
+          "cta": h["cta"].numpy().view(np.uint32), "y": h["y"].numpy().view(np.uint64)}
+    g.fill(first, n_local, out=hn)
+
+    stream = torch.cuda.Stream()
+    ctx = make_ctx(device=local, stream=stream)
+    with torch.cuda.stream(stream):
+        d = {k: v.to("cuda", non_blocking=True) for k, v in h.items()}
+        sid = torch.empty(max(n_local, 1), dtype=torch.int32, device="cuda")
+    stream.synchronize()
+    trace = sieve.load_trace(ctx, d["kid"], d["x"], num_kernels=cfg.K, cta=d["cta"], cycles=d["y"],
+                             first_id=first, adopt=True)
+
+    def step():
+        st = sieve.stratify(trace, stratum_of_invocation=sid)
+        sieve.predict(st, trace)
+        return st
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(v):
+        if world == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    clk = ClockSampler(local)
+    clk.start()
+    for _ in range(args.warmup):
+        st = step()
+    n_strata = len(st)
+    rounds = st.rounds
+
+    # ---- device-timed steps (trace resident in HBM; 2.4 GB of columns >> 126 MB L2) ----
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ctx.set_timing(True)
+    launches0 = sieve.kernel_launches()
+    barrier()
+    torch.cuda.synchronize()
+    clk.mark("t0")
+    ev0.record(stream)
+    for _ in range(args.steps):
+        st = step()
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    clk.mark("t1")
+    launches = sieve.kernel_launches() - launches0
+    ms = ev0.elapsed_time(ev1)
+    ms_max = max_over_ranks(ms)
+    phases = ctx.timing()
+    ctx.set_timing(False)
+    value = cfg.n * args.steps / (ms_max / 1000.0)
+
+    # ---- end-to-end through the C-ABI from pinned host buffers ----
+    e2e = None
+    if not args.no_e2e:
+        e_steps = max(1, min(args.steps, 5))
+        # warm once
+        tr_h = sieve.load_trace(ctx, hn["kid"], hn["x"], num_kernels=cfg.K, cta=hn["cta"], cycles=hn["y"],
+                                first_id=first)
+        sieve.predict(sieve.stratify(tr_h), tr_h)
+        del tr_h
+        barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(e_steps):
+            tr_h = sieve.load_trace(ctx, hn["kid"], hn["x"], num_kernels=cfg.K, cta=hn["cta"],
+                                    cycles=hn["y"], first_id=first)
+            st_h = sieve.stratify(tr_h)
+            pr = sieve.predict(st_h, tr_h)
+            del tr_h
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ems = max_over_ranks(e0.elapsed_time(e1))
+        e2e = {"value": cfg.n * e_steps / (ems / 1000.0), "unit": "invocations/s",
+               "h2d_bytes_per_step": int(n_local * 24),
+               "d2h_bytes_per_step": int(len(st_h) * 96 + 56), "steps": e_steps,
+               "note": "H2D of kid/x/cta/y from pinned host memory + stratify + predict; "
+                       "stratum table and prediction read back to the host"}
+    clk.stop()
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    peaks, peak_src = measured_peaks()
+    clocks = clk.summary()
+    nsm = torch.cuda.get_device_properties(local).multi_processor_count
+    kde_ms, kde_calls, kde_terms = phases["kde"]
+    fp64_peak = nsm * FP64_LANES_PER_SM * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12  # Top/s
+    roof = None
+    if kde_ms > 0:
+        achieved = KDE_FP64_OPS_PER_TERM * kde_terms / (kde_ms / 1000.0) / 1e12
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "kde_traffic.json")
+        if os.path.exists(tp):
+            with open(tp) as f:
+                traffic = json.load(f).get("dram_bytes_per_launch")
+        roof = {"kernel": "k_kde (fixed-point Gaussian KDE)", "bound": "alu", "achieved": achieved,
+                "peak": fp64_peak, "unit": "Top/s (FP64-pipe instructions)", "frac": achieved / fp64_peak,
+                "traffic": traffic, "share_of_step": kde_ms / ms,
+                "peak_source": f"{nsm} SMs x {FP64_LANES_PER_SM} FP64 lanes x sm_max_mhz "
+                               f"{peaks.get('sm_max_mhz')} ({peak_src} MEASURED_PEAKS.json)",
+                "work": f"{kde_terms / args.steps:.4g} in-window terms/step x {KDE_FP64_OPS_PER_TERM} FP64 ops"}
+    hbm = peaks.get("hbm_gbs", 6650.0)
+    phase_out = {}
+    for name, (pms, calls, work) in phases.items():
+        e = {"ms_per_step": pms / args.steps, "calls": calls}
+        if name in ("moments", "compact", "sort", "prefix", "assign") and pms > 0:
+            e["GB/s"] = work / (pms / 1000.0) / 1e9
+            e["hbm_frac"] = e["GB/s"] / hbm
+        phase_out[name] = e
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        rate, dt = cpu_oracle_rate(cfg, args.cpu_sample)
+        cpu = {"value": rate, "unit": "invocations/s", "cores": 1, "kind": "oracle",
+               "sample": f"first {args.cpu_sample} invocations of {cfg.name} (same generator), "
+                         f"{dt:.1f} s single-threaded"}
+    line = {"metric": "kernel invocations stratified/sec", "value": value, "unit": "invocations/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u64/u128 + f64", "data": "synthetic",
+            "config": {"workload": cfg.name, "invocations": cfg.n, "kernels": cfg.K,
+                       "grid_points": 1024, "theta": "2/5", "strata": n_strata, "rounds": rounds,
+                       "parallelism": f"dp{world} (contiguous invocation slices)",
+                       "l2": "inputs larger than L2 (24 B/invocation = 2.4 GB per step)"},
+            "clocks": clocks, "e2e": e2e, "gpu_launches": launches,
+            "roofline": roof, "phases": phase_out, "cpu_baseline": cpu}
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

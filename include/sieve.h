@@ -184,6 +184,28 @@ typedef struct {
                  trace's cycles column (SIEVE_EDOM if the trace has none). */
 int sieve_predict(sieve_strata s, sieve_trace t, const uint64_t* rep_cycles, sieve_prediction* out);
 
+/* ---- measurement ------------------------------------------------------------------------ */
+/* Per-phase device time of the calls made on this context, taken with CUDA events recorded on
+   the context's stream around each phase (off by default; enabling resets the counters).
+   `work` is the phase's algorithmic work unit count: bytes for the
+   streaming passes, in-window KDE terms for SIEVE_PHASE_KDE. */
+enum {
+  SIEVE_PHASE_MOMENTS = 0, /* pass A: per-kernel moments */
+  SIEVE_PHASE_COMPACT = 1, /* Tier-3 key compaction */
+  SIEVE_PHASE_SORT = 2,    /* radix sort of Tier-3 keys */
+  SIEVE_PHASE_PREFIX = 3,  /* u128 prefix sums of x, x^2 */
+  SIEVE_PHASE_KDE = 4,     /* fixed-point KDE (all rounds) */
+  SIEVE_PHASE_REFINE = 5,  /* valleys + part moments (all rounds) */
+  SIEVE_PHASE_ASSIGN = 6,  /* pass B: assignment + (stratum, CTA) statistics */
+  SIEVE_PHASE_REPS = 7,    /* entry compaction, sort, representatives */
+  SIEVE_PHASE_PREDICT = 8, /* prediction */
+  SIEVE_PHASE_COUNT = 9
+};
+int sieve_ctx_set_timing(sieve_ctx ctx, int enable);
+int sieve_timing_get(sieve_ctx ctx, uint32_t phase, double* ms, uint64_t* calls, uint64_t* work);
+/* number of kernels this process has launched through the library (all contexts) */
+uint64_t sieve_kernel_launches(void);
+
 /* ---- misc ----------------------------------------------------------------------------------- */
 const char* sieve_last_error(void); /* thread-local; valid until the next call on this thread */
 const char* sieve_version(void);

@@ -14,6 +14,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <atomic>
 #include <string>
 #include <vector>
 
@@ -63,6 +64,9 @@ extern "C" void sieve_limbs_to_u128(const uint64_t limbs[4], uint64_t* lo, uint6
 #define TRACE_MAGIC 0x51E7C7A1u
 #define STRATA_MAGIC 0x51E7C7A2u
 
+struct PhaseAcc { double ms = 0; u64 calls = 0; u64 work = 0; };
+struct PendingEv { int ph; cudaEvent_t a, b; };
+
 struct sieve_ctx_s {
   uint32_t magic = CTX_MAGIC;
   int device = 0;
@@ -72,7 +76,69 @@ struct sieve_ctx_s {
   sieve_alloc_fn af = nullptr;
   sieve_free_fn ff = nullptr;
   void* user = nullptr;
+  bool timing = false;
+  PhaseAcc acc[SIEVE_PHASE_COUNT];
+  std::vector<PendingEv> pending;
+  std::vector<cudaEvent_t> ev_pool;
 };
+
+static std::atomic<unsigned long long> g_launches{0};
+void sv_count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+extern "C" uint64_t sieve_kernel_launches(void) { return g_launches.load(); }
+
+// CUDA events around a phase on the ctx stream (only when timing is enabled)
+struct PhaseTimer {
+  sieve_ctx_s* c;
+  int ph;
+  cudaEvent_t a = nullptr;
+  PhaseTimer(sieve_ctx_s* cc, int p, u64 work) : c(cc), ph(p) {
+    if (!c->timing) return;
+    a = take();
+    cudaEventRecord(a, c->stream);
+    c->acc[ph].calls++;
+    c->acc[ph].work += work;
+  }
+  cudaEvent_t take() {
+    if (c->ev_pool.empty()) { cudaEvent_t e; cudaEventCreate(&e); return e; }
+    cudaEvent_t e = c->ev_pool.back();
+    c->ev_pool.pop_back();
+    return e;
+  }
+  void stop() {
+    if (!a) return;
+    cudaEvent_t b = take();
+    cudaEventRecord(b, c->stream);
+    c->pending.push_back({ph, a, b});
+    a = nullptr;
+  }
+  ~PhaseTimer() { stop(); }
+};
+
+// after the stream is synchronised: fold the recorded event pairs into the accumulators
+static void resolve_timing(sieve_ctx_s* c) {
+  for (auto& p : c->pending) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, p.a, p.b) == cudaSuccess) c->acc[p.ph].ms += ms;
+    c->ev_pool.push_back(p.a);
+    c->ev_pool.push_back(p.b);
+  }
+  c->pending.clear();
+}
+
+extern "C" int sieve_ctx_set_timing(sieve_ctx ctx, int enable) {
+  if (!ctx || ctx->magic != CTX_MAGIC) return sv_fail(SIEVE_EINVAL, "bad ctx");
+  ctx->timing = enable != 0;
+  for (auto& a : ctx->acc) a = PhaseAcc();
+  return SIEVE_OK;
+}
+
+extern "C" int sieve_timing_get(sieve_ctx ctx, uint32_t phase, double* ms, uint64_t* calls, uint64_t* work) {
+  if (!ctx || ctx->magic != CTX_MAGIC || phase >= SIEVE_PHASE_COUNT) return sv_fail(SIEVE_EINVAL, "bad ctx or phase");
+  if (ms) *ms = ctx->acc[phase].ms;
+  if (calls) *calls = ctx->acc[phase].calls;
+  if (work) *work = ctx->acc[phase].work;
+  return SIEVE_OK;
+}
 
 struct sieve_trace_s {
   uint32_t magic = TRACE_MAGIC;
@@ -211,6 +277,9 @@ extern "C" int sieve_ctx_set_allocator(sieve_ctx ctx, sieve_alloc_fn a, sieve_fr
 
 extern "C" void sieve_ctx_destroy(sieve_ctx ctx) {
   if (!ctx_ok(ctx)) return;
+  cudaSetDevice(ctx->device);
+  for (auto& p : ctx->pending) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
+  for (auto e : ctx->ev_pool) cudaEventDestroy(e);
   delete ctx->comm;
   ctx->magic = 0;
   delete ctx;
@@ -400,6 +469,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   // tot: [0..4) C_meas limbs (SUM), [4] max x (MAX), [5..8) error lanes (MAX)
   SV_TRY(tot.alloc(8));
   SV_CUDA(cudaMemsetAsync(tot.get(), 0, 8 * 8, S));
+  PhaseTimer tA(c, SIEVE_PHASE_MOMENTS, n * (12 + (t->y ? 8 : 0)));
   for (u32 k0 = 0; k0 < K; k0 += kt) {
     u32 kk = std::min(kt, K - k0);
     if (n) {
@@ -417,6 +487,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(h2d(c, mm.get(), mmh));
   }
   SV_CUDA(cudaGetLastError());
+  tA.stop();
   // AR-1: sums, then min/max (mm is interleaved min,max per kernel: reduce via a [2][K] copy)
   std::vector<u64> h_lanes, h_mm, h_tot, h_localn;
   if (c->comm) {
@@ -490,17 +561,24 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(h2d(c, d_t3rank.get(), t3rank));
     SV_TRY(keys.alloc(n3_local));
     SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
-    launch_t3_compact(t->kid, t->x, n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
+    {
+      PhaseTimer tm(c, SIEVE_PHASE_COMPACT, n * 12 + n3_local * 8);
+      launch_t3_compact(t->kid, t->x, n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
+    }
     {
       DBuf<char> tmp(c);
       SV_TRY(tmp.alloc(radix_sort_temp_bytes(n3_local, false)));
-      SV_TRY(radix_sort(keys.get(), nullptr, n3_local, nbits, tmp.get(), S));
+      PhaseTimer tm(c, SIEVE_PHASE_SORT, 0);
+      int passes = 0;
+      SV_TRY(radix_sort(keys.get(), nullptr, n3_local, nbits, tmp.get(), S, &passes));
+      if (c->timing) c->acc[SIEVE_PHASE_SORT].work += (u64)passes * n3_local * 16;
     }
     SV_TRY(P1.alloc(2 * (n3_local + 1)));
     SV_TRY(P2.alloc(2 * (n3_local + 1)));
     {
       DBuf<char> tmp(c);
       SV_TRY(tmp.alloc(prefix128_temp_bytes(n3_local)));
+      PhaseTimer tm(c, SIEVE_PHASE_PREFIX, n3_local * 8 + (n3_local + 1) * 32);
       launch_prefix128(keys.get(), n3_local, xmask, P1.get(), P2.get(), tmp.get(), S);
     }
     SV_CUDA(cudaGetLastError());
@@ -550,8 +628,10 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       u32 items = 0;
       SV_TRY(kde_plan(segs.get(), nseg, G, keys.get(), nkeys, xmask, tile_range.get(),
                       tile_items.get(), stemp.get(), &items, S));
+      PhaseTimer tm(c, SIEVE_PHASE_KDE, 0);
       launch_kde(segs.get(), nseg, G, keys.get(), xmask, tile_range.get(), tile_items.get(), items,
                  D.get(), counter.get() + 1, terms.get(), S);
+      tm.stop();
       SV_CUDA(cudaGetLastError());
     }
     if (c->comm) {  // AR-2: densities as 32-bit limbs
@@ -565,8 +645,10 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     DBuf<u32> ntk(c);
     SV_TRY(T.alloc((size_t)nseg * tstride));
     SV_TRY(ntk.alloc((size_t)nseg * 2));
+    PhaseTimer tv(c, SIEVE_PHASE_REFINE, 0);
     launch_valleys(segs.get(), nseg, G, P->valley_shift, D.get(), T.get(), tstride, ntk.get(),
                    ntk.get() + nseg, S);
+    tv.stop();
     std::vector<u32> h_ntk;
     SV_TRY(d2h(c, h_ntk, ntk.get(), (size_t)nseg * 2));
     SV_TRY(sync(c));
@@ -581,9 +663,11 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(pl.alloc((size_t)nparts * MOM_LANES));
     SV_TRY(pm.alloc((size_t)nparts * 2));
     SV_TRY(pab.alloc((size_t)nparts * 2));
+    PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
     launch_part_stats(segs.get(), nseg, T.get(), tstride, ntk.get(), d_off.get(), nparts,
                       nkeys ? keys.get() : nullptr, nkeys, bx, P1.get(), P2.get(), pl.get(),
                       pm.get(), pab.get(), S);
+    tp.stop();
     SV_CUDA(cudaGetLastError());
     SV_TRY(allreduce(c, pl.get(), (size_t)nparts * MOM_LANES, RED_SUM));   // AR-3
     SV_TRY(allreduce(c, pm.get(), nparts, RED_MIN));
@@ -638,6 +722,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(d2h(c, ht, terms.get(), 1));
     SV_TRY(sync(c));
     R->kde_terms = ht[0];
+    if (c->timing) c->acc[SIEVE_PHASE_KDE].work += ht[0];
   }
   P1.release(); P2.release(); keys.release();
 
@@ -681,8 +766,10 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     launch_fill_u64(gfirst.get(), cap, ~0ull, S);
     SV_CUDA(cudaMemsetAsync(errf.get(), 0, 32, S));
     GHash gh{gkeys.get(), gcnt.get(), gfirst.get(), cap};
+    PhaseTimer tb(c, SIEVE_PHASE_ASSIGN, n * (12 + (t->cta ? 4 : 0) + (sid_out ? 4 : 0)));
     launch_assign(t->kid, t->x, t->cta, n, t->first_id, d_ktab.get(), d_lows.get(), sid_out, gh,
                   errf.get(), assign_grid(), S);
+    tb.stop();
     SV_CUDA(cudaGetLastError());
     SV_TRY(ekey.alloc(cap)); SV_TRY(ecnt.alloc(cap)); SV_TRY(efirst.alloc(cap));
     SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
@@ -744,6 +831,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(h2d(c, idx.get(), iota));
   }
   SV_CUDA(cudaMemcpyAsync(sk.get(), ak.get(), Etot * 8, cudaMemcpyDeviceToDevice, S));
+  PhaseTimer tr(c, SIEVE_PHASE_REPS, 0);
   {
     DBuf<char> tmp(c);
     SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
@@ -759,12 +847,14 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   SV_TRY(h2d(c, d_tier.get(), tiers));
   launch_reps(sk.get(), scnt.get(), sfirst.get(), Etot, d_tier.get(), ns, rep.get(), rep.get() + ns, S);
   launch_rep_xy(rep.get(), ns, t->first_id, n, t->x, t->y, repxy.get(), S);
+  tr.stop();
   SV_CUDA(cudaGetLastError());
   SV_TRY(allreduce(c, repxy.get(), 2 * (size_t)ns, RED_SUM));   // AR-5: owner contributes
   std::vector<u64> h_rep, h_xy;
   SV_TRY(d2h(c, h_rep, rep.get(), 2 * (size_t)ns));
   SV_TRY(d2h(c, h_xy, repxy.get(), 2 * (size_t)ns));
   SV_TRY(sync(c));
+  resolve_timing(c);
 
   // ---------------- assemble --------------------------------------------------------------------
   R->st.resize(ns);
@@ -880,11 +970,14 @@ extern "C" int sieve_predict(sieve_strata s, sieve_trace t, const uint64_t* rep_
   DBuf<double> dout(c);
   SV_TRY(dW.alloc(hW.size())); SV_TRY(dx.alloc(ns)); SV_TRY(dy.alloc(ns)); SV_TRY(dout.alloc(4));
   SV_TRY(h2d(c, dW.get(), hW)); SV_TRY(h2d(c, dx.get(), hx)); SV_TRY(h2d(c, dy.get(), hy));
+  PhaseTimer tpr(c, SIEVE_PHASE_PREDICT, 0);
   launch_predict(dW.get(), dx.get(), dy.get(), ns, dout.get(), c->stream);
+  tpr.stop();
   SV_CUDA(cudaGetLastError());
   std::vector<double> r;
   SV_TRY(d2h(c, r, dout.get(), 4));
   SV_TRY(sync(c));
+  resolve_timing(c);
   out->predicted_cycles = r[0];
   out->predicted_ipc = r[3];
   out->total_instr_lo = (u64)s->total_instr;

@@ -125,7 +125,7 @@ void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 firs
   cudaFuncSetAttribute(k_assign, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   u64 maxgrid = (n + (u64)AS_THREADS * AS_IPT - 1) / ((u64)AS_THREADS * AS_IPT);
   if ((u64)grid > maxgrid) grid = (int)maxgrid;
-  k_assign<<<grid, AS_THREADS, smem, s>>>(kid, x, cta, n, first_id, ktab, lows, sid_out, gh, errflags);
+  SV_LAUNCH(k_assign, grid, AS_THREADS, smem, s)(kid, x, cta, n, first_id, ktab, lows, sid_out, gh, errflags);
 }
 
 __global__ void k_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst,
@@ -146,7 +146,7 @@ __global__ void k_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst,
 
 void launch_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst, unsigned long long* count,
                          cudaStream_t s) {
-  k_hash_compact<<<div_up(gh.cap, 256), 256, 0, s>>>(gh, okey, ocnt, ofirst, count);
+  SV_LAUNCH(k_hash_compact, div_up(gh.cap, 256), 256, 0, s)(gh, okey, ocnt, ofirst, count);
 }
 
 __global__ void k_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst) {
@@ -154,7 +154,7 @@ __global__ void k_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst) {
   if (i < n) dst[i] = src[idx[i]];
 }
 void launch_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst, cudaStream_t s) {
-  if (n) k_gather_u64<<<div_up(n, 256), 256, 0, s>>>(src, idx, n, dst);
+  if (n) SV_LAUNCH(k_gather_u64, div_up(n, 256), 256, 0, s)(src, idx, n, dst);
 }
 
 // one thread per stratum over its (sorted) entries; equal keys (from different ranks) merge
@@ -180,7 +180,7 @@ __global__ void k_reps(const u64* key, const u64* cnt, const u64* first, u64 E, 
 
 void launch_reps(const u64* key, const u64* cnt, const u64* first, u64 E, const u32* tier,
                  u32 nstrata, u64* rep_id, u64* rep_cta, cudaStream_t s) {
-  if (nstrata) k_reps<<<div_up(nstrata, 128), 128, 0, s>>>(key, cnt, first, E, tier, nstrata, rep_id, rep_cta);
+  if (nstrata) SV_LAUNCH(k_reps, div_up(nstrata, 128), 128, 0, s)(key, cnt, first, E, tier, nstrata, rep_id, rep_cta);
 }
 
 __global__ void k_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, const u64* x,
@@ -195,7 +195,7 @@ __global__ void k_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_loc
 
 void launch_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, const u64* x,
                    const u64* y, u64* out, cudaStream_t s) {
-  if (nstrata) k_rep_xy<<<div_up(nstrata, 128), 128, 0, s>>>(rep_id, nstrata, first_id, n_local, x, y, out);
+  if (nstrata) SV_LAUNCH(k_rep_xy, div_up(nstrata, 128), 128, 0, s)(rep_id, nstrata, first_id, n_local, x, y, out);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -203,7 +203,7 @@ __global__ void k_fill_u64(u64* p, u64 n, u64 v) {
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) p[i] = v;
 }
 void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s) {
-  if (n) k_fill_u64<<<min(div_up(n, 256), 4096u), 256, 0, s>>>(p, n, v);
+  if (n) SV_LAUNCH(k_fill_u64, min(div_up(n, 256), 4096u), 256, 0, s)(p, n, v);
 }
 
 __global__ void k_u128_to_limbs(const u64* src, u64 n, u64* limbs) {
@@ -215,8 +215,8 @@ __global__ void k_limbs_to_u128(const u64* limbs, u64 n, u64* dst) {
   if (i < n) limbs_to_u128(limbs + 4 * i, dst + 2 * i, dst + 2 * i + 1);
 }
 void launch_u128_to_limbs(const u64* src, u64 n, u64* limbs, cudaStream_t s) {
-  if (n) k_u128_to_limbs<<<div_up(n, 256), 256, 0, s>>>(src, n, limbs);
+  if (n) SV_LAUNCH(k_u128_to_limbs, div_up(n, 256), 256, 0, s)(src, n, limbs);
 }
 void launch_limbs_to_u128(const u64* limbs, u64 n, u64* dst, cudaStream_t s) {
-  if (n) k_limbs_to_u128<<<div_up(n, 256), 256, 0, s>>>(limbs, n, dst);
+  if (n) SV_LAUNCH(k_limbs_to_u128, div_up(n, 256), 256, 0, s)(limbs, n, dst);
 }

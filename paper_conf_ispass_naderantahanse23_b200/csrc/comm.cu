@@ -152,7 +152,7 @@ struct GroupComm : Comm {
       for (int r = 0; r < world; r++) pk.p[r] = g->ptrs[r];
       unsigned blocks = (unsigned)((n + 255) / 256);
       if (blocks > 4096) blocks = 4096;
-      k_group_reduce<<<blocks, 256, 0, s>>>(pk, world, n, (int)op, tmp);
+      SV_LAUNCH(k_group_reduce, blocks, 256, 0, s)(pk, world, n, (int)op, tmp);
       SV_CUDA(cudaGetLastError());
     }
     SV_CUDA(cudaStreamSynchronize(s));

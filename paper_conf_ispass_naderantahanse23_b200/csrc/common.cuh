@@ -72,3 +72,7 @@ __device__ __forceinline__ u32 lane_id() { return threadIdx.x & 31u; }
 // ------------------------------------------------------------------------------------------
 static inline unsigned div_up(u64 a, u64 b) { return (unsigned)((a + b - 1) / b); }
 int sv_num_sms();
+// every kernel launch of the library goes through SV_LAUNCH so the process-wide launch
+// count (sieve_kernel_launches) is exact
+void sv_count_launch();
+#define SV_LAUNCH(k, g, b, sm, st) sv_count_launch(), k<<<g, b, sm, st>>>

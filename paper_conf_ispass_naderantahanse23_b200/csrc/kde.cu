@@ -51,7 +51,7 @@ __global__ void k_seg_ranges(SegDev* segs, u32 nseg, const u64* keys, u64 nkeys)
 }
 
 void launch_seg_ranges(SegDev* segs, u32 nseg, const u64* keys, u64 nkeys, cudaStream_t s) {
-  if (nseg) k_seg_ranges<<<div_up(nseg, 128), 128, 0, s>>>(segs, nseg, keys, nkeys);
+  if (nseg) SV_LAUNCH(k_seg_ranges, div_up(nseg, 128), 128, 0, s)(segs, nseg, keys, nkeys);
 }
 
 // per (segment, tile): the local index range of values inside the tile's window, and the
@@ -84,7 +84,7 @@ int kde_plan(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 nkeys, u6
   (void)nkeys; (void)xmask;
   u32 tps = div_up(G, KDE_TJ);
   u64 nt = (u64)nseg * tps;
-  k_kde_tiles<<<div_up(nt, 128), 128, 0, s>>>(segs, nseg, G, tps, keys, tile_range, tile_items);
+  SV_LAUNCH(k_kde_tiles, div_up(nt, 128), 128, 0, s)(segs, nseg, G, tps, keys, tile_range, tile_items);
   // exclusive scan in place; tile_items[nt] receives the total
   scan_u32(tile_items, tile_items, nt, scan_temp, tile_items + nt, s);
   SV_CUDA(cudaMemcpyAsync(items_host, tile_items + nt, 4, cudaMemcpyDeviceToHost, s));
@@ -206,6 +206,6 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
   u32 grid = (u32)sv_num_sms() * (u32)per_sm;
   if (grid > items) grid = items;
   cudaMemsetAsync(work_counter, 0, 8, s);
-  k_kde<<<grid, KDE_TJ, 0, s>>>(segs, G, tps, keys, xmask, tile_range, tile_items, ntiles, items, D,
+  SV_LAUNCH(k_kde, grid, KDE_TJ, 0, s)(segs, G, tps, keys, xmask, tile_range, tile_items, ntiles, items, D,
                                  work_counter, terms);
 }

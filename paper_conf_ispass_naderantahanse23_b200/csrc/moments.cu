@@ -143,7 +143,7 @@ void launch_moments(const u32* kid, const u64* x, const u64* y, u64 n, u32 K, u3
   size_t smem = (size_t)kt * (8 + 8 + 4 + 12 + 16);
   cudaFuncSetAttribute(k_moments, cudaFuncAttributeMaxDynamicSharedMemorySize,
                        MOM_KT * (8 + 8 + 4 + 12 + 16));
-  k_moments<<<grid, MOM_THREADS, smem, s>>>(kid, x, y, n, K, k0, kt, part, blk_tot, errflags);
+  SV_LAUNCH(k_moments, grid, MOM_THREADS, smem, s)(kid, x, y, n, K, k0, kt, part, blk_tot, errflags);
 }
 
 // one thread per kernel: exact u128 sum over the blocks' partials, emitted as limb lanes
@@ -187,6 +187,6 @@ void launch_moments_reduce(const KMomPartial* part, const u64* blk_tot, int grid
                            u32 K, u64* lanes, u64* mm, u64* local_n, u64* tot_lanes, u64* tot_max,
                            bool do_totals, cudaStream_t s) {
   (void)K;
-  k_moments_reduce<<<div_up(kt, 256), 256, 0, s>>>(part, grid, k0, kt, lanes, mm, local_n);
-  if (do_totals) k_totals_reduce<<<1, 32, 0, s>>>(blk_tot, grid, tot_lanes, tot_max);
+  SV_LAUNCH(k_moments_reduce, div_up(kt, 256), 256, 0, s)(part, grid, k0, kt, lanes, mm, local_n);
+  if (do_totals) SV_LAUNCH(k_totals_reduce, 1, 32, 0, s)(blk_tot, grid, tot_lanes, tot_max);
 }

@@ -68,5 +68,5 @@ k_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, double* out) 
 
 void launch_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, double* out,
                     cudaStream_t s) {
-  k_predict<<<1, PR_THREADS, 0, s>>>(W, rx, ry, nstrata, out);
+  SV_LAUNCH(k_predict, 1, PR_THREADS, 0, s)(W, rx, ry, nstrata, out);
 }

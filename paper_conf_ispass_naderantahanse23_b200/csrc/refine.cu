@@ -69,7 +69,7 @@ k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, 
 
 void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T,
                     u32 tstride, u32* nt, u32* kind, cudaStream_t s) {
-  if (nseg) k_valleys<<<div_up(nseg, VAL_WARPS), 32 * VAL_WARPS, 0, s>>>(segs, nseg, G, shift, D, T,
+  if (nseg) SV_LAUNCH(k_valleys, div_up(nseg, VAL_WARPS), 32 * VAL_WARPS, 0, s)(segs, nseg, G, shift, D, T,
                                                                         tstride, nt, kind);
 }
 
@@ -124,6 +124,6 @@ void launch_part_stats(const SegDev* segs, u32 nseg, const u64* T, u32 tstride, 
                        const u32* part_off, u32 nparts, const u64* keys, u64 nkeys, u32 bx,
                        const u64* P1, const u64* P2, u64* lanes, u64* mm, u64* ab, cudaStream_t s) {
   if (nparts)
-    k_part_stats<<<div_up(nparts, 128), 128, 0, s>>>(segs, nseg, T, tstride, nt, part_off, nparts,
+    SV_LAUNCH(k_part_stats, div_up(nparts, 128), 128, 0, s)(segs, nseg, T, tstride, nt, part_off, nparts,
                                                       keys, nkeys, bx, P1, P2, lanes, mm, ab);
 }

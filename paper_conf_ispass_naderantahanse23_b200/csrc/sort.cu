@@ -117,9 +117,9 @@ size_t scan_u32_temp_bytes(u64 n) { return ((n + SC_TILE - 1) / SC_TILE + 2) * s
 void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s) {
   u32 nb = div_up(n ? n : 1, SC_TILE);
   u32* bsum = (u32*)temp;
-  k_scan_reduce<<<nb, SC_THREADS, 0, s>>>(in, n, bsum);
-  k_scan_blocks<<<1, SC_THREADS, 0, s>>>(bsum, nb, total);
-  k_scan_apply<<<nb, SC_THREADS, 0, s>>>(in, n, bsum, out);
+  SV_LAUNCH(k_scan_reduce, nb, SC_THREADS, 0, s)(in, n, bsum);
+  SV_LAUNCH(k_scan_blocks, 1, SC_THREADS, 0, s)(bsum, nb, total);
+  SV_LAUNCH(k_scan_apply, nb, SC_THREADS, 0, s)(in, n, bsum, out);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -163,7 +163,7 @@ void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u
   if (n == 0) return;
   u64 tiles = (n + (u64)CP_THREADS * CP_IPT - 1) / ((u64)CP_THREADS * CP_IPT);
   u64 grid = tiles < (u64)sv_num_sms() * 4 ? tiles : (u64)sv_num_sms() * 4;
-  k_t3_compact<<<(unsigned)grid, CP_THREADS, 0, s>>>(kid, x, n, t3rank, bx, keys_out, counter);
+  SV_LAUNCH(k_t3_compact, (unsigned)grid, CP_THREADS, 0, s)(kid, x, n, t3rank, bx, keys_out, counter);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -278,7 +278,8 @@ size_t radix_sort_temp_bytes(u64 n, bool with_vals) {
   return b;
 }
 
-int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s) {
+int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, int* passes) {
+  if (passes) *passes = 0;
   if (n <= 1 || nbits <= 0) return SIEVE_OK;
   u64 ntiles = (n + RS_TILE - 1) / RS_TILE;
   char* t = (char*)temp;
@@ -289,7 +290,7 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   void* stemp = t; t += ((scan_u32_temp_bytes(256 * ntiles) + 255) / 256) * 256;
   u64* dmask = (u64*)t;
   SV_CUDA(cudaMemsetAsync(dmask, 0, 8, s));
-  k_or_diff<<<sv_num_sms() * 2, 256, 0, s>>>(keys, n, dmask);
+  SV_LAUNCH(k_or_diff, sv_num_sms() * 2, 256, 0, s)(keys, n, dmask);
   u64 mask = 0;
   SV_CUDA(cudaMemcpyAsync(&mask, dmask, 8, cudaMemcpyDeviceToHost, s));
   SV_CUDA(cudaStreamSynchronize(s));
@@ -298,12 +299,13 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   u64* kin = keys; u32* vin = vals; u64* kout = kalt; u32* vout = valt;
   for (int shift = 0; shift < nbits; shift += 8) {
     if (((mask >> shift) & 255u) == 0) continue;   // constant digit: the pass is the identity
-    k_rs_hist<<<(unsigned)ntiles, RS_THREADS, 0, s>>>(kin, n, shift, (u32)ntiles, hist);
+    SV_LAUNCH(k_rs_hist, (unsigned)ntiles, RS_THREADS, 0, s)(kin, n, shift, (u32)ntiles, hist);
     scan_u32(hist, hist, 256 * ntiles, stemp, nullptr, s);
-    k_rs_scatter<<<(unsigned)ntiles, RS_THREADS, smem, s>>>(kin, vin, n, shift, (u32)ntiles, hist,
+    SV_LAUNCH(k_rs_scatter, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, shift, (u32)ntiles, hist,
                                                             kout, vout);
     u64* tk = kin; kin = kout; kout = tk;
     u32* tv = vin; vin = vout; vout = tv;
+    if (passes) (*passes)++;
   }
   if (kin != keys) {
     SV_CUDA(cudaMemcpyAsync(keys, kin, n * 8, cudaMemcpyDeviceToDevice, s));
@@ -414,7 +416,7 @@ void launch_prefix128(const u64* keys, u64 n, u64 xmask, u64* P1, u64* P2, void*
   // n+1 outputs: cover index n with one extra element slot
   u32 nb = div_up(n + 1, PX_TILE);
   Pair128* bsum = (Pair128*)temp;
-  k_px_reduce<<<nb, PX_THREADS, 0, s>>>(keys, n, xmask, bsum);
-  k_px_blocks<<<1, PX_THREADS, 0, s>>>(bsum, nb);
-  k_px_apply<<<nb, PX_THREADS, 0, s>>>(keys, n, xmask, bsum, P1, P2);
+  SV_LAUNCH(k_px_reduce, nb, PX_THREADS, 0, s)(keys, n, xmask, bsum);
+  SV_LAUNCH(k_px_blocks, 1, PX_THREADS, 0, s)(bsum, nb);
+  SV_LAUNCH(k_px_apply, nb, PX_THREADS, 0, s)(keys, n, xmask, bsum, P1, P2);
 }

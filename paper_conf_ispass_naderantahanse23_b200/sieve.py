@@ -34,8 +34,10 @@ EXPORTED = [
     "sieve_load_trace", "sieve_trace_free", "sieve_params_default", "sieve_stratify",
     "sieve_strata_count", "sieve_strata_copy", "sieve_strata_stats", "sieve_strata_free",
     "sieve_segment_count", "sieve_segment_get", "sieve_predict", "sieve_last_error",
-    "sieve_version", "sieve_u128_to_limbs", "sieve_limbs_to_u128",
+    "sieve_version", "sieve_u128_to_limbs", "sieve_limbs_to_u128", "sieve_ctx_set_timing",
+    "sieve_timing_get", "sieve_kernel_launches",
 ]
+PHASES = ["moments", "compact", "sort", "prefix", "kde", "refine", "assign", "reps", "predict"]
 
 
 class Params(ctypes.Structure):
@@ -89,6 +91,9 @@ def _load():
         "sieve_version": ([], ctypes.c_char_p),
         "sieve_u128_to_limbs": ([u64, u64, vp], None),
         "sieve_limbs_to_u128": ([vp, P(u64), P(u64)], None),
+        "sieve_ctx_set_timing": ([vp, i32], i32),
+        "sieve_timing_get": ([vp, u32, P(ctypes.c_double), P(u64), P(u64)], i32),
+        "sieve_kernel_launches": ([], u64),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -176,6 +181,19 @@ class Ctx:
         self.device, self.rank, self.world = device, rank, world if group is None else group.world
         self._group = group
 
+    def set_timing(self, enable=True):
+        _check(_L.sieve_ctx_set_timing(self._h, 1 if enable else 0), "sieve_ctx_set_timing")
+
+    def timing(self):
+        """{phase: (ms, calls, work)} accumulated since set_timing(True)."""
+        out = {}
+        for i, name in enumerate(PHASES):
+            ms, calls, work = ctypes.c_double(), ctypes.c_uint64(), ctypes.c_uint64()
+            _check(_L.sieve_timing_get(self._h, i, ctypes.byref(ms), ctypes.byref(calls),
+                                       ctypes.byref(work)), "sieve_timing_get")
+            out[name] = (ms.value, calls.value, work.value)
+        return out
+
     def close(self):
         if getattr(self, "_h", None):
             _L.sieve_ctx_destroy(self._h)
@@ -183,6 +201,10 @@ class Ctx:
 
     def __del__(self):
         self.close()
+
+
+def kernel_launches():
+    return _L.sieve_kernel_launches()
 
 
 def _col(a, dtype, device_ok=True):

@@ -54,6 +54,10 @@ def assert_tables_equal(gpu_table, ora_table):
 
 
 def assert_segments_equal(gs, os_):
+    # the library lists segments round by round; the oracle kernel by kernel: compare in
+    # (round, kernel, lo) order
+    key = lambda s: (s["round"], s["kernel_id"], s["lo"])
+    gs, os_ = sorted(gs, key=key), sorted(os_, key=key)
     assert len(gs) == len(os_)
     for a, b in zip(gs, os_):
         for k in ["kernel_id", "round", "split_kind", "n_cuts", "lo", "hi", "count"]:
