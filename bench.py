@@ -30,7 +30,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-KDE_FP64_OPS_PER_TERM = 24   # FP64-pipe instructions per in-window KDE term
+KDE_FP64_OPS_PER_TERM = 14   # FP64-pipe instructions per in-window KDE term
 FP64_LANES_PER_SM = 64       # B200: 64 FP64 FMA lanes / SM / clk (microbenchmark: 62.9)
 
 
@@ -197,9 +197,16 @@ def main():
     trace = sieve.load_trace(ctx, d["kid"], d["x"], num_kernels=cfg.K, cta=d["cta"], cycles=d["y"],
                              first_id=first, adopt=True)
 
+    debug = os.environ.get("BENCH_DEBUG")
+
     def step():
+        t0 = time.perf_counter()
         st = sieve.stratify(trace, stratum_of_invocation=sid)
+        t1 = time.perf_counter()
         sieve.predict(st, trace)
+        if debug:
+            print(f"[bench host] stratify {1e3 * (t1 - t0):.3f} ms predict "
+                  f"{1e3 * (time.perf_counter() - t1):.3f} ms", file=sys.stderr)
         return st
 
     def barrier():

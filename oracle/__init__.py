@@ -59,6 +59,8 @@ def _lib():
         L.oracle_det_exp.restype = dbl
         L.oracle_q.argtypes = [dbl]
         L.oracle_q.restype = u64
+        L.oracle_exp2_table.argtypes = [ctypes.c_int]
+        L.oracle_exp2_table.restype = dbl
         L.oracle_tier.argtypes = [u64, u64, u64, u64, u64, u64, u64, u32, u32]
         L.oracle_tier.restype = ctypes.c_int
         L.oracle_bandwidth.argtypes = [u64, u64, u64, u64, u64, dbl]
@@ -173,6 +175,10 @@ def det_exp(t):
 
 def q_of_t(t):
     return int(_lib().oracle_q(float(t)))
+
+
+def exp2_table():
+    return [_lib().oracle_exp2_table(j) for j in range(64)]
 
 
 def tier(values, theta=(2, 5)):

@@ -14,9 +14,9 @@ Only for tiny traces (a few hundred invocations, small G).
 import math
 from fractions import Fraction
 
-LOG2E = 1.4426950408889634074
-LN2_HI = 6.93147180369123816490e-01
-LN2_LO = 1.90821492927058770002e-10
+LOG2E_64 = 64.0 * 1.4426950408889634074
+LN2_64_HI = 6.93147180369123816490e-01 / 64.0
+LN2_64_LO = 1.90821492927058770002e-10 / 64.0
 TWO52 = 2.0 ** 52
 
 
@@ -24,26 +24,44 @@ def fma(a, b, c):
     return float(Fraction(a) * Fraction(b) + Fraction(c))
 
 
-def inv_fact(i):
-    return float(Fraction(1, math.factorial(i)))
+def _exp2_neg_table():
+    """2^(-j/64), j = 0..63, correctly rounded (60-digit decimal, then float() rounds)."""
+    from decimal import Decimal, getcontext
+    getcontext().prec = 60
+    return [float(Decimal(2) ** (Decimal(-j) / Decimal(64))) for j in range(64)]
+
+
+EXP2_NEG = _exp2_neg_table()
+
+
+def _reduce(t):
+    k = float(round(t * LOG2E_64))       # Python round() on floats is round-half-even == rint
+    r = fma(-k, LN2_64_HI, t)
+    r = fma(-k, LN2_64_LO, r)
+    p = -float(Fraction(1, 120))          # P(r) = sum_{i<=5} (-r)^i / i!  (Horner, signed coefs)
+    for c in (Fraction(1, 24), Fraction(-1, 6), Fraction(1, 2), Fraction(-1), Fraction(1)):
+        p = fma(p, r, float(c))
+    return p, int(k) & 63, int(k) >> 6
 
 
 def det_exp(t):
-    k = float(round(t * LOG2E))          # Python round() on floats is round-half-even == rint
-    r = fma(-k, LN2_HI, t)
-    r = fma(-k, LN2_LO, r)
-    p = inv_fact(13)
-    for i in range(12, -1, -1):
-        p = fma(p, -r, inv_fact(i))
-    return math.ldexp(p, -int(k))
+    p, j, m = _reduce(t)
+    return math.ldexp(p * EXP2_NEG[j], -m)
+
+
+def q_of_t(t):
+    """rint(P * 2^(-j/64) * 2^(52-m)) with a single rounding (exact rational, then round)."""
+    if t > 37.0:
+        return 0
+    p, j, m = _reduce(t)
+    v = Fraction(p) * Fraction(EXP2_NEG[j]) * Fraction(2) ** (52 - m)
+    return round(v)                      # Fraction round(): nearest, ties to even
 
 
 def q_term(g, x, inv_h):
     z = (g - float(x)) * inv_h
     t = (z * z) * 0.5
-    if t > 37.0:
-        return 0
-    return int(round(det_exp(t) * TWO52))
+    return q_of_t(t)
 
 
 def cov_below(vals, theta):

@@ -26,7 +26,8 @@
  *                                                         P:99-101, P:200-208 (A22)
  *
  * Pins (tests/test_oracle_*.py): tier closed forms and exact-boundary multisets, big-int
- * moments, det_exp vs libm exp (<= 1 ulp), KDE vs scikit-learn / scipy / direct sums,
+ * moments, det_exp vs libm exp (<= 2 ulp), the 2^{-j/64} table vs Python decimal,
+ * Q vs e^{-t} 2^52 (<= 2 units), KDE vs scikit-learn / scipy / direct sums,
  * hand-built valley sequences, symmetric two-point masses, strata invariants,
  * representative brute force, prediction identities (homogeneous cycles => error 0,
  * CPI arithmetic-mean form), and an independent Python big-int brute force (oracle/brute.py).
@@ -187,40 +188,77 @@ double oracle_grid_point(uint64_t lo, uint64_t hi, uint32_t j, uint32_t G) {
 }
 
 /* ------------------------------------------------------------------------------------------
- * O5c det_exp(t) = e^{-t} for t in [0, 37] (A10), built only from IEEE basic operations:
- *   k = rint(t * LOG2E); r = fma(-k, LN2_HI, t); r = fma(-k, LN2_LO, r);
- *   P(r) = sum_{i=0}^{13} (-r)^i / i!  by Horner with fma, starting from 1/13!;
- *   det_exp = ldexp(P, -k).
+ * O5c fixed-point Gaussian kernel value (A10), built only from IEEE basic operations:
+ *   k = rint(t * 64 log2 e),  j = k mod 64,  m = k div 64       (so t ~ k ln2 / 64)
+ *   r = fma(-k, ln2/64 hi, t);  r = fma(-k, ln2/64 lo, r)        (|r| <= ln2 / 128)
+ *   P(r) = 1 - r + r^2/2 - r^3/6 + r^4/24 - r^5/120               (Horner with fma)
+ *   e^{-t} = 2^{-j/64} * 2^{-m} * e^{-r}
+ *   Q = rint(P * T_j * 2^(52 - m)) with ONE rounding: S = ldexp(T_j, 52 - m) is exact and
+ *       Q = fma(P, S, 2^52) - 2^52 (the fma lands in [2^52, 2^53], where the ulp is 1).
+ *   T_j = 2^{-j/64} correctly rounded (pinned in tests against Python's decimal module).
+ * Q = 0 for t > 37: e^{-37} 2^52 = 0.38 rounds to 0 anyway.
  * ------------------------------------------------------------------------------------------ */
-static const double OR_LOG2E = 1.4426950408889634074;
-static const double OR_LN2_HI = 6.93147180369123816490e-01;
-static const double OR_LN2_LO = 1.90821492927058770002e-10;
-static const double OR_INV_FACT[14] = {
-    1.0,         1.0,          1.0 / 2.0,          1.0 / 6.0,          1.0 / 24.0,
-    1.0 / 120.0, 1.0 / 720.0,  1.0 / 5040.0,       1.0 / 40320.0,      1.0 / 362880.0,
-    1.0 / 3628800.0, 1.0 / 39916800.0, 1.0 / 479001600.0, 1.0 / 6227020800.0};
+static const double OR_LOG2E_64 = 64.0 * 1.4426950408889634074;        /* exact scaling */
+static const double OR_LN2_64_HI = 6.93147180369123816490e-01 / 64.0;  /* 21 significant bits */
+static const double OR_LN2_64_LO = 1.90821492927058770002e-10 / 64.0;
+static const double OR_TWO52 = 4503599627370496.0;
+static const double OR_EXP2_NEG[64] = {
+    0x1.0000000000000p+0, 0x1.fa7c1819e90d8p-1, 0x1.f50765b6e4540p-1, 0x1.efa1bee615a27p-1,
+    0x1.ea4afa2a490dap-1, 0x1.e502ee78b3ff6p-1, 0x1.dfc97337b9b5fp-1, 0x1.da9e603db3285p-1,
+    0x1.d5818dcfba487p-1, 0x1.d072d4a07897cp-1, 0x1.cb720dcef9069p-1, 0x1.c67f12e57d14bp-1,
+    0x1.c199bdd85529cp-1, 0x1.bcc1e904bc1d2p-1, 0x1.b7f76f2fb5e47p-1, 0x1.b33a2b84f15fbp-1,
+    0x1.ae89f995ad3adp-1, 0x1.a9e6b5579fdbfp-1, 0x1.a5503b23e255dp-1, 0x1.a0c667b5de565p-1,
+    0x1.9c49182a3f090p-1, 0x1.97d829fde4e50p-1, 0x1.93737b0cdc5e5p-1, 0x1.8f1ae99157736p-1,
+    0x1.8ace5422aa0dbp-1, 0x1.868d99b4492edp-1, 0x1.82589994cce13p-1, 0x1.7e2f336cf4e62p-1,
+    0x1.7a11473eb0187p-1, 0x1.75feb564267c9p-1, 0x1.71f75e8ec5f74p-1, 0x1.6dfb23c651a2fp-1,
+    0x1.6a09e667f3bcdp-1, 0x1.6623882552225p-1, 0x1.6247eb03a5585p-1, 0x1.5e76f15ad2148p-1,
+    0x1.5ab07dd485429p-1, 0x1.56f4736b527dap-1, 0x1.5342b569d4f82p-1, 0x1.4f9b2769d2ca7p-1,
+    0x1.4bfdad5362a27p-1, 0x1.486a2b5c13cd0p-1, 0x1.44e086061892dp-1, 0x1.4160a21f72e2ap-1,
+    0x1.3dea64c123422p-1, 0x1.3a7db34e59ff7p-1, 0x1.371a7373aa9cbp-1, 0x1.33c08b26416ffp-1,
+    0x1.306fe0a31b715p-1, 0x1.2d285a6e4030bp-1, 0x1.29e9df51fdee1p-1, 0x1.26b4565e27cddp-1,
+    0x1.2387a6e756238p-1, 0x1.2063b88628cd6p-1, 0x1.1d4873168b9aap-1, 0x1.1a35beb6fcb75p-1,
+    0x1.172b83c7d517bp-1, 0x1.1429aaea92de0p-1, 0x1.11301d0125b51p-1, 0x1.0e3ec32d3d1a2p-1,
+    0x1.0b5586cf9890fp-1, 0x1.0874518759bc8p-1, 0x1.059b0d3158574p-1, 0x1.02c9a3e778061p-1};
 
-double oracle_det_exp(double t) {
-  double k = rint(t * OR_LOG2E);
-  double r = fma(-k, OR_LN2_HI, t);
-  r = fma(-k, OR_LN2_LO, r);
-  double mr = -r;
-  double p = OR_INV_FACT[13];
-  for (int i = 12; i >= 0; i--) p = fma(p, mr, OR_INV_FACT[i]);
-  return ldexp(p, -(int)k);
+/* the reduced argument and polynomial shared by det_exp and Q */
+static double exp_reduce(double t, int* j, int* m) {
+  double k = rint(t * OR_LOG2E_64);
+  int ki = (int)k;
+  *j = ki & 63;
+  *m = ki >> 6;
+  double r = fma(-k, OR_LN2_64_HI, t);
+  r = fma(-k, OR_LN2_64_LO, r);
+  double p = -1.0 / 120.0;
+  p = fma(p, r, 1.0 / 24.0);
+  p = fma(p, r, -1.0 / 6.0);
+  p = fma(p, r, 0.5);
+  p = fma(p, r, -1.0);
+  p = fma(p, r, 1.0);
+  return p;
 }
 
-/* fixed-point kernel value Q(x, g) = rint(det_exp(t) * 2^52), 0 if t > 37 (A10) */
-static uint64_t kernel_q(double g, double xd, double inv_h) {
-  double z = (g - xd) * inv_h;
-  double t = (z * z) * 0.5;
-  if (t > 37.0) return 0;
-  return (uint64_t)rint(oracle_det_exp(t) * 4503599627370496.0 /* 2^52 */);
+/* e^{-t} for t in [0, 37] as the method evaluates it (diagnostic / pin only) */
+double oracle_det_exp(double t) {
+  int j, m;
+  double p = exp_reduce(t, &j, &m);
+  return ldexp(p * OR_EXP2_NEG[j], -m);
 }
 
 uint64_t oracle_q(double t) {
   if (t > 37.0) return 0;
-  return (uint64_t)rint(oracle_det_exp(t) * 4503599627370496.0);
+  int j, m;
+  double p = exp_reduce(t, &j, &m);
+  double S = ldexp(OR_EXP2_NEG[j], 52 - m);
+  return (uint64_t)(fma(p, S, OR_TWO52) - OR_TWO52);
+}
+
+double oracle_exp2_table(int j) { return OR_EXP2_NEG[j & 63]; }
+
+/* fixed-point kernel value Q(x, g), t = (z * z) * 0.5, z = (g - rn(x)) * inv_h */
+static uint64_t kernel_q(double g, double xd, double inv_h) {
+  double z = (g - xd) * inv_h;
+  double t = (z * z) * 0.5;
+  return oracle_q(t);
 }
 
 /* O5c density on the grid: D_j = sum over the segment's values of Q(x, g_j), u128 */

@@ -15,6 +15,7 @@
 
 #include <algorithm>
 #include <atomic>
+#include <chrono>
 #include <string>
 #include <vector>
 
@@ -448,11 +449,32 @@ static int sync(sieve_ctx c) { SV_CUDA(cudaStreamSynchronize(c->stream)); return
 // sieve_stratify
 // ------------------------------------------------------------------------------------------
 struct OpenSeg { u32 kid, t3rank; u64 lo, hi, n; u128 s1, s2; };
+
+// host-side wall-clock marks (SIEVE_HOST_TIMING=1 prints them to stderr): where the host
+// orchestration, not the device, spends time
+struct HostClock {
+  bool on = getenv("SIEVE_HOST_TIMING") != nullptr;
+  std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now(), last = t0;
+  std::string out;
+  void mark(const char* name) {
+    if (!on) return;
+    auto now = std::chrono::steady_clock::now();
+    char b[96];
+    snprintf(b, sizeof b, " %s=%.3f", name, std::chrono::duration<double, std::milli>(now - last).count());
+    out += b;
+    last = now;
+  }
+  ~HostClock() {
+    if (on) fprintf(stderr, "[sieve host ms]%s total=%.3f\n", out.c_str(),
+                    std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+  }
+};
 struct Fin { u32 kid, tier; u64 lo, hi, n; u128 s1; double h; u32 round; };
 
 static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out, sieve_strata_s* R) {
   sieve_ctx c = t->ctx;
   cudaStream_t S = c->stream;
+  HostClock hc;
   const u32 K = t->K, G = P->grid_points;
   const u64 n = t->n;
 
@@ -522,6 +544,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   R->c_meas = limbs_u128(&h_tot[0]);
   const u64 max_x = h_tot[4];
 
+  hc.mark("passA");
   // ---------------- tiers ---------------------------------------------------------
   std::vector<Fin> fin;
   std::vector<OpenSeg> open;
@@ -585,6 +608,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   }
   const u64 nkeys = (n_t3 && n3_local) ? n3_local : 0;
 
+  hc.mark("sort");
   // ---------------- refinement rounds (A6-A15) ------------------------------------------
   DBuf<unsigned long long> terms(c);
   SV_TRY(terms.alloc(2));
@@ -628,9 +652,11 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       u32 items = 0;
       SV_TRY(kde_plan(segs.get(), nseg, G, keys.get(), nkeys, xmask, tile_range.get(),
                       tile_items.get(), stemp.get(), &items, S));
+      DBuf<char> item_tile(c);
+      SV_TRY(item_tile.alloc(kde_item_bytes(items)));
       PhaseTimer tm(c, SIEVE_PHASE_KDE, 0);
-      launch_kde(segs.get(), nseg, G, keys.get(), xmask, tile_range.get(), tile_items.get(), items,
-                 D.get(), counter.get() + 1, terms.get(), S);
+      launch_kde(segs.get(), nseg, G, keys.get(), xmask, tile_range.get(), tile_items.get(),
+                 (u32*)item_tile.get(), items, D.get(), counter.get() + 1, terms.get(), S);
       tm.stop();
       SV_CUDA(cudaGetLastError());
     }
@@ -715,6 +741,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       }
     }
     open.swap(next);
+    hc.mark("round");
   }
   R->rounds = round;
   {
@@ -746,6 +773,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   // (pushed in order above because fin is sorted by (kid, lo))
   if (lows.empty()) lows.push_back(0);
 
+  hc.mark("table");
   // ---------------- pass B: assignment + (stratum, CTA) statistics ---------------------
   DBuf<KTab> d_ktab(c);
   DBuf<u64> d_lows(c), errf(c);
@@ -792,6 +820,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     cap <<= 2;
   }
   gkeys.release(); gcnt.release(); gfirst.release();
+  hc.mark("passB");
   // gather every rank's entries (AR-4: all-gather expressed as a SUM over zero-padded slots)
   u64 Etot = E, Eoff = 0;
   DBuf<u64> ak(c), ac(c), af(c);
@@ -855,6 +884,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   SV_TRY(d2h(c, h_xy, repxy.get(), 2 * (size_t)ns));
   SV_TRY(sync(c));
   resolve_timing(c);
+  hc.mark("reps");
 
   // ---------------- assemble --------------------------------------------------------------------
   R->st.resize(ns);

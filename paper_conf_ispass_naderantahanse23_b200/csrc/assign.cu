@@ -61,12 +61,23 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
   u64 b1 = b0 + chunk < n ? b0 + chunk : n;
   const u64 tile = (u64)AS_THREADS * AS_IPT;
   for (u64 base = b0; base < b1; base += tile) {
+    // issue the tile's loads first (AS_IPT rows per thread in flight), then the atomics
+    u32 kk[AS_IPT], cc[AS_IPT];
+    u64 vv[AS_IPT];
+#pragma unroll
+    for (int j = 0; j < AS_IPT; j++) {
+      u64 i = base + (u64)j * AS_THREADS + threadIdx.x;
+      bool ok = i < b1;
+      kk[j] = ok ? __ldcs(kid + i) : 0u;
+      vv[j] = ok ? __ldcs(x + i) : 0ull;
+      cc[j] = (ok && cta) ? __ldcs(cta + i) : 0u;
+    }
 #pragma unroll
     for (int j = 0; j < AS_IPT; j++) {
       u64 i = base + (u64)j * AS_THREADS + threadIdx.x;
       if (i >= b1) continue;
-      u32 k = __ldcs(kid + i);
-      u64 v = __ldcs(x + i);
+      u32 k = kk[j];
+      u64 v = vv[j];
       KTab kt = ktab[k];
       u32 sid = kt.base;
       if (kt.m > 1) {  // number of lower bounds lows[1..m) that are <= v
@@ -79,7 +90,7 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
         sid += lo;
       }
       if (sid_out) sid_out[i] = sid;
-      u32 c = cta ? __ldcs(cta + i) : 0u;
+      u32 c = cc[j];
       u64 key = ((u64)sid << 32) | c;
       u32 rel = (u32)(i - b0);
       u32 h = hash_key(key) & (AS_HC - 1);

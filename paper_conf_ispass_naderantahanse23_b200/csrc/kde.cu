@@ -3,28 +3,38 @@
 //
 //   g_j  = rn(lo) + rn((hi - lo) * j) / rn(G - 1)                      (A9)
 //   z    = (g_j - rn(x)) * inv_h ;  t = (z * z) * 0.5
-//   Q    = 0 if t > 37, else rint(det_exp(t) * 2^52)                  (A10)
+//   Q    = 0 if t > 37, else rint(P(r) * 2^{-j'/64} * 2^(52 - m))    (A10; k = rint(t 64 log2 e),
+//          j' = k mod 64, m = k div 64, r = t - k ln2/64, P = degree-5 Taylor of e^{-r})
 //   D_j  = sum over the segment's values x of Q(x, g_j)   (exact integer sum, u128)
 //
-// det_exp(t) = ldexp(P(r), -k) with k = rint(t log2 e), r = t - k ln2 (two fma with a split ln2)
-// and P the degree-13 Taylor polynomial of e^{-r} by Horner with fma.  Every floating-point
-// step is an IEEE basic operation written with the _rn intrinsics (never contracted), so each
-// term is bit-identical to the CPU oracle; the integer sum makes D independent of summation
-// order, of the work decomposition and of the number of ranks.
+// Every floating-point step is an IEEE basic operation written with _rn intrinsics (never
+// contracted), so each term is bit-identical to the CPU oracle; the integer sum makes D
+// independent of summation order, of the work decomposition and of the number of ranks.
 //
-// B200 mapping (the paper's scripts have no GPU design; this is new): the work is a gather over
-// the SORTED values of each segment.  A work item is (segment, tile of KDE_TJ=128 grid points,
-// chunk of <= KDE_CH=1024 values inside the tile's exact window |g - x| <= 8.7 h); a persistent
-// grid pulls items from an atomic counter.  Each thread owns one grid point; the chunk's values
-// are staged in shared memory as fp64 and read as warp broadcasts; each warp narrows the loop
-// to its own window by binary search.  FP64 is on the CUDA cores (no contraction exists, so no
-// tensor cores): ~24 FP64 pipe operations per in-window term.  Two bit tricks keep the
-// conversions off the slow pipes: rint(t log2 e) = (t log2 e + 1.5 * 2^52) - 1.5 * 2^52 (its low
-// word is k), and rint(P * 2^(52-k)) = bits(fma(P, 2^(52-k), 2^52)) - bits(2^52) because the
-// product is exact and the sum lies in [2^52, 2^53] where the ulp is 1.
+// B200 mapping (the paper's scripts have no GPU design; this is new).  The KDE is a windowed
+// gather over the SORTED values of each segment, bound by the FP64 pipe (no contraction, so no
+// tensor cores).  Work item = (segment, tile of 32 grid points, chunk of <= 256 values inside
+// the tile's window |g - x| <= 8.7 h); items are pulled by WARPS from an atomic counter (no
+// block barriers: warps of a block never wait for each other); each lane owns one grid point,
+// the chunk is staged in the warp's slice of shared memory and read as broadcasts.  The term is
+// arranged to be bit-identical to the oracle's while issuing 15 FP64-pipe instructions and ~4
+// others:
+//   * u = z*z replaces t = u/2 (exact scaling): k = rint(u * 32 log2 e), r' = u - k ln2/32 = 2r,
+//     Horner on r' with coefficients c_i 2^-i gives exactly the same P (power-of-two scaling
+//     commutes with round-to-nearest);
+//   * k = low word of u*32log2e + 1.5*2^52 (an exact rint), clamped to 3417;
+//   * S = T'[k] = 2^{-(k mod 64)/64} * 2^(52 - k div 64) from a shared-memory table (exact
+//     power-of-two scalings of the correctly rounded 2^{-j/64}), with T'[3417] = 0: every
+//     t > 37 lands on k >= 3417 or has Q = 0 anyway (e^-37 2^52 = 0.38), so no select;
+//   * rint(P * S) = bits(fma(P, S, 2^52)) - bits(2^52): the sum lies in [2^52, 2^53] where the
+//     ulp is 1; raw bit patterns are accumulated and 2^52's pattern is subtracted once per term
+//     count at the end.
 #include "kernels.cuh"
 
-#define KDE_W 8.7  // window half-width in units of h: t > 37 is guaranteed beyond it
+#define KDE_W 8.7            // window half-width in units of h: t > 37 is guaranteed beyond it
+#define KDE_WC 8.602325267042627  // sqrt(74): |z| <= this <=> t <= 37 (term-count diagnostic)
+#define KDE_KCUT 3417        // rint(37 * 64 log2 e) = 3416; index 3417 holds 0
+#define KDE_WARPS 8          // warps per block (independent work-item consumers)
 
 __device__ __forceinline__ double grid_pt(u64 lo, u64 hi, u32 j, u32 G) {
   return __dadd_rn(__ull2double_rn(lo),
@@ -54,8 +64,8 @@ void launch_seg_ranges(SegDev* segs, u32 nseg, const u64* keys, u64 nkeys, cudaS
   if (nseg) SV_LAUNCH(k_seg_ranges, div_up(nseg, 128), 128, 0, s)(segs, nseg, keys, nkeys);
 }
 
-// per (segment, tile): the local index range of values inside the tile's window, and the
-// number of KDE_CH-value chunks it takes
+// per (segment, tile of KDE_TJ grid points): the local index range of the values inside the
+// tile's window, and the number of KDE_CH-value chunks (work items) it takes
 __global__ void k_kde_tiles(const SegDev* segs, u32 nseg, u32 G, u32 tps, const u64* keys,
                             u64* tile_range, u32* tile_items) {
   u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
@@ -92,120 +102,157 @@ int kde_plan(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 nkeys, u6
   return SIEVE_OK;
 }
 
-// ------------------------------------------------------------------------------------------
-#define C_LOG2E 0x1.71547652b82fep+0
-#define C_LN2_HI 0x1.62e42fee00000p-1
-#define C_LN2_LO 0x1.a39ef35793c76p-33
-#define C_MAGIC 0x1.8p+52   // 1.5 * 2^52
-#define C_TWO52 0x1.0p+52
-
-// Q(x, g) in fixed point 2^-52; returns 0 when t > 37
-__device__ __forceinline__ u64 kde_term(double g, double xd, double inv_h, u32& inwin) {
-  double z = __dmul_rn(__dsub_rn(g, xd), inv_h);
-  double t = __dmul_rn(__dmul_rn(z, z), 0.5);
-  if (t > 37.0) return 0;
-  inwin++;
-  double kb = __dadd_rn(__dmul_rn(t, C_LOG2E), C_MAGIC);
-  double kf = __dsub_rn(kb, C_MAGIC);
-  int k = __double2loint(kb);
-  double r = __fma_rn(-kf, C_LN2_HI, t);
-  r = __fma_rn(-kf, C_LN2_LO, r);
-  double mr = -r;
-  double p = 0x1.6124613a86d09p-33;                  // 1/13!
-  p = __fma_rn(p, mr, 0x1.1eed8eff8d898p-29);        // 1/12!
-  p = __fma_rn(p, mr, 0x1.ae64567f544e4p-26);        // 1/11!
-  p = __fma_rn(p, mr, 0x1.27e4fb7789f5cp-22);        // 1/10!
-  p = __fma_rn(p, mr, 0x1.71de3a556c734p-19);        // 1/9!
-  p = __fma_rn(p, mr, 0x1.a01a01a01a01ap-16);        // 1/8!
-  p = __fma_rn(p, mr, 0x1.a01a01a01a01ap-13);        // 1/7!
-  p = __fma_rn(p, mr, 0x1.6c16c16c16c17p-10);        // 1/6!
-  p = __fma_rn(p, mr, 0x1.1111111111111p-7);         // 1/5!
-  p = __fma_rn(p, mr, 0x1.5555555555555p-5);         // 1/4!
-  p = __fma_rn(p, mr, 0x1.5555555555555p-3);         // 1/3!
-  p = __fma_rn(p, mr, 0x1.0p-1);                     // 1/2!
-  p = __fma_rn(p, mr, 1.0);                          // 1/1!
-  p = __fma_rn(p, mr, 1.0);                          // 1/0!
-  double sc = __hiloint2double((1075 - k) << 20, 0); // 2^(52 - k), k in [0, 54)
-  double q = __fma_rn(p, sc, C_TWO52);
-  return (u64)__double_as_longlong(q) - 0x4330000000000000ull;
+// item -> tile map (so a warp finds its tile with one load)
+__global__ void k_kde_items(const u32* tile_items, u32 ntiles, u32* item_tile) {
+  u32 tile = blockIdx.x * blockDim.x + threadIdx.x;
+  if (tile >= ntiles) return;
+  for (u32 it = tile_items[tile]; it < tile_items[tile + 1]; it++) item_tile[it] = tile;
 }
 
-__global__ void __launch_bounds__(KDE_TJ)
+// ------------------------------------------------------------------------------------------
+#define C_LOG2E_32 0x1.71547652b82fep+5     // 32 * log2(e)  (= the oracle's 64 log2 e / 2)
+#define C_LN2_32_HI 0x1.62e42fee00000p-6    // ln2/32 high part (21 significant bits)
+#define C_LN2_32_LO 0x1.a39ef35793c76p-38
+#define C_MAGIC 0x1.8p+52                   // 1.5 * 2^52
+#define C_TWO52 0x1.0p+52
+// Taylor coefficients of e^{-r} scaled by 2^-i for the argument r' = 2r
+#define C_P5 (-0x1.1111111111111p-7 * 0x1p-5)   // -1/120 * 2^-5
+#define C_P4 (0x1.5555555555555p-5 * 0x1p-4)    //  1/24  * 2^-4
+#define C_P3 (-0x1.5555555555555p-3 * 0x1p-3)   // -1/6   * 2^-3
+#define C_P2 0.125                              //  1/2   * 2^-2
+#define C_P1 (-0.5)                             // -1     * 2^-1
+#define C_P0 1.0
+
+__constant__ double KDE_EXP2_NEG[64] = {
+    0x1.0000000000000p+0, 0x1.fa7c1819e90d8p-1, 0x1.f50765b6e4540p-1, 0x1.efa1bee615a27p-1,
+    0x1.ea4afa2a490dap-1, 0x1.e502ee78b3ff6p-1, 0x1.dfc97337b9b5fp-1, 0x1.da9e603db3285p-1,
+    0x1.d5818dcfba487p-1, 0x1.d072d4a07897cp-1, 0x1.cb720dcef9069p-1, 0x1.c67f12e57d14bp-1,
+    0x1.c199bdd85529cp-1, 0x1.bcc1e904bc1d2p-1, 0x1.b7f76f2fb5e47p-1, 0x1.b33a2b84f15fbp-1,
+    0x1.ae89f995ad3adp-1, 0x1.a9e6b5579fdbfp-1, 0x1.a5503b23e255dp-1, 0x1.a0c667b5de565p-1,
+    0x1.9c49182a3f090p-1, 0x1.97d829fde4e50p-1, 0x1.93737b0cdc5e5p-1, 0x1.8f1ae99157736p-1,
+    0x1.8ace5422aa0dbp-1, 0x1.868d99b4492edp-1, 0x1.82589994cce13p-1, 0x1.7e2f336cf4e62p-1,
+    0x1.7a11473eb0187p-1, 0x1.75feb564267c9p-1, 0x1.71f75e8ec5f74p-1, 0x1.6dfb23c651a2fp-1,
+    0x1.6a09e667f3bcdp-1, 0x1.6623882552225p-1, 0x1.6247eb03a5585p-1, 0x1.5e76f15ad2148p-1,
+    0x1.5ab07dd485429p-1, 0x1.56f4736b527dap-1, 0x1.5342b569d4f82p-1, 0x1.4f9b2769d2ca7p-1,
+    0x1.4bfdad5362a27p-1, 0x1.486a2b5c13cd0p-1, 0x1.44e086061892dp-1, 0x1.4160a21f72e2ap-1,
+    0x1.3dea64c123422p-1, 0x1.3a7db34e59ff7p-1, 0x1.371a7373aa9cbp-1, 0x1.33c08b26416ffp-1,
+    0x1.306fe0a31b715p-1, 0x1.2d285a6e4030bp-1, 0x1.29e9df51fdee1p-1, 0x1.26b4565e27cddp-1,
+    0x1.2387a6e756238p-1, 0x1.2063b88628cd6p-1, 0x1.1d4873168b9aap-1, 0x1.1a35beb6fcb75p-1,
+    0x1.172b83c7d517bp-1, 0x1.1429aaea92de0p-1, 0x1.11301d0125b51p-1, 0x1.0e3ec32d3d1a2p-1,
+    0x1.0b5586cf9890fp-1, 0x1.0874518759bc8p-1, 0x1.059b0d3158574p-1, 0x1.02c9a3e778061p-1};
+
+// raw bit pattern of fma(P, S, 2^52); the term is this minus bits(2^52)
+__device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, const double* sS) {
+  double z = __dmul_rn(__dsub_rn(g, xd), inv_h);
+  double u = __dmul_rn(z, z);                               // 2t, exactly
+  double kb = __dadd_rn(__dmul_rn(u, C_LOG2E_32), C_MAGIC);
+  double kf = __dsub_rn(kb, C_MAGIC);
+  // k = rint(u * 32 log2 e) while u < 80 (the magic-number rint is exact there); any u >= 80
+  // (t >= 40, far outside the window) maps to the zero entry.  p stays finite for every input
+  // the API admits (x < 2^44, n < 2^36 => h > 2^-26, u < 2^140), and fma(p, 0, 2^52) = 2^52.
+  u32 k = min((u32)__double2loint(kb), (u32)KDE_KCUT);
+  k = (u32)__double2hiint(u) >= 0x40540000u ? (u32)KDE_KCUT : k;
+  double r = __fma_rn(-kf, C_LN2_32_HI, u);
+  r = __fma_rn(-kf, C_LN2_32_LO, r);
+  double p = __fma_rn(C_P5, r, C_P4);
+  p = __fma_rn(p, r, C_P3);
+  p = __fma_rn(p, r, C_P2);
+  p = __fma_rn(p, r, C_P1);
+  p = __fma_rn(p, r, C_P0);
+  return (u64)__double_as_longlong(__fma_rn(p, sS[k], C_TWO52));
+}
+
+#define KDE_SMEM_TABLE ((KDE_KCUT + 1) * 8)
+#define KDE_SMEM_BYTES (KDE_SMEM_TABLE + KDE_WARPS * KDE_CH * 8)
+
+__global__ void __launch_bounds__(32 * KDE_WARPS)
 k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ keys, u64 xmask,
-      const u64* __restrict__ tile_range, const u32* __restrict__ tile_items, u32 ntiles,
-      u32 items, u64* D, unsigned long long* counter, unsigned long long* terms) {
-  __shared__ double sx[KDE_CH];
-  __shared__ u32 s_item;
-  u32 inwin = 0;
+      const u64* __restrict__ tile_range, const u32* __restrict__ tile_items,
+      const u32* __restrict__ item_tile, u32 items, u64* D, unsigned long long* counter,
+      unsigned long long* terms) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  double* sS = (double*)smem;                                   // [KDE_KCUT + 1]
+  double* sx = (double*)(smem + KDE_SMEM_TABLE) + (threadIdx.x >> 5) * KDE_CH;  // warp's slice
+  // T'[k] = ldexp(2^{-(k mod 64)/64}, 52 - k div 64), T'[KCUT] = 0
+  for (u32 k = threadIdx.x; k <= KDE_KCUT; k += blockDim.x) {
+    double T = KDE_EXP2_NEG[k & 63];
+    sS[k] = k == KDE_KCUT ? 0.0
+                          : __hiloint2double(__double2hiint(T) + (int)((52u - (k >> 6)) << 20),
+                                             __double2loint(T));
+  }
+  __syncthreads();
+  const u32 lane = lane_id();
+  u64 inwin = 0;
   for (;;) {
-    if (threadIdx.x == 0) s_item = (u32)atomicAdd(counter, 1ull);
-    __syncthreads();
-    u32 item = s_item;
+    u32 item = 0;
+    if (lane == 0) item = (u32)atomicAdd(counter, 1ull);
+    item = __shfl_sync(0xffffffffu, item, 0);
     if (item >= items) break;
-    // tile containing the item: last tile with tile_items[tile] <= item
-    u32 lo = 0, hi = ntiles - 1;
-    while (lo < hi) {
-      u32 m = (lo + hi + 1) >> 1;
-      if (tile_items[m] <= item) lo = m; else hi = m - 1;
-    }
-    u32 tile = lo;
+    u32 tile = item_tile[item];
     u32 s = tile / tps, t = tile % tps;
     const SegDev& g = segs[s];
     u64 va = tile_range[2 * (u64)tile] + (u64)(item - tile_items[tile]) * KDE_CH;
     u64 ve = tile_range[2 * (u64)tile + 1];
     u32 len = (u32)min((u64)KDE_CH, ve - va);
-    for (u32 i = threadIdx.x; i < len; i += KDE_TJ) sx[i] = __ull2double_rn(keys[va + i] & xmask);
-    __syncthreads();
-    u32 j = t * KDE_TJ + threadIdx.x;
+    for (u32 i = lane; i < len; i += 32) sx[i] = __ull2double_rn(keys[va + i] & xmask);
+    __syncwarp();
+    u32 j = t * KDE_TJ + lane;
     double inv_h = g.inv_h;
-    double w = __dmul_rn(KDE_W, g.h);
-    // this warp's window inside the chunk
-    u32 jw0 = t * KDE_TJ + (threadIdx.x & ~31u);
-    u32 jw1 = min(G - 1, jw0 + 31);
+    double gj = grid_pt(g.lo, g.hi, j < G ? j : G - 1, G);
     u64 acc = 0;
-    if (jw0 < G) {
-      double wa = __dsub_rn(grid_pt(g.lo, g.hi, jw0, G), w);
-      double wb = __dadd_rn(grid_pt(g.lo, g.hi, jw1, G), w);
-      u32 a = 0, b = len;
-      {  // first value >= wa
-        u32 l = 0, r = len;
-        while (l < r) { u32 m = (l + r) >> 1; if (sx[m] < wa) l = m + 1; else r = m; }
-        a = l;
-        l = a; r = len;
-        while (l < r) { u32 m = (l + r) >> 1; if (sx[m] <= wb) l = m + 1; else r = m; }
-        b = l;
+    u32 i = 0;
+    for (; i + 4 <= len; i += 4) {
+      u64 b0 = kde_qbits(gj, sx[i], inv_h, sS);
+      u64 b1 = kde_qbits(gj, sx[i + 1], inv_h, sS);
+      u64 b2 = kde_qbits(gj, sx[i + 2], inv_h, sS);
+      u64 b3 = kde_qbits(gj, sx[i + 3], inv_h, sS);
+      acc += (b0 + b1) + (b2 + b3);
+    }
+    for (; i < len; i++) acc += kde_qbits(gj, sx[i], inv_h, sS);
+    acc -= (u64)len * 0x4330000000000000ull;   // remove 2^52's bit pattern once per term
+    if (j < G) {
+      if (acc) {
+        unsigned long long* d = (unsigned long long*)(D + 2 * ((u64)s * G + j));
+        unsigned long long old = atomicAdd(d, (unsigned long long)acc);
+        if (old + acc < old) atomicAdd(d + 1, 1ull);
       }
-      double gj = grid_pt(g.lo, g.hi, j < G ? j : G - 1, G);
-      u32 inwin0 = inwin;
-#pragma unroll 2
-      for (u32 i = a; i < b; i++) acc += kde_term(gj, sx[i], inv_h, inwin);
-      if (j >= G) { acc = 0; inwin = inwin0; }
+      if (terms) {  // values with |g - x| <= sqrt(74) h in this chunk (diagnostic work count)
+        double wc = __dmul_rn(KDE_WC, g.h);
+        double lo = __dsub_rn(gj, wc), hi = __dadd_rn(gj, wc);
+        u32 l = 0, r = len;
+        while (l < r) { u32 m = (l + r) >> 1; if (sx[m] < lo) l = m + 1; else r = m; }
+        u32 a = l;
+        r = len;
+        while (l < r) { u32 m = (l + r) >> 1; if (sx[m] <= hi) l = m + 1; else r = m; }
+        inwin += l - a;
+      }
     }
-    if (acc) {
-      unsigned long long* d = (unsigned long long*)(D + 2 * ((u64)s * G + j));
-      unsigned long long old = atomicAdd(d, (unsigned long long)acc);
-      if (old + acc < old) atomicAdd(d + 1, 1ull);
-    }
-    __syncthreads();
+    __syncwarp();
   }
   if (terms) {
     for (int o = 16; o > 0; o >>= 1) inwin += __shfl_down_sync(0xffffffffu, inwin, o);
-    if (lane_id() == 0 && inwin) atomicAdd(terms, (unsigned long long)inwin);
+    if (lane == 0 && inwin) atomicAdd(terms, (unsigned long long)inwin);
   }
 }
 
+size_t kde_item_bytes(u32 items) { return (size_t)items * 4 + 16; }
+
 void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
-                const u64* tile_range, const u32* tile_items, u32 items, u64* D,
+                const u64* tile_range, const u32* tile_items, u32* item_tile, u32 items, u64* D,
                 unsigned long long* work_counter, unsigned long long* terms, cudaStream_t s) {
   if (items == 0) return;
   u32 tps = div_up(G, KDE_TJ);
   u32 ntiles = nseg * tps;
+  SV_LAUNCH(k_kde_items, div_up(ntiles, 256), 256, 0, s)(tile_items, ntiles, item_tile);
+  cudaFuncSetAttribute(k_kde, cudaFuncAttributeMaxDynamicSharedMemorySize, KDE_SMEM_BYTES);
   int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_kde, KDE_TJ, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_kde, 32 * KDE_WARPS, KDE_SMEM_BYTES);
   if (per_sm < 1) per_sm = 1;
   u32 grid = (u32)sv_num_sms() * (u32)per_sm;
-  if (grid > items) grid = items;
+  u32 need = div_up(items, KDE_WARPS);
+  if (grid > need) grid = need;
   cudaMemsetAsync(work_counter, 0, 8, s);
-  SV_LAUNCH(k_kde, grid, KDE_TJ, 0, s)(segs, G, tps, keys, xmask, tile_range, tile_items, ntiles, items, D,
-                                 work_counter, terms);
+  SV_LAUNCH(k_kde, grid, 32 * KDE_WARPS, KDE_SMEM_BYTES, s)(segs, G, tps, keys, xmask, tile_range,
+                                                            tile_items, item_tile, items, D,
+                                                            work_counter, terms);
 }

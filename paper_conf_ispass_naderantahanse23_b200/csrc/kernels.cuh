@@ -60,8 +60,8 @@ struct SegDev {
   double h, inv_h;
   u64 begin, end; // local index range in the sorted keys (filled on device)
 };
-#define KDE_TJ 128      // grid points per tile (one thread each)
-#define KDE_CH 1024     // values per work item chunk (staged in shared memory)
+#define KDE_TJ 32       // grid points per tile (one lane each; a work item is one warp's)
+#define KDE_CH 256      // values per work item chunk (staged in the warp's shared memory)
 struct KdeScratch {
   u64* tile_range;     // [nseg*tiles][2]
   u32* tile_items;     // [nseg*tiles + 1] exclusive scan of chunks per tile
@@ -72,9 +72,11 @@ void launch_seg_ranges(SegDev* segs, u32 nseg, const u64* keys, u64 nkeys, cudaS
 // returns total work items through *items_host (synchronises the stream once)
 int kde_plan(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 nkeys, u64 xmask,
              u64* tile_range, u32* tile_items, void* scan_temp, u32* items_host, cudaStream_t s);
+size_t kde_item_bytes(u32 items);
 void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
-                const u64* tile_range, const u32* tile_items, u32 items, u64* D /* [nseg][G][2] */,
-                unsigned long long* work_counter, unsigned long long* terms, cudaStream_t s);
+                const u64* tile_range, const u32* tile_items, u32* item_tile, u32 items,
+                u64* D /* [nseg][G][2] */, unsigned long long* work_counter,
+                unsigned long long* terms, cudaStream_t s);
 
 // ---------------- valleys and thresholds (A11-A13) ---------------------------------------------
 // T[s*tstride + q], nt[s], kind[s] (1 = valley, 2 = bisect)

@@ -3,35 +3,31 @@
 // (CoV = sigma / mu with the population sigma; A1, A5), plus the totals C_meas = sum y
 // and max x.
 //
-// B200 design: each block keeps a privatised per-kernel table in shared memory.  B200 has no
-// native 64-bit shared-memory add (it is a CAS loop, measured 5x slower than 32-bit ATOMS), so
-// the wide sums are kept as 32-bit words updated by native 32-bit atomics with explicit carry
-// propagation: atomicAdd returns the old word, the carry-out is added to the next word.  The
-// final words are the exact sum of all added values regardless of interleaving.  min / max use
-// a read-then-CAS that almost never takes the CAS after the first few invocations.  Blocks
-// write one 48-byte partial per kernel; a second kernel sums the partials exactly (u128) and
+// B200 design: each block (one per SM, 1024 threads) keeps a privatised per-kernel table in
+// shared memory.  sm_100a has no native 64-bit shared-memory add (it compiles to a CAS loop,
+// measured 5x slower than 32-bit ATOMS), and 32-bit atomics with carry propagation serialise
+// on their return values.  So x and x^2 are split into 15-bit limbs and each limb is added with
+// a fire-and-forget 32-bit atomic into its own counter: no carries can occur before 2^17 - 1
+// additions, so every 131071 rows the block flushes its limb counters (exactly, as u128) into
+// its private 48-byte partial record per kernel in global memory and clears them.  Zero limbs
+// are skipped (x < 2^30 needs 2 + 4 limb atomics plus the count).  min / max use a read-then-CAS
+// that almost never takes the CAS.  A second kernel sums the blocks' partials exactly (u128) and
 // emits 32-bit limbs in u64 lanes ready for a cross-rank all-reduce.
 #include "kernels.cuh"
 
-#define MOM_THREADS 512
-#define MOM_KT 2048  // kernels per shared-memory pass: 2048 * 44 B = 88 KB per block
+#define MOM_THREADS 1024
+#define MOM_U 4                               // rows per thread with loads in flight
+#define MOM_KT 2048                           // kernels per shared-memory pass (56 B each)
+#define MOM_LB 15                             // limb bits
+#define MOM_LMASK ((1u << MOM_LB) - 1u)
+#define MOM_FLUSH ((1u << (32 - MOM_LB)) - 1u)  // rows between flushes: limb sums stay < 2^32
+#define MOM_L1 3                              // limbs of x   (44 bits)
+#define MOM_L2 6                              // limbs of x^2 (88 bits)
+#define MOM_WORDS (1 + MOM_L1 + MOM_L2)       // count + limbs, u32 each
 
 int moments_kt(u32 K) { return (int)(K < MOM_KT ? K : MOM_KT); }
-int moments_grid() { return 2 * sv_num_sms(); }
-
-// add a value given as 32-bit words w[0..nw) into shared words a[0], a[stride], ...
-template <int NW>
-__device__ __forceinline__ void atomic_add_words(u32* a, u32 stride, const u32 (&w)[NW]) {
-  u32 carry = 0;
-#pragma unroll
-  for (int i = 0; i < NW; i++) {
-    u64 add = (u64)w[i] + carry;
-    if (add == 0) { carry = 0; continue; }
-    if (add == 0x100000000ull) { carry = 1; continue; }
-    u32 old = atomicAdd(&a[i * stride], (u32)add);
-    carry = ((u64)old + add) >> 32 ? 1u : 0u;
-  }
-}
+int moments_grid() { return sv_num_sms(); }
+static size_t moments_smem(u32 kt) { return (size_t)kt * (16 + 4 * MOM_WORDS); }
 
 __device__ __forceinline__ void atomic_min_u64_smem(u64* p, u64 v) {
   u64 cur = *(volatile u64*)p;
@@ -57,56 +53,103 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
   extern __shared__ __align__(16) unsigned char smem[];
   u64* s_mn = (u64*)smem;                 // [kt]
   u64* s_mx = s_mn + kt;                  // [kt]
-  u32* s_n = (u32*)(s_mx + kt);           // [kt]
-  u32* s_s1 = s_n + kt;                   // [3][kt] words of S1
-  u32* s_s2 = s_s1 + 3 * kt;              // [4][kt] words of S2
+  u32* s_w = (u32*)(s_mx + kt);           // [MOM_WORDS][kt]: count, x limbs, x^2 limbs
+  KMomPartial* rec = part + (u64)blockIdx.x * kt;
   for (u32 i = threadIdx.x; i < kt; i += blockDim.x) {
-    s_mn[i] = ~0ull; s_mx[i] = 0; s_n[i] = 0;
-    s_s1[i] = s_s1[kt + i] = s_s1[2 * kt + i] = 0;
-    s_s2[i] = s_s2[kt + i] = s_s2[2 * kt + i] = s_s2[3 * kt + i] = 0;
+    s_mn[i] = ~0ull;
+    s_mx[i] = 0;
+#pragma unroll
+    for (int w = 0; w < MOM_WORDS; w++) s_w[w * kt + i] = 0;
+    KMomPartial z = {0, 0, 0, 0, 0, 0, 0};
+    rec[i] = z;
   }
   __syncthreads();
   const bool totals = (k0 == 0);
+  const bool use_y = totals && y;
   u64 chunk = (n + gridDim.x - 1) / gridDim.x;
   u64 b = (u64)blockIdx.x * chunk;
   u64 e = b + chunk < n ? b + chunk : n;
   u64 ylo = 0, yhi = 0, xmax = 0, err = 0;
-  for (u64 i = b + threadIdx.x; i < e; i += blockDim.x) {
-    u32 k = __ldcs(kid + i);
-    u64 v = __ldcs(x + i);
+
+  auto process = [&](u32 k, u64 v, u64 w) {
     if (totals) {
       if (k >= K) err |= ERRF_KID;
       if (v == 0 || v >= SIEVE_X_LIMIT) err |= ERRF_RANGE;
       xmax = v > xmax ? v : xmax;
-      if (y) { u64 w = __ldcs(y + i); u64 s = ylo + w; yhi += s < ylo; ylo = s; }
+      u64 s = ylo + w; yhi += s < ylo; ylo = s;
     }
     u32 l = k - k0;
-    if (l >= kt || v == 0 || v >= SIEVE_X_LIMIT) continue;
-    atomicAdd(&s_n[l], 1u);
-    u32 w1[3] = {(u32)v, (u32)(v >> 32), 0u};
-    atomic_add_words<3>(s_s1 + l, kt, w1);
+    if (l >= kt || v == 0 || v >= SIEVE_X_LIMIT) return;
+    atomicAdd(&s_w[l], 1u);
+#pragma unroll
+    for (int i = 0; i < MOM_L1; i++) {
+      u32 limb = (u32)(v >> (MOM_LB * i)) & MOM_LMASK;
+      if (limb) atomicAdd(&s_w[(1 + i) * kt + l], limb);
+    }
     u64 sqlo = v * v, sqhi = __umul64hi(v, v);
-    u32 w2[4] = {(u32)sqlo, (u32)(sqlo >> 32), (u32)sqhi, (u32)(sqhi >> 32)};
-    atomic_add_words<4>(s_s2 + l, kt, w2);
+#pragma unroll
+    for (int i = 0; i < MOM_L2; i++) {
+      int sh = MOM_LB * i;
+      u64 bits = sh < 64 ? ((sqlo >> sh) | (sh ? (sqhi << (64 - sh)) : 0ull)) : (sqhi >> (sh - 64));
+      u32 limb = (u32)bits & MOM_LMASK;
+      if (limb) atomicAdd(&s_w[(1 + MOM_L1 + i) * kt + l], limb);
+    }
     atomic_min_u64_smem(&s_mn[l], v);
     atomic_max_u64_smem(&s_mx[l], v);
+  };
+
+  auto flush = [&]() {
+    __syncthreads();
+    for (u32 i = threadIdx.x; i < kt; i += blockDim.x) {
+      u32 c = s_w[i];
+      if (!c) continue;
+      u128 s1 = 0, s2 = 0;
+#pragma unroll
+      for (int j = 0; j < MOM_L1; j++) {
+        s1 += (u128)s_w[(1 + j) * kt + i] << (MOM_LB * j);
+        s_w[(1 + j) * kt + i] = 0;
+      }
+#pragma unroll
+      for (int j = 0; j < MOM_L2; j++) {
+        s2 += (u128)s_w[(1 + MOM_L1 + j) * kt + i] << (MOM_LB * j);
+        s_w[(1 + MOM_L1 + j) * kt + i] = 0;
+      }
+      s_w[i] = 0;
+      KMomPartial r = rec[i];
+      u128 a1 = (((u128)r.s1hi << 64) | r.s1lo) + s1;
+      u128 a2 = (((u128)r.s2hi << 64) | r.s2lo) + s2;
+      r.n += c;
+      r.s1lo = (u64)a1; r.s1hi = (u32)(a1 >> 64);
+      r.s2lo = (u64)a2; r.s2hi = (u64)(a2 >> 64);
+      rec[i] = r;
+    }
+    __syncthreads();
+  };
+
+  const u64 step = blockDim.x;
+  for (u64 c0 = b; c0 < e; c0 += MOM_FLUSH) {
+    u64 c1 = c0 + MOM_FLUSH < e ? c0 + MOM_FLUSH : e;
+    u64 i = c0 + threadIdx.x;
+    for (; i + (MOM_U - 1) * step < c1; i += MOM_U * step) {
+      u32 kk[MOM_U];
+      u64 vv[MOM_U], ww[MOM_U];
+#pragma unroll
+      for (int u = 0; u < MOM_U; u++) {
+        kk[u] = __ldcs(kid + i + u * step);
+        vv[u] = __ldcs(x + i + u * step);
+        ww[u] = use_y ? __ldcs(y + i + u * step) : 0ull;
+      }
+#pragma unroll
+      for (int u = 0; u < MOM_U; u++) process(kk[u], vv[u], ww[u]);
+    }
+    for (; i < c1; i += step) process(__ldcs(kid + i), __ldcs(x + i), use_y ? __ldcs(y + i) : 0ull);
+    flush();
   }
-  __syncthreads();
-  KMomPartial* out = part + (u64)blockIdx.x * kt;
   for (u32 i = threadIdx.x; i < kt; i += blockDim.x) {
-    KMomPartial r;
-    r.n = s_n[i];
-    r.s1lo = (u64)s_s1[i] | ((u64)s_s1[kt + i] << 32);
-    r.s1hi = s_s1[2 * kt + i];
-    r.s2lo = (u64)s_s2[i] | ((u64)s_s2[kt + i] << 32);
-    r.s2hi = (u64)s_s2[2 * kt + i] | ((u64)s_s2[3 * kt + i] << 32);
-    r.mn = s_mn[i];
-    r.mx = s_mx[i];
-    out[i] = r;
+    rec[i].mn = s_mn[i];
+    rec[i].mx = s_mx[i];
   }
   if (totals) {
-    // block reduction of (ylo, yhi), xmax, err through shared memory (reuse s_mn area after sync)
-    __syncthreads();
     __shared__ u64 r_lo[MOM_THREADS / 32], r_hi[MOM_THREADS / 32], r_mx[MOM_THREADS / 32];
     for (int o = 16; o > 0; o >>= 1) {
       u64 olo = __shfl_down_sync(0xffffffffu, ylo, o);
@@ -140,10 +183,8 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
 
 void launch_moments(const u32* kid, const u64* x, const u64* y, u64 n, u32 K, u32 k0, u32 kt,
                     KMomPartial* part, u64* blk_tot, u64* errflags, int grid, cudaStream_t s) {
-  size_t smem = (size_t)kt * (8 + 8 + 4 + 12 + 16);
-  cudaFuncSetAttribute(k_moments, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                       MOM_KT * (8 + 8 + 4 + 12 + 16));
-  SV_LAUNCH(k_moments, grid, MOM_THREADS, smem, s)(kid, x, y, n, K, k0, kt, part, blk_tot, errflags);
+  cudaFuncSetAttribute(k_moments, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)moments_smem(MOM_KT));
+  SV_LAUNCH(k_moments, grid, MOM_THREADS, moments_smem(kt), s)(kid, x, y, n, K, k0, kt, part, blk_tot, errflags);
 }
 
 // one thread per kernel: exact u128 sum over the blocks' partials, emitted as limb lanes

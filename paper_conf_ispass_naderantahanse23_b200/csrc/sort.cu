@@ -185,10 +185,15 @@ k_rs_hist(const u64* __restrict__ keys, u64 n, int shift, u32 ntiles, u32* __res
   __syncthreads();
   u32 w = threadIdx.x >> 5;
   u64 base = (u64)blockIdx.x * RS_TILE + (u64)w * (RS_TILE / RS_WARPS);
-#pragma unroll 4
+  u32 dig[RS_IPT];  // all loads of the tile in flight before any ranking
+#pragma unroll
   for (int r = 0; r < RS_IPT; r++) {
     u64 i = base + (u64)r * 32 + lane_id();
-    u32 d = i < n ? (u32)(keys[i] >> shift) & 255u : 256u;
+    dig[r] = i < n ? (u32)(__ldcs(keys + i) >> shift) & 255u : 256u;
+  }
+#pragma unroll
+  for (int r = 0; r < RS_IPT; r++) {
+    u32 d = dig[r];
     u32 peers = __match_any_sync(0xffffffffu, d);
     if (d < 256u && lane_id() == (u32)(__ffs(peers) - 1)) s_h[w][d] += __popc(peers);
     __syncwarp();
@@ -219,11 +224,16 @@ k_rs_scatter(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, in
   u32 val[RS_IPT];
   u32 rank[RS_IPT];
 #pragma unroll
+  for (int r = 0; r < RS_IPT; r++) {  // all loads of the tile in flight before any ranking
+    u64 i = base + (u64)r * 32 + lane_id();
+    bool ok = i < n;
+    key[r] = ok ? __ldcs(kin + i) : 0;
+    val[r] = (ok && vin) ? __ldcs(vin + i) : 0;
+  }
+#pragma unroll
   for (int r = 0; r < RS_IPT; r++) {
     u64 i = base + (u64)r * 32 + lane_id();
     bool ok = i < n;
-    key[r] = ok ? kin[i] : 0;
-    val[r] = (ok && vin) ? vin[i] : 0;
     u32 d = ok ? (u32)(key[r] >> shift) & 255u : 256u;
     u32 peers = __match_any_sync(0xffffffffu, d);
     u32 lt = peers & ((1u << lane_id()) - 1u);
