@@ -30,7 +30,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-KDE_FP64_OPS_PER_TERM = 14   # FP64-pipe instructions per in-window KDE term
+KDE_FP64_OPS_PER_TERM = 13   # FP64-pipe instructions per in-window KDE term
 FP64_LANES_PER_SM = 64       # B200: 64 FP64 FMA lanes / SM / clk (microbenchmark: 62.9)
 
 
@@ -198,15 +198,19 @@ def main():
                              first_id=first, adopt=True)
 
     debug = os.environ.get("BENCH_DEBUG")
+    host_ms = {"stratify": [], "predict": []}
 
     def step():
         t0 = time.perf_counter()
         st = sieve.stratify(trace, stratum_of_invocation=sid)
         t1 = time.perf_counter()
         sieve.predict(st, trace)
+        t2 = time.perf_counter()
+        host_ms["stratify"].append(1e3 * (t1 - t0))
+        host_ms["predict"].append(1e3 * (t2 - t1))
         if debug:
-            print(f"[bench host] stratify {1e3 * (t1 - t0):.3f} ms predict "
-                  f"{1e3 * (time.perf_counter() - t1):.3f} ms", file=sys.stderr)
+            print(f"[bench host] stratify {1e3 * (t1 - t0):.3f} ms predict {1e3 * (t2 - t1):.3f} ms",
+                  file=sys.stderr)
         return st
 
     def barrier():
@@ -231,6 +235,8 @@ def main():
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ctx.set_timing(True)
     launches0 = sieve.kernel_launches()
+    host_ms["stratify"].clear()
+    host_ms["predict"].clear()
     barrier()
     torch.cuda.synchronize()
     clk.mark("t0")
@@ -325,7 +331,9 @@ def main():
                        "parallelism": f"dp{world} (contiguous invocation slices)",
                        "l2": "inputs larger than L2 (24 B/invocation = 2.4 GB per step)"},
             "clocks": clocks, "e2e": e2e, "gpu_launches": launches,
-            "roofline": roof, "phases": phase_out, "cpu_baseline": cpu}
+            "roofline": roof, "phases": phase_out,
+            "host_ms_per_step": {k: statistics.mean(v) for k, v in host_ms.items() if v},
+            "cpu_baseline": cpu}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

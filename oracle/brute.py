@@ -35,7 +35,8 @@ EXP2_NEG = _exp2_neg_table()
 
 
 def _reduce(t):
-    k = float(round(t * LOG2E_64))       # Python round() on floats is round-half-even == rint
+    # nearest integer to the EXACT product t * 64 log2 e (single rounding, ties to even)
+    k = float(round(Fraction(t) * Fraction(LOG2E_64)))
     r = fma(-k, LN2_64_HI, t)
     r = fma(-k, LN2_64_LO, r)
     p = -float(Fraction(1, 120))          # P(r) = sum_{i<=5} (-r)^i / i!  (Horner, signed coefs)

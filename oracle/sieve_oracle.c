@@ -189,7 +189,7 @@ double oracle_grid_point(uint64_t lo, uint64_t hi, uint32_t j, uint32_t G) {
 
 /* ------------------------------------------------------------------------------------------
  * O5c fixed-point Gaussian kernel value (A10), built only from IEEE basic operations:
- *   k = rint(t * 64 log2 e),  j = k mod 64,  m = k div 64       (so t ~ k ln2 / 64)
+ *   k = nearest integer to t * 64 log2 e (one rounding, fma), j = k mod 64, m = k div 64
  *   r = fma(-k, ln2/64 hi, t);  r = fma(-k, ln2/64 lo, r)        (|r| <= ln2 / 128)
  *   P(r) = 1 - r + r^2/2 - r^3/6 + r^4/24 - r^5/120               (Horner with fma)
  *   e^{-t} = 2^{-j/64} * 2^{-m} * e^{-r}
@@ -220,9 +220,11 @@ static const double OR_EXP2_NEG[64] = {
     0x1.172b83c7d517bp-1, 0x1.1429aaea92de0p-1, 0x1.11301d0125b51p-1, 0x1.0e3ec32d3d1a2p-1,
     0x1.0b5586cf9890fp-1, 0x1.0874518759bc8p-1, 0x1.059b0d3158574p-1, 0x1.02c9a3e778061p-1};
 
-/* the reduced argument and polynomial shared by det_exp and Q */
+/* the reduced argument and polynomial shared by det_exp and Q.  k is the integer nearest to
+ * t * 64 log2 e with a SINGLE rounding: fma(t, C, 1.5 * 2^52) lands in [2^52, 2^53) where the
+ * ulp is 1, and subtracting 1.5 * 2^52 back is exact. */
 static double exp_reduce(double t, int* j, int* m) {
-  double k = rint(t * OR_LOG2E_64);
+  double k = fma(t, OR_LOG2E_64, 6755399441055744.0) - 6755399441055744.0;
   int ki = (int)k;
   *j = ki & 63;
   *m = ki >> 6;

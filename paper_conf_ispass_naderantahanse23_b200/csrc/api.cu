@@ -81,6 +81,14 @@ struct sieve_ctx_s {
   PhaseAcc acc[SIEVE_PHASE_COUNT];
   std::vector<PendingEv> pending;
   std::vector<cudaEvent_t> ev_pool;
+  // per-call scratch arena: every temporary of a stratify / predict call is bump-allocated
+  // from one device buffer that is reset at the start of the next call (all work of a call is
+  // ordered on the ctx stream and synchronised before it returns).  A call that overflows
+  // gets the overflow from the allocator and the arena grows to the high-water mark, so
+  // steady-state calls never touch the allocator (no pool remapping, no fragmentation).
+  char* arena = nullptr;
+  size_t arena_cap = 0, arena_off = 0, arena_hw = 0;
+  std::vector<void*> overflow;
 };
 
 static std::atomic<unsigned long long> g_launches{0};
@@ -193,6 +201,37 @@ static void dfree(sieve_ctx c, void* p) {
   else cudaFreeAsync(p, c->stream);
 }
 
+static int arena_reset(sieve_ctx c) {
+  for (void* p : c->overflow) dfree(c, p);
+  c->overflow.clear();
+  if (c->arena_hw > c->arena_cap) {
+    if (c->arena) dfree(c, c->arena);
+    c->arena = nullptr;
+    c->arena_cap = 0;
+    size_t want = c->arena_hw + c->arena_hw / 8;
+    void* p;
+    SV_TRY(dalloc(c, &p, want));
+    c->arena = (char*)p;
+    c->arena_cap = want;
+  }
+  c->arena_off = 0;
+  c->arena_hw = 0;
+  return SIEVE_OK;
+}
+
+static int arena_alloc(sieve_ctx c, void** p, size_t bytes) {
+  bytes = (bytes + 255) / 256 * 256;
+  if (bytes == 0) bytes = 256;
+  size_t off = c->arena_off;
+  c->arena_off += bytes;
+  if (c->arena_off > c->arena_hw) c->arena_hw = c->arena_off;
+  if (c->arena_off <= c->arena_cap) { *p = c->arena + off; return SIEVE_OK; }
+  SV_TRY(dalloc(c, p, bytes));  // overflow this call; the arena grows at the next reset
+  c->overflow.push_back(*p);
+  return SIEVE_OK;
+}
+
+// a temporary device array of one call (freed wholesale at the next call's arena reset)
 template <typename T>
 struct DBuf {
   sieve_ctx c = nullptr;
@@ -202,13 +241,11 @@ struct DBuf {
   explicit DBuf(sieve_ctx cc) : c(cc) {}
   DBuf(const DBuf&) = delete;
   DBuf& operator=(const DBuf&) = delete;
-  ~DBuf() { release(); }
-  void release() { if (p) dfree(c, p); p = nullptr; n = 0; }
+  void release() { p = nullptr; n = 0; }
   int alloc(size_t count) {
-    release();
     n = count;
     void* q;
-    int st = dalloc(c, &q, count * sizeof(T));
+    int st = arena_alloc(c, &q, count * sizeof(T));
     p = (T*)q;
     return st;
   }
@@ -281,6 +318,9 @@ extern "C" void sieve_ctx_destroy(sieve_ctx ctx) {
   cudaSetDevice(ctx->device);
   for (auto& p : ctx->pending) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
+  for (void* p : ctx->overflow) dfree(ctx, p);
+  if (ctx->arena) dfree(ctx, ctx->arena);
+  cudaStreamSynchronize(ctx->stream);
   delete ctx->comm;
   ctx->magic = 0;
   delete ctx;
@@ -474,6 +514,7 @@ struct Fin { u32 kid, tier; u64 lo, hi, n; u128 s1; double h; u32 round; };
 static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out, sieve_strata_s* R) {
   sieve_ctx c = t->ctx;
   cudaStream_t S = c->stream;
+  SV_TRY(arena_reset(c));
   HostClock hc;
   const u32 K = t->K, G = P->grid_points;
   const u64 n = t->n;
@@ -575,7 +616,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   const u32 bx = std::max<u32>(1, bitlen(max_x));
   const u64 xmask = (bx >= 64) ? ~0ull : ((1ull << bx) - 1);
   const int nbits = (int)(bx + bitlen(n_t3 ? n_t3 - 1 : 0));
-  DBuf<u64> keys(c), P1(c), P2(c);
+  DBuf<u64> keys(c), Pb(c);
   DBuf<u32> d_t3rank(c);
   DBuf<unsigned long long> counter(c);
   SV_TRY(counter.alloc(4));
@@ -596,13 +637,10 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       SV_TRY(radix_sort(keys.get(), nullptr, n3_local, nbits, tmp.get(), S, &passes));
       if (c->timing) c->acc[SIEVE_PHASE_SORT].work += (u64)passes * n3_local * 16;
     }
-    SV_TRY(P1.alloc(2 * (n3_local + 1)));
-    SV_TRY(P2.alloc(2 * (n3_local + 1)));
+    SV_TRY(Pb.alloc(4 * block_prefix_entries(n3_local)));
     {
-      DBuf<char> tmp(c);
-      SV_TRY(tmp.alloc(prefix128_temp_bytes(n3_local)));
-      PhaseTimer tm(c, SIEVE_PHASE_PREFIX, n3_local * 8 + (n3_local + 1) * 32);
-      launch_prefix128(keys.get(), n3_local, xmask, P1.get(), P2.get(), tmp.get(), S);
+      PhaseTimer tm(c, SIEVE_PHASE_PREFIX, n3_local * 8);
+      launch_block_prefix(keys.get(), n3_local, xmask, Pb.get(), S);
     }
     SV_CUDA(cudaGetLastError());
   }
@@ -691,7 +729,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(pab.alloc((size_t)nparts * 2));
     PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
     launch_part_stats(segs.get(), nseg, T.get(), tstride, ntk.get(), d_off.get(), nparts,
-                      nkeys ? keys.get() : nullptr, nkeys, bx, P1.get(), P2.get(), pl.get(),
+                      nkeys ? keys.get() : nullptr, nkeys, bx, Pb.get(), pl.get(),
                       pm.get(), pab.get(), S);
     tp.stop();
     SV_CUDA(cudaGetLastError());
@@ -751,7 +789,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     R->kde_terms = ht[0];
     if (c->timing) c->acc[SIEVE_PHASE_KDE].work += ht[0];
   }
-  P1.release(); P2.release(); keys.release();
+  Pb.release(); keys.release();
 
   // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
   std::sort(fin.begin(), fin.end(), [](const Fin& a, const Fin& b) {
@@ -989,6 +1027,7 @@ extern "C" int sieve_predict(sieve_strata s, sieve_trace t, const uint64_t* rep_
   sieve_ctx c = t->ctx;
   SV_CUDA(cudaSetDevice(c->device));
   const u32 ns = (u32)s->st.size();
+  SV_TRY(arena_reset(c));
   std::vector<u64> hW(2 * (size_t)ns), hx(ns), hy(ns);
   for (u32 i = 0; i < ns; i++) {
     hW[2 * i] = s->st[i].instr_sum_lo;

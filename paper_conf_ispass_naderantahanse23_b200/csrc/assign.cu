@@ -16,11 +16,11 @@
 #include "kernels.cuh"
 
 #define AS_THREADS 512
-#define AS_IPT 4
+#define AS_IPT 8
 #define AS_HC 4096          // shared hash capacity (entries)
 #define AS_MAXP 32          // probes before falling back to the global table
 
-int assign_grid() { return 2 * sv_num_sms(); }
+int assign_grid() { return 3 * sv_num_sms(); }
 
 __device__ __forceinline__ u32 hash_key(u64 k) {
   return (u32)((k * 0x9E3779B97F4A7C15ull) >> 32);
@@ -72,13 +72,15 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
       vv[j] = ok ? __ldcs(x + i) : 0ull;
       cc[j] = (ok && cta) ? __ldcs(cta + i) : 0u;
     }
+    KTab kts[AS_IPT];  // per-kernel table rows (L1-resident), all requested before use
+#pragma unroll
+    for (int j = 0; j < AS_IPT; j++) kts[j] = ktab[kk[j]];
 #pragma unroll
     for (int j = 0; j < AS_IPT; j++) {
       u64 i = base + (u64)j * AS_THREADS + threadIdx.x;
       if (i >= b1) continue;
-      u32 k = kk[j];
       u64 v = vv[j];
-      KTab kt = ktab[k];
+      KTab kt = kts[j];
       u32 sid = kt.base;
       if (kt.m > 1) {  // number of lower bounds lows[1..m) that are <= v
         const u64* L = lows + kt.lows_off;
@@ -103,7 +105,7 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
         }
         if (cur == key) {
           atomicAdd(&hc[h], 1u);
-          atomicMin(&hf[h], rel);
+          if (*(volatile u32*)&hf[h] > rel) atomicMin(&hf[h], rel);  // rarely lowers it
           done = true;
           break;
         }

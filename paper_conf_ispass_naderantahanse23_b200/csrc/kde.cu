@@ -17,12 +17,13 @@
 // the tile's window |g - x| <= 8.7 h); items are pulled by WARPS from an atomic counter (no
 // block barriers: warps of a block never wait for each other); each lane owns one grid point,
 // the chunk is staged in the warp's slice of shared memory and read as broadcasts.  The term is
-// arranged to be bit-identical to the oracle's while issuing 15 FP64-pipe instructions and ~4
+// arranged to be bit-identical to the oracle's while issuing 13 FP64-pipe instructions and ~6
 // others:
-//   * u = z*z replaces t = u/2 (exact scaling): k = rint(u * 32 log2 e), r' = u - k ln2/32 = 2r,
+//   * u = z*z replaces t = u/2 (exact scaling): k = nearest integer to u * 32 log2 e (= t * 64
+//     log2 e, one rounding, via fma(u, 32 log2 e, 1.5 * 2^52)), r' = u - k ln2/32 = 2r,
 //     Horner on r' with coefficients c_i 2^-i gives exactly the same P (power-of-two scaling
 //     commutes with round-to-nearest);
-//   * k = low word of u*32log2e + 1.5*2^52 (an exact rint), clamped to 3417;
+//   * k = low word of that fma result, clamped to 3417;
 //   * S = T'[k] = 2^{-(k mod 64)/64} * 2^(52 - k div 64) from a shared-memory table (exact
 //     power-of-two scalings of the correctly rounded 2^{-j/64}), with T'[3417] = 0: every
 //     t > 37 lands on k >= 3417 or has Q = 0 anyway (e^-37 2^52 = 0.38), so no select;
@@ -102,11 +103,17 @@ int kde_plan(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 nkeys, u6
   return SIEVE_OK;
 }
 
-// item -> tile map (so a warp finds its tile with one load)
-__global__ void k_kde_items(const u32* tile_items, u32 ntiles, u32* item_tile) {
-  u32 tile = blockIdx.x * blockDim.x + threadIdx.x;
-  if (tile >= ntiles) return;
-  for (u32 it = tile_items[tile]; it < tile_items[tile + 1]; it++) item_tile[it] = tile;
+// item -> tile map (so a warp finds its tile with one load): one thread per item, binary
+// search of the last tile whose first item is <= it
+__global__ void k_kde_items(const u32* tile_items, u32 ntiles, u32 items, u32* item_tile) {
+  for (u32 it = blockIdx.x * blockDim.x + threadIdx.x; it < items; it += gridDim.x * blockDim.x) {
+    u32 lo = 0, hi = ntiles - 1;
+    while (lo < hi) {
+      u32 m = (lo + hi + 1) >> 1;
+      if (tile_items[m] <= it) lo = m; else hi = m - 1;
+    }
+    item_tile[it] = lo;
+  }
 }
 
 // ------------------------------------------------------------------------------------------
@@ -145,7 +152,7 @@ __constant__ double KDE_EXP2_NEG[64] = {
 __device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, const double* sS) {
   double z = __dmul_rn(__dsub_rn(g, xd), inv_h);
   double u = __dmul_rn(z, z);                               // 2t, exactly
-  double kb = __dadd_rn(__dmul_rn(u, C_LOG2E_32), C_MAGIC);
+  double kb = __fma_rn(u, C_LOG2E_32, C_MAGIC);             // one rounding: nearest integer
   double kf = __dsub_rn(kb, C_MAGIC);
   // k = rint(u * 32 log2 e) while u < 80 (the magic-number rint is exact there); any u >= 80
   // (t >= 40, far outside the window) maps to the zero entry.  p stays finite for every input
@@ -243,7 +250,7 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
   if (items == 0) return;
   u32 tps = div_up(G, KDE_TJ);
   u32 ntiles = nseg * tps;
-  SV_LAUNCH(k_kde_items, div_up(ntiles, 256), 256, 0, s)(tile_items, ntiles, item_tile);
+  SV_LAUNCH(k_kde_items, min(div_up(items, 256), 4096u), 256, 0, s)(tile_items, ntiles, items, item_tile);
   cudaFuncSetAttribute(k_kde, cudaFuncAttributeMaxDynamicSharedMemorySize, KDE_SMEM_BYTES);
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_kde, 32 * KDE_WARPS, KDE_SMEM_BYTES);

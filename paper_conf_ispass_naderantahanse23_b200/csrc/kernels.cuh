@@ -47,10 +47,12 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
                int* passes = nullptr);
 
 // ---------------- prefix sums of x and x^2 over sorted Tier-3 keys -----------------------------
-// P1[i] = sum_{j<i} x_j, P2[i] = sum_{j<i} x_j^2, as u128 pairs (lo, hi), i in [0, n]
-size_t prefix128_temp_bytes(u64 n);
-void launch_prefix128(const u64* keys, u64 n, u64 xmask, u64* P1, u64* P2, void* temp,
-                      cudaStream_t s);
+// block-boundary prefix sums of x and x^2 over the sorted Tier-3 keys
+#define PREFIX_BLOCK 4096
+u64 block_prefix_entries(u64 n);
+// Pb: [(n / PREFIX_BLOCK + 1) + 1][4] u64 = (S1 lo, S1 hi, S2 lo, S2 hi) exclusive prefixes at
+// block boundaries; the last entry is the total
+void launch_block_prefix(const u64* keys, u64 n, u64 xmask, u64* Pb, cudaStream_t s);
 
 // ---------------- KDE over open segments ([8], [36]; A6-A10) -----------------------------
 struct SegDev {
@@ -88,7 +90,7 @@ void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D
 // out: lanes[p*9..] (n, S1 limbs, S2 limbs), mm[p*2..] (min, max), ab[p*2..] value interval
 void launch_part_stats(const SegDev* segs, u32 nseg, const u64* T, u32 tstride, const u32* nt,
                        const u32* part_off, u32 nparts, const u64* keys, u64 nkeys, u32 bx,
-                       const u64* P1, const u64* P2, u64* lanes, u64* mm, u64* ab, cudaStream_t s);
+                       const u64* Pb, u64* lanes, u64* mm, u64* ab, cudaStream_t s);
 
 // ---------------- pass B: assignment + per-(stratum, CTA) statistics -------------------
 struct KTab {      // per kernel

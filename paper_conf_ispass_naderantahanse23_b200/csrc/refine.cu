@@ -34,7 +34,7 @@ k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, 
     u128 v = ((u128)hi << 64) | lo;
     mx = v > mx ? v : mx;
   }
-  if (lane_id() != 0) return;
+  mx = ((u128)__shfl_sync(0xffffffffu, (u64)(mx >> 64), 0) << 64) | __shfl_sync(0xffffffffu, (u64)mx, 0);
   SegDev g = segs[s];
   u128 delta = mx >> shift;
   if (delta < 1) delta = 1;
@@ -43,8 +43,17 @@ k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, 
   bool seek_min = false;
   u128 top = ((u128)d[1] << 64) | d[0], low = 0;
   u32 a = 0, b = 0;
-  for (u32 j = 1; j < G; j++) {
-    u128 v = ((u128)d[2 * j + 1] << 64) | d[2 * j];
+  u64 last_th = 0;
+  // every lane runs the (sequential) state machine on the same values: each 32-value chunk is
+  // one coalesced load, then broadcast value by value with shuffles (uniform control flow)
+  for (u32 j0 = 0; j0 < G; j0 += 32) {
+    u32 jl = j0 + lane_id();
+    u64 clo = jl < G ? d[2 * jl] : 0, chi = jl < G ? d[2 * jl + 1] : 0;
+    u32 cn = min(32u, G - j0);
+    for (u32 q = 0; q < cn; q++) {
+    u32 j = j0 + q;
+    u128 v = ((u128)__shfl_sync(0xffffffffu, chi, q) << 64) | __shfl_sync(0xffffffffu, clo, q);
+    if (j == 0) continue;
     if (!seek_min) {
       if (v > top) top = v;
       if (v + delta <= top) { seek_min = true; low = v; a = b = j; }
@@ -55,12 +64,18 @@ k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, 
         u32 m = (a + b) >> 1;
         double gm = grid_pt_r(g.lo, g.hi, m, G);
         u64 th = (u64)ceil(gm);
-        if (th > g.lo && th <= g.hi && (n == 0 || Ts[n - 1] != th)) Ts[n++] = th;
+        if (th > g.lo && th <= g.hi && (n == 0 || last_th != th)) {
+          if (lane_id() == 0) Ts[n] = th;
+          last_th = th;
+          n++;
+        }
         seek_min = false;
         top = v;
       }
     }
+    }
   }
+  if (lane_id() != 0) return;
   u32 k = 1;
   if (n == 0) { Ts[0] = (g.lo + g.hi + 1) >> 1; n = 1; k = 2; }  // value-range bisection (A13)
   nt[s] = n;
@@ -81,49 +96,104 @@ __device__ __forceinline__ u64 lb_u64(const u64* a, u64 b, u64 e, u64 v) {
   return b;
 }
 
-__global__ void k_part_stats(const SegDev* segs, u32 nseg, const u64* T, u32 tstride,
-                             const u32* nt, const u32* part_off, u32 nparts, const u64* keys,
-                             u64 nkeys, u32 bx, const u64* P1, const u64* P2, u64* lanes, u64* mm,
-                             u64* ab) {
-  u32 p = blockIdx.x * blockDim.x + threadIdx.x;
-  if (p >= nparts) return;
-  u32 lo = 0, hi = nseg - 1;  // last segment with part_off[s] <= p
-  while (lo < hi) {
-    u32 m = (lo + hi + 1) >> 1;
-    if (part_off[m] <= p) lo = m; else hi = m - 1;
+// One block per candidate part [a, b) of segment s (A13 f): its local index range [ia, ib) by
+// two binary searches, then n = ib - ia and
+//   S(ia, ib) = Pb[ib / B] - Pb[ia / B] + sum(keys[ib/B*B .. ib)) - sum(keys[ia/B*B .. ia))
+// from the block-boundary prefixes Pb and at most two partial blocks (B = PREFIX_BLOCK), in
+// exact modular u128 arithmetic.  Output: limb lanes (n, S1, S2), min / max, the interval.
+#define PS_THREADS 256
+__device__ __forceinline__ void ps_add(u64& s1, u64& s2lo, u64& s2hi, u64 x, bool neg) {
+  u64 qlo = x * x, qhi = __umul64hi(x, x);
+  if (neg) {  // two's complement of (x, x^2) in u64 / u128
+    s1 -= x;
+    u64 d = s2lo - qlo;
+    s2hi -= qhi + (s2lo < qlo ? 1ull : 0ull);
+    s2lo = d;
+  } else {
+    s1 += x;
+    u64 t = s2lo + qlo;
+    s2hi += qhi + (t < s2lo ? 1ull : 0ull);
+    s2lo = t;
   }
-  u32 s = lo, q = p - part_off[s];
-  SegDev g = segs[s];
-  const u64* Ts = T + (u64)s * tstride;
-  u64 a = q == 0 ? g.lo : Ts[q - 1];
-  u64 b = q == nt[s] ? g.hi + 1 : Ts[q];
-  u64 base = g.key_lo - g.lo;
-  u64 ia = 0, ib = 0;
-  if (nkeys) {
-    ia = lb_u64(keys, g.begin, g.end, base + a);
-    ib = lb_u64(keys, ia, g.end, base + b);
+}
+
+__global__ void __launch_bounds__(PS_THREADS)
+k_part_stats(const SegDev* segs, u32 nseg, const u64* T, u32 tstride, const u32* nt,
+             const u32* part_off, u32 nparts, const u64* keys, u64 nkeys, u32 bx, const u64* Pb,
+             u64* lanes, u64* mm, u64* ab) {
+  u32 p = blockIdx.x;
+  __shared__ u64 sh[4];
+  if (threadIdx.x == 0) {
+    u32 lo = 0, hi = nseg - 1;  // last segment with part_off[s] <= p
+    while (lo < hi) {
+      u32 m = (lo + hi + 1) >> 1;
+      if (part_off[m] <= p) lo = m; else hi = m - 1;
+    }
+    u32 s = lo, q = p - part_off[s];
+    SegDev g = segs[s];
+    const u64* Ts = T + (u64)s * tstride;
+    u64 a = q == 0 ? g.lo : Ts[q - 1];
+    u64 b = q == nt[s] ? g.hi + 1 : Ts[q];
+    u64 base = g.key_lo - g.lo;
+    u64 ia = 0, ib = 0;
+    if (nkeys) {
+      ia = lb_u64(keys, g.begin, g.end, base + a);
+      ib = lb_u64(keys, ia, g.end, base + b);
+    }
+    sh[0] = ia; sh[1] = ib;
+    ab[2 * (u64)p] = a;
+    ab[2 * (u64)p + 1] = b;
+  }
+  __syncthreads();
+  const u64 ia = sh[0], ib = sh[1];
+  const u64 xmask = (bx >= 64) ? ~0ull : ((1ull << bx) - 1);
+  // this thread's share of the two partial blocks (x^2 < 2^88, so S2 needs a u128)
+  u64 s1 = 0, s2lo = 0, s2hi = 0;
+  if (ib > ia) {
+    for (u64 j = (ib / PREFIX_BLOCK) * PREFIX_BLOCK + threadIdx.x; j < ib; j += PS_THREADS)
+      ps_add(s1, s2lo, s2hi, keys[j] & xmask, false);
+    for (u64 j = (ia / PREFIX_BLOCK) * PREFIX_BLOCK + threadIdx.x; j < ia; j += PS_THREADS)
+      ps_add(s1, s2lo, s2hi, keys[j] & xmask, true);
+  }
+  // block reduction (modular; S1 partial fits u64 once combined with the prefix as u128 below)
+  __shared__ u64 r1[PS_THREADS / 32], r2l[PS_THREADS / 32], r2h[PS_THREADS / 32];
+  for (int o = 16; o > 0; o >>= 1) {
+    u64 a1 = __shfl_down_sync(0xffffffffu, s1, o);
+    u64 al = __shfl_down_sync(0xffffffffu, s2lo, o);
+    u64 ah = __shfl_down_sync(0xffffffffu, s2hi, o);
+    s1 += a1;
+    u64 t = s2lo + al;
+    s2hi += ah + (t < s2lo ? 1ull : 0ull);
+    s2lo = t;
+  }
+  if (lane_id() == 0) { r1[threadIdx.x >> 5] = s1; r2l[threadIdx.x >> 5] = s2lo; r2h[threadIdx.x >> 5] = s2hi; }
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  u128 d1 = 0, d2 = 0;
+  for (int w = 0; w < PS_THREADS / 32; w++) {
+    d1 += (u128)(int64_t)r1[w];  // partial sums of S1 are < 2^57 in magnitude: sign-extend
+    d2 += ((u128)r2h[w] << 64) | r2l[w];
   }
   u64 n = ib - ia;
-  u128 s1 = 0, s2 = 0;
+  u128 S1 = 0, S2 = 0;
   if (n) {
-    s1 = (((u128)P1[2 * ib + 1] << 64) | P1[2 * ib]) - (((u128)P1[2 * ia + 1] << 64) | P1[2 * ia]);
-    s2 = (((u128)P2[2 * ib + 1] << 64) | P2[2 * ib]) - (((u128)P2[2 * ia + 1] << 64) | P2[2 * ia]);
+    const u64* Pe = Pb + 4 * (ib / PREFIX_BLOCK);
+    const u64* Pa = Pb + 4 * (ia / PREFIX_BLOCK);
+    S1 = ((((u128)Pe[1] << 64) | Pe[0]) - (((u128)Pa[1] << 64) | Pa[0])) + d1;
+    S2 = ((((u128)Pe[3] << 64) | Pe[2]) - (((u128)Pa[3] << 64) | Pa[2])) + d2;
   }
   u64* L = lanes + (u64)p * MOM_LANES;
   L[0] = n;
-  limbs_from_u128((u64)s1, (u64)(s1 >> 64), L + 1);
-  limbs_from_u128((u64)s2, (u64)(s2 >> 64), L + 5);
-  u64 xmask = (bx >= 64) ? ~0ull : ((1ull << bx) - 1);
+  limbs_from_u128((u64)S1, (u64)(S1 >> 64), L + 1);
+  limbs_from_u128((u64)S2, (u64)(S2 >> 64), L + 5);
   mm[p] = n ? (keys[ia] & xmask) : ~0ull;            // min (reduced with MIN)
   mm[nparts + p] = n ? (keys[ib - 1] & xmask) : 0;   // max (reduced with MAX)
-  ab[2 * (u64)p] = a;
-  ab[2 * (u64)p + 1] = b;
 }
 
 void launch_part_stats(const SegDev* segs, u32 nseg, const u64* T, u32 tstride, const u32* nt,
                        const u32* part_off, u32 nparts, const u64* keys, u64 nkeys, u32 bx,
-                       const u64* P1, const u64* P2, u64* lanes, u64* mm, u64* ab, cudaStream_t s) {
+                       const u64* Pb, u64* lanes, u64* mm, u64* ab, cudaStream_t s) {
   if (nparts)
-    SV_LAUNCH(k_part_stats, div_up(nparts, 128), 128, 0, s)(segs, nseg, T, tstride, nt, part_off, nparts,
-                                                      keys, nkeys, bx, P1, P2, lanes, mm, ab);
+    SV_LAUNCH(k_part_stats, nparts, PS_THREADS, 0, s)(segs, nseg, T, tstride, nt, part_off, nparts,
+                                                   keys, nkeys, bx, Pb, lanes, mm, ab);
 }

@@ -8,14 +8,13 @@
 // and passes whose 8 bits are constant over all keys (found by one OR-reduction of key ^ key0)
 // are skipped.
 //
-// Radix pass = reduce-then-scan: per-tile digit histograms (warp-aggregated with match.any),
-// one exclusive scan over the digit-major [digit][tile] matrix, then a scatter that ranks keys
-// stably inside the tile (match.any per 32-key round), stages them in shared memory in tile
-// order and writes runs of equal digits coalesced.
+// Radix passes are onesweep (see below): one kernel per digit with decoupled look-back.
+#include <algorithm>
+
 #include "kernels.cuh"
 
 #define RS_THREADS 256
-#define RS_IPT 16
+#define RS_IPT 8
 #define RS_TILE (RS_THREADS * RS_IPT)
 #define RS_WARPS (RS_THREADS / 32)
 
@@ -135,15 +134,21 @@ k_t3_compact(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n,
   const u64 tile = (u64)CP_THREADS * CP_IPT;
   for (u64 base = (u64)blockIdx.x * tile; base < n; base += (u64)gridDim.x * tile) {
     u64 key[CP_IPT];
+    u32 kk[CP_IPT];
     u32 cnt = 0;
+#pragma unroll
+    for (int j = 0; j < CP_IPT; j++) {  // all independent loads first
+      u64 i = base + (u64)j * CP_THREADS + threadIdx.x;
+      bool ok = i < n;
+      kk[j] = ok ? __ldcs(kid + i) : 0u;
+      key[j] = ok ? __ldcs(x + i) : ~0ull;
+    }
 #pragma unroll
     for (int j = 0; j < CP_IPT; j++) {
       u64 i = base + (u64)j * CP_THREADS + threadIdx.x;
-      key[j] = ~0ull;
-      if (i < n) {
-        u32 r = t3rank[__ldcs(kid + i)];
-        if (r != 0xFFFFFFFFu) { key[j] = ((u64)r << bx) + __ldcs(x + i); cnt++; }
-      }
+      u32 r = i < n ? __ldg(t3rank + kk[j]) : 0xFFFFFFFFu;
+      if (r != 0xFFFFFFFFu) { key[j] = ((u64)r << bx) + key[j]; cnt++; }
+      else key[j] = ~0ull;
     }
     __shared__ u32 tot;
     __shared__ unsigned long long gbase;
@@ -169,57 +174,69 @@ void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u
 // ------------------------------------------------------------------------------------------
 // radix sort
 // ------------------------------------------------------------------------------------------
-__global__ void k_or_diff(const u64* keys, u64 n, u64* mask) {
-  u64 k0 = keys[0];
-  u64 m = 0;
-  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x)
-    m |= keys[i] ^ k0;
-  for (int o = 16; o > 0; o >>= 1) m |= __shfl_down_sync(0xffffffffu, m, o);
-  if (lane_id() == 0 && m) atomicOr((unsigned long long*)mask, m);
-}
+// ------------------------------------------------------------------------------------------
+// Onesweep (single-pass per digit) radix sort.  One upfront kernel reads the keys once and
+// builds the global 256-bin histogram of EVERY digit position; the host reads them back once
+// (skipping digits whose histogram has a single non-empty bin: that pass is the identity) and
+// scans them into global digit bases.  Each digit pass is then ONE kernel: a block takes the
+// next tile from an atomic counter (so predecessors are always resident), ranks its keys
+// stably (match.any per 32-key round), publishes its per-digit counts, and obtains its
+// exclusive per-digit prefix by decoupled look-back over the predecessors' published
+// aggregates / inclusive prefixes (64-bit status words: 2 flag bits + 62-bit count), then
+// scatters through shared memory in runs of equal digits.  16 B of HBM traffic per key per
+// pass (read + write), versus 24 B for reduce-then-scan.
+// ------------------------------------------------------------------------------------------
+#define OS_FLAG_AGG (1ull << 62)
+#define OS_FLAG_PREFIX (2ull << 62)
+#define OS_VALUE_MASK ((1ull << 62) - 1)
+#define OS_MAX_PASSES 8
 
 __global__ void __launch_bounds__(RS_THREADS)
-k_rs_hist(const u64* __restrict__ keys, u64 n, int shift, u32 ntiles, u32* __restrict__ hist) {
-  __shared__ u32 s_h[RS_WARPS][256];
-  for (int i = threadIdx.x; i < RS_WARPS * 256; i += RS_THREADS) (&s_h[0][0])[i] = 0;
+k_os_hist(const u64* __restrict__ keys, u64 n, int npass, u32* __restrict__ ghist) {
+  extern __shared__ u32 s_hist[];  // [RS_WARPS/2][npass][256] (pairs of warps share a table)
+  const int tables = RS_WARPS / 2;
+  for (int i = threadIdx.x; i < tables * npass * 256; i += RS_THREADS) s_hist[i] = 0;
   __syncthreads();
-  u32 w = threadIdx.x >> 5;
-  u64 base = (u64)blockIdx.x * RS_TILE + (u64)w * (RS_TILE / RS_WARPS);
-  u32 dig[RS_IPT];  // all loads of the tile in flight before any ranking
-#pragma unroll
-  for (int r = 0; r < RS_IPT; r++) {
-    u64 i = base + (u64)r * 32 + lane_id();
-    dig[r] = i < n ? (u32)(__ldcs(keys + i) >> shift) & 255u : 256u;
-  }
-#pragma unroll
-  for (int r = 0; r < RS_IPT; r++) {
-    u32 d = dig[r];
-    u32 peers = __match_any_sync(0xffffffffu, d);
-    if (d < 256u && lane_id() == (u32)(__ffs(peers) - 1)) s_h[w][d] += __popc(peers);
-    __syncwarp();
+  u32* mine = s_hist + (threadIdx.x >> 6) * npass * 256;
+  for (u64 i = (u64)blockIdx.x * RS_THREADS + threadIdx.x; i < n; i += (u64)gridDim.x * RS_THREADS) {
+    u64 k = __ldcs(keys + i);
+    for (int p = 0; p < npass; p++) atomicAdd(&mine[p * 256 + ((k >> (8 * p)) & 255u)], 1u);
   }
   __syncthreads();
-  u32 d = threadIdx.x;  // RS_THREADS == 256 digits
-  u32 s = 0;
-#pragma unroll
-  for (int j = 0; j < RS_WARPS; j++) s += s_h[j][d];
-  hist[(u64)d * ntiles + blockIdx.x] = s;
+  for (int i = threadIdx.x; i < npass * 256; i += RS_THREADS) {
+    u32 s = 0;
+    for (int t = 0; t < tables; t++) s += s_hist[t * npass * 256 + i];
+    if (s) atomicAdd(&ghist[i], s);
+  }
 }
 
-__global__ void __launch_bounds__(RS_THREADS)
-k_rs_scatter(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int shift,
-             u32 ntiles, const u32* __restrict__ off, u64* __restrict__ kout,
-             u32* __restrict__ vout) {
+__device__ __forceinline__ u64 ld_volatile_u64(const u64* p) {
+  u64 v;
+  asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void st_volatile_u64(u64* p, u64 v) {
+  asm volatile("st.volatile.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+template <bool V>  // V: a u32 payload travels with each key
+__global__ void __launch_bounds__(RS_THREADS, 4)
+k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int shift,
+          const u32* __restrict__ gbase, u64* status, u32* tile_counter, u64* __restrict__ kout,
+          u32* __restrict__ vout) {
   extern __shared__ __align__(16) unsigned char smem[];
   u64* s_k = (u64*)smem;                        // [RS_TILE]
   u32* s_v = (u32*)(s_k + RS_TILE);             // [RS_TILE] (if values)
   __shared__ u32 s_wh[RS_WARPS][256];           // per-warp digit counts -> warp offsets
   __shared__ u32 s_td[256];                     // tile-local digit offsets
-  __shared__ u32 s_go[256];                     // global digit offsets of this tile
+  __shared__ u64 s_go[256];                     // global digit offsets of this tile
+  __shared__ u32 s_tile;
+  if (threadIdx.x == 0) s_tile = atomicAdd(tile_counter, 1u);
   for (int i = threadIdx.x; i < RS_WARPS * 256; i += RS_THREADS) (&s_wh[0][0])[i] = 0;
   __syncthreads();
+  const u32 tile = s_tile;
   u32 w = threadIdx.x >> 5;
-  u64 base = (u64)blockIdx.x * RS_TILE + (u64)w * (RS_TILE / RS_WARPS);
+  u64 base = (u64)tile * RS_TILE + (u64)w * (RS_TILE / RS_WARPS);
   u64 key[RS_IPT];
   u32 val[RS_IPT];
   u32 rank[RS_IPT];
@@ -228,7 +245,7 @@ k_rs_scatter(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, in
     u64 i = base + (u64)r * 32 + lane_id();
     bool ok = i < n;
     key[r] = ok ? __ldcs(kin + i) : 0;
-    val[r] = (ok && vin) ? __ldcs(vin + i) : 0;
+    if (V) val[r] = ok ? __ldcs(vin + i) : 0;
   }
 #pragma unroll
   for (int r = 0; r < RS_IPT; r++) {
@@ -244,15 +261,29 @@ k_rs_scatter(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, in
     __syncwarp();
   }
   __syncthreads();
-  {  // thread d: exclusive over warps, then exclusive over digits
+  {  // thread d: warp offsets, tile count, publish, look back, tile-local digit offsets
     u32 d = threadIdx.x;
     u32 run = 0;
 #pragma unroll
     for (int j = 0; j < RS_WARPS; j++) { u32 c = s_wh[j][d]; s_wh[j][d] = run; run += c; }
+    u64* my = status + (u64)tile * 256 + d;
+    u64 excl = 0;
+    if (tile == 0) {
+      st_volatile_u64(my, OS_FLAG_PREFIX | run);
+    } else {
+      st_volatile_u64(my, OS_FLAG_AGG | run);
+      for (u32 j = tile - 1;; j--) {
+        u64 v;
+        do { v = ld_volatile_u64(status + (u64)j * 256 + d); } while ((v >> 62) == 0);
+        excl += v & OS_VALUE_MASK;
+        if (v & OS_FLAG_PREFIX) break;
+      }
+      st_volatile_u64(my, OS_FLAG_PREFIX | (excl + run));
+    }
     __shared__ u32 tot;
     u32 ex = block_excl_scan<u32, RS_THREADS>(run, &tot);
     s_td[d] = ex;
-    s_go[d] = off[(u64)d * ntiles + blockIdx.x];
+    s_go[d] = (u64)gbase[d] + excl;
   }
   __syncthreads();
 #pragma unroll
@@ -262,57 +293,79 @@ k_rs_scatter(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, in
       u32 d = (u32)(key[r] >> shift) & 255u;
       u32 p = s_td[d] + s_wh[w][d] + rank[r];
       s_k[p] = key[r];
-      if (vin) s_v[p] = val[r];
+      if (V) s_v[p] = val[r];
     }
   }
   __syncthreads();
-  u64 tile_n = n - (u64)blockIdx.x * RS_TILE;
+  u64 tile_n = n - (u64)tile * RS_TILE;
   if (tile_n > RS_TILE) tile_n = RS_TILE;
   for (u32 j = threadIdx.x; j < tile_n; j += RS_THREADS) {
     u64 k = s_k[j];
     u32 d = (u32)(k >> shift) & 255u;
-    u64 o = (u64)s_go[d] + (j - s_td[d]);
+    u64 o = s_go[d] + (j - s_td[d]);
     kout[o] = k;
-    if (vin) vout[o] = s_v[j];
+    if (V) vout[o] = s_v[j];
   }
 }
 
+static size_t al256(size_t b) { return (b + 255) / 256 * 256; }
+
 size_t radix_sort_temp_bytes(u64 n, bool with_vals) {
   u64 ntiles = (n + RS_TILE - 1) / RS_TILE;
-  size_t b = 0;
-  b += ((n * 8 + 255) / 256) * 256;                       // alt keys
-  if (with_vals) b += ((n * 4 + 255) / 256) * 256;        // alt vals
-  b += ((256 * ntiles * 4 + 255) / 256) * 256;            // histogram / offsets
-  b += ((scan_u32_temp_bytes(256 * ntiles) + 255) / 256) * 256;
-  b += 256;                                               // diff mask
+  size_t b = al256(n * 8);                       // alt keys
+  if (with_vals) b += al256(n * 4);              // alt vals
+  b += al256(ntiles * 256 * 8);                  // look-back status words
+  b += al256(OS_MAX_PASSES * 256 * 4) * 2;       // histograms, bases
+  b += 256;                                      // tile counter
   return b;
 }
 
 int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, int* passes) {
   if (passes) *passes = 0;
   if (n <= 1 || nbits <= 0) return SIEVE_OK;
+  if (nbits > 8 * OS_MAX_PASSES) nbits = 8 * OS_MAX_PASSES;
+  const int npass = (nbits + 7) / 8;
   u64 ntiles = (n + RS_TILE - 1) / RS_TILE;
   char* t = (char*)temp;
-  u64* kalt = (u64*)t; t += ((n * 8 + 255) / 256) * 256;
+  u64* kalt = (u64*)t; t += al256(n * 8);
   u32* valt = nullptr;
-  if (vals) { valt = (u32*)t; t += ((n * 4 + 255) / 256) * 256; }
-  u32* hist = (u32*)t; t += ((256 * ntiles * 4 + 255) / 256) * 256;
-  void* stemp = t; t += ((scan_u32_temp_bytes(256 * ntiles) + 255) / 256) * 256;
-  u64* dmask = (u64*)t;
-  SV_CUDA(cudaMemsetAsync(dmask, 0, 8, s));
-  SV_LAUNCH(k_or_diff, sv_num_sms() * 2, 256, 0, s)(keys, n, dmask);
-  u64 mask = 0;
-  SV_CUDA(cudaMemcpyAsync(&mask, dmask, 8, cudaMemcpyDeviceToHost, s));
+  if (vals) { valt = (u32*)t; t += al256(n * 4); }
+  u64* status = (u64*)t; t += al256(ntiles * 256 * 8);
+  u32* ghist = (u32*)t; t += al256(OS_MAX_PASSES * 256 * 4);
+  u32* gbase = (u32*)t; t += al256(OS_MAX_PASSES * 256 * 4);
+  u32* tile_counter = (u32*)t;
+  SV_CUDA(cudaMemsetAsync(ghist, 0, (size_t)npass * 256 * 4, s));
+  size_t hsmem = (size_t)(RS_WARPS / 2) * npass * 256 * 4;
+  SV_CUDA(cudaFuncSetAttribute(k_os_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsmem));
+  u64 hgrid = std::min<u64>((n + RS_THREADS - 1) / RS_THREADS, (u64)sv_num_sms() * 4);
+  SV_LAUNCH(k_os_hist, (unsigned)hgrid, RS_THREADS, hsmem, s)(keys, n, npass, ghist);
+  u32 h[OS_MAX_PASSES * 256];
+  SV_CUDA(cudaMemcpyAsync(h, ghist, (size_t)npass * 256 * 4, cudaMemcpyDeviceToHost, s));
   SV_CUDA(cudaStreamSynchronize(s));
-  size_t smem = (size_t)RS_TILE * (8 + 4);
-  SV_CUDA(cudaFuncSetAttribute(k_rs_scatter, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  u32 bases[OS_MAX_PASSES * 256];
+  bool active[OS_MAX_PASSES];
+  for (int p = 0; p < npass; p++) {
+    u32 run = 0, nonzero = 0;
+    for (int d = 0; d < 256; d++) {
+      bases[p * 256 + d] = run;
+      run += h[p * 256 + d];
+      nonzero += h[p * 256 + d] != 0;
+    }
+    active[p] = nonzero > 1;  // a single non-empty bin: the pass is the identity
+  }
+  SV_CUDA(cudaMemcpyAsync(gbase, bases, (size_t)npass * 256 * 4, cudaMemcpyHostToDevice, s));
+  size_t smem = (size_t)RS_TILE * (vals ? 8 + 4 : 8);
   u64* kin = keys; u32* vin = vals; u64* kout = kalt; u32* vout = valt;
-  for (int shift = 0; shift < nbits; shift += 8) {
-    if (((mask >> shift) & 255u) == 0) continue;   // constant digit: the pass is the identity
-    SV_LAUNCH(k_rs_hist, (unsigned)ntiles, RS_THREADS, 0, s)(kin, n, shift, (u32)ntiles, hist);
-    scan_u32(hist, hist, 256 * ntiles, stemp, nullptr, s);
-    SV_LAUNCH(k_rs_scatter, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, shift, (u32)ntiles, hist,
-                                                            kout, vout);
+  for (int p = 0; p < npass; p++) {
+    if (!active[p]) continue;
+    SV_CUDA(cudaMemsetAsync(status, 0, ntiles * 256 * 8, s));
+    SV_CUDA(cudaMemsetAsync(tile_counter, 0, 4, s));
+    if (vals)
+      SV_LAUNCH(k_os_pass<true>, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, 8 * p, gbase + p * 256,
+                                                                     status, tile_counter, kout, vout);
+    else
+      SV_LAUNCH(k_os_pass<false>, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, 8 * p, gbase + p * 256,
+                                                                      status, tile_counter, kout, vout);
     u64* tk = kin; kin = kout; kout = tk;
     u32* tv = vin; vin = vout; vout = tv;
     if (passes) (*passes)++;
@@ -397,36 +450,15 @@ __global__ void __launch_bounds__(PX_THREADS) k_px_blocks(Pair128* bsum, u32 nb)
   }
 }
 
-__global__ void __launch_bounds__(PX_THREADS)
-k_px_apply(const u64* keys, u64 n, u64 xmask, const Pair128* bsum, u64* P1, u64* P2) {
-  u64 base = (u64)blockIdx.x * PX_TILE + (u64)threadIdx.x * PX_IPT;
-  Pair128 v[PX_IPT];
-  Pair128 s = pzero();
-#pragma unroll
-  for (int j = 0; j < PX_IPT; j++) {
-    v[j] = base + j < n ? px_val(keys[base + j], xmask) : pzero();
-    s += v[j];
-  }
-  __shared__ Pair128 tot;
-  Pair128 ex = block_excl_scan<Pair128, PX_THREADS>(s, &tot) + bsum[blockIdx.x];
-#pragma unroll
-  for (int j = 0; j < PX_IPT; j++) {
-    if (base + j <= n) {
-      P1[2 * (base + j)] = ex.a.lo; P1[2 * (base + j) + 1] = ex.a.hi;
-      P2[2 * (base + j)] = ex.b.lo; P2[2 * (base + j) + 1] = ex.b.hi;
-    }
-    ex += v[j];
-  }
-}
+static_assert(PX_TILE == PREFIX_BLOCK, "prefix block size");
 
-size_t prefix128_temp_bytes(u64 n) { return ((n + PX_TILE) / PX_TILE + 2) * sizeof(Pair128); }
+u64 block_prefix_entries(u64 n) { return (n + PX_TILE - 1) / PX_TILE + 1; }
 
-void launch_prefix128(const u64* keys, u64 n, u64 xmask, u64* P1, u64* P2, void* temp,
-                      cudaStream_t s) {
-  // n+1 outputs: cover index n with one extra element slot
-  u32 nb = div_up(n + 1, PX_TILE);
-  Pair128* bsum = (Pair128*)temp;
-  SV_LAUNCH(k_px_reduce, nb, PX_THREADS, 0, s)(keys, n, xmask, bsum);
-  SV_LAUNCH(k_px_blocks, 1, PX_THREADS, 0, s)(bsum, nb);
-  SV_LAUNCH(k_px_apply, nb, PX_THREADS, 0, s)(keys, n, xmask, bsum, P1, P2);
+// Pb[i] = (sum x, sum x^2) over keys[0, i * PREFIX_BLOCK), i = 0..nb (Pb[nb] = totals); part
+// sums need only these block boundaries plus at most two partial blocks (refine.cu)
+void launch_block_prefix(const u64* keys, u64 n, u64 xmask, u64* Pb, cudaStream_t s) {
+  u32 ne = (u32)block_prefix_entries(n);
+  Pair128* bsum = (Pair128*)Pb;
+  SV_LAUNCH(k_px_reduce, ne, PX_THREADS, 0, s)(keys, n, xmask, bsum);  // last block sums nothing
+  SV_LAUNCH(k_px_blocks, 1, PX_THREADS, 0, s)(bsum, ne);
 }

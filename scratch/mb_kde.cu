@@ -1,0 +1,52 @@
+// Throwaway microbenchmark: achievable rate of the KDE term's instruction mix (no memory).
+#include <cstdio>
+#include <cstdint>
+typedef unsigned long long u64; typedef unsigned u32;
+#define C_LOG2E_32 0x1.71547652b82fep+5
+#define C_LN2_32_HI 0x1.62e42fee00000p-6
+#define C_LN2_32_LO 0x1.a39ef35793c76p-38
+#define C_MAGIC 0x1.8p+52
+#define C_TWO52 0x1.0p+52
+#define C_P5 (-0x1.1111111111111p-7 * 0x1p-5)
+#define C_P4 (0x1.5555555555555p-5 * 0x1p-4)
+#define C_P3 (-0x1.5555555555555p-3 * 0x1p-3)
+__device__ __forceinline__ u64 q(double g, double xd, double inv_h, const double* sS) {
+  double z = __dmul_rn(__dsub_rn(g, xd), inv_h);
+  double u = __dmul_rn(z, z);
+  double kb = __dadd_rn(__dmul_rn(u, C_LOG2E_32), C_MAGIC);
+  double kf = __dsub_rn(kb, C_MAGIC);
+  u32 k = min((u32)__double2loint(kb), 3417u);
+  k = (u32)__double2hiint(u) >= 0x40540000u ? 3417u : k;
+  double r = __fma_rn(-kf, C_LN2_32_HI, u);
+  r = __fma_rn(-kf, C_LN2_32_LO, r);
+  double p = __fma_rn(C_P5, r, C_P4);
+  p = __fma_rn(p, r, C_P3); p = __fma_rn(p, r, 0.125); p = __fma_rn(p, r, -0.5); p = __fma_rn(p, r, 1.0);
+  return (u64)__double_as_longlong(__fma_rn(p, sS[k], C_TWO52));
+}
+template<int U, int NOTAB>
+__global__ void k(u64* out, int iters, double g0, double ih) {
+  __shared__ double sS[3418];
+  for (int i = threadIdx.x; i < 3418; i += blockDim.x) sS[i] = 1.0 + i * 1e-9;
+  __syncthreads();
+  double g = g0 + threadIdx.x * 0.37; u64 acc = 0; double x = 1000.0 + blockIdx.x;
+  for (int it = 0; it < iters; it++) {
+#pragma unroll
+    for (int u = 0; u < U; u++) acc += q(g, x + u, ih, sS);
+    x += U;
+  }
+  if (acc == 42) out[0] = acc;
+}
+int main() {
+  u64* o; cudaMalloc(&o, 8); cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
+  int iters = 20000; float ms;
+  auto run = [&](auto kern, int U, int blocksPerSM, int threads) {
+    for (int r = 0; r < 2; r++) { cudaEventRecord(a); kern<<<148 * blocksPerSM, threads>>>(o, iters, 1000.0, 0.01); cudaEventRecord(b); cudaEventSynchronize(b); }
+    cudaEventElapsedTime(&ms, a, b);
+    double terms = 148.0 * blocksPerSM * threads * (double)iters * U;
+    double tops = terms * 14 / (ms * 1e-3) / 1e12;
+    printf("U=%d blocks/SM=%d threads=%d: %.3f ms  %.3g terms/s  %.2f Top/s FP64 = %.1f%% of 18.61\n", U, blocksPerSM, threads, ms, terms / (ms * 1e-3), tops, 100 * tops / 18.61);
+  };
+  run(k<1,0>, 1, 4, 256); run(k<2,0>, 2, 4, 256); run(k<4,0>, 4, 4, 256); run(k<8,0>, 8, 4, 256);
+  run(k<4,0>, 4, 8, 256); run(k<4,0>, 4, 2, 256); run(k<2,0>, 2, 8, 256);
+  return 0;
+}
