@@ -155,6 +155,23 @@ int sieve_strata_copy(sieve_strata s, sieve_stratum* host_out, uint64_t cap);
 int sieve_strata_stats(sieve_strata s, uint32_t* rounds, uint64_t* kde_terms);
 void sieve_strata_free(sieve_strata s);
 
+/* ---- theta studies (Fig. 2, Fig. 10) -------------------- */
+
+/* Stratify for `count` thresholds theta_i = theta_num[i] / theta_den[i] (host arrays) in one
+   call: the per-kernel moments (pass A and its reduction) are computed once and reused; each
+   theta then runs tiering, the Tier-3 refinement and the assignment.  outs[i] receives the
+   strata for theta_i (free each with sieve_strata_free); on error none is returned.
+   Other fields of *p (grid, valley shift, ...) apply to every theta.  Collective if world > 1. */
+int sieve_stratify_sweep(sieve_trace t, const sieve_params* p, uint32_t count,
+                         const uint32_t* theta_num, const uint32_t* theta_den, sieve_strata* outs);
+
+/* Tier census (Fig. 2): for each theta_i, the number of kernels, invocations and instructions
+   (u128 as lo, hi) in Tier-1/2/3, from one moments pass.  kernels, invocations: HOST
+   [count][3]; instructions: nullable HOST [count][3][2].  Collective if world > 1. */
+int sieve_tier_census(sieve_trace t, uint32_t count, const uint32_t* theta_num,
+                      const uint32_t* theta_den, uint64_t* kernels, uint64_t* invocations,
+                      uint64_t* instructions);
+
 /* ---- debug: every KDE segment of every round (requires keep_debug = 1, else ESTATE) ---- */
 typedef struct {
   uint32_t kernel_id, round, split_kind /* 1 = valley, 2 = bisect */, n_cuts;

@@ -488,7 +488,9 @@ static int sync(sieve_ctx c) { SV_CUDA(cudaStreamSynchronize(c->stream)); return
 // ------------------------------------------------------------------------------------------
 // sieve_stratify
 // ------------------------------------------------------------------------------------------
-struct OpenSeg { u32 kid, t3rank; u64 lo, hi, n; u128 s1, s2; };
+// an open Tier-3 segment: global value range / moments (replicated) and this rank's index
+// range [b, e) in the sorted keys (local)
+struct OpenSeg { u32 kid, t3rank; u64 lo, hi, n; u128 s1, s2; u64 b, e; };
 
 // host-side wall-clock marks (SIEVE_HOST_TIMING=1 prints them to stderr): where the host
 // orchestration, not the device, spends time
@@ -511,15 +513,18 @@ struct HostClock {
 };
 struct Fin { u32 kid, tier; u64 lo, hi, n; u128 s1; double h; u32 round; };
 
-static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out, sieve_strata_s* R) {
+// pass A results on the host (replicated after AR-1): theta-independent, so a theta sweep or a
+// tier census computes them once
+struct MomentsHost {
+  std::vector<u64> lanes, mm, tot, localn;
+};
+
+// ---------------- pass A: per-kernel moments + totals -------------------
+static int moments_pass(sieve_trace t, MomentsHost* M) {
   sieve_ctx c = t->ctx;
   cudaStream_t S = c->stream;
-  SV_TRY(arena_reset(c));
-  HostClock hc;
-  const u32 K = t->K, G = P->grid_points;
+  const u32 K = t->K;
   const u64 n = t->n;
-
-  // ---------------- pass A: per-kernel moments + totals --------------------------------------
   const int gridA = moments_grid();
   const u32 kt = (u32)moments_kt(K);
   DBuf<KMomPartial> part(c);
@@ -579,11 +584,33 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(d2h(c, h_localn, local_n.get(), K));
     SV_TRY(sync(c));
   }
-  part.release(); blk_tot.release();
   if (h_tot[5]) return sv_fail(SIEVE_EINVAL, "kernel id >= num_kernels in the trace");
   if (h_tot[6]) return sv_fail(SIEVE_ERANGE, "instruction count 0 or >= 2^44 in the trace (A21)");
-  R->c_meas = limbs_u128(&h_tot[0]);
-  const u64 max_x = h_tot[4];
+  M->lanes.swap(h_lanes);
+  M->mm.swap(h_mm);
+  M->tot.swap(h_tot);
+  M->localn.swap(h_localn);
+  return SIEVE_OK;
+}
+
+static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out, sieve_strata_s* R,
+                         const MomentsHost* cached) {
+  sieve_ctx c = t->ctx;
+  cudaStream_t S = c->stream;
+  SV_TRY(arena_reset(c));
+  HostClock hc;
+  const u32 K = t->K, G = P->grid_points;
+  const u64 n = t->n;
+  MomentsHost own;
+  if (!cached) {
+    SV_TRY(moments_pass(t, &own));
+    cached = &own;
+  }
+  const std::vector<u64>& h_lanes = cached->lanes;
+  const std::vector<u64>& h_mm = cached->mm;
+  const std::vector<u64>& h_localn = cached->localn;
+  R->c_meas = limbs_u128(&cached->tot[0]);
+  const u64 max_x = cached->tot[4];
 
   hc.mark("passA");
   // ---------------- tiers ---------------------------------------------------------
@@ -606,8 +633,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       fin.push_back({k, 2, lo, hi, nk, s1, 0.0, 0});
     } else {                                                     // Tier-3 -> refinement
       t3rank[k] = n_t3++;
+      // the sorted keys are grouped by t3rank: this kernel's local range follows the previous
+      open.push_back({k, t3rank[k], lo, hi, nk, s1, s2, n3_local, n3_local + h_localn[k]});
       n3_local += h_localn[k];
-      open.push_back({k, t3rank[k], lo, hi, nk, s1, s2});
     }
   }
   R->total_instr = I;
@@ -671,7 +699,8 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       hs[s].hi = o.hi;
       hs[s].h = h;
       hs[s].inv_h = 1.0 / h;
-      hs[s].begin = hs[s].end = 0;
+      hs[s].begin = nkeys ? o.b : 0;  // local index range (no device search needed)
+      hs[s].end = nkeys ? o.e : 0;
     }
     DBuf<SegDev> segs(c);
     SV_TRY(segs.alloc(nseg));
@@ -680,16 +709,20 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(D.alloc((size_t)nseg * G * 2));
     SV_CUDA(cudaMemsetAsync(D.get(), 0, (size_t)nseg * G * 16, S));
     if (nkeys) {
-      launch_seg_ranges(segs.get(), nseg, keys.get(), nkeys, S);
       DBuf<u64> tile_range(c);
       DBuf<u32> tile_items(c);
       DBuf<char> stemp(c);
       SV_TRY(tile_range.alloc((size_t)nseg * tps * 2));
       SV_TRY(tile_items.alloc((size_t)nseg * tps + 1));
       SV_TRY(stemp.alloc(((size_t)nseg * tps / 4096 + 4) * 4));
-      u32 items = 0;
+      // work items are counted on the device; size the item map by a host-side bound so no
+      // synchronisation is needed here: a tile has at most ceil(segment length / KDE_CH) items
+      u64 items_bound = 0;
+      for (u32 s = 0; s < nseg; s++) items_bound += (u64)tps * ((open[s].e - open[s].b + KDE_CH - 1) / KDE_CH);
+      if (items_bound >= (1ull << 32)) return sv_fail(SIEVE_ELIMIT, "too many KDE work items");
+      u32 items = (u32)items_bound;
       SV_TRY(kde_plan(segs.get(), nseg, G, keys.get(), nkeys, xmask, tile_range.get(),
-                      tile_items.get(), stemp.get(), &items, S));
+                      tile_items.get(), stemp.get(), nullptr, S));
       DBuf<char> item_tile(c);
       SV_TRY(item_tile.alloc(kde_item_bytes(items)));
       PhaseTimer tm(c, SIEVE_PHASE_KDE, 0);
@@ -726,7 +759,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     DBuf<u64> pl(c), pm(c), pab(c);
     SV_TRY(pl.alloc((size_t)nparts * MOM_LANES));
     SV_TRY(pm.alloc((size_t)nparts * 2));
-    SV_TRY(pab.alloc((size_t)nparts * 2));
+    SV_TRY(pab.alloc((size_t)nparts * 4));
     PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
     launch_part_stats(segs.get(), nseg, T.get(), tstride, ntk.get(), d_off.get(), nparts,
                       nkeys ? keys.get() : nullptr, nkeys, bx, Pb.get(), pl.get(),
@@ -739,7 +772,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     std::vector<u64> h_pl, h_pm, h_ab;
     SV_TRY(d2h(c, h_pl, pl.get(), (size_t)nparts * MOM_LANES));
     SV_TRY(d2h(c, h_pm, pm.get(), (size_t)nparts * 2));
-    SV_TRY(d2h(c, h_ab, pab.get(), (size_t)nparts * 2));
+    SV_TRY(d2h(c, h_ab, pab.get(), (size_t)nparts * 4));
     std::vector<u64> h_D, h_T;
     if (R->keep_debug) {
       SV_TRY(d2h(c, h_D, D.get(), (size_t)nseg * G * 2));
@@ -775,7 +808,8 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         if (lo == hi || cov_lt(pn, s1, s2, P->theta_num, P->theta_den))
           fin.push_back({open[s].kid, 3, lo, hi, pn, s1, hh[s], round});
         else
-          next.push_back({open[s].kid, open[s].t3rank, lo, hi, pn, s1, s2});
+          next.push_back({open[s].kid, open[s].t3rank, lo, hi, pn, s1, s2, h_ab[4 * (size_t)p + 2],
+                          h_ab[4 * (size_t)p + 3]});
       }
     }
     open.swap(next);
@@ -947,31 +981,104 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   return SIEVE_OK;
 }
 
-extern "C" int sieve_stratify(sieve_trace t, const sieve_params* p, uint32_t* sid_out, sieve_strata* out) {
-  if (!out) return sv_fail(SIEVE_EINVAL, "out is NULL");
-  *out = nullptr;
-  if (!trace_ok(t)) return sv_fail(SIEVE_EINVAL, "bad trace handle");
-  sieve_params P;
-  if (p) P = *p; else sieve_params_default(&P);
-  if (P.theta_num == 0 || P.theta_den == 0) return sv_fail(SIEVE_EINVAL, "theta must be a positive fraction");
-  if (P.grid_points < 3 || P.grid_points > 65536) return sv_fail(SIEVE_EINVAL, "grid_points must be in [3, 65536]");
-  if (P.valley_shift > 120) return sv_fail(SIEVE_EINVAL, "valley_shift must be <= 120");
-  if (!(P.bw_scale > 0)) return sv_fail(SIEVE_EINVAL, "bw_scale must be > 0");
-  if (P.max_rounds == 0) P.max_rounds = 1;
+static int check_params(const sieve_params* p, sieve_params* P) {
+  if (p) *P = *p; else sieve_params_default(P);
+  if (P->theta_num == 0 || P->theta_den == 0) return sv_fail(SIEVE_EINVAL, "theta must be a positive fraction");
+  if (P->grid_points < 3 || P->grid_points > 65536) return sv_fail(SIEVE_EINVAL, "grid_points must be in [3, 65536]");
+  if (P->valley_shift > 120) return sv_fail(SIEVE_EINVAL, "valley_shift must be <= 120");
+  if (!(P->bw_scale > 0)) return sv_fail(SIEVE_EINVAL, "bw_scale must be > 0");
+  if (P->max_rounds == 0) P->max_rounds = 1;
+  return SIEVE_OK;
+}
+
+static int stratify_one(sieve_trace t, const sieve_params* P, uint32_t* sid_out, sieve_strata* out,
+                        const MomentsHost* cached) {
   sieve_ctx c = t->ctx;
-  SV_CUDA(cudaSetDevice(c->device));
   sieve_strata_s* R = new sieve_strata_s();
   R->ctx = c;
-  R->G = P.grid_points;
-  R->keep_debug = P.keep_debug != 0;
+  R->G = P->grid_points;
+  R->keep_debug = P->keep_debug != 0;
   R->has_cycles = t->y != nullptr;
-  int st = stratify_impl(t, &P, sid_out, R);
+  int st = stratify_impl(t, P, sid_out, R, cached);
   if (st != SIEVE_OK) {
     cudaStreamSynchronize(c->stream);
     delete R;
     return st;
   }
   *out = R;
+  return SIEVE_OK;
+}
+
+extern "C" int sieve_stratify(sieve_trace t, const sieve_params* p, uint32_t* sid_out, sieve_strata* out) {
+  if (!out) return sv_fail(SIEVE_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!trace_ok(t)) return sv_fail(SIEVE_EINVAL, "bad trace handle");
+  sieve_params P;
+  SV_TRY(check_params(p, &P));
+  SV_CUDA(cudaSetDevice(t->ctx->device));
+  return stratify_one(t, &P, sid_out, out, nullptr);
+}
+
+extern "C" int sieve_stratify_sweep(sieve_trace t, const sieve_params* p, uint32_t count,
+                                    const uint32_t* theta_num, const uint32_t* theta_den,
+                                    sieve_strata* outs) {
+  if (!outs || (count && (!theta_num || !theta_den))) return sv_fail(SIEVE_EINVAL, "NULL argument");
+  for (uint32_t i = 0; i < count; i++) outs[i] = nullptr;
+  if (!trace_ok(t)) return sv_fail(SIEVE_EINVAL, "bad trace handle");
+  sieve_params P;
+  SV_TRY(check_params(p, &P));
+  for (uint32_t i = 0; i < count; i++)
+    if (!theta_num[i] || !theta_den[i]) return sv_fail(SIEVE_EINVAL, "theta must be a positive fraction");
+  sieve_ctx c = t->ctx;
+  SV_CUDA(cudaSetDevice(c->device));
+  SV_TRY(arena_reset(c));
+  MomentsHost M;
+  SV_TRY(moments_pass(t, &M));  // pass A once for every theta
+  for (uint32_t i = 0; i < count; i++) {
+    P.theta_num = theta_num[i];
+    P.theta_den = theta_den[i];
+    int st = stratify_one(t, &P, nullptr, &outs[i], &M);
+    if (st != SIEVE_OK) {
+      for (uint32_t j = 0; j < i; j++) { sieve_strata_free(outs[j]); outs[j] = nullptr; }
+      return st;
+    }
+  }
+  return SIEVE_OK;
+}
+
+extern "C" int sieve_tier_census(sieve_trace t, uint32_t count, const uint32_t* theta_num,
+                                 const uint32_t* theta_den, uint64_t* kernels, uint64_t* invocations,
+                                 uint64_t* instructions) {
+  if (!trace_ok(t) || (count && (!theta_num || !theta_den || !kernels || !invocations)))
+    return sv_fail(SIEVE_EINVAL, "bad argument");
+  for (uint32_t i = 0; i < count; i++)
+    if (!theta_num[i] || !theta_den[i]) return sv_fail(SIEVE_EINVAL, "theta must be a positive fraction");
+  sieve_ctx c = t->ctx;
+  SV_CUDA(cudaSetDevice(c->device));
+  SV_TRY(arena_reset(c));
+  MomentsHost M;
+  SV_TRY(moments_pass(t, &M));
+  for (uint32_t i = 0; i < count; i++) {
+    u64 nk[3] = {0, 0, 0}, ni[3] = {0, 0, 0};
+    u128 ins[3] = {0, 0, 0};
+    for (u32 k = 0; k < t->K; k++) {
+      const u64* L = &M.lanes[(size_t)k * MOM_LANES];
+      if (!L[0]) continue;
+      u128 s1 = limbs_u128(L + 1), s2 = limbs_u128(L + 5);
+      int tier = M.mm[2 * k] == M.mm[2 * k + 1] ? 0 : (cov_lt(L[0], s1, s2, theta_num[i], theta_den[i]) ? 1 : 2);
+      nk[tier]++;
+      ni[tier] += L[0];
+      ins[tier] += s1;
+    }
+    for (int j = 0; j < 3; j++) {
+      kernels[3 * (size_t)i + j] = nk[j];
+      invocations[3 * (size_t)i + j] = ni[j];
+      if (instructions) {
+        instructions[6 * (size_t)i + 2 * j] = (u64)ins[j];
+        instructions[6 * (size_t)i + 2 * j + 1] = (u64)(ins[j] >> 64);
+      }
+    }
+  }
   return SIEVE_OK;
 }
 

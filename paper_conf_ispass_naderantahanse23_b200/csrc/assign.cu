@@ -16,11 +16,11 @@
 #include "kernels.cuh"
 
 #define AS_THREADS 512
-#define AS_IPT 8
+#define AS_IPT 4
 #define AS_HC 4096          // shared hash capacity (entries)
 #define AS_MAXP 32          // probes before falling back to the global table
 
-int assign_grid() { return 3 * sv_num_sms(); }
+int assign_grid() { return 2 * sv_num_sms(); }
 
 __device__ __forceinline__ u32 hash_key(u64 k) {
   return (u32)((k * 0x9E3779B97F4A7C15ull) >> 32);

@@ -96,16 +96,19 @@ int kde_plan(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 nkeys, u6
   u32 tps = div_up(G, KDE_TJ);
   u64 nt = (u64)nseg * tps;
   SV_LAUNCH(k_kde_tiles, div_up(nt, 128), 128, 0, s)(segs, nseg, G, tps, keys, tile_range, tile_items);
-  // exclusive scan in place; tile_items[nt] receives the total
+  // exclusive scan in place; tile_items[nt] receives the total (read on the device by k_kde)
   scan_u32(tile_items, tile_items, nt, scan_temp, tile_items + nt, s);
-  SV_CUDA(cudaMemcpyAsync(items_host, tile_items + nt, 4, cudaMemcpyDeviceToHost, s));
-  SV_CUDA(cudaStreamSynchronize(s));
+  if (items_host) {
+    SV_CUDA(cudaMemcpyAsync(items_host, tile_items + nt, 4, cudaMemcpyDeviceToHost, s));
+    SV_CUDA(cudaStreamSynchronize(s));
+  }
   return SIEVE_OK;
 }
 
 // item -> tile map (so a warp finds its tile with one load): one thread per item, binary
 // search of the last tile whose first item is <= it
-__global__ void k_kde_items(const u32* tile_items, u32 ntiles, u32 items, u32* item_tile) {
+__global__ void k_kde_items(const u32* tile_items, u32 ntiles, u32* item_tile) {
+  const u32 items = tile_items[ntiles];  // device-side total (no host round trip)
   for (u32 it = blockIdx.x * blockDim.x + threadIdx.x; it < items; it += gridDim.x * blockDim.x) {
     u32 lo = 0, hi = ntiles - 1;
     while (lo < hi) {
@@ -175,8 +178,9 @@ __device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, cons
 __global__ void __launch_bounds__(32 * KDE_WARPS)
 k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ keys, u64 xmask,
       const u64* __restrict__ tile_range, const u32* __restrict__ tile_items,
-      const u32* __restrict__ item_tile, u32 items, u64* D, unsigned long long* counter,
+      const u32* __restrict__ item_tile, u32 ntiles, u64* D, unsigned long long* counter,
       unsigned long long* terms) {
+  const u32 items = tile_items[ntiles];  // device-side total of work items
   extern __shared__ __align__(16) unsigned char smem[];
   double* sS = (double*)smem;                                   // [KDE_KCUT + 1]
   double* sx = (double*)(smem + KDE_SMEM_TABLE) + (threadIdx.x >> 5) * KDE_CH;  // warp's slice
@@ -250,7 +254,9 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
   if (items == 0) return;
   u32 tps = div_up(G, KDE_TJ);
   u32 ntiles = nseg * tps;
-  SV_LAUNCH(k_kde_items, min(div_up(items, 256), 4096u), 256, 0, s)(tile_items, ntiles, items, item_tile);
+  // `items` is a host-side upper bound: grids are sized by it, the kernels stop at the
+  // device-side count tile_items[ntiles]
+  SV_LAUNCH(k_kde_items, min(div_up(items, 256), 4096u), 256, 0, s)(tile_items, ntiles, item_tile);
   cudaFuncSetAttribute(k_kde, cudaFuncAttributeMaxDynamicSharedMemorySize, KDE_SMEM_BYTES);
   int per_sm = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_kde, 32 * KDE_WARPS, KDE_SMEM_BYTES);
@@ -260,6 +266,6 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
   if (grid > need) grid = need;
   cudaMemsetAsync(work_counter, 0, 8, s);
   SV_LAUNCH(k_kde, grid, 32 * KDE_WARPS, KDE_SMEM_BYTES, s)(segs, G, tps, keys, xmask, tile_range,
-                                                            tile_items, item_tile, items, D,
+                                                            tile_items, item_tile, ntiles, D,
                                                             work_counter, terms);
 }

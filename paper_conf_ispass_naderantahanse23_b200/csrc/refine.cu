@@ -141,8 +141,10 @@ k_part_stats(const SegDev* segs, u32 nseg, const u64* T, u32 tstride, const u32*
       ib = lb_u64(keys, ia, g.end, base + b);
     }
     sh[0] = ia; sh[1] = ib;
-    ab[2 * (u64)p] = a;
-    ab[2 * (u64)p + 1] = b;
+    ab[4 * (u64)p] = a;        // value interval [a, b)
+    ab[4 * (u64)p + 1] = b;
+    ab[4 * (u64)p + 2] = ia;   // this rank's index range in the sorted keys (next round's
+    ab[4 * (u64)p + 3] = ib;   // segment range if the part stays open)
   }
   __syncthreads();
   const u64 ia = sh[0], ib = sh[1];

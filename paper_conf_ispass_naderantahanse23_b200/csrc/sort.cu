@@ -14,7 +14,7 @@
 #include "kernels.cuh"
 
 #define RS_THREADS 256
-#define RS_IPT 8
+#define RS_IPT 16
 #define RS_TILE (RS_THREADS * RS_IPT)
 #define RS_WARPS (RS_THREADS / 32)
 
@@ -220,7 +220,7 @@ __device__ __forceinline__ void st_volatile_u64(u64* p, u64 v) {
 }
 
 template <bool V>  // V: a u32 payload travels with each key
-__global__ void __launch_bounds__(RS_THREADS, 4)
+__global__ void __launch_bounds__(RS_THREADS)
 k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int shift,
           const u32* __restrict__ gbase, u64* status, u32* tile_counter, u64* __restrict__ kout,
           u32* __restrict__ vout) {
@@ -355,6 +355,9 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   }
   SV_CUDA(cudaMemcpyAsync(gbase, bases, (size_t)npass * 256 * 4, cudaMemcpyHostToDevice, s));
   size_t smem = (size_t)RS_TILE * (vals ? 8 + 4 : 8);
+  SV_CUDA(cudaFuncSetAttribute(k_os_pass<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               RS_TILE * (8 + 4)));
+  SV_CUDA(cudaFuncSetAttribute(k_os_pass<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, RS_TILE * 8));
   u64* kin = keys; u32* vin = vals; u64* kout = kalt; u32* vout = valt;
   for (int p = 0; p < npass; p++) {
     if (!active[p]) continue;

@@ -35,7 +35,7 @@ EXPORTED = [
     "sieve_strata_count", "sieve_strata_copy", "sieve_strata_stats", "sieve_strata_free",
     "sieve_segment_count", "sieve_segment_get", "sieve_predict", "sieve_last_error",
     "sieve_version", "sieve_u128_to_limbs", "sieve_limbs_to_u128", "sieve_ctx_set_timing",
-    "sieve_timing_get", "sieve_kernel_launches",
+    "sieve_timing_get", "sieve_kernel_launches", "sieve_stratify_sweep", "sieve_tier_census",
 ]
 PHASES = ["moments", "compact", "sort", "prefix", "kde", "refine", "assign", "reps", "predict"]
 
@@ -94,6 +94,8 @@ def _load():
         "sieve_ctx_set_timing": ([vp, i32], i32),
         "sieve_timing_get": ([vp, u32, P(ctypes.c_double), P(u64), P(u64)], i32),
         "sieve_kernel_launches": ([], u64),
+        "sieve_stratify_sweep": ([vp, P(Params), u32, vp, vp, vp], i32),
+        "sieve_tier_census": ([vp, u32, vp, vp, vp, vp, vp], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -318,6 +320,37 @@ def stratify(trace, params=None, stratum_of_invocation=None, **kw):
     h = ctypes.c_void_p()
     _check(_L.sieve_stratify(trace._h, ctypes.byref(p), sid_ptr, ctypes.byref(h)), "sieve_stratify")
     return Strata(h)
+
+
+def _thetas(thetas):
+    num = np.ascontiguousarray([t[0] for t in thetas], np.uint32)
+    den = np.ascontiguousarray([t[1] for t in thetas], np.uint32)
+    return num, den
+
+
+def stratify_sweep(trace, thetas, params=None, **kw):
+    """sieve_stratify_sweep: one Strata per theta (num, den), pass A computed once."""
+    p = params if params is not None else default_params(**kw)
+    num, den = _thetas(thetas)
+    hs = (ctypes.c_void_p * len(thetas))()
+    _check(_L.sieve_stratify_sweep(trace._h, ctypes.byref(p), len(thetas),
+                                   num.ctypes.data_as(ctypes.c_void_p),
+                                   den.ctypes.data_as(ctypes.c_void_p), hs), "sieve_stratify_sweep")
+    return [Strata(ctypes.c_void_p(h)) for h in hs]
+
+
+def tier_census(trace, thetas):
+    """sieve_tier_census: per theta, (kernels[3], invocations[3], instructions[3]) per tier."""
+    num, den = _thetas(thetas)
+    k = np.zeros((len(thetas), 3), np.uint64)
+    inv = np.zeros((len(thetas), 3), np.uint64)
+    ins = np.zeros((len(thetas), 3, 2), np.uint64)
+    _check(_L.sieve_tier_census(trace._h, len(thetas), num.ctypes.data_as(ctypes.c_void_p),
+                                den.ctypes.data_as(ctypes.c_void_p), k.ctypes.data_as(ctypes.c_void_p),
+                                inv.ctypes.data_as(ctypes.c_void_p), ins.ctypes.data_as(ctypes.c_void_p)),
+           "sieve_tier_census")
+    instr = [[(int(ins[i, j, 1]) << 64) | int(ins[i, j, 0]) for j in range(3)] for i in range(len(thetas))]
+    return k, inv, instr
 
 
 def predict(strata, trace, rep_cycles=None):

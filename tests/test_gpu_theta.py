@@ -1,0 +1,53 @@
+"""NEXT-1: theta studies.  sieve_stratify_sweep must equal independent
+sieve_stratify / oracle runs for every theta (it only shares pass A), and sieve_tier_census must
+equal the oracle's tiers (Fig. 2 shape)."""
+import numpy as np
+import pytest
+
+import gen
+from tests.gpu_helpers import assert_tables_equal, run_oracle
+
+pytestmark = pytest.mark.gpu
+
+THETAS = [(1, 10), (1, 5), (2, 5), (1, 2), (1, 1)]
+
+
+def _trace(name, **kw):
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr = gen.make_trace(name, **kw)
+    ctx = sieve.Ctx(device=0)
+    trace = sieve.load_trace(ctx, tr["kid"], tr["x"], num_kernels=tr["K"], cta=tr["cta"], cycles=tr["y"])
+    return tr, ctx, trace
+
+
+@pytest.mark.parametrize("name", ["C1", "C2"])
+def test_sweep_equals_oracle_per_theta(name):
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr, ctx, trace = _trace(name)
+    outs = sieve.stratify_sweep(trace, THETAS)
+    assert len(outs) == len(THETAS)
+    for th, st in zip(THETAS, outs):
+        o = run_oracle(tr, theta=th)
+        assert_tables_equal(st.table, o.strata)
+        p = sieve.predict(st, trace)
+        q = o.predict()
+        assert abs(p["predicted_cycles"] - q["predicted_cycles"]) <= 1e-9 * q["predicted_cycles"]
+
+
+def test_census_matches_oracle_tiers():
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr, ctx, trace = _trace("C2")
+    k, inv, ins = sieve.tier_census(trace, THETAS)
+    x = tr["x"].astype(object)
+    for i, th in enumerate(THETAS):
+        o = run_oracle(tr, theta=th)
+        st = o.strata
+        for t in (1, 2, 3):
+            rows = st["tier"] == t
+            assert k[i, t - 1] == len(np.unique(st["kernel_id"][rows]))
+            assert inv[i, t - 1] == int(st["count"][rows].sum())
+            W = sum((int(h) << 64) | int(l) for l, h in zip(st["instr_sum_lo"][rows], st["instr_sum_hi"][rows]))
+            assert ins[i][t - 1] == W
+    # monotone in theta: a larger threshold never moves a kernel up a tier
+    assert np.all(np.diff(k[:, 2].astype(np.int64)) <= 0)
+    assert sum(inv[0]) == len(tr["kid"])
