@@ -201,6 +201,14 @@ typedef struct {
                  trace's cycles column (SIEVE_EDOM if the trace has none). */
 int sieve_predict(sieve_strata s, sieve_trace t, const uint64_t* rep_cycles, sieve_prediction* out);
 
+/* Predict for M cycle sources at once (Fig. 9: the same
+   representatives simulated on M architectures): rep_cycles is a required HOST array
+   [M][n_strata]; out is a HOST array [M].  The predicted relative speedup of architecture b
+   over a is out[a].predicted_cycles / out[b].predicted_cycles.  measured_cycles / error /
+   speedup refer to the trace's own cycles column (NaN without one). */
+int sieve_predict_multi(sieve_strata s, sieve_trace t, uint32_t M, const uint64_t* rep_cycles,
+                        sieve_prediction* out);
+
 /* ---- measurement ------------------------------------------------------------------------ */
 /* Per-phase device time of the calls made on this context, taken with CUDA events recorded on
    the context's stream around each phase (off by default; enabling resets the counters).

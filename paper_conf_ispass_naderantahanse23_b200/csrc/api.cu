@@ -726,8 +726,13 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       DBuf<char> item_tile(c);
       SV_TRY(item_tile.alloc(kde_item_bytes(items)));
       PhaseTimer tm(c, SIEVE_PHASE_KDE, 0);
+      // the unguarded KDE variant needs |z| < 9645 for every evaluated pair: window 8.7 h plus
+      // KDE_TJ - 1 grid steps, so max Delta / h < 300 suffices (true for realistic segments)
+      bool guard = false;
+      for (u32 s = 0; s < nseg; s++)
+        if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 300.0 * hs[s].h) guard = true;
       launch_kde(segs.get(), nseg, G, keys.get(), xmask, tile_range.get(), tile_items.get(),
-                 (u32*)item_tile.get(), items, D.get(), counter.get() + 1, terms.get(), S);
+                 (u32*)item_tile.get(), items, D.get(), counter.get() + 1, terms.get(), guard, S);
       tm.stop();
       SV_CUDA(cudaGetLastError());
     }
@@ -1128,45 +1133,66 @@ extern "C" int sieve_segment_get(sieve_strata s, uint64_t idx, sieve_segment* ou
 // ------------------------------------------------------------------------------------------
 static double u128_to_double_host(u128 v) { return (double)v; }  // libgcc: correctly rounded
 
-extern "C" int sieve_predict(sieve_strata s, sieve_trace t, const uint64_t* rep_cycles, sieve_prediction* out) {
+// M predictions at once: rep_cycles is [M][n_strata] (nullable iff M == 1: the trace's cycles)
+static int predict_impl(sieve_strata s, sieve_trace t, u32 M, const uint64_t* rep_cycles,
+                        sieve_prediction* out) {
   if (!strata_ok(s) || !trace_ok(t) || !out) return sv_fail(SIEVE_EINVAL, "bad handle");
-  if (!rep_cycles && !s->has_cycles) return sv_fail(SIEVE_EDOM, "no cycle source for the representatives");
+  if (!rep_cycles && (M != 1 || !s->has_cycles))
+    return sv_fail(SIEVE_EDOM, "no cycle source for the representatives");
   sieve_ctx c = t->ctx;
   SV_CUDA(cudaSetDevice(c->device));
   const u32 ns = (u32)s->st.size();
   SV_TRY(arena_reset(c));
-  std::vector<u64> hW(2 * (size_t)ns), hx(ns), hy(ns);
+  std::vector<u64> hW(2 * (size_t)ns), hx(ns), hy((size_t)M * ns);
   for (u32 i = 0; i < ns; i++) {
     hW[2 * i] = s->st[i].instr_sum_lo;
     hW[2 * i + 1] = s->st[i].instr_sum_hi;
     hx[i] = s->st[i].rep_instr;
-    hy[i] = rep_cycles ? rep_cycles[i] : s->st[i].rep_cycles;
   }
+  for (u32 m = 0; m < M; m++)
+    for (u32 i = 0; i < ns; i++)
+      hy[(size_t)m * ns + i] = rep_cycles ? rep_cycles[(size_t)m * ns + i] : s->st[i].rep_cycles;
   DBuf<u64> dW(c), dx(c), dy(c);
   DBuf<double> dout(c);
-  SV_TRY(dW.alloc(hW.size())); SV_TRY(dx.alloc(ns)); SV_TRY(dy.alloc(ns)); SV_TRY(dout.alloc(4));
+  SV_TRY(dW.alloc(hW.size())); SV_TRY(dx.alloc(ns)); SV_TRY(dy.alloc(hy.size()));
+  SV_TRY(dout.alloc(4 * (size_t)M));
   SV_TRY(h2d(c, dW.get(), hW)); SV_TRY(h2d(c, dx.get(), hx)); SV_TRY(h2d(c, dy.get(), hy));
   PhaseTimer tpr(c, SIEVE_PHASE_PREDICT, 0);
-  launch_predict(dW.get(), dx.get(), dy.get(), ns, dout.get(), c->stream);
+  launch_predict(dW.get(), dx.get(), dy.get(), ns, M, dout.get(), c->stream);
   tpr.stop();
   SV_CUDA(cudaGetLastError());
   std::vector<double> r;
-  SV_TRY(d2h(c, r, dout.get(), 4));
+  SV_TRY(d2h(c, r, dout.get(), 4 * (size_t)M));
   SV_TRY(sync(c));
   resolve_timing(c);
-  out->predicted_cycles = r[0];
-  out->predicted_ipc = r[3];
-  out->total_instr_lo = (u64)s->total_instr;
-  out->total_instr_hi = (u64)(s->total_instr >> 64);
-  if (s->has_cycles) {
-    double cm = u128_to_double_host(s->c_meas);
-    out->measured_cycles = cm;
-    out->error = s->c_meas == 0 ? NAN : fabs(r[0] - cm) / cm;
-    out->speedup = cm / r[1];
-  } else {
-    out->measured_cycles = NAN;
-    out->error = NAN;
-    out->speedup = NAN;
+  for (u32 m = 0; m < M; m++) {
+    const double* rm = &r[4 * (size_t)m];
+    sieve_prediction& o = out[m];
+    o.predicted_cycles = rm[0];
+    o.predicted_ipc = rm[3];
+    o.total_instr_lo = (u64)s->total_instr;
+    o.total_instr_hi = (u64)(s->total_instr >> 64);
+    if (s->has_cycles) {
+      double cm = u128_to_double_host(s->c_meas);
+      o.measured_cycles = cm;
+      o.error = s->c_meas == 0 ? NAN : fabs(rm[0] - cm) / cm;
+      o.speedup = cm / rm[1];
+    } else {
+      o.measured_cycles = NAN;
+      o.error = NAN;
+      o.speedup = NAN;
+    }
   }
   return SIEVE_OK;
+}
+
+extern "C" int sieve_predict(sieve_strata s, sieve_trace t, const uint64_t* rep_cycles, sieve_prediction* out) {
+  return predict_impl(s, t, 1, rep_cycles, out);
+}
+
+extern "C" int sieve_predict_multi(sieve_strata s, sieve_trace t, uint32_t M, const uint64_t* rep_cycles,
+                                   sieve_prediction* out) {
+  if (M == 0) return SIEVE_OK;
+  if (!rep_cycles) return sv_fail(SIEVE_EINVAL, "rep_cycles [M][n_strata] is required");
+  return predict_impl(s, t, M, rep_cycles, out);
 }

@@ -62,7 +62,7 @@ struct SegDev {
   double h, inv_h;
   u64 begin, end; // local index range in the sorted keys (filled on device)
 };
-#define KDE_TJ 32       // grid points per tile (one lane each; a work item is one warp's)
+#define KDE_TJ 32       // grid points per tile (a work item is one warp's: one point per lane)
 #define KDE_CH 256      // values per work item chunk (staged in the warp's shared memory)
 struct KdeScratch {
   u64* tile_range;     // [nseg*tiles][2]
@@ -78,7 +78,7 @@ size_t kde_item_bytes(u32 items);
 void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
                 const u64* tile_range, const u32* tile_items, u32* item_tile, u32 items,
                 u64* D /* [nseg][G][2] */, unsigned long long* work_counter,
-                unsigned long long* terms, cudaStream_t s);
+                unsigned long long* terms, bool guard, cudaStream_t s);
 
 // ---------------- valleys and thresholds (A11-A13) ---------------------------------------------
 // T[s*tstride + q], nt[s], kind[s] (1 = valley, 2 = bisect)
@@ -124,7 +124,8 @@ void launch_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, co
 // ---------------- prediction ----------------------------------------------
 // strata: W (lo,hi), rep x, rep y ; out[0] = C_pred, out[1] = sum y_rep, out[2] = I (double),
 // out[3] = IPC
-void launch_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, double* out,
+// ry: [M][nstrata] (one cycle vector per architecture); out: [M][4]
+void launch_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, u32 M, double* out,
                     cudaStream_t s);
 
 // ---------------- misc -------------------------------------------------------------------------

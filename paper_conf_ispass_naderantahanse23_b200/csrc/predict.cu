@@ -35,6 +35,9 @@ __global__ void __launch_bounds__(PR_THREADS)
 k_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, double* out) {
   __shared__ DD s_c[PR_THREADS], s_i[PR_THREADS];
   __shared__ DD s_y[PR_THREADS];
+  // block m predicts for the m-th cycle vector (one architecture each)
+  ry += (u64)blockIdx.x * nstrata;
+  out += 4 * (u64)blockIdx.x;
   DD c = {0.0, 0.0}, I = {0.0, 0.0}, Y = {0.0, 0.0};
   for (u32 s = threadIdx.x; s < nstrata; s += PR_THREADS) {
     double w = u128_to_double(W[2 * (u64)s], W[2 * (u64)s + 1]);
@@ -66,7 +69,8 @@ k_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, double* out) 
   }
 }
 
-void launch_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, double* out,
+// ry: [M][nstrata]; out: [M][4]
+void launch_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, u32 M, double* out,
                     cudaStream_t s) {
-  SV_LAUNCH(k_predict, 1, PR_THREADS, 0, s)(W, rx, ry, nstrata, out);
+  if (M) SV_LAUNCH(k_predict, M, PR_THREADS, 0, s)(W, rx, ry, nstrata, out);
 }

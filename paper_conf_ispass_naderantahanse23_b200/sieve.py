@@ -36,6 +36,7 @@ EXPORTED = [
     "sieve_segment_count", "sieve_segment_get", "sieve_predict", "sieve_last_error",
     "sieve_version", "sieve_u128_to_limbs", "sieve_limbs_to_u128", "sieve_ctx_set_timing",
     "sieve_timing_get", "sieve_kernel_launches", "sieve_stratify_sweep", "sieve_tier_census",
+    "sieve_predict_multi",
 ]
 PHASES = ["moments", "compact", "sort", "prefix", "kde", "refine", "assign", "reps", "predict"]
 
@@ -96,6 +97,7 @@ def _load():
         "sieve_kernel_launches": ([], u64),
         "sieve_stratify_sweep": ([vp, P(Params), u32, vp, vp, vp], i32),
         "sieve_tier_census": ([vp, u32, vp, vp, vp, vp, vp], i32),
+        "sieve_predict_multi": ([vp, vp, u32, vp, P(_Prediction)], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -351,6 +353,23 @@ def tier_census(trace, thetas):
            "sieve_tier_census")
     instr = [[(int(ins[i, j, 1]) << 64) | int(ins[i, j, 0]) for j in range(3)] for i in range(len(thetas))]
     return k, inv, instr
+
+
+def _pred_dict(out):
+    return {"predicted_cycles": out.predicted_cycles, "predicted_ipc": out.predicted_ipc,
+            "measured_cycles": out.measured_cycles, "error": out.error, "speedup": out.speedup,
+            "total_instr": (out.total_instr_hi << 64) | out.total_instr_lo}
+
+
+def predict_multi(strata, trace, rep_cycles):
+    """sieve_predict_multi: rep_cycles [M][n_strata] (one row per architecture) -> M dicts."""
+    rc = np.ascontiguousarray(rep_cycles, np.uint64)
+    if rc.ndim != 2 or rc.shape[1] != len(strata):
+        raise ValueError("rep_cycles must be [M][n_strata]")
+    outs = (_Prediction * rc.shape[0])()
+    _check(_L.sieve_predict_multi(strata._h, trace._h, rc.shape[0], rc.ctypes.data_as(ctypes.c_void_p),
+                                  outs), "sieve_predict_multi")
+    return [_pred_dict(o) for o in outs]
 
 
 def predict(strata, trace, rep_cycles=None):

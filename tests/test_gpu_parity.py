@@ -146,6 +146,22 @@ def test_edge_cases():
     assert e.value.code == -7
 
 
+@pytest.mark.parametrize("G", [3, 5, 1024])
+def test_kde_guarded_variant(G):
+    # a huge outlier makes grid steps >> h at small G, so the KDE must take its guarded path
+    # (u >= 80 sent to the zero entry explicitly); results must not change
+    n = 50_000
+    x = np.full(n, 1000, np.uint64)
+    x[::997] = 1000 + np.arange(len(x[::997]), dtype=np.uint64) * 3
+    x[-1] = 10 ** 12
+    tr = {"kid": np.zeros(n, np.uint32), "x": x, "cta": np.full(n, 128, np.uint32),
+          "y": x * 2, "K": 1}
+    g = run_gpu(tr, G=G, keep_debug=True)
+    o = run_oracle(tr, G=G, keep_debug=True)
+    assert_tables_equal(g["table"], o.strata)
+    assert_segments_equal(g["segments"], o.segments())
+
+
 def test_many_kernels_multiple_smem_passes():
     # K > 2048 makes pass A run several kernel-id ranges
     rng = np.random.default_rng(3)

@@ -51,3 +51,23 @@ def test_census_matches_oracle_tiers():
     # monotone in theta: a larger threshold never moves a kernel up a tier
     assert np.all(np.diff(k[:, 2].astype(np.int64)) <= 0)
     assert sum(inv[0]) == len(tr["kid"])
+
+
+def test_predict_multi_architecture():
+    """NEXT-2 (Fig. 9): the same representatives with M cycle vectors."""
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr, ctx, trace = _trace("C2")
+    st = sieve.stratify(trace)
+    o = run_oracle(tr)
+    ns = len(st)
+    rng = np.random.default_rng(0)
+    base = st.table["rep_cycles"].astype(np.uint64)
+    rc = np.stack([base, base * 2, rng.integers(1, 1 << 40, ns).astype(np.uint64)])
+    preds = sieve.predict_multi(st, trace, rc)
+    for m in range(3):
+        q = o.predict(rc[m])
+        assert abs(preds[m]["predicted_cycles"] - q["predicted_cycles"]) <= 1e-9 * q["predicted_cycles"]
+    # doubling every representative's cycles doubles the prediction (relative speedup 2)
+    assert abs(preds[1]["predicted_cycles"] / preds[0]["predicted_cycles"] - 2.0) < 1e-12
+    single = sieve.predict(st, trace)
+    assert preds[0]["predicted_cycles"] == single["predicted_cycles"]
