@@ -89,6 +89,12 @@ struct sieve_ctx_s {
   char* arena = nullptr;
   size_t arena_cap = 0, arena_off = 0, arena_hw = 0;
   std::vector<void*> overflow;
+  // the same scheme in pinned host memory for the orchestrator's staged copies
+  char* pin = nullptr;
+  size_t pin_cap = 0, pin_off = 0, pin_hw = 0;
+  std::vector<void*> pin_overflow;
+  struct Pend { void* dst; void* pinned; size_t bytes; };
+  std::vector<Pend> pend;
 };
 
 static std::atomic<unsigned long long> g_launches{0};
@@ -201,7 +207,35 @@ static void dfree(sieve_ctx c, void* p) {
   else cudaFreeAsync(p, c->stream);
 }
 
+static int pin_alloc(sieve_ctx c, void** p, size_t bytes) {
+  bytes = (bytes + 255) / 256 * 256;
+  if (bytes == 0) bytes = 256;
+  size_t off = c->pin_off;
+  c->pin_off += bytes;
+  if (c->pin_off > c->pin_hw) c->pin_hw = c->pin_off;
+  if (c->pin_off <= c->pin_cap) { *p = c->pin + off; return SIEVE_OK; }
+  SV_CUDA(cudaHostAlloc(p, bytes, cudaHostAllocDefault));
+  c->pin_overflow.push_back(*p);
+  return SIEVE_OK;
+}
+
 static int arena_reset(sieve_ctx c) {
+  // pinned staging: every copy of the previous call completed before it returned
+  c->pend.clear();
+  for (void* p : c->pin_overflow) cudaFreeHost(p);
+  c->pin_overflow.clear();
+  if (c->pin_hw > c->pin_cap) {
+    if (c->pin) cudaFreeHost(c->pin);
+    c->pin = nullptr;
+    c->pin_cap = 0;
+    size_t want = c->pin_hw + c->pin_hw / 4 + 4096;
+    void* p;
+    SV_CUDA(cudaHostAlloc(&p, want, cudaHostAllocDefault));
+    c->pin = (char*)p;
+    c->pin_cap = want;
+  }
+  c->pin_off = 0;
+  c->pin_hw = 0;
   for (void* p : c->overflow) dfree(c, p);
   c->overflow.clear();
   if (c->arena_hw > c->arena_cap) {
@@ -321,6 +355,8 @@ extern "C" void sieve_ctx_destroy(sieve_ctx ctx) {
   for (void* p : ctx->overflow) dfree(ctx, p);
   if (ctx->arena) dfree(ctx, ctx->arena);
   cudaStreamSynchronize(ctx->stream);
+  for (void* p : ctx->pin_overflow) cudaFreeHost(p);
+  if (ctx->pin) cudaFreeHost(ctx->pin);
   delete ctx->comm;
   ctx->magic = 0;
   delete ctx;
@@ -472,18 +508,38 @@ static int allreduce(sieve_ctx c, u64* buf, size_t n, ReduceOp op) {
   return c->comm->allreduce(buf, n, op, c->stream);
 }
 
+// Host <-> device copies of the orchestrator go through a per-call PINNED staging arena: a
+// copy to or from pageable memory would make cudaMemcpyAsync synchronise the stream (H2D) or
+// block the host until the copy ran (D2H).  d2h only queues the copy; the data lands in the
+// vector at the next sync(c), so several read-backs share one synchronisation.
+static int d2h_raw(sieve_ctx c, void* dst, const void* d, size_t bytes) {
+  if (!bytes) return SIEVE_OK;
+  void* p;
+  SV_TRY(pin_alloc(c, &p, bytes));
+  SV_CUDA(cudaMemcpyAsync(p, d, bytes, cudaMemcpyDeviceToHost, c->stream));
+  c->pend.push_back({dst, p, bytes});
+  return SIEVE_OK;
+}
 template <typename T>
 static int d2h(sieve_ctx c, std::vector<T>& h, const T* d, size_t n) {
   h.resize(n);
-  if (n) SV_CUDA(cudaMemcpyAsync(h.data(), d, n * sizeof(T), cudaMemcpyDeviceToHost, c->stream));
-  return SIEVE_OK;
+  return d2h_raw(c, h.data(), d, n * sizeof(T));
 }
 template <typename T>
 static int h2d(sieve_ctx c, T* d, const std::vector<T>& h) {
-  if (!h.empty()) SV_CUDA(cudaMemcpyAsync(d, h.data(), h.size() * sizeof(T), cudaMemcpyHostToDevice, c->stream));
+  if (h.empty()) return SIEVE_OK;
+  void* p;
+  SV_TRY(pin_alloc(c, &p, h.size() * sizeof(T)));
+  memcpy(p, h.data(), h.size() * sizeof(T));
+  SV_CUDA(cudaMemcpyAsync(d, p, h.size() * sizeof(T), cudaMemcpyHostToDevice, c->stream));
   return SIEVE_OK;
 }
-static int sync(sieve_ctx c) { SV_CUDA(cudaStreamSynchronize(c->stream)); return SIEVE_OK; }
+static int sync(sieve_ctx c) {
+  SV_CUDA(cudaStreamSynchronize(c->stream));
+  for (auto& q : c->pend) memcpy(q.dst, q.pinned, q.bytes);
+  c->pend.clear();
+  return SIEVE_OK;
+}
 
 // ------------------------------------------------------------------------------------------
 // sieve_stratify
@@ -662,7 +718,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       SV_TRY(tmp.alloc(radix_sort_temp_bytes(n3_local, false)));
       PhaseTimer tm(c, SIEVE_PHASE_SORT, 0);
       int passes = 0;
-      SV_TRY(radix_sort(keys.get(), nullptr, n3_local, nbits, tmp.get(), S, &passes));
+      void* pinned;
+      SV_TRY(pin_alloc(c, &pinned, RADIX_PINNED_BYTES));
+      SV_TRY(radix_sort(keys.get(), nullptr, n3_local, nbits, tmp.get(), S, pinned, &passes));
       if (c->timing) c->acc[SIEVE_PHASE_SORT].work += (u64)passes * n3_local * 16;
     }
     SV_TRY(Pb.alloc(4 * block_prefix_entries(n3_local)));
@@ -821,13 +879,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     hc.mark("round");
   }
   R->rounds = round;
-  {
-    std::vector<unsigned long long> ht;
-    SV_TRY(d2h(c, ht, terms.get(), 1));
-    SV_TRY(sync(c));
-    R->kde_terms = ht[0];
-    if (c->timing) c->acc[SIEVE_PHASE_KDE].work += ht[0];
-  }
+  // the KDE term count is read back with the representatives at the end (no extra sync)
+  std::vector<unsigned long long> h_terms;
+  SV_TRY(d2h(c, h_terms, terms.get(), 1));
   Pb.release(); keys.release();
 
   // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
@@ -885,13 +939,15 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(d2h(c, hcnt, counter.get(), 1));
     SV_TRY(sync(c));
     // the retry decision must be identical on every rank
-    DBuf<u64> fl(c);
-    SV_TRY(fl.alloc(1));
-    SV_TRY(h2d(c, fl.get(), std::vector<u64>{hflag[2]}));
-    SV_TRY(allreduce(c, fl.get(), 1, RED_MAX));
-    std::vector<u64> gfl;
-    SV_TRY(d2h(c, gfl, fl.get(), 1));
-    SV_TRY(sync(c));
+    std::vector<u64> gfl{hflag[2]};
+    if (c->comm) {
+      DBuf<u64> fl(c);
+      SV_TRY(fl.alloc(1));
+      SV_TRY(h2d(c, fl.get(), gfl));
+      SV_TRY(allreduce(c, fl.get(), 1, RED_MAX));
+      SV_TRY(d2h(c, gfl, fl.get(), 1));
+      SV_TRY(sync(c));
+    }
     if (!gfl[0]) { E = hcnt[0]; break; }
     if (attempt > 6) return sv_fail(SIEVE_ENOMEM, "(stratum, CTA) table kept overflowing");
     cap <<= 2;
@@ -941,7 +997,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   {
     DBuf<char> tmp(c);
     SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
-    SV_TRY(radix_sort(sk.get(), idx.get(), Etot, 32 + (int)bitlen(ns ? ns - 1 : 0), tmp.get(), S));
+    void* pinned;
+    SV_TRY(pin_alloc(c, &pinned, RADIX_PINNED_BYTES));
+    SV_TRY(radix_sort(sk.get(), idx.get(), Etot, 32 + (int)bitlen(ns ? ns - 1 : 0), tmp.get(), S, pinned));
   }
   launch_gather_u64(ak.get() + Etot, idx.get(), Etot, scnt.get(), S);
   launch_gather_u64(ak.get() + 2 * Etot, idx.get(), Etot, sfirst.get(), S);
@@ -961,6 +1019,8 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   SV_TRY(d2h(c, h_xy, repxy.get(), 2 * (size_t)ns));
   SV_TRY(sync(c));
   resolve_timing(c);
+  R->kde_terms = h_terms[0];
+  if (c->timing) c->acc[SIEVE_PHASE_KDE].work += h_terms[0];
   hc.mark("reps");
 
   // ---------------- assemble --------------------------------------------------------------------

@@ -15,12 +15,16 @@
 // number of ranks or blocks.
 #include "kernels.cuh"
 
-#define AS_THREADS 512
+#define AS_THREADS 1024
 #define AS_IPT 4
-#define AS_HC 4096          // shared hash capacity (entries)
+#define AS_HC 8192          // shared hash capacity (entries): 128 KB, one block per SM
+#define AS_FLUSH (3 * AS_HC / 4)      // flush to the L2 table when this full
 #define AS_MAXP 32          // probes before falling back to the global table
 
-int assign_grid() { return 2 * sv_num_sms(); }
+// One block per SM with a large table: a block's contiguous chunk sees nearly every (stratum,
+// CTA) pair of the trace (thousands), so a small table would flush -- i.e. issue contended L2
+// atomics on the same hot keys from every block -- many times per block.
+int assign_grid() { return sv_num_sms(); }
 
 __device__ __forceinline__ u32 hash_key(u64 k) {
   return (u32)((k * 0x9E3779B97F4A7C15ull) >> 32);
@@ -115,7 +119,7 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
     }
     __syncthreads();
     bool last = base + tile >= b1;
-    if (s_fill > AS_HC / 2 || last) {
+    if (s_fill > AS_FLUSH || last) {  // rows that find no slot go to the L2 table directly
       for (u32 e = threadIdx.x; e < AS_HC; e += AS_THREADS) {
         u64 key = hk[e];
         if (key != HASH_EMPTY) {

@@ -43,7 +43,9 @@ void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u
 // ---------------- LSD radix sort (u64 keys, optional u32 payload) ----------------------------
 size_t radix_sort_temp_bytes(u64 n, bool with_vals);
 // sorts keys[0..n) on bits [0, nbits); result in keys/vals (in place via internal ping-pong)
-int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s,
+// pinned: >= RADIX_PINNED_BYTES of pinned host memory for the one histogram read-back
+#define RADIX_PINNED_BYTES (2 * 8 * 256 * 4)
+int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, void* pinned,
                int* passes = nullptr);
 
 // ---------------- prefix sums of x and x^2 over sorted Tier-3 keys -----------------------------

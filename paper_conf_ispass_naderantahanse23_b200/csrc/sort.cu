@@ -320,7 +320,8 @@ size_t radix_sort_temp_bytes(u64 n, bool with_vals) {
   return b;
 }
 
-int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, int* passes) {
+int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, void* pinned,
+               int* passes) {
   if (passes) *passes = 0;
   if (n <= 1 || nbits <= 0) return SIEVE_OK;
   if (nbits > 8 * OS_MAX_PASSES) nbits = 8 * OS_MAX_PASSES;
@@ -339,10 +340,11 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   SV_CUDA(cudaFuncSetAttribute(k_os_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsmem));
   u64 hgrid = std::min<u64>((n + RS_THREADS - 1) / RS_THREADS, (u64)sv_num_sms() * 4);
   SV_LAUNCH(k_os_hist, (unsigned)hgrid, RS_THREADS, hsmem, s)(keys, n, npass, ghist);
-  u32 h[OS_MAX_PASSES * 256];
+  // pinned staging: a pageable copy would block on / synchronise the stream differently
+  u32* h = (u32*)pinned;
+  u32* bases = h + OS_MAX_PASSES * 256;
   SV_CUDA(cudaMemcpyAsync(h, ghist, (size_t)npass * 256 * 4, cudaMemcpyDeviceToHost, s));
   SV_CUDA(cudaStreamSynchronize(s));
-  u32 bases[OS_MAX_PASSES * 256];
   bool active[OS_MAX_PASSES];
   for (int p = 0; p < npass; p++) {
     u32 run = 0, nonzero = 0;
