@@ -229,6 +229,7 @@ def main():
     for _ in range(args.warmup):
         st = step()
     n_strata = len(st)
+    st_terms, kde_eval = st.kde_terms, st.kde_evaluated
     rounds = st.rounds
 
     # ---- device-timed steps (trace resident in HBM; 2.4 GB of columns >> 126 MB L2) ----
@@ -307,7 +308,8 @@ def main():
                 "traffic": traffic, "share_of_step": kde_ms / ms,
                 "peak_source": f"{nsm} SMs x {FP64_LANES_PER_SM} FP64 lanes x sm_max_mhz "
                                f"{peaks.get('sm_max_mhz')} ({peak_src} MEASURED_PEAKS.json)",
-                "work": f"{kde_terms / args.steps:.4g} in-window terms/step x {KDE_FP64_OPS_PER_TERM} FP64 ops"}
+                "work": f"{kde_terms / args.steps:.4g} in-window terms/step x {KDE_FP64_OPS_PER_TERM} FP64 ops",
+                "evaluated_per_in_window": kde_eval / max(1, st_terms)}
     hbm = peaks.get("hbm_gbs", 6650.0)
     phase_out = {}
     for name, (pms, calls, work) in phases.items():

@@ -73,8 +73,9 @@ typedef void (*sieve_free_fn)(void* p, void* stream, void* user);
 int sieve_get_unique_id(uint8_t out[128]);
 
 /* Create a context on CUDA device `cuda_device` using stream `cuda_stream` (a cudaStream_t,
-   NULL = the legacy default stream).  world == 1: no communicator (nccl_id must be NULL).
-   world > 1: ncclCommInitRank(world, *nccl_id, rank) -- one process (or thread) per GPU. */
+   NULL = the legacy default stream).  world > 1: ncclCommInitRank(world, *nccl_id, rank) --
+   one process per GPU.  world == 1: no communicator if nccl_id is NULL; with an id, a one-rank
+   NCCL communicator (the multi-rank code path on a single GPU, for testing). */
 int sieve_ctx_create(int cuda_device, void* cuda_stream, int rank, int world,
                      const uint8_t* nccl_id, sieve_ctx* out);
 
@@ -152,7 +153,10 @@ int sieve_strata_count(sieve_strata s, uint64_t* n);
 /* copy min(cap, count) strata to a HOST array */
 int sieve_strata_copy(sieve_strata s, sieve_stratum* host_out, uint64_t cap);
 /* refinement rounds used, KDE terms evaluated (diagnostics) */
-int sieve_strata_stats(sieve_strata s, uint32_t* rounds, uint64_t* kde_terms);
+/* rounds: refinement rounds; kde_terms: in-window (|g - x| <= sqrt(74) h) KDE terms;
+   kde_evaluated: (grid point, value) pairs the KDE kernel evaluated (in-window + wasted) */
+int sieve_strata_stats(sieve_strata s, uint32_t* rounds, uint64_t* kde_terms,
+                       uint64_t* kde_evaluated);
 void sieve_strata_free(sieve_strata s);
 
 /* ---- theta studies (Fig. 2, Fig. 10) -------------------- */
@@ -230,6 +234,16 @@ int sieve_ctx_set_timing(sieve_ctx ctx, int enable);
 int sieve_timing_get(sieve_ctx ctx, uint32_t phase, double* ms, uint64_t* calls, uint64_t* work);
 /* number of kernels this process has launched through the library (all contexts) */
 uint64_t sieve_kernel_launches(void);
+
+/* ---- within-stratum cycle variability (Fig. 4; NEXT-2) ---------------------- */
+/* For every stratum, the coefficient of variation of its members' cycle counts,
+   cov_s = sigma_pop(y) / mean(y) = sqrt(n S2 - S1^2) / S1 from exact integer sums (0 if S1 = 0),
+   and their average weighted by the strata's instruction weights W_s / I (reading A25).
+     sid       DEVICE [n_local] u32: stratum_of_invocation from sieve_stratify on this trace
+     cov       nullable HOST [n_strata]; weighted: nullable HOST scalar
+   SIEVE_EDOM without a cycles column; SIEVE_ERANGE if a cycle count is >= 2^48.
+   Collective if world > 1. */
+int sieve_cycle_cov(sieve_strata s, sieve_trace t, const uint32_t* sid, double* cov, double* weighted);
 
 /* ---- misc ----------------------------------------------------------------------------------- */
 const char* sieve_last_error(void); /* thread-local; valid until the next call on this thread */

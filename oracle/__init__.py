@@ -59,6 +59,8 @@ def _lib():
         L.oracle_det_exp.restype = dbl
         L.oracle_q.argtypes = [dbl]
         L.oracle_q.restype = u64
+        L.oracle_cycle_cov.argtypes = [vp, vp, vp, ctypes.POINTER(dbl)]
+        L.oracle_cycle_cov.restype = ctypes.c_int
         L.oracle_exp2_table.argtypes = [ctypes.c_int]
         L.oracle_exp2_table.restype = dbl
         L.oracle_tier.argtypes = [u64, u64, u64, u64, u64, u64, u64, u32, u32]
@@ -138,6 +140,16 @@ class Result:
                         "count": int(m3[2]), "bandwidth": h.value, "d_lo": dlo, "d_hi": dhi,
                         "cuts": cuts})
         return out
+
+    def cycle_cov(self, cycles):
+        """Per-stratum CoV of the members' cycles and its instruction-weighted mean (Fig. 4)."""
+        cyc = np.ascontiguousarray(cycles, np.uint64)
+        cov = np.zeros(len(self.strata), np.float64)
+        w = ctypes.c_double()
+        rc = _lib().oracle_cycle_cov(self._h, _p(cyc), _p(cov), ctypes.byref(w))
+        if rc != 0:
+            raise OracleError(rc)
+        return cov, w.value
 
     def predict(self, rep_cycles=None):
         pr = _Pred()

@@ -654,6 +654,54 @@ int oracle_predict(const oracle_result* R, const uint64_t* rep_cycles, oracle_pr
   return OR_OK;
 }
 
+/* ------------------------------------------------------------------------------------------
+ * Within-stratum cycle variability (Fig. 4): per stratum, the coefficient of
+ * variation of the members' cycle counts, cov_s = sigma_pop(y) / mu(y) = sqrt(n S2 - S1^2) / S1
+ * (exact integers, one rounding each for the root argument, the root and the division;
+ * 0 if S1 == 0), and the average weighted by the strata's instruction weights w_s = W_s / I
+ * (reading A25: the paper says "(weighted) average" without naming the weights; Sieve's own
+ * weights are the natural choice).  Cycles must be < 2^48.
+ * ------------------------------------------------------------------------------------------ */
+int oracle_cycle_cov(const oracle_result* R, const uint64_t* cycles, double* cov, double* weighted) {
+  uint64_t ns = R->n_strata;
+  uint64_t* cnt = (uint64_t*)calloc(ns ? ns : 1, sizeof(uint64_t));
+  u128* s1 = (u128*)calloc(ns ? ns : 1, sizeof(u128));
+  u256* s2 = (u256*)calloc(ns ? ns : 1, sizeof(u256));
+  for (uint64_t i = 0; i < R->n; i++) {
+    uint32_t s = R->sid[i];
+    uint64_t y = cycles[i];
+    if (y >= ((uint64_t)1 << 48)) { free(cnt); free(s1); free(s2); return OR_ERANGE; }
+    cnt[s]++;
+    s1[s] += y;
+    u256 q = u256_mul128((u128)y, (u128)y);
+    u128 lo = ((u128)s2[s].w[1] << 64) | s2[s].w[0];
+    u128 sum = lo + (((u128)q.w[1] << 64) | q.w[0]);
+    u128 carry = sum < lo ? 1 : 0;
+    s2[s].w[0] = (uint64_t)sum; s2[s].w[1] = (uint64_t)(sum >> 64);
+    u128 hi = ((u128)s2[s].w[3] << 64) | s2[s].w[2];
+    hi += carry + (((u128)q.w[3] << 64) | q.w[2]);
+    s2[s].w[2] = (uint64_t)hi; s2[s].w[3] = (uint64_t)(hi >> 64);
+  }
+  __float128 acc = 0, I = 0;
+  for (uint64_t s = 0; s < ns; s++) {
+    double c = 0.0;
+    if (s1[s] != 0) {
+      /* n S2 - S1^2 with n < 2^36 and S2 < 2^132: compute n * S2 limb by limb */
+      u256 nS2 = u256_mul_u64(s2[s], cnt[s]);
+      u256 d = u256_sub(nS2, u256_mul128(s1[s], s1[s]));
+      c = sqrt(u256_to_double(d)) / (double)s1[s];
+    }
+    if (cov) cov[s] = c;
+    const oracle_stratum* o = &R->strata[s];
+    __float128 W = (__float128)(((u128)o->instr_sum_hi << 64) | o->instr_sum_lo);
+    acc += W * c;
+    I += W;
+  }
+  if (weighted) *weighted = ns ? (double)(acc / I) : 0.0;
+  free(cnt); free(s1); free(s2);
+  return OR_OK;
+}
+
 /* accessors */
 uint64_t oracle_strata_count(const oracle_result* R) { return R->n_strata; }
 void oracle_strata_copy(const oracle_result* R, oracle_stratum* dst) {

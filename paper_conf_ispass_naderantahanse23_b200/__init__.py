@@ -4,7 +4,7 @@ See include/sieve.h for the C-ABI and DESIGN.md for the design.  The binding onl
 arguments; every step of the path runs in the library's sm_100a kernels.
 """
 from .sieve import (ADOPT, EXPORTED, LIB_PATH, MEM_DEVICE, MEM_HOST, PHASES, STRATUM_DTYPE, Ctx,
-                    Group, Params, SieveError, Strata, Trace, default_params, get_unique_id,
+                    Group, Params, SieveError, Strata, Trace, cycle_cov, default_params, get_unique_id,
                     kernel_launches, limbs_to_u128, load_trace, predict, predict_multi, stratify,
                     stratify_sweep, tier_census, u128_to_limbs, version)
 from . import distributed  # noqa: F401

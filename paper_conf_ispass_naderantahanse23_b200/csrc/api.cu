@@ -180,7 +180,7 @@ struct sieve_strata_s {
   bool keep_debug = false;
   u32 G = 0;
   u32 rounds = 0;
-  u64 kde_terms = 0;
+  u64 kde_terms = 0, kde_evaluated = 0;
   u128 total_instr = 0, c_meas = 0;
   bool has_cycles = false;
 };
@@ -316,12 +316,12 @@ static int ctx_common(int dev, void* stream, sieve_ctx* out, sieve_ctx_s** c) {
 extern "C" int sieve_ctx_create(int cuda_device, void* cuda_stream, int rank, int world,
                                 const uint8_t* nccl_id, sieve_ctx* out) {
   if (world < 1 || rank < 0 || rank >= world) return sv_fail(SIEVE_EINVAL, "bad rank/world");
-  if ((world == 1) != (nccl_id == nullptr)) return sv_fail(SIEVE_EINVAL, "nccl_id must be NULL iff world == 1");
+  if (world > 1 && nccl_id == nullptr) return sv_fail(SIEVE_EINVAL, "world > 1 needs an nccl_id");
   sieve_ctx_s* c;
   SV_TRY(ctx_common(cuda_device, cuda_stream, out, &c));
   c->rank = rank;
   c->world = world;
-  if (world > 1) {
+  if (nccl_id) {  // world == 1 with an id: a one-rank NCCL communicator (exercises the NCCL path)
     int st = nccl_comm_create(rank, world, nccl_id, &c->comm);
     if (st != SIEVE_OK) { delete c; return st; }
   }
@@ -881,7 +881,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   R->rounds = round;
   // the KDE term count is read back with the representatives at the end (no extra sync)
   std::vector<unsigned long long> h_terms;
-  SV_TRY(d2h(c, h_terms, terms.get(), 1));
+  SV_TRY(d2h(c, h_terms, terms.get(), 2));
   Pb.release(); keys.release();
 
   // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
@@ -1020,6 +1020,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   SV_TRY(sync(c));
   resolve_timing(c);
   R->kde_terms = h_terms[0];
+  R->kde_evaluated = h_terms[1];
   if (c->timing) c->acc[SIEVE_PHASE_KDE].work += h_terms[0];
   hc.mark("reps");
 
@@ -1158,10 +1159,12 @@ extern "C" int sieve_strata_copy(sieve_strata s, sieve_stratum* host_out, uint64
   if (m) memcpy(host_out, s->st.data(), m * sizeof(sieve_stratum));
   return SIEVE_OK;
 }
-extern "C" int sieve_strata_stats(sieve_strata s, uint32_t* rounds, uint64_t* terms) {
+extern "C" int sieve_strata_stats(sieve_strata s, uint32_t* rounds, uint64_t* terms,
+                                  uint64_t* evaluated) {
   if (!strata_ok(s)) return sv_fail(SIEVE_EINVAL, "bad strata handle");
   if (rounds) *rounds = s->rounds;
   if (terms) *terms = s->kde_terms;
+  if (evaluated) *evaluated = s->kde_evaluated;
   return SIEVE_OK;
 }
 extern "C" void sieve_strata_free(sieve_strata s) {
@@ -1192,6 +1195,66 @@ extern "C" int sieve_segment_get(sieve_strata s, uint64_t idx, sieve_segment* ou
 // sieve_predict
 // ------------------------------------------------------------------------------------------
 static double u128_to_double_host(u128 v) { return (double)v; }  // libgcc: correctly rounded
+
+// ------------------------------------------------------------------------------------------
+// sieve_cycle_cov: within-stratum cycle CoV (Fig. 4; reading A25: instruction
+// weights for the average)
+// ------------------------------------------------------------------------------------------
+extern "C" int sieve_cycle_cov(sieve_strata s, sieve_trace t, const uint32_t* sid, double* cov,
+                               double* weighted) {
+  if (!strata_ok(s) || !trace_ok(t)) return sv_fail(SIEVE_EINVAL, "bad handle");
+  if (!t->y) return sv_fail(SIEVE_EDOM, "the trace has no cycles column");
+  if (t->n && !sid) return sv_fail(SIEVE_EINVAL, "stratum_of_invocation (device) is required");
+  sieve_ctx c = t->ctx;
+  SV_CUDA(cudaSetDevice(c->device));
+  SV_TRY(arena_reset(c));
+  const u32 ns = (u32)s->st.size();
+  DBuf<char> part(c);
+  DBuf<u64> lanes(c), errf(c);
+  SV_TRY(part.alloc(group_moments_part_bytes(ns ? ns : 1)));
+  SV_TRY(lanes.alloc((size_t)ns * GM_LANES));
+  SV_TRY(errf.alloc(1));
+  SV_CUDA(cudaMemsetAsync(errf.get(), 0, 8, c->stream));
+  if (ns) launch_group_moments(sid, t->y, t->n, ns, (GMomPartial*)part.get(), lanes.get(), errf.get(), c->stream);
+  SV_CUDA(cudaGetLastError());
+  SV_TRY(allreduce(c, lanes.get(), (size_t)ns * GM_LANES, RED_SUM));
+  SV_TRY(allreduce(c, errf.get(), 1, RED_MAX));
+  std::vector<u64> h_l, h_e;
+  SV_TRY(d2h(c, h_l, lanes.get(), (size_t)ns * GM_LANES));
+  SV_TRY(d2h(c, h_e, errf.get(), 1));
+  SV_TRY(sync(c));
+  if (h_e[0]) return sv_fail(SIEVE_ERANGE, "cycle counts must be < 2^48 for sieve_cycle_cov");
+  long double acc = 0, I = 0;
+  for (u32 i = 0; i < ns; i++) {
+    const u64* L = &h_l[(size_t)i * GM_LANES];
+    u128 s1 = limbs_u128(L + 1);
+    // S2 from 6 limb lanes (can exceed 2^128 across ranks)
+    W256 s2 = {{0, 0, 0, 0}};
+    {
+      u128 carry = 0;
+      u64 w32[8] = {0};
+      for (int j = 0; j < 6; j++) {
+        u128 v = (u128)L[5 + j] + carry;
+        w32[j] = (u64)(v & 0xFFFFFFFFull);
+        carry = v >> 32;
+      }
+      w32[6] = (u64)(carry & 0xFFFFFFFFull);
+      w32[7] = (u64)(carry >> 32);
+      for (int j = 0; j < 4; j++) s2.w[j] = w32[2 * j] | (w32[2 * j + 1] << 32);
+    }
+    double cv = 0.0;
+    if (s1 != 0) {
+      W256 d = w256_sub(w256_mul_small(s2, L[0]), w256_mul(s1, s1));
+      cv = sqrt(w256_to_double(d)) / (double)s1;
+    }
+    if (cov) cov[i] = cv;
+    long double W = (long double)(((u128)s->st[i].instr_sum_hi << 64) | s->st[i].instr_sum_lo);
+    acc += W * cv;
+    I += W;
+  }
+  if (weighted) *weighted = ns ? (double)(acc / I) : 0.0;
+  return SIEVE_OK;
+}
 
 // M predictions at once: rep_cycles is [M][n_strata] (nullable iff M == 1: the trace's cycles)
 static int predict_impl(sieve_strata s, sieve_trace t, u32 M, const uint64_t* rep_cycles,

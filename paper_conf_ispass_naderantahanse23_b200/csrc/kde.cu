@@ -236,6 +236,10 @@ k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ k
     acc -= (u64)nterm * 0x4330000000000000ull;
 #pragma unroll
     for (int o = KDE_TJ; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    if (terms && lane == 0) {  // evaluated (lane, value) pairs of this item, wasted ones included
+      u32 live = min((u32)KDE_TJ, G - t * KDE_TJ);
+      atomicAdd(terms + 1, (unsigned long long)live * len);
+    }
     if (j < G && slice == 0) {
       if (acc) {
         unsigned long long* d = (unsigned long long*)(D + 2 * ((u64)s * G + j));

@@ -130,6 +130,14 @@ void launch_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, co
 void launch_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, u32 M, double* out,
                     cudaStream_t s);
 
+// ---------------- within-stratum cycle moments (Fig. 4 diagnostic) ----------------------------
+struct GMomPartial { u64 n, s1lo, s1hi, s2lo, s2hi; };
+#define GM_LANES 11   // n, S1 (4 limbs), S2 (6 limbs)
+size_t group_moments_part_bytes(u32 nstrata);
+// lanes: [nstrata][GM_LANES]; errflag set to 1 if a cycle count >= 2^48 is seen
+void launch_group_moments(const u32* sid, const u64* y, u64 n, u32 nstrata, GMomPartial* part,
+                          u64* lanes, u64* errflag, cudaStream_t s);
+
 // ---------------- misc -------------------------------------------------------------------------
 void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s);
 // cross-rank encoding of u128 pairs [n][2] <-> 4 limbs [n][4]

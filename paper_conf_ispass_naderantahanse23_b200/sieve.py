@@ -36,7 +36,7 @@ EXPORTED = [
     "sieve_segment_count", "sieve_segment_get", "sieve_predict", "sieve_last_error",
     "sieve_version", "sieve_u128_to_limbs", "sieve_limbs_to_u128", "sieve_ctx_set_timing",
     "sieve_timing_get", "sieve_kernel_launches", "sieve_stratify_sweep", "sieve_tier_census",
-    "sieve_predict_multi",
+    "sieve_predict_multi", "sieve_cycle_cov",
 ]
 PHASES = ["moments", "compact", "sort", "prefix", "kde", "refine", "assign", "reps", "predict"]
 
@@ -83,7 +83,7 @@ def _load():
         "sieve_stratify": ([vp, P(Params), vp, P(vp)], i32),
         "sieve_strata_count": ([vp, P(u64)], i32),
         "sieve_strata_copy": ([vp, vp, u64], i32),
-        "sieve_strata_stats": ([vp, P(u32), P(u64)], i32),
+        "sieve_strata_stats": ([vp, P(u32), P(u64), P(u64)], i32),
         "sieve_strata_free": ([vp], None),
         "sieve_segment_count": ([vp, P(u64)], i32),
         "sieve_segment_get": ([vp, u64, P(_Segment), vp, vp, vp], i32),
@@ -98,6 +98,7 @@ def _load():
         "sieve_stratify_sweep": ([vp, P(Params), u32, vp, vp, vp], i32),
         "sieve_tier_census": ([vp, u32, vp, vp, vp, vp, vp], i32),
         "sieve_predict_multi": ([vp, vp, u32, vp, P(_Prediction)], i32),
+        "sieve_cycle_cov": ([vp, vp, vp, vp, P(ctypes.c_double)], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -279,9 +280,10 @@ class Strata:
         if n.value:
             _check(_L.sieve_strata_copy(h, self.table.ctypes.data_as(ctypes.c_void_p), n.value),
                    "sieve_strata_copy")
-        r, t = ctypes.c_uint32(), ctypes.c_uint64()
-        _check(_L.sieve_strata_stats(h, ctypes.byref(r), ctypes.byref(t)), "sieve_strata_stats")
-        self.rounds, self.kde_terms = r.value, t.value
+        r, t, ev = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint64()
+        _check(_L.sieve_strata_stats(h, ctypes.byref(r), ctypes.byref(t), ctypes.byref(ev)),
+               "sieve_strata_stats")
+        self.rounds, self.kde_terms, self.kde_evaluated = r.value, t.value, ev.value
 
     def __len__(self):
         return len(self.table)
@@ -370,6 +372,15 @@ def predict_multi(strata, trace, rep_cycles):
     _check(_L.sieve_predict_multi(strata._h, trace._h, rc.shape[0], rc.ctypes.data_as(ctypes.c_void_p),
                                   outs), "sieve_predict_multi")
     return [_pred_dict(o) for o in outs]
+
+
+def cycle_cov(strata, trace, stratum_of_invocation):
+    """sieve_cycle_cov: per-stratum CoV of member cycles + instruction-weighted mean (Fig. 4)."""
+    cov = np.zeros(len(strata), np.float64)
+    w = ctypes.c_double()
+    _check(_L.sieve_cycle_cov(strata._h, trace._h, ctypes.c_void_p(stratum_of_invocation.data_ptr()),
+                              cov.ctypes.data_as(ctypes.c_void_p), ctypes.byref(w)), "sieve_cycle_cov")
+    return cov, w.value
 
 
 def predict(strata, trace, rep_cycles=None):

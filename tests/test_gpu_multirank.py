@@ -73,3 +73,20 @@ def test_group_rank_with_empty_slice():
     o = run_oracle(tr)
     for table, _, _ in res:
         assert_tables_equal(table, o.strata)
+
+
+def test_nccl_path_single_rank():
+    """The NCCL communicator path (dlopen of libnccl, ncclCommInitRank, ncclAllReduce on every
+    reduction) with one rank must give exactly the no-communicator result."""
+    import torch
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr = gen.make_trace("C2")
+    one = run_gpu(tr)
+    uid = sieve.get_unique_id()
+    ctx = sieve.Ctx(device=0, rank=0, world=1, nccl_id=uid)
+    trace = sieve.load_trace(ctx, tr["kid"], tr["x"], num_kernels=tr["K"], cta=tr["cta"], cycles=tr["y"])
+    sid = torch.empty(len(tr["kid"]), dtype=torch.int32, device="cuda")
+    st = sieve.stratify(trace, stratum_of_invocation=sid)
+    torch.cuda.synchronize()
+    assert st.table.tobytes() == one["table"].tobytes()
+    assert np.array_equal(sid.cpu().numpy().view(np.uint32), one["sid"])

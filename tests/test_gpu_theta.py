@@ -71,3 +71,20 @@ def test_predict_multi_architecture():
     assert abs(preds[1]["predicted_cycles"] / preds[0]["predicted_cycles"] - 2.0) < 1e-12
     single = sieve.predict(st, trace)
     assert preds[0]["predicted_cycles"] == single["predicted_cycles"]
+
+
+@pytest.mark.parametrize("name", ["C1", "C2"])
+def test_cycle_cov_matches_oracle(name):
+    """Fig. 4 diagnostic: per-stratum cycle CoV bit-identical to the oracle."""
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    from tests.gpu_helpers import run_gpu
+    tr = gen.make_trace(name)
+    g = run_gpu(tr)
+    import torch
+    sid = torch.from_numpy(g["sid"].view(np.int32)).cuda()
+    cov, w = sieve.cycle_cov(g["strata"], g["trace"], sid)
+    o = run_oracle(tr)
+    ocov, ow = o.cycle_cov(tr["y"])
+    assert np.array_equal(cov, ocov)
+    assert abs(w - ow) <= 1e-12 * max(ow, 1e-300)
+    assert 0.0 <= w < 0.5     # within-stratum cycle variability is small (P:228: 0.09 mean)

@@ -207,3 +207,31 @@ def test_errors():
 def test_empty_trace():
     r = oracle.stratify(np.zeros(0, np.uint32), np.zeros(0, np.uint64), 4)
     assert len(r.strata) == 0
+
+
+# ---------------------------------------------------------------- cycle CoV (Fig. 4)
+def test_cycle_cov_definition_and_closed_forms():
+    tr = gen.make_trace("C1")
+    r = oracle.stratify(tr["kid"], tr["x"], tr["K"], tr["cta"], tr["y"])
+    cov, wmean = r.cycle_cov(tr["y"])
+    st = r.strata
+    order = np.argsort(r.sid, kind="stable")
+    bounds = np.searchsorted(r.sid[order], np.arange(len(st) + 1))
+    W = [(int(h) << 64) | int(l) for l, h in zip(st["instr_sum_lo"], st["instr_sum_hi"])]
+    want = []
+    for s in range(len(st)):
+        ys = [Fraction(int(v)) for v in tr["y"][order[bounds[s]:bounds[s + 1]]]]
+        mu = sum(ys) / len(ys)
+        var = sum((v - mu) ** 2 for v in ys) / len(ys)     # population (A1 / A25)
+        want.append(math.sqrt(float(var)) / float(mu))
+    assert np.allclose(cov, want, rtol=1e-14, atol=0)
+    assert math.isclose(wmean, sum(w * c for w, c in zip(W, want)) / sum(W), rel_tol=1e-14)
+    # closed forms: constant cycles -> 0; members {y, 3y} -> sigma = y, mu = 2y -> 0.5
+    kid = np.zeros(4, np.uint32)
+    x = np.array([100, 100, 100, 100], np.uint64)
+    r2 = oracle.stratify(kid, x, 1, None, np.array([7, 7, 7, 7], np.uint64))
+    assert r2.cycle_cov(np.array([7, 7, 7, 7], np.uint64))[0][0] == 0.0
+    y = np.array([5, 15, 5, 15], np.uint64)
+    assert r2.cycle_cov(y)[0][0] == 0.5
+    with pytest.raises(oracle.OracleError):
+        r2.cycle_cov(np.array([1, 1, 1, 1 << 48], np.uint64))
