@@ -113,6 +113,32 @@ int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_id, uint32_
                      const uint64_t* cycles, uint32_t mem, sieve_trace* out);
 void sieve_trace_free(sieve_trace t);
 
+/* Load the profile from its CSV export ("converted into a readable CSV file which serves
+   as input"), parsed and interned on the GPU.  One row per invocation in
+   launch order (invocation id = first_id + data-row index).  Quoted fields may contain the
+   delimiter; numbers may carry thousands separators; newlines inside fields are not allowed.
+   Kernel names (quote characters removed) are interned into dense ids in order of first
+   appearance, identified by a 64-bit FNV-1a hash of their bytes.
+     data, bytes  the CSV text: HOST (mem = SIEVE_MEM_HOST) or DEVICE (SIEVE_MEM_DEVICE)
+     spec         0-based columns; col_cta / col_cycles = -1 if absent; header_lines to skip
+     num_kernels  nullable: receives the number of distinct names
+   SIEVE_EINVAL on a malformed row, SIEVE_ERANGE beyond 65536 names or 2^32 rows. */
+typedef struct {
+  int32_t col_kernel, col_instr, col_cta, col_cycles;
+  uint32_t header_lines;
+  char delimiter;
+} sieve_csv_spec;
+int sieve_load_csv(sieve_ctx ctx, const char* data, uint64_t bytes, uint32_t mem,
+                   const sieve_csv_spec* spec, uint64_t first_id, sieve_trace* out,
+                   uint32_t* num_kernels);
+/* copy a trace's columns (n_local rows) back into HOST buffers; every pointer is nullable and a
+   column the trace does not hold is left untouched.  Synchronises the context's stream. */
+int sieve_trace_copy(sieve_trace t, uint32_t* kernel_id, uint64_t* instr, uint32_t* cta,
+                     uint64_t* cycles, uint64_t* n_local, uint32_t* num_kernels);
+/* names of a CSV-loaded trace in id order, each followed by '\n', into a HOST buffer of cap
+   bytes; *needed receives the total size (call with buf = NULL to size it) */
+int sieve_trace_kernel_names(sieve_trace t, char* buf, uint64_t cap, uint64_t* needed);
+
 /* ---- stratification ------------------------------------------------------------ */
 typedef struct {
   uint32_t theta_num, theta_den; /* theta = num/den, exact rational (P:85 default 0.4 = 2/5; A3) */

@@ -165,6 +165,7 @@ struct sieve_trace_s {
   u32* cta = nullptr;
   u64* y = nullptr;
   bool owned = true;
+  std::vector<std::string> names;  // kernel names by id (traces loaded from CSV)
 };
 
 struct SegDebug {
@@ -1318,4 +1319,163 @@ extern "C" int sieve_predict_multi(sieve_strata s, sieve_trace t, uint32_t M, co
   if (M == 0) return SIEVE_OK;
   if (!rep_cycles) return sv_fail(SIEVE_EINVAL, "rep_cycles [M][n_strata] is required");
   return predict_impl(s, t, M, rep_cycles, out);
+}
+
+// ------------------------------------------------------------------------------------------
+// sieve_load_csv: the profiler's CSV parsed and interned on the GPU
+// ------------------------------------------------------------------------------------------
+extern "C" int sieve_load_csv(sieve_ctx ctx, const char* data, uint64_t bytes, uint32_t mem,
+                              const sieve_csv_spec* spec, uint64_t first_id, sieve_trace* out,
+                              uint32_t* num_kernels) {
+  if (!out) return sv_fail(SIEVE_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!ctx_ok(ctx) || !spec || (bytes && !data)) return sv_fail(SIEVE_EINVAL, "bad argument");
+  if (spec->col_kernel < 0 || spec->col_instr < 0) return sv_fail(SIEVE_EINVAL, "kernel and instruction columns are required");
+  if (mem & ~1u) return sv_fail(SIEVE_EINVAL, "mem must be SIEVE_MEM_HOST or SIEVE_MEM_DEVICE");
+  sieve_ctx c = ctx;
+  cudaStream_t S = c->stream;
+  SV_CUDA(cudaSetDevice(c->device));
+  SV_TRY(arena_reset(c));
+  // the bytes on the device, and on the host (for the names)
+  const unsigned char* dbuf = (const unsigned char*)data;
+  std::vector<char> hostcopy;
+  const char* hbuf = data;
+  if (!(mem & SIEVE_MEM_DEVICE)) {
+    DBuf<unsigned char> db(c);
+    SV_TRY(db.alloc(bytes ? bytes : 1));
+    if (bytes) SV_CUDA(cudaMemcpyAsync(db.get(), data, bytes, cudaMemcpyHostToDevice, S));
+    dbuf = db.get();
+  } else {
+    hostcopy.resize(bytes);
+    if (bytes) SV_CUDA(cudaMemcpyAsync(hostcopy.data(), data, bytes, cudaMemcpyDeviceToHost, S));
+    hbuf = hostcopy.data();
+  }
+  // 1. line ends
+  const u64 nt = csv_tiles(bytes);
+  DBuf<u32> tiles(c);
+  DBuf<char> stemp(c);
+  SV_TRY(tiles.alloc(nt + 1));
+  SV_TRY(stemp.alloc(scan_u32_temp_bytes(nt + 1)));
+  SV_CUDA(cudaMemsetAsync(tiles.get(), 0, (nt + 1) * 4, S));
+  launch_csv_count(dbuf, bytes, tiles.get(), stemp.get(), S);
+  std::vector<u32> h_nl;
+  SV_TRY(d2h(c, h_nl, tiles.get() + nt, 1));
+  SV_TRY(sync(c));
+  const u64 nends = h_nl[0];
+  DBuf<u64> ends(c);
+  SV_TRY(ends.alloc(nends + 1));
+  launch_csv_ends(dbuf, bytes, tiles.get(), ends.get(), S);
+  bool trailing = bytes > 0 && hbuf[bytes - 1] == '\n';
+  const u64 nlines = nends + (bytes > 0 && !trailing ? 1 : 0);
+  const u64 nrows = nlines > spec->header_lines ? nlines - spec->header_lines : 0;
+  if (nrows >= (1ull << 32)) return sv_fail(SIEVE_ERANGE, "more than 2^32 - 1 rows");
+  // 2. parse
+  DBuf<u64> hash(c), npos(c), errf(c);
+  DBuf<u32> row(c);
+  SV_TRY(hash.alloc(nrows)); SV_TRY(npos.alloc(2 * nrows)); SV_TRY(errf.alloc(1)); SV_TRY(row.alloc(nrows));
+  SV_CUDA(cudaMemsetAsync(errf.get(), 0, 8, S));
+  sieve_trace_s* t = new sieve_trace_s();
+  t->ctx = c; t->n = nrows; t->first_id = first_id; t->owned = true;
+  auto fail = [&](int st) { cudaStreamSynchronize(S); sieve_trace_free(t); return st; };
+#define CSV_TRY(e) do { int _s = (e); if (_s != SIEVE_OK) return fail(_s); } while (0)
+  void* p;
+  int st = SIEVE_OK;
+  if ((st = dalloc(c, &p, nrows * 4 + 16)) != SIEVE_OK) return fail(st);
+  t->kid = (u32*)p;
+  if ((st = dalloc(c, &p, nrows * 8 + 16)) != SIEVE_OK) return fail(st);
+  t->x = (u64*)p;
+  if (spec->col_cta >= 0) { if ((st = dalloc(c, &p, nrows * 4 + 16)) != SIEVE_OK) return fail(st); t->cta = (u32*)p; }
+  if (spec->col_cycles >= 0) { if ((st = dalloc(c, &p, nrows * 8 + 16)) != SIEVE_OK) return fail(st); t->y = (u64*)p; }
+  CsvSpec cs{spec->col_kernel, spec->col_instr, spec->col_cta, spec->col_cycles, (unsigned char)spec->delimiter};
+  launch_csv_parse(dbuf, bytes, ends.get(), nends, spec->header_lines, nrows, cs, hash.get(), row.get(),
+                   npos.get(), t->x, t->cta, t->y, errf.get(), S);
+  // 3. intern names: stable sort by hash, distinct heads, ids by first appearance
+  std::vector<u64> h_err, h_names;
+  std::vector<u32> h_nd;
+  u64 nd = 0;
+  if (nrows) {
+    {
+      DBuf<char> tmp(c);
+      if ((st = tmp.alloc(radix_sort_temp_bytes(nrows, true))) != SIEVE_OK) return fail(st);
+      if ((st = pin_alloc(c, &p, RADIX_PINNED_BYTES)) != SIEVE_OK) return fail(st);
+      if ((st = radix_sort(hash.get(), row.get(), nrows, 64, tmp.get(), S, p)) != SIEVE_OK) return fail(st);
+    }
+    DBuf<u32> flag(c), seg(c);
+    DBuf<char> st2(c);
+    CSV_TRY(flag.alloc(nrows)); CSV_TRY(seg.alloc(nrows + 1)); CSV_TRY(st2.alloc(scan_u32_temp_bytes(nrows)));
+    launch_csv_heads(hash.get(), nrows, flag.get(), S);
+    scan_u32(flag.get(), seg.get(), nrows, st2.get(), seg.get() + nrows, S);
+    CSV_TRY(d2h(c, h_nd, seg.get() + nrows, 1));
+    CSV_TRY(d2h(c, h_err, errf.get(), 1));
+    if ((st = sync(c)) != SIEVE_OK) return fail(st);
+    nd = h_nd[0];
+    if (h_err[0]) return fail(sv_fail(SIEVE_EINVAL, "malformed CSV row (missing field or non-integer count)"));
+    if (nd > SIEVE_MAX_K) return fail(sv_fail(SIEVE_ERANGE, "more than 65536 distinct kernel names"));
+    DBuf<u64> fkey(c), names(c);
+    DBuf<u32> fval(c), id_of(c);
+    CSV_TRY(fkey.alloc(nd)); CSV_TRY(fval.alloc(nd)); CSV_TRY(id_of.alloc(nd)); CSV_TRY(names.alloc(2 * nd));
+    launch_csv_firsts(flag.get(), seg.get(), row.get(), nrows, fkey.get(), fval.get(), S);
+    {
+      DBuf<char> tmp(c);
+      if ((st = tmp.alloc(radix_sort_temp_bytes(nd, true))) != SIEVE_OK) return fail(st);
+      if ((st = pin_alloc(c, &p, RADIX_PINNED_BYTES)) != SIEVE_OK) return fail(st);
+      if ((st = radix_sort(fkey.get(), fval.get(), nd, 32, tmp.get(), S, p)) != SIEVE_OK) return fail(st);
+    }
+    launch_csv_ids(fval.get(), nd, id_of.get(), flag.get(), seg.get(), row.get(), nrows, t->kid, S);
+    launch_gather_pairs(npos.get(), fkey.get(), nd, names.get(), S);  // first row of each id
+    CSV_TRY(d2h(c, h_names, names.get(), 2 * nd));
+    if ((st = sync(c)) != SIEVE_OK) return fail(st);
+    { cudaError_t ce = cudaGetLastError(); if (ce) return fail(sv_cuda(ce, "csv kernels", __LINE__)); }
+  }
+  t->K = nd ? (u32)nd : 1;
+  t->names.resize(nd);
+  for (u64 d = 0; d < nd; d++) {
+    std::string s;
+    const char* q = hbuf + h_names[2 * d];
+    for (u64 i = 0; i < h_names[2 * d + 1]; i++) if (q[i] != '"') s.push_back(q[i]);
+    t->names[d] = s;
+  }
+  if (num_kernels) *num_kernels = (uint32_t)nd;
+  *out = t;
+#undef CSV_TRY
+  return SIEVE_OK;
+}
+
+// copy a trace's columns back to HOST buffers (each nullable; a column the trace lacks is left
+// untouched); *n_local / *num_kernels nullable
+extern "C" int sieve_trace_copy(sieve_trace t, uint32_t* kernel_id, uint64_t* instr, uint32_t* cta,
+                                uint64_t* cycles, uint64_t* n_local, uint32_t* num_kernels) {
+  if (!trace_ok(t)) return sv_fail(SIEVE_EINVAL, "bad trace handle");
+  sieve_ctx c = t->ctx;
+  SV_CUDA(cudaSetDevice(c->device));
+  if (n_local) *n_local = t->n;
+  if (num_kernels) *num_kernels = t->K;
+  auto cp = [&](void* dst, const void* src, size_t bytes) -> int {
+    if (dst && src && bytes) SV_CUDA(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, c->stream));
+    return SIEVE_OK;
+  };
+  SV_TRY(cp(kernel_id, t->kid, t->n * 4));
+  SV_TRY(cp(instr, t->x, t->n * 8));
+  SV_TRY(cp(cta, t->cta, t->n * 4));
+  SV_TRY(cp(cycles, t->y, t->n * 8));
+  SV_CUDA(cudaStreamSynchronize(c->stream));
+  return SIEVE_OK;
+}
+
+// kernel names of a CSV-loaded trace, in id order, each terminated by '\n'; *needed = bytes
+extern "C" int sieve_trace_kernel_names(sieve_trace t, char* buf, uint64_t cap, uint64_t* needed) {
+  if (!trace_ok(t)) return sv_fail(SIEVE_EINVAL, "bad trace handle");
+  u64 need = 0;
+  for (auto& s : t->names) need += s.size() + 1;
+  if (needed) *needed = need;
+  if (buf) {
+    u64 o = 0;
+    for (auto& s : t->names) {
+      if (o + s.size() + 1 > cap) break;
+      memcpy(buf + o, s.data(), s.size());
+      o += s.size();
+      buf[o++] = '\n';
+    }
+  }
+  return SIEVE_OK;
 }

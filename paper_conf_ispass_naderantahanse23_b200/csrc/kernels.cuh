@@ -138,6 +138,26 @@ size_t group_moments_part_bytes(u32 nstrata);
 void launch_group_moments(const u32* sid, const u64* y, u64 n, u32 nstrata, GMomPartial* part,
                           u64* lanes, u64* errflag, cudaStream_t s);
 
+// ---------------- CSV profile ingest (NEXT-4) ---------------------------------------------------
+struct CsvSpec { int col_kernel, col_instr, col_cta, col_cycles; int delim; };
+u64 csv_tiles(u64 nbytes);
+// tile_count: [tiles + 1]; after the first launch tile_count[tiles] = number of '\n'
+void launch_csv_count(const unsigned char* buf, u64 nbytes, u32* tile_count, void* scan_temp,
+                      cudaStream_t s);
+void launch_csv_ends(const unsigned char* buf, u64 nbytes, const u32* tile_off, u64* ends,
+                     cudaStream_t s);
+void launch_csv_parse(const unsigned char* buf, u64 nbytes, const u64* ends, u64 nends,
+                      u64 first_line, u64 nrows, CsvSpec spec, u64* hash, u32* row, u64* name_pos,
+                      u64* x, u32* cta, u64* y, u64* errflag, cudaStream_t s);
+void launch_csv_heads(const u64* h, u64 n, u32* flag, cudaStream_t s);
+void launch_csv_firsts(const u32* flag, const u32* seg, const u32* row, u64 n, u64* first_key,
+                       u32* first_val, cudaStream_t s);
+void launch_csv_ids(const u32* order, u64 nd, u32* id_of, const u32* flag, const u32* seg,
+                    const u32* row, u64 n, u32* kid, cudaStream_t s);
+void launch_gather_pairs(const u64* src, const u64* idx, u64 n, u64* dst, cudaStream_t s);
+void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s);
+size_t scan_u32_temp_bytes(u64 n);
+
 // ---------------- misc -------------------------------------------------------------------------
 void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s);
 // cross-rank encoding of u128 pairs [n][2] <-> 4 limbs [n][4]

@@ -36,7 +36,8 @@ EXPORTED = [
     "sieve_segment_count", "sieve_segment_get", "sieve_predict", "sieve_last_error",
     "sieve_version", "sieve_u128_to_limbs", "sieve_limbs_to_u128", "sieve_ctx_set_timing",
     "sieve_timing_get", "sieve_kernel_launches", "sieve_stratify_sweep", "sieve_tier_census",
-    "sieve_predict_multi", "sieve_cycle_cov",
+    "sieve_predict_multi", "sieve_cycle_cov", "sieve_load_csv", "sieve_trace_copy",
+    "sieve_trace_kernel_names",
 ]
 PHASES = ["moments", "compact", "sort", "prefix", "kde", "refine", "assign", "reps", "predict"]
 
@@ -60,6 +61,12 @@ class _Prediction(ctypes.Structure):
                 ("measured_cycles", ctypes.c_double), ("error", ctypes.c_double),
                 ("speedup", ctypes.c_double), ("total_instr_lo", ctypes.c_uint64),
                 ("total_instr_hi", ctypes.c_uint64)]
+
+
+class CsvSpec(ctypes.Structure):
+    _fields_ = [("col_kernel", ctypes.c_int32), ("col_instr", ctypes.c_int32),
+                ("col_cta", ctypes.c_int32), ("col_cycles", ctypes.c_int32),
+                ("header_lines", ctypes.c_uint32), ("delimiter", ctypes.c_char)]
 
 
 def _load():
@@ -99,6 +106,9 @@ def _load():
         "sieve_tier_census": ([vp, u32, vp, vp, vp, vp, vp], i32),
         "sieve_predict_multi": ([vp, vp, u32, vp, P(_Prediction)], i32),
         "sieve_cycle_cov": ([vp, vp, vp, vp, P(ctypes.c_double)], i32),
+        "sieve_load_csv": ([vp, vp, u64, u32, P(CsvSpec), u64, P(vp), P(u32)], i32),
+        "sieve_trace_copy": ([vp, vp, vp, vp, vp, P(u64), P(u32)], i32),
+        "sieve_trace_kernel_names": ([vp, vp, u64, P(u64)], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -259,6 +269,49 @@ def load_trace(ctx, kernel_id, instr, num_kernels, cta=None, cycles=None, first_
     _check(_L.sieve_load_trace(ctx._h, n, first_id, num_kernels, cols[0][0], cols[1][0], cols[2][0],
                                cols[3][0], mem, ctypes.byref(h)), "sieve_load_trace")
     return Trace(h, ctx, n, [c[2] for c in cols] if adopt else None)
+
+
+def load_csv(ctx, data, col_kernel, col_instr, col_cta=-1, col_cycles=-1, header_lines=1,
+             delimiter=",", first_id=0):
+    """sieve_load_csv: `data` is the CSV text (bytes / str on the host, or a CUDA uint8 tensor).
+    Returns (Trace, names) with names[i] the kernel name of id i (first-appearance order)."""
+    spec = CsvSpec(col_kernel, col_instr, col_cta, col_cycles, header_lines, delimiter.encode())
+    keep = None
+    if isinstance(data, str):
+        data = data.encode()
+    if isinstance(data, (bytes, bytearray)):
+        keep = ctypes.create_string_buffer(bytes(data), len(data))
+        ptr, nbytes, mem = ctypes.cast(keep, ctypes.c_void_p), len(data), MEM_HOST
+    else:
+        import torch
+        if not (isinstance(data, torch.Tensor) and data.is_cuda and data.dtype == torch.uint8):
+            raise TypeError("data must be bytes, str or a CUDA uint8 tensor")
+        ptr, nbytes, mem = ctypes.c_void_p(data.data_ptr()), data.numel(), MEM_DEVICE
+    h, nk = ctypes.c_void_p(), ctypes.c_uint32()
+    _check(_L.sieve_load_csv(ctx._h, ptr, nbytes, mem, ctypes.byref(spec), first_id, ctypes.byref(h),
+                             ctypes.byref(nk)), "sieve_load_csv")
+    n = ctypes.c_uint64()
+    _check(_L.sieve_trace_copy(h, None, None, None, None, ctypes.byref(n), None), "sieve_trace_copy")
+    t = Trace(h, ctx, n.value, None)
+    need = ctypes.c_uint64()
+    _check(_L.sieve_trace_kernel_names(h, None, 0, ctypes.byref(need)), "sieve_trace_kernel_names")
+    buf = ctypes.create_string_buffer(max(1, need.value))
+    _check(_L.sieve_trace_kernel_names(h, buf, need.value, ctypes.byref(need)), "sieve_trace_kernel_names")
+    names = buf.raw[:need.value].decode(errors="replace").split("\n")[:-1] if need.value else []
+    assert len(names) == nk.value
+    t.names = names
+    return t, names
+
+
+def trace_columns(trace, cta=True, cycles=True):
+    """sieve_trace_copy: the trace's columns as host numpy arrays (kid, x, cta|None, y|None)."""
+    n = trace.n
+    kid, x = np.zeros(n, np.uint32), np.zeros(n, np.uint64)
+    c = np.zeros(n, np.uint32) if cta else None
+    y = np.zeros(n, np.uint64) if cycles else None
+    ptr = lambda a: None if a is None else a.ctypes.data_as(ctypes.c_void_p)
+    _check(_L.sieve_trace_copy(trace._h, ptr(kid), ptr(x), ptr(c), ptr(y), None, None), "sieve_trace_copy")
+    return kid, x, c, y
 
 
 def default_params(**kw):
