@@ -61,7 +61,9 @@ def report(rep):
 def traffic(rep, kname):
     per = []
     for r, u in raw_rows(rep):
-        if r.get("Kernel Name", "").split("(")[0] != kname:
+        base = r.get("Kernel Name", "").split("(")[0]
+        base = base[5:] if base.startswith("void ") else base
+        if base.split("<")[0] != kname:
             continue
         b = 0.0
         for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
