@@ -61,6 +61,8 @@ def _lib():
         L.oracle_q.restype = u64
         L.oracle_cycle_cov.argtypes = [vp, vp, vp, ctypes.POINTER(dbl)]
         L.oracle_cycle_cov.restype = ctypes.c_int
+        L.oracle_min_strata.argtypes = [u64, u32, vp, vp, u32, u32, u64, vp, vp, u64, ctypes.POINTER(u64)]
+        L.oracle_min_strata.restype = ctypes.c_int
         L.oracle_exp2_table.argtypes = [ctypes.c_int]
         L.oracle_exp2_table.restype = dbl
         L.oracle_tier.argtypes = [u64, u64, u64, u64, u64, u64, u64, u32, u32]
@@ -178,6 +180,30 @@ def stratify(kid, x, K, cta=None, cycles=None, ids=None, theta=(2, 5), G=1024, v
     if rc != 0:
         raise OracleError(rc)
     return Result(h, len(kid), G)
+
+
+def min_strata(kid, x, K, theta=(2, 5), max_distinct=1 << 62):
+    """NEXT-3 (reading A28): exact minimum strata per kernel and the canonical optimal cuts.
+    -> (counts[K] as uint32, list of per-kernel cut lists)."""
+    kid = np.ascontiguousarray(kid, np.uint32)
+    x = np.ascontiguousarray(x, np.uint64)
+    counts = np.zeros(K, np.uint32)
+    nc = ctypes.c_uint64()
+    rc = _lib().oracle_min_strata(len(kid), K, _p(kid), _p(x), theta[0], theta[1], max_distinct,
+                                  _p(counts), None, 0, ctypes.byref(nc))
+    if rc != 0:
+        raise OracleError(rc)
+    cuts = np.zeros(max(1, nc.value), np.uint64)
+    rc = _lib().oracle_min_strata(len(kid), K, _p(kid), _p(x), theta[0], theta[1], max_distinct,
+                                  _p(counts), _p(cuts), nc.value, ctypes.byref(nc))
+    if rc != 0:
+        raise OracleError(rc)
+    per, o = [], 0
+    for c in counts.tolist():
+        k = c - 1 if 2 <= c < 0xFFFFFFFF else 0
+        per.append([int(v) for v in cuts[o:o + k]])
+        o += k
+    return counts, per
 
 
 # ---- step functions exported for the pin tests ----

@@ -198,3 +198,24 @@ def predict(strata, cycles=None, rep_cycles=None):
         out["error"] = float(abs(c_pred - cm) / cm) if cm else math.nan
         out["speedup"] = float(Fraction(cm, sum(ys)))
     return out
+
+
+def min_strata(vals, theta=Fraction(2, 5)):
+    """NEXT-3 by exhaustion (reading A28): every way of cutting the sorted distinct values into
+    runs; the minimum count whose runs all have CoV < theta (Fractions, population sigma), and
+    the canonical optimum = the one whose cut positions, read from the last, are smallest."""
+    from itertools import combinations
+    d = sorted(set(int(v) for v in vals))
+    m = len(d)
+    groups = {v: [w for w in vals if int(w) == v] for v in d}
+    for k in range(1, m + 1):
+        found = []
+        for cut in combinations(range(1, m), k - 1):
+            bounds = (0,) + cut + (m,)
+            if all(cov_below([w for v in d[bounds[t]:bounds[t + 1]] for w in groups[v]], theta)
+                   for t in range(k)):
+                found.append(cut)
+        if found:
+            best = min(found, key=lambda c: tuple(reversed(c)))
+            return k, [d[i] for i in best]
+    raise AssertionError("unreachable: single values are always valid")

@@ -702,6 +702,97 @@ int oracle_cycle_cov(const oracle_result* R, const uint64_t* cycles, double* cov
   return OR_OK;
 }
 
+/* ------------------------------------------------------------------------------------------
+ * NEXT-3: the exact minimum number of strata ("(1) minimises the number of strata such
+ * that (2) the CoV of each stratum is below theta"; reading A28).  Per kernel, over its distinct
+ * instruction counts v_1 < ... < v_m with multiplicities c_1..c_m, a stratum is a run of
+ * consecutive distinct values; f(0) = 0 and
+ *     f(j) = min { f(i) + 1 : 0 <= i < j, CoV(v_{i+1..j}) < theta }      (O3's exact test),
+ * which always has the candidate i = j - 1 (one value: CoV 0).  The optimum is f(m); the
+ * canonical optimal partition takes, at every step of the backtrack from j = m, the SMALLEST
+ * i attaining f(j) - 1, and the cuts reported are the lowest value of every stratum but the
+ * first, ascending.  A kernel that is one valid stratum (Tier-1/2) has f(m) = 1 and no cuts; a
+ * kernel with more than max_distinct distinct values that is not is skipped (UINT32_MAX).
+ * counts[K]; cuts (nullable) receives the cuts of kernels 0..K-1 in order.
+ * ------------------------------------------------------------------------------------------ */
+static int cmp_u64(const void* a, const void* b) {
+  uint64_t x = *(const uint64_t*)a, y = *(const uint64_t*)b;
+  return x < y ? -1 : x > y;
+}
+
+int oracle_min_strata(uint64_t n, uint32_t K, const uint32_t* kid, const uint64_t* x, uint32_t p,
+                      uint32_t q, uint64_t max_distinct, uint32_t* counts, uint64_t* cuts,
+                      uint64_t cuts_cap, uint64_t* n_cuts) {
+  uint64_t total_cuts = 0;
+  uint64_t* vals = (uint64_t*)malloc((n ? n : 1) * sizeof(uint64_t));
+  if (!vals) return OR_ENOMEM;
+  for (uint32_t k = 0; k < K; k++) {
+    /* O1: the kernel's instruction counts, sorted */
+    uint64_t nk = 0;
+    for (uint64_t i = 0; i < n; i++) if (kid[i] == k) vals[nk++] = x[i];
+    counts[k] = 0;
+    if (!nk) continue;
+    qsort(vals, nk, sizeof(uint64_t), cmp_u64);
+    /* distinct values and their multiplicities; prefix sums N, S1, S2 over them */
+    uint64_t m = 0;
+    uint64_t* v = (uint64_t*)malloc(nk * sizeof(uint64_t));
+    uint64_t* c = (uint64_t*)malloc(nk * sizeof(uint64_t));
+    for (uint64_t i = 0; i < nk; i++) {
+      if (i == 0 || vals[i] != vals[i - 1]) { v[m] = vals[i]; c[m] = 0; m++; }
+      c[m - 1]++;
+    }
+    uint64_t* N = (uint64_t*)malloc((m + 1) * sizeof(uint64_t));
+    u128* S1 = (u128*)malloc((m + 1) * sizeof(u128));
+    u128* S2 = (u128*)malloc((m + 1) * sizeof(u128));
+    N[0] = 0; S1[0] = 0; S2[0] = 0;
+    for (uint64_t i = 0; i < m; i++) {
+      N[i + 1] = N[i] + c[i];
+      S1[i + 1] = S1[i] + (u128)c[i] * v[i];
+      S2[i + 1] = S2[i] + (u128)c[i] * v[i] * v[i];
+    }
+    uint32_t best = 0;
+    uint32_t* f = NULL;
+    uint64_t* arg = NULL;
+    if (cov_below(N[m], S1[m], S2[m], p, q)) {
+      best = 1;                                   /* the whole kernel is one valid stratum */
+    } else if (m > max_distinct) {
+      best = UINT32_MAX;                          /* skipped */
+    } else {
+      f = (uint32_t*)malloc((m + 1) * sizeof(uint32_t));
+      arg = (uint64_t*)malloc((m + 1) * sizeof(uint64_t));
+      f[0] = 0;
+      for (uint64_t j = 1; j <= m; j++) {
+        f[j] = UINT32_MAX;
+        for (uint64_t i = 0; i < j; i++) {
+          if (f[i] + 1 < f[j] &&
+              cov_below(N[j] - N[i], S1[j] - S1[i], S2[j] - S2[i], p, q)) {
+            f[j] = f[i] + 1;
+            arg[j] = i;                           /* strict < keeps the smallest i */
+          }
+        }
+      }
+      best = f[m];
+      /* backtrack: the cuts are v at the start index of every stratum but the first */
+      uint64_t nc = best - 1;
+      if (cuts && total_cuts + nc <= cuts_cap) {
+        uint64_t j = m, w = total_cuts + nc;
+        while (j > 0) {
+          uint64_t i = arg[j];
+          if (i > 0) cuts[--w] = v[i];
+          j = i;
+        }
+      }
+      total_cuts += nc;
+    }
+    counts[k] = best;
+    free(f); free(arg); free(N); free(S1); free(S2); free(v); free(c);
+  }
+  free(vals);
+  if (n_cuts) *n_cuts = total_cuts;
+  if (cuts && total_cuts > cuts_cap) return OR_ERANGE;
+  return OR_OK;
+}
+
 /* accessors */
 uint64_t oracle_strata_count(const oracle_result* R) { return R->n_strata; }
 void oracle_strata_copy(const oracle_result* R, oracle_stratum* dst) {
