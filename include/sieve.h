@@ -261,6 +261,23 @@ int sieve_timing_get(sieve_ctx ctx, uint32_t phase, double* ms, uint64_t* calls,
 /* number of kernels this process has launched through the library (all contexts) */
 uint64_t sieve_kernel_launches(void);
 
+/* ---- exact minimum number of strata (NEXT-3; reading A28) -------------- */
+/* P:89 asks the Tier-3 split to "(1) minimise the number of strata such that (2) the CoV of
+   each stratum is below theta".  This diagnostic computes that optimum exactly, per kernel,
+   over runs of its sorted distinct instruction counts: f(0) = 0, f(j) = min f(i) + 1 over the
+   runs (i, j] with CoV < theta (the exact u256 test of the tiering), ties -> smallest i.
+     counts      HOST [num_kernels]: 0 = no invocations, 1 = Tier-1/2 (one valid stratum), the
+                 optimum for Tier-3 kernels, UINT32_MAX = skipped (more than max_distinct
+                 distinct values; 0 selects 16384 -- the DP is O(m^2) per kernel)
+     cuts        nullable HOST [cuts_cap]: per kernel in id order, the lowest instruction count
+                 of every optimal stratum but the first, ascending (the canonical optimum: the
+                 backtrack from the top takes the smallest start at every step)
+     n_cuts      nullable: total number of cuts (call with cuts = NULL to size the buffer)
+   SIEVE_ERANGE if cuts_cap < *n_cuts; SIEVE_ESTATE on a multi-rank context (single-rank
+   diagnostic).  Synchronises the stream. */
+int sieve_min_strata(sieve_trace t, uint32_t theta_num, uint32_t theta_den, uint32_t max_distinct,
+                     uint32_t* counts, uint64_t* cuts, uint64_t cuts_cap, uint64_t* n_cuts);
+
 /* ---- within-stratum cycle variability (Fig. 4; NEXT-2) ---------------------- */
 /* For every stratum, the coefficient of variation of its members' cycle counts,
    cov_s = sigma_pop(y) / mean(y) = sqrt(n S2 - S1^2) / S1 from exact integer sums (0 if S1 = 0),

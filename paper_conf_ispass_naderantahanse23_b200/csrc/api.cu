@@ -1149,6 +1149,104 @@ extern "C" int sieve_tier_census(sieve_trace t, uint32_t count, const uint32_t* 
   return SIEVE_OK;
 }
 
+// ------------------------------------------------------------------------------------------
+// sieve_min_strata: the exact optimum of P:89's "(1)" (NEXT-3, reading A28)
+// ------------------------------------------------------------------------------------------
+extern "C" int sieve_min_strata(sieve_trace t, uint32_t theta_num, uint32_t theta_den,
+                                uint32_t max_distinct, uint32_t* counts, uint64_t* cuts,
+                                uint64_t cuts_cap, uint64_t* n_cuts) {
+  if (!trace_ok(t) || !counts) return sv_fail(SIEVE_EINVAL, "bad argument");
+  if (!theta_num || !theta_den) return sv_fail(SIEVE_EINVAL, "theta must be a positive fraction");
+  sieve_ctx c = t->ctx;
+  if (c->comm) return sv_fail(SIEVE_ESTATE, "sieve_min_strata is a single-rank diagnostic");
+  cudaStream_t S = c->stream;
+  SV_CUDA(cudaSetDevice(c->device));
+  SV_TRY(arena_reset(c));
+  MomentsHost M;
+  SV_TRY(moments_pass(t, &M));
+  const u32 K = t->K;
+  std::vector<u32> t3rank(K, 0xFFFFFFFFu), t3kid;
+  u64 n3 = 0;
+  for (u32 k = 0; k < K; k++) {
+    const u64* L = &M.lanes[(size_t)k * MOM_LANES];
+    counts[k] = 0;
+    if (!L[0]) continue;
+    counts[k] = 1;
+    if (M.mm[2 * k] == M.mm[2 * k + 1] || cov_lt(L[0], limbs_u128(L + 1), limbs_u128(L + 5), theta_num, theta_den))
+      continue;  // Tier-1/2: one valid stratum
+    t3rank[k] = (u32)t3kid.size();
+    t3kid.push_back(k);
+    n3 += L[0];
+  }
+  const u32 nk = (u32)t3kid.size();
+  u64 total = 0;
+  std::vector<u64> h_cuts;
+  if (nk) {
+    const u32 bx = std::max<u32>(1, bitlen(M.tot[4]));
+    const u64 xmask = (bx >= 64) ? ~0ull : ((1ull << bx) - 1);
+    const int nbits = (int)(bx + bitlen(nk - 1));
+    DBuf<u64> keys(c);
+    DBuf<u32> d_t3rank(c), flag(c), seg(c);
+    DBuf<unsigned long long> counter(c);
+    SV_TRY(counter.alloc(1));
+    SV_TRY(d_t3rank.alloc(K));
+    SV_TRY(h2d(c, d_t3rank.get(), t3rank));
+    SV_TRY(keys.alloc(n3));
+    SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
+    launch_t3_compact(t->kid, t->x, t->n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
+    {
+      DBuf<char> tmp(c);
+      void* pinned;
+      SV_TRY(tmp.alloc(radix_sort_temp_bytes(n3, false)));
+      SV_TRY(pin_alloc(c, &pinned, RADIX_PINNED_BYTES));
+      SV_TRY(radix_sort(keys.get(), nullptr, n3, nbits, tmp.get(), S, pinned));
+    }
+    // run-length encoding: distinct keys, run starts, Tier-3 rank starts
+    DBuf<char> stemp(c);
+    SV_TRY(flag.alloc(n3)); SV_TRY(seg.alloc(n3 + 1)); SV_TRY(stemp.alloc(scan_u32_temp_bytes(n3)));
+    launch_csv_heads(keys.get(), n3, flag.get(), S);
+    scan_u32(flag.get(), seg.get(), n3, stemp.get(), seg.get() + n3, S);
+    std::vector<u32> h_nu;
+    SV_TRY(d2h(c, h_nu, seg.get() + n3, 1));
+    SV_TRY(sync(c));
+    const u64 nu = h_nu[0];
+    DBuf<u64> ukey(c), Pn(c), dcuts(c), doff(c), out(c);
+    DBuf<u32> ustart(c), kstart(c), f(c), arg(c), dcount(c);
+    DBuf<u128> P1(c), P2(c);
+    SV_TRY(ukey.alloc(nu)); SV_TRY(ustart.alloc(nu + 1)); SV_TRY(kstart.alloc(nk + 1));
+    SV_TRY(Pn.alloc(nu + nk)); SV_TRY(P1.alloc(nu + nk)); SV_TRY(P2.alloc(nu + nk));
+    SV_TRY(f.alloc(nu + nk)); SV_TRY(arg.alloc(nu + nk)); SV_TRY(dcount.alloc(nk)); SV_TRY(dcuts.alloc(nu));
+    std::vector<u32> ends = {(u32)n3};
+    std::vector<u32> kend = {(u32)nu};
+    SV_TRY(h2d(c, ustart.get() + nu, ends));
+    SV_TRY(h2d(c, kstart.get() + nk, kend));
+    launch_rle(keys.get(), flag.get(), seg.get(), n3, bx, ukey.get(), ustart.get(), kstart.get(), S);
+    const u32 cap = max_distinct ? max_distinct : 16384u;
+    launch_min_strata(ukey.get(), ustart.get(), kstart.get(), nk, xmask, theta_num, theta_den, cap,
+                      Pn.get(), P1.get(), P2.get(), f.get(), arg.get(), dcount.get(), dcuts.get(), S);
+    std::vector<u32> h_count;
+    SV_TRY(d2h(c, h_count, dcount.get(), nk));
+    SV_TRY(sync(c));
+    SV_CUDA(cudaGetLastError());
+    std::vector<u64> off(nk);
+    for (u32 r = 0; r < nk; r++) {
+      off[r] = total;
+      counts[t3kid[r]] = h_count[r];
+      if (h_count[r] >= 2 && h_count[r] != 0xFFFFFFFFu) total += h_count[r] - 1;
+    }
+    if (cuts && total && total <= cuts_cap) {
+      SV_TRY(doff.alloc(nk)); SV_TRY(out.alloc(total));
+      SV_TRY(h2d(c, doff.get(), off));
+      launch_dp_gather(kstart.get(), dcount.get(), doff.get(), dcuts.get(), nk, out.get(), S);
+      SV_TRY(d2h_raw(c, cuts, out.get(), total * 8));
+      SV_TRY(sync(c));
+    }
+  }
+  if (n_cuts) *n_cuts = total;
+  if (cuts && total > cuts_cap) return sv_fail(SIEVE_ERANGE, "cuts_cap is smaller than *n_cuts");
+  return SIEVE_OK;
+}
+
 extern "C" int sieve_strata_count(sieve_strata s, uint64_t* n) {
   if (!strata_ok(s) || !n) return sv_fail(SIEVE_EINVAL, "bad strata handle");
   *n = s->st.size();

@@ -1,0 +1,222 @@
+// dp.cu -- exact minimum number of strata ("(1) minimises
+// the number of strata such that (2) the CoV of each stratum is below theta"; A28).
+//
+// Per Tier-3 kernel, over its distinct instruction counts (run-length encoded from the sorted
+// Tier-3 keys): f(0) = 0, f(j) = min { f(i) + 1 : CoV(values i+1..j) < theta }, ties -> the
+// smallest i; the backtrack from m gives the canonical optimal cuts.  One 1024-thread block per
+// kernel: block-wide u128 prefix sums of (count, count*v, count*v^2), then the O(m^2) DP with
+// the threads spread over i for every j (one block-wide min per j).  Each (i, j) test is the
+// exact u256 comparison q^2 (n S2 - S1^2) < p^2 S1^2, decided in fp64 when the ratio is
+// further than 1e-12 (relative) from the boundary -- far beyond the fp64 error of the ratio
+// (< 8 ulp), so the decision is always the exact one.
+#include "kernels.cuh"
+
+#define DP_THREADS 1024
+
+struct U256 { u64 w[4]; };
+
+__device__ __forceinline__ U256 mul128(u128 a, u128 b) {
+  u64 a0 = (u64)a, a1 = (u64)(a >> 64), b0 = (u64)b, b1 = (u64)(b >> 64);
+  u128 p00 = (u128)a0 * b0, p01 = (u128)a0 * b1, p10 = (u128)a1 * b0, p11 = (u128)a1 * b1;
+  U256 r;
+  r.w[0] = (u64)p00;
+  u128 mid = (p00 >> 64) + (u64)p01 + (u64)p10;
+  r.w[1] = (u64)mid;
+  u128 hi = (mid >> 64) + (p01 >> 64) + (p10 >> 64) + p11;
+  r.w[2] = (u64)hi;
+  r.w[3] = (u64)(hi >> 64);
+  return r;
+}
+__device__ __forceinline__ U256 mul_u64(U256 a, u64 m) {
+  U256 r;
+  u128 c = 0;
+#pragma unroll
+  for (int i = 0; i < 4; i++) {
+    u128 t = (u128)a.w[i] * m + c;
+    r.w[i] = (u64)t;
+    c = t >> 64;
+  }
+  return r;
+}
+__device__ __forceinline__ U256 sub256(U256 a, U256 b) {
+  U256 r;
+  u64 br = 0;
+#pragma unroll
+  for (int i = 0; i < 4; i++) {
+    u64 t = a.w[i] - b.w[i];
+    u64 b1 = a.w[i] < b.w[i];
+    r.w[i] = t - br;
+    br = b1 | (t < br);
+  }
+  return r;
+}
+__device__ __forceinline__ bool lt256(U256 a, U256 b) {
+#pragma unroll
+  for (int i = 3; i >= 0; i--)
+    if (a.w[i] != b.w[i]) return a.w[i] < b.w[i];
+  return false;
+}
+__device__ __forceinline__ double to_d(u128 v) {
+  return fma((double)(u64)(v >> 64), 18446744073709551616.0, (double)(u64)v);
+}
+
+// CoV < p/q of a run with n values, sums s1, s2 (exact decision; fp64 fast path)
+__device__ __forceinline__ bool run_ok(u64 n, u128 s1, u128 s2, u32 p, u32 q, double bound) {
+  double d1 = to_d(s1);
+  double r = ((double)n * to_d(s2)) / (d1 * d1);  // = 1 + CoV^2
+  if (r < bound * (1.0 - 1e-12)) return true;
+  if (r > bound * (1.0 + 1e-12)) return false;
+  U256 nS2 = mul128((u128)n, s2);
+  U256 sq = mul128(s1, s1);
+  U256 lhs = mul_u64(sub256(nS2, sq), (u64)q * q);
+  U256 rhs = mul_u64(sq, (u64)p * p);
+  return lt256(lhs, rhs);
+}
+
+__device__ __forceinline__ u64 block_min_u64(u64 v, u64* red) {
+  for (int o = 16; o > 0; o >>= 1) {
+    u64 w = __shfl_xor_sync(0xffffffffu, v, o);
+    v = w < v ? w : v;
+  }
+  if (lane_id() == 0) red[threadIdx.x >> 5] = v;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    v = threadIdx.x < (DP_THREADS / 32) ? red[threadIdx.x] : ~0ull;
+    for (int o = 16; o > 0; o >>= 1) {
+      u64 w = __shfl_xor_sync(0xffffffffu, v, o);
+      v = w < v ? w : v;
+    }
+    if (threadIdx.x == 0) red[32] = v;
+  }
+  __syncthreads();
+  u64 r = red[32];
+  return r;
+}
+
+// per Tier-3 rank r: distinct values ukey[kstart[r] .. kstart[r+1]), run starts ustart[] (with
+// ustart[nu] = nkeys).  Scratch at offset kstart[r] + r: prefix arrays of m + 1 entries.
+__global__ void __launch_bounds__(DP_THREADS)
+k_min_strata(const u64* __restrict__ ukey, const u32* __restrict__ ustart, const u32* __restrict__ kstart,
+             u64 xmask, u32 p, u32 q, u32 max_distinct, u64* __restrict__ Pn, u128* __restrict__ P1,
+             u128* __restrict__ P2, u32* __restrict__ f, u32* __restrict__ arg, u32* __restrict__ count,
+             u64* __restrict__ cuts) {
+  __shared__ u64 s_n[DP_THREADS];
+  __shared__ u128 s_1[DP_THREADS], s_2[DP_THREADS];
+  __shared__ u64 red[33];
+  const u32 r = blockIdx.x;
+  const u32 b = kstart[r], m = kstart[r + 1] - b;
+  const u64 off = (u64)b + r;
+  const double bound = 1.0 + ((double)p * p) / ((double)q * q);
+  // whole kernel valid?  (never for a Tier-3 kernel, but cheap and keeps the kernel general)
+  // prefix sums: thread t owns a contiguous chunk
+  const u32 T = DP_THREADS, t = threadIdx.x;
+  const u32 chunk = (m + T - 1) / T;
+  const u32 c0 = min(m, t * chunk), c1 = min(m, c0 + chunk);
+  u64 ln = 0;
+  u128 l1 = 0, l2 = 0;
+  for (u32 i = c0; i < c1; i++) {
+    u64 v = ukey[b + i] & xmask, c = ustart[b + i + 1] - ustart[b + i];
+    ln += c;
+    l1 += (u128)c * v;
+    l2 += (u128)c * ((u128)v * v);
+  }
+  s_n[t] = ln; s_1[t] = l1; s_2[t] = l2;
+  __syncthreads();
+  if (t == 0) {
+    u64 an = 0;
+    u128 a1 = 0, a2 = 0;
+    for (u32 w = 0; w < T; w++) {
+      u64 xn = s_n[w]; u128 x1 = s_1[w], x2 = s_2[w];
+      s_n[w] = an; s_1[w] = a1; s_2[w] = a2;
+      an += xn; a1 += x1; a2 += x2;
+    }
+  }
+  __syncthreads();
+  ln = s_n[t]; l1 = s_1[t]; l2 = s_2[t];
+  for (u32 i = c0; i < c1; i++) {
+    Pn[off + i] = ln; P1[off + i] = l1; P2[off + i] = l2;
+    u64 v = ukey[b + i] & xmask, c = ustart[b + i + 1] - ustart[b + i];
+    ln += c;
+    l1 += (u128)c * v;
+    l2 += (u128)c * ((u128)v * v);
+  }
+  if (c1 == m && (c0 < c1 || t == 0)) { Pn[off + m] = ln; P1[off + m] = l1; P2[off + m] = l2; }
+  if (t == 0) f[off] = 0;
+  __syncthreads();
+  if (run_ok(Pn[off + m], P1[off + m], P2[off + m], p, q, bound)) {
+    if (t == 0) count[r] = 1;
+    return;
+  }
+  if (m > max_distinct) {
+    if (t == 0) count[r] = 0xFFFFFFFFu;
+    return;
+  }
+  for (u32 j = 1; j <= m; j++) {
+    const u64 nj = Pn[off + j];
+    const u128 sj1 = P1[off + j], sj2 = P2[off + j];
+    // candidate i = j - 1 (one distinct value) is always valid: an upper bound for pruning
+    const u32 ub = f[off + j - 1] + 1;
+    u64 best = ((u64)ub << 32) | (j - 1);
+    for (u32 i = t; i + 1 < j; i += T) {
+      u32 fi = f[off + i];
+      if (fi + 1 > ub) continue;          // cannot beat (or tie) i = j - 1 with a smaller i
+      u64 key = ((u64)(fi + 1) << 32) | i;
+      if (key >= best) continue;
+      if (run_ok(nj - Pn[off + i], sj1 - P1[off + i], sj2 - P2[off + i], p, q, bound)) best = key;
+    }
+    best = block_min_u64(best, red);
+    if (t == 0) { f[off + j] = (u32)(best >> 32); arg[off + j] = (u32)best; }
+    __syncthreads();
+  }
+  if (t == 0) {
+    u32 fm = f[off + m];
+    count[r] = fm;
+    // cuts (lowest value of every stratum but the first), ascending, at cuts[b .. b + fm - 1)
+    u32 j = m, w = fm - 1;
+    while (j > 0) {
+      u32 i = arg[off + j];
+      if (i > 0) cuts[b + (--w)] = ukey[b + i] & xmask;
+      j = i;
+    }
+  }
+}
+
+// run heads of sorted keys -> unique keys, run starts (ustart[nu] = n), Tier-3 rank starts
+__global__ void k_rle(const u64* __restrict__ keys, const u32* __restrict__ flag,
+                      const u32* __restrict__ seg, u64 n, u32 bx, u64* __restrict__ ukey,
+                      u32* __restrict__ ustart, u32* __restrict__ kstart) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n || !flag[i]) return;
+  u32 d = seg[i];
+  u64 k = keys[i];
+  ukey[d] = k;
+  ustart[d] = (u32)i;
+  if (i == 0 || (keys[i - 1] >> bx) != (k >> bx)) kstart[k >> bx] = d;
+}
+
+__global__ void k_dp_gather(const u32* __restrict__ kstart, const u32* __restrict__ count,
+                            const u64* __restrict__ off, const u64* __restrict__ cuts,
+                            u64* __restrict__ out) {
+  const u32 r = blockIdx.x;
+  const u32 c = count[r];
+  if (c < 2 || c == 0xFFFFFFFFu) return;
+  for (u32 i = threadIdx.x; i + 1 < c; i += blockDim.x) out[off[r] + i] = cuts[kstart[r] + i];
+}
+
+void launch_rle(const u64* keys, const u32* flag, const u32* seg, u64 n, u32 bx, u64* ukey,
+                u32* ustart, u32* kstart, cudaStream_t s) {
+  if (n) SV_LAUNCH(k_rle, div_up(n, 256), 256, 0, s)(keys, flag, seg, n, bx, ukey, ustart, kstart);
+}
+
+void launch_min_strata(const u64* ukey, const u32* ustart, const u32* kstart, u32 nk, u64 xmask,
+                       u32 p, u32 q, u32 max_distinct, u64* Pn, u128* P1, u128* P2, u32* f, u32* arg,
+                       u32* count, u64* cuts, cudaStream_t s) {
+  if (nk)
+    SV_LAUNCH(k_min_strata, nk, DP_THREADS, 0, s)(ukey, ustart, kstart, xmask, p, q, max_distinct,
+                                                  Pn, P1, P2, f, arg, count, cuts);
+}
+
+void launch_dp_gather(const u32* kstart, const u32* count, const u64* off, const u64* cuts, u32 nk,
+                      u64* out, cudaStream_t s) {
+  if (nk) SV_LAUNCH(k_dp_gather, nk, 256, 0, s)(kstart, count, off, cuts, out);
+}

@@ -158,6 +158,15 @@ void launch_gather_pairs(const u64* src, const u64* idx, u64 n, u64* dst, cudaSt
 void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s);
 size_t scan_u32_temp_bytes(u64 n);
 
+// ---------------- exact min-strata DP (NEXT-3) --------------------------------------------------
+void launch_rle(const u64* keys, const u32* flag, const u32* seg, u64 n, u32 bx, u64* ukey,
+                u32* ustart, u32* kstart, cudaStream_t s);
+void launch_min_strata(const u64* ukey, const u32* ustart, const u32* kstart, u32 nk, u64 xmask,
+                       u32 p, u32 q, u32 max_distinct, u64* Pn, u128* P1, u128* P2, u32* f, u32* arg,
+                       u32* count, u64* cuts, cudaStream_t s);
+void launch_dp_gather(const u32* kstart, const u32* count, const u64* off, const u64* cuts, u32 nk,
+                      u64* out, cudaStream_t s);
+
 // ---------------- misc -------------------------------------------------------------------------
 void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s);
 // cross-rank encoding of u128 pairs [n][2] <-> 4 limbs [n][4]

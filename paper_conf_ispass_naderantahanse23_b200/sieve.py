@@ -37,7 +37,7 @@ EXPORTED = [
     "sieve_version", "sieve_u128_to_limbs", "sieve_limbs_to_u128", "sieve_ctx_set_timing",
     "sieve_timing_get", "sieve_kernel_launches", "sieve_stratify_sweep", "sieve_tier_census",
     "sieve_predict_multi", "sieve_cycle_cov", "sieve_load_csv", "sieve_trace_copy",
-    "sieve_trace_kernel_names",
+    "sieve_trace_kernel_names", "sieve_min_strata",
 ]
 PHASES = ["moments", "compact", "sort", "prefix", "kde", "refine", "assign", "reps", "predict"]
 
@@ -109,6 +109,7 @@ def _load():
         "sieve_load_csv": ([vp, vp, u64, u32, P(CsvSpec), u64, P(vp), P(u32)], i32),
         "sieve_trace_copy": ([vp, vp, vp, vp, vp, P(u64), P(u32)], i32),
         "sieve_trace_kernel_names": ([vp, vp, u64, P(u64)], i32),
+        "sieve_min_strata": ([vp, u32, u32, u32, vp, vp, u64, P(u64)], i32),
     }
     for name, (args, res) in sig.items():
         f = getattr(L, name)
@@ -243,8 +244,9 @@ def _col(a, dtype, device_ok=True):
 
 
 class Trace:
-    def __init__(self, h, ctx, n, keep):
+    def __init__(self, h, ctx, n, keep, num_kernels=None):
         self._h, self.ctx, self.n, self._keep = h, ctx, n, keep
+        self.num_kernels = num_kernels
 
     def close(self):
         if getattr(self, "_h", None):
@@ -268,7 +270,7 @@ def load_trace(ctx, kernel_id, instr, num_kernels, cta=None, cycles=None, first_
     h = ctypes.c_void_p()
     _check(_L.sieve_load_trace(ctx._h, n, first_id, num_kernels, cols[0][0], cols[1][0], cols[2][0],
                                cols[3][0], mem, ctypes.byref(h)), "sieve_load_trace")
-    return Trace(h, ctx, n, [c[2] for c in cols] if adopt else None)
+    return Trace(h, ctx, n, [c[2] for c in cols] if adopt else None, num_kernels)
 
 
 def load_csv(ctx, data, col_kernel, col_instr, col_cta=-1, col_cycles=-1, header_lines=1,
@@ -290,9 +292,9 @@ def load_csv(ctx, data, col_kernel, col_instr, col_cta=-1, col_cycles=-1, header
     h, nk = ctypes.c_void_p(), ctypes.c_uint32()
     _check(_L.sieve_load_csv(ctx._h, ptr, nbytes, mem, ctypes.byref(spec), first_id, ctypes.byref(h),
                              ctypes.byref(nk)), "sieve_load_csv")
-    n = ctypes.c_uint64()
-    _check(_L.sieve_trace_copy(h, None, None, None, None, ctypes.byref(n), None), "sieve_trace_copy")
-    t = Trace(h, ctx, n.value, None)
+    n, kk = ctypes.c_uint64(), ctypes.c_uint32()
+    _check(_L.sieve_trace_copy(h, None, None, None, None, ctypes.byref(n), ctypes.byref(kk)), "sieve_trace_copy")
+    t = Trace(h, ctx, n.value, None, kk.value)
     need = ctypes.c_uint64()
     _check(_L.sieve_trace_kernel_names(h, None, 0, ctypes.byref(need)), "sieve_trace_kernel_names")
     buf = ctypes.create_string_buffer(max(1, need.value))
@@ -301,6 +303,27 @@ def load_csv(ctx, data, col_kernel, col_instr, col_cta=-1, col_cycles=-1, header
     assert len(names) == nk.value
     t.names = names
     return t, names
+
+
+def min_strata(trace, theta=(2, 5), max_distinct=0, num_kernels=None):
+    """sieve_min_strata (NEXT-3): exact minimum strata per kernel and the canonical optimal
+    cuts -> (counts uint32[K], list of per-kernel cut lists)."""
+    K = num_kernels if num_kernels is not None else trace.num_kernels
+    counts = np.zeros(K, np.uint32)
+    nc = ctypes.c_uint64()
+    cp = counts.ctypes.data_as(ctypes.c_void_p)
+    _check(_L.sieve_min_strata(trace._h, theta[0], theta[1], max_distinct, cp, None, 0, ctypes.byref(nc)),
+           "sieve_min_strata")
+    cuts = np.zeros(max(1, nc.value), np.uint64)
+    _check(_L.sieve_min_strata(trace._h, theta[0], theta[1], max_distinct, cp,
+                               cuts.ctypes.data_as(ctypes.c_void_p), nc.value, ctypes.byref(nc)),
+           "sieve_min_strata")
+    per, o = [], 0
+    for c in counts.tolist():
+        k = c - 1 if 2 <= c < 0xFFFFFFFF else 0
+        per.append([int(v) for v in cuts[o:o + k]])
+        o += k
+    return counts, per
 
 
 def trace_columns(trace, cta=True, cycles=True):
