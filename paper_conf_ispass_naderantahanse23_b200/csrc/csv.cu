@@ -72,7 +72,8 @@ __device__ __forceinline__ bool parse_u64(const unsigned char* p, u32 len, u64* 
   for (u32 i = 0; i < len; i++) {
     unsigned char ch = p[i];
     if (ch >= '0' && ch <= '9') {
-      if (v > (~0ull - 9) / 10) return false;
+      const u64 q = ~0ull / 10;  // 1844674407370955161: v * 10 + d fits iff v < q or v == q, d <= 5
+      if (v > q || (v == q && (u32)(ch - '0') > (u32)(~0ull % 10))) return false;
       v = v * 10 + (ch - '0');
       any = true;
     } else if (ch == ',' || ch == '"' || ch == ' ' || ch == '_' || ch == '\r' || ch == '\t') {

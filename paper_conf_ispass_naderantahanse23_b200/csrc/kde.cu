@@ -35,7 +35,15 @@
 #define KDE_W 8.7            // window half-width in units of h: t > 37 is guaranteed beyond it
 #define KDE_WC 8.602325267042627  // sqrt(74): |z| <= this <=> t <= 37 (term-count diagnostic)
 #define KDE_KCUT 3417        // rint(37 * 64 log2 e) = 3416; index 3417 holds 0
+#ifndef KDE_WARPS
 #define KDE_WARPS 8          // warps per block (independent work-item consumers)
+#endif
+#ifndef KDE_MINB
+#define KDE_MINB 3           // min resident blocks per SM (register budget: 85 / thread)
+#endif
+#ifndef KDE_UNROLL
+#define KDE_UNROLL 8         // terms in flight per lane
+#endif
 #define KDE_V (32 / KDE_TJ)  // value slices per warp
 
 __device__ __forceinline__ double grid_pt(u64 lo, u64 hi, u32 j, u32 G) {
@@ -152,25 +160,31 @@ __constant__ double KDE_EXP2_NEG[64] = {
     0x1.172b83c7d517bp-1, 0x1.1429aaea92de0p-1, 0x1.11301d0125b51p-1, 0x1.0e3ec32d3d1a2p-1,
     0x1.0b5586cf9890fp-1, 0x1.0874518759bc8p-1, 0x1.059b0d3158574p-1, 0x1.02c9a3e778061p-1};
 
+// coefficients without a short (upper-word) immediate form: the constant bank
+__constant__ double c_kde[6] = {C_LOG2E_32, C_LN2_32_HI, C_LN2_32_LO, C_P5, C_P4, C_P3};
+
+struct KdeRegs { double log2e, magic; };  // operands that must sit in registers (see below)
+
 // raw bit pattern of fma(P, S, 2^52); the term is this minus bits(2^52)
 template <bool GUARD>
-__device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, const double* sS) {
+__device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, const double* sS,
+                                         KdeRegs R) {
   double z = __dmul_rn(__dsub_rn(g, xd), inv_h);
   double u = __dmul_rn(z, z);                               // 2t, exactly
-  double kb = __fma_rn(u, C_LOG2E_32, C_MAGIC);             // one rounding: nearest integer
+  double kb = __fma_rn(u, R.log2e, R.magic);                // one rounding: nearest integer
   double kf = __dsub_rn(kb, C_MAGIC);
   // k = rint(u * 32 log2 e); any k >= 3417 (t > 37) maps to the zero entry.  The low word of kb
   // is k while k < 2^32, i.e. u < 9.3e7: the host proves |z| < 9645 for every (lane, value)
-  // pair of a launch when max Delta/h < 300 (window 8.7 h plus KDE_TJ-1 = 31 grid steps) and runs the
-  // unguarded variant; otherwise any u >= 80 is sent to the zero entry explicitly.  p stays
-  // finite for every input the API admits (x < 2^44, n < 2^36 => h > 2^-26, u < 2^140), and
-  // fma(p, 0, 2^52) = 2^52.
+  // pair of a launch when max Delta/h < 300 (window 8.7 h plus KDE_TJ-1 = 31 grid steps) and
+  // runs the unguarded variant; otherwise any u >= 80 is sent to the zero entry explicitly.  p
+  // stays finite for every input the API admits (x < 2^44, n < 2^36 => h > 2^-26, u < 2^140),
+  // and fma(p, 0, 2^52) = 2^52.
   u32 k = min((u32)__double2loint(kb), (u32)KDE_KCUT);
   if (GUARD) k = (u32)__double2hiint(u) >= 0x40540000u ? (u32)KDE_KCUT : k;
-  double r = __fma_rn(-kf, C_LN2_32_HI, u);
-  r = __fma_rn(-kf, C_LN2_32_LO, r);
-  double p = __fma_rn(C_P5, r, C_P4);
-  p = __fma_rn(p, r, C_P3);
+  double r = __fma_rn(-kf, c_kde[1], u);
+  r = __fma_rn(-kf, c_kde[2], r);
+  double p = __fma_rn(c_kde[3], r, c_kde[4]);
+  p = __fma_rn(p, r, c_kde[5]);
   p = __fma_rn(p, r, C_P2);
   p = __fma_rn(p, r, C_P1);
   p = __fma_rn(p, r, C_P0);
@@ -185,7 +199,7 @@ __device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, cons
 // shuffles.  (Measured: 32 x 1 beats 8 x 4 -- the narrower value window of 8 x 4 saves ~10%
 // out-of-window terms but quadruples the per-item overhead at equal chunk size.)
 template <bool GUARD>
-__global__ void __launch_bounds__(32 * KDE_WARPS)
+__global__ void __launch_bounds__(32 * KDE_WARPS, KDE_MINB)
 k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ keys, u64 xmask,
       const u64* __restrict__ tile_range, const u32* __restrict__ tile_items,
       const u32* __restrict__ item_tile, u32 ntiles, u64* D, unsigned long long* counter,
@@ -204,6 +218,11 @@ k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ k
   __syncthreads();
   const u32 lane = lane_id();
   u64 inwin = 0;
+  // the fma that forms kb has two constant operands and a DFMA takes at most one constant:
+  // load both into registers once (opaque to the compiler, so it cannot re-materialise them)
+  KdeRegs R;
+  asm volatile("mov.b64 %0, %1;" : "=d"(R.log2e) : "d"(c_kde[0]));
+  asm volatile("mov.b64 %0, %1;" : "=d"(R.magic) : "d"(C_MAGIC));
   for (;;) {
     u32 item = 0;
     if (lane == 0) item = (u32)atomicAdd(counter, 1ull);
@@ -223,14 +242,25 @@ k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ k
     double gj = grid_pt(g.lo, g.hi, j < G ? j : G - 1, G);
     u64 acc = 0;
     u32 i = slice;
+    const double* sSb = sS;
+#if KDE_UNROLL > 4
+    for (; i + (KDE_UNROLL - 1) * KDE_V < len; i += KDE_UNROLL * KDE_V) {
+      u64 b[KDE_UNROLL];
+#pragma unroll
+      for (int q = 0; q < KDE_UNROLL; q++) b[q] = kde_qbits<GUARD>(gj, sx[i + q * KDE_V], inv_h, sSb, R);
+#pragma unroll
+      for (int q = 1; q < KDE_UNROLL; q++) b[0] += b[q];  // integer sums: order is irrelevant
+      acc += b[0];
+    }
+#endif
     for (; i + 3 * KDE_V < len; i += 4 * KDE_V) {
-      u64 b0 = kde_qbits<GUARD>(gj, sx[i], inv_h, sS);
-      u64 b1 = kde_qbits<GUARD>(gj, sx[i + KDE_V], inv_h, sS);
-      u64 b2 = kde_qbits<GUARD>(gj, sx[i + 2 * KDE_V], inv_h, sS);
-      u64 b3 = kde_qbits<GUARD>(gj, sx[i + 3 * KDE_V], inv_h, sS);
+      u64 b0 = kde_qbits<GUARD>(gj, sx[i], inv_h, sSb, R);
+      u64 b1 = kde_qbits<GUARD>(gj, sx[i + KDE_V], inv_h, sSb, R);
+      u64 b2 = kde_qbits<GUARD>(gj, sx[i + 2 * KDE_V], inv_h, sSb, R);
+      u64 b3 = kde_qbits<GUARD>(gj, sx[i + 3 * KDE_V], inv_h, sSb, R);
       acc += (b0 + b1) + (b2 + b3);
     }
-    for (; i < len; i += KDE_V) acc += kde_qbits<GUARD>(gj, sx[i], inv_h, sS);
+    for (; i < len; i += KDE_V) acc += kde_qbits<GUARD>(gj, sx[i], inv_h, sSb, R);
     // remove 2^52's bit pattern once per term this lane evaluated, then sum the value slices
     u32 nterm = len > slice ? (len - slice + KDE_V - 1) / KDE_V : 0;
     acc -= (u64)nterm * 0x4330000000000000ull;

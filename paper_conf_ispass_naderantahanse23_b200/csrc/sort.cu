@@ -252,7 +252,15 @@ k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int s
     u64 i = base + (u64)r * 32 + lane_id();
     bool ok = i < n;
     u32 d = ok ? (u32)(key[r] >> shift) & 255u : 256u;
-    u32 peers = __match_any_sync(0xffffffffu, d);
+    // lanes with the same digit: 8 ballots (one per digit bit) plus validity, ANDed -- cheaper
+    // than MATCH.ANY, which serialises in the MIO pipe
+    u32 peers = __ballot_sync(0xffffffffu, ok);
+    if (!ok) peers = ~peers;
+#pragma unroll
+    for (int b = 0; b < 8; b++) {
+      u32 m = __ballot_sync(0xffffffffu, (d >> b) & 1u);
+      peers &= ((d >> b) & 1u) ? m : ~m;
+    }
     u32 lt = peers & ((1u << lane_id()) - 1u);
     u32 cur = d < 256u ? s_wh[w][d] : 0;
     rank[r] = cur + __popc(lt);

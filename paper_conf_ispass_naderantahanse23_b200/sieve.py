@@ -16,7 +16,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsieve.so")
+# SIEVE_LIB_PATH: an alternative build of the same library (A/B measurements of kernel variants)
+LIB_PATH = os.environ.get("SIEVE_LIB_PATH") or os.path.join(_HERE, "libsieve.so")
 
 SIEVE_OK, SIEVE_EINVAL, SIEVE_ERANGE, SIEVE_ENOMEM = 0, -1, -2, -3
 SIEVE_ECUDA, SIEVE_ENCCL, SIEVE_EDOM, SIEVE_ELIMIT, SIEVE_ESTATE = -4, -5, -6, -7, -8

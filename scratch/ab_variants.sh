@@ -1,0 +1,9 @@
+#!/bin/bash
+# A/B: bench.py phase times for every build/variants/libsieve_*.so (and the default build)
+for so in default build/variants/libsieve_*.so; do
+  if [ "$so" = default ]; then unset SIEVE_LIB_PATH; else export SIEVE_LIB_PATH=$PWD/$so; fi
+  timeout 300 python bench.py --steps 10 --warmup 3 --no-e2e --no-cpu-baseline 2>/dev/null | python -c "
+import json,sys
+d=json.loads(sys.stdin.read())
+print('$so', round(d['ms_per_step'],3), 'kde', round(d['phases']['kde']['ms_per_step'],3), 'frac', round(d['roofline']['frac'],4), 'sort', round(d['phases']['sort']['ms_per_step'],3))"
+done

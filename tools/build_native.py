@@ -71,6 +71,27 @@ def build_lib(force=False):
     return out
 
 
+def build_variant(name, source, defines):
+    """A/B builds: the library with one source compiled under extra -D flags, written to
+    build/variants/libsieve_<name>.so (select it with SIEVE_LIB_PATH)."""
+    build_lib()
+    objdir = os.path.join(ROOT, "build", "obj")
+    vdir = os.path.join(ROOT, "build", "variants")
+    os.makedirs(vdir, exist_ok=True)
+    objs = []
+    for s in cuda_sources():
+        o = os.path.join(objdir, os.path.basename(s) + ".o")
+        if os.path.basename(s) == source:
+            o = os.path.join(vdir, f"{name}_{source}.o")
+            _run([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-ffp-contract=off",
+                  *[f"-D{d}" for d in defines], "-I", os.path.join(ROOT, "include"),
+                  "-I", os.path.join(PKG, "csrc"), "-x", "cu", "-c", s, "-o", o])
+        objs.append(o)
+    out = os.path.join(vdir, f"libsieve_{name}.so")
+    _run([NVCC, *ARCH, "-shared", "-o", out, *objs, "-lcudart_static", "-ldl", "-lpthread", "-lrt"])
+    return out
+
+
 def build_all(force=False):
     build_gen(force)
     build_oracle(force)
