@@ -13,8 +13,15 @@
 
 #include "kernels.cuh"
 
+#ifndef RS_THREADS
 #define RS_THREADS 256
+#endif
+#ifndef RS_IPT
 #define RS_IPT 16
+#endif
+#ifndef RS_MINB
+#define RS_MINB 2
+#endif
 #define RS_TILE (RS_THREADS * RS_IPT)
 #define RS_WARPS (RS_THREADS / 32)
 
@@ -190,6 +197,9 @@ void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u
 #define OS_FLAG_PREFIX (2ull << 62)
 #define OS_VALUE_MASK ((1ull << 62) - 1)
 #define OS_MAX_PASSES 8
+#ifndef OS_LB
+#define OS_LB 4   // predecessors read per look-back step
+#endif
 
 __global__ void __launch_bounds__(RS_THREADS)
 k_os_hist(const u64* __restrict__ keys, u64 n, int npass, u32* __restrict__ ghist) {
@@ -210,17 +220,19 @@ k_os_hist(const u64* __restrict__ keys, u64 n, int npass, u32* __restrict__ ghis
   }
 }
 
+// look-back status words: GPU-scope relaxed accesses (served by L2; volatile would be
+// system scope).  Each word is written whole, so a reader sees either 0 or a complete value.
 __device__ __forceinline__ u64 ld_volatile_u64(const u64* p) {
   u64 v;
-  asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
 __device__ __forceinline__ void st_volatile_u64(u64* p, u64 v) {
-  asm volatile("st.volatile.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
 template <bool V>  // V: a u32 payload travels with each key
-__global__ void __launch_bounds__(RS_THREADS)
+__global__ void __launch_bounds__(RS_THREADS, RS_MINB)
 k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int shift,
           const u32* __restrict__ gbase, u64* status, u32* tile_counter, u64* __restrict__ kout,
           u32* __restrict__ vout) {
@@ -280,11 +292,21 @@ k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int s
       st_volatile_u64(my, OS_FLAG_PREFIX | run);
     } else {
       st_volatile_u64(my, OS_FLAG_AGG | run);
-      for (u32 j = tile - 1;; j--) {
-        u64 v;
-        do { v = ld_volatile_u64(status + (u64)j * 256 + d); } while ((v >> 62) == 0);
-        excl += v & OS_VALUE_MASK;
-        if (v & OS_FLAG_PREFIX) break;
+      // look back OS_LB predecessors at a time: their status loads are in flight together
+      // (each is an L2 round trip, possibly to the other die)
+      bool done = false;
+      for (int j0 = (int)tile - 1; !done; j0 -= OS_LB) {
+        u64 v[OS_LB];
+#pragma unroll
+        for (int q = 0; q < OS_LB; q++)
+          v[q] = j0 - q >= 0 ? ld_volatile_u64(status + (u64)(j0 - q) * 256 + d) : OS_FLAG_PREFIX;
+#pragma unroll
+        for (int q = 0; q < OS_LB; q++) {
+          if (done) break;
+          while ((v[q] >> 62) == 0) v[q] = ld_volatile_u64(status + (u64)(j0 - q) * 256 + d);
+          excl += v[q] & OS_VALUE_MASK;
+          if (v[q] & OS_FLAG_PREFIX) done = true;
+        }
       }
       st_volatile_u64(my, OS_FLAG_PREFIX | (excl + run));
     }
