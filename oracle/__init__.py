@@ -216,7 +216,7 @@ def q_of_t(t):
 
 
 def exp2_table():
-    return [_lib().oracle_exp2_table(j) for j in range(64)]
+    return [_lib().oracle_exp2_table(j) for j in range(256)]
 
 
 def tier(values, theta=(2, 5)):

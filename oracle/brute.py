@@ -14,9 +14,9 @@ Only for tiny traces (a few hundred invocations, small G).
 import math
 from fractions import Fraction
 
-LOG2E_64 = 64.0 * 1.4426950408889634074
-LN2_64_HI = 6.93147180369123816490e-01 / 64.0
-LN2_64_LO = 1.90821492927058770002e-10 / 64.0
+LOG2E_256 = 256.0 * 1.4426950408889634074
+LN2_256 = float.fromhex("0x1.62e42fefa39efp-9")     # rn(ln 2) / 256
+KMAX = 10526
 TWO52 = 2.0 ** 52
 
 
@@ -25,37 +25,43 @@ def fma(a, b, c):
 
 
 def _exp2_neg_table():
-    """2^(-j/64), j = 0..63, correctly rounded (60-digit decimal, then float() rounds)."""
+    """2^(-j/256), j = 0..255, correctly rounded (60-digit decimal, then float() rounds)."""
     from decimal import Decimal, getcontext
     getcontext().prec = 60
-    return [float(Decimal(2) ** (Decimal(-j) / Decimal(64))) for j in range(64)]
+    return [float(Decimal(2) ** (Decimal(-j) / Decimal(256))) for j in range(256)]
 
 
 EXP2_NEG = _exp2_neg_table()
 
 
-def _reduce(t):
-    # nearest integer to the EXACT product t * 64 log2 e (single rounding, ties to even)
-    k = float(round(Fraction(t) * Fraction(LOG2E_64)))
-    r = fma(-k, LN2_64_HI, t)
-    r = fma(-k, LN2_64_LO, r)
-    p = -float(Fraction(1, 120))          # P(r) = sum_{i<=5} (-r)^i / i!  (Horner, signed coefs)
-    for c in (Fraction(1, 24), Fraction(-1, 6), Fraction(1, 2), Fraction(-1), Fraction(1)):
+def _k(t):
+    # nearest integer to the EXACT product t * 256 log2 e (single rounding, ties to even)
+    return round(Fraction(t) * Fraction(LOG2E_256))
+
+
+def _reduce(t, k):
+    r = fma(-float(k), LN2_256, t)
+    p = -float(Fraction(1, 6))           # P(r) = 1 - r + r^2/2 - r^3/6 (Horner, signed coefs)
+    for c in (Fraction(1, 2), Fraction(-1), Fraction(1)):
         p = fma(p, r, float(c))
-    return p, int(k) & 63, int(k) >> 6
+    return p, k & 255, k >> 8
 
 
 def det_exp(t):
-    p, j, m = _reduce(t)
+    k = _k(t)
+    if k > KMAX:
+        return 0.0
+    p, j, m = _reduce(t, k)
     return math.ldexp(p * EXP2_NEG[j], -m)
 
 
 def q_of_t(t):
-    """rint(P * 2^(-j/64) * 2^(52-m)) with a single rounding (exact rational, then round)."""
-    if t > 37.0:
+    """rint(P * 2^(-j/256) * 2^(40-m)) with a single rounding (exact rational, then round)."""
+    k = _k(t)
+    if k > KMAX:
         return 0
-    p, j, m = _reduce(t)
-    v = Fraction(p) * Fraction(EXP2_NEG[j]) * Fraction(2) ** (52 - m)
+    p, j, m = _reduce(t, k)
+    v = Fraction(p) * Fraction(EXP2_NEG[j]) * Fraction(2) ** (40 - m)
     return round(v)                      # Fraction round(): nearest, ties to even
 
 

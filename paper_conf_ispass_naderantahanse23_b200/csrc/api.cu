@@ -785,11 +785,11 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       DBuf<char> item_tile(c);
       SV_TRY(item_tile.alloc(kde_item_bytes(items)));
       PhaseTimer tm(c, SIEVE_PHASE_KDE, 0);
-      // the unguarded KDE variant needs |z| < 9645 for every evaluated pair: window 8.7 h plus
-      // KDE_TJ - 1 grid steps, so max Delta / h < 300 suffices (true for realistic segments)
+      // the unguarded KDE variant needs |z| < 4800 for every evaluated pair: window 7.6 h plus
+      // KDE_TJ - 1 grid steps, so max Delta / h < 150 suffices (true for realistic segments)
       bool guard = false;
       for (u32 s = 0; s < nseg; s++)
-        if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 300.0 * hs[s].h) guard = true;
+        if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 150.0 * hs[s].h) guard = true;
       launch_kde(segs.get(), nseg, G, keys.get(), xmask, tile_range.get(), tile_items.get(),
                  (u32*)item_tile.get(), items, D.get(), counter.get() + 1, terms.get(), guard, S);
       tm.stop();

@@ -11,7 +11,7 @@ import pytest
 import oracle
 from oracle import brute
 
-TWO52 = 2.0 ** 52
+TWO40 = 2.0 ** 40   # A10: densities in units of 2^-40 of one kernel's peak
 
 
 # ---------------------------------------------------------------- O3 tiers
@@ -68,41 +68,48 @@ def test_tier_theta_variants():
 def _decimal_exp2_neg(j):
     from decimal import Decimal, getcontext
     getcontext().prec = 60
-    return float(Decimal(2) ** (Decimal(-j) / Decimal(64)))
+    return float(Decimal(2) ** (Decimal(-j) / Decimal(256)))
 
 
 def test_exp2_tables_correctly_rounded():
     # the oracle's table and the CUDA path's table (kde.cu literals) are each pinned to the
-    # correctly rounded 2^(-j/64); the two sides share no table generator
+    # correctly rounded 2^(-j/256); the two sides share no table generator
     import os
     import re
-    want = [_decimal_exp2_neg(j) for j in range(64)]
+    want = [_decimal_exp2_neg(j) for j in range(256)]
     assert oracle.exp2_table() == want
     src = open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
                             "paper_conf_ispass_naderantahanse23_b200", "csrc", "kde.cu")).read()
-    body = src[src.index("KDE_EXP2_NEG[64]"):]
+    body = src[src.index("KDE_EXP2_NEG[256]"):]
     body = body[body.index("{") + 1:body.index("}")]
     got = [float.fromhex(h) for h in re.findall(r"0x[0-9a-fA-F.]+p[+-]?\d+", body)]
     assert got == want
 
 
-def test_det_exp_within_two_ulp_of_libm():
+def test_det_exp_relative_accuracy():
+    # degree-3 Taylor on |r| <= ln2/512 plus the one-fma reduction: relative error < 2^-42
+    from decimal import Decimal, getcontext
+    getcontext().prec = 40
     rng = random.Random(7)
-    ts = [0.0, 1e-300, 0.5, 1.0, math.log(2), 36.99, 37.0] + [rng.uniform(0, 37) for _ in range(20000)]
+    ts = [0.0, 1e-300, 0.5, 1.0, math.log(2), 28.4, 28.5] + [rng.uniform(0, 28.5) for _ in range(20000)]
     for t in ts:
-        e = math.exp(-t)
-        d = oracle.det_exp(t)
-        assert abs(d - e) <= 2 * math.ulp(e), (t, d, e)
+        e = Decimal(-t).exp()
+        d = Decimal(oracle.det_exp(t))
+        assert abs(d - e) <= e * Decimal(2) ** -42, (t, d, e)
 
 
 def test_q_close_to_exact_exponential():
-    # Q(t) is within 2 units (of 2^-52) of e^{-t} 2^52 over the whole window
+    # Q(t) is within 1 unit (of 2^-40) of e^{-t} 2^40 over the whole window
     from decimal import Decimal, getcontext
     getcontext().prec = 50
     rng = random.Random(9)
-    for t in [0.0, 1e-9, 0.3, 1.0, 5.0, 20.0, 36.9] + [rng.uniform(0, 37) for _ in range(3000)]:
-        exact = (Decimal(-t).exp() * Decimal(2) ** 52)
-        assert abs(Decimal(oracle.q_of_t(t)) - exact) <= 2, t
+    worst = 0
+    for t in [0.0, 1e-9, 0.3, 1.0, 5.0, 20.0, 28.4] + [rng.uniform(0, 28.6) for _ in range(5000)]:
+        exact = (Decimal(-t).exp() * Decimal(2) ** 40)
+        err = abs(Decimal(oracle.q_of_t(t)) - exact)
+        worst = max(worst, err)
+        assert err <= 1, t
+    assert worst > Decimal("0.4")   # the rounding is really to integers at 2^-40
 
 
 def test_q_matches_exact_fma_emulation():
@@ -110,18 +117,20 @@ def test_q_matches_exact_fma_emulation():
     # dropped / added rounding step in the oracle differs somewhere
     rng = random.Random(11)
     for _ in range(2000):
-        t = rng.uniform(0, 37)
+        t = rng.uniform(0, 28.6)
         assert oracle.q_of_t(t) == brute.q_of_t(t)
         assert oracle.det_exp(t) == brute.det_exp(t)
 
 
 def test_q_cutoff_and_peak():
-    assert oracle.q_of_t(0.0) == 2 ** 52
-    assert oracle.q_of_t(37.0) == round(math.exp(-37) * TWO52)   # 0.38 -> 0
-    assert oracle.q_of_t(37.0000001) == 0
-    assert abs(oracle.q_of_t(36.0) - math.exp(-36.0) * TWO52) <= 1
-    # exp(-37) * 2^52 < 0.5: the cutoff drops nothing the rounding would keep
-    assert math.exp(-37) * TWO52 < 0.5
+    assert oracle.q_of_t(0.0) == 2 ** 40
+    assert oracle.q_of_t(1.0) == round(math.exp(-1.0) * TWO40)
+    # k = rint(t 256 log2 e) > 10526 <=> t > 28.5014 -> 0; e^-28.5014 2^40 = 0.46 rounds to 0
+    # anyway, so the cutoff drops nothing the rounding would keep
+    assert oracle.q_of_t(28.5) == 0 and oracle.q_of_t(28.6) == 0 and oracle.q_of_t(1e300) == 0
+    assert math.exp(-28.5) * TWO40 < 0.5
+    assert oracle.q_of_t(27.0) == round(math.exp(-27.0) * TWO40)     # 2.06 -> 2
+    assert oracle.q_of_t(28.0) == round(math.exp(-28.0) * TWO40)     # 0.76 -> 1
 
 
 # ---------------------------------------------------------------- bandwidth ([36]; A8)
@@ -166,7 +175,7 @@ def test_kde_against_sklearn_and_scipy():
     vals = np.clip(np.round(vals), 1, None).astype(np.uint64)
     lo, hi, G = int(vals.min()), int(vals.max()), 256
     h = oracle.bandwidth([int(v) for v in vals])
-    D = np.array([float(d) for d in oracle.kde(vals, lo, hi, h, G)]) / TWO52
+    D = np.array([float(d) for d in oracle.kde(vals, lo, hi, h, G)]) / TWO40
     grid = np.array([oracle.grid_point(lo, hi, j, G) for j in range(G)])
     n = len(vals)
     kd = KernelDensity(kernel="gaussian", bandwidth=h).fit(vals.astype(np.float64)[:, None])
