@@ -37,10 +37,10 @@
 #define KDE_WC 7.54983443527075   // sqrt(57): |z| <= this <=> t <= 28.5 (term-count diagnostic)
 #define KDE_KCUT 10527       // k > 10526 = rint(28.5 * 256 log2 e) -> index 10527 holds 0
 #ifndef KDE_WARPS
-#define KDE_WARPS 8          // warps per block (independent work-item consumers)
+#define KDE_WARPS 12         // warps per block (independent work-item consumers)
 #endif
 #ifndef KDE_MINB
-#define KDE_MINB 3           // min resident blocks per SM (register budget: 85 / thread)
+#define KDE_MINB 2           // resident blocks per SM (84 KB table + 24 KB staging each)
 #endif
 #ifndef KDE_UNROLL
 #define KDE_UNROLL 8         // terms in flight per lane

@@ -65,7 +65,9 @@ struct SegDev {
   u64 begin, end; // local index range in the sorted keys (filled on device)
 };
 #define KDE_TJ 32       // grid points per tile (a work item is one warp's: one point per lane)
+#ifndef KDE_CH
 #define KDE_CH 256      // values per work item chunk (staged in the warp's shared memory)
+#endif
 struct KdeScratch {
   u64* tile_range;     // [nseg*tiles][2]
   u32* tile_items;     // [nseg*tiles + 1] exclusive scan of chunks per tile

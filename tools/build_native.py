@@ -72,8 +72,9 @@ def build_lib(force=False):
 
 
 def build_variant(name, source, defines):
-    """A/B builds: the library with one source compiled under extra -D flags, written to
-    build/variants/libsieve_<name>.so (select it with SIEVE_LIB_PATH)."""
+    """A/B builds: the library with some sources (a file name or a list) compiled under extra
+    -D flags, written to build/variants/libsieve_<name>.so (select it with SIEVE_LIB_PATH)."""
+    sources = [source] if isinstance(source, str) else list(source)
     build_lib()
     objdir = os.path.join(ROOT, "build", "obj")
     vdir = os.path.join(ROOT, "build", "variants")
@@ -81,8 +82,8 @@ def build_variant(name, source, defines):
     objs = []
     for s in cuda_sources():
         o = os.path.join(objdir, os.path.basename(s) + ".o")
-        if os.path.basename(s) == source:
-            o = os.path.join(vdir, f"{name}_{source}.o")
+        if os.path.basename(s) in sources:
+            o = os.path.join(vdir, f"{name}_{os.path.basename(s)}.o")
             _run([NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-ffp-contract=off",
                   *[f"-D{d}" for d in defines], "-I", os.path.join(ROOT, "include"),
                   "-I", os.path.join(PKG, "csrc"), "-x", "cu", "-c", s, "-o", o])
