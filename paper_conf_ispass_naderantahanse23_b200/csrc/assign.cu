@@ -16,7 +16,9 @@
 #include "kernels.cuh"
 
 #define AS_THREADS 1024
-#define AS_IPT 4
+#ifndef AS_IPT
+#define AS_IPT 8
+#endif
 #define AS_HC 8192          // shared hash capacity (entries): 128 KB, one block per SM
 #define AS_FLUSH (3 * AS_HC / 4)      // flush to the L2 table when this full
 #define AS_MAXP 32          // probes before falling back to the global table

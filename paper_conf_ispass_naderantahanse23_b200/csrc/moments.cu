@@ -16,7 +16,9 @@
 #include "kernels.cuh"
 
 #define MOM_THREADS 1024
-#define MOM_U 4                               // rows per thread with loads in flight
+#ifndef MOM_U
+#define MOM_U 2                               // rows per thread with loads in flight (A/B: 2 >= 4, 8 > 16)
+#endif
 #define MOM_KT 2048                           // kernels per shared-memory pass (56 B each)
 #define MOM_LB 15                             // limb bits
 #define MOM_LMASK ((1u << MOM_LB) - 1u)

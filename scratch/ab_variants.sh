@@ -5,5 +5,6 @@ for so in default build/variants/libsieve_*.so; do
   timeout 300 python bench.py --steps 10 --warmup 3 --no-e2e --no-cpu-baseline 2>/dev/null | python -c "
 import json,sys
 d=json.loads(sys.stdin.read())
-print('$so', round(d['ms_per_step'],3), 'kde', round(d['phases']['kde']['ms_per_step'],3), 'frac', round(d['roofline']['frac'],4), 'sort', round(d['phases']['sort']['ms_per_step'],3))"
+ph={k: round(v['ms_per_step'],3) for k,v in d['phases'].items()}
+print('$so', round(d['ms_per_step'],3), ph)"
 done
