@@ -719,9 +719,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       SV_TRY(tmp.alloc(radix_sort_temp_bytes(n3_local, false)));
       PhaseTimer tm(c, SIEVE_PHASE_SORT, 0);
       int passes = 0;
-      void* pinned;
-      SV_TRY(pin_alloc(c, &pinned, RADIX_PINNED_BYTES));
-      SV_TRY(radix_sort(keys.get(), nullptr, n3_local, nbits, tmp.get(), S, pinned, &passes));
+      SV_TRY(radix_sort(keys.get(), nullptr, n3_local, nbits, tmp.get(), S, &passes));
       if (c->timing) c->acc[SIEVE_PHASE_SORT].work += (u64)passes * n3_local * 16;
     }
     SV_TRY(Pb.alloc(4 * block_prefix_entries(n3_local)));
@@ -811,38 +809,41 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
                    ntk.get() + nseg, S);
     tv.stop();
     std::vector<u32> h_ntk;
-    SV_TRY(d2h(c, h_ntk, ntk.get(), (size_t)nseg * 2));
-    SV_TRY(sync(c));
-    std::vector<u32> part_off(nseg + 1);
+    std::vector<u64> h_pl, h_pmin, h_pmax, h_ab, h_D, h_T;
+    std::vector<u32> part_off;
     u32 nparts = 0;
-    for (u32 s = 0; s < nseg; s++) { part_off[s] = nparts; nparts += h_ntk[s] + 1; }
-    part_off[nseg] = nparts;
-    DBuf<u32> d_off(c);
-    SV_TRY(d_off.alloc(nseg + 1));
-    SV_TRY(h2d(c, d_off.get(), part_off));
-    DBuf<u64> pl(c), pm(c), pab(c);
-    SV_TRY(pl.alloc((size_t)nparts * MOM_LANES));
-    SV_TRY(pm.alloc((size_t)nparts * 2));
-    SV_TRY(pab.alloc((size_t)nparts * 4));
-    PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
-    launch_part_stats(segs.get(), nseg, T.get(), tstride, ntk.get(), d_off.get(), nparts,
-                      nkeys ? keys.get() : nullptr, nkeys, bx, Pb.get(), pl.get(),
-                      pm.get(), pab.get(), S);
-    tp.stop();
-    SV_CUDA(cudaGetLastError());
-    SV_TRY(allreduce(c, pl.get(), (size_t)nparts * MOM_LANES, RED_SUM));   // AR-3
-    SV_TRY(allreduce(c, pm.get(), nparts, RED_MIN));
-    SV_TRY(allreduce(c, pm.get() + nparts, nparts, RED_MAX));
-    std::vector<u64> h_pl, h_pm, h_ab;
-    SV_TRY(d2h(c, h_pl, pl.get(), (size_t)nparts * MOM_LANES));
-    SV_TRY(d2h(c, h_pm, pm.get(), (size_t)nparts * 2));
-    SV_TRY(d2h(c, h_ab, pab.get(), (size_t)nparts * 4));
-    std::vector<u64> h_D, h_T;
-    if (R->keep_debug) {
-      SV_TRY(d2h(c, h_D, D.get(), (size_t)nseg * G * 2));
-      SV_TRY(d2h(c, h_T, T.get(), (size_t)nseg * tstride));
+    {
+      SV_TRY(d2h(c, h_ntk, ntk.get(), (size_t)nseg * 2));
+      SV_TRY(sync(c));
+      part_off.resize(nseg + 1);
+      for (u32 s = 0; s < nseg; s++) { part_off[s] = nparts; nparts += h_ntk[s] + 1; }
+      part_off[nseg] = nparts;
+      DBuf<u32> d_off(c);
+      SV_TRY(d_off.alloc(nseg + 1));
+      SV_TRY(h2d(c, d_off.get(), part_off));
+      DBuf<u64> pl(c), pm(c), pab(c);
+      SV_TRY(pl.alloc((size_t)nparts * MOM_LANES));
+      SV_TRY(pm.alloc((size_t)nparts * 2));
+      SV_TRY(pab.alloc((size_t)nparts * 4));
+      PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
+      launch_part_stats(segs.get(), nseg, T.get(), tstride, ntk.get(), d_off.get(), nparts,
+                        nkeys ? keys.get() : nullptr, nkeys, bx, Pb.get(), pl.get(),
+                        pm.get(), pab.get(), S);
+      tp.stop();
+      SV_CUDA(cudaGetLastError());
+      SV_TRY(allreduce(c, pl.get(), (size_t)nparts * MOM_LANES, RED_SUM));   // AR-3
+      SV_TRY(allreduce(c, pm.get(), nparts, RED_MIN));
+      SV_TRY(allreduce(c, pm.get() + nparts, nparts, RED_MAX));
+      SV_TRY(d2h(c, h_pl, pl.get(), (size_t)nparts * MOM_LANES));
+      SV_TRY(d2h(c, h_pmin, pm.get(), (size_t)nparts));
+      SV_TRY(d2h(c, h_pmax, pm.get() + nparts, (size_t)nparts));
+      SV_TRY(d2h(c, h_ab, pab.get(), (size_t)nparts * 4));
+      if (R->keep_debug) {
+        SV_TRY(d2h(c, h_D, D.get(), (size_t)nseg * G * 2));
+        SV_TRY(d2h(c, h_T, T.get(), (size_t)nseg * tstride));
+      }
+      SV_TRY(sync(c));
     }
-    SV_TRY(sync(c));
     std::vector<OpenSeg> next;
     for (u32 s = 0; s < nseg; s++) {
       if (R->keep_debug) {
@@ -868,7 +869,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         u64 pn = L[0];
         if (!pn) continue;  // empty part: dropped (A13 f)
         u128 s1 = limbs_u128(L + 1), s2 = limbs_u128(L + 5);
-        u64 lo = h_pm[p], hi = h_pm[nparts + p];
+        u64 lo = h_pmin[p], hi = h_pmax[p];
         if (lo == hi || cov_lt(pn, s1, s2, P->theta_num, P->theta_den))
           fin.push_back({open[s].kid, 3, lo, hi, pn, s1, hh[s], round});
         else
@@ -927,8 +928,8 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_CUDA(cudaMemsetAsync(errf.get(), 0, 32, S));
     GHash gh{gkeys.get(), gcnt.get(), gfirst.get(), cap};
     PhaseTimer tb(c, SIEVE_PHASE_ASSIGN, n * (12 + (t->cta ? 4 : 0) + (sid_out ? 4 : 0)));
-    launch_assign(t->kid, t->x, t->cta, n, t->first_id, d_ktab.get(), d_lows.get(), sid_out, gh,
-                  errf.get(), assign_grid(), S);
+    launch_assign(t->kid, t->x, t->cta, n, t->first_id, d_ktab.get(), d_lows.get(), K,
+                  (u32)lows.size(), sid_out, gh, errf.get(), assign_grid(), S);
     tb.stop();
     SV_CUDA(cudaGetLastError());
     SV_TRY(ekey.alloc(cap)); SV_TRY(ecnt.alloc(cap)); SV_TRY(efirst.alloc(cap));
@@ -998,9 +999,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   {
     DBuf<char> tmp(c);
     SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
-    void* pinned;
-    SV_TRY(pin_alloc(c, &pinned, RADIX_PINNED_BYTES));
-    SV_TRY(radix_sort(sk.get(), idx.get(), Etot, 32 + (int)bitlen(ns ? ns - 1 : 0), tmp.get(), S, pinned));
+    SV_TRY(radix_sort(sk.get(), idx.get(), Etot, 32 + (int)bitlen(ns ? ns - 1 : 0), tmp.get(), S));
   }
   launch_gather_u64(ak.get() + Etot, idx.get(), Etot, scnt.get(), S);
   launch_gather_u64(ak.get() + 2 * Etot, idx.get(), Etot, sfirst.get(), S);
@@ -1196,10 +1195,8 @@ extern "C" int sieve_min_strata(sieve_trace t, uint32_t theta_num, uint32_t thet
     launch_t3_compact(t->kid, t->x, t->n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
     {
       DBuf<char> tmp(c);
-      void* pinned;
       SV_TRY(tmp.alloc(radix_sort_temp_bytes(n3, false)));
-      SV_TRY(pin_alloc(c, &pinned, RADIX_PINNED_BYTES));
-      SV_TRY(radix_sort(keys.get(), nullptr, n3, nbits, tmp.get(), S, pinned));
+      SV_TRY(radix_sort(keys.get(), nullptr, n3, nbits, tmp.get(), S));
     }
     // run-length encoding: distinct keys, run starts, Tier-3 rank starts
     DBuf<char> stemp(c);
@@ -1495,8 +1492,7 @@ extern "C" int sieve_load_csv(sieve_ctx ctx, const char* data, uint64_t bytes, u
     {
       DBuf<char> tmp(c);
       if ((st = tmp.alloc(radix_sort_temp_bytes(nrows, true))) != SIEVE_OK) return fail(st);
-      if ((st = pin_alloc(c, &p, RADIX_PINNED_BYTES)) != SIEVE_OK) return fail(st);
-      if ((st = radix_sort(hash.get(), row.get(), nrows, 64, tmp.get(), S, p)) != SIEVE_OK) return fail(st);
+      if ((st = radix_sort(hash.get(), row.get(), nrows, 64, tmp.get(), S)) != SIEVE_OK) return fail(st);
     }
     DBuf<u32> flag(c), seg(c);
     DBuf<char> st2(c);
@@ -1516,8 +1512,7 @@ extern "C" int sieve_load_csv(sieve_ctx ctx, const char* data, uint64_t bytes, u
     {
       DBuf<char> tmp(c);
       if ((st = tmp.alloc(radix_sort_temp_bytes(nd, true))) != SIEVE_OK) return fail(st);
-      if ((st = pin_alloc(c, &p, RADIX_PINNED_BYTES)) != SIEVE_OK) return fail(st);
-      if ((st = radix_sort(fkey.get(), fval.get(), nd, 32, tmp.get(), S, p)) != SIEVE_OK) return fail(st);
+      if ((st = radix_sort(fkey.get(), fval.get(), nd, 32, tmp.get(), S)) != SIEVE_OK) return fail(st);
     }
     launch_csv_ids(fval.get(), nd, id_of.get(), flag.get(), seg.get(), row.get(), nrows, t->kid, S);
     launch_gather_pairs(npos.get(), fkey.get(), nd, names.get(), S);  // first row of each id

@@ -50,15 +50,28 @@ __device__ void ghash_update(GHash gh, u64 key, u64 cnt, u64 first, u64* errflag
   atomicMax((unsigned long long*)&errflags[2], 1ull);  // global table full: caller retries bigger
 }
 
+// SMEM_TAB: the per-kernel table and the strata lower bounds are staged in shared memory next
+// to the hash (every row looks them up; from global memory the dependent loads of the binary
+// search and the LSU queue were the kernel's main stalls)
+#define AS_TAB_BUDGET (96 * 1024)
+template <bool SMEM_TAB>
 __global__ void __launch_bounds__(AS_THREADS)
 k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __restrict__ cta,
-         u64 n, u64 first_id, const KTab* __restrict__ ktab, const u64* __restrict__ lows,
-         u32* __restrict__ sid_out, GHash gh, u64* errflags) {
+         u64 n, u64 first_id, const KTab* __restrict__ g_ktab, const u64* __restrict__ g_lows,
+         u32 K, u32 nlows, u32* __restrict__ sid_out, GHash gh, u64* errflags) {
   extern __shared__ __align__(16) unsigned char smem[];
   u64* hk = (u64*)smem;              // [AS_HC]
   u32* hc = (u32*)(hk + AS_HC);      // [AS_HC]
   u32* hf = hc + AS_HC;              // [AS_HC]
+  KTab* s_ktab = (KTab*)(hf + AS_HC);          // [K]       (SMEM_TAB)
+  u64* s_lows = (u64*)(s_ktab + K);             // [nlows]   (SMEM_TAB)
+  const KTab* ktab = SMEM_TAB ? s_ktab : g_ktab;
+  const u64* lows = SMEM_TAB ? s_lows : g_lows;
   __shared__ u32 s_fill;
+  if (SMEM_TAB) {
+    for (u32 i = threadIdx.x; i < K; i += AS_THREADS) s_ktab[i] = g_ktab[i];
+    for (u32 i = threadIdx.x; i < nlows; i += AS_THREADS) s_lows[i] = g_lows[i];
+  }
   for (u32 i = threadIdx.x; i < AS_HC; i += AS_THREADS) { hk[i] = HASH_EMPTY; hc[i] = 0; hf[i] = 0xFFFFFFFFu; }
   if (threadIdx.x == 0) s_fill = 0;
   __syncthreads();
@@ -137,14 +150,22 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
 }
 
 void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 first_id,
-                   const KTab* ktab, const u64* lows, u32* sid_out, GHash gh, u64* errflags,
-                   int grid, cudaStream_t s) {
+                   const KTab* ktab, const u64* lows, u32 K, u32 nlows, u32* sid_out, GHash gh,
+                   u64* errflags, int grid, cudaStream_t s) {
   if (n == 0) return;
   size_t smem = (size_t)AS_HC * (8 + 4 + 4);
-  cudaFuncSetAttribute(k_assign, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  size_t tab = (size_t)K * sizeof(KTab) + (size_t)nlows * 8;
   u64 maxgrid = (n + (u64)AS_THREADS * AS_IPT - 1) / ((u64)AS_THREADS * AS_IPT);
   if ((u64)grid > maxgrid) grid = (int)maxgrid;
-  SV_LAUNCH(k_assign, grid, AS_THREADS, smem, s)(kid, x, cta, n, first_id, ktab, lows, sid_out, gh, errflags);
+  if (tab <= AS_TAB_BUDGET) {
+    cudaFuncSetAttribute(k_assign<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(smem + tab));
+    SV_LAUNCH(k_assign<true>, grid, AS_THREADS, smem + tab, s)(kid, x, cta, n, first_id, ktab, lows, K,
+                                                                nlows, sid_out, gh, errflags);
+  } else {
+    cudaFuncSetAttribute(k_assign<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    SV_LAUNCH(k_assign<false>, grid, AS_THREADS, smem, s)(kid, x, cta, n, first_id, ktab, lows, K,
+                                                           nlows, sid_out, gh, errflags);
+  }
 }
 
 __global__ void k_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst,

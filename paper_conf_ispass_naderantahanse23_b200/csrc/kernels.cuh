@@ -42,10 +42,9 @@ void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u
 
 // ---------------- LSD radix sort (u64 keys, optional u32 payload) ----------------------------
 size_t radix_sort_temp_bytes(u64 n, bool with_vals);
-// sorts keys[0..n) on bits [0, nbits); result in keys/vals (in place via internal ping-pong)
-// pinned: >= RADIX_PINNED_BYTES of pinned host memory for the one histogram read-back
-#define RADIX_PINNED_BYTES (2 * 8 * 256 * 4)
-int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, void* pinned,
+// sorts keys[0..n) on bits [0, nbits); result in keys/vals (in place via internal ping-pong);
+// stream-ordered, no host synchronisation
+int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s,
                int* passes = nullptr);
 
 // ---------------- prefix sums of x and x^2 over sorted Tier-3 keys -----------------------------
@@ -95,7 +94,6 @@ void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D
 void launch_part_stats(const SegDev* segs, u32 nseg, const u64* T, u32 tstride, const u32* nt,
                        const u32* part_off, u32 nparts, const u64* keys, u64 nkeys, u32 bx,
                        const u64* Pb, u64* lanes, u64* mm, u64* ab, cudaStream_t s);
-
 // ---------------- pass B: assignment + per-(stratum, CTA) statistics -------------------
 struct KTab {      // per kernel
   u32 base;        // global id of its first stratum
@@ -112,8 +110,8 @@ struct GHash {     // global (sid, cta) table
 #define HASH_EMPTY 0xFFFFFFFFFFFFFFFFull
 int assign_grid();
 void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 first_id,
-                   const KTab* ktab, const u64* lows, u32* sid_out, GHash gh, u64* errflags,
-                   int grid, cudaStream_t s);
+                   const KTab* ktab, const u64* lows, u32 K, u32 nlows, u32* sid_out, GHash gh,
+                   u64* errflags, int grid, cudaStream_t s);
 // compact occupied entries into (key, cnt, first) arrays; *count (device) += entries
 void launch_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst, unsigned long long* count,
                          cudaStream_t s);

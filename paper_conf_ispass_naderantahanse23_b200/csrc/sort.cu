@@ -338,6 +338,13 @@ k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int s
   }
 }
 
+// exclusive scan of each pass's 256-bin histogram (one block of 256 threads per pass)
+__global__ void __launch_bounds__(RS_THREADS) k_os_scan(const u32* __restrict__ ghist, u32* __restrict__ gbase) {
+  __shared__ u32 tot;
+  u32 v = ghist[blockIdx.x * 256 + threadIdx.x];
+  gbase[blockIdx.x * 256 + threadIdx.x] = block_excl_scan<u32, RS_THREADS>(v, &tot);
+}
+
 static size_t al256(size_t b) { return (b + 255) / 256 * 256; }
 
 size_t radix_sort_temp_bytes(u64 n, bool with_vals) {
@@ -350,8 +357,7 @@ size_t radix_sort_temp_bytes(u64 n, bool with_vals) {
   return b;
 }
 
-int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, void* pinned,
-               int* passes) {
+int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, int* passes) {
   if (passes) *passes = 0;
   if (n <= 1 || nbits <= 0) return SIEVE_OK;
   if (nbits > 8 * OS_MAX_PASSES) nbits = 8 * OS_MAX_PASSES;
@@ -370,29 +376,16 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   SV_CUDA(cudaFuncSetAttribute(k_os_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsmem));
   u64 hgrid = std::min<u64>((n + RS_THREADS - 1) / RS_THREADS, (u64)sv_num_sms() * 4);
   SV_LAUNCH(k_os_hist, (unsigned)hgrid, RS_THREADS, hsmem, s)(keys, n, npass, ghist);
-  // pinned staging: a pageable copy would block on / synchronise the stream differently
-  u32* h = (u32*)pinned;
-  u32* bases = h + OS_MAX_PASSES * 256;
-  SV_CUDA(cudaMemcpyAsync(h, ghist, (size_t)npass * 256 * 4, cudaMemcpyDeviceToHost, s));
-  SV_CUDA(cudaStreamSynchronize(s));
-  bool active[OS_MAX_PASSES];
-  for (int p = 0; p < npass; p++) {
-    u32 run = 0, nonzero = 0;
-    for (int d = 0; d < 256; d++) {
-      bases[p * 256 + d] = run;
-      run += h[p * 256 + d];
-      nonzero += h[p * 256 + d] != 0;
-    }
-    active[p] = nonzero > 1;  // a single non-empty bin: the pass is the identity
-  }
-  SV_CUDA(cudaMemcpyAsync(gbase, bases, (size_t)npass * 256 * 4, cudaMemcpyHostToDevice, s));
+  // digit bases on the device (no host round trip): every pass runs -- a pass over a digit
+  // that is constant across all keys is a stable identity permutation, so skipping it would only
+  // save time, never change the result
+  SV_LAUNCH(k_os_scan, npass, RS_THREADS, 0, s)(ghist, gbase);
   size_t smem = (size_t)RS_TILE * (vals ? 8 + 4 : 8);
   SV_CUDA(cudaFuncSetAttribute(k_os_pass<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                RS_TILE * (8 + 4)));
   SV_CUDA(cudaFuncSetAttribute(k_os_pass<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, RS_TILE * 8));
   u64* kin = keys; u32* vin = vals; u64* kout = kalt; u32* vout = valt;
   for (int p = 0; p < npass; p++) {
-    if (!active[p]) continue;
     SV_CUDA(cudaMemsetAsync(status, 0, ntiles * 256 * 8, s));
     SV_CUDA(cudaMemsetAsync(tile_counter, 0, 4, s));
     if (vals)
