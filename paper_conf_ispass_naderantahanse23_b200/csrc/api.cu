@@ -95,6 +95,11 @@ struct sieve_ctx_s {
   std::vector<void*> pin_overflow;
   struct Pend { void* dst; void* pinned; size_t bytes; };
   std::vector<Pend> pend;
+  // SIEVE_HOST_TIMING: host-side accounting of the synchronisations of a call
+  int hs_n = 0;
+  double hs_wait = 0, hs_between = 0;
+  std::string hs_list;
+  std::chrono::steady_clock::time_point hs_last{};
 };
 
 static std::atomic<unsigned long long> g_launches{0};
@@ -535,7 +540,27 @@ static int h2d(sieve_ctx c, T* d, const std::vector<T>& h) {
   SV_CUDA(cudaMemcpyAsync(d, p, h.size() * sizeof(T), cudaMemcpyHostToDevice, c->stream));
   return SIEVE_OK;
 }
+static bool host_timing() {
+  static const bool on = getenv("SIEVE_HOST_TIMING") != nullptr;
+  return on;
+}
 static int sync(sieve_ctx c) {
+  if (host_timing()) {
+    auto t0 = std::chrono::steady_clock::now();
+    if (c->hs_n) {
+      double b = std::chrono::duration<double, std::milli>(t0 - c->hs_last).count();
+      c->hs_between += b;
+      char tmp[32];
+      snprintf(tmp, sizeof tmp, " %.3f", b);
+      c->hs_list += tmp;
+    }
+    cudaError_t e = cudaStreamSynchronize(c->stream);
+    auto t1 = std::chrono::steady_clock::now();
+    c->hs_wait += std::chrono::duration<double, std::milli>(t1 - t0).count();
+    c->hs_n++;
+    c->hs_last = t1;
+    SV_CUDA(e);
+  }
   SV_CUDA(cudaStreamSynchronize(c->stream));
   for (auto& q : c->pend) memcpy(q.dst, q.pinned, q.bytes);
   c->pend.clear();
@@ -552,7 +577,8 @@ struct OpenSeg { u32 kid, t3rank; u64 lo, hi, n; u128 s1, s2; u64 b, e; };
 // host-side wall-clock marks (SIEVE_HOST_TIMING=1 prints them to stderr): where the host
 // orchestration, not the device, spends time
 struct HostClock {
-  bool on = getenv("SIEVE_HOST_TIMING") != nullptr;
+  bool on = host_timing();
+  sieve_ctx c = nullptr;
   std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now(), last = t0;
   std::string out;
   void mark(const char* name) {
@@ -564,8 +590,11 @@ struct HostClock {
     last = now;
   }
   ~HostClock() {
-    if (on) fprintf(stderr, "[sieve host ms]%s total=%.3f\n", out.c_str(),
-                    std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    if (!on) return;
+    fprintf(stderr, "[sieve host ms]%s total=%.3f syncs=%d wait=%.3f between=%.3f [%s ]\n", out.c_str(),
+            std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count(),
+            c ? c->hs_n : 0, c ? c->hs_wait : 0.0, c ? c->hs_between : 0.0, c ? c->hs_list.c_str() : "");
+    if (c) { c->hs_n = 0; c->hs_wait = c->hs_between = 0; c->hs_list.clear(); }
   }
 };
 struct Fin { u32 kid, tier; u64 lo, hi, n; u128 s1; double h; u32 round; };
@@ -656,6 +685,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   cudaStream_t S = c->stream;
   SV_TRY(arena_reset(c));
   HostClock hc;
+  hc.c = c;
   const u32 K = t->K, G = P->grid_points;
   const u64 n = t->n;
   MomentsHost own;
@@ -814,7 +844,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     u32 nparts = 0;
     {
       SV_TRY(d2h(c, h_ntk, ntk.get(), (size_t)nseg * 2));
+      hc.mark("v");
       SV_TRY(sync(c));
+      hc.mark("vs");
       part_off.resize(nseg + 1);
       for (u32 s = 0; s < nseg; s++) { part_off[s] = nparts; nparts += h_ntk[s] + 1; }
       part_off[nseg] = nparts;
@@ -842,7 +874,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         SV_TRY(d2h(c, h_D, D.get(), (size_t)nseg * G * 2));
         SV_TRY(d2h(c, h_T, T.get(), (size_t)nseg * tstride));
       }
+      hc.mark("p");
       SV_TRY(sync(c));
+      hc.mark("ps");
     }
     std::vector<OpenSeg> next;
     for (u32 s = 0; s < nseg; s++) {

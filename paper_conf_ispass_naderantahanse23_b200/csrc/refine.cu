@@ -12,50 +12,27 @@ __device__ __forceinline__ double grid_pt_r(u64 lo, u64 hi, u32 j, u32 G) {
                    __ddiv_rn(__ull2double_rn((hi - lo) * (u64)j), __uint2double_rn(G - 1)));
 }
 
-// Valley scan of one segment per warp: the warp stages D in shared memory (coalesced), lane 0
-// runs the two-state hysteresis machine (A11): delta = max(1, max_j D_j >> shift); in seek_max
-// track the running maximum and switch when D_j + delta <= max; in seek_min track the first run
-// of the minimum and emit its midpoint once D_j >= min + delta.  Edges are never valleys.
-#define VAL_WARPS 4
-__global__ void __launch_bounds__(32 * VAL_WARPS)
-k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, u32 tstride,
-          u32* nt, u32* kind) {
-  u32 w = threadIdx.x >> 5;
-  u32 s = blockIdx.x * VAL_WARPS + w;
-  if (s >= nseg) return;
-  const u64* d = D + 2 * (u64)s * G;
-  // max over the segment (warp reduction on u128 as (hi, lo))
-  u128 mx = 0;
-  for (u32 j = lane_id(); j < G; j += 32) {
-    u128 v = ((u128)d[2 * j + 1] << 64) | d[2 * j];
-    mx = v > mx ? v : mx;
-  }
-  for (int o = 16; o > 0; o >>= 1) {
-    u64 lo = __shfl_down_sync(0xffffffffu, (u64)mx, o);
-    u64 hi = __shfl_down_sync(0xffffffffu, (u64)(mx >> 64), o);
-    u128 v = ((u128)hi << 64) | lo;
-    mx = v > mx ? v : mx;
-  }
-  mx = ((u128)__shfl_sync(0xffffffffu, (u64)(mx >> 64), 0) << 64) | __shfl_sync(0xffffffffu, (u64)mx, 0);
-  SegDev g = segs[s];
-  u128 delta = mx >> shift;
+// Valley scan of one segment per warp: the warp stages D in shared memory (coalesced) and
+// reduces its maximum; then lane 0 runs the two-state hysteresis machine (A11) straight from
+// shared memory (the loads do not depend on the state, so they run ahead of the dependent
+// compare chain): delta = max(1, max_j D_j >> shift); in seek_max track the running maximum and
+// switch when D_j + delta <= max; in seek_min track the first run of the minimum and emit its
+// midpoint once D_j >= min + delta.  Edges are never valleys.
+// the state machine over D (values read as (lo, hi) word pairs); V = u64 when every D_j < 2^63
+// (then v + delta cannot wrap), else u128.  Returns the number of thresholds written to Ts.
+template <typename V>
+__device__ __forceinline__ u32 valley_machine(const u64* src, u32 G, V mx, u32 shift, const SegDev& g,
+                                              u64* Ts) {
+  V delta = shift >= 8 * sizeof(V) ? (V)0 : (V)(mx >> shift);
   if (delta < 1) delta = 1;
-  u64* Ts = T + (u64)s * tstride;
   u32 n = 0;
   bool seek_min = false;
-  u128 top = ((u128)d[1] << 64) | d[0], low = 0;
+  V top = sizeof(V) == 8 ? (V)src[0] : (V)(((u128)src[1] << 64) | src[0]), low = 0;
   u32 a = 0, b = 0;
   u64 last_th = 0;
-  // every lane runs the (sequential) state machine on the same values: each 32-value chunk is
-  // one coalesced load, then broadcast value by value with shuffles (uniform control flow)
-  for (u32 j0 = 0; j0 < G; j0 += 32) {
-    u32 jl = j0 + lane_id();
-    u64 clo = jl < G ? d[2 * jl] : 0, chi = jl < G ? d[2 * jl + 1] : 0;
-    u32 cn = min(32u, G - j0);
-    for (u32 q = 0; q < cn; q++) {
-    u32 j = j0 + q;
-    u128 v = ((u128)__shfl_sync(0xffffffffu, chi, q) << 64) | __shfl_sync(0xffffffffu, clo, q);
-    if (j == 0) continue;
+#pragma unroll 4
+  for (u32 j = 1; j < G; j++) {
+    V v = sizeof(V) == 8 ? (V)src[2 * j] : (V)(((u128)src[2 * j + 1] << 64) | src[2 * j]);
     if (!seek_min) {
       if (v > top) top = v;
       if (v + delta <= top) { seek_min = true; low = v; a = b = j; }
@@ -67,7 +44,7 @@ k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, 
         double gm = grid_pt_r(g.lo, g.hi, m, G);
         u64 th = (u64)ceil(gm);
         if (th > g.lo && th <= g.hi && (n == 0 || last_th != th)) {
-          if (lane_id() == 0) Ts[n] = th;
+          Ts[n] = th;
           last_th = th;
           n++;
         }
@@ -75,9 +52,44 @@ k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, 
         top = v;
       }
     }
-    }
   }
+  return n;
+}
+
+#define VAL_WARPS 4
+#define VAL_GMAX 2048   // segments with more grid points fall back to reading D from global memory
+__global__ void __launch_bounds__(32 * VAL_WARPS)
+k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, u32 tstride,
+          u32* nt, u32* kind) {
+  extern __shared__ __align__(16) unsigned char vsm[];
+  u32 w = threadIdx.x >> 5;
+  u32 s = blockIdx.x * VAL_WARPS + w;
+  if (s >= nseg) return;
+  const u64* d = D + 2 * (u64)s * G;
+  const bool staged = G <= VAL_GMAX;
+  u64* sd = (u64*)vsm + (u64)w * 2 * G;
+  // stage + max over the segment (warp reduction on u128 as (hi, lo))
+  u128 mx = 0;
+  for (u32 j = lane_id(); j < G; j += 32) {
+    u64 lo = d[2 * j], hi = d[2 * j + 1];
+    if (staged) { sd[2 * j] = lo; sd[2 * j + 1] = hi; }
+    u128 v = ((u128)hi << 64) | lo;
+    mx = v > mx ? v : mx;
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    u64 lo = __shfl_down_sync(0xffffffffu, (u64)mx, o);
+    u64 hi = __shfl_down_sync(0xffffffffu, (u64)(mx >> 64), o);
+    u128 v = ((u128)hi << 64) | lo;
+    mx = v > mx ? v : mx;
+  }
+  __syncwarp();
   if (lane_id() != 0) return;
+  const u64* src = staged ? sd : d;
+  SegDev g = segs[s];
+  u64* Ts = T + (u64)s * tstride;
+  u32 n = 0;
+  if ((u64)(mx >> 63) == 0) n = valley_machine<u64>(src, G, (u64)mx, shift, g, Ts);  // usual: D < 2^63
+  else n = valley_machine<u128>(src, G, mx, shift, g, Ts);
   u32 k = 1;
   if (n == 0) { Ts[0] = (g.lo + g.hi + 1) >> 1; n = 1; k = 2; }  // value-range bisection (A13)
   nt[s] = n;
@@ -86,8 +98,11 @@ k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, 
 
 void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T,
                     u32 tstride, u32* nt, u32* kind, cudaStream_t s) {
-  if (nseg) SV_LAUNCH(k_valleys, div_up(nseg, VAL_WARPS), 32 * VAL_WARPS, 0, s)(segs, nseg, G, shift, D, T,
-                                                                        tstride, nt, kind);
+  if (!nseg) return;
+  size_t smem = G <= VAL_GMAX ? (size_t)VAL_WARPS * 2 * G * 8 : 0;
+  cudaFuncSetAttribute(k_valleys, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)((size_t)VAL_WARPS * 2 * VAL_GMAX * 8));
+  SV_LAUNCH(k_valleys, div_up(nseg, VAL_WARPS), 32 * VAL_WARPS, smem, s)(segs, nseg, G, shift, D, T,
+                                                                  tstride, nt, kind);
 }
 
 __device__ __forceinline__ u64 lb_u64(const u64* a, u64 b, u64 e, u64 v) {
