@@ -179,8 +179,10 @@ int sieve_strata_count(sieve_strata s, uint64_t* n);
 /* copy min(cap, count) strata to a HOST array */
 int sieve_strata_copy(sieve_strata s, sieve_stratum* host_out, uint64_t cap);
 /* refinement rounds used, KDE terms evaluated (diagnostics) */
-/* rounds: refinement rounds; kde_terms: in-window (|g - x| <= sqrt(74) h) KDE terms;
-   kde_evaluated: (grid point, value) pairs the KDE kernel evaluated (in-window + wasted) */
+/* rounds: refinement rounds; kde_terms: in-window KDE terms, i.e. (grid point j, value x) pairs
+   of every round with rn(g_j - w) <= x <= rn(g_j + w), w = rn(sqrt(57) h) (0 when term counting
+   is off, see sieve_ctx_set_term_count); kde_evaluated: (grid point, value) pairs the KDE kernel
+   evaluated (in-window + wasted) */
 int sieve_strata_stats(sieve_strata s, uint32_t* rounds, uint64_t* kde_terms,
                        uint64_t* kde_evaluated);
 void sieve_strata_free(sieve_strata s);
@@ -247,8 +249,8 @@ int sieve_predict_multi(sieve_strata s, sieve_trace t, uint32_t M, const uint64_
 enum {
   SIEVE_PHASE_MOMENTS = 0, /* pass A: per-kernel moments */
   SIEVE_PHASE_COMPACT = 1, /* Tier-3 key compaction */
-  SIEVE_PHASE_SORT = 2,    /* radix sort of Tier-3 keys */
-  SIEVE_PHASE_PREFIX = 3,  /* u128 prefix sums of x, x^2 */
+  SIEVE_PHASE_SORT = 2,    /* per round: sort of the open segments' values by (segment, grid cell) */
+  SIEVE_PHASE_PREFIX = 3,  /* reserved (0): the former u128 prefix sums */
   SIEVE_PHASE_KDE = 4,     /* fixed-point KDE (all rounds) */
   SIEVE_PHASE_REFINE = 5,  /* valleys + part moments (all rounds) */
   SIEVE_PHASE_ASSIGN = 6,  /* pass B: assignment + (stratum, CTA) statistics */
@@ -257,6 +259,10 @@ enum {
   SIEVE_PHASE_COUNT = 9
 };
 int sieve_ctx_set_timing(sieve_ctx ctx, int enable);
+/* In-window KDE term counting (the KDE's algorithmic work count, sieve_strata_stats), on by
+   default: one per-value grid search per round on top of the cell sort.  It changes no result;
+   a timing loop over identical inputs may count once and switch it off. */
+int sieve_ctx_set_term_count(sieve_ctx ctx, int enable);
 int sieve_timing_get(sieve_ctx ctx, uint32_t phase, double* ms, uint64_t* calls, uint64_t* work);
 /* number of kernels this process has launched through the library (all contexts) */
 uint64_t sieve_kernel_launches(void);

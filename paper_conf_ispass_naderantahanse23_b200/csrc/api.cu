@@ -97,6 +97,7 @@ struct sieve_ctx_s {
   std::vector<Pend> pend;
   // SIEVE_HOST_TIMING: host-side accounting of the synchronisations of a call
   int hs_n = 0;
+  bool count_terms = true;  // in-window KDE term count (sieve_ctx_set_term_count)
   double hs_wait = 0, hs_between = 0;
   std::string hs_list;
   std::chrono::steady_clock::time_point hs_last{};
@@ -149,6 +150,12 @@ extern "C" int sieve_ctx_set_timing(sieve_ctx ctx, int enable) {
   if (!ctx || ctx->magic != CTX_MAGIC) return sv_fail(SIEVE_EINVAL, "bad ctx");
   ctx->timing = enable != 0;
   for (auto& a : ctx->acc) a = PhaseAcc();
+  return SIEVE_OK;
+}
+
+extern "C" int sieve_ctx_set_term_count(sieve_ctx ctx, int enable) {
+  if (!ctx || ctx->magic != CTX_MAGIC) return sv_fail(SIEVE_EINVAL, "bad ctx");
+  ctx->count_terms = enable != 0;
   return SIEVE_OK;
 }
 
@@ -572,7 +579,8 @@ static int sync(sieve_ctx c) {
 // ------------------------------------------------------------------------------------------
 // an open Tier-3 segment: global value range / moments (replicated) and this rank's index
 // range [b, e) in the sorted keys (local)
-struct OpenSeg { u32 kid, t3rank; u64 lo, hi, n; u128 s1, s2; u64 b, e; };
+// rounds > 1: its values are [b, e) of `src` (sorted cell keys, x = key >> src_shift)
+struct OpenSeg { u32 kid, t3rank; u64 lo, hi, n; u128 s1, s2; u64 b, e; const u64* src; u32 src_shift; };
 
 // host-side wall-clock marks (SIEVE_HOST_TIMING=1 prints them to stderr): where the host
 // orchestration, not the device, spends time
@@ -721,17 +729,15 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     } else {                                                     // Tier-3 -> refinement
       t3rank[k] = n_t3++;
       // the sorted keys are grouped by t3rank: this kernel's local range follows the previous
-      open.push_back({k, t3rank[k], lo, hi, nk, s1, s2, n3_local, n3_local + h_localn[k]});
+      open.push_back({k, t3rank[k], lo, hi, nk, s1, s2, n3_local, n3_local + h_localn[k], nullptr, 0});
       n3_local += h_localn[k];
     }
   }
   R->total_instr = I;
 
-  // ---------------- Tier-3 keys: compact, sort, prefix sums ----------------------------------
+  // ---------------- Tier-3 keys: compaction ----------------------------------------------------
   const u32 bx = std::max<u32>(1, bitlen(max_x));
-  const u64 xmask = (bx >= 64) ? ~0ull : ((1ull << bx) - 1);
-  const int nbits = (int)(bx + bitlen(n_t3 ? n_t3 - 1 : 0));
-  DBuf<u64> keys(c), Pb(c);
+  DBuf<u64> keys(c);
   DBuf<u32> d_t3rank(c);
   DBuf<unsigned long long> counter(c);
   SV_TRY(counter.alloc(4));
@@ -740,86 +746,132 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(h2d(c, d_t3rank.get(), t3rank));
     SV_TRY(keys.alloc(n3_local));
     SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
-    {
-      PhaseTimer tm(c, SIEVE_PHASE_COMPACT, n * 12 + n3_local * 8);
-      launch_t3_compact(t->kid, t->x, n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
-    }
-    {
-      DBuf<char> tmp(c);
-      SV_TRY(tmp.alloc(radix_sort_temp_bytes(n3_local, false)));
-      PhaseTimer tm(c, SIEVE_PHASE_SORT, 0);
-      int passes = 0;
-      SV_TRY(radix_sort(keys.get(), nullptr, n3_local, nbits, tmp.get(), S, &passes));
-      if (c->timing) c->acc[SIEVE_PHASE_SORT].work += (u64)passes * n3_local * 16;
-    }
-    SV_TRY(Pb.alloc(4 * block_prefix_entries(n3_local)));
-    {
-      PhaseTimer tm(c, SIEVE_PHASE_PREFIX, n3_local * 8);
-      launch_block_prefix(keys.get(), n3_local, xmask, Pb.get(), S);
-    }
+    PhaseTimer tm(c, SIEVE_PHASE_COMPACT, n * 12 + n3_local * 8);
+    launch_t3_compact(t->kid, t->x, n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
     SV_CUDA(cudaGetLastError());
   }
   const u64 nkeys = (n_t3 && n3_local) ? n3_local : 0;
 
-  hc.mark("sort");
+  hc.mark("compact");
   // ---------------- refinement rounds (A6-A15) ------------------------------------------
+  // Each round sorts the open segments' values by (segment, grid cell) (bucket.cu: the segmented
+  // sort the KDE windows and the part moments need), evaluates the fixed-point KDE, finds the
+  // valleys and reduces the candidate parts exactly.  Round 1 reads the compacted keys (open
+  // segment s = Tier-3 kernel of rank s); round r > 1 reads, for each re-opened part, its range
+  // of whole cells in the sorted keys of round r-1.  The packed sort key (x << ib) | cell index
+  // bounds the cells of one sort by 2^(64 - bx): a round with more open segments than that runs
+  // in batches (the decisions are per segment, so batching changes no result).
   DBuf<unsigned long long> terms(c);
   SV_TRY(terms.alloc(2));
   SV_CUDA(cudaMemsetAsync(terms.get(), 0, 16, S));
   u32 round = 0;
   const u32 tstride = G / 2 + 1;
   const u32 tps = div_up(G, KDE_TJ);
+  const u64 max_cells = bx >= 63 ? 0 : (1ull << (64 - bx)) - 1;  // idx <= ncell must fit
+  if (!open.empty() && max_cells < G) return sv_fail(SIEVE_ELIMIT, "instruction counts too wide for the cell sort key");
+  for (auto& o : open) { o.src = keys.get(); o.src_shift = 0; }
   while (!open.empty()) {
     round++;
     if (round > P->max_rounds) return sv_fail(SIEVE_ELIMIT, "Tier-3 refinement exceeded max_rounds");
-    const u32 nseg = (u32)open.size();
+    std::vector<OpenSeg> next;
+    const u32 nopen = (u32)open.size();
+    u32 batch = (u32)std::min<u64>(nopen, std::min<u64>(max_cells / G, 0xFFFFFFFEull / G));
+    if (const char* e = getenv("SIEVE_SEG_BATCH"))  // test hook: force small batches
+      batch = std::max<u32>(1, std::min<u32>(batch, (u32)atoi(e)));
+    // batches: runs of segments with one source array, at most `batch` segments each
+    std::vector<u32> bstart;
+    for (u32 s = 0; s < nopen; s++)
+      if (bstart.empty() || s - bstart.back() == batch || open[s].src != open[s - 1].src) bstart.push_back(s);
+    bstart.push_back(nopen);
+    for (size_t bi = 0; bi + 1 < bstart.size(); bi++) {
+    const u32 s0 = bstart[bi];
+    const u32 nseg = bstart[bi + 1] - s0;
+    const OpenSeg* op = open.data() + s0;
+    const u64 ncell = (u64)nseg * G;
+    const u32 ib = std::max<u32>(1, bitlen(ncell));
     std::vector<SegDev> hs(nseg);
     std::vector<double> hh(nseg);
+    std::vector<BucketChunk> chunks;
+    u64 maxlen = 0;  // largest segment (local values)
     for (u32 s = 0; s < nseg; s++) {
-      const OpenSeg& o = open[s];
+      const OpenSeg& o = op[s];
       double h = scott_h(o.n, o.s1, o.s2, P->bw_scale);
       hh[s] = h;
-      u64 base = (u64)o.t3rank << bx;
-      hs[s].key_lo = base + o.lo;
-      hs[s].key_hi = base + o.hi;
       hs[s].lo = o.lo;
       hs[s].hi = o.hi;
       hs[s].h = h;
       hs[s].inv_h = 1.0 / h;
-      hs[s].begin = nkeys ? o.b : 0;  // local index range (no device search needed)
-      hs[s].end = nkeys ? o.e : 0;
+      hs[s].cq = (double)(G - 1) / (double)(o.hi - o.lo);
+      u64 len = round == 1 ? h_localn[o.kid] : o.e - o.b;
+      maxlen = std::max(maxlen, len);
+      if (round > 1)
+        for (u64 b = o.b; b < o.e; b += BK_CHUNK)
+          chunks.push_back({s, (u32)std::min<u64>(BK_CHUNK, o.e - b), b});
     }
+    if (round == 1)  // the open segments are the Tier-3 kernels in t3rank order
+      for (u32 s = 0; s < nseg; s++)
+        if (op[s].t3rank != s0 + s) return sv_fail(SIEVE_ESTATE, "internal: round-1 segment order");
+    const u64* src = op[0].src;  // one source per batch (see bstart)
+    const u32 src_shift = op[0].src_shift;
+    const u64 nin = round == 1 ? nkeys : (u64)chunks.size() * BK_CHUNK;
     DBuf<SegDev> segs(c);
+    DBuf<double> gtab(c);
+    DBuf<u32> off(c);
+    DBuf<u64> ck(c);
+    DBuf<BucketChunk> d_chunks(c);
     SV_TRY(segs.alloc(nseg));
     SV_TRY(h2d(c, segs.get(), hs));
+    SV_TRY(gtab.alloc(ncell));
+    SV_TRY(off.alloc(ncell + 1));
+    SV_TRY(ck.alloc(std::max<u64>(nin, 1)));
+    {
+      DBuf<char> tmp(c);
+      SV_TRY(tmp.alloc(radix_sort_temp_bytes(nin, false)));
+      if (!chunks.empty()) {
+        SV_TRY(d_chunks.alloc(chunks.size()));
+        SV_TRY(h2d(c, d_chunks.get(), chunks));
+      }
+      PhaseTimer tm(c, SIEVE_PHASE_SORT, nin * 8);
+      launch_grid_tab(segs.get(), nseg, G, gtab.get(), S);
+      launch_cellkey(round == 1 ? nullptr : d_chunks.get(), src, nin, round == 1 ? bx : 64, src_shift,
+                     segs.get(), G, gtab.get(), ib, (u32)ncell, s0, ck.get(),
+                     c->count_terms ? terms.get() : nullptr, S);
+      int passes = 0;
+      SV_TRY(radix_sort(ck.get(), nullptr, nin, (int)ib, tmp.get(), S, &passes));
+      if (c->timing) c->acc[SIEVE_PHASE_SORT].work += (u64)passes * nin * 16;
+      launch_cell_offsets(ck.get(), nin, ib, (u32)ncell, off.get(), S);
+      SV_CUDA(cudaGetLastError());
+    }
     DBuf<u64> D(c);
     SV_TRY(D.alloc((size_t)nseg * G * 2));
     SV_CUDA(cudaMemsetAsync(D.get(), 0, (size_t)nseg * G * 16, S));
-    if (nkeys) {
+    if (nin) {
       DBuf<u64> tile_range(c);
       DBuf<u32> tile_items(c);
       DBuf<char> stemp(c);
       SV_TRY(tile_range.alloc((size_t)nseg * tps * 2));
       SV_TRY(tile_items.alloc((size_t)nseg * tps + 1));
-      SV_TRY(stemp.alloc(((size_t)nseg * tps / 4096 + 4) * 4));
+      SV_TRY(stemp.alloc(scan_u32_temp_bytes((u64)nseg * tps)));
       // work items are counted on the device; size the item map by a host-side bound so no
-      // synchronisation is needed here: a tile has at most ceil(segment length / KDE_CH) items
+      // synchronisation is needed here: a tile has at most ceil(segment values / KDE_CH) items
       u64 items_bound = 0;
-      for (u32 s = 0; s < nseg; s++) items_bound += (u64)tps * ((open[s].e - open[s].b + KDE_CH - 1) / KDE_CH);
+      for (u32 s = 0; s < nseg; s++) {
+        u64 len = round == 1 ? h_localn[op[s].kid] : op[s].e - op[s].b;
+        items_bound += (u64)tps * ((len + KDE_CH - 1) / KDE_CH);
+      }
       if (items_bound >= (1ull << 32)) return sv_fail(SIEVE_ELIMIT, "too many KDE work items");
       u32 items = (u32)items_bound;
-      SV_TRY(kde_plan(segs.get(), nseg, G, keys.get(), nkeys, xmask, tile_range.get(),
-                      tile_items.get(), stemp.get(), nullptr, S));
+      kde_plan(segs.get(), nseg, G, gtab.get(), off.get(), tile_range.get(), tile_items.get(), stemp.get(), S);
       DBuf<char> item_tile(c);
       SV_TRY(item_tile.alloc(kde_item_bytes(items)));
       PhaseTimer tm(c, SIEVE_PHASE_KDE, 0);
       // the unguarded KDE variant needs |z| < 4800 for every evaluated pair: window 7.6 h plus
-      // KDE_TJ - 1 grid steps, so max Delta / h < 150 suffices (true for realistic segments)
+      // KDE_TJ - 1 grid steps plus two boundary cells, so max Delta / h < 140 suffices
       bool guard = false;
       for (u32 s = 0; s < nseg; s++)
-        if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 150.0 * hs[s].h) guard = true;
-      launch_kde(segs.get(), nseg, G, keys.get(), xmask, tile_range.get(), tile_items.get(),
-                 (u32*)item_tile.get(), items, D.get(), counter.get() + 1, terms.get(), guard, S);
+        if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 140.0 * hs[s].h) guard = true;
+      launch_kde(segs.get(), nseg, G, ck.get(), ib, tile_range.get(), tile_items.get(),
+                 (u32*)item_tile.get(), items, D.get(), counter.get() + 1, terms.get() + 1, guard, S);
       tm.stop();
       SV_CUDA(cudaGetLastError());
     }
@@ -857,10 +909,16 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       SV_TRY(pl.alloc((size_t)nparts * MOM_LANES));
       SV_TRY(pm.alloc((size_t)nparts * 2));
       SV_TRY(pab.alloc((size_t)nparts * 4));
+      SV_CUDA(cudaMemsetAsync(pl.get(), 0, (size_t)nparts * MOM_LANES * 8, S));
+      launch_fill_u64(pm.get(), nparts, ~0ull, S);
+      SV_CUDA(cudaMemsetAsync(pm.get() + nparts, 0, (size_t)nparts * 8, S));
+      DBuf<u32> pitems(c);
+      DBuf<char> ptemp(c);
+      SV_TRY(pitems.alloc(nparts + 1));
+      SV_TRY(ptemp.alloc(scan_u32_temp_bytes(nparts)));
       PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
-      launch_part_stats(segs.get(), nseg, T.get(), tstride, ntk.get(), d_off.get(), nparts,
-                        nkeys ? keys.get() : nullptr, nkeys, bx, Pb.get(), pl.get(),
-                        pm.get(), pab.get(), S);
+      launch_part_stats(segs.get(), nseg, G, gtab.get(), off.get(), T.get(), tstride, ntk.get(), d_off.get(),
+                        nparts, ck.get(), ib, pitems.get(), ptemp.get(), pl.get(), pm.get(), pab.get(), S);
       tp.stop();
       SV_CUDA(cudaGetLastError());
       SV_TRY(allreduce(c, pl.get(), (size_t)nparts * MOM_LANES, RED_SUM));   // AR-3
@@ -878,17 +936,16 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       SV_TRY(sync(c));
       hc.mark("ps");
     }
-    std::vector<OpenSeg> next;
     for (u32 s = 0; s < nseg; s++) {
       if (R->keep_debug) {
         SegDebug sd;
-        sd.meta.kernel_id = open[s].kid;
+        sd.meta.kernel_id = op[s].kid;
         sd.meta.round = round;
         sd.meta.split_kind = h_ntk[nseg + s];
         sd.meta.n_cuts = h_ntk[s];
-        sd.meta.lo = open[s].lo;
-        sd.meta.hi = open[s].hi;
-        sd.meta.count = open[s].n;
+        sd.meta.lo = op[s].lo;
+        sd.meta.hi = op[s].hi;
+        sd.meta.count = op[s].n;
         sd.meta.bandwidth = hh[s];
         sd.dlo.resize(G); sd.dhi.resize(G);
         for (u32 j = 0; j < G; j++) {
@@ -905,12 +962,13 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         u128 s1 = limbs_u128(L + 1), s2 = limbs_u128(L + 5);
         u64 lo = h_pmin[p], hi = h_pmax[p];
         if (lo == hi || cov_lt(pn, s1, s2, P->theta_num, P->theta_den))
-          fin.push_back({open[s].kid, 3, lo, hi, pn, s1, hh[s], round});
-        else
-          next.push_back({open[s].kid, open[s].t3rank, lo, hi, pn, s1, s2, h_ab[4 * (size_t)p + 2],
-                          h_ab[4 * (size_t)p + 3]});
+          fin.push_back({op[s].kid, 3, lo, hi, pn, s1, hh[s], round});
+        else  // re-opened: its values are [ia, ib) of this batch's sorted keys (x << ib)
+          next.push_back({op[s].kid, op[s].t3rank, lo, hi, pn, s1, s2, h_ab[4 * (size_t)p + 2],
+                          h_ab[4 * (size_t)p + 3], ck.get(), ib});
       }
     }
+    }  // batches
     open.swap(next);
     hc.mark("round");
   }
@@ -918,7 +976,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   // the KDE term count is read back with the representatives at the end (no extra sync)
   std::vector<unsigned long long> h_terms;
   SV_TRY(d2h(c, h_terms, terms.get(), 2));
-  Pb.release(); keys.release();
+  keys.release();
 
   // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
   std::sort(fin.begin(), fin.end(), [](const Fin& a, const Fin& b) {

@@ -13,7 +13,7 @@
 // independent of summation order, of the work decomposition and of the number of ranks.
 //
 // B200 mapping (the paper's scripts have no GPU design; this is new).  The KDE is a windowed
-// gather over the SORTED values of each segment, bound by the FP64 pipe (no contraction, so no
+// gather over the values of each segment grouped by grid cell (bucket.cu), bound by the FP64 pipe (no contraction, so no
 // tensor cores).  Work item = (segment, tile of 32 grid points, chunk of <= 256 values inside
 // the tile's window |g - x| <= 7.6 h); items are pulled by WARPS from an atomic counter (no
 // block barriers: warps of a block never wait for each other); each lane owns one grid point,
@@ -34,7 +34,6 @@
 #include "kernels.cuh"
 
 #define KDE_W 7.6            // window half-width in units of h: k > 10526 (t > 28.5014) beyond it
-#define KDE_WC 7.54983443527075   // sqrt(57): |z| <= this <=> t <= 28.5 (term-count diagnostic)
 #define KDE_KCUT 10527       // k > 10526 = rint(28.5 * 256 log2 e) -> index 10527 holds 0
 #ifndef KDE_WARPS
 #define KDE_WARPS 12         // warps per block (independent work-item consumers)
@@ -52,67 +51,40 @@ __device__ __forceinline__ double grid_pt(u64 lo, u64 hi, u32 j, u32 G) {
                    __ddiv_rn(__ull2double_rn((hi - lo) * (u64)j), __uint2double_rn(G - 1)));
 }
 
-__device__ __forceinline__ u64 lower_bound_u64(const u64* a, u64 b, u64 e, u64 v) {
-  while (b < e) {
-    u64 m = (b + e) >> 1;
-    if (a[m] < v) b = m + 1; else e = m;
-  }
-  return b;
-}
-
-// ------------------------------------------------------------------------------------------
-__global__ void k_seg_ranges(SegDev* segs, u32 nseg, const u64* keys, u64 nkeys) {
-  u32 s = blockIdx.x * blockDim.x + threadIdx.x;
-  if (s >= nseg) return;
-  SegDev g = segs[s];
-  u64 b = lower_bound_u64(keys, 0, nkeys, g.key_lo);
-  u64 e = g.key_hi == ~0ull ? nkeys : lower_bound_u64(keys, b, nkeys, g.key_hi + 1);
-  segs[s].begin = b;
-  segs[s].end = e;
-}
-
-void launch_seg_ranges(SegDev* segs, u32 nseg, const u64* keys, u64 nkeys, cudaStream_t s) {
-  if (nseg) SV_LAUNCH(k_seg_ranges, div_up(nseg, 128), 128, 0, s)(segs, nseg, keys, nkeys);
-}
-
-// per (segment, tile of KDE_TJ grid points): the local index range of the values inside the
-// tile's window, and the number of KDE_CH-value chunks (work items) it takes
-__global__ void k_kde_tiles(const SegDev* segs, u32 nseg, u32 G, u32 tps, const u64* keys,
-                            u64* tile_range, u32* tile_items) {
+// per (segment, tile of KDE_TJ grid points): the range of bucketed values in the cells that meet
+// the tile's window [g_j0 - 7.6 h, g_j1 + 7.6 h], and the number of KDE_CH-value chunks (work
+// items) it takes.  Values of the two boundary cells that lie outside the window are evaluated
+// too; their terms are exactly 0 (k > 10526).
+__global__ void k_kde_tiles(const SegDev* segs, u32 nseg, u32 G, u32 tps, const double* gtab,
+                            const u32* off, u64* tile_range, u32* tile_items) {
   u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (id >= (u64)nseg * tps) return;
   u32 s = (u32)(id / tps), t = (u32)(id % tps);
   SegDev g = segs[s];
+  const double* gt = gtab + (u64)s * G;
   u32 j0 = t * KDE_TJ;
   u32 j1 = min(G - 1, j0 + KDE_TJ - 1);
   double w = __dmul_rn(KDE_W, g.h);
-  double ga = __dsub_rn(grid_pt(g.lo, g.hi, j0, G), w);
-  double gb = __dadd_rn(grid_pt(g.lo, g.hi, j1, G), w);
-  u64 base = g.key_lo - g.lo;
+  double ga = __dsub_rn(gt[j0], w);
+  double gb = __dadd_rn(gt[j1], w);
   u64 xa = ga <= (double)g.lo ? g.lo : (u64)floor(ga);
   u64 xb = gb >= (double)g.hi ? g.hi : (u64)ceil(gb);
-  u64 a = lower_bound_u64(keys, g.begin, g.end, base + xa);
-  u64 z = lower_bound_u64(keys, a, g.end, base + xb + 1);
+  u32 ca = cell_of(gt, G, g.lo, g.cq, xa), cb = cell_of(gt, G, g.lo, g.cq, xb);
+  u64 a = off[(u64)s * G + ca];
+  u64 z = off[(u64)s * G + cb + 1];
   tile_range[2 * id] = a;
   tile_range[2 * id + 1] = z;
   tile_items[id] = (u32)((z - a + KDE_CH - 1) / KDE_CH);
 }
 
-void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s);
 
-int kde_plan(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 nkeys, u64 xmask,
-             u64* tile_range, u32* tile_items, void* scan_temp, u32* items_host, cudaStream_t s) {
-  (void)nkeys; (void)xmask;
+void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
+              u64* tile_range, u32* tile_items, void* scan_temp, cudaStream_t s) {
   u32 tps = div_up(G, KDE_TJ);
   u64 nt = (u64)nseg * tps;
-  SV_LAUNCH(k_kde_tiles, div_up(nt, 128), 128, 0, s)(segs, nseg, G, tps, keys, tile_range, tile_items);
+  SV_LAUNCH(k_kde_tiles, div_up(nt, 128), 128, 0, s)(segs, nseg, G, tps, gtab, off, tile_range, tile_items);
   // exclusive scan in place; tile_items[nt] receives the total (read on the device by k_kde)
   scan_u32(tile_items, tile_items, nt, scan_temp, tile_items + nt, s);
-  if (items_host) {
-    SV_CUDA(cudaMemcpyAsync(items_host, tile_items + nt, 4, cudaMemcpyDeviceToHost, s));
-    SV_CUDA(cudaStreamSynchronize(s));
-  }
-  return SIEVE_OK;
 }
 
 // item -> tile map (so a warp finds its tile with one load): one thread per item, binary
@@ -221,7 +193,8 @@ __device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, cons
   double kf = __dsub_rn(kb, C_MAGIC);
   // k = rint(u * 128 log2 e); any k > 10526 maps to the zero entry.  The low word of kb is k
   // while k < 2^32, i.e. u < 2.3e7: the host proves |z| < 4800 for every (lane, value) pair of
-  // a launch when max Delta/h < 150 (window 7.6 h plus KDE_TJ-1 = 31 grid steps) and runs the
+  // a launch when max Delta/h < 140 (window 7.6 h plus KDE_TJ-1 = 31 grid steps plus the two
+  // boundary cells of the bucketed range: 7.6 + 33 * 140 < 4800) and runs the
   // unguarded variant; otherwise any u >= 80 is sent to the zero entry explicitly.  p stays
   // finite for every input the API admits (x < 2^44, n < 2^36 => h > 2^-26, u < 2^140), and
   // fma(p, 0, 2^52) = 2^52.
@@ -243,10 +216,10 @@ __device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, cons
 // out-of-window terms but quadruples the per-item overhead at equal chunk size.)
 template <bool GUARD>
 __global__ void __launch_bounds__(32 * KDE_WARPS, KDE_MINB)
-k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ keys, u64 xmask,
+k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ vals, u32 vshift,
       const u64* __restrict__ tile_range, const u32* __restrict__ tile_items,
       const u32* __restrict__ item_tile, u32 ntiles, u64* D, unsigned long long* counter,
-      unsigned long long* terms) {
+      unsigned long long* evaluated) {
   const u32 items = tile_items[ntiles];  // device-side total of work items
   extern __shared__ __align__(16) unsigned char smem[];
   double* sS = (double*)smem;                                   // [KDE_KCUT + 1]
@@ -260,7 +233,6 @@ k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ k
   }
   __syncthreads();
   const u32 lane = lane_id();
-  u64 inwin = 0;
   // the fma that forms kb has two constant operands and a DFMA takes at most one constant:
   // load both into registers once (opaque to the compiler, so it cannot re-materialise them)
   KdeRegs R;
@@ -277,7 +249,7 @@ k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ k
     u64 va = tile_range[2 * (u64)tile] + (u64)(item - tile_items[tile]) * KDE_CH;
     u64 ve = tile_range[2 * (u64)tile + 1];
     u32 len = (u32)min((u64)KDE_CH, ve - va);
-    for (u32 i = lane; i < len; i += 32) sx[i] = __ull2double_rn(keys[va + i] & xmask);
+    for (u32 i = lane; i < len; i += 32) sx[i] = __ull2double_rn(vals[va + i] >> vshift);
     __syncwarp();
     const u32 slice = lane / KDE_TJ;
     u32 j = t * KDE_TJ + lane % KDE_TJ;
@@ -309,40 +281,24 @@ k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ k
     acc -= (u64)nterm * 0x4330000000000000ull;
 #pragma unroll
     for (int o = KDE_TJ; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if (terms && lane == 0) {  // evaluated (lane, value) pairs of this item, wasted ones included
+    if (evaluated && lane == 0) {  // evaluated (lane, value) pairs of this item, wasted ones included
       u32 live = min((u32)KDE_TJ, G - t * KDE_TJ);
-      atomicAdd(terms + 1, (unsigned long long)live * len);
+      atomicAdd(evaluated, (unsigned long long)live * len);
     }
-    if (j < G && slice == 0) {
-      if (acc) {
-        unsigned long long* d = (unsigned long long*)(D + 2 * ((u64)s * G + j));
-        unsigned long long old = atomicAdd(d, (unsigned long long)acc);
-        if (old + acc < old) atomicAdd(d + 1, 1ull);
-      }
-      if (terms) {  // values with |g - x| <= sqrt(74) h in this chunk (diagnostic work count)
-        double wc = __dmul_rn(KDE_WC, g.h);
-        double lo = __dsub_rn(gj, wc), hi = __dadd_rn(gj, wc);
-        u32 l = 0, r = len;
-        while (l < r) { u32 m = (l + r) >> 1; if (sx[m] < lo) l = m + 1; else r = m; }
-        u32 a = l;
-        r = len;
-        while (l < r) { u32 m = (l + r) >> 1; if (sx[m] <= hi) l = m + 1; else r = m; }
-        inwin += l - a;
-      }
+    if (j < G && slice == 0 && acc) {
+      unsigned long long* d = (unsigned long long*)(D + 2 * ((u64)s * G + j));
+      unsigned long long old = atomicAdd(d, (unsigned long long)acc);
+      if (old + acc < old) atomicAdd(d + 1, 1ull);
     }
     __syncwarp();
-  }
-  if (terms) {
-    for (int o = 16; o > 0; o >>= 1) inwin += __shfl_down_sync(0xffffffffu, inwin, o);
-    if (lane == 0 && inwin) atomicAdd(terms, (unsigned long long)inwin);
   }
 }
 
 size_t kde_item_bytes(u32 items) { return (size_t)items * 4 + 16; }
 
-void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
-                const u64* tile_range, const u32* tile_items, u32* item_tile, u32 items, u64* D,
-                unsigned long long* work_counter, unsigned long long* terms, bool guard,
+void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const u64* tile_range,
+                const u32* tile_items, u32* item_tile, u32 items, u64* D,
+                unsigned long long* work_counter, unsigned long long* evaluated, bool guard,
                 cudaStream_t s) {
   if (items == 0) return;
   u32 tps = div_up(G, KDE_TJ);
@@ -359,7 +315,7 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
   u32 need = div_up(items, KDE_WARPS);
   if (grid > need) grid = need;
   cudaMemsetAsync(work_counter, 0, 8, s);
-  SV_LAUNCH(kern, grid, 32 * KDE_WARPS, KDE_SMEM_BYTES, s)(segs, G, tps, keys, xmask, tile_range,
-                                                           tile_items, item_tile, ntiles, D,
-                                                           work_counter, terms);
+  SV_LAUNCH(kern, grid, 32 * KDE_WARPS, KDE_SMEM_BYTES, s)(segs, G, tps, vals, vshift, tile_range, tile_items,
+                                                           item_tile, ntiles, D, work_counter,
+                                                           evaluated);
 }

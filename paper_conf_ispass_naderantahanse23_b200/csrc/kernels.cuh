@@ -42,46 +42,67 @@ void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u
 
 // ---------------- LSD radix sort (u64 keys, optional u32 payload) ----------------------------
 size_t radix_sort_temp_bytes(u64 n, bool with_vals);
-// sorts keys[0..n) on bits [0, nbits); result in keys/vals (in place via internal ping-pong);
+// sorts keys[0..n) by bits [0, nbits) (higher bits ride along); result in keys/vals (in place via
+// internal ping-pong);
 // stream-ordered, no host synchronisation
 int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s,
                int* passes = nullptr);
 
-// ---------------- prefix sums of x and x^2 over sorted Tier-3 keys -----------------------------
-// block-boundary prefix sums of x and x^2 over the sorted Tier-3 keys
-#define PREFIX_BLOCK 4096
-u64 block_prefix_entries(u64 n);
-// Pb: [(n / PREFIX_BLOCK + 1) + 1][4] u64 = (S1 lo, S1 hi, S2 lo, S2 hi) exclusive prefixes at
-// block boundaries; the last entry is the total
-void launch_block_prefix(const u64* keys, u64 n, u64 xmask, u64* Pb, cudaStream_t s);
+void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s);
+size_t scan_u32_temp_bytes(u64 n);
 
 // ---------------- KDE over open segments ([8], [36]; A6-A10) -----------------------------
 struct SegDev {
-  u64 key_lo;   // (t3rank << bx) + lo   -- first key of the segment's value range
-  u64 key_hi;   // (t3rank << bx) + hi   -- last key (inclusive)
   u64 lo, hi;   // value range [lo, hi] (global, replicated)
   double h, inv_h;
-  u64 begin, end; // local index range in the sorted keys (filled on device)
+  double cq;    // (G - 1) / (hi - lo): cell estimate (made exact against the grid table)
 };
+#define KDE_WC 7.54983443527075   // sqrt(57): |z| <= this <=> t <= 28.5 (in-window term count)
 #define KDE_TJ 32       // grid points per tile (a work item is one warp's: one point per lane)
 #ifndef KDE_CH
 #define KDE_CH 256      // values per work item chunk (staged in the warp's shared memory)
 #endif
-struct KdeScratch {
-  u64* tile_range;     // [nseg*tiles][2]
-  u32* tile_items;     // [nseg*tiles + 1] exclusive scan of chunks per tile
-  void* scan_temp;
-  unsigned long long* work_counter;
-};
-void launch_seg_ranges(SegDev* segs, u32 nseg, const u64* keys, u64 nkeys, cudaStream_t s);
-// returns total work items through *items_host (synchronises the stream once)
-int kde_plan(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 nkeys, u64 xmask,
-             u64* tile_range, u32* tile_items, void* scan_temp, u32* items_host, cudaStream_t s);
+// per (segment, tile of KDE_TJ grid points): the range of bucketed values whose cells meet the
+// tile's window, chunked into work items; tile_items[nseg * tiles] receives the item total
+void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
+              u64* tile_range, u32* tile_items, void* scan_temp, cudaStream_t s);
 size_t kde_item_bytes(u32 items);
-void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* keys, u64 xmask,
-                const u64* tile_range, const u32* tile_items, u32* item_tile, u32 items,
+void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const u64* tile_range,
+                const u32* tile_items, u32* item_tile, u32 items,
                 u64* D /* [nseg][G][2] */, unsigned long long* work_counter,
-                unsigned long long* terms, bool guard, cudaStream_t s);
+                unsigned long long* evaluated, bool guard, cudaStream_t s);
+
+// ---------------- segmented sort by (open segment, grid cell) (a2) ----------------------------
+// rounds > 1 read each re-opened part's range of the previous round's sorted keys in chunks of
+// BK_CHUNK values: chunk c supplies outputs [c * BK_CHUNK, c * BK_CHUNK + len)
+struct BucketChunk { u32 seg; u32 len; u64 begin; };
+#define BK_CHUNK 2048
+// max j with g[j] <= x, for lo <= x (so the answer exists); cq = (G - 1) / (hi - lo) gives the
+// estimate, which is exact unless x lies within rounding error of a grid point: the two table
+// entries that confirm it are loaded together (one L2 round trip), and a miss walks the table
+// (g is non-decreasing in j)
+__device__ __forceinline__ u32 cell_of(const double* g, u32 G, u64 lo, double cq, u64 x) {
+  double xd = __ull2double_rn(x);  // exact: x < 2^44
+  double e = __dmul_rn(__ull2double_rn(x - lo), cq);
+  u32 j = e >= (double)(G - 1) ? G - 1 : (u32)e;
+  u32 j1 = j + 1 < G ? j + 1 : j;
+  double g0 = __ldg(g + j), g1 = __ldg(g + j1);
+  if (g0 <= xd && (j1 == j || g1 > xd)) return j;
+  while (j + 1 < G && __ldg(g + j + 1) <= xd) j++;
+  while (j > 0 && __ldg(g + j) > xd) j--;
+  return j;
+}
+
+// gtab[s * G + j] = g_j of segment s (A9)
+void launch_grid_tab(const SegDev* segs, u32 nseg, u32 G, double* gtab, cudaStream_t s);
+// out[i] = (x << ib) | idx, idx = s * G + cell(x) (ncell if x is outside [lo, hi] of segment s);
+// chunks == nullptr: in = tagged Tier-3 keys (s = (key >> bx) - seg0, keys of other segments get
+// the sentinel), else x = in[..] >> in_shift; *inwin += in-window KDE terms
+void launch_cellkey(const BucketChunk* chunks, const u64* in, u64 nin, u32 bx, u32 in_shift,
+                    const SegDev* segs, u32 G, const double* gtab, u32 ib, u32 ncell, u32 seg0,
+                    u64* out, unsigned long long* inwin, cudaStream_t s);
+// off[c] = first position of the idx-sorted keys with idx >= c, c = 0..ncell
+void launch_cell_offsets(const u64* keys, u64 n, u32 ib, u32 ncell, u32* off, cudaStream_t s);
 
 // ---------------- valleys and thresholds (A11-A13) ---------------------------------------------
 // T[s*tstride + q], nt[s], kind[s] (1 = valley, 2 = bisect)
@@ -90,10 +111,13 @@ void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D
 
 // ---------------- part moments (A13 f) ----------------------------------------------------------
 // parts of segment s: q = 0..nt[s]; part_off[s] = first part index (exclusive scan of nt+1)
-// out: lanes[p*9..] (n, S1 limbs, S2 limbs), mm[p*2..] (min, max), ab[p*2..] value interval
-void launch_part_stats(const SegDev* segs, u32 nseg, const u64* T, u32 tstride, const u32* nt,
-                       const u32* part_off, u32 nparts, const u64* keys, u64 nkeys, u32 bx,
-                       const u64* Pb, u64* lanes, u64* mm, u64* ab, cudaStream_t s);
+// out (accumulated: lanes zeroed, mm[0..nparts) = ~0 and mm[nparts..2 nparts) = 0 by the
+// caller): lanes[p*9..] (n, S1 limbs, S2 limbs), mm (min, max), ab[p*4..] = value interval
+// [a, b) and this rank's superset range [ia, ib) in the bucketed values
+void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
+                       const u64* T, u32 tstride, const u32* nt, const u32* part_off, u32 nparts,
+                       const u64* vals, u32 vshift, u32* items /* [nparts + 1] */, void* scan_temp,
+                       u64* lanes, u64* mm, u64* ab, cudaStream_t s);
 // ---------------- pass B: assignment + per-(stratum, CTA) statistics -------------------
 struct KTab {      // per kernel
   u32 base;        // global id of its first stratum
@@ -155,8 +179,6 @@ void launch_csv_firsts(const u32* flag, const u32* seg, const u32* row, u64 n, u
 void launch_csv_ids(const u32* order, u64 nd, u32* id_of, const u32* flag, const u32* seg,
                     const u32* row, u64 n, u32* kid, cudaStream_t s);
 void launch_gather_pairs(const u64* src, const u64* idx, u64 n, u64* dst, cudaStream_t s);
-void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s);
-size_t scan_u32_temp_bytes(u64 n);
 
 // ---------------- exact min-strata DP (NEXT-3) --------------------------------------------------
 void launch_rle(const u64* keys, const u32* flag, const u32* seg, u64 n, u32 bx, u64* ukey,

@@ -1,12 +1,10 @@
-// sort.cu -- Tier-3 key compaction, LSD radix sort of 64-bit packed keys, exclusive scans and
-// the u128 prefix sums of x and x^2 over the sorted Tier-3 values.
+// sort.cu -- Tier-3 key compaction, LSD radix sort of 64-bit packed keys and exclusive scans.
 //
-// The north_star path sorts (kernel, instruction count) to group each high-CoV kernel's
-// invocations by value (the KDE windows and the part moments need them contiguous).  Only
-// Tier-3 invocations are sorted (A-series reading "sort only Tier-3 keys"); the
-// key is (t3rank << bx) + x with bx = bitlen(max x), so only ceil(bits / 8) digit passes run,
-// and passes whose 8 bits are constant over all keys (found by one OR-reduction of key ^ key0)
-// are skipped.
+// The compaction gathers the Tier-3 invocations as keys (t3rank << bx) + x (bx = bitlen(max x));
+// the stratification groups them by (segment, grid cell) with the counting sort of bucket.cu.
+// The radix sort orders the (stratum, CTA) entries of pass B, the name hashes of the CSV ingest
+// and the Tier-3 keys of the exact min-strata DP (which needs every distinct value in order):
+// only the digit passes whose 8 bits vary over the keys run (one histogram read decides).
 //
 // Radix passes are onesweep (see below): one kernel per digit with decoupled look-back.
 #include <algorithm>
@@ -202,14 +200,14 @@ void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u
 #endif
 
 __global__ void __launch_bounds__(RS_THREADS)
-k_os_hist(const u64* __restrict__ keys, u64 n, int npass, u32* __restrict__ ghist) {
+k_os_hist(const u64* __restrict__ keys, u64 n, int npass, u64 kmask, u32* __restrict__ ghist) {
   extern __shared__ u32 s_hist[];  // [RS_WARPS/2][npass][256] (pairs of warps share a table)
   const int tables = RS_WARPS / 2;
   for (int i = threadIdx.x; i < tables * npass * 256; i += RS_THREADS) s_hist[i] = 0;
   __syncthreads();
   u32* mine = s_hist + (threadIdx.x >> 6) * npass * 256;
   for (u64 i = (u64)blockIdx.x * RS_THREADS + threadIdx.x; i < n; i += (u64)gridDim.x * RS_THREADS) {
-    u64 k = __ldcs(keys + i);
+    u64 k = __ldcs(keys + i) & kmask;
     for (int p = 0; p < npass; p++) atomicAdd(&mine[p * 256 + ((k >> (8 * p)) & 255u)], 1u);
   }
   __syncthreads();
@@ -233,7 +231,7 @@ __device__ __forceinline__ void st_volatile_u64(u64* p, u64 v) {
 
 template <bool V>  // V: a u32 payload travels with each key
 __global__ void __launch_bounds__(RS_THREADS, RS_MINB)
-k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int shift,
+k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int shift, u32 dmask,
           const u32* __restrict__ gbase, u64* status, u32* tile_counter, u64* __restrict__ kout,
           u32* __restrict__ vout) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -263,7 +261,7 @@ k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int s
   for (int r = 0; r < RS_IPT; r++) {
     u64 i = base + (u64)r * 32 + lane_id();
     bool ok = i < n;
-    u32 d = ok ? (u32)(key[r] >> shift) & 255u : 256u;
+    u32 d = ok ? (u32)(key[r] >> shift) & dmask : 256u;
     // lanes with the same digit: 8 ballots (one per digit bit) plus validity, ANDed -- cheaper
     // than MATCH.ANY, which serialises in the MIO pipe
     u32 peers = __ballot_sync(0xffffffffu, ok);
@@ -320,7 +318,7 @@ k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int s
   for (int r = 0; r < RS_IPT; r++) {
     u64 i = base + (u64)r * 32 + lane_id();
     if (i < n) {
-      u32 d = (u32)(key[r] >> shift) & 255u;
+      u32 d = (u32)(key[r] >> shift) & dmask;
       u32 p = s_td[d] + s_wh[w][d] + rank[r];
       s_k[p] = key[r];
       if (V) s_v[p] = val[r];
@@ -331,7 +329,7 @@ k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int s
   if (tile_n > RS_TILE) tile_n = RS_TILE;
   for (u32 j = threadIdx.x; j < tile_n; j += RS_THREADS) {
     u64 k = s_k[j];
-    u32 d = (u32)(k >> shift) & 255u;
+    u32 d = (u32)(k >> shift) & dmask;
     u64 o = s_go[d] + (j - s_td[d]);
     kout[o] = k;
     if (V) vout[o] = s_v[j];
@@ -375,7 +373,7 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   size_t hsmem = (size_t)(RS_WARPS / 2) * npass * 256 * 4;
   SV_CUDA(cudaFuncSetAttribute(k_os_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsmem));
   u64 hgrid = std::min<u64>((n + RS_THREADS - 1) / RS_THREADS, (u64)sv_num_sms() * 4);
-  SV_LAUNCH(k_os_hist, (unsigned)hgrid, RS_THREADS, hsmem, s)(keys, n, npass, ghist);
+  SV_LAUNCH(k_os_hist, (unsigned)hgrid, RS_THREADS, hsmem, s)(keys, n, npass, nbits >= 64 ? ~0ull : (1ull << nbits) - 1, ghist);
   // digit bases on the device (no host round trip): every pass runs -- a pass over a digit
   // that is constant across all keys is a stable identity permutation, so skipping it would only
   // save time, never change the result
@@ -386,13 +384,15 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   SV_CUDA(cudaFuncSetAttribute(k_os_pass<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, RS_TILE * 8));
   u64* kin = keys; u32* vin = vals; u64* kout = kalt; u32* vout = valt;
   for (int p = 0; p < npass; p++) {
+    // digits above nbits are masked off (keys may carry payload bits there)
+    const u32 dmask = 8 * p + 8 <= nbits ? 255u : (1u << (nbits - 8 * p)) - 1u;
     SV_CUDA(cudaMemsetAsync(status, 0, ntiles * 256 * 8, s));
     SV_CUDA(cudaMemsetAsync(tile_counter, 0, 4, s));
     if (vals)
-      SV_LAUNCH(k_os_pass<true>, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, 8 * p, gbase + p * 256,
+      SV_LAUNCH(k_os_pass<true>, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, 8 * p, dmask, gbase + p * 256,
                                                                      status, tile_counter, kout, vout);
     else
-      SV_LAUNCH(k_os_pass<false>, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, 8 * p, gbase + p * 256,
+      SV_LAUNCH(k_os_pass<false>, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, 8 * p, dmask, gbase + p * 256,
                                                                       status, tile_counter, kout, vout);
     u64* tk = kin; kin = kout; kout = tk;
     u32* tv = vin; vin = vout; vout = tv;
@@ -404,89 +404,4 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   }
   SV_CUDA(cudaGetLastError());
   return SIEVE_OK;
-}
-
-// ------------------------------------------------------------------------------------------
-// u128 prefix sums of x and x^2 over the sorted keys (x = key & xmask)
-// ------------------------------------------------------------------------------------------
-// POD u128 / pair types (no constructors: they live in __shared__ memory)
-struct U128 { u64 lo, hi; };
-struct Pair128 { U128 a, b; };
-__device__ __forceinline__ U128 add128v(U128 x, U128 y) {
-  U128 r; r.lo = x.lo + y.lo; r.hi = x.hi + y.hi + (r.lo < x.lo ? 1ull : 0ull); return r;
-}
-__device__ __forceinline__ U128 sub128v(U128 x, U128 y) {
-  U128 r; r.lo = x.lo - y.lo; r.hi = x.hi - y.hi - (x.lo < y.lo ? 1ull : 0ull); return r;
-}
-__device__ __forceinline__ Pair128 operator+(const Pair128& x, const Pair128& y) {
-  Pair128 r; r.a = add128v(x.a, y.a); r.b = add128v(x.b, y.b); return r;
-}
-__device__ __forceinline__ Pair128& operator+=(Pair128& x, const Pair128& y) { x = x + y; return x; }
-__device__ __forceinline__ Pair128 operator-(const Pair128& x, const Pair128& y) {
-  Pair128 r; r.a = sub128v(x.a, y.a); r.b = sub128v(x.b, y.b); return r;
-}
-__device__ __forceinline__ Pair128 pzero() { Pair128 r; r.a.lo = r.a.hi = r.b.lo = r.b.hi = 0; return r; }
-template <>
-__device__ __forceinline__ Pair128 sv_zero<Pair128>() { return pzero(); }
-template <>
-__device__ __forceinline__ Pair128 warp_incl_scan<Pair128>(Pair128 v) {
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    Pair128 n;
-    n.a.lo = __shfl_up_sync(0xffffffffu, v.a.lo, o); n.a.hi = __shfl_up_sync(0xffffffffu, v.a.hi, o);
-    n.b.lo = __shfl_up_sync(0xffffffffu, v.b.lo, o); n.b.hi = __shfl_up_sync(0xffffffffu, v.b.hi, o);
-    if ((int)lane_id() >= o) v += n;
-  }
-  return v;
-}
-
-#define PX_THREADS 512
-#define PX_IPT 8
-#define PX_TILE (PX_THREADS * PX_IPT)
-
-__device__ __forceinline__ Pair128 px_val(u64 key, u64 xmask) {
-  u64 x = key & xmask;
-  Pair128 r; r.a.lo = x; r.a.hi = 0; r.b.lo = x * x; r.b.hi = __umul64hi(x, x); return r;
-}
-
-__global__ void __launch_bounds__(PX_THREADS)
-k_px_reduce(const u64* keys, u64 n, u64 xmask, Pair128* bsum) {
-  u64 base = (u64)blockIdx.x * PX_TILE + (u64)threadIdx.x * PX_IPT;
-  Pair128 s = pzero();
-#pragma unroll
-  for (int j = 0; j < PX_IPT; j++)
-    if (base + j < n) s += px_val(keys[base + j], xmask);
-  __shared__ Pair128 tot;
-  block_excl_scan<Pair128, PX_THREADS>(s, &tot);
-  if (threadIdx.x == 0) bsum[blockIdx.x] = tot;
-}
-
-__global__ void __launch_bounds__(PX_THREADS) k_px_blocks(Pair128* bsum, u32 nb) {
-  __shared__ Pair128 carry_s;
-  if (threadIdx.x == 0) carry_s = pzero();
-  __syncthreads();
-  for (u32 b0 = 0; b0 < nb; b0 += PX_THREADS) {
-    u32 i = b0 + threadIdx.x;
-    Pair128 v = i < nb ? bsum[i] : pzero();
-    __shared__ Pair128 tot;
-    Pair128 ex = block_excl_scan<Pair128, PX_THREADS>(v, &tot);
-    Pair128 c = carry_s;
-    if (i < nb) bsum[i] = c + ex;
-    __syncthreads();
-    if (threadIdx.x == 0) carry_s = c + tot;
-    __syncthreads();
-  }
-}
-
-static_assert(PX_TILE == PREFIX_BLOCK, "prefix block size");
-
-u64 block_prefix_entries(u64 n) { return (n + PX_TILE - 1) / PX_TILE + 1; }
-
-// Pb[i] = (sum x, sum x^2) over keys[0, i * PREFIX_BLOCK), i = 0..nb (Pb[nb] = totals); part
-// sums need only these block boundaries plus at most two partial blocks (refine.cu)
-void launch_block_prefix(const u64* keys, u64 n, u64 xmask, u64* Pb, cudaStream_t s) {
-  u32 ne = (u32)block_prefix_entries(n);
-  Pair128* bsum = (Pair128*)Pb;
-  SV_LAUNCH(k_px_reduce, ne, PX_THREADS, 0, s)(keys, n, xmask, bsum);  // last block sums nothing
-  SV_LAUNCH(k_px_blocks, 1, PX_THREADS, 0, s)(bsum, ne);
 }

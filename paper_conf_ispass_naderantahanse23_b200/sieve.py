@@ -36,6 +36,7 @@ EXPORTED = [
     "sieve_strata_count", "sieve_strata_copy", "sieve_strata_stats", "sieve_strata_free",
     "sieve_segment_count", "sieve_segment_get", "sieve_predict", "sieve_last_error",
     "sieve_version", "sieve_u128_to_limbs", "sieve_limbs_to_u128", "sieve_ctx_set_timing",
+    "sieve_ctx_set_term_count",
     "sieve_timing_get", "sieve_kernel_launches", "sieve_stratify_sweep", "sieve_tier_census",
     "sieve_predict_multi", "sieve_cycle_cov", "sieve_load_csv", "sieve_trace_copy",
     "sieve_trace_kernel_names", "sieve_min_strata",
@@ -101,6 +102,7 @@ def _load():
         "sieve_u128_to_limbs": ([u64, u64, vp], None),
         "sieve_limbs_to_u128": ([vp, P(u64), P(u64)], None),
         "sieve_ctx_set_timing": ([vp, i32], i32),
+        "sieve_ctx_set_term_count": ([vp, i32], i32),
         "sieve_timing_get": ([vp, u32, P(ctypes.c_double), P(u64), P(u64)], i32),
         "sieve_kernel_launches": ([], u64),
         "sieve_stratify_sweep": ([vp, P(Params), u32, vp, vp, vp], i32),
@@ -197,6 +199,10 @@ class Ctx:
         self._h = h
         self.device, self.rank, self.world = device, rank, world if group is None else group.world
         self._group = group
+
+    def set_term_count(self, enable=True):
+        """In-window KDE term counting (strata.kde_terms); on by default."""
+        _check(_L.sieve_ctx_set_term_count(self._h, 1 if enable else 0), "sieve_ctx_set_term_count")
 
     def set_timing(self, enable=True):
         _check(_L.sieve_ctx_set_timing(self._h, 1 if enable else 0), "sieve_ctx_set_timing")

@@ -183,3 +183,39 @@ def test_homogeneous_prediction_exact():
     g = run_gpu(tr)
     p = sieve.predict(g["strata"], g["trace"])
     assert p["error"] < 1e-12
+
+
+@pytest.mark.parametrize("name,n", [("C1", None), ("C2", 200_000)])
+def test_kde_in_window_term_count(name, n):
+    """The in-window KDE term count (the roofline's work unit, counted per value in the bucket
+    pass) equals a brute-force count over the oracle's segments: pairs (grid point j, value x)
+    of every segment of every round with rn(g_j - w) <= x <= rn(g_j + w), w = rn(sqrt(57) h)."""
+    tr = gen.make_trace(name, n=n) if n else gen.make_trace(name)
+    G = 1024
+    g = run_gpu(tr, G=G)
+    o = run_oracle(tr, G=G, keep_debug=True)
+    wc = np.float64(7.54983443527075)
+    j = np.arange(G, dtype=np.int64)
+    total = 0
+    for seg in o.segments():
+        k, lo, hi, h = seg["kernel_id"], int(seg["lo"]), int(seg["hi"]), np.float64(seg["bandwidth"])
+        xs = tr["x"][(tr["kid"] == k) & (tr["x"] >= lo) & (tr["x"] <= hi)]
+        xs = np.sort(xs.astype(np.float64))  # exact: x < 2^44
+        gj = np.float64(lo) + ((hi - lo) * j).astype(np.float64) / np.float64(G - 1)
+        w = wc * h
+        a = np.searchsorted(xs, gj - w, side="left")
+        b = np.searchsorted(xs, gj + w, side="right")
+        total += int((b - a).sum())
+    assert g["terms"] == total
+
+
+def test_segment_batches_change_nothing(monkeypatch):
+    """A round whose open segments exceed one cell sort's key space runs in batches; forcing
+    batches of 3 segments (test hook) must reproduce the oracle exactly."""
+    tr = gen.make_trace("C2", n=150_000)
+    monkeypatch.setenv("SIEVE_SEG_BATCH", "3")
+    g = run_gpu(tr, keep_debug=True)
+    o = run_oracle(tr, keep_debug=True)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+    assert_segments_equal(g["segments"], o.segments())
