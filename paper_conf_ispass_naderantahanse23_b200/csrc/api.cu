@@ -98,6 +98,9 @@ struct sieve_ctx_s {
   // SIEVE_HOST_TIMING: host-side accounting of the synchronisations of a call
   int hs_n = 0;
   bool count_terms = true;  // in-window KDE term count (sieve_ctx_set_term_count)
+  // mapped (zero-copy) pinned host memory: kernels write each round's part results here
+  u64* mapped = nullptr;
+  size_t mapped_cap = 0;
   double hs_wait = 0, hs_between = 0;
   std::string hs_list;
   std::chrono::steady_clock::time_point hs_last{};
@@ -229,6 +232,27 @@ static int pin_alloc(sieve_ctx c, void** p, size_t bytes) {
   if (c->pin_off <= c->pin_cap) { *p = c->pin + off; return SIEVE_OK; }
   SV_CUDA(cudaHostAlloc(p, bytes, cudaHostAllocDefault));
   c->pin_overflow.push_back(*p);
+  return SIEVE_OK;
+}
+
+// a mapped pinned host buffer of at least `bytes` (grown, never shrunk; its contents are only
+// valid between a kernel that writes it and the host's read after the next stream sync)
+static int mapped_get(sieve_ctx c, size_t bytes, u64** host, u64** dev) {
+  if (bytes > c->mapped_cap) {
+    SV_CUDA(cudaStreamSynchronize(c->stream));  // the old buffer may still be written
+    if (c->mapped) cudaFreeHost(c->mapped);
+    c->mapped = nullptr;
+    c->mapped_cap = 0;
+    size_t want = bytes + bytes / 2 + 4096;
+    void* p;
+    SV_CUDA(cudaHostAlloc(&p, want, cudaHostAllocMapped | cudaHostAllocPortable));
+    c->mapped = (u64*)p;
+    c->mapped_cap = want;
+  }
+  void* d;
+  SV_CUDA(cudaHostGetDevicePointer(&d, c->mapped, 0));
+  *host = c->mapped;
+  *dev = (u64*)d;
   return SIEVE_OK;
 }
 
@@ -370,6 +394,7 @@ extern "C" void sieve_ctx_destroy(sieve_ctx ctx) {
   cudaStreamSynchronize(ctx->stream);
   for (void* p : ctx->pin_overflow) cudaFreeHost(p);
   if (ctx->pin) cudaFreeHost(ctx->pin);
+  if (ctx->mapped) cudaFreeHost(ctx->mapped);
   delete ctx->comm;
   ctx->magic = 0;
   delete ctx;
@@ -883,59 +908,65 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       launch_limbs_to_u128(lim.get(), (u64)nseg * G, D.get(), S);
     }
     DBuf<u64> T(c);
-    DBuf<u32> ntk(c);
+    DBuf<u32> ntk(c), d_off(c);
     SV_TRY(T.alloc((size_t)nseg * tstride));
     SV_TRY(ntk.alloc((size_t)nseg * 2));
+    SV_TRY(d_off.alloc(nseg + 1));
     PhaseTimer tv(c, SIEVE_PHASE_REFINE, 0);
     launch_valleys(segs.get(), nseg, G, P->valley_shift, D.get(), T.get(), tstride, ntk.get(),
                    ntk.get() + nseg, S);
+    launch_part_offsets(ntk.get(), nseg, d_off.get(), S);
     tv.stop();
-    std::vector<u32> h_ntk;
-    std::vector<u64> h_pl, h_pmin, h_pmax, h_ab, h_D, h_T;
-    std::vector<u32> part_off;
-    u32 nparts = 0;
-    {
-      SV_TRY(d2h(c, h_ntk, ntk.get(), (size_t)nseg * 2));
+    // Part moments.  One rank: the part count stays on the device (buffers sized by the bound
+    // nseg * tstride), the results are packed into mapped host memory and the round costs ONE
+    // host synchronisation.  Several ranks: the all-reduces need the part count on the host.
+    u32 cap = nseg * tstride;
+    if (c->comm) {
+      std::vector<u32> h_np;
+      SV_TRY(d2h(c, h_np, d_off.get() + nseg, 1));
       hc.mark("v");
       SV_TRY(sync(c));
       hc.mark("vs");
-      part_off.resize(nseg + 1);
-      for (u32 s = 0; s < nseg; s++) { part_off[s] = nparts; nparts += h_ntk[s] + 1; }
-      part_off[nseg] = nparts;
-      DBuf<u32> d_off(c);
-      SV_TRY(d_off.alloc(nseg + 1));
-      SV_TRY(h2d(c, d_off.get(), part_off));
-      DBuf<u64> pl(c), pm(c), pab(c);
-      SV_TRY(pl.alloc((size_t)nparts * MOM_LANES));
-      SV_TRY(pm.alloc((size_t)nparts * 2));
-      SV_TRY(pab.alloc((size_t)nparts * 4));
-      SV_CUDA(cudaMemsetAsync(pl.get(), 0, (size_t)nparts * MOM_LANES * 8, S));
-      launch_fill_u64(pm.get(), nparts, ~0ull, S);
-      SV_CUDA(cudaMemsetAsync(pm.get() + nparts, 0, (size_t)nparts * 8, S));
-      DBuf<u32> pitems(c);
-      DBuf<char> ptemp(c);
-      SV_TRY(pitems.alloc(nparts + 1));
-      SV_TRY(ptemp.alloc(scan_u32_temp_bytes(nparts)));
+      cap = std::max<u32>(1, h_np[0]);
+    }
+    DBuf<u64> pl(c), pm(c), pab(c);
+    SV_TRY(pl.alloc((size_t)cap * MOM_LANES));
+    SV_TRY(pm.alloc((size_t)cap * 2));
+    SV_TRY(pab.alloc((size_t)cap * 4));
+    SV_CUDA(cudaMemsetAsync(pl.get(), 0, (size_t)cap * MOM_LANES * 8, S));
+    launch_fill_u64(pm.get(), cap, ~0ull, S);
+    SV_CUDA(cudaMemsetAsync(pm.get() + cap, 0, (size_t)cap * 8, S));
+    DBuf<u32> pitems(c);
+    DBuf<char> ptemp(c);
+    SV_TRY(pitems.alloc(cap + 1));
+    SV_TRY(ptemp.alloc(scan_u32_temp_bytes(cap)));
+    {
       PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
       launch_part_stats(segs.get(), nseg, G, gtab.get(), off.get(), T.get(), tstride, ntk.get(), d_off.get(),
-                        nparts, ck.get(), ib, pitems.get(), ptemp.get(), pl.get(), pm.get(), pab.get(), S);
-      tp.stop();
+                        cap, ck.get(), ib, pitems.get(), ptemp.get(), pl.get(), pm.get(), pab.get(), S);
       SV_CUDA(cudaGetLastError());
-      SV_TRY(allreduce(c, pl.get(), (size_t)nparts * MOM_LANES, RED_SUM));   // AR-3
-      SV_TRY(allreduce(c, pm.get(), nparts, RED_MIN));
-      SV_TRY(allreduce(c, pm.get() + nparts, nparts, RED_MAX));
-      SV_TRY(d2h(c, h_pl, pl.get(), (size_t)nparts * MOM_LANES));
-      SV_TRY(d2h(c, h_pmin, pm.get(), (size_t)nparts));
-      SV_TRY(d2h(c, h_pmax, pm.get() + nparts, (size_t)nparts));
-      SV_TRY(d2h(c, h_ab, pab.get(), (size_t)nparts * 4));
-      if (R->keep_debug) {
-        SV_TRY(d2h(c, h_D, D.get(), (size_t)nseg * G * 2));
-        SV_TRY(d2h(c, h_T, T.get(), (size_t)nseg * tstride));
-      }
-      hc.mark("p");
-      SV_TRY(sync(c));
-      hc.mark("ps");
     }
+    SV_TRY(allreduce(c, pl.get(), (size_t)cap * MOM_LANES, RED_SUM));   // AR-3 (cap = parts here)
+    SV_TRY(allreduce(c, pm.get(), cap, RED_MIN));
+    SV_TRY(allreduce(c, pm.get() + cap, cap, RED_MAX));
+    u64 *hrec = nullptr, *drec = nullptr;
+    SV_TRY(mapped_get(c, (1 + (size_t)cap * PART_REC) * 8, &hrec, &drec));
+    launch_part_pack(d_off.get(), nseg, cap, pl.get(), pm.get(), pab.get(), drec, S);
+    std::vector<u32> h_ntk;
+    std::vector<u64> h_D, h_T;
+    SV_TRY(d2h(c, h_ntk, ntk.get(), (size_t)nseg * 2));
+    if (R->keep_debug) {
+      SV_TRY(d2h(c, h_D, D.get(), (size_t)nseg * G * 2));
+      SV_TRY(d2h(c, h_T, T.get(), (size_t)nseg * tstride));
+    }
+    hc.mark("p");
+    SV_TRY(sync(c));
+    hc.mark("ps");
+    std::vector<u32> part_off(nseg + 1);
+    u32 nparts = 0;
+    for (u32 s = 0; s < nseg; s++) { part_off[s] = nparts; nparts += h_ntk[s] + 1; }
+    part_off[nseg] = nparts;
+    if (hrec[0] != nparts) return sv_fail(SIEVE_ESTATE, "internal: part count mismatch");
     for (u32 s = 0; s < nseg; s++) {
       if (R->keep_debug) {
         SegDebug sd;
@@ -956,16 +987,16 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         R->segs.push_back(std::move(sd));
       }
       for (u32 p = part_off[s]; p < part_off[s + 1]; p++) {
-        const u64* L = &h_pl[(size_t)p * MOM_LANES];
+        const u64* L = hrec + 1 + (size_t)p * PART_REC;  // {lanes[9], min, max, ia, ib}
         u64 pn = L[0];
         if (!pn) continue;  // empty part: dropped (A13 f)
         u128 s1 = limbs_u128(L + 1), s2 = limbs_u128(L + 5);
-        u64 lo = h_pmin[p], hi = h_pmax[p];
+        u64 lo = L[MOM_LANES], hi = L[MOM_LANES + 1];
         if (lo == hi || cov_lt(pn, s1, s2, P->theta_num, P->theta_den))
           fin.push_back({op[s].kid, 3, lo, hi, pn, s1, hh[s], round});
         else  // re-opened: its values are [ia, ib) of this batch's sorted keys (x << ib)
-          next.push_back({op[s].kid, op[s].t3rank, lo, hi, pn, s1, s2, h_ab[4 * (size_t)p + 2],
-                          h_ab[4 * (size_t)p + 3], ck.get(), ib});
+          next.push_back({op[s].kid, op[s].t3rank, lo, hi, pn, s1, s2, L[MOM_LANES + 2],
+                          L[MOM_LANES + 3], ck.get(), ib});
       }
     }
     }  // batches

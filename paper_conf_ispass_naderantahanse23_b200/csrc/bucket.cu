@@ -179,13 +179,51 @@ void launch_cell_offsets(const u64* keys, u64 n, u32 ib, u32 ncell, u32* off, cu
 #define PS_THREADS 256
 #define PS_CH 8192      // values per work item
 
-// one thread per part: value interval, bucketed range, work items
+// part offsets on the device (one block): part_off[s] = sum over s' < s of (nt[s'] + 1),
+// part_off[nseg] = number of parts -- the host needs no copy of the cut counts before the part
+// moments are launched
+__global__ void __launch_bounds__(1024) k_part_offsets(const u32* __restrict__ nt, u32 nseg, u32* part_off) {
+  __shared__ u32 carry;
+  __shared__ u32 wsum[32];
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  for (u32 b = 0; b < nseg; b += 1024) {
+    u32 s = b + threadIdx.x;
+    u32 v = s < nseg ? nt[s] + 1 : 0;
+    u32 inc = v;
+    for (int o = 1; o < 32; o <<= 1) {
+      u32 t = __shfl_up_sync(0xffffffffu, inc, o);
+      if ((int)lane_id() >= o) inc += t;
+    }
+    if (lane_id() == 31) wsum[threadIdx.x >> 5] = inc;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+      u32 w = wsum[threadIdx.x], wi = w;
+      for (int o = 1; o < 32; o <<= 1) {
+        u32 t = __shfl_up_sync(0xffffffffu, wi, o);
+        if ((int)lane_id() >= o) wi += t;
+      }
+      wsum[threadIdx.x] = wi - w;
+    }
+    __syncthreads();
+    u32 c0 = carry;
+    if (s < nseg) part_off[s] = c0 + wsum[threadIdx.x >> 5] + inc - v;
+    __syncthreads();
+    if (threadIdx.x == 1023) carry = c0 + wsum[31] + inc;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) part_off[nseg] = carry;
+}
+
+// one thread per part slot (p < cap; the live count is part_off[nseg]): value interval,
+// bucketed range, work items (0 for dead slots)
 __global__ void k_part_ranges(const SegDev* __restrict__ segs, u32 nseg, u32 G,
                               const double* __restrict__ gtab, const u32* __restrict__ off,
                               const u64* __restrict__ T, u32 tstride, const u32* __restrict__ nt,
-                              const u32* __restrict__ part_off, u32 nparts, u64* ab, u32* items) {
+                              const u32* __restrict__ part_off, u32 cap, u64* ab, u32* items) {
   u32 p = blockIdx.x * blockDim.x + threadIdx.x;
-  if (p >= nparts) return;
+  if (p >= cap) return;
+  if (p >= part_off[nseg]) { items[p] = 0; return; }
   u32 lo = 0, hi = nseg - 1;  // last segment with part_off[s] <= p
   while (lo < hi) {
     u32 m = (lo + hi + 1) >> 1;
@@ -209,12 +247,12 @@ __global__ void k_part_ranges(const SegDev* __restrict__ segs, u32 nseg, u32 G,
 // work items (part, chunk of PS_CH values of its range), pulled grid-stride; each block reduces
 // its chunk exactly and adds it into the part's limb lanes / min / max with 64-bit atomics
 __global__ void __launch_bounds__(PS_THREADS)
-k_part_stats(const u64* __restrict__ ab, const u32* __restrict__ item_off, u32 nparts,
+k_part_stats(const u64* __restrict__ ab, const u32* __restrict__ item_off, u32 cap,
              const u64* __restrict__ vals, u32 vshift, u64* lanes, u64* mm) {
   __shared__ u64 r[PS_THREADS / 32][7];
-  const u32 total = item_off[nparts];
+  const u32 total = item_off[cap];
   for (u32 item = blockIdx.x; item < total; item += gridDim.x) {
-    u32 lo = 0, hi = nparts - 1;  // last part with item_off[p] <= item
+    u32 lo = 0, hi = cap - 1;  // last part with item_off[p] <= item
     while (lo < hi) {
       u32 m = (lo + hi + 1) >> 1;
       if (item_off[m] <= item) lo = m; else hi = m - 1;
@@ -265,20 +303,45 @@ k_part_stats(const u64* __restrict__ ab, const u32* __restrict__ item_off, u32 n
         for (int k = 0; k < 8; k++)
           if (l[k]) atomicAdd(L + 1 + k, (unsigned long long)l[k]);
         atomicMin((unsigned long long*)&mm[p], (unsigned long long)mn);
-        atomicMax((unsigned long long*)&mm[nparts + p], (unsigned long long)mx);
+        atomicMax((unsigned long long*)&mm[cap + p], (unsigned long long)mx);
       }
     }
     __syncthreads();
   }
 }
 
+void launch_part_offsets(const u32* nt, u32 nseg, u32* part_off, cudaStream_t s) {
+  SV_LAUNCH(k_part_offsets, 1, 1024, 0, s)(nt, nseg, part_off);
+}
+
 void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
-                       const u64* T, u32 tstride, const u32* nt, const u32* part_off, u32 nparts,
+                       const u64* T, u32 tstride, const u32* nt, const u32* part_off, u32 cap,
                        const u64* vals, u32 vshift, u32* items, void* scan_temp, u64* lanes, u64* mm,
                        u64* ab, cudaStream_t s) {
-  if (!nparts) return;
-  SV_LAUNCH(k_part_ranges, div_up(nparts, 128), 128, 0, s)(segs, nseg, G, gtab, off, T, tstride, nt,
-                                                          part_off, nparts, ab, items);
-  scan_u32(items, items, nparts, scan_temp, items + nparts, s);
-  SV_LAUNCH(k_part_stats, (u32)sv_num_sms() * 8, PS_THREADS, 0, s)(ab, items, nparts, vals, vshift, lanes, mm);
+  if (!cap) return;
+  SV_LAUNCH(k_part_ranges, div_up(cap, 128), 128, 0, s)(segs, nseg, G, gtab, off, T, tstride, nt,
+                                                       part_off, cap, ab, items);
+  scan_u32(items, items, cap, scan_temp, items + cap, s);
+  SV_LAUNCH(k_part_stats, (u32)sv_num_sms() * 8, PS_THREADS, 0, s)(ab, items, cap, vals, vshift, lanes, mm);
+}
+
+// the round's results in one record per live part, written straight into mapped (zero-copy)
+// host memory: out[0] = number of parts, then per part {lanes[9], min, max, ia, ib}
+__global__ void k_part_pack(const u32* __restrict__ part_off, u32 nseg, u32 cap, const u64* __restrict__ lanes,
+                            const u64* __restrict__ mm, const u64* __restrict__ ab, u64* out) {
+  const u32 nparts = part_off[nseg];
+  u32 p = blockIdx.x * blockDim.x + threadIdx.x;
+  if (p == 0) out[0] = nparts;
+  if (p >= nparts) return;
+  u64* o = out + 1 + (u64)p * PART_REC;
+  for (int k = 0; k < MOM_LANES; k++) o[k] = lanes[(u64)p * MOM_LANES + k];
+  o[MOM_LANES] = mm[p];
+  o[MOM_LANES + 1] = mm[cap + p];
+  o[MOM_LANES + 2] = ab[4 * (u64)p + 2];
+  o[MOM_LANES + 3] = ab[4 * (u64)p + 3];
+}
+
+void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, const u64* mm,
+                      const u64* ab, u64* out, cudaStream_t s) {
+  SV_LAUNCH(k_part_pack, div_up(std::max<u32>(cap, 1), 128), 128, 0, s)(part_off, nseg, cap, lanes, mm, ab, out);
 }

@@ -110,14 +110,20 @@ void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D
                     u32 tstride, u32* nt, u32* kind, cudaStream_t s);
 
 // ---------------- part moments (A13 f) ----------------------------------------------------------
-// parts of segment s: q = 0..nt[s]; part_off[s] = first part index (exclusive scan of nt+1)
-// out (accumulated: lanes zeroed, mm[0..nparts) = ~0 and mm[nparts..2 nparts) = 0 by the
-// caller): lanes[p*9..] (n, S1 limbs, S2 limbs), mm (min, max), ab[p*4..] = value interval
-// [a, b) and this rank's superset range [ia, ib) in the bucketed values
+// parts of segment s: q = 0..nt[s]; part_off[s] = first part index (exclusive scan of nt + 1, on
+// the device), part_off[nseg] = number of parts (<= cap = nseg * tstride)
+void launch_part_offsets(const u32* nt, u32 nseg, u32* part_off, cudaStream_t s);
+// out (accumulated: lanes zeroed, mm[0..cap) = ~0 and mm[cap..2 cap) = 0 by the caller):
+// lanes[p*9..] (n, S1 limbs, S2 limbs), mm (min, max), ab[p*4..] = value interval [a, b) and this
+// rank's superset range [ia, ib) in the bucketed values
 void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
-                       const u64* T, u32 tstride, const u32* nt, const u32* part_off, u32 nparts,
-                       const u64* vals, u32 vshift, u32* items /* [nparts + 1] */, void* scan_temp,
+                       const u64* T, u32 tstride, const u32* nt, const u32* part_off, u32 cap,
+                       const u64* vals, u32 vshift, u32* items /* [cap + 1] */, void* scan_temp,
                        u64* lanes, u64* mm, u64* ab, cudaStream_t s);
+#define PART_REC (MOM_LANES + 4)
+// out[0] = parts, out[1 + p * PART_REC ..] = {lanes[9], min, max, ia, ib} (mapped host memory)
+void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, const u64* mm,
+                      const u64* ab, u64* out, cudaStream_t s);
 // ---------------- pass B: assignment + per-(stratum, CTA) statistics -------------------
 struct KTab {      // per kernel
   u32 base;        // global id of its first stratum
