@@ -25,10 +25,11 @@ def fma(a, b, c):
 
 
 def _exp2_neg_table():
-    """2^(-j/256), j = 0..255, correctly rounded (60-digit decimal, then float() rounds)."""
+    """2^(-j/256), j = 1..255, correctly rounded (60-digit decimal, then float() rounds); entry 0
+    is 1 - 2^-53 (A10: no term is an exact half-integer)."""
     from decimal import Decimal, getcontext
     getcontext().prec = 60
-    return [float(Decimal(2) ** (Decimal(-j) / Decimal(256))) for j in range(256)]
+    return [1.0 - 2.0 ** -53] + [float(Decimal(2) ** (Decimal(-j) / Decimal(256))) for j in range(1, 256)]
 
 
 EXP2_NEG = _exp2_neg_table()

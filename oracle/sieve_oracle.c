@@ -195,7 +195,10 @@ double oracle_grid_point(uint64_t lo, uint64_t hi, uint32_t j, uint32_t G) {
  *   e^{-t} = 2^{-j/256} * 2^{-m} * e^{-r}
  *   Q = rint(P * T_j * 2^(40 - m)) with ONE rounding: S = ldexp(T_j, 40 - m) is exact and
  *       Q = fma(P, S, 2^52) - 2^52 (the fma lands in [2^52, 2^53), where the ulp is 1).
- *   T_j = 2^{-j/256} correctly rounded (pinned in tests against Python's decimal module).
+ *   T_j = 2^{-j/256} correctly rounded for j >= 1 (pinned in tests against Python's decimal
+ *       module), T_0 = 1 - 2^-53: with every T_j having fewer than 12 trailing zero bits in its
+ *       significand, P * S can never be an exact half-integer (pinned), so Q does not depend on
+ *       a tie rule and a sum of terms may be rounded into an accumulator in any order.
  * Q = 0 for k > 10526 (t > 28.5014): there e^{-t} 2^40 < 0.47 rounds to 0 anyway.
  * Fixed point at 2^-40 of one kernel's peak: the relative accuracy of P T_j (< 2^-42) keeps
  * every Q within one unit of e^{-t} 2^40 (pinned).
@@ -205,7 +208,7 @@ static const double OR_LN2_256 = 0x1.62e42fefa39efp-9;                  /* rn(ln
 static const double OR_TWO52 = 4503599627370496.0;
 static const double OR_KMAX = 10526.0;                                  /* rint(28.5 * 256 log2 e) */
 static const double OR_EXP2_NEG[256] = {
-    0x1.0000000000000p+0, 0x1.fe9d96b2a23d9p-1, 0x1.fd3c22b8f71f1p-1, 0x1.fbdba3692d514p-1,
+    0x1.fffffffffffffp-1, /* 1 - 2^-53, not 1: see T_j above */ 0x1.fe9d96b2a23d9p-1, 0x1.fd3c22b8f71f1p-1, 0x1.fbdba3692d514p-1,
     0x1.fa7c1819e90d8p-1, 0x1.f91d802243c89p-1, 0x1.f7bfdad9cbe14p-1, 0x1.f6632798844f8p-1,
     0x1.f50765b6e4540p-1, 0x1.f3ac948dd7274p-1, 0x1.f252b376bba97p-1, 0x1.f0f9c1cb6412ap-1,
     0x1.efa1bee615a27p-1, 0x1.ee4aaa2188510p-1, 0x1.ecf482d8e67f1p-1, 0x1.eb9f4867cca6ep-1,

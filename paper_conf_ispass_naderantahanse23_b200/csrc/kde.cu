@@ -112,8 +112,9 @@ __global__ void k_kde_items(const u32* tile_items, u32 ntiles, u32* item_tile) {
 #define C_P1 (-0.5)                             // -1       * 2^-1
 #define C_P0 1.0
 
+// 2^(-j/256) correctly rounded for j >= 1; entry 0 is 1 - 2^-53 (A10: no exact ties, see kde_acc)
 __constant__ double KDE_EXP2_NEG[256] = {
-    0x1.0000000000000p+0, 0x1.fe9d96b2a23d9p-1, 0x1.fd3c22b8f71f1p-1, 0x1.fbdba3692d514p-1,
+    0x1.fffffffffffffp-1, 0x1.fe9d96b2a23d9p-1, 0x1.fd3c22b8f71f1p-1, 0x1.fbdba3692d514p-1,
     0x1.fa7c1819e90d8p-1, 0x1.f91d802243c89p-1, 0x1.f7bfdad9cbe14p-1, 0x1.f6632798844f8p-1,
     0x1.f50765b6e4540p-1, 0x1.f3ac948dd7274p-1, 0x1.f252b376bba97p-1, 0x1.f0f9c1cb6412ap-1,
     0x1.efa1bee615a27p-1, 0x1.ee4aaa2188510p-1, 0x1.ecf482d8e67f1p-1, 0x1.eb9f4867cca6ep-1,
@@ -183,10 +184,14 @@ __constant__ double c_kde[3] = {C_LOG2E_128, C_LN2_128, C_P3};
 
 struct KdeRegs { double log2e, magic; };  // operands that must sit in registers (see below)
 
-// raw bit pattern of fma(P, S, 2^52); the term is this minus bits(2^52)
+// acc + Q: the term's final fma adds rint(P * S) straight into an integer-valued accumulator in
+// [2^52, 2^53) (ulp 1).  rn(acc + P*S) = acc + rint(P*S) exactly because P*S is never an exact
+// half-integer: with p, s the odd significands of P and S, P*S = p*s*2^(a+b) has fraction 1/2
+// only if a + b = -1, which needs >= 12 trailing zero bits in T_j' (A10 sets T_0 = 1 - 2^-53; the
+// other entries have <= 6, pinned in tests), so the sum is exact in any order.
 template <bool GUARD>
-__device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, const double* sS,
-                                         KdeRegs R) {
+__device__ __forceinline__ double kde_acc(double g, double xd, double inv_h, const double* sS,
+                                          KdeRegs R, double acc) {
   double z = __dmul_rn(__dsub_rn(g, xd), inv_h);
   double u = __dmul_rn(z, z);                               // 2t, exactly
   double kb = __fma_rn(u, R.log2e, R.magic);                // one rounding: nearest integer
@@ -197,14 +202,14 @@ __device__ __forceinline__ u64 kde_qbits(double g, double xd, double inv_h, cons
   // boundary cells of the bucketed range: 7.6 + 33 * 140 < 4800) and runs the
   // unguarded variant; otherwise any u >= 80 is sent to the zero entry explicitly.  p stays
   // finite for every input the API admits (x < 2^44, n < 2^36 => h > 2^-26, u < 2^140), and
-  // fma(p, 0, 2^52) = 2^52.
+  // fma(p, 0, acc) = acc.
   u32 k = min((u32)__double2loint(kb), (u32)KDE_KCUT);
   if (GUARD) k = (u32)__double2hiint(u) >= 0x40540000u ? (u32)KDE_KCUT : k;
   double r = __fma_rn(-kf, c_kde[1], u);
   double p = __fma_rn(c_kde[2], r, C_P2);
   p = __fma_rn(p, r, C_P1);
   p = __fma_rn(p, r, C_P0);
-  return (u64)__double_as_longlong(__fma_rn(p, sS[k], C_TWO52));
+  return __fma_rn(p, sS[k], acc);
 }
 
 #define KDE_SMEM_TABLE ((KDE_KCUT + 1) * 8)
@@ -255,30 +260,23 @@ k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ v
     u32 j = t * KDE_TJ + lane % KDE_TJ;
     double inv_h = g.inv_h;
     double gj = grid_pt(g.lo, g.hi, j < G ? j : G - 1, G);
-    u64 acc = 0;
     u32 i = slice;
     const double* sSb = sS;
-#if KDE_UNROLL > 4
+    // KDE_UNROLL independent accumulators, each an integer in [2^52, 2^53): a lane adds at most
+    // KDE_CH terms of <= 2^40 per item
+    double ac[KDE_UNROLL];
+#pragma unroll
+    for (int q = 0; q < KDE_UNROLL; q++) ac[q] = C_TWO52;
     for (; i + (KDE_UNROLL - 1) * KDE_V < len; i += KDE_UNROLL * KDE_V) {
-      u64 b[KDE_UNROLL];
 #pragma unroll
-      for (int q = 0; q < KDE_UNROLL; q++) b[q] = kde_qbits<GUARD>(gj, sx[i + q * KDE_V], inv_h, sSb, R);
+      for (int q = 0; q < KDE_UNROLL; q++) ac[q] = kde_acc<GUARD>(gj, sx[i + q * KDE_V], inv_h, sSb, R, ac[q]);
+    }
 #pragma unroll
-      for (int q = 1; q < KDE_UNROLL; q++) b[0] += b[q];  // integer sums: order is irrelevant
-      acc += b[0];
-    }
-#endif
-    for (; i + 3 * KDE_V < len; i += 4 * KDE_V) {
-      u64 b0 = kde_qbits<GUARD>(gj, sx[i], inv_h, sSb, R);
-      u64 b1 = kde_qbits<GUARD>(gj, sx[i + KDE_V], inv_h, sSb, R);
-      u64 b2 = kde_qbits<GUARD>(gj, sx[i + 2 * KDE_V], inv_h, sSb, R);
-      u64 b3 = kde_qbits<GUARD>(gj, sx[i + 3 * KDE_V], inv_h, sSb, R);
-      acc += (b0 + b1) + (b2 + b3);
-    }
-    for (; i < len; i += KDE_V) acc += kde_qbits<GUARD>(gj, sx[i], inv_h, sSb, R);
-    // remove 2^52's bit pattern once per term this lane evaluated, then sum the value slices
-    u32 nterm = len > slice ? (len - slice + KDE_V - 1) / KDE_V : 0;
-    acc -= (u64)nterm * 0x4330000000000000ull;
+    for (int q = 0; q < KDE_UNROLL - 1; q++)
+      if (i + q * KDE_V < len) ac[q] = kde_acc<GUARD>(gj, sx[i + q * KDE_V], inv_h, sSb, R, ac[q]);
+    u64 acc = 0;
+#pragma unroll
+    for (int q = 0; q < KDE_UNROLL; q++) acc += (u64)__double_as_longlong(ac[q]) - 0x4330000000000000ull;
 #pragma unroll
     for (int o = KDE_TJ; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
     if (evaluated && lane == 0) {  // evaluated (lane, value) pairs of this item, wasted ones included

@@ -73,10 +73,11 @@ def _decimal_exp2_neg(j):
 
 def test_exp2_tables_correctly_rounded():
     # the oracle's table and the CUDA path's table (kde.cu literals) are each pinned to the
-    # correctly rounded 2^(-j/256); the two sides share no table generator
+    # correctly rounded 2^(-j/256) for j >= 1 and to 1 - 2^-53 for j = 0 (A10); the two sides
+    # share no table generator
     import os
     import re
-    want = [_decimal_exp2_neg(j) for j in range(256)]
+    want = [1.0 - 2.0 ** -53] + [_decimal_exp2_neg(j) for j in range(1, 256)]
     assert oracle.exp2_table() == want
     src = open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
                             "paper_conf_ispass_naderantahanse23_b200", "csrc", "kde.cu")).read()
@@ -84,6 +85,34 @@ def test_exp2_tables_correctly_rounded():
     body = body[body.index("{") + 1:body.index("}")]
     got = [float.fromhex(h) for h in re.findall(r"0x[0-9a-fA-F.]+p[+-]?\d+", body)]
     assert got == want
+
+
+def test_q_terms_are_never_ties():
+    """A10: P * T_j * 2^(40-m) is never an exact half-integer, so rint needs no tie rule and the
+    GPU may round each term into an integer-valued fp64 accumulator (kde.cu kde_acc).  P*S =
+    p*s*2^(a+b) (p, s odd) has fraction 1/2 only if a + b = -1.  P < 2 has a <= 0, and
+    S = T * 2^(40-m) with tz trailing zero bits in T's significand has b = tz - 13 - m, so a tie
+    needs tz >= 12 + m.  Pin: every table entry has fewer than 12."""
+    import struct
+    for j, v in enumerate(oracle.exp2_table()):
+        bits = struct.unpack("<Q", struct.pack("<d", v))[0]
+        mant = (bits & ((1 << 52) - 1)) | (1 << 52)
+        tz = (mant & -mant).bit_length() - 1
+        assert tz < 12, (j, tz)
+    # and directly: random terms of every table entry are never exact half-integers, while the
+    # exact power of two T = 1 would produce ties (the reason for 1 - 2^-53)
+    rng = random.Random(11)
+    ties_with_one = 0
+    for _ in range(20000):
+        p = 1.0 + rng.randint(-2 ** 40, 2 ** 40) * 2.0 ** -52
+        p = math.ldexp(math.floor(math.ldexp(p, 41)), -41) if rng.random() < 0.5 else p
+        m = rng.randint(0, 41)
+        for T in (oracle.exp2_table()[rng.randrange(256)],):
+            v = Fraction(p) * Fraction(T) * Fraction(2) ** (40 - m)
+            assert v - math.floor(v) != Fraction(1, 2)
+        w = Fraction(p) * Fraction(2) ** (40 - m)
+        ties_with_one += (w - math.floor(w) == Fraction(1, 2))
+    assert ties_with_one > 0
 
 
 def test_det_exp_relative_accuracy():
