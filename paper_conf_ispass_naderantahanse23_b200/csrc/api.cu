@@ -1040,107 +1040,109 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   SV_TRY(h2d(c, d_lows.get(), lows));
   u64 cap = 1;
   while (cap < std::max<u64>(1u << 16, 8ull * ns)) cap <<= 1;
-  DBuf<u64> gkeys(c), gcnt(c), gfirst(c);
-  u64 E = 0;
-  DBuf<u64> ekey(c), ecnt(c), efirst(c);
+  // One rank: the (stratum, CTA) entries go to the representatives without a host round trip --
+  // the compacted arrays are pre-filled with neutral entries (key ~0 sorts last, count 0), so
+  // every later launch can be sized by the table capacity; the overflow flag is read with the
+  // representatives (one synchronisation) and an overflow redoes pass B with a bigger table.
+  // Several ranks: the entry counts are exchanged first (AR-4 needs them on the host).
+  std::vector<u64> h_rep, h_xy, hflag;
   for (int attempt = 0;; attempt++) {
+    if (attempt > 6) return sv_fail(SIEVE_ENOMEM, "(stratum, CTA) table kept overflowing");
+    DBuf<u64> gkeys(c), gcnt(c), gfirst(c), ent(c);
     SV_TRY(gkeys.alloc(cap)); SV_TRY(gcnt.alloc(cap)); SV_TRY(gfirst.alloc(cap));
     launch_fill_u64(gkeys.get(), cap, HASH_EMPTY, S);
     SV_CUDA(cudaMemsetAsync(gcnt.get(), 0, cap * 8, S));
     launch_fill_u64(gfirst.get(), cap, ~0ull, S);
     SV_CUDA(cudaMemsetAsync(errf.get(), 0, 32, S));
     GHash gh{gkeys.get(), gcnt.get(), gfirst.get(), cap};
-    PhaseTimer tb(c, SIEVE_PHASE_ASSIGN, n * (12 + (t->cta ? 4 : 0) + (sid_out ? 4 : 0)));
-    launch_assign(t->kid, t->x, t->cta, n, t->first_id, d_ktab.get(), d_lows.get(), K,
-                  (u32)lows.size(), sid_out, gh, errf.get(), assign_grid(), S);
-    tb.stop();
+    {
+      PhaseTimer tb(c, SIEVE_PHASE_ASSIGN, n * (12 + (t->cta ? 4 : 0) + (sid_out ? 4 : 0)));
+      launch_assign(t->kid, t->x, t->cta, n, t->first_id, d_ktab.get(), d_lows.get(), K,
+                    (u32)lows.size(), sid_out, gh, errf.get(), assign_grid(), S);
+    }
     SV_CUDA(cudaGetLastError());
-    SV_TRY(ekey.alloc(cap)); SV_TRY(ecnt.alloc(cap)); SV_TRY(efirst.alloc(cap));
+    // ent = [keys | counts | firsts], cap each
+    SV_TRY(ent.alloc(cap * 3));
+    launch_fill_u64(ent.get(), cap, ~0ull, S);
+    SV_CUDA(cudaMemsetAsync(ent.get() + cap, 0, cap * 8, S));
+    launch_fill_u64(ent.get() + 2 * cap, cap, ~0ull, S);
     SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
-    launch_hash_compact(gh, ekey.get(), ecnt.get(), efirst.get(), counter.get(), S);
-    std::vector<u64> hflag;
-    std::vector<unsigned long long> hcnt;
-    SV_TRY(d2h(c, hflag, errf.get(), 4));
-    SV_TRY(d2h(c, hcnt, counter.get(), 1));
-    SV_TRY(sync(c));
-    // the retry decision must be identical on every rank
-    std::vector<u64> gfl{hflag[2]};
+    launch_hash_compact(gh, ent.get(), ent.get() + cap, ent.get() + 2 * cap, counter.get(), S);
+    u64 Etot = cap;
+    const u64* ak = ent.get();
+    DBuf<u64> akb(c);
     if (c->comm) {
+      std::vector<unsigned long long> hcnt;
+      SV_TRY(d2h(c, hflag, errf.get(), 4));
+      SV_TRY(d2h(c, hcnt, counter.get(), 1));
+      SV_TRY(sync(c));
+      // the retry decision must be identical on every rank
+      std::vector<u64> gfl{hflag[2]};
       DBuf<u64> fl(c);
       SV_TRY(fl.alloc(1));
       SV_TRY(h2d(c, fl.get(), gfl));
       SV_TRY(allreduce(c, fl.get(), 1, RED_MAX));
       SV_TRY(d2h(c, gfl, fl.get(), 1));
       SV_TRY(sync(c));
+      if (gfl[0]) { cap <<= 2; continue; }
+      const u64 E = hcnt[0];
+      // gather every rank's entries (AR-4: all-gather expressed as a SUM over zero-padded slots)
+      DBuf<u64> cnts(c);
+      SV_TRY(cnts.alloc(c->world));
+      std::vector<u64> mine(c->world, 0);
+      mine[c->rank] = E;
+      SV_TRY(h2d(c, cnts.get(), mine));
+      SV_TRY(allreduce(c, cnts.get(), c->world, RED_SUM));
+      std::vector<u64> all;
+      SV_TRY(d2h(c, all, cnts.get(), c->world));
+      SV_TRY(sync(c));
+      Etot = 0;
+      u64 Eoff = 0;
+      for (int r = 0; r < c->world; r++) { if (r == c->rank) Eoff = Etot; Etot += all[r]; }
+      SV_TRY(akb.alloc(std::max<u64>(Etot, 1) * 3));
+      SV_CUDA(cudaMemsetAsync(akb.get(), 0, Etot * 3 * 8, S));
+      SV_CUDA(cudaMemcpyAsync(akb.get() + Eoff, ent.get(), E * 8, cudaMemcpyDeviceToDevice, S));
+      SV_CUDA(cudaMemcpyAsync(akb.get() + Etot + Eoff, ent.get() + cap, E * 8, cudaMemcpyDeviceToDevice, S));
+      SV_CUDA(cudaMemcpyAsync(akb.get() + 2 * Etot + Eoff, ent.get() + 2 * cap, E * 8, cudaMemcpyDeviceToDevice, S));
+      SV_TRY(allreduce(c, akb.get(), Etot * 3, RED_SUM));
+      ak = akb.get();
     }
-    if (!gfl[0]) { E = hcnt[0]; break; }
-    if (attempt > 6) return sv_fail(SIEVE_ENOMEM, "(stratum, CTA) table kept overflowing");
-    cap <<= 2;
-  }
-  gkeys.release(); gcnt.release(); gfirst.release();
-  hc.mark("passB");
-  // gather every rank's entries (AR-4: all-gather expressed as a SUM over zero-padded slots)
-  u64 Etot = E, Eoff = 0;
-  DBuf<u64> ak(c), ac(c), af(c);
-  if (c->comm) {
-    DBuf<u64> cnts(c);
-    SV_TRY(cnts.alloc(c->world));
-    std::vector<u64> mine(c->world, 0);
-    mine[c->rank] = E;
-    SV_TRY(h2d(c, cnts.get(), mine));
-    SV_TRY(allreduce(c, cnts.get(), c->world, RED_SUM));
-    std::vector<u64> all;
-    SV_TRY(d2h(c, all, cnts.get(), c->world));
+    hc.mark("passB");
+    // sort entries by (stratum, CTA) with their index as payload, then gather count / first;
+    // nbits covers every stratum id with a spare bit, so a neutral key (~0) sorts last
+    DBuf<u32> idx(c);
+    DBuf<u64> sk(c), scnt(c), sfirst(c);
+    SV_TRY(idx.alloc(std::max<u64>(Etot, 1)));
+    SV_TRY(sk.alloc(std::max<u64>(Etot, 1))); SV_TRY(scnt.alloc(std::max<u64>(Etot, 1)));
+    SV_TRY(sfirst.alloc(std::max<u64>(Etot, 1)));
+    launch_iota_u32(idx.get(), Etot, S);
+    SV_CUDA(cudaMemcpyAsync(sk.get(), ak, Etot * 8, cudaMemcpyDeviceToDevice, S));
+    PhaseTimer tr(c, SIEVE_PHASE_REPS, 0);
+    {
+      DBuf<char> tmp(c);
+      SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
+      SV_TRY(radix_sort(sk.get(), idx.get(), Etot, 32 + (int)bitlen(ns), tmp.get(), S));
+    }
+    launch_gather_u64(ak + Etot, idx.get(), Etot, scnt.get(), S);
+    launch_gather_u64(ak + 2 * Etot, idx.get(), Etot, sfirst.get(), S);
+    DBuf<u32> d_tier(c);
+    DBuf<u64> rep(c), repxy(c);
+    SV_TRY(d_tier.alloc(ns));
+    SV_TRY(rep.alloc(2 * (size_t)ns));
+    SV_TRY(repxy.alloc(2 * (size_t)ns));
+    SV_TRY(h2d(c, d_tier.get(), tiers));
+    launch_reps(sk.get(), scnt.get(), sfirst.get(), Etot, d_tier.get(), ns, rep.get(), rep.get() + ns, S);
+    launch_rep_xy(rep.get(), ns, t->first_id, n, t->x, t->y, repxy.get(), S);
+    tr.stop();
+    SV_CUDA(cudaGetLastError());
+    SV_TRY(allreduce(c, repxy.get(), 2 * (size_t)ns, RED_SUM));   // AR-5: owner contributes
+    SV_TRY(d2h(c, h_rep, rep.get(), 2 * (size_t)ns));
+    SV_TRY(d2h(c, h_xy, repxy.get(), 2 * (size_t)ns));
+    if (!c->comm) SV_TRY(d2h(c, hflag, errf.get(), 4));
     SV_TRY(sync(c));
-    Etot = 0;
-    for (int r = 0; r < c->world; r++) { if (r == c->rank) Eoff = Etot; Etot += all[r]; }
-    SV_TRY(ak.alloc(Etot * 3));
-    SV_CUDA(cudaMemsetAsync(ak.get(), 0, Etot * 3 * 8, S));
-    SV_CUDA(cudaMemcpyAsync(ak.get() + Eoff, ekey.get(), E * 8, cudaMemcpyDeviceToDevice, S));
-    SV_CUDA(cudaMemcpyAsync(ak.get() + Etot + Eoff, ecnt.get(), E * 8, cudaMemcpyDeviceToDevice, S));
-    SV_CUDA(cudaMemcpyAsync(ak.get() + 2 * Etot + Eoff, efirst.get(), E * 8, cudaMemcpyDeviceToDevice, S));
-    SV_TRY(allreduce(c, ak.get(), Etot * 3, RED_SUM));
-  } else {
-    SV_TRY(ak.alloc(Etot * 3));
-    SV_CUDA(cudaMemcpyAsync(ak.get(), ekey.get(), E * 8, cudaMemcpyDeviceToDevice, S));
-    SV_CUDA(cudaMemcpyAsync(ak.get() + Etot, ecnt.get(), E * 8, cudaMemcpyDeviceToDevice, S));
-    SV_CUDA(cudaMemcpyAsync(ak.get() + 2 * Etot, efirst.get(), E * 8, cudaMemcpyDeviceToDevice, S));
+    if (!c->comm && hflag[2]) { cap <<= 2; continue; }
+    break;
   }
-  ekey.release(); ecnt.release(); efirst.release();
-  // sort entries by (stratum, CTA) with their index as payload, then gather count / first
-  DBuf<u32> idx(c);
-  DBuf<u64> sk(c), scnt(c), sfirst(c);
-  SV_TRY(idx.alloc(Etot));
-  SV_TRY(sk.alloc(Etot)); SV_TRY(scnt.alloc(Etot)); SV_TRY(sfirst.alloc(Etot));
-  {
-    std::vector<u32> iota(Etot);
-    for (u64 i = 0; i < Etot; i++) iota[i] = (u32)i;
-    SV_TRY(h2d(c, idx.get(), iota));
-  }
-  SV_CUDA(cudaMemcpyAsync(sk.get(), ak.get(), Etot * 8, cudaMemcpyDeviceToDevice, S));
-  PhaseTimer tr(c, SIEVE_PHASE_REPS, 0);
-  {
-    DBuf<char> tmp(c);
-    SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
-    SV_TRY(radix_sort(sk.get(), idx.get(), Etot, 32 + (int)bitlen(ns ? ns - 1 : 0), tmp.get(), S));
-  }
-  launch_gather_u64(ak.get() + Etot, idx.get(), Etot, scnt.get(), S);
-  launch_gather_u64(ak.get() + 2 * Etot, idx.get(), Etot, sfirst.get(), S);
-  DBuf<u32> d_tier(c);
-  DBuf<u64> rep(c), repxy(c);
-  SV_TRY(d_tier.alloc(ns));
-  SV_TRY(rep.alloc(2 * (size_t)ns));
-  SV_TRY(repxy.alloc(2 * (size_t)ns));
-  SV_TRY(h2d(c, d_tier.get(), tiers));
-  launch_reps(sk.get(), scnt.get(), sfirst.get(), Etot, d_tier.get(), ns, rep.get(), rep.get() + ns, S);
-  launch_rep_xy(rep.get(), ns, t->first_id, n, t->x, t->y, repxy.get(), S);
-  tr.stop();
-  SV_CUDA(cudaGetLastError());
-  SV_TRY(allreduce(c, repxy.get(), 2 * (size_t)ns, RED_SUM));   // AR-5: owner contributes
-  std::vector<u64> h_rep, h_xy;
-  SV_TRY(d2h(c, h_rep, rep.get(), 2 * (size_t)ns));
-  SV_TRY(d2h(c, h_xy, repxy.get(), 2 * (size_t)ns));
-  SV_TRY(sync(c));
   resolve_timing(c);
   R->kde_terms = h_terms[0];
   R->kde_evaluated = h_terms[1];

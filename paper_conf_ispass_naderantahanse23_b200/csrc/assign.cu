@@ -189,6 +189,14 @@ void launch_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst, unsigned l
   SV_LAUNCH(k_hash_compact, div_up(gh.cap, 256), 256, 0, s)(gh, okey, ocnt, ofirst, count);
 }
 
+__global__ void k_iota_u32(u32* p, u64 n) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = (u32)i;
+}
+void launch_iota_u32(u32* p, u64 n, cudaStream_t s) {
+  if (n) SV_LAUNCH(k_iota_u32, div_up(n, 256), 256, 0, s)(p, n);
+}
+
 __global__ void k_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst) {
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) dst[i] = src[idx[i]];

@@ -146,6 +146,7 @@ void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 firs
 void launch_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst, unsigned long long* count,
                          cudaStream_t s);
 void launch_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst, cudaStream_t s);
+void launch_iota_u32(u32* p, u64 n, cudaStream_t s);
 // reduce duplicates of equal keys (sorted) and pick each stratum's representative
 void launch_reps(const u64* key, const u64* cnt, const u64* first, u64 E, const u32* tier,
                  u32 nstrata, u64* rep_id, u64* rep_cta, cudaStream_t s);

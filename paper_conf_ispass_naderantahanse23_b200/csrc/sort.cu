@@ -235,6 +235,7 @@ k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int s
           const u32* __restrict__ gbase, u64* status, u32* tile_counter, u64* __restrict__ kout,
           u32* __restrict__ vout) {
   extern __shared__ __align__(16) unsigned char smem[];
+  const int dbits = __popc(dmask);
   u64* s_k = (u64*)smem;                        // [RS_TILE]
   u32* s_v = (u32*)(s_k + RS_TILE);             // [RS_TILE] (if values)
   __shared__ u32 s_wh[RS_WARPS][256];           // per-warp digit counts -> warp offsets
@@ -268,6 +269,7 @@ k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int s
     if (!ok) peers = ~peers;
 #pragma unroll
     for (int b = 0; b < 8; b++) {
+      if (b >= dbits) break;  // narrow last digit: fewer ballots (uniform branch)
       u32 m = __ballot_sync(0xffffffffu, (d >> b) & 1u);
       peers &= ((d >> b) & 1u) ? m : ~m;
     }
