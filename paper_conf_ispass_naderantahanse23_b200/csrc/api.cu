@@ -896,7 +896,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       for (u32 s = 0; s < nseg; s++)
         if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 140.0 * hs[s].h) guard = true;
       launch_kde(segs.get(), nseg, G, ck.get(), ib, tile_range.get(), tile_items.get(),
-                 (u32*)item_tile.get(), items, D.get(), counter.get() + 1, terms.get() + 1, guard, S);
+                 item_tile.get(), items, D.get(), terms.get() + 1, guard, S);
       tm.stop();
       SV_CUDA(cudaGetLastError());
     }

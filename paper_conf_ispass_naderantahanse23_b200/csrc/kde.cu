@@ -36,10 +36,10 @@
 #define KDE_W 7.6            // window half-width in units of h: k > 10526 (t > 28.5014) beyond it
 #define KDE_KCUT 10527       // k > 10526 = rint(28.5 * 256 log2 e) -> index 10527 holds 0
 #ifndef KDE_WARPS
-#define KDE_WARPS 12         // warps per block (independent work-item consumers)
+#define KDE_WARPS 24         // warps per block (independent work-item consumers)
 #endif
 #ifndef KDE_MINB
-#define KDE_MINB 2           // resident blocks per SM (84 KB table + 24 KB staging each)
+#define KDE_MINB 1           // resident blocks per SM: one 64 KB table shared by 24 warps
 #endif
 #ifndef KDE_UNROLL
 #define KDE_UNROLL 8         // terms in flight per lane
@@ -87,9 +87,25 @@ void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32
   scan_u32(tile_items, tile_items, nt, scan_temp, tile_items + nt, s);
 }
 
-// item -> tile map (so a warp finds its tile with one load): one thread per item, binary
-// search of the last tile whose first item is <= it
-__global__ void k_kde_items(const u32* tile_items, u32 ntiles, u32* item_tile) {
+// one work item's descriptor, built on the device so a warp can prefetch it with one
+// asynchronous 48-byte copy: value range, first grid point and the segment's grid parameters
+struct __align__(16) KdeItem {
+  u64 va;        // first value (index into the sorted cell keys)
+  u32 len;       // values (<= KDE_CH)
+  u32 j0;        // first grid point of the tile
+  u64 lo, hi;    // segment range (grid g_j = rn(lo) + rn((hi - lo) j) / rn(G - 1))
+  double inv_h;
+  u32 s;         // segment
+  unsigned short live;    // grid points of the tile that exist (< KDE_TJ only in the last tile)
+  unsigned short fast;    // 1: every evaluated |z| < 18.8 (Delta / h < 0.33), so MODE 0 is exact
+};
+static_assert(sizeof(KdeItem) == 48, "KdeItem is copied as three 16-byte pieces");
+
+// item -> descriptor: one thread per item, binary search of the last tile whose first item is
+// <= it
+__global__ void k_kde_items(const SegDev* __restrict__ segs, u32 G, u32 tps,
+                            const u64* __restrict__ tile_range, const u32* __restrict__ tile_items,
+                            u32 ntiles, KdeItem* __restrict__ desc) {
   const u32 items = tile_items[ntiles];  // device-side total (no host round trip)
   for (u32 it = blockIdx.x * blockDim.x + threadIdx.x; it < items; it += gridDim.x * blockDim.x) {
     u32 lo = 0, hi = ntiles - 1;
@@ -97,9 +113,33 @@ __global__ void k_kde_items(const u32* tile_items, u32 ntiles, u32* item_tile) {
       u32 m = (lo + hi + 1) >> 1;
       if (tile_items[m] <= it) lo = m; else hi = m - 1;
     }
-    item_tile[it] = lo;
+    const u32 tile = lo, s = tile / tps, t = tile % tps;
+    const SegDev g = segs[s];
+    KdeItem d;
+    d.va = tile_range[2 * (u64)tile] + (u64)(it - tile_items[tile]) * KDE_CH;
+    d.len = (u32)min((u64)KDE_CH, tile_range[2 * (u64)tile + 1] - d.va);
+    d.j0 = t * KDE_TJ;
+    d.lo = g.lo;
+    d.hi = g.hi;
+    d.inv_h = g.inv_h;
+    d.s = s;
+    d.live = (unsigned short)min((u32)KDE_TJ, G - d.j0);
+    // |z| <= 7.6 (window) + 33 grid steps (31 lanes + the two boundary cells) in units of h
+    d.fast = (double)(g.hi - g.lo) < 0.33 * g.h * (double)(G - 1);
+    desc[it] = d;
   }
 }
+
+__device__ __forceinline__ void cp_async8(void* sdst, const void* gsrc) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"((u32)__cvta_generic_to_shared(sdst)),
+               "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async16(void* sdst, const void* gsrc) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"((u32)__cvta_generic_to_shared(sdst)),
+               "l"(gsrc) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
 // ------------------------------------------------------------------------------------------
 #define C_LOG2E_128 0x1.71547652b82fep+7     // 128 * log2(e)  (= the oracle's 256 log2 e / 2)
@@ -189,46 +229,109 @@ struct KdeRegs { double log2e, magic; };  // operands that must sit in registers
 // half-integer: with p, s the odd significands of P and S, P*S = p*s*2^(a+b) has fraction 1/2
 // only if a + b = -1, which needs >= 12 trailing zero bits in T_j' (A10 sets T_0 = 1 - 2^-53; the
 // other entries have <= 6, pinned in tests), so the sum is exact in any order.
-template <bool GUARD>
+#ifndef KDE_SPLIT
+#define KDE_SPLIT 1          // 1: lane-replicated 256-entry table + exponent arithmetic (below)
+#endif
+#define KDE_KCLAMP 16383     // KDE_SPLIT: k is clamped here; m = k div 256 <= 63 keeps S normal
+
+// MODE 0: no clamp (the item's |z| < 18.8, so k < 65536 and the byte permutes below see k
+// itself; with m = k div 256 <= 255 the scaled entry stays normal); MODE 1: k clamped to
+// KDE_KCLAMP; MODE 2: clamp plus the explicit large-u guard (see below).
+template <int MODE>
 __device__ __forceinline__ double kde_acc(double g, double xd, double inv_h, const double* sS,
                                           KdeRegs R, double acc) {
   double z = __dmul_rn(__dsub_rn(g, xd), inv_h);
   double u = __dmul_rn(z, z);                               // 2t, exactly
   double kb = __fma_rn(u, R.log2e, R.magic);                // one rounding: nearest integer
   double kf = __dsub_rn(kb, C_MAGIC);
-  // k = rint(u * 128 log2 e); any k > 10526 maps to the zero entry.  The low word of kb is k
+  // k = rint(u * 128 log2 e); any k > 10526 contributes 0.  The low word of kb is k
   // while k < 2^32, i.e. u < 2.3e7: the host proves |z| < 4800 for every (lane, value) pair of
   // a launch when max Delta/h < 140 (window 7.6 h plus KDE_TJ-1 = 31 grid steps plus the two
   // boundary cells of the bucketed range: 7.6 + 33 * 140 < 4800) and runs the
-  // unguarded variant; otherwise any u >= 80 is sent to the zero entry explicitly.  p stays
-  // finite for every input the API admits (x < 2^44, n < 2^36 => h > 2^-26, u < 2^140), and
-  // fma(p, 0, acc) = acc.
+  // unguarded variant; otherwise any u >= 80 is sent to a zero-contribution index explicitly.
+  // p stays finite for every input the API admits (x < 2^44, n < 2^36 => h > 2^-26, u < 2^140).
+#if KDE_SPLIT
+  // S = T'[k] = (2^{-(k mod 256)/256} 2^40) * 2^-(k div 256): the 256-entry table is replicated
+  // once per lane (entry e of replica l at byte 256 e + 8 l, so the lanes of every 128-byte
+  // wavefront hit distinct bank pairs: conflict-free for any pattern of k), and the power of
+  // two is applied exactly by subtracting (k div 256) from the exponent field.  The byte
+  // permutes give (k mod 256) << 8 and (k div 256) << 16 in one instruction each.  For
+  // 10526 < k <= KDE_KCLAMP, P * S <= 1.0014 * 2^(40 - 10527/256) < 0.47, so
+  // fma(P, S, acc) = acc exactly: the term is 0 as A10 defines, with no select.
+  u32 k = (u32)__double2loint(kb);
+  if (MODE >= 1) k = min(k, (u32)KDE_KCLAMP);
+  if (MODE == 2) k = (u32)__double2hiint(u) >= 0x40540000u ? (u32)KDE_KCLAMP : k;
+  double T = *(const double*)((const char*)sS + __byte_perm(k, 0u, 0x4404u));
+  double S = __hiloint2double(__double2hiint(T) - (int)(__byte_perm(k, 0u, 0x4144u) << 4),
+                              __double2loint(T));
+#else
+  // fma(p, 0, acc) = acc for the zero entry T'[KDE_KCUT]
   u32 k = min((u32)__double2loint(kb), (u32)KDE_KCUT);
-  if (GUARD) k = (u32)__double2hiint(u) >= 0x40540000u ? (u32)KDE_KCUT : k;
+  if (MODE == 2) k = (u32)__double2hiint(u) >= 0x40540000u ? (u32)KDE_KCUT : k;
+  double S = sS[k];
+#endif
   double r = __fma_rn(-kf, c_kde[1], u);
   double p = __fma_rn(c_kde[2], r, C_P2);
   p = __fma_rn(p, r, C_P1);
   p = __fma_rn(p, r, C_P0);
-  return __fma_rn(p, sS[k], acc);
+  return __fma_rn(p, S, acc);
 }
 
+#if KDE_SPLIT
+#define KDE_SMEM_TABLE (256 * 32 * 8)
+#else
 #define KDE_SMEM_TABLE ((KDE_KCUT + 1) * 8)
-#define KDE_SMEM_BYTES (KDE_SMEM_TABLE + KDE_WARPS * KDE_CH * 8)
+#endif
+// one lane's sum over the item's values: KDE_UNROLL independent accumulators, each an integer
+// in [2^52, 2^53) (a lane adds at most KDE_CH terms of <= 2^40 per item)
+template <int MODE>
+__device__ __forceinline__ u64 kde_item_sum(double gj, const double* sx, u32 i, u32 len, double inv_h,
+                                            const double* sSb, KdeRegs R) {
+  double ac[KDE_UNROLL];
+#pragma unroll
+  for (int q = 0; q < KDE_UNROLL; q++) ac[q] = C_TWO52;
+  for (; i + (KDE_UNROLL - 1) * KDE_V < len; i += KDE_UNROLL * KDE_V) {
+#pragma unroll
+    for (int q = 0; q < KDE_UNROLL; q++) ac[q] = kde_acc<MODE>(gj, sx[i + q * KDE_V], inv_h, sSb, R, ac[q]);
+  }
+#pragma unroll
+  for (int q = 0; q < KDE_UNROLL - 1; q++)
+    if (i + q * KDE_V < len) ac[q] = kde_acc<MODE>(gj, sx[i + q * KDE_V], inv_h, sSb, R, ac[q]);
+  u64 acc = 0;
+#pragma unroll
+  for (int q = 0; q < KDE_UNROLL; q++) acc += (u64)__double_as_longlong(ac[q]) - 0x4330000000000000ull;
+  return acc;
+}
+
+// per warp: two value buffers (double-buffered asynchronous staging) and a ring of three item
+// descriptors (current, next, the one after)
+#define KDE_WARP_BYTES (2 * KDE_CH * 8 + 3 * 48)
+#define KDE_SMEM_BYTES (KDE_SMEM_TABLE + KDE_WARPS * KDE_WARP_BYTES)
 
 // A warp owns KDE_TJ grid points x KDE_V = 32 / KDE_TJ value slices: lane l evaluates grid
 // point j0 + l % KDE_TJ over the values i = l / KDE_TJ + m * KDE_V; slices are summed with
 // shuffles.  (Measured: 32 x 1 beats 8 x 4 -- the narrower value window of 8 x 4 saves ~10%
 // out-of-window terms but quadruples the per-item overhead at equal chunk size.)
+//
+// Items are dealt to warps round-robin (item w, w + W, w + 2W, ...; W warps in the grid; items
+// cost about the same) so every warp knows its future items, and a three-stage cp.async
+// pipeline keeps all global latency off the FP64 pipe: while item k is evaluated, the values of
+// item k + 1 and the descriptor of item k + 2 are in flight.  Densities are accumulated with
+// fire-and-forget reductions of two limbs (low 32 bits, the rest) into D[2j], D[2j + 1];
+// k_kde_fix turns them into the u128 D_j afterwards.
 template <bool GUARD>
 __global__ void __launch_bounds__(32 * KDE_WARPS, KDE_MINB)
-k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ vals, u32 vshift,
-      const u64* __restrict__ tile_range, const u32* __restrict__ tile_items,
-      const u32* __restrict__ item_tile, u32 ntiles, u64* D, unsigned long long* counter,
-      unsigned long long* evaluated) {
-  const u32 items = tile_items[ntiles];  // device-side total of work items
+k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
+      const u64* __restrict__ vals, u32 vshift, u64* D, unsigned long long* evaluated) {
   extern __shared__ __align__(16) unsigned char smem[];
-  double* sS = (double*)smem;                                   // [KDE_KCUT + 1]
-  double* sx = (double*)(smem + KDE_SMEM_TABLE) + (threadIdx.x >> 5) * KDE_CH;  // warp's slice
+  double* sS = (double*)smem;
+#if KDE_SPLIT
+  // replica l of entry e at double index 32 e + l: 2^{-e/256} * 2^40 (exact scaling)
+  for (u32 q = threadIdx.x; q < 256 * 32; q += blockDim.x) {
+    double T = KDE_EXP2_NEG[q >> 5];
+    sS[q] = __hiloint2double(__double2hiint(T) + 40 * (1 << 20), __double2loint(T));
+  }
+#else
   // T'[k] = ldexp(2^{-(k mod 256)/256}, 40 - k div 256), T'[KCUT] = 0
   for (u32 k = threadIdx.x; k <= KDE_KCUT; k += blockDim.x) {
     double T = KDE_EXP2_NEG[k & 255];
@@ -236,74 +339,114 @@ k_kde(const SegDev* __restrict__ segs, u32 G, u32 tps, const u64* __restrict__ v
                           : __hiloint2double(__double2hiint(T) + (40 - (int)(k >> 8)) * (1 << 20),
                                              __double2loint(T));
   }
-  __syncthreads();
+#endif
+  __syncthreads();  // the last block-wide barrier: warps run independently from here
+  const u32 items = *n_items;  // device-side total of work items
   const u32 lane = lane_id();
+  const u32 W = gridDim.x * KDE_WARPS;
+  u32 it = blockIdx.x * KDE_WARPS + (threadIdx.x >> 5);
+  if (it >= items) return;
+  unsigned char* wsm = smem + KDE_SMEM_TABLE + (threadIdx.x >> 5) * KDE_WARP_BYTES;
+  double* const buf0 = (double*)wsm;   // value buffers buf0 + b * KDE_CH, b = 0, 1
+  KdeItem* sd = (KdeItem*)(wsm + 2 * KDE_CH * 8);
+#if KDE_SPLIT
+  const double* sSb = sS + lane;   // this lane's table replica
+#else
+  const double* sSb = sS;
+#endif
+  KdeRegs R;
   // the fma that forms kb has two constant operands and a DFMA takes at most one constant:
   // load both into registers once (opaque to the compiler, so it cannot re-materialise them)
-  KdeRegs R;
   asm volatile("mov.b64 %0, %1;" : "=d"(R.log2e) : "d"(c_kde[0]));
   asm volatile("mov.b64 %0, %1;" : "=d"(R.magic) : "d"(C_MAGIC));
+
+  auto fetch_desc = [&](u32 item, KdeItem* dst) {
+    if (lane < 3) cp_async16((char*)dst + 16 * lane, (const char*)(desc + item) + 16 * lane);
+  };
+  auto fetch_vals = [&](const KdeItem* d, double* dst) {
+    const u64* src = vals + d->va;
+    const u32 len = d->len;
+#pragma unroll
+    for (u32 q = 0; q < KDE_CH / 32; q++) {
+      const u32 i = lane + 32 * q;
+      if (i < len) cp_async8(dst + i, src + i);
+    }
+  };
+  // prologue: descriptor of the first item, then its values and the second item's descriptor
+  fetch_desc(it, sd);
+  cp_async_commit();
+  cp_async_wait_all();
+  __syncwarp();
+  fetch_vals(sd, buf0);
+  if (it + W < items) fetch_desc(it + W, sd + 1);
+  cp_async_commit();
+  u32 cur = 0, b = 0;   // ring slot of the current descriptor, current value buffer
   for (;;) {
-    u32 item = 0;
-    if (lane == 0) item = (u32)atomicAdd(counter, 1ull);
-    item = __shfl_sync(0xffffffffu, item, 0);
-    if (item >= items) break;
-    u32 tile = item_tile[item];
-    u32 s = tile / tps, t = tile % tps;
-    const SegDev& g = segs[s];
-    u64 va = tile_range[2 * (u64)tile] + (u64)(item - tile_items[tile]) * KDE_CH;
-    u64 ve = tile_range[2 * (u64)tile + 1];
-    u32 len = (u32)min((u64)KDE_CH, ve - va);
-    for (u32 i = lane; i < len; i += 32) sx[i] = __ull2double_rn(vals[va + i] >> vshift);
+    cp_async_wait_all();  // values of this item, descriptor of the next (issued one item ago)
+    __syncwarp();
+    const KdeItem* cd = sd + cur;
+    const u32 nxt = cur == 2 ? 0 : cur + 1, nn = nxt == 2 ? 0 : nxt + 1;
+    const u32 it1 = it + W;
+    if (it1 < items) {
+      fetch_vals(sd + nxt, buf0 + (b ^ 1) * KDE_CH);
+      if (it1 + W < items) fetch_desc(it1 + W, sd + nn);
+    }
+    cp_async_commit();
+    double* sx = buf0 + b * KDE_CH;
+    const u32 len = cd->len;
+    // each lane converts the values it copied itself (x = key >> vshift, exactly rounded)
+#pragma unroll
+    for (u32 q = 0; q < KDE_CH / 32; q++) {
+      const u32 i = lane + 32 * q;
+      if (i < len) sx[i] = __ull2double_rn((u64)__double_as_longlong(sx[i]) >> vshift);
+    }
     __syncwarp();
     const u32 slice = lane / KDE_TJ;
-    u32 j = t * KDE_TJ + lane % KDE_TJ;
-    double inv_h = g.inv_h;
-    double gj = grid_pt(g.lo, g.hi, j < G ? j : G - 1, G);
-    u32 i = slice;
-    const double* sSb = sS;
-    // KDE_UNROLL independent accumulators, each an integer in [2^52, 2^53): a lane adds at most
-    // KDE_CH terms of <= 2^40 per item
-    double ac[KDE_UNROLL];
-#pragma unroll
-    for (int q = 0; q < KDE_UNROLL; q++) ac[q] = C_TWO52;
-    for (; i + (KDE_UNROLL - 1) * KDE_V < len; i += KDE_UNROLL * KDE_V) {
-#pragma unroll
-      for (int q = 0; q < KDE_UNROLL; q++) ac[q] = kde_acc<GUARD>(gj, sx[i + q * KDE_V], inv_h, sSb, R, ac[q]);
-    }
-#pragma unroll
-    for (int q = 0; q < KDE_UNROLL - 1; q++)
-      if (i + q * KDE_V < len) ac[q] = kde_acc<GUARD>(gj, sx[i + q * KDE_V], inv_h, sSb, R, ac[q]);
-    u64 acc = 0;
-#pragma unroll
-    for (int q = 0; q < KDE_UNROLL; q++) acc += (u64)__double_as_longlong(ac[q]) - 0x4330000000000000ull;
+    const u32 j = cd->j0 + lane % KDE_TJ;
+    const double inv_h = cd->inv_h;
+    const double gj = grid_pt(cd->lo, cd->hi, j < G ? j : G - 1, G);
+    u64 acc = (!GUARD && cd->fast) ? kde_item_sum<0>(gj, sx, slice, len, inv_h, sSb, R)
+                                   : kde_item_sum<GUARD ? 2 : 1>(gj, sx, slice, len, inv_h, sSb, R);
 #pragma unroll
     for (int o = KDE_TJ; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
-    if (evaluated && lane == 0) {  // evaluated (lane, value) pairs of this item, wasted ones included
-      u32 live = min((u32)KDE_TJ, G - t * KDE_TJ);
-      atomicAdd(evaluated, (unsigned long long)live * len);
-    }
+    // evaluated (lane, value) pairs of this item, wasted ones included
+    if (evaluated && lane == 0) atomicAdd(evaluated, (unsigned long long)cd->live * len);
     if (j < G && slice == 0 && acc) {
-      unsigned long long* d = (unsigned long long*)(D + 2 * ((u64)s * G + j));
-      unsigned long long old = atomicAdd(d, (unsigned long long)acc);
-      if (old + acc < old) atomicAdd(d + 1, 1ull);
+      unsigned long long* d = (unsigned long long*)(D + 2 * ((u64)cd->s * G + j));
+      atomicAdd(d, acc & 0xFFFFFFFFull);                 // < 2^32 items per grid point: exact
+      if (acc >> 32) atomicAdd(d + 1, acc >> 32);
     }
-    __syncwarp();
+    __syncwarp();  // buffer b and descriptor slot cur are refilled from the next iteration on
+    it = it1;
+    if (it >= items) break;
+    cur = nxt;
+    b ^= 1;
   }
 }
 
-size_t kde_item_bytes(u32 items) { return (size_t)items * 4 + 16; }
+// D[2j] (sum of low 32-bit limbs), D[2j + 1] (sum of high parts) -> u128 D_j
+__global__ void k_kde_fix(u64* D, u64 n) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  u64 lo = D[2 * i], hi = D[2 * i + 1];
+  u64 l = lo + (hi << 32);
+  D[2 * i] = l;
+  D[2 * i + 1] = (hi >> 32) + (l < lo);
+}
+
+size_t kde_item_bytes(u32 items) { return (size_t)items * sizeof(KdeItem) + 16; }
 
 void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const u64* tile_range,
-                const u32* tile_items, u32* item_tile, u32 items, u64* D,
-                unsigned long long* work_counter, unsigned long long* evaluated, bool guard,
-                cudaStream_t s) {
+                const u32* tile_items, void* item_desc, u32 items, u64* D,
+                unsigned long long* evaluated, bool guard, cudaStream_t s) {
   if (items == 0) return;
   u32 tps = div_up(G, KDE_TJ);
   u32 ntiles = nseg * tps;
   // `items` is a host-side upper bound: grids are sized by it, the kernels stop at the
   // device-side count tile_items[ntiles]
-  SV_LAUNCH(k_kde_items, min(div_up(items, 256), 4096u), 256, 0, s)(tile_items, ntiles, item_tile);
+  KdeItem* desc = (KdeItem*)item_desc;
+  SV_LAUNCH(k_kde_items, min(div_up(items, 256), 4096u), 256, 0, s)(segs, G, tps, tile_range, tile_items,
+                                                                     ntiles, desc);
   auto kern = guard ? k_kde<true> : k_kde<false>;
   cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, KDE_SMEM_BYTES);
   int per_sm = 0;
@@ -312,8 +455,8 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift
   u32 grid = (u32)sv_num_sms() * (u32)per_sm;
   u32 need = div_up(items, KDE_WARPS);
   if (grid > need) grid = need;
-  cudaMemsetAsync(work_counter, 0, 8, s);
-  SV_LAUNCH(kern, grid, 32 * KDE_WARPS, KDE_SMEM_BYTES, s)(segs, G, tps, vals, vshift, tile_range, tile_items,
-                                                           item_tile, ntiles, D, work_counter,
+  SV_LAUNCH(kern, grid, 32 * KDE_WARPS, KDE_SMEM_BYTES, s)(desc, tile_items + ntiles, G, vals, vshift, D,
                                                            evaluated);
+  u64 nd = (u64)nseg * G;
+  SV_LAUNCH(k_kde_fix, div_up(nd, 256), 256, 0, s)(D, nd);
 }

@@ -68,9 +68,8 @@ void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32
               u64* tile_range, u32* tile_items, void* scan_temp, cudaStream_t s);
 size_t kde_item_bytes(u32 items);
 void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const u64* tile_range,
-                const u32* tile_items, u32* item_tile, u32 items,
-                u64* D /* [nseg][G][2] */, unsigned long long* work_counter,
-                unsigned long long* evaluated, bool guard, cudaStream_t s);
+                const u32* tile_items, void* item_desc /* kde_item_bytes(items) */, u32 items,
+                u64* D /* [nseg][G][2] */, unsigned long long* evaluated, bool guard, cudaStream_t s);
 
 // ---------------- segmented sort by (open segment, grid cell) (a2) ----------------------------
 // rounds > 1 read each re-opened part's range of the previous round's sorted keys in chunks of
