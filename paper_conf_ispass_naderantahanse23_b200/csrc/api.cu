@@ -554,7 +554,7 @@ static int d2h_raw(sieve_ctx c, void* dst, const void* d, size_t bytes) {
   if (!bytes) return SIEVE_OK;
   void* p;
   SV_TRY(pin_alloc(c, &p, bytes));
-  SV_CUDA(cudaMemcpyAsync(p, d, bytes, cudaMemcpyDeviceToHost, c->stream));
+  launch_copy(p, d, bytes, c->stream);  // SM copy into the UVA-mapped staging (no copy engine)
   c->pend.push_back({dst, p, bytes});
   return SIEVE_OK;
 }
@@ -569,7 +569,7 @@ static int h2d(sieve_ctx c, T* d, const std::vector<T>& h) {
   void* p;
   SV_TRY(pin_alloc(c, &p, h.size() * sizeof(T)));
   memcpy(p, h.data(), h.size() * sizeof(T));
-  SV_CUDA(cudaMemcpyAsync(d, p, h.size() * sizeof(T), cudaMemcpyHostToDevice, c->stream));
+  launch_copy(d, p, h.size() * sizeof(T), c->stream);  // SM copy from the UVA-mapped staging
   return SIEVE_OK;
 }
 static bool host_timing() {
@@ -683,14 +683,14 @@ static int moments_pass(sieve_trace t, MomentsHost* M) {
     SV_TRY(mx.alloc(K + 4));
     SV_CUDA(cudaMemcpy2DAsync(mn.get(), 8, mm.get(), 16, 8, K, cudaMemcpyDeviceToDevice, S));
     SV_CUDA(cudaMemcpy2DAsync(mx.get(), 8, mm.get() + 1, 16, 8, K, cudaMemcpyDeviceToDevice, S));
-    SV_CUDA(cudaMemcpyAsync(mx.get() + K, tot.get() + 4, 4 * 8, cudaMemcpyDeviceToDevice, S));
+    launch_copy(mx.get() + K, tot.get() + 4, 4 * 8, S);
     SV_TRY(allreduce(c, lanes.get(), (size_t)K * MOM_LANES, RED_SUM));
     SV_TRY(allreduce(c, tot.get(), 4, RED_SUM));
     SV_TRY(allreduce(c, mn.get(), K, RED_MIN));
     SV_TRY(allreduce(c, mx.get(), K + 4, RED_MAX));
     SV_CUDA(cudaMemcpy2DAsync(mm.get(), 16, mn.get(), 8, 8, K, cudaMemcpyDeviceToDevice, S));
     SV_CUDA(cudaMemcpy2DAsync(mm.get() + 1, 16, mx.get(), 8, 8, K, cudaMemcpyDeviceToDevice, S));
-    SV_CUDA(cudaMemcpyAsync(tot.get() + 4, mx.get() + K, 4 * 8, cudaMemcpyDeviceToDevice, S));
+    launch_copy(tot.get() + 4, mx.get() + K, 4 * 8, S);
     SV_TRY(d2h(c, h_lanes, lanes.get(), (size_t)K * MOM_LANES));
     SV_TRY(d2h(c, h_mm, mm.get(), (size_t)K * 2));
     SV_TRY(d2h(c, h_tot, tot.get(), 8));
@@ -1116,7 +1116,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(sk.alloc(std::max<u64>(Etot, 1))); SV_TRY(scnt.alloc(std::max<u64>(Etot, 1)));
     SV_TRY(sfirst.alloc(std::max<u64>(Etot, 1)));
     launch_iota_u32(idx.get(), Etot, S);
-    SV_CUDA(cudaMemcpyAsync(sk.get(), ak, Etot * 8, cudaMemcpyDeviceToDevice, S));
+    launch_copy(sk.get(), ak, Etot * 8, S);
     PhaseTimer tr(c, SIEVE_PHASE_REPS, 0);
     {
       DBuf<char> tmp(c);

@@ -13,6 +13,9 @@
 // The global table's contents (not its slot order) are deterministic; entries are compacted,
 // gathered across ranks, radix-sorted by key and reduced, so the result is identical for any
 // number of ranks or blocks.
+#include <algorithm>
+#include <cstdint>
+
 #include "kernels.cuh"
 
 #define AS_THREADS 1024
@@ -247,6 +250,28 @@ void launch_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, co
 }
 
 // ------------------------------------------------------------------------------------------
+// Copies issued by the SMs instead of the copy engines: the path's small host<->device tables
+// (through the pinned staging arena, which UVA maps into the device's address space) and its
+// device-to-device moves.  A concurrent bulk H2D on another stream (sieve_load_trace of the next
+// trace) occupies the copy engines for tens of milliseconds; copy-engine work queued behind it
+// would stall every synchronisation of this call.
+__global__ void k_copy_words(u32* __restrict__ dst, const u32* __restrict__ src, u64 n) {
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) dst[i] = src[i];
+}
+__global__ void k_copy_bytes(unsigned char* __restrict__ dst, const unsigned char* __restrict__ src, u64 n) {
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) dst[i] = src[i];
+}
+void launch_copy(void* dst, const void* src, u64 bytes, cudaStream_t s) {
+  if (!bytes) return;
+  if ((((uintptr_t)dst | (uintptr_t)src | bytes) & 3) == 0) {
+    u64 n = bytes / 4;
+    SV_LAUNCH(k_copy_words, (unsigned)std::min<u64>(div_up(n, 256), 2048), 256, 0, s)((u32*)dst, (const u32*)src, n);
+  } else {
+    SV_LAUNCH(k_copy_bytes, (unsigned)std::min<u64>(div_up(bytes, 256), 2048), 256, 0, s)(
+        (unsigned char*)dst, (const unsigned char*)src, bytes);
+  }
+}
+
 __global__ void k_fill_u64(u64* p, u64 n, u64 v) {
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) p[i] = v;
 }

@@ -197,6 +197,8 @@ void launch_dp_gather(const u32* kstart, const u32* count, const u64* off, const
 
 // ---------------- misc -------------------------------------------------------------------------
 void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s);
+// SM-driven copy (device or pinned host memory on either side; no copy engine)
+void launch_copy(void* dst, const void* src, u64 bytes, cudaStream_t s);
 // cross-rank encoding of u128 pairs [n][2] <-> 4 limbs [n][4]
 void launch_u128_to_limbs(const u64* src, u64 n, u64* limbs, cudaStream_t s);
 void launch_limbs_to_u128(const u64* limbs, u64 n, u64* dst, cudaStream_t s);

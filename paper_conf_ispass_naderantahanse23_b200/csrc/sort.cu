@@ -401,8 +401,8 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
     if (passes) (*passes)++;
   }
   if (kin != keys) {
-    SV_CUDA(cudaMemcpyAsync(keys, kin, n * 8, cudaMemcpyDeviceToDevice, s));
-    if (vals) SV_CUDA(cudaMemcpyAsync(vals, vin, n * 4, cudaMemcpyDeviceToDevice, s));
+    launch_copy(keys, kin, n * 8, s);
+    if (vals) launch_copy(vals, vin, n * 4, s);
   }
   SV_CUDA(cudaGetLastError());
   return SIEVE_OK;
