@@ -30,7 +30,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-KDE_FP64_OPS_PER_TERM = 10   # FP64-pipe instructions per in-window KDE term
+KDE_FP64_OPS_PER_TERM = 9    # FP64-pipe instructions per in-window KDE term
 FP64_LANES_PER_SM = 64       # B200: 64 FP64 FMA lanes / SM / clk (microbenchmark: 62.9)
 
 

@@ -66,8 +66,12 @@ def q_of_t(t):
     return round(v)                      # Fraction round(): nearest, ties to even
 
 
-def q_term(g, x, inv_h):
-    z = (g - float(x)) * inv_h
+def q_term(g, x, inv_h, lo):
+    """A10: z = rn(rn(g - lo) / h') - rn(rn(x - lo) / h') with 1/h' = inv_h (Python floats are
+    IEEE doubles; x - lo is an exact integer below 2^44, so float() of it is exact)"""
+    gs = (g - float(lo)) * inv_h
+    xs = float(x - lo) * inv_h
+    z = gs - xs
     t = (z * z) * 0.5
     return q_of_t(t)
 
@@ -97,7 +101,7 @@ def grid(lo, hi, G):
 
 def kde(vals, lo, hi, h, G):
     inv_h = 1.0 / h
-    return [sum(q_term(g, x, inv_h) for x in vals) for g in grid(lo, hi, G)]
+    return [sum(q_term(g, x, inv_h, lo) for x in vals) for g in grid(lo, hi, G)]
 
 
 def valley_cuts(D, shift):

@@ -309,9 +309,13 @@ uint64_t oracle_q(double t) {
 
 double oracle_exp2_table(int j) { return OR_EXP2_NEG[j & 255]; }
 
-/* fixed-point kernel value Q(x, g), t = (z * z) * 0.5, z = (g - rn(x)) * inv_h */
-static uint64_t kernel_q(double g, double xd, double inv_h) {
-  double z = (g - xd) * inv_h;
+/* fixed-point kernel value Q(x, g) (A10): both points are measured from the segment's lo in
+ * units of h, gs = rn(rn(g - rn(lo)) * inv_h) and xs = rn(rn(x - lo) * inv_h) (x - lo is an exact
+ * integer), z = gs - xs, t = (z * z) * 0.5 */
+static double scaled_value(uint64_t x, uint64_t lo, double inv_h) { return (double)(x - lo) * inv_h; }
+static double scaled_grid(double g, uint64_t lo, double inv_h) { return (g - (double)lo) * inv_h; }
+static uint64_t kernel_q(double gs, double xs) {
+  double z = gs - xs;
   double t = (z * z) * 0.5;
   return oracle_q(t);
 }
@@ -321,9 +325,9 @@ static void kde_grid(const uint64_t* v, uint64_t m, uint64_t lo, uint64_t hi, do
                      uint32_t G, u128* D) {
   double inv_h = 1.0 / h;
   for (uint32_t j = 0; j < G; j++) {
-    double g = grid_point(lo, hi, j, G);
+    double gs = scaled_grid(grid_point(lo, hi, j, G), lo, inv_h);
     u128 acc = 0;
-    for (uint64_t i = 0; i < m; i++) acc += kernel_q(g, (double)v[i], inv_h);
+    for (uint64_t i = 0; i < m; i++) acc += kernel_q(gs, scaled_value(v[i], lo, inv_h));
     D[j] = acc;
   }
 }

@@ -2,7 +2,7 @@
 // ("Kernel Density Estimation [8], [36]"; readings A6-A10 in DESIGN.md section 3):
 //
 //   g_j  = rn(lo) + rn((hi - lo) * j) / rn(G - 1)                      (A9)
-//   z    = (g_j - rn(x)) * inv_h ;  t = (z * z) * 0.5
+//   z    = rn(rn(g_j - rn(lo)) * inv_h) - rn(rn(x - lo) * inv_h) ;  t = (z * z) * 0.5
 //   Q    = 0 if k > 10526, else rint(P(r) * 2^{-j'/256} * 2^(40 - m))   (A10; k = rint(t 256
 //          log2 e), j' = k mod 256, m = k div 256, r = t - k rn(ln2/256), P = degree-3 Taylor
 //          of e^{-r})
@@ -13,21 +13,21 @@
 // independent of summation order, of the work decomposition and of the number of ranks.
 //
 // B200 mapping (the paper's scripts have no GPU design; this is new).  The KDE is a windowed
-// gather over the values of each segment grouped by grid cell (bucket.cu), bound by the FP64 pipe (no contraction, so no
-// tensor cores).  Work item = (segment, tile of 32 grid points, chunk of <= 256 values inside
-// the tile's window |g - x| <= 7.6 h); items are pulled by WARPS from an atomic counter (no
-// block barriers: warps of a block never wait for each other); each lane owns one grid point,
-// the chunk is staged in the warp's slice of shared memory and read as broadcasts.  The term is
-// arranged to be bit-identical to the oracle's while issuing 10 FP64-pipe instructions and ~5
-// others:
+// gather over the values of each segment grouped by grid cell (bucket.cu), bound by the FP64
+// pipe (no contraction, so no tensor cores).  Work item = (segment, tile of 32 grid points,
+// chunk of <= 256 values inside the tile's window |g - x| <= 7.6 h); items are dealt to warps
+// round-robin and staged by a per-warp cp.async pipeline (see k_kde); each lane owns one grid
+// point and reads the staged values as shared-memory broadcasts.  The term is arranged to be
+// bit-identical to the oracle's while issuing 9 FP64-pipe instructions and ~6 others:
+//   * xs (per value, at staging) and gs (per lane, per item) are the A10 scaled coordinates,
+//     so z = gs - xs is one subtraction;
 //   * u = z*z replaces t = u/2 (exact scaling): k = nearest integer to u * 128 log2 e (= t * 256
 //     log2 e, one rounding, via fma(u, 128 log2 e, 1.5 * 2^52)), r' = u - k rn(ln2)/128 = 2r,
 //     Horner on r' with coefficients c_i 2^-i gives exactly the same P (power-of-two scaling
 //     commutes with round-to-nearest);
-//   * k = low word of that fma result, clamped to 10527;
-//   * S = T'[k] = 2^{-(k mod 256)/256} * 2^(40 - k div 256) from a shared-memory table (exact
-//     power-of-two scalings of the correctly rounded 2^{-j/256}), with T'[10527] = 0, so the
-//     cutoff k > 10526 needs no select;
+//   * k = low word of that fma result;
+//   * S = 2^{-(k mod 256)/256} * 2^(40 - k div 256): a lane-replicated 256-entry table and an
+//     exponent-field subtraction (kde_acc); terms with k > 10526 contribute exactly 0;
 //   * rint(P * S) = bits(fma(P, S, 2^52)) - bits(2^52): the sum lies in [2^52, 2^53) where the
 //     ulp is 1; raw bit patterns are accumulated and 2^52's pattern is subtracted once per term
 //     count at the end.
@@ -238,9 +238,9 @@ struct KdeRegs { double log2e, magic; };  // operands that must sit in registers
 // itself; with m = k div 256 <= 255 the scaled entry stays normal); MODE 1: k clamped to
 // KDE_KCLAMP; MODE 2: clamp plus the explicit large-u guard (see below).
 template <int MODE>
-__device__ __forceinline__ double kde_acc(double g, double xd, double inv_h, const double* sS,
-                                          KdeRegs R, double acc) {
-  double z = __dmul_rn(__dsub_rn(g, xd), inv_h);
+__device__ __forceinline__ double kde_acc(double gs, double xs, const double* sS, KdeRegs R,
+                                          double acc) {
+  double z = __dsub_rn(gs, xs);                             // A10: both scaled from lo by 1/h
   double u = __dmul_rn(z, z);                               // 2t, exactly
   double kb = __fma_rn(u, R.log2e, R.magic);                // one rounding: nearest integer
   double kf = __dsub_rn(kb, C_MAGIC);
@@ -285,18 +285,18 @@ __device__ __forceinline__ double kde_acc(double g, double xd, double inv_h, con
 // one lane's sum over the item's values: KDE_UNROLL independent accumulators, each an integer
 // in [2^52, 2^53) (a lane adds at most KDE_CH terms of <= 2^40 per item)
 template <int MODE>
-__device__ __forceinline__ u64 kde_item_sum(double gj, const double* sx, u32 i, u32 len, double inv_h,
+__device__ __forceinline__ u64 kde_item_sum(double gs, const double* sx, u32 i, u32 len,
                                             const double* sSb, KdeRegs R) {
   double ac[KDE_UNROLL];
 #pragma unroll
   for (int q = 0; q < KDE_UNROLL; q++) ac[q] = C_TWO52;
   for (; i + (KDE_UNROLL - 1) * KDE_V < len; i += KDE_UNROLL * KDE_V) {
 #pragma unroll
-    for (int q = 0; q < KDE_UNROLL; q++) ac[q] = kde_acc<MODE>(gj, sx[i + q * KDE_V], inv_h, sSb, R, ac[q]);
+    for (int q = 0; q < KDE_UNROLL; q++) ac[q] = kde_acc<MODE>(gs, sx[i + q * KDE_V], sSb, R, ac[q]);
   }
 #pragma unroll
   for (int q = 0; q < KDE_UNROLL - 1; q++)
-    if (i + q * KDE_V < len) ac[q] = kde_acc<MODE>(gj, sx[i + q * KDE_V], inv_h, sSb, R, ac[q]);
+    if (i + q * KDE_V < len) ac[q] = kde_acc<MODE>(gs, sx[i + q * KDE_V], sSb, R, ac[q]);
   u64 acc = 0;
 #pragma unroll
   for (int q = 0; q < KDE_UNROLL; q++) acc += (u64)__double_as_longlong(ac[q]) - 0x4330000000000000ull;
@@ -394,19 +394,23 @@ k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
     cp_async_commit();
     double* sx = buf0 + b * KDE_CH;
     const u32 len = cd->len;
-    // each lane converts the values it copied itself (x = key >> vshift, exactly rounded)
+    // each lane converts the values it copied itself: x = key >> vshift (lo <= x <= hi), then
+    // xs = rn(rn(x - lo) * inv_h) (A10; x - lo is an exact integer below 2^44)
+    const u64 lo = cd->lo;
+    const double inv_h = cd->inv_h;
 #pragma unroll
     for (u32 q = 0; q < KDE_CH / 32; q++) {
       const u32 i = lane + 32 * q;
-      if (i < len) sx[i] = __ull2double_rn((u64)__double_as_longlong(sx[i]) >> vshift);
+      if (i < len)
+        sx[i] = __dmul_rn(__ull2double_rn(((u64)__double_as_longlong(sx[i]) >> vshift) - lo), inv_h);
     }
     __syncwarp();
     const u32 slice = lane / KDE_TJ;
     const u32 j = cd->j0 + lane % KDE_TJ;
-    const double inv_h = cd->inv_h;
-    const double gj = grid_pt(cd->lo, cd->hi, j < G ? j : G - 1, G);
-    u64 acc = (!GUARD && cd->fast) ? kde_item_sum<0>(gj, sx, slice, len, inv_h, sSb, R)
-                                   : kde_item_sum<GUARD ? 2 : 1>(gj, sx, slice, len, inv_h, sSb, R);
+    // gs = rn(rn(g_j - rn(lo)) * inv_h) (A10)
+    const double gs = __dmul_rn(__dsub_rn(grid_pt(lo, cd->hi, j < G ? j : G - 1, G), __ull2double_rn(lo)), inv_h);
+    u64 acc = (!GUARD && cd->fast) ? kde_item_sum<0>(gs, sx, slice, len, sSb, R)
+                                   : kde_item_sum<GUARD ? 2 : 1>(gs, sx, slice, len, sSb, R);
 #pragma unroll
     for (int o = KDE_TJ; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
     // evaluated (lane, value) pairs of this item, wasted ones included

@@ -189,14 +189,19 @@ void launch_moments(const u32* kid, const u64* x, const u64* y, u64 n, u32 K, u3
   SV_LAUNCH(k_moments, grid, MOM_THREADS, moments_smem(kt), s)(kid, x, y, n, K, k0, kt, part, blk_tot, errflags);
 }
 
-// one thread per kernel: exact u128 sum over the blocks' partials, emitted as limb lanes
+// one warp per kernel: the lanes stride over the blocks' partials, exact u128 sums reduced by
+// shuffles, emitted as limb lanes
+__device__ __forceinline__ u128 shfl_xor_u128(u128 v, int o) {
+  u64 lo = __shfl_xor_sync(0xffffffffu, (u64)v, o), hi = __shfl_xor_sync(0xffffffffu, (u64)(v >> 64), o);
+  return ((u128)hi << 64) | lo;
+}
 __global__ void k_moments_reduce(const KMomPartial* __restrict__ part, int grid, u32 k0, u32 kt,
                                  u64* lanes, u64* mm, u64* local_n) {
-  u32 l = blockIdx.x * blockDim.x + threadIdx.x;
-  if (l >= kt) return;
+  u32 l = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (l >= kt) return;  // warp-uniform
   u128 n = 0, s1 = 0, s2 = 0;
   u64 mn = ~0ull, mx = 0;
-  for (int b = 0; b < grid; b++) {
+  for (int b = lane_id(); b < grid; b += 32) {
     KMomPartial r = part[(u64)b * kt + l];
     n += r.n;
     s1 += ((u128)r.s1hi << 64) | r.s1lo;
@@ -204,6 +209,16 @@ __global__ void k_moments_reduce(const KMomPartial* __restrict__ part, int grid,
     mn = r.mn < mn ? r.mn : mn;
     mx = r.mx > mx ? r.mx : mx;
   }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    n += shfl_xor_u128(n, o);
+    s1 += shfl_xor_u128(s1, o);
+    s2 += shfl_xor_u128(s2, o);
+    u64 omn = __shfl_xor_sync(0xffffffffu, mn, o), omx = __shfl_xor_sync(0xffffffffu, mx, o);
+    mn = omn < mn ? omn : mn;
+    mx = omx > mx ? omx : mx;
+  }
+  if (lane_id() != 0) return;
   u32 k = k0 + l;
   u64* L = lanes + (u64)k * MOM_LANES;
   L[0] = (u64)n;
@@ -215,13 +230,20 @@ __global__ void k_moments_reduce(const KMomPartial* __restrict__ part, int grid,
 }
 
 __global__ void k_totals_reduce(const u64* blk_tot, int grid, u64* tot_lanes, u64* tot_max) {
-  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  if (blockIdx.x != 0 || threadIdx.x >= 32) return;
   u128 c = 0;
   u64 mx = 0;
-  for (int b = 0; b < grid; b++) {
+  for (int b = lane_id(); b < grid; b += 32) {
     c += ((u128)blk_tot[3 * b + 1] << 64) | blk_tot[3 * b];
     mx = blk_tot[3 * b + 2] > mx ? blk_tot[3 * b + 2] : mx;
   }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    c += shfl_xor_u128(c, o);
+    u64 omx = __shfl_xor_sync(0xffffffffu, mx, o);
+    mx = omx > mx ? omx : mx;
+  }
+  if (lane_id() != 0) return;
   limbs_from_u128((u64)c, (u64)(c >> 64), tot_lanes);
   tot_max[0] = mx;
 }
@@ -230,6 +252,6 @@ void launch_moments_reduce(const KMomPartial* part, const u64* blk_tot, int grid
                            u32 K, u64* lanes, u64* mm, u64* local_n, u64* tot_lanes, u64* tot_max,
                            bool do_totals, cudaStream_t s) {
   (void)K;
-  SV_LAUNCH(k_moments_reduce, div_up(kt, 256), 256, 0, s)(part, grid, k0, kt, lanes, mm, local_n);
+  SV_LAUNCH(k_moments_reduce, div_up((u64)kt * 32, 256), 256, 0, s)(part, grid, k0, kt, lanes, mm, local_n);
   if (do_totals) SV_LAUNCH(k_totals_reduce, 1, 32, 0, s)(blk_tot, grid, tot_lanes, tot_max);
 }
