@@ -19,8 +19,11 @@
 #include "kernels.cuh"
 
 #define AS_THREADS 1024
+#ifndef AS_PIPE
+#define AS_PIPE 1           // the next tile's rows are loaded while this tile is processed
+#endif                      // (A/B on C4: 0.96 -> 0.73 ms against 8 rows per thread unpipelined)
 #ifndef AS_IPT
-#define AS_IPT 8
+#define AS_IPT (AS_PIPE ? 4 : 8)
 #endif
 #define AS_HC 8192          // shared hash capacity (entries): 128 KB, one block per SM
 #define AS_FLUSH (3 * AS_HC / 4)      // flush to the L2 table when this full
@@ -82,18 +85,29 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
   u64 b0 = (u64)blockIdx.x * chunk;
   u64 b1 = b0 + chunk < n ? b0 + chunk : n;
   const u64 tile = (u64)AS_THREADS * AS_IPT;
-  for (u64 base = b0; base < b1; base += tile) {
-    // issue the tile's loads first (AS_IPT rows per thread in flight), then the atomics
-    u32 kk[AS_IPT], cc[AS_IPT];
-    u64 vv[AS_IPT];
+  u32 kk[AS_IPT], cc[AS_IPT];
+  u64 vv[AS_IPT];
+  auto load_tile = [&](u64 base, u32* k_, u64* v_, u32* c_) {
 #pragma unroll
     for (int j = 0; j < AS_IPT; j++) {
       u64 i = base + (u64)j * AS_THREADS + threadIdx.x;
       bool ok = i < b1;
-      kk[j] = ok ? __ldcs(kid + i) : 0u;
-      vv[j] = ok ? __ldcs(x + i) : 0ull;
-      cc[j] = (ok && cta) ? __ldcs(cta + i) : 0u;
+      k_[j] = ok ? __ldcs(kid + i) : 0u;
+      v_[j] = ok ? __ldcs(x + i) : 0ull;
+      c_[j] = (ok && cta) ? __ldcs(cta + i) : 0u;
     }
+  };
+#if AS_PIPE
+  load_tile(b0, kk, vv, cc);
+#endif
+  for (u64 base = b0; base < b1; base += tile) {
+#if AS_PIPE
+    u32 nk[AS_IPT], nc[AS_IPT];
+    u64 nv[AS_IPT];
+    load_tile(base + tile, nk, nv, nc);   // in flight while this tile is processed
+#else
+    load_tile(base, kk, vv, cc);          // the tile's loads first, then the atomics
+#endif
     KTab kts[AS_IPT];  // per-kernel table rows (L1-resident), all requested before use
 #pragma unroll
     for (int j = 0; j < AS_IPT; j++) kts[j] = ktab[kk[j]];
@@ -149,6 +163,10 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
       if (threadIdx.x == 0) s_fill = 0;
       __syncthreads();
     }
+#if AS_PIPE
+#pragma unroll
+    for (int j = 0; j < AS_IPT; j++) { kk[j] = nk[j]; vv[j] = nv[j]; cc[j] = nc[j]; }
+#endif
   }
 }
 

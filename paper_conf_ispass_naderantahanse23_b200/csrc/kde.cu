@@ -31,18 +31,20 @@
 //   * rint(P * S) = bits(fma(P, S, 2^52)) - bits(2^52): the sum lies in [2^52, 2^53) where the
 //     ulp is 1; raw bit patterns are accumulated and 2^52's pattern is subtracted once per term
 //     count at the end.
+#include <cstdlib>
+
 #include "kernels.cuh"
 
 #define KDE_W 7.6            // window half-width in units of h: k > 10526 (t > 28.5014) beyond it
 #define KDE_KCUT 10527       // k > 10526 = rint(28.5 * 256 log2 e) -> index 10527 holds 0
 #ifndef KDE_WARPS
-#define KDE_WARPS 24         // warps per block (independent work-item consumers)
+#define KDE_WARPS 16         // warps per block (A/B on C4: 16 x 16 terms in flight beat 24 x 8, 28 x 6, 12 x 24)
 #endif
 #ifndef KDE_MINB
-#define KDE_MINB 1           // resident blocks per SM: one 64 KB table shared by 24 warps
+#define KDE_MINB 1           // resident blocks per SM: one 64 KB table shared by the block
 #endif
 #ifndef KDE_UNROLL
-#define KDE_UNROLL 8         // terms in flight per lane
+#define KDE_UNROLL 16        // terms in flight per lane
 #endif
 #define KDE_V (32 / KDE_TJ)  // value slices per warp
 
@@ -322,7 +324,8 @@ __device__ __forceinline__ u64 kde_item_sum(double gs, const double* sx, u32 i, 
 template <bool GUARD>
 __global__ void __launch_bounds__(32 * KDE_WARPS, KDE_MINB)
 k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
-      const u64* __restrict__ vals, u32 vshift, u64* D, unsigned long long* evaluated) {
+      const u64* __restrict__ vals, u32 vshift, u64* D, unsigned long long* evaluated,
+      bool allow_fast) {
   extern __shared__ __align__(16) unsigned char smem[];
   double* sS = (double*)smem;
 #if KDE_SPLIT
@@ -409,7 +412,7 @@ k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
     const u32 j = cd->j0 + lane % KDE_TJ;
     // gs = rn(rn(g_j - rn(lo)) * inv_h) (A10)
     const double gs = __dmul_rn(__dsub_rn(grid_pt(lo, cd->hi, j < G ? j : G - 1, G), __ull2double_rn(lo)), inv_h);
-    u64 acc = (!GUARD && cd->fast) ? kde_item_sum<0>(gs, sx, slice, len, sSb, R)
+    u64 acc = (!GUARD && allow_fast && cd->fast) ? kde_item_sum<0>(gs, sx, slice, len, sSb, R)
                                    : kde_item_sum<GUARD ? 2 : 1>(gs, sx, slice, len, sSb, R);
 #pragma unroll
     for (int o = KDE_TJ; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
@@ -451,6 +454,11 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift
   KdeItem* desc = (KdeItem*)item_desc;
   SV_LAUNCH(k_kde_items, min(div_up(items, 256), 4096u), 256, 0, s)(segs, G, tps, tile_range, tile_items,
                                                                      ntiles, desc);
+  // test hook SIEVE_KDE_FORCE: 1 = never the unclamped fast path, 2 = always the guarded
+  // variant (all three evaluate identical terms; the parity tests run each)
+  const char* force = getenv("SIEVE_KDE_FORCE");
+  const int fm = force ? atoi(force) : 0;
+  if (fm >= 2) guard = true;
   auto kern = guard ? k_kde<true> : k_kde<false>;
   cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, KDE_SMEM_BYTES);
   int per_sm = 0;
@@ -460,7 +468,7 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift
   u32 need = div_up(items, KDE_WARPS);
   if (grid > need) grid = need;
   SV_LAUNCH(kern, grid, 32 * KDE_WARPS, KDE_SMEM_BYTES, s)(desc, tile_items + ntiles, G, vals, vshift, D,
-                                                           evaluated);
+                                                           evaluated, fm == 0);
   u64 nd = (u64)nseg * G;
   SV_LAUNCH(k_kde_fix, div_up(nd, 256), 256, 0, s)(D, nd);
 }

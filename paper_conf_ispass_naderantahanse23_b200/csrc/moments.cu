@@ -16,9 +16,12 @@
 #include "kernels.cuh"
 
 #define MOM_THREADS 1024
-#ifndef MOM_U
-#define MOM_U 2                               // rows per thread with loads in flight (A/B: 2 >= 4, 8 > 16)
+#ifndef MOM_PIPE
+#define MOM_PIPE 1                            // next rows loaded while these are processed
 #endif
+#ifndef MOM_U
+#define MOM_U 1                               // rows per thread per step (A/B pipelined: 1 < 2 < 4;
+#endif                                        // unpipelined 2 was 10% slower than pipelined 1)
 #define MOM_KT 2048                           // kernels per shared-memory pass (56 B each)
 #define MOM_LB 15                             // limb bits
 #define MOM_LMASK ((1u << MOM_LB) - 1u)
@@ -132,6 +135,30 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
   for (u64 c0 = b; c0 < e; c0 += MOM_FLUSH) {
     u64 c1 = c0 + MOM_FLUSH < e ? c0 + MOM_FLUSH : e;
     u64 i = c0 + threadIdx.x;
+#if MOM_PIPE
+    // the next MOM_U rows are loaded while these are processed
+    u32 kk[MOM_U];
+    u64 vv[MOM_U], ww[MOM_U];
+    auto load = [&](u64 at, u32* k_, u64* v_, u64* w_) {
+#pragma unroll
+      for (int u = 0; u < MOM_U; u++) {
+        const bool ok = at + u * step < c1;
+        k_[u] = ok ? __ldcs(kid + at + u * step) : 0u;
+        v_[u] = ok ? __ldcs(x + at + u * step) : 0ull;
+        w_[u] = ok && use_y ? __ldcs(y + at + u * step) : 0ull;
+      }
+    };
+    if (i + (MOM_U - 1) * step < c1) load(i, kk, vv, ww);
+    for (; i + (MOM_U - 1) * step < c1; i += MOM_U * step) {
+      u32 nk[MOM_U];
+      u64 nv[MOM_U], nw[MOM_U];
+      load(i + MOM_U * step, nk, nv, nw);   // rows past c1 load as 0 and are never processed
+#pragma unroll
+      for (int u = 0; u < MOM_U; u++) process(kk[u], vv[u], ww[u]);
+#pragma unroll
+      for (int u = 0; u < MOM_U; u++) { kk[u] = nk[u]; vv[u] = nv[u]; ww[u] = nw[u]; }
+    }
+#else
     for (; i + (MOM_U - 1) * step < c1; i += MOM_U * step) {
       u32 kk[MOM_U];
       u64 vv[MOM_U], ww[MOM_U];
@@ -144,6 +171,7 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
 #pragma unroll
       for (int u = 0; u < MOM_U; u++) process(kk[u], vv[u], ww[u]);
     }
+#endif
     for (; i < c1; i += step) process(__ldcs(kid + i), __ldcs(x + i), use_y ? __ldcs(y + i) : 0ull);
     flush();
   }

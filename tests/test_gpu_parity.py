@@ -219,3 +219,18 @@ def test_segment_batches_change_nothing(monkeypatch):
     assert_tables_equal(g["table"], o.strata)
     assert np.array_equal(g["sid"], o.sid)
     assert_segments_equal(g["segments"], o.segments())
+
+
+@pytest.mark.parametrize("mode", ["1", "2"])
+def test_kde_evaluation_modes_identical(monkeypatch, mode):
+    """The KDE evaluates a term three ways (kde.cu kde_acc MODE 0: no k clamp on items proven
+    |z| < 18.8; 1: clamped; 2: clamped plus the large-u guard).  The test hook forces the
+    slower modes on a whole C2-shaped trace; every density, cut and stratum must still equal the
+    oracle's (MODE 0 is what the other parity tests exercise)."""
+    tr = gen.make_trace("C2", n=200_000)
+    monkeypatch.setenv("SIEVE_KDE_FORCE", mode)
+    g = run_gpu(tr, keep_debug=True)
+    o = run_oracle(tr, keep_debug=True)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+    assert_segments_equal(g["segments"], o.segments())
