@@ -325,6 +325,8 @@ def main():
         e2e = {"value": cfg.n * e_steps / (ems / 1000.0), "unit": "invocations/s",
                "h2d_bytes_per_step": int(n_local * 24),
                "d2h_bytes_per_step": int(out["strata"] * 96 + 56), "steps": e_steps,
+               # the step is bound by the PCIe H2D of the columns: the rate it implies
+               "h2d_GBps_per_rank": n_local * 24 * e_steps / (ems / 1000.0) / 1e9,
                "note": "every step: H2D of kid/x/cta/y from pinned host memory (sieve_load_trace) + "
                        "stratify + predict, stratum table and prediction read back; "
                        + ("double-buffered over two contexts (step i+1's H2D overlaps step i)"

@@ -38,6 +38,31 @@ int sv_cuda(cudaError_t e, const char* what, int line) {
 extern "C" const char* sieve_last_error(void) { return t_err.c_str(); }
 extern "C" const char* sieve_version(void) { return "sieve-b200 0.1 (sm_100a)"; }
 
+cudaError_t sv_set_smem(const void* fn, int bytes) {
+  // small lock-free cache of (kernel, device) -> largest size already set; a race only repeats
+  // an idempotent driver call
+  struct E { std::atomic<const void*> fn; std::atomic<int> dev, bytes; };
+  static E cache[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  for (auto& e : cache) {
+    const void* f = e.fn.load(std::memory_order_acquire);
+    if (f == fn && e.dev.load() == dev) {
+      if (e.bytes.load() >= bytes) return cudaSuccess;
+      cudaError_t r = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+      if (r == cudaSuccess) e.bytes.store(bytes);
+      return r;
+    }
+    if (f == nullptr) {
+      cudaError_t r = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+      const void* expect = nullptr;
+      if (r == cudaSuccess && e.fn.compare_exchange_strong(expect, fn)) { e.dev.store(dev); e.bytes.store(bytes); }
+      return r;
+    }
+  }
+  return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+}
+
 int sv_num_sms() {
   static int cache[64] = {0};
   int dev = 0;
@@ -858,11 +883,13 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       }
       PhaseTimer tm(c, SIEVE_PHASE_SORT, nin * 8);
       launch_grid_tab(segs.get(), nseg, G, gtab.get(), S);
+      // the cell keys go where an odd number of radix passes ends in ck (no copy-back)
+      u64* ck_in = radix_sort_keys_input(ck.get(), nin, (int)ib, tmp.get());
       launch_cellkey(round == 1 ? nullptr : d_chunks.get(), src, nin, round == 1 ? bx : 64, src_shift,
-                     segs.get(), G, gtab.get(), ib, (u32)ncell, s0, ck.get(),
+                     segs.get(), G, gtab.get(), ib, (u32)ncell, s0, ck_in,
                      c->count_terms ? terms.get() : nullptr, S);
       int passes = 0;
-      SV_TRY(radix_sort(ck.get(), nullptr, nin, (int)ib, tmp.get(), S, &passes));
+      SV_TRY(radix_sort(ck.get(), nullptr, nin, (int)ib, tmp.get(), S, &passes, ck_in != ck.get()));
       if (c->timing) c->acc[SIEVE_PHASE_SORT].work += (u64)passes * nin * 16;
       launch_cell_offsets(ck.get(), nin, ib, (u32)ncell, off.get(), S);
       SV_CUDA(cudaGetLastError());
@@ -1116,12 +1143,23 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(sk.alloc(std::max<u64>(Etot, 1))); SV_TRY(scnt.alloc(std::max<u64>(Etot, 1)));
     SV_TRY(sfirst.alloc(std::max<u64>(Etot, 1)));
     launch_iota_u32(idx.get(), Etot, S);
-    launch_copy(sk.get(), ak, Etot * 8, S);
     PhaseTimer tr(c, SIEVE_PHASE_REPS, 0);
-    {
+    if (c->comm) {  // equal (stratum, CTA) keys from several ranks must end up adjacent
+      launch_copy(sk.get(), ak, Etot * 8, S);
       DBuf<char> tmp(c);
       SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
       SV_TRY(radix_sort(sk.get(), idx.get(), Etot, 32 + (int)bitlen(ns), tmp.get(), S));
+    } else {
+      // one rank: every (stratum, CTA) key occurs once, so grouping by stratum suffices (the
+      // dominant CTA and the first invocation do not depend on the order within a stratum):
+      // sort the stratum ids alone (neutral slots map to ns and sort last), then gather the keys
+      DBuf<u64> sid(c);
+      SV_TRY(sid.alloc(std::max<u64>(Etot, 1)));
+      launch_entry_sids(ak, Etot, ns, sid.get(), S);
+      DBuf<char> tmp(c);
+      SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
+      SV_TRY(radix_sort(sid.get(), idx.get(), Etot, (int)bitlen(ns), tmp.get(), S));
+      launch_gather_u64(ak, idx.get(), Etot, sk.get(), S);
     }
     launch_gather_u64(ak + Etot, idx.get(), Etot, scnt.get(), S);
     launch_gather_u64(ak + 2 * Etot, idx.get(), Etot, sfirst.get(), S);

@@ -179,11 +179,11 @@ void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 firs
   u64 maxgrid = (n + (u64)AS_THREADS * AS_IPT - 1) / ((u64)AS_THREADS * AS_IPT);
   if ((u64)grid > maxgrid) grid = (int)maxgrid;
   if (tab <= AS_TAB_BUDGET) {
-    cudaFuncSetAttribute(k_assign<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(smem + tab));
+    sv_smem_attr(k_assign<true>, (int)(smem + tab));
     SV_LAUNCH(k_assign<true>, grid, AS_THREADS, smem + tab, s)(kid, x, cta, n, first_id, ktab, lows, K,
                                                                 nlows, sid_out, gh, errflags);
   } else {
-    cudaFuncSetAttribute(k_assign<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    sv_smem_attr(k_assign<false>, (int)smem);
     SV_LAUNCH(k_assign<false>, grid, AS_THREADS, smem, s)(kid, x, cta, n, first_id, ktab, lows, K,
                                                            nlows, sid_out, gh, errflags);
   }
@@ -216,6 +216,15 @@ __global__ void k_iota_u32(u32* p, u64 n) {
 }
 void launch_iota_u32(u32* p, u64 n, cudaStream_t s) {
   if (n) SV_LAUNCH(k_iota_u32, div_up(n, 256), 256, 0, s)(p, n);
+}
+
+// stratum id of every compacted (stratum, CTA) entry; neutral slots (key ~0) map to ns
+__global__ void k_entry_sids(const u64* key, u64 n, u32 ns, u64* out) {
+  u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) { u64 s = key[i] >> 32; out[i] = s < ns ? s : ns; }
+}
+void launch_entry_sids(const u64* key, u64 n, u32 ns, u64* out, cudaStream_t s) {
+  if (n) SV_LAUNCH(k_entry_sids, div_up(n, 256), 256, 0, s)(key, n, ns, out);
 }
 
 __global__ void k_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst) {

@@ -76,3 +76,9 @@ int sv_num_sms();
 // count (sieve_kernel_launches) is exact
 void sv_count_launch();
 #define SV_LAUNCH(k, g, b, sm, st) sv_count_launch(), k<<<g, b, sm, st>>>
+
+// cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once per (kernel, device, size): launchers
+// run on the host between synchronisations, where every driver call is GPU idle time
+cudaError_t sv_set_smem(const void* fn, int bytes);
+template <typename F>
+inline cudaError_t sv_smem_attr(F* fn, int bytes) { return sv_set_smem((const void*)fn, bytes); }

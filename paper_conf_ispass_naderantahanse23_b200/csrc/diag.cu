@@ -108,7 +108,7 @@ void launch_group_moments(const u32* sid, const u64* y, u64 n, u32 nstrata, GMom
   const u32 kt = (u32)group_moments_kt(nstrata);
   const int grid = sv_num_sms();
   size_t smem = (size_t)kt * GM_WORDS * 4;
-  cudaFuncSetAttribute(k_group_moments, cudaFuncAttributeMaxDynamicSharedMemorySize, GM_KT * GM_WORDS * 4);
+  sv_smem_attr(k_group_moments, GM_KT * GM_WORDS * 4);
   for (u32 k0 = 0; k0 < nstrata; k0 += kt) {
     u32 kk = nstrata - k0 < kt ? nstrata - k0 : kt;
     if (n) SV_LAUNCH(k_group_moments, grid, GM_THREADS, smem, s)(sid, y, n, k0, kk, part, errflag);

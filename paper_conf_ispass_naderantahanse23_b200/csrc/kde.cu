@@ -460,10 +460,15 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift
   const int fm = force ? atoi(force) : 0;
   if (fm >= 2) guard = true;
   auto kern = guard ? k_kde<true> : k_kde<false>;
-  cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, KDE_SMEM_BYTES);
-  int per_sm = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * KDE_WARPS, KDE_SMEM_BYTES);
-  if (per_sm < 1) per_sm = 1;
+  sv_smem_attr(kern, KDE_SMEM_BYTES);
+  static int occ[2][64];  // resident blocks per SM, per variant and device (queried once)
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int& per_sm = occ[guard][dev & 63];
+  if (per_sm < 1) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 32 * KDE_WARPS, KDE_SMEM_BYTES);
+    if (per_sm < 1) per_sm = 1;
+  }
   u32 grid = (u32)sv_num_sms() * (u32)per_sm;
   u32 need = div_up(items, KDE_WARPS);
   if (grid > need) grid = need;

@@ -46,7 +46,11 @@ size_t radix_sort_temp_bytes(u64 n, bool with_vals);
 // internal ping-pong);
 // stream-ordered, no host synchronisation
 int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s,
-               int* passes = nullptr);
+               int* passes = nullptr, bool keys_in_alt = false);
+// keys-only sorts: where the producer should write the n keys so that radix_sort(..., keys_in_alt
+// = (returned != keys)) ends in `keys` without a copy-back (odd pass counts start in the alternate
+// buffer, which leads `temp`)
+u64* radix_sort_keys_input(u64* keys, u64 n, int nbits, void* temp);
 
 void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s);
 size_t scan_u32_temp_bytes(u64 n);
@@ -144,6 +148,7 @@ void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 firs
 // compact occupied entries into (key, cnt, first) arrays; *count (device) += entries
 void launch_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst, unsigned long long* count,
                          cudaStream_t s);
+void launch_entry_sids(const u64* key, u64 n, u32 ns, u64* out, cudaStream_t s);
 void launch_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst, cudaStream_t s);
 void launch_iota_u32(u32* p, u64 n, cudaStream_t s);
 // reduce duplicates of equal keys (sorted) and pick each stratum's representative

@@ -213,7 +213,7 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
 
 void launch_moments(const u32* kid, const u64* x, const u64* y, u64 n, u32 K, u32 k0, u32 kt,
                     KMomPartial* part, u64* blk_tot, u64* errflags, int grid, cudaStream_t s) {
-  cudaFuncSetAttribute(k_moments, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)moments_smem(MOM_KT));
+  sv_smem_attr(k_moments, (int)moments_smem(MOM_KT));
   SV_LAUNCH(k_moments, grid, MOM_THREADS, moments_smem(kt), s)(kid, x, y, n, K, k0, kt, part, blk_tot, errflags);
 }
 

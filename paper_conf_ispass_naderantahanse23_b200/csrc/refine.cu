@@ -189,7 +189,7 @@ void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D
                     u32 tstride, u32* nt, u32* kind, cudaStream_t s) {
   if (!nseg) return;
   size_t smem = G <= VAL_GMAX ? (size_t)VAL_WARPS * 2 * G * 8 : 0;
-  cudaFuncSetAttribute(k_valleys, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)((size_t)VAL_WARPS * 2 * VAL_GMAX * 8));
+  sv_smem_attr(k_valleys, (int)((size_t)VAL_WARPS * 2 * VAL_GMAX * 8));
   SV_LAUNCH(k_valleys, div_up(nseg, VAL_WARPS), 32 * VAL_WARPS, smem, s)(segs, nseg, G, shift, D, T,
                                                                   tstride, nt, kind);
 }

@@ -357,9 +357,20 @@ size_t radix_sort_temp_bytes(u64 n, bool with_vals) {
   return b;
 }
 
-int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, int* passes) {
+u64* radix_sort_keys_input(u64* keys, u64 n, int nbits, void* temp) {
+  if (n <= 1 || nbits <= 0) return keys;
+  const int npass = (std::min(nbits, 8 * OS_MAX_PASSES) + 7) / 8;
+  (void)n;
+  return (npass & 1) ? (u64*)temp : keys;  // the alternate key buffer leads the temp block
+}
+
+int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s, int* passes,
+               bool keys_in_alt) {
   if (passes) *passes = 0;
-  if (n <= 1 || nbits <= 0) return SIEVE_OK;
+  if (n <= 1 || nbits <= 0) {
+    if (keys_in_alt && n) launch_copy(keys, temp, n * 8, s);
+    return SIEVE_OK;
+  }
   if (nbits > 8 * OS_MAX_PASSES) nbits = 8 * OS_MAX_PASSES;
   const int npass = (nbits + 7) / 8;
   u64 ntiles = (n + RS_TILE - 1) / RS_TILE;
@@ -373,18 +384,18 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   u32* tile_counter = (u32*)t;
   SV_CUDA(cudaMemsetAsync(ghist, 0, (size_t)npass * 256 * 4, s));
   size_t hsmem = (size_t)(RS_WARPS / 2) * npass * 256 * 4;
-  SV_CUDA(cudaFuncSetAttribute(k_os_hist, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsmem));
+  SV_CUDA(sv_smem_attr(k_os_hist, (int)hsmem));
   u64 hgrid = std::min<u64>((n + RS_THREADS - 1) / RS_THREADS, (u64)sv_num_sms() * 4);
-  SV_LAUNCH(k_os_hist, (unsigned)hgrid, RS_THREADS, hsmem, s)(keys, n, npass, nbits >= 64 ? ~0ull : (1ull << nbits) - 1, ghist);
+  SV_LAUNCH(k_os_hist, (unsigned)hgrid, RS_THREADS, hsmem, s)(keys_in_alt ? kalt : keys, n, npass, nbits >= 64 ? ~0ull : (1ull << nbits) - 1, ghist);
   // digit bases on the device (no host round trip): every pass runs -- a pass over a digit
   // that is constant across all keys is a stable identity permutation, so skipping it would only
   // save time, never change the result
   SV_LAUNCH(k_os_scan, npass, RS_THREADS, 0, s)(ghist, gbase);
   size_t smem = (size_t)RS_TILE * (vals ? 8 + 4 : 8);
-  SV_CUDA(cudaFuncSetAttribute(k_os_pass<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               RS_TILE * (8 + 4)));
-  SV_CUDA(cudaFuncSetAttribute(k_os_pass<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, RS_TILE * 8));
+  SV_CUDA(sv_smem_attr(k_os_pass<true>, RS_TILE * (8 + 4)));
+  SV_CUDA(sv_smem_attr(k_os_pass<false>, RS_TILE * 8));
   u64* kin = keys; u32* vin = vals; u64* kout = kalt; u32* vout = valt;
+  if (keys_in_alt) { kin = kalt; kout = keys; }  // keys-only: the producer wrote the alt buffer
   for (int p = 0; p < npass; p++) {
     // digits above nbits are masked off (keys may carry payload bits there)
     const u32 dmask = 8 * p + 8 <= nbits ? 255u : (1u << (nbits - 8 * p)) - 1u;
