@@ -876,7 +876,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(ck.alloc(std::max<u64>(nin, 1)));
     {
       DBuf<char> tmp(c);
-      SV_TRY(tmp.alloc(radix_sort_temp_bytes(nin, false)));
+      SV_TRY(tmp.alloc(radix_sort_temp_bytes(nin, false, (int)ib)));
       if (!chunks.empty()) {
         SV_TRY(d_chunks.alloc(chunks.size()));
         SV_TRY(h2d(c, d_chunks.get(), chunks));
@@ -1147,7 +1147,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     if (c->comm) {  // equal (stratum, CTA) keys from several ranks must end up adjacent
       launch_copy(sk.get(), ak, Etot * 8, S);
       DBuf<char> tmp(c);
-      SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
+      SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true, 32 + (int)bitlen(ns))));
       SV_TRY(radix_sort(sk.get(), idx.get(), Etot, 32 + (int)bitlen(ns), tmp.get(), S));
     } else {
       // one rank: every (stratum, CTA) key occurs once, so grouping by stratum suffices (the
@@ -1157,7 +1157,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       SV_TRY(sid.alloc(std::max<u64>(Etot, 1)));
       launch_entry_sids(ak, Etot, ns, sid.get(), S);
       DBuf<char> tmp(c);
-      SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true)));
+      SV_TRY(tmp.alloc(radix_sort_temp_bytes(Etot, true, (int)bitlen(ns))));
       SV_TRY(radix_sort(sid.get(), idx.get(), Etot, (int)bitlen(ns), tmp.get(), S));
       launch_gather_u64(ak, idx.get(), Etot, sk.get(), S);
     }
@@ -1358,7 +1358,7 @@ extern "C" int sieve_min_strata(sieve_trace t, uint32_t theta_num, uint32_t thet
     launch_t3_compact(t->kid, t->x, t->n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
     {
       DBuf<char> tmp(c);
-      SV_TRY(tmp.alloc(radix_sort_temp_bytes(n3, false)));
+      SV_TRY(tmp.alloc(radix_sort_temp_bytes(n3, false, nbits)));
       SV_TRY(radix_sort(keys.get(), nullptr, n3, nbits, tmp.get(), S));
     }
     // run-length encoding: distinct keys, run starts, Tier-3 rank starts
@@ -1674,7 +1674,7 @@ extern "C" int sieve_load_csv(sieve_ctx ctx, const char* data, uint64_t bytes, u
     launch_csv_firsts(flag.get(), seg.get(), row.get(), nrows, fkey.get(), fval.get(), S);
     {
       DBuf<char> tmp(c);
-      if ((st = tmp.alloc(radix_sort_temp_bytes(nd, true))) != SIEVE_OK) return fail(st);
+      if ((st = tmp.alloc(radix_sort_temp_bytes(nd, true, 32))) != SIEVE_OK) return fail(st);
       if ((st = radix_sort(fkey.get(), fval.get(), nd, 32, tmp.get(), S)) != SIEVE_OK) return fail(st);
     }
     launch_csv_ids(fval.get(), nd, id_of.get(), flag.get(), seg.get(), row.get(), nrows, t->kid, S);

@@ -30,6 +30,9 @@
 #include "kernels.cuh"
 
 #define BK_THREADS 256
+#ifndef BK_U
+#define BK_U 2            // values per thread in flight (A/B: 1, 2, 4 within noise; 8 slower)
+#endif
 
 __device__ __forceinline__ double grid_pt_b(u64 lo, u64 hi, u32 j, u32 G) {
   return __dadd_rn(__ull2double_rn(lo),
@@ -103,27 +106,40 @@ k_cellkey(const BucketChunk* __restrict__ chunks, u32 nchunks, const u64* __rest
   const u32 nseg = ncell / G;
   const u64 xmask = bx >= 64 ? ~0ull : ((1ull << bx) - 1);
   u64 win = 0;
-  const u64 stride = (u64)gridDim.x * BK_THREADS;
-  for (u64 i = (u64)blockIdx.x * BK_THREADS + threadIdx.x; i < nin; i += stride) {
-    u64 x;
-    u32 s;
-    if (!chunks) {  // round 1: tagged Tier-3 keys, one output per input
-      u64 v = __ldcs(in + i);
-      s = (u32)(v >> bx) - seg0;  // this batch's segments are t3rank seg0 .. seg0 + nseg - 1
-      x = v & xmask;
-      if (s >= nseg) {
-        out[i] = ncell;
-        continue;
+  // BK_U values per thread per step, all loaded before any is processed (latency hiding)
+  const u64 stride = (u64)gridDim.x * BK_THREADS * BK_U;
+  for (u64 i0 = (u64)blockIdx.x * BK_THREADS * BK_U + threadIdx.x; i0 < nin; i0 += stride) {
+    u64 xs[BK_U];
+    u32 ss[BK_U];
+#pragma unroll
+    for (int u = 0; u < BK_U; u++) {
+      const u64 i = i0 + (u64)u * BK_THREADS;
+      ss[u] = 0xFFFFFFFFu;  // sentinel: out of range / padding / another batch
+      xs[u] = 0;
+      if (i >= nin) continue;
+      if (!chunks) {  // round 1: tagged Tier-3 keys, one output per input
+        const u64 v = __ldcs(in + i);
+        const u32 s = (u32)(v >> bx) - seg0;  // this batch's segments are t3rank seg0 .. seg0 + nseg - 1
+        xs[u] = v & xmask;
+        if (s < nseg) ss[u] = s;
+      } else {        // later rounds: output i lies in chunk c (chunks hold BK_CHUNK values each)
+        const BucketChunk ch = chunks[i / BK_CHUNK];
+        const u32 r = (u32)(i % BK_CHUNK);
+        if (r < ch.len) {  // else padding of a short chunk: sorts to the end
+          ss[u] = ch.seg;
+          xs[u] = __ldcs(in + ch.begin + r) >> in_shift;
+        }
       }
-    } else {        // later rounds: output i lies in chunk c (chunks hold BK_CHUNK values each)
-      const BucketChunk ch = chunks[i / BK_CHUNK];
-      const u32 r = (u32)(i % BK_CHUNK);
-      if (r >= ch.len) {  // padding of a short chunk: sorts to the end
-        out[i] = ncell;
-        continue;
-      }
-      s = ch.seg;
-      x = __ldcs(in + ch.begin + r) >> in_shift;
+    }
+#pragma unroll
+    for (int u = 0; u < BK_U; u++) {
+    const u64 i = i0 + (u64)u * BK_THREADS;
+    if (i >= nin) continue;
+    const u64 x = xs[u];
+    const u32 s = ss[u];
+    if (s == 0xFFFFFFFFu) {
+      out[i] = ncell;
+      continue;
     }
     const SegDev& g = segs[s];
     u64 lo = g.lo, hi = g.hi;
@@ -135,6 +151,7 @@ k_cellkey(const BucketChunk* __restrict__ chunks, u32 nchunks, const u64* __rest
       if (inwin) win += inwin_count(gf, G, cq, __dmul_rn(KDE_WC, g.h), x);
     }
     out[i] = (x << ib) | idx;
+    }
   }
   if (inwin) {
     for (int o = 16; o > 0; o >>= 1) win += __shfl_down_sync(0xffffffffu, win, o);
@@ -146,7 +163,7 @@ void launch_cellkey(const BucketChunk* chunks, const u64* in, u64 nin, u32 bx, u
                     const SegDev* segs, u32 G, const double* gtab, u32 ib, u32 ncell, u32 seg0,
                     u64* out, unsigned long long* inwin, cudaStream_t s) {
   if (!nin) return;
-  u64 grid = std::min<u64>((nin + BK_THREADS - 1) / BK_THREADS, (u64)sv_num_sms() * 8);
+  u64 grid = std::min<u64>((nin + BK_THREADS * BK_U - 1) / (BK_THREADS * BK_U), (u64)sv_num_sms() * 8);
   SV_LAUNCH(k_cellkey, (u32)grid, BK_THREADS, 0, s)(chunks, 0, in, nin, bx, in_shift, segs, G, gtab,
                                                     ib, ncell, seg0, out, inwin);
 }

@@ -41,7 +41,7 @@ void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u
                        u64* keys_out, unsigned long long* counter, cudaStream_t s);
 
 // ---------------- LSD radix sort (u64 keys, optional u32 payload) ----------------------------
-size_t radix_sort_temp_bytes(u64 n, bool with_vals);
+size_t radix_sort_temp_bytes(u64 n, bool with_vals, int nbits = 64);  // nbits as passed to radix_sort
 // sorts keys[0..n) by bits [0, nbits) (higher bits ride along); result in keys/vals (in place via
 // internal ping-pong);
 // stream-ordered, no host synchronisation

@@ -347,13 +347,14 @@ __global__ void __launch_bounds__(RS_THREADS) k_os_scan(const u32* __restrict__ 
 
 static size_t al256(size_t b) { return (b + 255) / 256 * 256; }
 
-size_t radix_sort_temp_bytes(u64 n, bool with_vals) {
+size_t radix_sort_temp_bytes(u64 n, bool with_vals, int nbits) {
   u64 ntiles = (n + RS_TILE - 1) / RS_TILE;
+  const u64 np = (u64)(std::max(1, std::min(nbits, 8 * OS_MAX_PASSES)) + 7) / 8;
   size_t b = al256(n * 8);                       // alt keys
   if (with_vals) b += al256(n * 4);              // alt vals
-  b += al256(ntiles * 256 * 8);                  // look-back status words
+  b += al256(np * ntiles * 256 * 8);             // look-back status words, one set per pass
   b += al256(OS_MAX_PASSES * 256 * 4) * 2;       // histograms, bases
-  b += 256;                                      // tile counter
+  b += 256;                                      // tile counters, one per pass
   return b;
 }
 
@@ -378,11 +379,14 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   u64* kalt = (u64*)t; t += al256(n * 8);
   u32* valt = nullptr;
   if (vals) { valt = (u32*)t; t += al256(n * 4); }
-  u64* status = (u64*)t; t += al256(ntiles * 256 * 8);
+  u64* status = (u64*)t; t += al256((u64)npass * ntiles * 256 * 8);  // as radix_sort_temp_bytes(nbits)
   u32* ghist = (u32*)t; t += al256(OS_MAX_PASSES * 256 * 4);
   u32* gbase = (u32*)t; t += al256(OS_MAX_PASSES * 256 * 4);
   u32* tile_counter = (u32*)t;
   SV_CUDA(cudaMemsetAsync(ghist, 0, (size_t)npass * 256 * 4, s));
+  // every pass has its own status words and tile counter: one memset each for the whole sort
+  SV_CUDA(cudaMemsetAsync(status, 0, (size_t)npass * ntiles * 256 * 8, s));
+  SV_CUDA(cudaMemsetAsync(tile_counter, 0, OS_MAX_PASSES * 4, s));
   size_t hsmem = (size_t)(RS_WARPS / 2) * npass * 256 * 4;
   SV_CUDA(sv_smem_attr(k_os_hist, (int)hsmem));
   u64 hgrid = std::min<u64>((n + RS_THREADS - 1) / RS_THREADS, (u64)sv_num_sms() * 4);
@@ -399,14 +403,13 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   for (int p = 0; p < npass; p++) {
     // digits above nbits are masked off (keys may carry payload bits there)
     const u32 dmask = 8 * p + 8 <= nbits ? 255u : (1u << (nbits - 8 * p)) - 1u;
-    SV_CUDA(cudaMemsetAsync(status, 0, ntiles * 256 * 8, s));
-    SV_CUDA(cudaMemsetAsync(tile_counter, 0, 4, s));
+    u64* st = status + (u64)p * ntiles * 256;
     if (vals)
       SV_LAUNCH(k_os_pass<true>, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, 8 * p, dmask, gbase + p * 256,
-                                                                     status, tile_counter, kout, vout);
+                                                                     st, tile_counter + p, kout, vout);
     else
       SV_LAUNCH(k_os_pass<false>, (unsigned)ntiles, RS_THREADS, smem, s)(kin, vin, n, 8 * p, dmask, gbase + p * 256,
-                                                                      status, tile_counter, kout, vout);
+                                                                      st, tile_counter + p, kout, vout);
     u64* tk = kin; kin = kout; kout = tk;
     u32* tv = vin; vin = vout; vout = tv;
     if (passes) (*passes)++;
