@@ -160,6 +160,26 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def pin_to_gpu_numa(dev):
+    """Run this rank on the CPU cores next to its GPU (NVML's affinity mask), before any host
+    buffer is touched: the generator's threads then place the pinned trace columns in the GPU's
+    NUMA node, and the e2e H2D reads local memory.  Returns the core count, or None."""
+    try:
+        import pynvml
+        pynvml.nvmlInit()
+        h = pynvml.nvmlDeviceGetHandleByIndex(dev)
+        words = (os.cpu_count() + 63) // 64
+        mask = pynvml.nvmlDeviceGetCpuAffinity(h, words)
+        cpus = [64 * w + b for w, m in enumerate(mask) for b in range(64) if (m >> b) & 1]
+        cpus = [c for c in cpus if c in os.sched_getaffinity(0)]
+        if cpus:
+            os.sched_setaffinity(0, cpus)
+            return len(cpus)
+    except Exception:
+        pass
+    return None
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -173,6 +193,7 @@ def main():
 
     rank, world = int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    cpus = pin_to_gpu_numa(local)
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
@@ -327,6 +348,7 @@ def main():
                "d2h_bytes_per_step": int(out["strata"] * 96 + 56), "steps": e_steps,
                # the step is bound by the PCIe H2D of the columns: the rate it implies
                "h2d_GBps_per_rank": n_local * 24 * e_steps / (ems / 1000.0) / 1e9,
+               "host_cores_near_gpu": cpus,   # NVML affinity the rank was pinned to (None: not pinned)
                "note": "every step: H2D of kid/x/cta/y from pinned host memory (sieve_load_trace) + "
                        "stratify + predict, stratum table and prediction read back; "
                        + ("double-buffered over two contexts (step i+1's H2D overlaps step i)"

@@ -115,11 +115,46 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_apply(const u32* in, u64 n,
   }
 }
 
+// small scans (up to SC_SMALL tiles: the per-round KDE tile and part counts) in ONE block that
+// walks the tiles with a carry: one launch instead of three (the host launch cost between
+// synchronisations is GPU idle time)
+#define SC_SMALL 4
+__global__ void __launch_bounds__(SC_THREADS) k_scan_single(const u32* in, u64 n, u32* out, u32* total) {
+  __shared__ u32 carry_s;
+  if (threadIdx.x == 0) carry_s = 0;
+  __syncthreads();
+  for (u64 t0 = 0; t0 < n; t0 += SC_TILE) {
+    const u64 base = t0 + (u64)threadIdx.x * SC_IPT;
+    u32 v[SC_IPT];
+    u32 sum = 0;
+#pragma unroll
+    for (int j = 0; j < SC_IPT; j++) {
+      v[j] = base + j < n ? in[base + j] : 0;
+      sum += v[j];
+    }
+    __shared__ u32 tot;
+    u32 ex = block_excl_scan<u32, SC_THREADS>(sum, &tot) + carry_s;
+#pragma unroll
+    for (int j = 0; j < SC_IPT; j++) {
+      if (base + j < n) out[base + j] = ex;
+      ex += v[j];
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) carry_s += tot;
+    __syncthreads();
+  }
+  if (threadIdx.x == 0 && total) *total = carry_s;
+}
+
 size_t scan_u32_temp_bytes(u64 n) { return ((n + SC_TILE - 1) / SC_TILE + 2) * sizeof(u32); }
 
 // exclusive scan in -> out (may alias); total (device pointer, nullable) receives the sum
 void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s) {
   u32 nb = div_up(n ? n : 1, SC_TILE);
+  if (nb <= SC_SMALL) {
+    SV_LAUNCH(k_scan_single, 1, SC_THREADS, 0, s)(in, n, out, total);
+    return;
+  }
   u32* bsum = (u32*)temp;
   SV_LAUNCH(k_scan_reduce, nb, SC_THREADS, 0, s)(in, n, bsum);
   SV_LAUNCH(k_scan_blocks, 1, SC_THREADS, 0, s)(bsum, nb, total);
@@ -379,14 +414,13 @@ int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t 
   u64* kalt = (u64*)t; t += al256(n * 8);
   u32* valt = nullptr;
   if (vals) { valt = (u32*)t; t += al256(n * 4); }
+  // status words (one set per pass) | histograms | tile counters (one per pass) | digit bases:
+  // the first three are zeroed by ONE memset for the whole sort
   u64* status = (u64*)t; t += al256((u64)npass * ntiles * 256 * 8);  // as radix_sort_temp_bytes(nbits)
   u32* ghist = (u32*)t; t += al256(OS_MAX_PASSES * 256 * 4);
-  u32* gbase = (u32*)t; t += al256(OS_MAX_PASSES * 256 * 4);
-  u32* tile_counter = (u32*)t;
-  SV_CUDA(cudaMemsetAsync(ghist, 0, (size_t)npass * 256 * 4, s));
-  // every pass has its own status words and tile counter: one memset each for the whole sort
-  SV_CUDA(cudaMemsetAsync(status, 0, (size_t)npass * ntiles * 256 * 8, s));
-  SV_CUDA(cudaMemsetAsync(tile_counter, 0, OS_MAX_PASSES * 4, s));
+  u32* tile_counter = (u32*)t; t += 256;
+  u32* gbase = (u32*)t;
+  SV_CUDA(cudaMemsetAsync(status, 0, (size_t)((char*)gbase - (char*)status), s));
   size_t hsmem = (size_t)(RS_WARPS / 2) * npass * 256 * 4;
   SV_CUDA(sv_smem_attr(k_os_hist, (int)hsmem));
   u64 hgrid = std::min<u64>((n + RS_THREADS - 1) / RS_THREADS, (u64)sv_num_sms() * 4);

@@ -1,0 +1,73 @@
+// Throwaway microbenchmark: FP64-pipe rate of the current KDE term (9 FP64 ops + lane-replicated
+// table + byte permutes) in a register-only loop, against variants without the table / int ops.
+#include <cstdio>
+#include <cstdint>
+typedef unsigned long long u64; typedef unsigned u32;
+#define C_LOG2E_128 0x1.71547652b82fep+7
+#define C_LN2_128 0x1.62e42fefa39efp-8
+#define C_MAGIC 0x1.8p+52
+#define C_TWO52 0x1.0p+52
+#define C_P3 (-0x1.5555555555555p-3 * 0x1p-3)
+__constant__ double c_kde[3] = {C_LOG2E_128, C_LN2_128, C_P3};
+template <int V>
+__device__ __forceinline__ double term(double gs, double xs, const double* sS, double L, double M, double acc) {
+  double z = __dsub_rn(gs, xs);
+  double u = __dmul_rn(z, z);
+  double kb = __fma_rn(u, L, M);
+  double kf = __dsub_rn(kb, C_MAGIC);
+  double r = __fma_rn(-kf, c_kde[1], u);
+  double p = __fma_rn(c_kde[2], r, 0.125);
+  p = __fma_rn(p, r, -0.5);
+  p = __fma_rn(p, r, 1.0);
+  double S;
+  if (V == 0) {
+    u32 k = (u32)__double2loint(kb);
+    double T = *(const double*)((const char*)sS + __byte_perm(k, 0u, 0x4404u));
+    S = __hiloint2double(__double2hiint(T) - (int)(__byte_perm(k, 0u, 0x4144u) << 4), __double2loint(T));
+  } else {
+    S = kf;  // no table, no int ops
+  }
+  return __fma_rn(p, S, acc);
+}
+template <int V, int U>
+__global__ void __launch_bounds__(512, 1) k(double* out, int iters, double g0) {
+  extern __shared__ double sS[];
+  for (int i = threadIdx.x; i < 256 * 32; i += blockDim.x) sS[i] = 0x1p40 * (1.0 - (i >> 5) * 1e-3);
+  __syncthreads();
+  const double* sSb = sS + (threadIdx.x & 31);
+  double L, M;
+  asm volatile("mov.b64 %0, %1;" : "=d"(L) : "d"(c_kde[0]));
+  asm volatile("mov.b64 %0, %1;" : "=d"(M) : "d"(C_MAGIC));
+  double ac[U];
+  for (int q = 0; q < U; q++) ac[q] = C_TWO52;
+  double gs = g0 + threadIdx.x * 0.03;
+  for (int it = 0; it < iters; it++) {
+    double xs = it * 1e-3;
+#pragma unroll
+    for (int q = 0; q < U; q++) ac[q] = term<V>(gs, xs + q * 0.01, sSb, L, M, ac[q]);
+  }
+  double s = 0; for (int q = 0; q < U; q++) s += ac[q];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+template <int V, int U>
+void run(const char* name, double* d, int iters) {
+  cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
+  cudaFuncSetAttribute(k<V, U>, cudaFuncAttributeMaxDynamicSharedMemorySize, 65536);
+  k<V, U><<<148, 512, 65536>>>(d, 10, 1.0);
+  cudaEventRecord(a);
+  k<V, U><<<148, 512, 65536>>>(d, iters, 1.0);
+  cudaEventRecord(b); cudaEventSynchronize(b);
+  float ms; cudaEventElapsedTime(&ms, a, b);
+  double ops = 148.0 * 512 * iters * U * 9;
+  int clk; cudaDeviceGetAttribute(&clk, cudaDevAttrClockRate, 0);
+  double peak = 148.0 * 64 * clk * 1e3;
+  printf("%-22s %8.3f ms  %.2f T FP64-pipe/s  %.1f%% of %.2f T\n", name, ms, ops / ms / 1e9, 100 * ops / ms / 1e9 / (peak / 1e12), peak / 1e12);
+}
+int main() {
+  double* d; cudaMalloc(&d, 148 * 512 * 8);
+  run<0, 16>("term+table u16", d, 4000);
+  run<1, 16>("term no-table u16", d, 4000);
+  run<0, 8>("term+table u8", d, 8000);
+  run<0, 24>("term+table u24", d, 2700);
+  return 0;
+}
