@@ -9,18 +9,29 @@ typedef unsigned long long u64; typedef unsigned u32;
 #define C_TWO52 0x1.0p+52
 #define C_P3 (-0x1.5555555555555p-3 * 0x1p-3)
 __constant__ double c_kde[3] = {C_LOG2E_128, C_LN2_128, C_P3};
+__device__ double g_one = 1.0, g_nz = -0.0, g_nmagic = -C_MAGIC;
+struct Ops { double one, nz, nmagic; };
 template <int V>
-__device__ __forceinline__ double term(double gs, double xs, const double* sS, double L, double M, double acc) {
-  double z = __dsub_rn(gs, xs);
-  double u = __dmul_rn(z, z);
-  double kb = __fma_rn(u, L, M);
-  double kf = __dsub_rn(kb, C_MAGIC);
+__device__ __forceinline__ double term(double gs, double xs, const double* sS, double L, double M, double acc,
+                                       Ops o = Ops{1.0, -0.0, -C_MAGIC}) {
+  double z, u, kf, kb;
+  if (V >= 2) {  // every add / mul as a DFMA with opaque register operands (same roundings)
+    z = __fma_rn(xs, -o.one, gs);
+    u = __fma_rn(z, z, o.nz);
+    kb = __fma_rn(u, L, M);
+    kf = __fma_rn(kb, o.one, o.nmagic);
+  } else {
+    z = __dsub_rn(gs, xs);
+    u = __dmul_rn(z, z);
+    kb = __fma_rn(u, L, M);
+    kf = __dsub_rn(kb, C_MAGIC);
+  }
   double r = __fma_rn(-kf, c_kde[1], u);
   double p = __fma_rn(c_kde[2], r, 0.125);
   p = __fma_rn(p, r, -0.5);
   p = __fma_rn(p, r, 1.0);
   double S;
-  if (V == 0) {
+  if (V == 0 || V == 2) {
     u32 k = (u32)__double2loint(kb);
     double T = *(const double*)((const char*)sS + __byte_perm(k, 0u, 0x4404u));
     S = __hiloint2double(__double2hiint(T) - (int)(__byte_perm(k, 0u, 0x4144u) << 4), __double2loint(T));
@@ -41,10 +52,25 @@ __global__ void __launch_bounds__(512, 1) k(double* out, int iters, double g0) {
   double ac[U];
   for (int q = 0; q < U; q++) ac[q] = C_TWO52;
   double gs = g0 + threadIdx.x * 0.03;
+  Ops o;
+  asm volatile("mov.b64 %0, %1;" : "=d"(o.one) : "d"(g_one));
+  asm volatile("mov.b64 %0, %1;" : "=d"(o.nz) : "d"(g_nz));
+  asm volatile("mov.b64 %0, %1;" : "=d"(o.nmagic) : "d"(g_nmagic));
+  if (V >= 4) {  // raw pipe tests: 9 independent chains of one op kind
+    double a[U];
+    for (int q = 0; q < U; q++) a[q] = gs + q;
+    for (int it = 0; it < iters; it++)
+#pragma unroll
+      for (int r = 0; r < 9; r++)
+#pragma unroll
+        for (int q = 0; q < U; q++)
+          a[q] = V == 4 ? __dadd_rn(a[q], o.nz) : V == 5 ? __dmul_rn(a[q], o.one) : __fma_rn(a[q], o.one, o.nz);
+    for (int q = 0; q < U; q++) ac[q] = a[q];
+  } else
   for (int it = 0; it < iters; it++) {
     double xs = it * 1e-3;
 #pragma unroll
-    for (int q = 0; q < U; q++) ac[q] = term<V>(gs, xs + q * 0.01, sSb, L, M, ac[q]);
+    for (int q = 0; q < U; q++) ac[q] = term<V>(gs, xs + q * 0.01, sSb, L, M, ac[q], o);
   }
   double s = 0; for (int q = 0; q < U; q++) s += ac[q];
   out[blockIdx.x * blockDim.x + threadIdx.x] = s;
@@ -67,7 +93,10 @@ int main() {
   double* d; cudaMalloc(&d, 148 * 512 * 8);
   run<0, 16>("term+table u16", d, 4000);
   run<1, 16>("term no-table u16", d, 4000);
-  run<0, 8>("term+table u8", d, 8000);
-  run<0, 24>("term+table u24", d, 2700);
+  run<2, 16>("all-DFMA term+table", d, 4000);
+  run<3, 16>("all-DFMA no-table", d, 4000);
+  run<4, 16>("DADD only", d, 4000);
+  run<5, 16>("DMUL only", d, 4000);
+  run<6, 16>("DFMA only", d, 4000);
   return 0;
 }
