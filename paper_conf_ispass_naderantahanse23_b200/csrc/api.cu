@@ -883,13 +883,16 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       }
       PhaseTimer tm(c, SIEVE_PHASE_SORT, nin * 8);
       launch_grid_tab(segs.get(), nseg, G, gtab.get(), S);
-      // the cell keys go where an odd number of radix passes ends in ck (no copy-back)
+      // the cell keys go where an odd number of radix passes ends in ck (no copy-back), and
+      // k_cellkey accumulates the sort's digit histograms as it writes them (no histogram read)
       u64* ck_in = radix_sort_keys_input(ck.get(), nin, (int)ib, tmp.get());
+      u32* ghist = (nin > 1 && ib <= 24) ? radix_sort_prepare(nin, false, (int)ib, tmp.get(), S) : nullptr;
       launch_cellkey(round == 1 ? nullptr : d_chunks.get(), src, nin, round == 1 ? bx : 64, src_shift,
                      segs.get(), G, gtab.get(), ib, (u32)ncell, s0, ck_in,
-                     c->count_terms ? terms.get() : nullptr, S);
+                     c->count_terms ? terms.get() : nullptr, ghist, S);
       int passes = 0;
-      SV_TRY(radix_sort(ck.get(), nullptr, nin, (int)ib, tmp.get(), S, &passes, ck_in != ck.get()));
+      SV_TRY(radix_sort(ck.get(), nullptr, nin, (int)ib, tmp.get(), S, &passes, ck_in != ck.get(),
+                        ghist != nullptr));
       if (c->timing) c->acc[SIEVE_PHASE_SORT].work += (u64)passes * nin * 16;
       launch_cell_offsets(ck.get(), nin, ib, (u32)ncell, off.get(), S);
       SV_CUDA(cudaGetLastError());

@@ -102,7 +102,14 @@ __device__ __forceinline__ u32 inwin_count(const GridFn& g, u32 G, double cq, do
 __global__ void __launch_bounds__(BK_THREADS)
 k_cellkey(const BucketChunk* __restrict__ chunks, u32 nchunks, const u64* __restrict__ in, u64 nin,
           u32 bx, u32 in_shift, const SegDev* __restrict__ segs, u32 G, const double* __restrict__ gtab,
-          u32 ib, u32 ncell, u32 seg0, u64* __restrict__ out, unsigned long long* inwin) {
+          u32 ib, u32 ncell, u32 seg0, u64* __restrict__ out, unsigned long long* inwin,
+          u32* __restrict__ ghist) {
+  // ghist != nullptr: the radix sort's digit histograms of the output keys over bits [0, ib)
+  // (the cell index) are accumulated here, so the sort skips its own histogram read
+  __shared__ u32 s_hist[3 * 256];
+  const int npass = ghist ? (int)((ib + 7) / 8) : 0;   // ib <= 24 on this path (see launch)
+  for (int i = threadIdx.x; i < npass * 256; i += BK_THREADS) s_hist[i] = 0;
+  if (ghist) __syncthreads();
   const u32 nseg = ncell / G;
   const u64 xmask = bx >= 64 ? ~0ull : ((1ull << bx) - 1);
   u64 win = 0;
@@ -139,6 +146,7 @@ k_cellkey(const BucketChunk* __restrict__ chunks, u32 nchunks, const u64* __rest
     const u32 s = ss[u];
     if (s == 0xFFFFFFFFu) {
       out[i] = ncell;
+      for (int p = 0; p < npass; p++) atomicAdd(&s_hist[p * 256 + ((ncell >> (8 * p)) & 255u)], 1u);
       continue;
     }
     const SegDev& g = segs[s];
@@ -151,7 +159,13 @@ k_cellkey(const BucketChunk* __restrict__ chunks, u32 nchunks, const u64* __rest
       if (inwin) win += inwin_count(gf, G, cq, __dmul_rn(KDE_WC, g.h), x);
     }
     out[i] = (x << ib) | idx;
+    for (int p = 0; p < npass; p++) atomicAdd(&s_hist[p * 256 + ((idx >> (8 * p)) & 255u)], 1u);
     }
+  }
+  if (ghist) {
+    __syncthreads();
+    for (int i = threadIdx.x; i < npass * 256; i += BK_THREADS)
+      if (s_hist[i]) atomicAdd(&ghist[i], s_hist[i]);
   }
   if (inwin) {
     for (int o = 16; o > 0; o >>= 1) win += __shfl_down_sync(0xffffffffu, win, o);
@@ -161,11 +175,12 @@ k_cellkey(const BucketChunk* __restrict__ chunks, u32 nchunks, const u64* __rest
 
 void launch_cellkey(const BucketChunk* chunks, const u64* in, u64 nin, u32 bx, u32 in_shift,
                     const SegDev* segs, u32 G, const double* gtab, u32 ib, u32 ncell, u32 seg0,
-                    u64* out, unsigned long long* inwin, cudaStream_t s) {
+                    u64* out, unsigned long long* inwin, u32* ghist, cudaStream_t s) {
   if (!nin) return;
+  if (ib > 24) ghist = nullptr;  // (the caller then lets the sort build its histograms)
   u64 grid = std::min<u64>((nin + BK_THREADS * BK_U - 1) / (BK_THREADS * BK_U), (u64)sv_num_sms() * 8);
   SV_LAUNCH(k_cellkey, (u32)grid, BK_THREADS, 0, s)(chunks, 0, in, nin, bx, in_shift, segs, G, gtab,
-                                                    ib, ncell, seg0, out, inwin);
+                                                    ib, ncell, seg0, out, inwin, ghist);
 }
 
 // off[c] = first position of the sorted keys with idx >= c, c = 0..ncell (position i writes the

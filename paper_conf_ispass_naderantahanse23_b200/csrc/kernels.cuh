@@ -46,11 +46,15 @@ size_t radix_sort_temp_bytes(u64 n, bool with_vals, int nbits = 64);  // nbits a
 // internal ping-pong);
 // stream-ordered, no host synchronisation
 int radix_sort(u64* keys, u32* vals, u64 n, int nbits, void* temp, cudaStream_t s,
-               int* passes = nullptr, bool keys_in_alt = false);
+               int* passes = nullptr, bool keys_in_alt = false, bool prepared = false);
 // keys-only sorts: where the producer should write the n keys so that radix_sort(..., keys_in_alt
 // = (returned != keys)) ends in `keys` without a copy-back (odd pass counts start in the alternate
 // buffer, which leads `temp`)
 u64* radix_sort_keys_input(u64* keys, u64 n, int nbits, void* temp);
+// optional: zero the sort's scratch now and return its digit-histogram array (npass x 256 u32),
+// for a producer that accumulates the histograms of the keys it writes; then call radix_sort
+// with prepared = true (it skips its zeroing and its histogram pass)
+u32* radix_sort_prepare(u64 n, bool with_vals, int nbits, void* temp, cudaStream_t s);
 
 void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s);
 size_t scan_u32_temp_bytes(u64 n);
@@ -103,7 +107,8 @@ void launch_grid_tab(const SegDev* segs, u32 nseg, u32 G, double* gtab, cudaStre
 // the sentinel), else x = in[..] >> in_shift; *inwin += in-window KDE terms
 void launch_cellkey(const BucketChunk* chunks, const u64* in, u64 nin, u32 bx, u32 in_shift,
                     const SegDev* segs, u32 G, const double* gtab, u32 ib, u32 ncell, u32 seg0,
-                    u64* out, unsigned long long* inwin, cudaStream_t s);
+                    u64* out, unsigned long long* inwin, u32* ghist /* nullable: radix_sort_prepare */,
+                    cudaStream_t s);
 // off[c] = first position of the idx-sorted keys with idx >= c, c = 0..ncell
 void launch_cell_offsets(const u64* keys, u64 n, u32 ib, u32 ncell, u32* off, cudaStream_t s);
 
