@@ -402,7 +402,10 @@ def main():
             "config": {"workload": cfg.name, "invocations": cfg.n, "kernels": cfg.K,
                        "grid_points": 1024, "theta": "2/5", "strata": n_strata, "rounds": rounds,
                        "parallelism": f"dp{world} (contiguous invocation slices)",
-                       "l2": "inputs larger than L2 (24 B/invocation = 2.4 GB per step)"},
+                       "l2": (f"inputs larger than L2 (24 B/invocation = {cfg.n * 24 / 1e9:.3g} GB per step)"
+                              if cfg.n * 24 > 126e6 else
+                              f"inputs ({cfg.n * 24 / 1e6:.3g} MB) fit in L2 and L2 is not flushed: "
+                              "not a valid bench configuration, parity / smoke use only")},
             "clocks": clocks, "e2e": e2e, "gpu_launches": launches,
             "roofline": roof, "phases": phase_out,
             "host_ms_per_step": {k: statistics.mean(v) for k, v in host_ms.items() if v},
