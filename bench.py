@@ -291,7 +291,7 @@ def main():
     # issuing collectives from two threads could interleave differently across ranks).
     e2e = None
     if not args.no_e2e:
-        e_steps = max(2, min(args.steps, 6))
+        e_steps = max(4, min(args.steps, 10))   # >= 2 loads per context: a steadier PCIe average
         lanes = [(ctx, stream)]
         if world == 1:
             stream2 = torch.cuda.Stream()

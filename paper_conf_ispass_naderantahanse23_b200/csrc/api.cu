@@ -899,7 +899,20 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     }
     DBuf<u64> D(c);
     SV_TRY(D.alloc((size_t)nseg * G * 2));
-    SV_CUDA(cudaMemsetAsync(D.get(), 0, (size_t)nseg * G * 16, S));
+    // part buffers (one rank: sized by the bound nseg * tstride, see below) are initialised with
+    // the densities in one launch
+    u32 cap = nseg * tstride;
+    DBuf<u64> pl(c), pm(c), pab(c);
+    if (!c->comm) {
+      SV_TRY(pl.alloc((size_t)cap * MOM_LANES));
+      SV_TRY(pm.alloc((size_t)cap * 2));
+      SV_TRY(pab.alloc((size_t)cap * 4));
+      FillRegions fr{{D.get(), pl.get(), pm.get(), pm.get() + cap},
+                     {(u64)nseg * G * 2, (u64)cap * MOM_LANES, cap, cap}, {0, 0, ~0ull, 0}, 4};
+      launch_fill_multi(fr, S);
+    } else {
+      SV_CUDA(cudaMemsetAsync(D.get(), 0, (size_t)nseg * G * 16, S));
+    }
     if (nin) {
       DBuf<u64> tile_range(c);
       DBuf<u32> tile_items(c);
@@ -950,7 +963,6 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     // Part moments.  One rank: the part count stays on the device (buffers sized by the bound
     // nseg * tstride), the results are packed into mapped host memory and the round costs ONE
     // host synchronisation.  Several ranks: the all-reduces need the part count on the host.
-    u32 cap = nseg * tstride;
     if (c->comm) {
       std::vector<u32> h_np;
       SV_TRY(d2h(c, h_np, d_off.get() + nseg, 1));
@@ -959,13 +971,14 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       hc.mark("vs");
       cap = std::max<u32>(1, h_np[0]);
     }
-    DBuf<u64> pl(c), pm(c), pab(c);
-    SV_TRY(pl.alloc((size_t)cap * MOM_LANES));
-    SV_TRY(pm.alloc((size_t)cap * 2));
-    SV_TRY(pab.alloc((size_t)cap * 4));
-    SV_CUDA(cudaMemsetAsync(pl.get(), 0, (size_t)cap * MOM_LANES * 8, S));
-    launch_fill_u64(pm.get(), cap, ~0ull, S);
-    SV_CUDA(cudaMemsetAsync(pm.get() + cap, 0, (size_t)cap * 8, S));
+    if (c->comm) {
+      SV_TRY(pl.alloc((size_t)cap * MOM_LANES));
+      SV_TRY(pm.alloc((size_t)cap * 2));
+      SV_TRY(pab.alloc((size_t)cap * 4));
+      SV_CUDA(cudaMemsetAsync(pl.get(), 0, (size_t)cap * MOM_LANES * 8, S));
+      launch_fill_u64(pm.get(), cap, ~0ull, S);
+      SV_CUDA(cudaMemsetAsync(pm.get() + cap, 0, (size_t)cap * 8, S));
+    }
     DBuf<u32> pitems(c);
     DBuf<char> ptemp(c);
     SV_TRY(pitems.alloc(cap + 1));
@@ -1040,9 +1053,21 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   keys.release();
 
   // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
-  std::sort(fin.begin(), fin.end(), [](const Fin& a, const Fin& b) {
-    return a.kid != b.kid ? a.kid < b.kid : a.lo < b.lo;
-  });
+  {  // counting sort by kernel, then by lo inside each kernel's (short) run: O(#strata + K)
+    std::vector<u32> cnt(K + 1, 0);
+    for (const Fin& f : fin) cnt[f.kid + 1]++;
+    for (u32 k = 0; k < K; k++) cnt[k + 1] += cnt[k];
+    std::vector<Fin> by(fin.size());
+    {
+      std::vector<u32> pos(cnt.begin(), cnt.end() - 1);
+      for (const Fin& f : fin) by[pos[f.kid]++] = f;
+    }
+    for (u32 k = 0; k < K; k++)
+      if (cnt[k + 1] - cnt[k] > 1)
+        std::sort(by.begin() + cnt[k], by.begin() + cnt[k + 1],
+                  [](const Fin& a, const Fin& b) { return a.lo < b.lo; });
+    fin.swap(by);
+  }
   const u32 ns = (u32)fin.size();
   std::vector<KTab> ktab(K, KTab{0, 0, 0, 0});
   std::vector<u64> lows;

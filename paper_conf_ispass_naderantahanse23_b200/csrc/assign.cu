@@ -305,6 +305,17 @@ __global__ void k_fill_u64(u64* p, u64 n, u64 v) {
 void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s) {
   if (n) SV_LAUNCH(k_fill_u64, min(div_up(n, 256), 4096u), 256, 0, s)(p, n, v);
 }
+// several fills in one launch (FILL_MAX regions): per-round buffer initialisation
+__global__ void k_fill_multi(FillRegions r) {
+  for (int q = 0; q < r.k; q++)
+    for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < r.n[q]; i += (u64)gridDim.x * blockDim.x)
+      r.p[q][i] = r.v[q];
+}
+void launch_fill_multi(const FillRegions& r, cudaStream_t s) {
+  u64 mx = 0;
+  for (int q = 0; q < r.k; q++) mx = r.n[q] > mx ? r.n[q] : mx;
+  if (mx) SV_LAUNCH(k_fill_multi, min(div_up(mx, 256), 4096u), 256, 0, s)(r);
+}
 
 __global__ void k_u128_to_limbs(const u64* src, u64 n, u64* limbs) {
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;

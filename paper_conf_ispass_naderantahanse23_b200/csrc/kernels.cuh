@@ -207,6 +207,9 @@ void launch_dp_gather(const u32* kstart, const u32* count, const u64* off, const
 
 // ---------------- misc -------------------------------------------------------------------------
 void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s);
+#define FILL_MAX 4
+struct FillRegions { u64* p[FILL_MAX]; u64 n[FILL_MAX]; u64 v[FILL_MAX]; int k; };
+void launch_fill_multi(const FillRegions& r, cudaStream_t s);
 // SM-driven copy (device or pinned host memory on either side; no copy engine)
 void launch_copy(void* dst, const void* src, u64 bytes, cudaStream_t s);
 // cross-rank encoding of u128 pairs [n][2] <-> 4 limbs [n][4]

@@ -15,7 +15,7 @@ template <int V>
 __device__ __forceinline__ double term(double gs, double xs, const double* sS, double L, double M, double acc,
                                        Ops o = Ops{1.0, -0.0, -C_MAGIC}) {
   double z, u, kf, kb;
-  if (V >= 2) {  // every add / mul as a DFMA with opaque register operands (same roundings)
+  if (V >= 2 && V < 7) {  // every add / mul as a DFMA with opaque register operands (same roundings)
     z = __fma_rn(xs, -o.one, gs);
     u = __fma_rn(z, z, o.nz);
     kb = __fma_rn(u, L, M);
@@ -31,7 +31,23 @@ __device__ __forceinline__ double term(double gs, double xs, const double* sS, d
   p = __fma_rn(p, r, -0.5);
   p = __fma_rn(p, r, 1.0);
   double S;
-  if (V == 0 || V == 2) {
+  if (V == 7) {  // address by ONE byte permute: the lane's replica offset lies in byte 0 and the
+                 // table at a 64 KB-aligned shared address, so no add is needed
+    u32 k = (u32)__double2loint(kb);
+    u32 a = __byte_perm(k, (u32)(size_t)sS, 0x7604u);
+    double T;
+    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(T) : "r"(a));
+    S = __hiloint2double(__double2hiint(T) - (int)(__byte_perm(k, 0u, 0x4144u) << 4), __double2loint(T));
+  } else if (V == 10) {  // full k-indexed table (10,528 entries, bank conflicts), clamp
+    u32 k = min((u32)__double2loint(kb), 10527u);
+    S = sS[k];
+  } else if (V == 8) {  // table load, no exponent adjust
+    u32 k = (u32)__double2loint(kb);
+    S = *(const double*)((const char*)sS + __byte_perm(k, 0u, 0x4404u));
+  } else if (V == 9) {  // exponent adjust on kf, no table load
+    u32 k = (u32)__double2loint(kb);
+    S = __hiloint2double(__double2hiint(kf) - (int)(__byte_perm(k, 0u, 0x4144u) << 4), __double2loint(kf));
+  } else if (V == 0 || V == 2) {
     u32 k = (u32)__double2loint(kb);
     double T = *(const double*)((const char*)sS + __byte_perm(k, 0u, 0x4404u));
     S = __hiloint2double(__double2hiint(T) - (int)(__byte_perm(k, 0u, 0x4144u) << 4), __double2loint(T));
@@ -43,9 +59,18 @@ __device__ __forceinline__ double term(double gs, double xs, const double* sS, d
 template <int V, int U>
 __global__ void __launch_bounds__(512, 1) k(double* out, int iters, double g0) {
   extern __shared__ double sS[];
-  for (int i = threadIdx.x; i < 256 * 32; i += blockDim.x) sS[i] = 0x1p40 * (1.0 - (i >> 5) * 1e-3);
+  for (int i = threadIdx.x; i < (V == 10 ? 10528 : 256 * 32); i += blockDim.x) sS[i] = 0x1p40 * (1.0 - (i >> 5) * 1e-3);
   __syncthreads();
-  const double* sSb = sS + (threadIdx.x & 31);
+  const double* sSb = V == 10 ? sS : sS + (threadIdx.x & 31);
+  if (V == 7) {  // table copy at the first 64 KB-aligned shared address inside the dynamic block
+    const u32 b0 = (u32)__cvta_generic_to_shared(sS);
+    const u32 tb = (b0 + 0xFFFFu) & ~0xFFFFu;
+    double* tab = sS + (tb - b0) / 8;
+    for (int i = threadIdx.x; i < 256 * 32; i += blockDim.x) tab[i] = 0x1p40 * (1.0 - (i >> 5) * 1e-3);
+    __syncthreads();
+    sSb = (const double*)(size_t)(tb + 8 * (threadIdx.x & 31));
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0 && iters < 20) printf("dynamic smem shared offset 0x%x\n", (u32)__cvta_generic_to_shared(sS));
   double L, M;
   asm volatile("mov.b64 %0, %1;" : "=d"(L) : "d"(c_kde[0]));
   asm volatile("mov.b64 %0, %1;" : "=d"(M) : "d"(C_MAGIC));
@@ -56,7 +81,7 @@ __global__ void __launch_bounds__(512, 1) k(double* out, int iters, double g0) {
   asm volatile("mov.b64 %0, %1;" : "=d"(o.one) : "d"(g_one));
   asm volatile("mov.b64 %0, %1;" : "=d"(o.nz) : "d"(g_nz));
   asm volatile("mov.b64 %0, %1;" : "=d"(o.nmagic) : "d"(g_nmagic));
-  if (V >= 4) {  // raw pipe tests: 9 independent chains of one op kind
+  if (V >= 4 && V < 7) {  // raw pipe tests: 9 independent chains of one op kind
     double a[U];
     for (int q = 0; q < U; q++) a[q] = gs + q;
     for (int it = 0; it < iters; it++)
@@ -78,10 +103,11 @@ __global__ void __launch_bounds__(512, 1) k(double* out, int iters, double g0) {
 template <int V, int U>
 void run(const char* name, double* d, int iters) {
   cudaEvent_t a, b; cudaEventCreate(&a); cudaEventCreate(&b);
-  cudaFuncSetAttribute(k<V, U>, cudaFuncAttributeMaxDynamicSharedMemorySize, 65536);
-  k<V, U><<<148, 512, 65536>>>(d, 10, 1.0);
+  const int sm = V == 7 ? 0x20000 : V == 10 ? 10528 * 8 : 65536;
+  cudaFuncSetAttribute(k<V, U>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+  k<V, U><<<148, 512, sm>>>(d, 10, 1.0);
   cudaEventRecord(a);
-  k<V, U><<<148, 512, 65536>>>(d, iters, 1.0);
+  k<V, U><<<148, 512, sm>>>(d, iters, 1.0);
   cudaEventRecord(b); cudaEventSynchronize(b);
   float ms; cudaEventElapsedTime(&ms, a, b);
   double ops = 148.0 * 512 * iters * U * 9;
@@ -92,6 +118,10 @@ void run(const char* name, double* d, int iters) {
 int main() {
   double* d; cudaMalloc(&d, 148 * 512 * 8);
   run<0, 16>("term+table u16", d, 4000);
+  run<7, 16>("term+table 1-PRMT addr", d, 4000);
+  run<8, 16>("table load, no exp adj", d, 4000);
+  run<10, 16>("full k table (conflicts)", d, 4000);
+  run<9, 16>("exp adj, no table load", d, 4000);
   run<1, 16>("term no-table u16", d, 4000);
   run<2, 16>("all-DFMA term+table", d, 4000);
   run<3, 16>("all-DFMA no-table", d, 4000);
