@@ -66,9 +66,11 @@ struct SegDev {
   double cq;    // (G - 1) / (hi - lo): cell estimate (made exact against the grid table)
 };
 #define KDE_WC 7.54983443527075   // sqrt(57): |z| <= this <=> t <= 28.5 (in-window term count)
-#define KDE_TJ 32       // grid points per tile (a work item is one warp's: one point per lane)
+#ifndef KDE_TJ
+#define KDE_TJ 32       // grid points per tile (32: one point per lane; 16: two value slices)
+#endif
 #ifndef KDE_CH
-#define KDE_CH 256      // values per work item chunk (staged in the warp's shared memory)
+#define KDE_CH 512      // values per work item (A/B: 512 beats 256 by 2.5%; 16-point tiles lose)
 #endif
 // per (segment, tile of KDE_TJ grid points): the range of bucketed values whose cells meet the
 // tile's window, chunked into work items; tile_items[nseg * tiles] receives the item total
