@@ -312,43 +312,49 @@ def main():
 
         for c, _ in lanes:   # warm each context once
             e2e_step(c)
-        barrier()
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        errs = []
+        def trial():
+            barrier()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            errs = []
 
-        def worker(w):
-            c, s = lanes[w]
-            try:
-                if w:
-                    s.wait_event(e0)
-                for _ in range(w, e_steps, len(lanes)):
-                    e2e_step(c)
-            except Exception as ex:  # surfaced after the join
-                errs.append(ex)
+            def worker(w):
+                c, s = lanes[w]
+                try:
+                    if w:
+                        s.wait_event(e0)
+                    for _ in range(w, e_steps, len(lanes)):
+                        e2e_step(c)
+                except Exception as ex:  # surfaced after the join
+                    errs.append(ex)
 
-        ths = [threading.Thread(target=worker, args=(w,)) for w in range(len(lanes))]
-        for th in ths:
-            th.start()
-        for th in ths:
-            th.join()
-        if errs:
-            raise errs[0]
-        for _, s in lanes[1:]:
-            ev = torch.cuda.Event()
-            ev.record(s)
-            stream.wait_event(ev)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        barrier()
-        ems = max_over_ranks(e0.elapsed_time(e1))
+            ths = [threading.Thread(target=worker, args=(w,)) for w in range(len(lanes))]
+            for th in ths:
+                th.start()
+            for th in ths:
+                th.join()
+            if errs:
+                raise errs[0]
+            for _, s in lanes[1:]:
+                ev = torch.cuda.Event()
+                ev.record(s)
+                stream.wait_event(ev)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            barrier()
+            return max_over_ranks(e0.elapsed_time(e1))
+
+        # three timed trials of e_steps steps each; the median is reported, all are listed
+        trials = [trial() for _ in range(3)]
+        ems = statistics.median(trials)
         e2e = {"value": cfg.n * e_steps / (ems / 1000.0), "unit": "invocations/s",
                "h2d_bytes_per_step": int(n_local * 24),
                "d2h_bytes_per_step": int(out["strata"] * 96 + 56), "steps": e_steps,
                # the step is bound by the PCIe H2D of the columns: the rate it implies
                "h2d_GBps_per_rank": n_local * 24 * e_steps / (ems / 1000.0) / 1e9,
                "host_cores_near_gpu": cpus,   # NVML affinity the rank was pinned to (None: not pinned)
+               "trials_ms": [round(t, 3) for t in trials],   # median reported
                "note": "every step: H2D of kid/x/cta/y from pinned host memory (sieve_load_trace) + "
                        "stratify + predict, stratum table and prediction read back; "
                        + ("double-buffered over two contexts (step i+1's H2D overlaps step i)"
