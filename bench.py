@@ -345,7 +345,10 @@ def main():
             barrier()
             return max_over_ranks(e0.elapsed_time(e1))
 
-        # three timed trials of e_steps steps each; the median is reported, all are listed
+        # one untimed pipelined trial first (both contexts' traces and arenas alive together for the
+        # first time: the memory pools grow here), then three timed trials of e_steps steps each;
+        # the median is reported, all are listed
+        trial()
         trials = [trial() for _ in range(3)]
         ems = statistics.median(trials)
         e2e = {"value": cfg.n * e_steps / (ems / 1000.0), "unit": "invocations/s",
