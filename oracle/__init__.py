@@ -69,6 +69,8 @@ def _lib():
         L.oracle_tier.restype = ctypes.c_int
         L.oracle_bandwidth.argtypes = [u64, u64, u64, u64, u64, dbl]
         L.oracle_bandwidth.restype = dbl
+        L.oracle_u256_to_double.argtypes = [vp]
+        L.oracle_u256_to_double.restype = dbl
         L.oracle_grid_point.argtypes = [u64, u64, u32, u32]
         L.oracle_grid_point.restype = dbl
         L.oracle_kde.argtypes = [vp, u64, u64, u64, dbl, u32, vp, vp]
@@ -235,6 +237,24 @@ def bandwidth(values, bw_scale=1.06):
     a, b = _split(s1)
     c, d = _split(s2)
     return _lib().oracle_bandwidth(n, a, b, c, d, bw_scale)
+
+
+def tier_moments(n, s1, s2, lo, hi, theta=(2, 5)):
+    """O3 on explicit exact moments (n, S1, S2 as Python ints) -- the wide-regime pin hook."""
+    a, b = _split(s1)
+    c, d = _split(s2)
+    return _lib().oracle_tier(n, a, b, c, d, lo, hi, theta[0], theta[1])
+
+
+def bandwidth_moments(n, s1, s2, bw_scale=1.06):
+    a, b = _split(s1)
+    c, d = _split(s2)
+    return _lib().oracle_bandwidth(n, a, b, c, d, bw_scale)
+
+
+def u256_to_double(v):
+    w = np.array([(int(v) >> (64 * i)) & ((1 << 64) - 1) for i in range(4)], np.uint64)
+    return _lib().oracle_u256_to_double(_p(w))
 
 
 def grid_point(lo, hi, j, G):

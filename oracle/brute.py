@@ -86,8 +86,10 @@ def cov_below(vals, theta):
 
 def bandwidth(vals, bw_scale):
     n = len(vals)
-    s1 = sum(vals)
-    s2 = sum(v * v for v in vals)
+    return bandwidth_from_moments(n, sum(vals), sum(v * v for v in vals), bw_scale)
+
+
+def bandwidth_from_moments(n, s1, s2, bw_scale):
     num = n * s2 - s1 * s1                # exact integer
     var = float(num) / (float(n) * float(n))   # float(int) is correctly rounded
     h_raw = (bw_scale * math.sqrt(var)) * math.pow(float(n), -0.2)
@@ -128,7 +130,8 @@ def valley_cuts(D, shift):
 
 
 def stratify(kid, x, K, cta=None, cycles=None, theta=Fraction(2, 5), G=64, shift=10,
-             bw_scale=1.06, max_rounds=64):
+             bw_scale=1.06, max_rounds=64, split_kinds=None):
+    """split_kinds: optional list that receives 1 (valley) or 2 (bisection) per KDE segment"""
     n = len(kid)
     kid = [int(k) for k in kid]
     x = [int(v) for v in x]
@@ -159,6 +162,8 @@ def stratify(kid, x, K, cta=None, cycles=None, theta=Fraction(2, 5), G=64, shift
                 gs = grid(lo, hi, G)
                 T = sorted({math.ceil(gs[m]) for m in valley_cuts(D, shift)})
                 T = [t for t in T if lo < t <= hi]
+                if split_kinds is not None:
+                    split_kinds.append(1 if T else 2)
                 if not T:
                     T = [(lo + hi + 1) // 2]
                 bounds = [0] + T + [1 << 64]

@@ -30,7 +30,10 @@
  * Q vs e^{-t} 2^40 (<= 1 unit), KDE vs scikit-learn / scipy / direct sums,
  * hand-built valley sequences, symmetric two-point masses, strata invariants,
  * representative brute force, prediction identities (homogeneous cycles => error 0,
- * CPI arithmetic-mean form), and an independent Python big-int brute force (oracle/brute.py).
+ * CPI arithmetic-mean form), an independent Python big-int brute force (oracle/brute.py), and
+ * the wide regime (tests/test_oracle_wide.py): u256 -> double vs Python float(int), tiers at
+ * n S2 >= 2^128 vs the CoV definition in Fractions, h vs Scott's closed form, D_j >= 2^63, the
+ * bisection fallback on a unimodal density.
  *
  * Build: gcc -O2 -std=c11 -ffp-contract=off -fPIC -shared (no -ffast-math: every
  * floating-point step must be the IEEE basic operation written here).
@@ -135,6 +138,12 @@ static double u256_to_double(u256 a) {
   for (int b = 0; b < s; b++)
     if ((a.w[b / 64] >> (b % 64)) & 1u) { sticky = 1; break; }
   return ldexp((double)(t | sticky), s); /* >= 11 dropped bits, so the sticky LSB is exact */
+}
+
+/* test hook (pinned against Python's correctly rounded float(int)): w = 4 little-endian limbs */
+double oracle_u256_to_double(const uint64_t* w) {
+  u256 a = {{w[0], w[1], w[2], w[3]}};
+  return u256_to_double(a);
 }
 
 /* ------------------------------------------------------------------------------------------

@@ -1,0 +1,70 @@
+"""Workload for compute-sanitizer (memcheck / racecheck / synccheck): C1 and a 200k-invocation
+slice of C2 through sieve_stratify + sieve_predict (keep_debug on, so every KDE segment is read
+back), plus C1 over an in-process 2-rank group (the multi-rank reduction kernels).
+
+    compute-sanitizer --tool racecheck python tools/sanitize_run.py [--no-group]
+"""
+import os
+import sys
+import threading
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import gen  # noqa: E402
+import paper_conf_ispass_naderantahanse23_b200 as sieve  # noqa: E402
+from paper_conf_ispass_naderantahanse23_b200.distributed import shard_bounds  # noqa: E402
+
+
+def one(tr, n=None, G=1024):
+    n = len(tr["kid"]) if n is None else n
+    ctx = sieve.Ctx(device=0)
+    t = sieve.load_trace(ctx, tr["kid"][:n], tr["x"][:n], num_kernels=tr["K"], cta=tr["cta"][:n],
+                         cycles=tr["y"][:n])
+    sid = torch.empty(n, dtype=torch.int32, device="cuda")
+    st = sieve.stratify(t, stratum_of_invocation=sid, grid_points=G, keep_debug=1)
+    segs = st.segments(G)
+    p = sieve.predict(st, t)
+    torch.cuda.synchronize()
+    print(f"n={n} strata={len(st.table)} rounds={st.rounds} segments={len(segs)} "
+          f"pred={p['predicted_cycles']:.6g}", flush=True)
+
+
+def group(tr, world=2):
+    grp = sieve.Group(world)
+    n = len(tr["kid"])
+    errs = []
+
+    def rank_main(r):
+        try:
+            torch.cuda.set_device(0)
+            s = torch.cuda.Stream()
+            ctx = sieve.Ctx(device=0, stream=s, rank=r, group=grp)
+            first, cnt = shard_bounds(n, world, r)
+            sl = slice(first, first + cnt)
+            t = sieve.load_trace(ctx, tr["kid"][sl], tr["x"][sl], num_kernels=tr["K"],
+                                 cta=tr["cta"][sl], cycles=tr["y"][sl], first_id=first)
+            st = sieve.stratify(t)
+            sieve.predict(st, t)
+            s.synchronize()
+        except Exception as e:  # reported below
+            errs.append((r, repr(e)))
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join()
+    assert not errs, errs
+    print(f"group world={world} ok", flush=True)
+
+
+if __name__ == "__main__":
+    one(gen.make_trace("C1"))
+    one(gen.make_trace("C2"), n=200_000)
+    if "--no-group" not in sys.argv:
+        group(gen.make_trace("C1"))
+    print("sanitize workload done")
