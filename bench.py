@@ -44,7 +44,112 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=1_000_000)
+    ap.add_argument("--no-ncu-traffic", action="store_true",
+                    help="skip the ncu DRAM-traffic capture that runs before the timed steps")
+    ap.add_argument("--ncu-child", action="store_true", help=argparse.SUPPRESS)
     return ap.parse_args()
+
+
+def host_info():
+    """the host the CPU oracle ran on: model name and core count (cpu_baseline)"""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count(),
+            "affinity_cores": len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else None}
+
+
+# kernels whose DRAM traffic bench reports (ncu capture before the timed steps), with the
+# algorithmic bytes the method needs per unit (DESIGN.md 5): per invocation for the streaming
+# passes over the trace, per launch for the KDE (its work unit is the term, not bytes)
+TRAFFIC_KERNELS = {
+    "k_kde": None,
+    "k_moments": 20,          # kid 4 + x 8 + y 8 (pass A)
+    "k_assign": 20,           # kid 4 + x 8 + cta 4 in, sid 4 out (pass B)
+    "k_t3_compact": 12,       # kid 4 + x 8 in (+ 8 B per Tier-3 key out, reported separately)
+}
+
+
+def ncu_traffic(args, n):
+    """DRAM bytes of the dominant and the streaming kernels, measured by ncu on one stratify step
+    of the same workload in a child process (before this process touches the GPU, so the two do
+    not share it).  Numbers under the profiler are traffic only, never timing."""
+    import shutil
+    import tempfile
+    ncu = shutil.which("ncu") or ("/usr/local/cuda/bin/ncu" if os.path.exists("/usr/local/cuda/bin/ncu") else None)
+    if ncu is None:
+        return {"unavailable": "ncu not found"}
+    log = tempfile.NamedTemporaryFile(prefix="sieve_ncu_", suffix=".csv", delete=False).name
+    regex = "regex:^(" + "|".join(TRAFFIC_KERNELS) + ")$"
+    cmd = [ncu, "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum", "--kernel-name-base", "function",
+           "--kernel-name", regex, "--csv", "--log-file", log, sys.executable, os.path.abspath(__file__),
+           "--ncu-child", "--config", args.config, "--steps", "1", "--warmup", "0"]
+    try:
+        r = subprocess.run(cmd, stdout=subprocess.DEVNULL, stderr=subprocess.PIPE, timeout=300, text=True)
+    except (subprocess.TimeoutExpired, OSError) as e:
+        return {"unavailable": f"ncu capture failed: {type(e).__name__}"}
+    import csv
+    per = {}
+    try:
+        with open(log) as f:
+            rows = [row for row in csv.reader(f) if len(row) > 10]
+        hdr = rows[0]
+        ki, mi, vi, ui = hdr.index("Kernel Name"), hdr.index("Metric Name"), hdr.index("Metric Value"), hdr.index("Metric Unit")
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9}
+        ids = hdr.index("ID")
+        launches = {}
+        for row in rows[1:]:
+            name = row[ki].split("(")[0].split("<")[0].strip()
+            if name.startswith("void "):
+                name = name[5:]
+            v = float(row[vi].replace(",", "")) * scale.get(row[ui], 1)
+            e = per.setdefault(name, {"dram_bytes": 0.0})
+            e["dram_bytes"] += v
+            launches.setdefault(name, set()).add(row[ids])
+        for name, e in per.items():
+            e["launches"] = len(launches[name])
+            e["dram_bytes_per_launch"] = e["dram_bytes"] / e["launches"]
+            alg = TRAFFIC_KERNELS.get(name)
+            if alg:
+                e["B_per_inv"] = e["dram_bytes"] / n
+                e["algorithmic_B_per_inv"] = alg
+    except (OSError, ValueError, IndexError) as e:
+        return {"unavailable": f"ncu output unreadable: {type(e).__name__} ({r.stderr[-200:] if r.stderr else ''})"}
+    finally:
+        try:
+            os.unlink(log)
+        except OSError:
+            pass
+    if not per:
+        return {"unavailable": "ncu captured no kernel (" + (r.stderr or "").strip()[-200:] + ")"}
+    return {"by_kernel": per, "how": "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum, one stratify "
+                                      "step of the same workload in a child process before the timed steps"}
+
+
+def run_ncu_child(args):
+    """the workload ncu_traffic() profiles: one stratify of the bench trace (device-resident)"""
+    import numpy as np
+    import torch
+    import gen
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    cfg = gen.get_config(args.config)
+    g = gen.Generator(cfg)
+    tr = g.fill(0, cfg.n)
+    d = {k: torch.from_numpy(tr[k].view(np.int64 if tr[k].dtype == np.uint64 else np.int32)).cuda()
+         for k in ("kid", "x", "cta", "y")}
+    ctx = sieve.Ctx(device=0)
+    t = sieve.load_trace(ctx, d["kid"], d["x"], num_kernels=cfg.K, cta=d["cta"], cycles=d["y"], adopt=True)
+    sid = torch.empty(cfg.n, dtype=torch.int32, device="cuda")
+    ctx.set_term_count(False)
+    st = sieve.stratify(t, stratum_of_invocation=sid)
+    sieve.predict(st, t)
+    torch.cuda.synchronize()
 
 
 def measured_peaks():
@@ -154,7 +259,7 @@ def run_reference(args):
             "vs_baseline": None, "dtype": "u64/u128 + f64", "data": "synthetic",
             "config": {"workload": cfg.name, "invocations": cfg.n, "kernels": cfg.K, "sample": per_step},
             "cpu_baseline": {"value": value, "unit": "invocations/s", "cores": 1, "kind": "oracle",
-                             "sample": sample},
+                             "sample": sample, "host": host_info()},
             "e2e": {"value": value, "unit": "invocations/s", "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -184,6 +289,14 @@ def main():
     args = parse()
     if args.impl == "reference":
         return run_reference(args)
+    if args.ncu_child:
+        return run_ncu_child(args)
+    rank0 = int(os.environ.get("RANK", "0")) == 0
+    world0 = int(os.environ.get("WORLD_SIZE", "1"))
+    traffic = None
+    if rank0 and world0 == 1 and not args.no_ncu_traffic:
+        import gen as _gen
+        traffic = ncu_traffic(args, _gen.get_config(args.config).n)
     import numpy as np
     import torch
     import torch.distributed as dist
@@ -266,8 +379,12 @@ def main():
     torch.cuda.synchronize()
     clk.mark("t0")
     ev0.record(stream)
+    marks = []   # per-step boundaries on the same stream (recording an event never synchronises)
     for _ in range(args.steps):
         st = step()
+        e = torch.cuda.Event(enable_timing=True)
+        e.record(stream)
+        marks.append(e)
     ev1.record(stream)
     torch.cuda.synchronize()
     barrier()
@@ -275,6 +392,7 @@ def main():
     launches = sieve.kernel_launches() - launches0
     ms = ev0.elapsed_time(ev1)
     ms_max = max_over_ranks(ms)
+    per_step = [ev0.elapsed_time(marks[0])] + [marks[i - 1].elapsed_time(marks[i]) for i in range(1, len(marks))]
     phases = ctx.timing()
     ctx.set_timing(False)
     value = cfg.n * args.steps / (ms_max / 1000.0)
@@ -378,14 +496,12 @@ def main():
     roof = None
     if kde_ms > 0:
         achieved = KDE_FP64_OPS_PER_TERM * kde_terms / (kde_ms / 1000.0) / 1e12
-        traffic = None
-        tp = os.path.join(ROOT, "profiles", "kde_traffic.json")
-        if os.path.exists(tp):
-            with open(tp) as f:
-                traffic = json.load(f).get("dram_bytes_per_launch")
+        kde_traffic = None
+        if traffic and "by_kernel" in traffic and "k_kde" in traffic["by_kernel"]:
+            kde_traffic = traffic["by_kernel"]["k_kde"]["dram_bytes_per_launch"]
         roof = {"kernel": "k_kde (fixed-point Gaussian KDE)", "bound": "alu", "achieved": achieved,
                 "peak": fp64_peak, "unit": "Top/s (FP64-pipe instructions)", "frac": achieved / fp64_peak,
-                "traffic": traffic, "share_of_step": kde_ms / ms,
+                "traffic": kde_traffic, "share_of_step": kde_ms / ms,
                 "peak_source": f"{nsm} SMs x {FP64_LANES_PER_SM} FP64 lanes x sm_max_mhz "
                                f"{peaks.get('sm_max_mhz')} ({peak_src} MEASURED_PEAKS.json)",
                 "work": f"{kde_terms / args.steps:.4g} in-window terms/step x {KDE_FP64_OPS_PER_TERM} FP64 ops",
@@ -403,10 +519,11 @@ def main():
         rate, dt = cpu_oracle_rate(cfg, args.cpu_sample)
         cpu = {"value": rate, "unit": "invocations/s", "cores": 1, "kind": "oracle",
                "sample": f"first {args.cpu_sample} invocations of {cfg.name} (same generator), "
-                         f"{dt:.1f} s single-threaded"}
+                         f"{dt:.1f} s single-threaded", "host": host_info()}
     line = {"metric": "kernel invocations stratified/sec", "value": value, "unit": "invocations/s",
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "strong",
+            "ms_per_step_median": statistics.median(per_step), "ms_per_step_min": min(per_step),
             "vs_baseline": None, "dtype": "u64/u128 + f64", "data": "synthetic",
             "config": {"workload": cfg.name, "invocations": cfg.n, "kernels": cfg.K,
                        "grid_points": 1024, "theta": "2/5", "strata": n_strata, "rounds": rounds,
@@ -416,7 +533,7 @@ def main():
                               f"inputs ({cfg.n * 24 / 1e6:.3g} MB) fit in L2 and L2 is not flushed: "
                               "not a valid bench configuration, parity / smoke use only")},
             "clocks": clocks, "e2e": e2e, "gpu_launches": launches,
-            "roofline": roof, "phases": phase_out,
+            "roofline": roof, "phases": phase_out, "dram_traffic": traffic,
             "host_ms_per_step": {k: statistics.mean(v) for k, v in host_ms.items() if v},
             "cpu_baseline": cpu}
     print(json.dumps(line), flush=True)

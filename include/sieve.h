@@ -89,6 +89,13 @@ void sieve_group_destroy(sieve_group g);
 int sieve_ctx_create_in_group(int cuda_device, void* cuda_stream, sieve_group g, int rank,
                               sieve_ctx* out);
 
+/* Device-memory hooks (e.g. PyTorch's caching allocator); alloc and free are both set or both
+   NULL (NULL restores cudaMallocAsync / cudaFreeAsync on the ctx stream).  Every buffer is
+   released through the allocator that made it: a trace's owned columns keep their allocator
+   until sieve_trace_free, and the context's scratch arena is returned to its allocator by this
+   call (the next call grows a new arena from the new hooks).  The hooks must stay callable until
+   every buffer they made is freed.  Not to be called while another call on ctx runs.
+   Errors: EINVAL (bad ctx, only one hook given), ECUDA. */
 int sieve_ctx_set_allocator(sieve_ctx ctx, sieve_alloc_fn alloc, sieve_free_fn free_fn, void* user);
 void sieve_ctx_destroy(sieve_ctx ctx);
 
@@ -212,7 +219,7 @@ typedef struct {
 } sieve_segment;
 
 int sieve_segment_count(sieve_strata s, uint64_t* n);
-/* density_lo/hi: nullable HOST arrays [G]: D_j as u128 = hi:lo (fixed point 2^-52);
+/* density_lo/hi: nullable HOST arrays [G]: D_j as u128 = hi:lo (fixed point 2^-40, A10);
    cuts: nullable HOST array [n_cuts]: integer thresholds (x < T left, x >= T right; A12) */
 int sieve_segment_get(sieve_strata s, uint64_t idx, sieve_segment* out, uint64_t* density_lo,
                       uint64_t* density_hi, uint64_t* cuts);

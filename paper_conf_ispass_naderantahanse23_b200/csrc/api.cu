@@ -93,6 +93,13 @@ extern "C" void sieve_limbs_to_u128(const uint64_t limbs[4], uint64_t* lo, uint6
 struct PhaseAcc { double ms = 0; u64 calls = 0; u64 work = 0; };
 struct PendingEv { int ph; cudaEvent_t a, b; };
 
+// the allocator a device buffer came from: it is always released through the same one, even
+// after sieve_ctx_set_allocator changed the context's hooks
+struct Owner {
+  sieve_free_fn ff = nullptr;  // nullptr: cudaMallocAsync / cudaFreeAsync
+  void* user = nullptr;
+};
+
 struct sieve_ctx_s {
   uint32_t magic = CTX_MAGIC;
   int device = 0;
@@ -112,8 +119,9 @@ struct sieve_ctx_s {
   // gets the overflow from the allocator and the arena grows to the high-water mark, so
   // steady-state calls never touch the allocator (no pool remapping, no fragmentation).
   char* arena = nullptr;
+  Owner arena_owner;
   size_t arena_cap = 0, arena_off = 0, arena_hw = 0;
-  std::vector<void*> overflow;
+  std::vector<std::pair<void*, Owner>> overflow;
   // the same scheme in pinned host memory for the orchestrator's staged copies
   char* pin = nullptr;
   size_t pin_cap = 0, pin_off = 0, pin_hw = 0;
@@ -205,6 +213,7 @@ struct sieve_trace_s {
   u32* cta = nullptr;
   u64* y = nullptr;
   bool owned = true;
+  Owner owner;                     // allocator of the owned columns
   std::vector<std::string> names;  // kernel names by id (traces loaded from CSV)
 };
 
@@ -242,9 +251,10 @@ static int dalloc(sieve_ctx c, void** p, size_t bytes) {
   SV_CUDA(cudaMallocAsync(p, bytes, c->stream));
   return SIEVE_OK;
 }
-static void dfree(sieve_ctx c, void* p) {
+static Owner cur_owner(sieve_ctx c) { return Owner{c->ff, c->user}; }
+static void dfree(sieve_ctx c, const Owner& o, void* p) {
   if (!p) return;
-  if (c->ff) c->ff(p, (void*)c->stream, c->user);
+  if (o.ff) o.ff(p, (void*)c->stream, o.user);
   else cudaFreeAsync(p, c->stream);
 }
 
@@ -298,16 +308,17 @@ static int arena_reset(sieve_ctx c) {
   }
   c->pin_off = 0;
   c->pin_hw = 0;
-  for (void* p : c->overflow) dfree(c, p);
+  for (auto& q : c->overflow) dfree(c, q.second, q.first);
   c->overflow.clear();
   if (c->arena_hw > c->arena_cap) {
-    if (c->arena) dfree(c, c->arena);
+    if (c->arena) dfree(c, c->arena_owner, c->arena);
     c->arena = nullptr;
     c->arena_cap = 0;
     size_t want = c->arena_hw + c->arena_hw / 8;
     void* p;
     SV_TRY(dalloc(c, &p, want));
     c->arena = (char*)p;
+    c->arena_owner = cur_owner(c);
     c->arena_cap = want;
   }
   c->arena_off = 0;
@@ -323,7 +334,7 @@ static int arena_alloc(sieve_ctx c, void** p, size_t bytes) {
   if (c->arena_off > c->arena_hw) c->arena_hw = c->arena_off;
   if (c->arena_off <= c->arena_cap) { *p = c->arena + off; return SIEVE_OK; }
   SV_TRY(dalloc(c, p, bytes));  // overflow this call; the arena grows at the next reset
-  c->overflow.push_back(*p);
+  c->overflow.push_back({*p, cur_owner(c)});
   return SIEVE_OK;
 }
 
@@ -405,6 +416,17 @@ extern "C" int sieve_ctx_create_in_group(int cuda_device, void* cuda_stream, sie
 
 extern "C" int sieve_ctx_set_allocator(sieve_ctx ctx, sieve_alloc_fn a, sieve_free_fn f, void* user) {
   if (!ctx_ok(ctx) || (!a) != (!f)) return sv_fail(SIEVE_EINVAL, "bad ctx or allocator pair");
+  SV_CUDA(cudaSetDevice(ctx->device));
+  // the scratch arena goes back to the allocator it came from now (no call is in flight: every
+  // call synchronises before it returns), so the next call grows a new one from the new hooks;
+  // traces keep their owner and are released through it by sieve_trace_free
+  SV_CUDA(cudaStreamSynchronize(ctx->stream));
+  for (auto& q : ctx->overflow) dfree(ctx, q.second, q.first);
+  ctx->overflow.clear();
+  if (ctx->arena) dfree(ctx, ctx->arena_owner, ctx->arena);
+  ctx->arena = nullptr;
+  ctx->arena_cap = ctx->arena_off = 0;
+  SV_CUDA(cudaStreamSynchronize(ctx->stream));
   ctx->af = a; ctx->ff = f; ctx->user = user;
   return SIEVE_OK;
 }
@@ -414,8 +436,8 @@ extern "C" void sieve_ctx_destroy(sieve_ctx ctx) {
   cudaSetDevice(ctx->device);
   for (auto& p : ctx->pending) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
   for (auto e : ctx->ev_pool) cudaEventDestroy(e);
-  for (void* p : ctx->overflow) dfree(ctx, p);
-  if (ctx->arena) dfree(ctx, ctx->arena);
+  for (auto& q : ctx->overflow) dfree(ctx, q.second, q.first);
+  if (ctx->arena) dfree(ctx, ctx->arena_owner, ctx->arena);
   cudaStreamSynchronize(ctx->stream);
   for (void* p : ctx->pin_overflow) cudaFreeHost(p);
   if (ctx->pin) cudaFreeHost(ctx->pin);
@@ -454,6 +476,7 @@ extern "C" int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_
   SV_CUDA(cudaSetDevice(ctx->device));
   sieve_trace_s* t = new sieve_trace_s();
   t->ctx = ctx; t->n = n_local; t->first_id = first_id; t->K = K; t->owned = !adopt;
+  t->owner = cur_owner(ctx);
   if (adopt) {
     t->kid = (u32*)kernel_id; t->x = (u64*)instr; t->cta = (u32*)cta; t->y = (u64*)cycles;
   } else {
@@ -480,7 +503,8 @@ extern "C" void sieve_trace_free(sieve_trace t) {
   if (!t || t->magic != TRACE_MAGIC) return;
   if (t->owned && ctx_ok(t->ctx)) {
     cudaSetDevice(t->ctx->device);
-    dfree(t->ctx, t->kid); dfree(t->ctx, t->x); dfree(t->ctx, t->cta); dfree(t->ctx, t->y);
+    const Owner& o = t->owner;
+    dfree(t->ctx, o, t->kid); dfree(t->ctx, o, t->x); dfree(t->ctx, o, t->cta); dfree(t->ctx, o, t->y);
     cudaStreamSynchronize(t->ctx->stream);
   }
   t->magic = 0;
@@ -569,6 +593,11 @@ static inline u32 bitlen(u64 v) { return v ? 64 - __builtin_clzll(v) : 0; }
 static int allreduce(sieve_ctx c, u64* buf, size_t n, ReduceOp op) {
   if (!c->comm) return SIEVE_OK;
   return c->comm->allreduce(buf, n, op, c->stream);
+}
+// several all-reduces as one collective step (one NCCL group = one fused launch)
+static int allreduce_group(sieve_ctx c, std::initializer_list<ARReq> reqs) {
+  if (!c->comm) return SIEVE_OK;
+  return c->comm->allreduce_group(reqs.begin(), (int)reqs.size(), c->stream);
 }
 
 // Host <-> device copies of the orchestrator go through a per-call PINNED staging arena: a
@@ -669,8 +698,8 @@ static int moments_pass(sieve_trace t, MomentsHost* M) {
   cudaStream_t S = c->stream;
   const u32 K = t->K;
   const u64 n = t->n;
-  const int gridA = moments_grid();
   const u32 kt = (u32)moments_kt(K);
+  const int gridA = moments_grid(kt);
   DBuf<KMomPartial> part(c);
   DBuf<u64> blk_tot(c), lanes(c), mm(c), local_n(c), tot(c);
   SV_TRY(part.alloc((size_t)gridA * kt));
@@ -703,19 +732,12 @@ static int moments_pass(sieve_trace t, MomentsHost* M) {
   // AR-1: sums, then min/max (mm is interleaved min,max per kernel: reduce via a [2][K] copy)
   std::vector<u64> h_lanes, h_mm, h_tot, h_localn;
   if (c->comm) {
-    DBuf<u64> mn(c), mx(c);
-    SV_TRY(mn.alloc(K + 1));
-    SV_TRY(mx.alloc(K + 4));
-    SV_CUDA(cudaMemcpy2DAsync(mn.get(), 8, mm.get(), 16, 8, K, cudaMemcpyDeviceToDevice, S));
-    SV_CUDA(cudaMemcpy2DAsync(mx.get(), 8, mm.get() + 1, 16, 8, K, cudaMemcpyDeviceToDevice, S));
-    launch_copy(mx.get() + K, tot.get() + 4, 4 * 8, S);
-    SV_TRY(allreduce(c, lanes.get(), (size_t)K * MOM_LANES, RED_SUM));
-    SV_TRY(allreduce(c, tot.get(), 4, RED_SUM));
-    SV_TRY(allreduce(c, mn.get(), K, RED_MIN));
-    SV_TRY(allreduce(c, mx.get(), K + 4, RED_MAX));
-    SV_CUDA(cudaMemcpy2DAsync(mm.get(), 16, mn.get(), 8, 8, K, cudaMemcpyDeviceToDevice, S));
-    SV_CUDA(cudaMemcpy2DAsync(mm.get() + 1, 16, mx.get(), 8, 8, K, cudaMemcpyDeviceToDevice, S));
-    launch_copy(tot.get() + 4, mx.get() + K, 4 * 8, S);
+    // AR-1, one grouped step: SUM of the limb lanes and C_meas; MAX of (min, max) per kernel with
+    // the mins complemented (min(a, b) = ~max(~a, ~b)), max x and the error lanes
+    launch_complement(mm.get(), K, 2, S);
+    SV_TRY(allreduce_group(c, {{lanes.get(), (size_t)K * MOM_LANES, RED_SUM}, {tot.get(), 4, RED_SUM},
+                               {mm.get(), (size_t)K * 2, RED_MAX}, {tot.get() + 4, 4, RED_MAX}}));
+    launch_complement(mm.get(), K, 2, S);
     SV_TRY(d2h(c, h_lanes, lanes.get(), (size_t)K * MOM_LANES));
     SV_TRY(d2h(c, h_mm, mm.get(), (size_t)K * 2));
     SV_TRY(d2h(c, h_tot, tot.get(), 8));
@@ -901,17 +923,19 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(D.alloc((size_t)nseg * G * 2));
     // part buffers (one rank: sized by the bound nseg * tstride, see below) are initialised with
     // the densities in one launch
-    u32 cap = nseg * tstride;
+    // Part slots: a guess of PART_GUESS parts per segment (never more than the bound
+    // nseg * tstride), so neither the part moments nor their all-reduce wait for the host to learn
+    // the part count; a round with more parts than slots redoes its part moments with the exact
+    // count, which every rank reads after the round's one synchronisation (so all ranks agree).
+    u32 cap = (u32)std::min<u64>((u64)nseg * tstride, (u64)nseg * PART_GUESS + 64);
     DBuf<u64> pl(c), pm(c), pab(c);
-    if (!c->comm) {
-      SV_TRY(pl.alloc((size_t)cap * MOM_LANES));
-      SV_TRY(pm.alloc((size_t)cap * 2));
-      SV_TRY(pab.alloc((size_t)cap * 4));
+    SV_TRY(pl.alloc((size_t)cap * MOM_LANES));
+    SV_TRY(pm.alloc((size_t)cap * 2));
+    SV_TRY(pab.alloc((size_t)cap * 4));
+    {
       FillRegions fr{{D.get(), pl.get(), pm.get(), pm.get() + cap},
                      {(u64)nseg * G * 2, (u64)cap * MOM_LANES, cap, cap}, {0, 0, ~0ull, 0}, 4};
       launch_fill_multi(fr, S);
-    } else {
-      SV_CUDA(cudaMemsetAsync(D.get(), 0, (size_t)nseg * G * 16, S));
     }
     if (nin) {
       DBuf<u64> tile_range(c);
@@ -922,12 +946,15 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       SV_TRY(stemp.alloc(scan_u32_temp_bytes((u64)nseg * tps)));
       // work items are counted on the device; size the item map by a host-side bound so no
       // synchronisation is needed here: a tile has at most ceil(segment values / KDE_CH) items
-      u64 items_bound = 0;
+      u64 items_bound = 0, global_bound = 0;
       for (u32 s = 0; s < nseg; s++) {
         u64 len = round == 1 ? h_localn[op[s].kid] : op[s].e - op[s].b;
         items_bound += (u64)tps * ((len + KDE_CH - 1) / KDE_CH);
+        global_bound += (u64)tps * ((op[s].n + KDE_CH - 1) / KDE_CH);  // replicated on every rank
       }
-      if (items_bound >= (1ull << 32)) return sv_fail(SIEVE_ELIMIT, "too many KDE work items");
+      // the limit is decided on the segments' GLOBAL counts, identical on every rank, so no rank
+      // returns while the others enter AR-2 (the local bound is at most the global one)
+      if (global_bound >= (1ull << 32)) return sv_fail(SIEVE_ELIMIT, "too many KDE work items");
       u32 items = (u32)items_bound;
       kde_plan(segs.get(), nseg, G, gtab.get(), off.get(), tile_range.get(), tile_items.get(), stemp.get(), S);
       DBuf<char> item_tile(c);
@@ -939,16 +966,13 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       for (u32 s = 0; s < nseg; s++)
         if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 140.0 * hs[s].h) guard = true;
       launch_kde(segs.get(), nseg, G, ck.get(), ib, tile_range.get(), tile_items.get(),
-                 item_tile.get(), items, D.get(), terms.get() + 1, guard, S);
+                 item_tile.get(), items, D.get(), terms.get() + 1, guard, !c->comm, S);
       tm.stop();
       SV_CUDA(cudaGetLastError());
     }
-    if (c->comm) {  // AR-2: densities as 32-bit limbs
-      DBuf<u64> lim(c);
-      SV_TRY(lim.alloc((size_t)nseg * G * 4));
-      launch_u128_to_limbs(D.get(), (u64)nseg * G, lim.get(), S);
-      SV_TRY(allreduce(c, lim.get(), (size_t)nseg * G * 4, RED_SUM));
-      launch_limbs_to_u128(lim.get(), (u64)nseg * G, D.get(), S);
+    if (c->comm) {  // AR-2: the densities' two u64 lanes per grid point (16 B), then normalise
+      SV_TRY(allreduce(c, D.get(), (size_t)nseg * G * 2, RED_SUM));
+      launch_kde_fix(D.get(), (u64)nseg * G, S);
     }
     DBuf<u64> T(c);
     DBuf<u32> ntk(c), d_off(c);
@@ -960,41 +984,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
                    ntk.get() + nseg, S);
     launch_part_offsets(ntk.get(), nseg, d_off.get(), S);
     tv.stop();
-    // Part moments.  One rank: the part count stays on the device (buffers sized by the bound
-    // nseg * tstride), the results are packed into mapped host memory and the round costs ONE
-    // host synchronisation.  Several ranks: the all-reduces need the part count on the host.
-    if (c->comm) {
-      std::vector<u32> h_np;
-      SV_TRY(d2h(c, h_np, d_off.get() + nseg, 1));
-      hc.mark("v");
-      SV_TRY(sync(c));
-      hc.mark("vs");
-      cap = std::max<u32>(1, h_np[0]);
-    }
-    if (c->comm) {
-      SV_TRY(pl.alloc((size_t)cap * MOM_LANES));
-      SV_TRY(pm.alloc((size_t)cap * 2));
-      SV_TRY(pab.alloc((size_t)cap * 4));
-      SV_CUDA(cudaMemsetAsync(pl.get(), 0, (size_t)cap * MOM_LANES * 8, S));
-      launch_fill_u64(pm.get(), cap, ~0ull, S);
-      SV_CUDA(cudaMemsetAsync(pm.get() + cap, 0, (size_t)cap * 8, S));
-    }
-    DBuf<u32> pitems(c);
-    DBuf<char> ptemp(c);
-    SV_TRY(pitems.alloc(cap + 1));
-    SV_TRY(ptemp.alloc(scan_u32_temp_bytes(cap)));
-    {
-      PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
-      launch_part_stats(segs.get(), nseg, G, gtab.get(), off.get(), T.get(), tstride, ntk.get(), d_off.get(),
-                        cap, ck.get(), ib, pitems.get(), ptemp.get(), pl.get(), pm.get(), pab.get(), S);
-      SV_CUDA(cudaGetLastError());
-    }
-    SV_TRY(allreduce(c, pl.get(), (size_t)cap * MOM_LANES, RED_SUM));   // AR-3 (cap = parts here)
-    SV_TRY(allreduce(c, pm.get(), cap, RED_MIN));
-    SV_TRY(allreduce(c, pm.get() + cap, cap, RED_MAX));
-    u64 *hrec = nullptr, *drec = nullptr;
-    SV_TRY(mapped_get(c, (1 + (size_t)cap * PART_REC) * 8, &hrec, &drec));
-    launch_part_pack(d_off.get(), nseg, cap, pl.get(), pm.get(), pab.get(), drec, S);
+    // Part moments (AR-3 as one grouped step: SUM of the limb lanes, MAX of the complemented
+    // mins and of the maxes), packed into mapped host memory: ONE host synchronisation per round
+    // at any rank count.
     std::vector<u32> h_ntk;
     std::vector<u64> h_D, h_T;
     SV_TRY(d2h(c, h_ntk, ntk.get(), (size_t)nseg * 2));
@@ -1002,9 +994,39 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       SV_TRY(d2h(c, h_D, D.get(), (size_t)nseg * G * 2));
       SV_TRY(d2h(c, h_T, T.get(), (size_t)nseg * tstride));
     }
-    hc.mark("p");
-    SV_TRY(sync(c));
-    hc.mark("ps");
+    u64 *hrec = nullptr, *drec = nullptr;
+    for (int pass = 0;; pass++) {
+      DBuf<u32> pitems(c);
+      DBuf<char> ptemp(c);
+      SV_TRY(pitems.alloc(cap + 1));
+      SV_TRY(ptemp.alloc(scan_u32_temp_bytes(cap)));
+      {
+        PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
+        launch_part_stats(segs.get(), nseg, G, gtab.get(), off.get(), T.get(), tstride, ntk.get(), d_off.get(),
+                          cap, ck.get(), ib, pitems.get(), ptemp.get(), pl.get(), pm.get(), pab.get(), S);
+        SV_CUDA(cudaGetLastError());
+      }
+      if (c->comm) {
+        launch_complement(pm.get(), cap, 1, S);
+        SV_TRY(allreduce_group(c, {{pl.get(), (size_t)cap * MOM_LANES, RED_SUM}, {pm.get(), (size_t)cap * 2, RED_MAX}}));
+        launch_complement(pm.get(), cap, 1, S);
+      }
+      SV_TRY(mapped_get(c, (1 + (size_t)cap * PART_REC) * 8, &hrec, &drec));
+      launch_part_pack(d_off.get(), nseg, cap, pl.get(), pm.get(), pab.get(), drec, S);
+      hc.mark("p");
+      SV_TRY(sync(c));
+      hc.mark("ps");
+      const u64 live = hrec[0];  // replicated: every rank computed the same cuts from the same D
+      if (live <= cap) break;
+      if (pass > 0) return sv_fail(SIEVE_ESTATE, "internal: part count grew");
+      cap = (u32)live;  // more parts than slots: redo this round's part moments with the exact count
+      SV_TRY(pl.alloc((size_t)cap * MOM_LANES));
+      SV_TRY(pm.alloc((size_t)cap * 2));
+      SV_TRY(pab.alloc((size_t)cap * 4));
+      FillRegions fr{{pl.get(), pm.get(), pm.get() + cap, nullptr},
+                     {(u64)cap * MOM_LANES, cap, cap, 0}, {0, ~0ull, 0, 0}, 3};
+      launch_fill_multi(fr, S);
+    }
     std::vector<u32> part_off(nseg + 1);
     u32 nparts = 0;
     for (u32 s = 0; s < nseg; s++) { part_off[s] = nparts; nparts += h_ntk[s] + 1; }
@@ -1127,33 +1149,22 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     const u64* ak = ent.get();
     DBuf<u64> akb(c);
     if (c->comm) {
-      std::vector<unsigned long long> hcnt;
-      SV_TRY(d2h(c, hflag, errf.get(), 4));
-      SV_TRY(d2h(c, hcnt, counter.get(), 1));
-      SV_TRY(sync(c));
-      // the retry decision must be identical on every rank
-      std::vector<u64> gfl{hflag[2]};
-      DBuf<u64> fl(c);
-      SV_TRY(fl.alloc(1));
-      SV_TRY(h2d(c, fl.get(), gfl));
-      SV_TRY(allreduce(c, fl.get(), 1, RED_MAX));
-      SV_TRY(d2h(c, gfl, fl.get(), 1));
-      SV_TRY(sync(c));
-      if (gfl[0]) { cap <<= 2; continue; }
-      const u64 E = hcnt[0];
-      // gather every rank's entries (AR-4: all-gather expressed as a SUM over zero-padded slots)
-      DBuf<u64> cnts(c);
-      SV_TRY(cnts.alloc(c->world));
-      std::vector<u64> mine(c->world, 0);
-      mine[c->rank] = E;
-      SV_TRY(h2d(c, cnts.get(), mine));
-      SV_TRY(allreduce(c, cnts.get(), c->world, RED_SUM));
+      // one exchange of world + 1 lanes (SUM) and ONE synchronisation: [0] = ranks whose table
+      // overflowed (the retry decision is then identical on every rank), [1 + r] = rank r's
+      // entry count (the offsets of the all-gather below)
+      DBuf<u64> xw(c);
+      SV_TRY(xw.alloc((size_t)c->world + 1));
+      launch_exchange_prep(errf.get() + 2, counter.get(), c->comm->rank, c->world, xw.get(), S);
+      SV_TRY(allreduce(c, xw.get(), (size_t)c->world + 1, RED_SUM));
       std::vector<u64> all;
-      SV_TRY(d2h(c, all, cnts.get(), c->world));
+      SV_TRY(d2h(c, all, xw.get(), (size_t)c->world + 1));
       SV_TRY(sync(c));
+      if (all[0]) { cap <<= 2; continue; }
+      const u64 E = all[1 + c->rank];
+      // gather every rank's entries (AR-4: all-gather expressed as a SUM over zero-padded slots)
       Etot = 0;
       u64 Eoff = 0;
-      for (int r = 0; r < c->world; r++) { if (r == c->rank) Eoff = Etot; Etot += all[r]; }
+      for (int r = 0; r < c->world; r++) { if (r == c->rank) Eoff = Etot; Etot += all[1 + r]; }
       SV_TRY(akb.alloc(std::max<u64>(Etot, 1) * 3));
       SV_CUDA(cudaMemsetAsync(akb.get(), 0, Etot * 3 * 8, S));
       SV_CUDA(cudaMemcpyAsync(akb.get() + Eoff, ent.get(), E * 8, cudaMemcpyDeviceToDevice, S));
@@ -1662,6 +1673,7 @@ extern "C" int sieve_load_csv(sieve_ctx ctx, const char* data, uint64_t bytes, u
   SV_CUDA(cudaMemsetAsync(errf.get(), 0, 8, S));
   sieve_trace_s* t = new sieve_trace_s();
   t->ctx = c; t->n = nrows; t->first_id = first_id; t->owned = true;
+  t->owner = cur_owner(c);
   auto fail = [&](int st) { cudaStreamSynchronize(S); sieve_trace_free(t); return st; };
 #define CSV_TRY(e) do { int _s = (e); if (_s != SIEVE_OK) return fail(_s); } while (0)
   void* p;

@@ -331,3 +331,24 @@ void launch_u128_to_limbs(const u64* src, u64 n, u64* limbs, cudaStream_t s) {
 void launch_limbs_to_u128(const u64* limbs, u64 n, u64* dst, cudaStream_t s) {
   if (n) SV_LAUNCH(k_limbs_to_u128, div_up(n, 256), 256, 0, s)(limbs, n, dst);
 }
+
+// MIN folded into MAX for the grouped cross-rank reductions: min(a, b) = ~max(~a, ~b)
+__global__ void k_complement(u64* p, u64 n, u64 stride) {
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x)
+    p[i * stride] = ~p[i * stride];
+}
+void launch_complement(u64* p, u64 n, u64 stride, cudaStream_t s) {
+  if (n) SV_LAUNCH(k_complement, min(div_up(n, 256), 4096u), 256, 0, s)(p, n, stride);
+}
+
+// pass B's exchange word set (one SUM all-reduce of world + 1 lanes, no host round trip before
+// it): x[0] = this rank's table-overflow flag, x[1 + r] = rank r's entry count (0 elsewhere)
+__global__ void k_exchange_prep(const u64* flag, const unsigned long long* count, int rank, int world, u64* x) {
+  int i = threadIdx.x;
+  if (i == 0) x[0] = flag[0] ? 1ull : 0ull;
+  if (i < world) x[1 + i] = i == rank ? (u64)count[0] : 0ull;
+}
+void launch_exchange_prep(const u64* flag, const unsigned long long* count, int rank, int world, u64* x,
+                          cudaStream_t s) {
+  SV_LAUNCH(k_exchange_prep, 1, ((world + 31) / 32) * 32, 0, s)(flag, count, rank, world, x);
+}

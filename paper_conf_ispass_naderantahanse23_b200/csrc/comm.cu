@@ -28,6 +28,7 @@ typedef int (*fn_init_rank)(nccl_comm_t*, int, nccl_uid_t, int);
 typedef int (*fn_allreduce)(const void*, void*, size_t, int, int, nccl_comm_t, cudaStream_t);
 typedef int (*fn_destroy)(nccl_comm_t);
 typedef const char* (*fn_errstr)(int);
+typedef int (*fn_group)(void);
 
 static struct {
   void* h = nullptr;
@@ -36,6 +37,7 @@ static struct {
   fn_allreduce allreduce;
   fn_destroy destroy;
   fn_errstr errstr;
+  fn_group group_start, group_end;
 } g_nccl;
 
 static int nccl_load() {
@@ -55,7 +57,10 @@ static int nccl_load() {
   g_nccl.allreduce = (fn_allreduce)dlsym(h, "ncclAllReduce");
   g_nccl.destroy = (fn_destroy)dlsym(h, "ncclCommDestroy");
   g_nccl.errstr = (fn_errstr)dlsym(h, "ncclGetErrorString");
-  if (!g_nccl.get_uid || !g_nccl.init_rank || !g_nccl.allreduce || !g_nccl.destroy)
+  g_nccl.group_start = (fn_group)dlsym(h, "ncclGroupStart");
+  g_nccl.group_end = (fn_group)dlsym(h, "ncclGroupEnd");
+  if (!g_nccl.get_uid || !g_nccl.init_rank || !g_nccl.allreduce || !g_nccl.destroy ||
+      !g_nccl.group_start || !g_nccl.group_end)
     return sv_fail(SIEVE_ENCCL, "libnccl is missing required symbols");
   g_nccl.h = h;
   return SIEVE_OK;
@@ -80,10 +85,20 @@ struct NcclComm : Comm {
   ~NcclComm() override {
     if (c) g_nccl.destroy(c);
   }
-  int allreduce(u64* buf, size_t n, ReduceOp op, cudaStream_t s) override {
-    if (n == 0) return SIEVE_OK;
-    int nop = op == RED_SUM ? 0 : (op == RED_MAX ? 2 : 3);
-    return nccl_check(g_nccl.allreduce(buf, buf, n, 5 /* ncclUint64 */, nop, c, s), "ncclAllReduce");
+  int allreduce_group(const ARReq* reqs, int nreq, cudaStream_t s) override {
+    int live = 0;
+    for (int i = 0; i < nreq; i++) live += reqs[i].n != 0;
+    if (!live) return SIEVE_OK;
+    SV_TRY(nccl_check(g_nccl.group_start(), "ncclGroupStart"));
+    int st = SIEVE_OK;
+    for (int i = 0; i < nreq && st == SIEVE_OK; i++) {
+      if (!reqs[i].n) continue;
+      const int nop = reqs[i].op == RED_SUM ? 0 : (reqs[i].op == RED_MAX ? 2 : 3);
+      st = nccl_check(g_nccl.allreduce(reqs[i].buf, reqs[i].buf, reqs[i].n, 5 /* ncclUint64 */, nop, c, s),
+                      "ncclAllReduce");
+    }
+    const int ge = nccl_check(g_nccl.group_end(), "ncclGroupEnd");
+    return st != SIEVE_OK ? st : ge;
   }
 };
 
@@ -104,6 +119,7 @@ int nccl_comm_create(int rank, int world, const uint8_t id[128], Comm** out) {
 // in-process group
 // ------------------------------------------------------------------------------------------
 #define GROUP_MAX 16
+#define GROUP_MAXREQ 8
 struct sieve_group_s {
   int magic = 0x5e6e0001;
   int world = 0;
@@ -111,7 +127,8 @@ struct sieve_group_s {
   std::condition_variable cv;
   int arrived = 0;
   long generation = 0;
-  u64* ptrs[GROUP_MAX] = {};
+  u64* ptrs[GROUP_MAX][GROUP_MAXREQ] = {};
+  int err[GROUP_MAX] = {};
   void barrier() {
     std::unique_lock<std::mutex> lk(m);
     long gen = generation;
@@ -138,32 +155,51 @@ __global__ void k_group_reduce(PtrPack pk, int world, size_t n, int op, u64* out
   }
 }
 
+// first CUDA failure of a step, kept so the rank still reaches every barrier of the step (a rank
+// that returned early would leave the others waiting forever)
+#define GC_CUDA(x)                                                   \
+  do {                                                               \
+    cudaError_t _e = (x);                                            \
+    if (_e != cudaSuccess && st == SIEVE_OK) st = sv_cuda(_e, #x, __LINE__); \
+  } while (0)
+
 struct GroupComm : Comm {
   sieve_group_s* g = nullptr;
-  int allreduce(u64* buf, size_t n, ReduceOp op, cudaStream_t s) override {
+  int allreduce_group(const ARReq* reqs, int nreq, cudaStream_t s) override {
     // every rank must take part even with n == 0 (identical call sequence on all ranks)
-    SV_CUDA(cudaStreamSynchronize(s));
-    g->ptrs[rank] = buf;
+    int st = SIEVE_OK;
+    if (nreq > GROUP_MAXREQ) return sv_fail(SIEVE_EINVAL, "internal: too many grouped all-reduces");
+    GC_CUDA(cudaStreamSynchronize(s));
+    for (int i = 0; i < nreq; i++) g->ptrs[rank][i] = reqs[i].buf;
+    g->err[rank] = st;
     g->barrier();
-    u64* tmp = nullptr;
-    if (n) {
-      SV_CUDA(cudaMallocAsync((void**)&tmp, n * 8, s));
+    // a rank whose stream failed makes every rank return an error from this step (together)
+    bool peer_failed = false;
+    for (int r = 0; r < world; r++) peer_failed |= g->err[r] != SIEVE_OK;
+    if (peer_failed && st == SIEVE_OK) st = sv_fail(SIEVE_ECUDA, "another rank of the group failed");
+    u64* tmp[GROUP_MAXREQ] = {};
+    for (int i = 0; i < nreq && st == SIEVE_OK; i++) {
+      const size_t n = reqs[i].n;
+      if (!n) continue;
+      GC_CUDA(cudaMallocAsync((void**)&tmp[i], n * 8, s));
+      if (st != SIEVE_OK) break;
       PtrPack pk;
-      for (int r = 0; r < world; r++) pk.p[r] = g->ptrs[r];
+      for (int r = 0; r < world; r++) pk.p[r] = g->ptrs[r][i];
       unsigned blocks = (unsigned)((n + 255) / 256);
       if (blocks > 4096) blocks = 4096;
-      SV_LAUNCH(k_group_reduce, blocks, 256, 0, s)(pk, world, n, (int)op, tmp);
-      SV_CUDA(cudaGetLastError());
+      SV_LAUNCH(k_group_reduce, blocks, 256, 0, s)(pk, world, n, (int)reqs[i].op, tmp[i]);
+      GC_CUDA(cudaGetLastError());
     }
-    SV_CUDA(cudaStreamSynchronize(s));
+    GC_CUDA(cudaStreamSynchronize(s));
     g->barrier();  // all ranks have read every buffer
-    if (n) {
-      SV_CUDA(cudaMemcpyAsync(buf, tmp, n * 8, cudaMemcpyDeviceToDevice, s));
-      SV_CUDA(cudaFreeAsync(tmp, s));
-      SV_CUDA(cudaStreamSynchronize(s));
+    for (int i = 0; i < nreq; i++) {
+      if (!tmp[i]) continue;
+      if (st == SIEVE_OK) GC_CUDA(cudaMemcpyAsync(reqs[i].buf, tmp[i], reqs[i].n * 8, cudaMemcpyDeviceToDevice, s));
+      GC_CUDA(cudaFreeAsync(tmp[i], s));
     }
+    GC_CUDA(cudaStreamSynchronize(s));
     g->barrier();  // nobody reuses a published pointer before everyone copied
-    return SIEVE_OK;
+    return st;
   }
 };
 

@@ -9,11 +9,25 @@
 
 #include "common.cuh"
 
+// one in-place all-reduce of n u64 lanes
+struct ARReq {
+  u64* buf;
+  size_t n;
+  ReduceOp op;
+};
+
 struct Comm {
   int rank = 0, world = 1;
   virtual ~Comm() {}
-  // in-place all-reduce of n u64 lanes on `s`; returns SIEVE_OK or an error status
-  virtual int allreduce(u64* buf, size_t n, ReduceOp op, cudaStream_t s) = 0;
+  // in-place all-reduces of several buffers on `s` as ONE collective step (NCCL: one
+  // ncclGroupStart/End group, i.e. one fused launch; in-process group: one set of barriers);
+  // every rank passes the same sequence of (n, op).  Returns SIEVE_OK or an error status, and
+  // never leaves the other ranks of the group waiting (an error is returned after the step).
+  virtual int allreduce_group(const ARReq* reqs, int nreq, cudaStream_t s) = 0;
+  int allreduce(u64* buf, size_t n, ReduceOp op, cudaStream_t s) {
+    ARReq r{buf, n, op};
+    return allreduce_group(&r, 1, s);
+  }
 };
 
 int nccl_unique_id(uint8_t out[128]);

@@ -15,7 +15,7 @@
 // B200 mapping (the paper's scripts have no GPU design; this is new).  The KDE is a windowed
 // gather over the values of each segment grouped by grid cell (bucket.cu), bound by the FP64
 // pipe (no contraction, so no tensor cores).  Work item = (segment, tile of 32 grid points,
-// chunk of <= 256 values inside the tile's window |g - x| <= 7.6 h); items are dealt to warps
+// chunk of <= KDE_CH = 512 values inside the tile's window |g - x| <= 7.6 h); items are dealt to warps
 // round-robin and staged by a per-warp cp.async pipeline (see k_kde); each lane owns one grid
 // point and reads the staged values as shared-memory broadcasts.  The term is arranged to be
 // bit-identical to the oracle's while issuing 9 FP64-pipe instructions and ~6 others:
@@ -445,8 +445,11 @@ size_t kde_item_bytes(u32 items) { return (size_t)items * sizeof(KdeItem) + 16; 
 
 void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const u64* tile_range,
                 const u32* tile_items, void* item_desc, u32 items, u64* D,
-                unsigned long long* evaluated, bool guard, cudaStream_t s) {
-  if (items == 0) return;
+                unsigned long long* evaluated, bool guard, bool fix, cudaStream_t s) {
+  if (items == 0) {
+    if (fix) launch_kde_fix(D, (u64)nseg * G, s);
+    return;
+  }
   u32 tps = div_up(G, KDE_TJ);
   u32 ntiles = nseg * tps;
   // `items` is a host-side upper bound: grids are sized by it, the kernels stop at the
@@ -474,6 +477,9 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift
   if (grid > need) grid = need;
   SV_LAUNCH(kern, grid, 32 * KDE_WARPS, KDE_SMEM_BYTES, s)(desc, tile_items + ntiles, G, vals, vshift, D,
                                                            evaluated, fm == 0);
-  u64 nd = (u64)nseg * G;
-  SV_LAUNCH(k_kde_fix, div_up(nd, 256), 256, 0, s)(D, nd);
+  if (fix) launch_kde_fix(D, (u64)nseg * G, s);
+}
+
+void launch_kde_fix(u64* D, u64 npoints, cudaStream_t s) {
+  if (npoints) SV_LAUNCH(k_kde_fix, div_up(npoints, 256), 256, 0, s)(D, npoints);
 }

@@ -28,7 +28,7 @@ struct MomentsScratch {
   u32 kt;
 };
 int moments_kt(u32 K);  // kernels per smem pass
-int moments_grid();
+int moments_grid(u32 kt);
 void launch_moments(const u32* kid, const u64* x, const u64* y, u64 n, u32 K, u32 k0, u32 kt,
                     KMomPartial* part, u64* blk_tot, u64* errflags, int grid, cudaStream_t s);
 void launch_moments_reduce(const KMomPartial* part, const u64* blk_tot, int grid, u32 k0, u32 kt,
@@ -77,9 +77,14 @@ struct SegDev {
 void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
               u64* tile_range, u32* tile_items, void* scan_temp, cudaStream_t s);
 size_t kde_item_bytes(u32 items);
+// D[2j] accumulates the low 32-bit limbs of the item sums, D[2j + 1] the rest (both are plain
+// u64 sums: several ranks may all-reduce them as they are); fix = true normalises them into the
+// u128 D_j right away (else call launch_kde_fix after the cross-rank sum)
 void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const u64* tile_range,
                 const u32* tile_items, void* item_desc /* kde_item_bytes(items) */, u32 items,
-                u64* D /* [nseg][G][2] */, unsigned long long* evaluated, bool guard, cudaStream_t s);
+                u64* D /* [nseg][G][2] */, unsigned long long* evaluated, bool guard, bool fix,
+                cudaStream_t s);
+void launch_kde_fix(u64* D, u64 npoints, cudaStream_t s);
 
 // ---------------- segmented sort by (open segment, grid cell) (a2) ----------------------------
 // rounds > 1 read each re-opened part's range of the previous round's sorted keys in chunks of
@@ -131,6 +136,8 @@ void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, 
                        const u64* vals, u32 vshift, u32* items /* [cap + 1] */, void* scan_temp,
                        u64* lanes, u64* mm, u64* ab, cudaStream_t s);
 #define PART_REC (MOM_LANES + 4)
+#define PART_GUESS 16   // part slots per open segment before the exact count is known (a round
+                        // with more parts redoes its part moments once with the exact count)
 // out[0] = parts, out[1 + p * PART_REC ..] = {lanes[9], min, max, ia, ib} (mapped host memory)
 void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, const u64* mm,
                       const u64* ab, u64* out, cudaStream_t s);
@@ -217,3 +224,8 @@ void launch_copy(void* dst, const void* src, u64 bytes, cudaStream_t s);
 // cross-rank encoding of u128 pairs [n][2] <-> 4 limbs [n][4]
 void launch_u128_to_limbs(const u64* src, u64 n, u64* limbs, cudaStream_t s);
 void launch_limbs_to_u128(const u64* limbs, u64 n, u64* dst, cudaStream_t s);
+// p[i * stride] = ~p[i * stride], i < n (a MIN all-reduce becomes a MAX on complemented lanes)
+void launch_complement(u64* p, u64 n, u64 stride, cudaStream_t s);
+// x[0] = (flag[0] != 0), x[1 + r] = (r == rank ? count[0] : 0), r < world
+void launch_exchange_prep(const u64* flag, const unsigned long long* count, int rank, int world, u64* x,
+                          cudaStream_t s);

@@ -30,8 +30,12 @@
 #define MOM_L2 6                              // limbs of x^2 (88 bits)
 #define MOM_WORDS (1 + MOM_L1 + MOM_L2)       // count + limbs, u32 each
 
+#ifndef MOM_MINB
+#define MOM_MINB 1                            // resident blocks per SM (A/B on C4: 2 x 1024 threads caps the
+                                              // kernel at 32 registers and spills: 0.72 -> 3.0 ms)
+#endif
+
 int moments_kt(u32 K) { return (int)(K < MOM_KT ? K : MOM_KT); }
-int moments_grid() { return sv_num_sms(); }
 static size_t moments_smem(u32 kt) { return (size_t)kt * (16 + 4 * MOM_WORDS); }
 
 __device__ __forceinline__ void atomic_min_u64_smem(u64* p, u64 v) {
@@ -51,7 +55,7 @@ __device__ __forceinline__ void atomic_max_u64_smem(u64* p, u64 v) {
   }
 }
 
-__global__ void __launch_bounds__(MOM_THREADS)
+__global__ void __launch_bounds__(MOM_THREADS, MOM_MINB)
 k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __restrict__ y,
           u64 n, u32 K, u32 k0, u32 kt, KMomPartial* __restrict__ part,
           u64* __restrict__ blk_tot, u64* errflags) {
@@ -209,6 +213,23 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
       blk_tot[blockIdx.x * 3 + 2] = mx;
     }
   }
+}
+
+// blocks of pass A: every SM holds as many blocks as its shared memory takes for this kt (two
+// at K <= 2048: twice the warps to hide the shared-atomic latency), queried once per (device, kt)
+int moments_grid(u32 kt) {
+  static int cache[64][2] = {};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int* e = cache[dev & 63];
+  if (e[0] != (int)kt || e[1] < 1) {
+    sv_smem_attr(k_moments, (int)moments_smem(MOM_KT));
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_moments, MOM_THREADS, moments_smem(kt));
+    e[0] = (int)kt;
+    e[1] = per_sm < 1 ? 1 : per_sm;
+  }
+  return sv_num_sms() * e[1];
 }
 
 void launch_moments(const u32* kid, const u64* x, const u64* y, u64 n, u32 K, u32 k0, u32 kt,

@@ -1,12 +1,11 @@
 // sort.cu -- Tier-3 key compaction, LSD radix sort of 64-bit packed keys and exclusive scans.
 //
-// The compaction gathers the Tier-3 invocations as keys (t3rank << bx) + x (bx = bitlen(max x));
-// the stratification groups them by (segment, grid cell) with the counting sort of bucket.cu.
-// The radix sort orders the (stratum, CTA) entries of pass B, the name hashes of the CSV ingest
-// and the Tier-3 keys of the exact min-strata DP (which needs every distinct value in order):
-// only the digit passes whose 8 bits vary over the keys run (one histogram read decides).
-//
-// Radix passes are onesweep (see below): one kernel per digit with decoupled look-back.
+// The compaction gathers the Tier-3 invocations as keys (t3rank << bx) + x (bx = bitlen(max x)).
+// The radix sort orders them per refinement round by (segment, grid cell) (bucket.cu: the cell
+// keys' low bits), and also the (stratum, CTA) entries of pass B, the name hashes of the CSV
+// ingest and the Tier-3 keys of the exact min-strata DP.  It runs one onesweep pass per 8-bit
+// digit of the key bits it is asked to sort (see below): digit histograms and bases are computed
+// on the device, with no host read-back.
 #include <algorithm>
 
 #include "kernels.cuh"

@@ -200,6 +200,34 @@ class Ctx:
         self.device, self.rank, self.world = device, rank, world if group is None else group.world
         self._group = group
 
+    def set_allocator(self, alloc=None, free=None):
+        """sieve_ctx_set_allocator: alloc(nbytes, stream_handle) -> device pointer (int) and
+        free(ptr, stream_handle), e.g. torch_caching_allocator(); None, None restores the
+        library's cudaMallocAsync.  Buffers are always released by the allocator that made them."""
+        if (alloc is None) != (free is None):
+            raise ValueError("alloc and free must both be given or both be None")
+        if alloc is None:
+            self._hooks = None
+            _check(_L.sieve_ctx_set_allocator(self._h, None, None, None), "sieve_ctx_set_allocator")
+            return
+
+        def _a(nbytes, stream, user):
+            try:
+                return int(alloc(int(nbytes), stream or 0)) or None
+            except Exception:  # the library reports SIEVE_ENOMEM for a NULL result
+                return None
+
+        def _f(ptr, stream, user):
+            free(int(ptr), stream or 0)
+
+        a, f = _ALLOC_FN(_a), _FREE_FN(_f)
+        # the hooks must outlive every buffer they made: keep them with the context (and with
+        # any trace created while they were set, see load_trace)
+        self._hooks_live = getattr(self, "_hooks_live", []) + [(a, f)]
+        self._hooks = (a, f)
+        _check(_L.sieve_ctx_set_allocator(self._h, ctypes.cast(a, ctypes.c_void_p),
+                                          ctypes.cast(f, ctypes.c_void_p), None), "sieve_ctx_set_allocator")
+
     def set_term_count(self, enable=True):
         """In-window KDE term counting (strata.kde_terms); on by default."""
         _check(_L.sieve_ctx_set_term_count(self._h, 1 if enable else 0), "sieve_ctx_set_term_count")
@@ -224,6 +252,23 @@ class Ctx:
 
     def __del__(self):
         self.close()
+
+
+_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
+_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
+
+
+def torch_caching_allocator(device=0):
+    """(alloc, free) hooks that take device memory from PyTorch's caching allocator."""
+    import torch
+
+    def alloc(nbytes, stream):
+        return torch.cuda.caching_allocator_alloc(nbytes, device, stream)
+
+    def free(ptr, stream):
+        torch.cuda.caching_allocator_delete(ptr)
+
+    return alloc, free
 
 
 def kernel_launches():
@@ -274,10 +319,20 @@ def load_trace(ctx, kernel_id, instr, num_kernels, cta=None, cycles=None, first_
     on_dev = kinds == {True}
     mem = (MEM_DEVICE if on_dev else MEM_HOST) | (ADOPT if adopt else 0)
     n = len(kernel_id)
+    for name, c in zip(("instr", "cta", "cycles"), (instr, cta, cycles)):
+        if c is not None and len(c) != n:  # the library reads n rows of every column
+            raise ValueError(f"{name} has {len(c)} rows, kernel_id has {n}")
+    if on_dev:
+        import torch
+        devs = {c[2].device.index for c in cols if c[2] is not None}
+        if devs != {ctx.device}:
+            raise ValueError(f"device columns must live on cuda:{ctx.device}")
     h = ctypes.c_void_p()
     _check(_L.sieve_load_trace(ctx._h, n, first_id, num_kernels, cols[0][0], cols[1][0], cols[2][0],
                                cols[3][0], mem, ctypes.byref(h)), "sieve_load_trace")
-    return Trace(h, ctx, n, [c[2] for c in cols] if adopt else None, num_kernels)
+    t = Trace(h, ctx, n, [c[2] for c in cols] if adopt else None, num_kernels)
+    t._hooks = getattr(ctx, "_hooks", None)  # the allocator that owns the copied columns
+    return t
 
 
 def load_csv(ctx, data, col_kernel, col_instr, col_cta=-1, col_cycles=-1, header_lines=1,
@@ -398,11 +453,24 @@ class Strata:
         self.close()
 
 
+def _check_sid(t, trace):
+    """stratum ids are written / read by the kernels as a DEVICE uint32 array of n_local entries"""
+    import torch
+    if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype in (torch.int32, torch.uint32)
+            and t.is_contiguous()):
+        raise TypeError("stratum_of_invocation must be a contiguous CUDA int32/uint32 tensor")
+    if t.numel() < trace.n:
+        raise ValueError(f"stratum_of_invocation has {t.numel()} entries, the trace {trace.n}")
+    if t.device.index != trace.ctx.device:
+        raise ValueError(f"stratum_of_invocation must live on cuda:{trace.ctx.device}")
+
+
 def stratify(trace, params=None, stratum_of_invocation=None, **kw):
     """sieve_stratify; stratum_of_invocation: optional CUDA int32/uint32 tensor [n_local]."""
     p = params if params is not None else default_params(**kw)
     sid_ptr = None
     if stratum_of_invocation is not None:
+        _check_sid(stratum_of_invocation, trace)
         sid_ptr = ctypes.c_void_p(stratum_of_invocation.data_ptr())
     h = ctypes.c_void_p()
     _check(_L.sieve_stratify(trace._h, ctypes.byref(p), sid_ptr, ctypes.byref(h)), "sieve_stratify")
@@ -459,6 +527,7 @@ def predict_multi(strata, trace, rep_cycles):
 
 def cycle_cov(strata, trace, stratum_of_invocation):
     """sieve_cycle_cov: per-stratum CoV of member cycles + instruction-weighted mean (Fig. 4)."""
+    _check_sid(stratum_of_invocation, trace)
     cov = np.zeros(len(strata), np.float64)
     w = ctypes.c_double()
     _check(_L.sieve_cycle_cov(strata._h, trace._h, ctypes.c_void_p(stratum_of_invocation.data_ptr()),
@@ -471,6 +540,8 @@ def predict(strata, trace, rep_cycles=None):
     rc = None
     if rep_cycles is not None:
         rc = np.ascontiguousarray(rep_cycles, np.uint64)
+        if rc.ndim != 1 or len(rc) != len(strata):  # the library reads n_strata values
+            raise ValueError(f"rep_cycles must have one entry per stratum ({len(strata)})")
     _check(_L.sieve_predict(strata._h, trace._h, None if rc is None else rc.ctypes.data_as(ctypes.c_void_p),
                             ctypes.byref(out)), "sieve_predict")
     return {"predicted_cycles": out.predicted_cycles, "predicted_ipc": out.predicted_ipc,

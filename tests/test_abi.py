@@ -56,3 +56,34 @@ def test_product_never_imports_oracle():
 
 def test_stratum_struct_size(lib):
     assert lib.STRATUM_DTYPE.itemsize == 96
+
+
+def test_binding_validates_before_the_library_reads():
+    """the binding rejects arguments the library would read out of bounds"""
+    import numpy as np
+    import torch
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    kid = np.zeros(10, np.uint32)
+    x = np.ones(9, np.uint64)
+
+    class _Ctx:  # no GPU needed: the checks run before any library call
+        device = 0
+        _h = None
+    with pytest.raises(ValueError):
+        sieve.load_trace(_Ctx(), kid, x, num_kernels=1)
+    with pytest.raises(ValueError):
+        sieve.load_trace(_Ctx(), kid, np.ones(10, np.uint64), num_kernels=1, cycles=np.ones(3, np.uint64))
+
+    class _Trace:
+        n = 10
+        ctx = _Ctx()
+    with pytest.raises(TypeError):
+        sieve.sieve._check_sid(torch.zeros(10, dtype=torch.int32), _Trace())   # host tensor
+
+    class _Strata:
+        _h = None
+
+        def __len__(self):
+            return 5
+    with pytest.raises(ValueError):
+        sieve.predict(_Strata(), _Trace(), rep_cycles=np.ones(4, np.uint64))

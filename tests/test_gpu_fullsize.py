@@ -62,7 +62,11 @@ def test_c4_full_size_sampled_parity():
     for want, lo, hi, m in [(3, 20_000, 250_000, 5), (3, 50, 20_000, 3), (2, 1000, 10 ** 7, 4), (1, 1, 10 ** 8, 4)]:
         cand = [k for k, t in tier_of.items() if t == want and lo <= counts[k] <= hi]
         pick += list(rng.choice(cand, size=min(m, len(cand)), replace=False))
-    assert len(pick) >= 10
+    # the two largest Tier-3 kernels (~600k invocations each: the widest KDE segments of C4)
+    t3 = [k for k, t in tier_of.items() if t == 3]
+    pick += sorted(t3, key=lambda k: -counts[k])[:2]
+    pick = sorted(set(int(k) for k in pick))
+    assert len(pick) >= 12
     rows = np.nonzero(np.isin(tr["kid"], pick))[0]
     o = oracle.stratify(tr["kid"][rows], tr["x"][rows], cfg.K, tr["cta"][rows], tr["y"][rows],
                         ids=rows.astype(np.uint64))

@@ -2,7 +2,7 @@
 # one gpurun call: parity tests on the default build, A/B bench of every variant, ncu of k_kde
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests -m gpu -x -q ${TESTS:-} > gpurun_out/ab_tests.log 2>&1; echo tests_rc=$? >> gpurun_out/ab_tests.log
-bash scratch/ab_variants.sh > gpurun_out/ab.log 2>&1
+bash tools/ab_variants.sh > gpurun_out/ab.log 2>&1
 if [ -n "$NCU" ]; then
   for so in default $NCU_VARIANTS; do
     if [ "$so" = default ]; then unset SIEVE_LIB_PATH; tag=default; else export SIEVE_LIB_PATH=$PWD/$so; tag=$(basename $so .so); fi
