@@ -626,6 +626,44 @@ static int h2d(sieve_ctx c, T* d, const std::vector<T>& h) {
   launch_copy(d, p, h.size() * sizeof(T), c->stream);  // SM copy from the UVA-mapped staging
   return SIEVE_OK;
 }
+// Several host <-> device copies of the orchestrator in ONE launch: queue them with add_h2d /
+// add_d2h (staged through the pinned arena like h2d / d2h), then flush() before the kernels that
+// read the uploaded tables; read-backs land in their vectors at the next sync(c).
+struct CopyBatch {
+  sieve_ctx c;
+  CopyRegions r{};
+  explicit CopyBatch(sieve_ctx cc) : c(cc) { r.k = 0; }
+  int add_raw(void* dst, const void* src, size_t bytes) {
+    if (!bytes) return SIEVE_OK;
+    if (r.k == COPY_MAX) SV_TRY(flush());
+    r.dst[r.k] = dst; r.src[r.k] = src; r.bytes[r.k] = bytes; r.k++;
+    return SIEVE_OK;
+  }
+  template <typename T>
+  int add_h2d(T* d, const std::vector<T>& h) {
+    if (h.empty()) return SIEVE_OK;
+    void* p;
+    SV_TRY(pin_alloc(c, &p, h.size() * sizeof(T)));
+    memcpy(p, h.data(), h.size() * sizeof(T));
+    return add_raw(d, p, h.size() * sizeof(T));
+  }
+  template <typename T>
+  int add_d2h(std::vector<T>& h, const T* d, size_t n) {
+    h.resize(n);
+    if (!n) return SIEVE_OK;
+    void* p;
+    SV_TRY(pin_alloc(c, &p, n * sizeof(T)));
+    c->pend.push_back({h.data(), p, n * sizeof(T)});
+    return add_raw(p, d, n * sizeof(T));
+  }
+  int flush() {
+    launch_copy_multi(r, c->stream);
+    r.k = 0;
+    SV_CUDA(cudaGetLastError());
+    return SIEVE_OK;
+  }
+};
+
 static bool host_timing() {
   static const bool on = getenv("SIEVE_HOST_TIMING") != nullptr;
   return on;
@@ -690,6 +728,11 @@ struct Fin { u32 kid, tier; u64 lo, hi, n; u128 s1; double h; u32 round; };
 // tier census computes them once
 struct MomentsHost {
   std::vector<u64> lanes, mm, tot, localn;
+  // pass A's per-block partials on the device (arena memory of THIS call; null when cached from
+  // another call or when the kernels took several shared-memory passes)
+  const KMomPartial* part = nullptr;
+  int part_grid = 0;
+  u32 part_kt = 0;
 };
 
 // ---------------- pass A: per-kernel moments + totals -------------------
@@ -738,20 +781,19 @@ static int moments_pass(sieve_trace t, MomentsHost* M) {
     SV_TRY(allreduce_group(c, {{lanes.get(), (size_t)K * MOM_LANES, RED_SUM}, {tot.get(), 4, RED_SUM},
                                {mm.get(), (size_t)K * 2, RED_MAX}, {tot.get() + 4, 4, RED_MAX}}));
     launch_complement(mm.get(), K, 2, S);
-    SV_TRY(d2h(c, h_lanes, lanes.get(), (size_t)K * MOM_LANES));
-    SV_TRY(d2h(c, h_mm, mm.get(), (size_t)K * 2));
-    SV_TRY(d2h(c, h_tot, tot.get(), 8));
-    SV_TRY(d2h(c, h_localn, local_n.get(), K));
-    SV_TRY(sync(c));
-  } else {
-    SV_TRY(d2h(c, h_lanes, lanes.get(), (size_t)K * MOM_LANES));
-    SV_TRY(d2h(c, h_mm, mm.get(), (size_t)K * 2));
-    SV_TRY(d2h(c, h_tot, tot.get(), 8));
-    SV_TRY(d2h(c, h_localn, local_n.get(), K));
+  }
+  {
+    CopyBatch cb(c);
+    SV_TRY(cb.add_d2h(h_lanes, lanes.get(), (size_t)K * MOM_LANES));
+    SV_TRY(cb.add_d2h(h_mm, mm.get(), (size_t)K * 2));
+    SV_TRY(cb.add_d2h(h_tot, tot.get(), 8));
+    SV_TRY(cb.add_d2h(h_localn, local_n.get(), K));
+    SV_TRY(cb.flush());
     SV_TRY(sync(c));
   }
   if (h_tot[5]) return sv_fail(SIEVE_EINVAL, "kernel id >= num_kernels in the trace");
   if (h_tot[6]) return sv_fail(SIEVE_ERANGE, "instruction count 0 or >= 2^44 in the trace (A21)");
+  if (K <= kt) { M->part = part.get(); M->part_grid = gridA; M->part_kt = kt; }
   M->lanes.swap(h_lanes);
   M->mm.swap(h_mm);
   M->tot.swap(h_tot);
@@ -807,7 +849,10 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   }
   R->total_instr = I;
 
-  // ---------------- Tier-3 keys: compaction ----------------------------------------------------
+  // ---------------- Tier-3 values: compaction ---------------------------------------------------
+  // grouped path (G <= GROUP_MAXG): the Tier-3 rows' x grouped by segment (t3rank) at the bases
+  // the local counts give; radix path: tagged keys (t3rank << bx) + x in row order
+  const bool grouped = G <= GROUP_MAXG && !getenv("SIEVE_CELL_RADIX");
   const u32 bx = std::max<u32>(1, bitlen(max_x));
   DBuf<u64> keys(c);
   DBuf<u32> d_t3rank(c);
@@ -815,10 +860,28 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   SV_TRY(counter.alloc(4));
   if (n_t3 && n3_local) {
     SV_TRY(d_t3rank.alloc(K));
-    SV_TRY(h2d(c, d_t3rank.get(), t3rank));
+    CopyBatch cb(c);
+    SV_TRY(cb.add_h2d(d_t3rank.get(), t3rank));
     SV_TRY(keys.alloc(n3_local));
-    SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
+    if (!grouped) {
+      SV_TRY(cb.flush());
+      SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
+    }
     PhaseTimer tm(c, SIEVE_PHASE_COMPACT, n * 12 + n3_local * 8);
+    if (grouped) {
+      std::vector<u32> sb(2 * (size_t)n_t3);   // [segment bases | kernel of each segment]
+      for (u32 s = 0; s < n_t3; s++) { sb[s] = (u32)open[s].b; sb[n_t3 + s] = open[s].kid; }
+      DBuf<u32> d_sb(c), cur(c);
+      DBuf<char> gtmp(c);
+      SV_TRY(d_sb.alloc(2 * (size_t)n_t3));
+      SV_TRY(cur.alloc(n_t3));
+      SV_TRY(gtmp.alloc(group_t3_temp_bytes(n_t3)));
+      SV_TRY(cb.add_h2d(d_sb.get(), sb));
+      SV_TRY(cb.flush());
+      if (n_t3 > GROUP_T3_SMEM_MAX) SV_CUDA(cudaMemsetAsync(cur.get(), 0, (size_t)n_t3 * 4, S));  // global-cursor path
+      launch_group_t3(t->kid, t->x, n, d_t3rank.get(), n_t3, d_sb.get(), cur.get(), keys.get(), gtmp.get(),
+                      cached == &own ? own.part : nullptr, own.part_grid, own.part_kt, d_sb.get() + n_t3, S);
+    } else
     launch_t3_compact(t->kid, t->x, n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
     SV_CUDA(cudaGetLastError());
   }
@@ -840,14 +903,15 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   const u32 tstride = G / 2 + 1;
   const u32 tps = div_up(G, KDE_TJ);
   const u64 max_cells = bx >= 63 ? 0 : (1ull << (64 - bx)) - 1;  // idx <= ncell must fit
-  if (!open.empty() && max_cells < G) return sv_fail(SIEVE_ELIMIT, "instruction counts too wide for the cell sort key");
+  if (!grouped && !open.empty() && max_cells < G)
+    return sv_fail(SIEVE_ELIMIT, "instruction counts too wide for the cell sort key");
   for (auto& o : open) { o.src = keys.get(); o.src_shift = 0; }
   while (!open.empty()) {
     round++;
     if (round > P->max_rounds) return sv_fail(SIEVE_ELIMIT, "Tier-3 refinement exceeded max_rounds");
     std::vector<OpenSeg> next;
     const u32 nopen = (u32)open.size();
-    u32 batch = (u32)std::min<u64>(nopen, std::min<u64>(max_cells / G, 0xFFFFFFFEull / G));
+    u32 batch = grouped ? nopen : (u32)std::min<u64>(nopen, std::min<u64>(max_cells / G, 0xFFFFFFFEull / G));
     if (const char* e = getenv("SIEVE_SEG_BATCH"))  // test hook: force small batches
       batch = std::max<u32>(1, std::min<u32>(batch, (u32)atoi(e)));
     // batches: runs of segments with one source array, at most `batch` segments each
@@ -864,7 +928,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     std::vector<SegDev> hs(nseg);
     std::vector<double> hh(nseg);
     std::vector<BucketChunk> chunks;
+    std::vector<u32> seg_chunk;  // grouped path: first chunk of every segment
     u64 maxlen = 0;  // largest segment (local values)
+    u64 nsup = 0;    // grouped path: values of the segments' source ranges
     for (u32 s = 0; s < nseg; s++) {
       const OpenSeg& o = op[s];
       double h = scott_h(o.n, o.s1, o.s2, P->bw_scale);
@@ -876,33 +942,67 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       hs[s].cq = (double)(G - 1) / (double)(o.hi - o.lo);
       u64 len = round == 1 ? h_localn[o.kid] : o.e - o.b;
       maxlen = std::max(maxlen, len);
-      if (round > 1)
+      if (grouped) {  // every round reads each segment's contiguous source range [b, e)
+        seg_chunk.push_back((u32)chunks.size());
+        nsup += o.e - o.b;
+        for (u64 b = o.b; b < o.e; b += GROUP_CH)
+          chunks.push_back({s, (u32)std::min<u64>(GROUP_CH, o.e - b), b});
+      } else if (round > 1) {
         for (u64 b = o.b; b < o.e; b += BK_CHUNK)
           chunks.push_back({s, (u32)std::min<u64>(BK_CHUNK, o.e - b), b});
+      }
     }
+    if (grouped) seg_chunk.push_back((u32)chunks.size());
     if (round == 1)  // the open segments are the Tier-3 kernels in t3rank order
       for (u32 s = 0; s < nseg; s++)
         if (op[s].t3rank != s0 + s) return sv_fail(SIEVE_ESTATE, "internal: round-1 segment order");
     const u64* src = op[0].src;  // one source per batch (see bstart)
     const u32 src_shift = op[0].src_shift;
-    const u64 nin = round == 1 ? nkeys : (u64)chunks.size() * BK_CHUNK;
+    const u64 nin = grouped ? nsup : (round == 1 ? nkeys : (u64)chunks.size() * BK_CHUNK);
+    const u32 vsh = grouped ? 0 : ib;  // the grouped values are raw x; cell keys carry x above ib
     DBuf<SegDev> segs(c);
     DBuf<double> gtab(c);
     DBuf<u32> off(c);
     DBuf<u64> ck(c);
     DBuf<BucketChunk> d_chunks(c);
     SV_TRY(segs.alloc(nseg));
-    SV_TRY(h2d(c, segs.get(), hs));
+    CopyBatch rcb(c);   // this round's tables: one upload
+    SV_TRY(rcb.add_h2d(segs.get(), hs));
     SV_TRY(gtab.alloc(ncell));
     SV_TRY(off.alloc(ncell + 1));
     SV_TRY(ck.alloc(std::max<u64>(nin, 1)));
+    if (grouped) {
+      const u32 nch = (u32)chunks.size();
+      DBuf<unsigned short> cells(c);
+      DBuf<u32> hist(c), rel(c), tot(c), d_sc(c);
+      DBuf<char> stemp(c);
+      SV_TRY(cells.alloc((size_t)std::max<u32>(nch, 1) * GROUP_CH));
+      SV_TRY(hist.alloc((size_t)std::max<u32>(nch, 1) * G));
+      SV_TRY(rel.alloc((size_t)std::max<u32>(nch, 1) * G));
+      SV_TRY(tot.alloc(ncell));
+      SV_TRY(d_sc.alloc(nseg + 1));
+      SV_TRY(stemp.alloc(scan_u32_temp_bytes(ncell)));
+      if (nch) {
+        SV_TRY(d_chunks.alloc(nch));
+        SV_TRY(rcb.add_h2d(d_chunks.get(), chunks));
+      }
+      SV_TRY(rcb.add_h2d(d_sc.get(), seg_chunk));
+      SV_TRY(rcb.flush());
+      PhaseTimer tm(c, SIEVE_PHASE_SORT, nin * 36 + (u64)nch * G * 16);
+      launch_grid_tab(segs.get(), nseg, G, gtab.get(), S);
+      launch_cell_group(d_chunks.get(), nch, src, segs.get(), nseg, G, d_sc.get(), cells.get(), hist.get(),
+                        rel.get(), tot.get(), off.get(), stemp.get(), ck.get(),
+                        c->count_terms ? terms.get() : nullptr, S);
+      SV_CUDA(cudaGetLastError());
+    } else
     {
       DBuf<char> tmp(c);
       SV_TRY(tmp.alloc(radix_sort_temp_bytes(nin, false, (int)ib)));
       if (!chunks.empty()) {
         SV_TRY(d_chunks.alloc(chunks.size()));
-        SV_TRY(h2d(c, d_chunks.get(), chunks));
+        SV_TRY(rcb.add_h2d(d_chunks.get(), chunks));
       }
+      SV_TRY(rcb.flush());
       PhaseTimer tm(c, SIEVE_PHASE_SORT, nin * 8);
       launch_grid_tab(segs.get(), nseg, G, gtab.get(), S);
       // the cell keys go where an odd number of radix passes ends in ck (no copy-back), and
@@ -965,7 +1065,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       bool guard = false;
       for (u32 s = 0; s < nseg; s++)
         if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 140.0 * hs[s].h) guard = true;
-      launch_kde(segs.get(), nseg, G, ck.get(), ib, tile_range.get(), tile_items.get(),
+      launch_kde(segs.get(), nseg, G, ck.get(), vsh, tile_range.get(), tile_items.get(),
                  item_tile.get(), items, D.get(), terms.get() + 1, guard, !c->comm, S);
       tm.stop();
       SV_CUDA(cudaGetLastError());
@@ -989,11 +1089,13 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     // at any rank count.
     std::vector<u32> h_ntk;
     std::vector<u64> h_D, h_T;
-    SV_TRY(d2h(c, h_ntk, ntk.get(), (size_t)nseg * 2));
+    CopyBatch ecb(c);   // read back with the part records at the round's synchronisation
+    SV_TRY(ecb.add_d2h(h_ntk, ntk.get(), (size_t)nseg * 2));
     if (R->keep_debug) {
-      SV_TRY(d2h(c, h_D, D.get(), (size_t)nseg * G * 2));
-      SV_TRY(d2h(c, h_T, T.get(), (size_t)nseg * tstride));
+      SV_TRY(ecb.add_d2h(h_D, D.get(), (size_t)nseg * G * 2));
+      SV_TRY(ecb.add_d2h(h_T, T.get(), (size_t)nseg * tstride));
     }
+    SV_TRY(ecb.flush());
     u64 *hrec = nullptr, *drec = nullptr;
     for (int pass = 0;; pass++) {
       DBuf<u32> pitems(c);
@@ -1003,7 +1105,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       {
         PhaseTimer tp(c, SIEVE_PHASE_REFINE, 0);
         launch_part_stats(segs.get(), nseg, G, gtab.get(), off.get(), T.get(), tstride, ntk.get(), d_off.get(),
-                          cap, ck.get(), ib, pitems.get(), ptemp.get(), pl.get(), pm.get(), pab.get(), S);
+                          cap, ck.get(), vsh, pitems.get(), ptemp.get(), pl.get(), pm.get(), pab.get(), S);
         SV_CUDA(cudaGetLastError());
       }
       if (c->comm) {
@@ -1061,7 +1163,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
           fin.push_back({op[s].kid, 3, lo, hi, pn, s1, hh[s], round});
         else  // re-opened: its values are [ia, ib) of this batch's sorted keys (x << ib)
           next.push_back({op[s].kid, op[s].t3rank, lo, hi, pn, s1, s2, L[MOM_LANES + 2],
-                          L[MOM_LANES + 3], ck.get(), ib});
+                          L[MOM_LANES + 3], ck.get(), vsh});
       }
     }
     }  // batches
@@ -1071,7 +1173,6 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   R->rounds = round;
   // the KDE term count is read back with the representatives at the end (no extra sync)
   std::vector<unsigned long long> h_terms;
-  SV_TRY(d2h(c, h_terms, terms.get(), 2));
   keys.release();
 
   // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
@@ -1113,8 +1214,12 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   SV_TRY(d_ktab.alloc(K));
   SV_TRY(d_lows.alloc(lows.size()));
   SV_TRY(errf.alloc(4));
-  SV_TRY(h2d(c, d_ktab.get(), ktab));
-  SV_TRY(h2d(c, d_lows.get(), lows));
+  {
+    CopyBatch cb(c);
+    SV_TRY(cb.add_h2d(d_ktab.get(), ktab));
+    SV_TRY(cb.add_h2d(d_lows.get(), lows));
+    SV_TRY(cb.flush());
+  }
   u64 cap = 1;
   while (cap < std::max<u64>(1u << 16, 8ull * ns)) cap <<= 1;
   // One rank: the (stratum, CTA) entries go to the representatives without a host round trip --
@@ -1207,15 +1312,24 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(d_tier.alloc(ns));
     SV_TRY(rep.alloc(2 * (size_t)ns));
     SV_TRY(repxy.alloc(2 * (size_t)ns));
-    SV_TRY(h2d(c, d_tier.get(), tiers));
+    {
+      CopyBatch cb(c);
+      SV_TRY(cb.add_h2d(d_tier.get(), tiers));
+      SV_TRY(cb.flush());
+    }
     launch_reps(sk.get(), scnt.get(), sfirst.get(), Etot, d_tier.get(), ns, rep.get(), rep.get() + ns, S);
     launch_rep_xy(rep.get(), ns, t->first_id, n, t->x, t->y, repxy.get(), S);
     tr.stop();
     SV_CUDA(cudaGetLastError());
     SV_TRY(allreduce(c, repxy.get(), 2 * (size_t)ns, RED_SUM));   // AR-5: owner contributes
-    SV_TRY(d2h(c, h_rep, rep.get(), 2 * (size_t)ns));
-    SV_TRY(d2h(c, h_xy, repxy.get(), 2 * (size_t)ns));
-    if (!c->comm) SV_TRY(d2h(c, hflag, errf.get(), 4));
+    {
+      CopyBatch cb(c);
+      SV_TRY(cb.add_d2h(h_rep, rep.get(), 2 * (size_t)ns));
+      SV_TRY(cb.add_d2h(h_xy, repxy.get(), 2 * (size_t)ns));
+      if (!c->comm) SV_TRY(cb.add_d2h(hflag, errf.get(), 4));
+      if (h_terms.empty()) SV_TRY(cb.add_d2h(h_terms, terms.get(), 2));
+      SV_TRY(cb.flush());
+    }
     SV_TRY(sync(c));
     if (!c->comm && hflag[2]) { cap <<= 2; continue; }
     break;
@@ -1577,7 +1691,11 @@ static int predict_impl(sieve_strata s, sieve_trace t, u32 M, const uint64_t* re
   DBuf<double> dout(c);
   SV_TRY(dW.alloc(hW.size())); SV_TRY(dx.alloc(ns)); SV_TRY(dy.alloc(hy.size()));
   SV_TRY(dout.alloc(4 * (size_t)M));
-  SV_TRY(h2d(c, dW.get(), hW)); SV_TRY(h2d(c, dx.get(), hx)); SV_TRY(h2d(c, dy.get(), hy));
+  {
+    CopyBatch cb(c);
+    SV_TRY(cb.add_h2d(dW.get(), hW)); SV_TRY(cb.add_h2d(dx.get(), hx)); SV_TRY(cb.add_h2d(dy.get(), hy));
+    SV_TRY(cb.flush());
+  }
   PhaseTimer tpr(c, SIEVE_PHASE_PREDICT, 0);
   launch_predict(dW.get(), dx.get(), dy.get(), ns, M, dout.get(), c->stream);
   tpr.stop();

@@ -28,6 +28,10 @@
 #define AS_HC 8192          // shared hash capacity (entries): 128 KB, one block per SM
 #define AS_FLUSH (3 * AS_HC / 4)      // flush to the L2 table when this full
 #define AS_MAXP 32          // probes before falling back to the global table
+#ifndef AS_CHECK
+#define AS_CHECK 16         // tiles between the block barriers that check the table's fill (A/B on C4:
+                            // every tile 0.73 ms, every 4 tiles 0.60, every 16 tiles 0.55)
+#endif
 
 // One block per SM with a large table: a block's contiguous chunk sees nearly every (stratum,
 // CTA) pair of the trace (thousands), so a small table would flush -- i.e. issue contended L2
@@ -87,6 +91,7 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
   const u64 tile = (u64)AS_THREADS * AS_IPT;
   u32 kk[AS_IPT], cc[AS_IPT];
   u64 vv[AS_IPT];
+  u32 tiles_done = 0;
   auto load_tile = [&](u64 base, u32* k_, u64* v_, u32* c_) {
 #pragma unroll
     for (int j = 0; j < AS_IPT; j++) {
@@ -149,8 +154,18 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
       }
       if (!done) ghash_update(gh, key, 1, first_id + i, errflags);
     }
-    __syncthreads();
     bool last = base + tile >= b1;
+    ++tiles_done;
+    // the fill check needs a block barrier: every AS_CHECK tiles (a full table only sends rows
+    // to the L2 table directly, it is never wrong)
+    if (tiles_done % AS_CHECK != 0 && !last) {
+#if AS_PIPE
+#pragma unroll
+      for (int j = 0; j < AS_IPT; j++) { kk[j] = nk[j]; vv[j] = nv[j]; cc[j] = nc[j]; }
+#endif
+      continue;
+    }
+    __syncthreads();
     if (s_fill > AS_FLUSH || last) {  // rows that find no slot go to the L2 table directly
       for (u32 e = threadIdx.x; e < AS_HC; e += AS_THREADS) {
         u64 key = hk[e];
@@ -297,6 +312,33 @@ void launch_copy(void* dst, const void* src, u64 bytes, cudaStream_t s) {
     SV_LAUNCH(k_copy_bytes, (unsigned)std::min<u64>(div_up(bytes, 256), 2048), 256, 0, s)(
         (unsigned char*)dst, (const unsigned char*)src, bytes);
   }
+}
+
+// several copies in ONE launch (blockIdx.y = region): the orchestrator's small host <-> device
+// tables of one step go together (each separate copy was a launch plus a PCIe round trip)
+__global__ void k_copy_multi(CopyRegions r) {
+  const int q = blockIdx.y;
+  if (q >= r.k) return;
+  unsigned char* d = (unsigned char*)r.dst[q];
+  const unsigned char* sp = (const unsigned char*)r.src[q];
+  const u64 n = r.bytes[q];
+  const u64 stride = (u64)gridDim.x * blockDim.x;
+  const u64 t = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if ((((uintptr_t)d | (uintptr_t)sp) & 7) == 0) {
+    const u64 nw = n / 8;
+    for (u64 i = t; i < nw; i += stride) ((u64*)d)[i] = ((const u64*)sp)[i];
+    for (u64 i = nw * 8 + t; i < n; i += stride) d[i] = sp[i];
+  } else {
+    for (u64 i = t; i < n; i += stride) d[i] = sp[i];
+  }
+}
+void launch_copy_multi(const CopyRegions& r, cudaStream_t s) {
+  if (r.k <= 0) return;
+  u64 mx = 0;
+  for (int q = 0; q < r.k; q++) mx = r.bytes[q] > mx ? r.bytes[q] : mx;
+  if (!mx) return;
+  dim3 grid(std::min<u64>(div_up(mx, 256 * 8), 512), r.k);
+  SV_LAUNCH(k_copy_multi, grid, 256, 0, s)(r);
 }
 
 __global__ void k_fill_u64(u64* p, u64 n, u64 v) {

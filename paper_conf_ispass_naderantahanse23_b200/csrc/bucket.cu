@@ -377,3 +377,341 @@ void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, 
                       const u64* ab, u64* out, cudaStream_t s) {
   SV_LAUNCH(k_part_pack, div_up(std::max<u32>(cap, 1), 128), 128, 0, s)(part_off, nseg, cap, lanes, mm, ab, out);
 }
+
+// ==========================================================================================
+// Cell GROUPING by counting sort (the default path for G <= GROUP_MAXG): the KDE windows and the
+// part moments only need the values grouped by (segment, cell) -- the order inside a cell is
+// irrelevant (exact integer sums, see the header) -- so no stable radix ranking is needed.
+//   round 1   k_group_t3  : Tier-3 rows of the trace -> raw x grouped by segment (t3rank), at
+//                           bases known from pass A's local counts; one shared atomic per Tier-3
+//                           row and one global atomic per (tile, segment)
+//   each round, over chunks of <= GR_CH values of one segment's range:
+//             k_cell_hist : cell of every value (u16, 0xFFFF outside the segment's [lo, hi]) and
+//                           the chunk's per-cell counts
+//             k_cell_walk : per (segment, cell): offsets of the chunks inside the cell, cell total
+//             scan_u32    : off[s * G + c] = first position of cell c of segment s (packed)
+//             k_cell_scatter: values staged in shared memory in cell order, written out in runs
+// Traffic per value and round: 8 B read (hist) + 2 B cell write + (8 + 2) B read + 8 B write
+// (scatter), against 16 B per onesweep pass x 3 passes + 16 B for the radix path's cell keys.
+// ==========================================================================================
+#define GR_THREADS 512
+#define GR_CH 8192          // values per chunk (one block), 16 per thread
+#define GT_ROWS 16          // trace rows per thread per tile in k_group_t3
+#define GT_SMEM_MAX GROUP_T3_SMEM_MAX   // segments handled with a shared-memory counter table
+
+__global__ void __launch_bounds__(GR_THREADS)
+k_group_t3(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, const u32* __restrict__ t3rank,
+           u32 n_t3, const u32* __restrict__ seg_base, u32* __restrict__ cursor, u64* __restrict__ out) {
+  extern __shared__ u32 s_cnt[];      // [n_t3]: tile counts, then the tile's output bases
+  __shared__ u32 s_list[GR_THREADS * GT_ROWS];
+  __shared__ u32 s_nlist;
+  const bool smem = n_t3 <= GT_SMEM_MAX;
+  if (smem)
+    for (u32 i = threadIdx.x; i < n_t3; i += GR_THREADS) s_cnt[i] = 0;
+  if (threadIdx.x == 0) s_nlist = 0;
+  __syncthreads();
+  const u64 tile = (u64)GR_THREADS * GT_ROWS;
+  for (u64 base = (u64)blockIdx.x * tile; base < n; base += (u64)gridDim.x * tile) {
+    u32 t[GT_ROWS], r[GT_ROWS];
+    u64 v[GT_ROWS];
+#pragma unroll
+    for (int j = 0; j < GT_ROWS; j++) {   // all loads first
+      const u64 i = base + (u64)j * GR_THREADS + threadIdx.x;
+      const bool ok = i < n;
+      t[j] = ok ? __ldcs(kid + i) : 0u;
+      v[j] = ok ? __ldcs(x + i) : 0ull;
+      if (!ok) t[j] = 0xFFFFFFFFu;
+    }
+#pragma unroll
+    for (int j = 0; j < GT_ROWS; j++) {
+      if (t[j] != 0xFFFFFFFFu) t[j] = __ldg(t3rank + t[j]);
+      if (t[j] == 0xFFFFFFFFu) continue;
+      if (smem) {
+        r[j] = atomicAdd(&s_cnt[t[j]], 1u);
+        if (r[j] == 0) s_list[atomicAdd(&s_nlist, 1u)] = t[j];
+      } else {
+        r[j] = seg_base[t[j]] + atomicAdd(&cursor[t[j]], 1u);
+      }
+    }
+    if (smem) {
+      __syncthreads();
+      const u32 nl = s_nlist;
+      for (u32 q = threadIdx.x; q < nl; q += GR_THREADS) {  // reserve one range per segment
+        const u32 s = s_list[q];
+        s_cnt[s] = seg_base[s] + atomicAdd(&cursor[s], s_cnt[s]);
+      }
+      __syncthreads();
+#pragma unroll
+      for (int j = 0; j < GT_ROWS; j++)
+        if (t[j] != 0xFFFFFFFFu) out[s_cnt[t[j]] + r[j]] = v[j];
+      __syncthreads();
+      for (u32 q = threadIdx.x; q < nl; q += GR_THREADS) s_cnt[s_list[q]] = 0;
+      if (threadIdx.x == 0) s_nlist = 0;
+      __syncthreads();
+    } else {
+#pragma unroll
+      for (int j = 0; j < GT_ROWS; j++)
+        if (t[j] != 0xFFFFFFFFu) out[r[j]] = v[j];
+    }
+  }
+}
+
+// The default round-1 grouping (n_t3 <= GT_SMEM_MAX): blocks own fixed contiguous row ranges;
+// k_t3_count counts each block's Tier-3 rows per segment, k_t3_offsets turns the counts into
+// each (segment, block) output base, and k_t3_scatter writes every Tier-3 row at its block's
+// next position of its segment (a shared-memory atomic): no global atomics, no per-tile barriers.
+#define T3_THREADS 512
+#define T3_SC_THREADS 1024   // k_t3_scatter (one block per SM when it reuses pass A's row ranges)
+#define T3_U 8               // rows per thread in flight
+__device__ __forceinline__ void t3_range(u64 n, u32 nb, u32 b, u64* r0, u64* r1) {
+  const u64 chunk = (n + nb - 1) / nb;
+  *r0 = min(n, (u64)b * chunk);
+  *r1 = min(n, *r0 + chunk);
+}
+
+__global__ void __launch_bounds__(T3_THREADS)
+k_t3_count(const u32* __restrict__ kid, u64 n, const u32* __restrict__ t3rank, u32 n_t3, u32* __restrict__ cnt) {
+  extern __shared__ u32 s_c[];   // [n_t3]
+  for (u32 i = threadIdx.x; i < n_t3; i += T3_THREADS) s_c[i] = 0;
+  __syncthreads();
+  u64 r0, r1;
+  t3_range(n, gridDim.x, blockIdx.x, &r0, &r1);
+  for (u64 i0 = r0 + threadIdx.x; i0 < r1; i0 += (u64)T3_THREADS * T3_U) {
+    u32 k[T3_U];
+#pragma unroll
+    for (int u = 0; u < T3_U; u++) {
+      const u64 i = i0 + (u64)u * T3_THREADS;
+      k[u] = i < r1 ? __ldcs(kid + i) : 0xFFFFFFFFu;
+    }
+#pragma unroll
+    for (int u = 0; u < T3_U; u++) {
+      const u32 t = k[u] != 0xFFFFFFFFu ? __ldg(t3rank + k[u]) : 0xFFFFFFFFu;
+      if (t != 0xFFFFFFFFu) atomicAdd(&s_c[t], 1u);
+    }
+  }
+  __syncthreads();
+  for (u32 t = threadIdx.x; t < n_t3; t += T3_THREADS) cnt[(u64)t * gridDim.x + blockIdx.x] = s_c[t];
+}
+
+// one warp per segment: exclusive scan of its per-block counts, offset by the segment's base;
+// part != nullptr: the counts are pass A's per-block kernel counts (part[b * kt + kernel].n, the
+// same row ranges), t3kern[t] = the kernel of segment t
+__global__ void k_t3_offsets(u32* __restrict__ cnt, u32 nb, u32 n_t3, const u32* __restrict__ seg_base,
+                             const KMomPartial* __restrict__ part, u32 kt, const u32* __restrict__ t3kern) {
+  const u32 t = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (t >= n_t3) return;
+  u32 carry = seg_base[t];
+  u32* row = cnt + (u64)t * nb;
+  const u32 kk = part ? t3kern[t] : 0u;
+  for (u32 b0 = 0; b0 < nb; b0 += 32) {
+    const u32 b = b0 + lane_id();
+    const u32 v = b < nb ? (part ? part[(u64)b * kt + kk].n : row[b]) : 0u;
+    u32 inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const u32 q = __shfl_up_sync(0xffffffffu, inc, o);
+      if ((int)lane_id() >= o) inc += q;
+    }
+    if (b < nb) row[b] = carry + inc - v;
+    carry += __shfl_sync(0xffffffffu, inc, 31);
+  }
+}
+
+__global__ void __launch_bounds__(T3_SC_THREADS)
+k_t3_scatter(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, const u32* __restrict__ t3rank,
+             u32 n_t3, const u32* __restrict__ off, u64* __restrict__ out) {
+  extern __shared__ u32 s_cur[];   // [n_t3]: this block's next output position per segment
+  for (u32 t = threadIdx.x; t < n_t3; t += T3_SC_THREADS) s_cur[t] = off[(u64)t * gridDim.x + blockIdx.x];
+  __syncthreads();
+  u64 r0, r1;
+  t3_range(n, gridDim.x, blockIdx.x, &r0, &r1);
+  for (u64 i0 = r0 + threadIdx.x; i0 < r1; i0 += (u64)T3_SC_THREADS * T3_U) {
+    u32 t[T3_U];
+    u64 v[T3_U];
+#pragma unroll
+    for (int u = 0; u < T3_U; u++) {
+      const u64 i = i0 + (u64)u * T3_SC_THREADS;
+      t[u] = i < r1 ? __ldcs(kid + i) : 0xFFFFFFFFu;
+    }
+#pragma unroll
+    for (int u = 0; u < T3_U; u++) t[u] = t[u] != 0xFFFFFFFFu ? __ldg(t3rank + t[u]) : 0xFFFFFFFFu;
+    // x only for the Tier-3 rows: a 32-byte sector none of whose rows is Tier-3 is never read
+#pragma unroll
+    for (int u = 0; u < T3_U; u++) v[u] = t[u] != 0xFFFFFFFFu ? __ldcs(x + i0 + (u64)u * T3_SC_THREADS) : 0ull;
+#pragma unroll
+    for (int u = 0; u < T3_U; u++)
+      if (t[u] != 0xFFFFFFFFu) out[atomicAdd(&s_cur[t[u]], 1u)] = v[u];
+  }
+}
+
+size_t group_t3_temp_bytes(u32 n_t3) { return (size_t)n_t3 * sv_num_sms() * 4 * 4 + 256; }
+
+void launch_group_t3(const u32* kid, const u64* x, u64 n, const u32* t3rank, u32 n_t3, const u32* seg_base,
+                     u32* cursor, u64* out, void* temp, const KMomPartial* part, int part_grid, u32 part_kt,
+                     const u32* t3kern, cudaStream_t s) {
+  if (!n || !n_t3) return;
+  if (n_t3 <= GT_SMEM_MAX) {
+    // pass A's per-block kernel counts over the same row ranges, when the caller has them
+    const bool reuse = part && part_grid > 0;
+    const u32 nb = reuse ? (u32)part_grid
+                         : (u32)std::min<u64>((u64)sv_num_sms() * 4, (n + T3_THREADS - 1) / T3_THREADS);
+    u32* cnt = (u32*)temp;   // [n_t3][nb]
+    const size_t sm = (size_t)n_t3 * 4;
+    sv_smem_attr(k_t3_count, GT_SMEM_MAX * 4);
+    sv_smem_attr(k_t3_scatter, GT_SMEM_MAX * 4);
+    if (!reuse) SV_LAUNCH(k_t3_count, nb, T3_THREADS, sm, s)(kid, n, t3rank, n_t3, cnt);
+    SV_LAUNCH(k_t3_offsets, div_up((u64)n_t3 * 32, 256), 256, 0, s)(cnt, nb, n_t3, seg_base,
+                                                                    reuse ? part : nullptr, part_kt, t3kern);
+    SV_LAUNCH(k_t3_scatter, nb, T3_SC_THREADS, sm, s)(kid, x, n, t3rank, n_t3, cnt, out);
+    return;
+  }
+  // many Tier-3 kernels: global cursors (k_group_t3's global-atomic branch)
+  const u64 tiles = (n + (u64)GR_THREADS * GT_ROWS - 1) / ((u64)GR_THREADS * GT_ROWS);
+  const u64 grid = std::min<u64>(tiles, (u64)sv_num_sms() * 2);
+  SV_LAUNCH(k_group_t3, (u32)grid, GR_THREADS, 0, s)(kid, x, n, t3rank, n_t3, seg_base, cursor, out);
+}
+
+// per chunk: cells (u16) and the chunk's per-cell counts (hist[chunk * G + c]); the counts are
+// accumulated two cells per 32-bit word (a chunk holds <= GR_CH < 2^16 values)
+__global__ void __launch_bounds__(GR_THREADS)
+k_cell_hist(const BucketChunk* __restrict__ chunks, const u64* __restrict__ src, const SegDev* __restrict__ segs,
+            u32 G, unsigned short* __restrict__ cells, u32* __restrict__ hist, unsigned long long* inwin) {
+  extern __shared__ u32 s_h2[];       // [ceil(G / 2)]
+  const BucketChunk ch = chunks[blockIdx.x];
+  const u32 gw = (G + 1) / 2;
+  for (u32 i = threadIdx.x; i < gw; i += GR_THREADS) s_h2[i] = 0;
+  __syncthreads();
+  const SegDev g = segs[ch.seg];
+  const GridFn gf{__ull2double_rn(g.lo), __uint2double_rn(G - 1), g.hi - g.lo};
+  const double w = __dmul_rn(KDE_WC, g.h);
+  u64 win = 0;
+  for (u32 i = threadIdx.x; i < ch.len; i += GR_THREADS) {
+    const u64 x = __ldcs(src + ch.begin + i);
+    unsigned short c = 0xFFFFu;
+    if (x >= g.lo && x <= g.hi) {   // a superset range holds a neighbouring part's boundary cell
+      const u32 cc = cell_arith(gf, G, g.cq, g.lo, x);
+      c = (unsigned short)cc;
+      atomicAdd(&s_h2[cc >> 1], 1u << (16 * (cc & 1)));
+      if (inwin) win += inwin_count(gf, G, g.cq, w, x);
+    }
+    cells[(u64)blockIdx.x * GR_CH + i] = c;
+  }
+  __syncthreads();
+  u32* hc = hist + (u64)blockIdx.x * G;
+  for (u32 c = threadIdx.x; c < G; c += GR_THREADS) hc[c] = (s_h2[c >> 1] >> (16 * (c & 1))) & 0xFFFFu;
+  if (inwin) {
+    for (int o = 16; o > 0; o >>= 1) win += __shfl_down_sync(0xffffffffu, win, o);
+    if (lane_id() == 0 && win) atomicAdd(inwin, (unsigned long long)win);
+  }
+}
+
+// per (segment s, cell c): rel[chunk * G + c] = values of cell c in the earlier chunks of s,
+// tot[s * G + c] = all of them (one thread walks the segment's chunks; consecutive threads read
+// consecutive cells of a chunk)
+__global__ void k_cell_walk(const u32* __restrict__ seg_chunk, u32 nseg, u32 G, const u32* __restrict__ hist,
+                            u32* __restrict__ rel, u32* __restrict__ tot) {
+  const u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (id >= (u64)nseg * G) return;
+  const u32 s = (u32)(id / G), c = (u32)(id % G);
+  u32 run = 0;
+  for (u32 k = seg_chunk[s]; k < seg_chunk[s + 1]; k++) {
+    rel[(u64)k * G + c] = run;
+    run += hist[(u64)k * G + c];
+  }
+  tot[id] = run;
+}
+
+// exclusive prefix of v over a GR_THREADS block; *total receives the block sum
+__device__ __forceinline__ u32 block_excl_scan_u32(u32 v, u32* total) {
+  __shared__ u32 s_w[GR_THREADS / 32];
+  u32 inc = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const u32 t = __shfl_up_sync(0xffffffffu, inc, o);
+    if ((int)lane_id() >= o) inc += t;
+  }
+  const u32 w = threadIdx.x >> 5;
+  if (lane_id() == 31) s_w[w] = inc;
+  __syncthreads();
+  if (w == 0) {
+    const u32 t = lane_id() < GR_THREADS / 32 ? s_w[lane_id()] : 0u;
+    u32 ti = t;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const u32 q = __shfl_up_sync(0xffffffffu, ti, o);
+      if ((int)lane_id() >= o) ti += q;
+    }
+    if (lane_id() < GR_THREADS / 32) s_w[lane_id()] = ti - t;
+    if (lane_id() == GR_THREADS / 32 - 1) *total = ti;
+  }
+  __syncthreads();
+  const u32 r = s_w[w] + inc - v;
+  __syncthreads();
+  return r;
+}
+
+// per chunk: each value's destination = off[s * G + c] + rel[chunk][c] + its rank among the
+// chunk's values of cell c.  The chunk is first staged in shared memory in cell order (local
+// positions from a block scan of its counts), then written out so that consecutive threads
+// write consecutive addresses of one cell's run.
+__global__ void __launch_bounds__(GR_THREADS)
+k_cell_scatter(const BucketChunk* __restrict__ chunks, const u64* __restrict__ src,
+               const unsigned short* __restrict__ cells, u32 G, const u32* __restrict__ hist,
+               const u32* __restrict__ rel, const u32* __restrict__ off, u64* __restrict__ out) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  u64* s_v = (u64*)smem;                          // [GR_CH]
+  unsigned short* s_c = (unsigned short*)(s_v + GR_CH);   // [GR_CH]
+  u32* s_ls = (u32*)(s_c + GR_CH);                // [G]: local exclusive scan of the counts
+  u32* s_gb = s_ls + G;                           // [G]: global base of the chunk's cell run
+  u32* s_cur = s_gb + G;                          // [G]: rank counters
+  const BucketChunk ch = chunks[blockIdx.x];
+  const u32* hc = hist + (u64)blockIdx.x * G;
+  const u32* rc = rel + (u64)blockIdx.x * G;
+  const u32* oc = off + (u64)ch.seg * G;
+  // block-wide exclusive scan of the G counts (G / GR_THREADS per thread, then the block)
+  const u32 per = (G + GR_THREADS - 1) / GR_THREADS;
+  const u32 c0 = threadIdx.x * per;
+  u32 sum = 0;
+  for (u32 c = c0; c < c0 + per && c < G; c++) sum += hc[c];
+  __shared__ u32 tot;
+  u32 ex = block_excl_scan_u32(sum, &tot);
+  for (u32 c = c0; c < c0 + per && c < G; c++) {
+    s_ls[c] = ex;
+    ex += hc[c];
+    s_gb[c] = oc[c] + rc[c];
+    s_cur[c] = 0;
+  }
+  __syncthreads();
+  for (u32 i = threadIdx.x; i < ch.len; i += GR_THREADS) {
+    const unsigned short c = cells[(u64)blockIdx.x * GR_CH + i];
+    if (c == 0xFFFFu) continue;
+    const u32 p = s_ls[c] + atomicAdd(&s_cur[c], 1u);
+    s_v[p] = __ldcs(src + ch.begin + i);
+    s_c[p] = c;
+  }
+  __syncthreads();
+  for (u32 p = threadIdx.x; p < tot; p += GR_THREADS) {
+    const u32 c = s_c[p];
+    out[s_gb[c] + (p - s_ls[c])] = s_v[p];
+  }
+}
+
+size_t cell_scatter_smem(u32 G) { return (size_t)GR_CH * 10 + (size_t)G * 12; }
+
+void launch_cell_group(const BucketChunk* chunks, u32 nchunks, const u64* src, const SegDev* segs, u32 nseg,
+                       u32 G, const u32* seg_chunk, unsigned short* cells, u32* hist, u32* rel, u32* tot,
+                       u32* off, void* scan_temp, u64* out, unsigned long long* inwin, cudaStream_t s) {
+  const u64 ncell = (u64)nseg * G;
+  if (nchunks) {
+    const size_t hs = (size_t)(G + 1) / 2 * 4;
+    sv_smem_attr(k_cell_hist, (int)hs);
+    SV_LAUNCH(k_cell_hist, nchunks, GR_THREADS, hs, s)(chunks, src, segs, G, cells, hist, inwin);
+  }
+  SV_LAUNCH(k_cell_walk, div_up(ncell, 256), 256, 0, s)(seg_chunk, nseg, G, hist, rel, tot);
+  scan_u32(tot, off, ncell, scan_temp, off + ncell, s);
+  if (nchunks) {
+    const size_t ss = cell_scatter_smem(G);
+    sv_smem_attr(k_cell_scatter, (int)ss);
+    SV_LAUNCH(k_cell_scatter, nchunks, GR_THREADS, ss, s)(chunks, src, cells, G, hist, rel, off, out);
+  }
+}

@@ -119,6 +119,27 @@ void launch_cellkey(const BucketChunk* chunks, const u64* in, u64 nin, u32 bx, u
 // off[c] = first position of the idx-sorted keys with idx >= c, c = 0..ncell
 void launch_cell_offsets(const u64* keys, u64 n, u32 ib, u32 ncell, u32* off, cudaStream_t s);
 
+// ---- cell grouping by counting sort (bucket.cu; the default for G <= GROUP_MAXG) ----
+#define GROUP_MAXG 8192
+#define GROUP_CH 8192   // values per chunk (= GR_CH in bucket.cu)
+#define GROUP_T3_SMEM_MAX 16384   // Tier-3 kernels the round-1 grouping counts in shared memory
+// round 1: the Tier-3 rows' x grouped by t3rank at out[seg_base[t3rank] ...] (cursor zeroed)
+size_t group_t3_temp_bytes(u32 n_t3);
+// part (nullable): pass A's per-block partials of this trace (part_grid blocks x part_kt kernels,
+// every kernel in one pass), whose per-block counts then give the output bases directly;
+// t3kern[t] = the kernel of segment t (read only with part)
+void launch_group_t3(const u32* kid, const u64* x, u64 n, const u32* t3rank, u32 n_t3, const u32* seg_base,
+                     u32* cursor, u64* out, void* temp /* group_t3_temp_bytes(n_t3) */,
+                     const KMomPartial* part, int part_grid, u32 part_kt, const u32* t3kern, cudaStream_t s);
+// chunks (<= GROUP_CH values of one segment's source range each, the chunks of segment s are
+// seg_chunk[s] .. seg_chunk[s + 1] - 1) -> out grouped by (segment, cell) with
+// off[s * G + c] = first position of cell c of segment s, off[nseg * G] = values grouped
+// (values outside their segment's [lo, hi] are dropped); cells [nchunks * GROUP_CH], hist / rel
+// [nchunks * G], tot [nseg * G] scratch; *inwin += in-window KDE terms (nullable)
+void launch_cell_group(const BucketChunk* chunks, u32 nchunks, const u64* src, const SegDev* segs, u32 nseg,
+                       u32 G, const u32* seg_chunk, unsigned short* cells, u32* hist, u32* rel, u32* tot,
+                       u32* off, void* scan_temp, u64* out, unsigned long long* inwin, cudaStream_t s);
+
 // ---------------- valleys and thresholds (A11-A13) ---------------------------------------------
 // T[s*tstride + q], nt[s], kind[s] (1 = valley, 2 = bisect)
 void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T,
@@ -221,6 +242,9 @@ struct FillRegions { u64* p[FILL_MAX]; u64 n[FILL_MAX]; u64 v[FILL_MAX]; int k; 
 void launch_fill_multi(const FillRegions& r, cudaStream_t s);
 // SM-driven copy (device or pinned host memory on either side; no copy engine)
 void launch_copy(void* dst, const void* src, u64 bytes, cudaStream_t s);
+#define COPY_MAX 8
+struct CopyRegions { void* dst[COPY_MAX]; const void* src[COPY_MAX]; u64 bytes[COPY_MAX]; int k; };
+void launch_copy_multi(const CopyRegions& r, cudaStream_t s);
 // cross-rank encoding of u128 pairs [n][2] <-> 4 limbs [n][4]
 void launch_u128_to_limbs(const u64* src, u64 n, u64* limbs, cudaStream_t s);
 void launch_limbs_to_u128(const u64* limbs, u64 n, u64* dst, cudaStream_t s);

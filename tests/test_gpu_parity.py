@@ -54,6 +54,20 @@ def test_grid_sizes(G):
     assert_segments_equal(g["segments"], o.segments())
 
 
+@pytest.mark.parametrize("G,radix", [(1024, True), (10000, False)])
+def test_cell_radix_path(G, radix, monkeypatch):
+    """the onesweep cell-key path (forced by SIEVE_CELL_RADIX, and taken for G > GROUP_MAXG) gives
+    the same densities, cuts and strata as the grouped default"""
+    if radix:
+        monkeypatch.setenv("SIEVE_CELL_RADIX", "1")
+    tr = gen.make_trace("C2", n=150_000)
+    g = run_gpu(tr, G=G, keep_debug=True)
+    o = run_oracle(tr, G=G, keep_debug=True)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+    assert_segments_equal(g["segments"], o.segments())
+
+
 @pytest.mark.parametrize("theta", [(1, 10), (1, 2), (1, 1), (3, 7)])
 def test_theta_values(theta):
     tr = gen.make_trace("C2", n=100_000)
