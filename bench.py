@@ -360,7 +360,7 @@ def main():
 
     clk = ClockSampler(local)
     clk.start()
-    for _ in range(args.warmup):
+    for _ in range(max(1, args.warmup)):   # at least one: the table sizes below come from it
         st = step()
     n_strata = len(st)
     st_terms, kde_eval = st.kde_terms, st.kde_evaluated

@@ -277,7 +277,8 @@ uint64_t sieve_kernel_launches(void);
 /* ---- exact minimum number of strata (NEXT-3; reading A28) -------------- */
 /* P:89 asks the Tier-3 split to "(1) minimise the number of strata such that (2) the CoV of
    each stratum is below theta".  This diagnostic computes that optimum exactly, per kernel,
-   over runs of its sorted distinct instruction counts: f(0) = 0, f(j) = min f(i) + 1 over the
+   among strata that are value intervals (the only kind Sieve builds), i.e. over runs of its
+   sorted distinct instruction counts: f(0) = 0, f(j) = min f(i) + 1 over the
    runs (i, j] with CoV < theta (the exact u256 test of the tiering), ties -> smallest i.
      counts      HOST [num_kernels]: 0 = no invocations, 1 = Tier-1/2 (one valid stratum), the
                  optimum for Tier-3 kernels, UINT32_MAX = skipped (more than max_distinct

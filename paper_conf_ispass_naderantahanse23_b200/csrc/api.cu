@@ -134,6 +134,7 @@ struct sieve_ctx_s {
   // mapped (zero-copy) pinned host memory: kernels write each round's part results here
   u64* mapped = nullptr;
   size_t mapped_cap = 0;
+  u64* scan_state = nullptr;   // single-pass scans (sort.cu), zero-initialised at creation
   double hs_wait = 0, hs_between = 0;
   std::string hs_list;
   std::chrono::steady_clock::time_point hs_last{};
@@ -383,6 +384,12 @@ static int ctx_common(int dev, void* stream, sieve_ctx* out, sieve_ctx_s** c) {
   *c = new sieve_ctx_s();
   (*c)->device = dev;
   (*c)->stream = (cudaStream_t)stream;
+  void* st = nullptr;
+  const size_t sb = (SCAN_SP_MAX_TILES + 2) * sizeof(u64);
+  cudaError_t e = cudaMalloc(&st, sb);
+  if (e == cudaSuccess) e = cudaMemset(st, 0, sb);
+  if (e != cudaSuccess) { if (st) cudaFree(st); delete *c; return sv_cuda(e, "scan state", __LINE__); }
+  (*c)->scan_state = (u64*)st;
   return SIEVE_OK;
 }
 
@@ -442,6 +449,7 @@ extern "C" void sieve_ctx_destroy(sieve_ctx ctx) {
   for (void* p : ctx->pin_overflow) cudaFreeHost(p);
   if (ctx->pin) cudaFreeHost(ctx->pin);
   if (ctx->mapped) cudaFreeHost(ctx->mapped);
+  if (ctx->scan_state) cudaFree(ctx->scan_state);
   delete ctx->comm;
   ctx->magic = 0;
   delete ctx;
@@ -724,6 +732,12 @@ struct HostClock {
 };
 struct Fin { u32 kid, tier; u64 lo, hi, n; u128 s1; double h; u32 round; };
 
+// the calling thread's scans use this context's single-pass scan state for the call's duration
+struct ScanScope {
+  explicit ScanScope(sieve_ctx c) { scan_set_state(c->scan_state); }
+  ~ScanScope() { scan_set_state(nullptr); }
+};
+
 // pass A results on the host (replicated after AR-1): theta-independent, so a theta sweep or a
 // tier census computes them once
 struct MomentsHost {
@@ -806,6 +820,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   sieve_ctx c = t->ctx;
   cudaStream_t S = c->stream;
   SV_TRY(arena_reset(c));
+  ScanScope scan_scope(c);
   HostClock hc;
   hc.c = c;
   const u32 K = t->K, G = P->grid_points;
@@ -940,6 +955,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       hs[s].h = h;
       hs[s].inv_h = 1.0 / h;
       hs[s].cq = (double)(G - 1) / (double)(o.hi - o.lo);
+      hs[s].cm = cell_margin(o.lo, o.hi, G);
       u64 len = round == 1 ? h_localn[o.kid] : o.e - o.b;
       maxlen = std::max(maxlen, len);
       if (grouped) {  // every round reads each segment's contiguous source range [b, e)
@@ -1066,14 +1082,13 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       for (u32 s = 0; s < nseg; s++)
         if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 140.0 * hs[s].h) guard = true;
       launch_kde(segs.get(), nseg, G, ck.get(), vsh, tile_range.get(), tile_items.get(),
-                 item_tile.get(), items, D.get(), terms.get() + 1, guard, !c->comm, S);
+                 item_tile.get(), items, D.get(), terms.get() + 1, guard, false, S);
       tm.stop();
       SV_CUDA(cudaGetLastError());
     }
-    if (c->comm) {  // AR-2: the densities' two u64 lanes per grid point (16 B), then normalise
-      SV_TRY(allreduce(c, D.get(), (size_t)nseg * G * 2, RED_SUM));
-      launch_kde_fix(D.get(), (u64)nseg * G, S);
-    }
+    // AR-2: the densities' two u64 lanes per grid point (16 B), summed as the KDE left them;
+    // k_valleys normalises them to u128
+    if (c->comm) SV_TRY(allreduce(c, D.get(), (size_t)nseg * G * 2, RED_SUM));
     DBuf<u64> T(c);
     DBuf<u32> ntk(c), d_off(c);
     SV_TRY(T.alloc((size_t)nseg * tstride));
@@ -1081,21 +1096,20 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     SV_TRY(d_off.alloc(nseg + 1));
     PhaseTimer tv(c, SIEVE_PHASE_REFINE, 0);
     launch_valleys(segs.get(), nseg, G, P->valley_shift, D.get(), T.get(), tstride, ntk.get(),
-                   ntk.get() + nseg, S);
+                   ntk.get() + nseg, R->keep_debug, S);
     launch_part_offsets(ntk.get(), nseg, d_off.get(), S);
     tv.stop();
     // Part moments (AR-3 as one grouped step: SUM of the limb lanes, MAX of the complemented
     // mins and of the maxes), packed into mapped host memory: ONE host synchronisation per round
     // at any rank count.
-    std::vector<u32> h_ntk;
+    std::vector<u32> h_ntk(2 * (size_t)nseg);   // cut counts and split kinds, from the part records
     std::vector<u64> h_D, h_T;
-    CopyBatch ecb(c);   // read back with the part records at the round's synchronisation
-    SV_TRY(ecb.add_d2h(h_ntk, ntk.get(), (size_t)nseg * 2));
     if (R->keep_debug) {
+      CopyBatch ecb(c);   // read back with the part records at the round's synchronisation
       SV_TRY(ecb.add_d2h(h_D, D.get(), (size_t)nseg * G * 2));
       SV_TRY(ecb.add_d2h(h_T, T.get(), (size_t)nseg * tstride));
+      SV_TRY(ecb.flush());
     }
-    SV_TRY(ecb.flush());
     u64 *hrec = nullptr, *drec = nullptr;
     for (int pass = 0;; pass++) {
       DBuf<u32> pitems(c);
@@ -1113,12 +1127,17 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         SV_TRY(allreduce_group(c, {{pl.get(), (size_t)cap * MOM_LANES, RED_SUM}, {pm.get(), (size_t)cap * 2, RED_MAX}}));
         launch_complement(pm.get(), cap, 1, S);
       }
-      SV_TRY(mapped_get(c, (1 + (size_t)cap * PART_REC) * 8, &hrec, &drec));
-      launch_part_pack(d_off.get(), nseg, cap, pl.get(), pm.get(), pab.get(), drec, S);
+      SV_TRY(mapped_get(c, (1 + (size_t)cap * PART_REC + nseg) * 8, &hrec, &drec));
+      launch_part_pack(d_off.get(), nseg, cap, pl.get(), pm.get(), pab.get(), ntk.get(), drec, S);
       hc.mark("p");
       SV_TRY(sync(c));
       hc.mark("ps");
       const u64 live = hrec[0];  // replicated: every rank computed the same cuts from the same D
+      for (u32 q = 0; q < nseg; q++) {
+        const u64 w = hrec[1 + (size_t)cap * PART_REC + q];
+        h_ntk[q] = (u32)w;
+        h_ntk[nseg + q] = (u32)(w >> 32);
+      }
       if (live <= cap) break;
       if (pass > 0) return sv_fail(SIEVE_ESTATE, "internal: part count grew");
       cap = (u32)live;  // more parts than slots: redo this round's part moments with the exact count

@@ -29,8 +29,8 @@
 #define AS_FLUSH (3 * AS_HC / 4)      // flush to the L2 table when this full
 #define AS_MAXP 32          // probes before falling back to the global table
 #ifndef AS_CHECK
-#define AS_CHECK 16         // tiles between the block barriers that check the table's fill (A/B on C4:
-                            // every tile 0.73 ms, every 4 tiles 0.60, every 16 tiles 0.55)
+#define AS_CHECK 32         // tiles between the block barriers that check the table's fill (A/B on C4:
+                            // every tile 0.73 ms, every 4 tiles 0.60, 16: 0.55, 32: 0.54, 128: 0.53)
 #endif
 
 // One block per SM with a large table: a block's contiguous chunk sees nearly every (stratum,

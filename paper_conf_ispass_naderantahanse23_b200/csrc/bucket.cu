@@ -360,11 +360,15 @@ void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, 
 // the round's results in one record per live part, written straight into mapped (zero-copy)
 // host memory: out[0] = number of parts, then per part {lanes[9], min, max, ia, ib}
 __global__ void k_part_pack(const u32* __restrict__ part_off, u32 nseg, u32 cap, const u64* __restrict__ lanes,
-                            const u64* __restrict__ mm, const u64* __restrict__ ab, u64* out) {
+                            const u64* __restrict__ mm, const u64* __restrict__ ab, const u32* __restrict__ ntk,
+                            u64* out) {
   const u32 nparts = part_off[nseg];
   u32 p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p == 0) out[0] = nparts;
-  if (p >= nparts) return;
+  // per segment: cut count and split kind (after the cap part slots)
+  for (u32 q = p; q < nseg; q += gridDim.x * blockDim.x)
+    out[1 + (u64)cap * PART_REC + q] = (u64)ntk[q] | ((u64)ntk[nseg + q] << 32);
+  if (p >= nparts || p >= cap) return;
   u64* o = out + 1 + (u64)p * PART_REC;
   for (int k = 0; k < MOM_LANES; k++) o[k] = lanes[(u64)p * MOM_LANES + k];
   o[MOM_LANES] = mm[p];
@@ -374,8 +378,9 @@ __global__ void k_part_pack(const u32* __restrict__ part_off, u32 nseg, u32 cap,
 }
 
 void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, const u64* mm,
-                      const u64* ab, u64* out, cudaStream_t s) {
-  SV_LAUNCH(k_part_pack, div_up(std::max<u32>(cap, 1), 128), 128, 0, s)(part_off, nseg, cap, lanes, mm, ab, out);
+                      const u64* ab, const u32* ntk, u64* out, cudaStream_t s) {
+  SV_LAUNCH(k_part_pack, div_up(std::max<u32>(std::max(cap, nseg), 1), 128), 128, 0, s)(part_off, nseg, cap, lanes,
+                                                                                    mm, ab, ntk, out);
 }
 
 // ==========================================================================================
@@ -585,11 +590,26 @@ k_cell_hist(const BucketChunk* __restrict__ chunks, const u64* __restrict__ src,
   const GridFn gf{__ull2double_rn(g.lo), __uint2double_rn(G - 1), g.hi - g.lo};
   const double w = __dmul_rn(KDE_WC, g.h);
   u64 win = 0;
-  for (u32 i = threadIdx.x; i < ch.len; i += GR_THREADS) {
-    const u64 x = __ldcs(src + ch.begin + i);
+  u64 xv[GR_CH / GR_THREADS];
+#pragma unroll
+  for (int q = 0; q < GR_CH / GR_THREADS; q++) {   // the thread's loads first
+    const u32 i = threadIdx.x + q * GR_THREADS;
+    xv[q] = i < ch.len ? __ldcs(src + ch.begin + i) : 0ull;
+  }
+#pragma unroll
+  for (int q = 0; q < GR_CH / GR_THREADS; q++) {
+    const u32 i = threadIdx.x + q * GR_THREADS;
+    if (i >= ch.len) continue;
+    const u64 x = xv[q];
     unsigned short c = 0xFFFFu;
     if (x >= g.lo && x <= g.hi) {   // a superset range holds a neighbouring part's boundary cell
-      const u32 cc = cell_arith(gf, G, g.cq, g.lo, x);
+      // fast path: the estimate is far enough from both neighbouring grid points (SegDev.cm) to
+      // decide the cell without evaluating them; else the exact search on the grid
+      const double e = __dmul_rn(__ull2double_rn(x - g.lo), g.cq);
+      const double jf = floor(e);
+      const double f = e - jf;   // exact: e and jf share the binade's ulp grid
+      const u32 cc = (f > g.cm && f < 1.0 - g.cm && jf < (double)(G - 1)) ? (u32)jf
+                                                                         : cell_arith(gf, G, g.cq, g.lo, x);
       c = (unsigned short)cc;
       atomicAdd(&s_h2[cc >> 1], 1u << (16 * (cc & 1)));
       if (inwin) win += inwin_count(gf, G, g.cq, w, x);
@@ -682,11 +702,21 @@ k_cell_scatter(const BucketChunk* __restrict__ chunks, const u64* __restrict__ s
     s_cur[c] = 0;
   }
   __syncthreads();
-  for (u32 i = threadIdx.x; i < ch.len; i += GR_THREADS) {
-    const unsigned short c = cells[(u64)blockIdx.x * GR_CH + i];
+  // all of the thread's loads first (GR_CH / GR_THREADS values), then the shared-memory placement
+  u64 xv[GR_CH / GR_THREADS];
+  unsigned short cv[GR_CH / GR_THREADS];
+#pragma unroll
+  for (int q = 0; q < GR_CH / GR_THREADS; q++) {
+    const u32 i = threadIdx.x + q * GR_THREADS;
+    cv[q] = i < ch.len ? cells[(u64)blockIdx.x * GR_CH + i] : (unsigned short)0xFFFFu;
+    xv[q] = cv[q] != 0xFFFFu ? __ldcs(src + ch.begin + i) : 0ull;
+  }
+#pragma unroll
+  for (int q = 0; q < GR_CH / GR_THREADS; q++) {
+    const unsigned short c = cv[q];
     if (c == 0xFFFFu) continue;
     const u32 p = s_ls[c] + atomicAdd(&s_cur[c], 1u);
-    s_v[p] = __ldcs(src + ch.begin + i);
+    s_v[p] = xv[q];
     s_c[p] = c;
   }
   __syncthreads();

@@ -57,6 +57,10 @@ u64* radix_sort_keys_input(u64* keys, u64 n, int nbits, void* temp);
 u32* radix_sort_prepare(u64 n, bool with_vals, int nbits, void* temp, cudaStream_t s);
 
 void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s);
+// the calling thread's single-pass scan state (a context's persistent, zero-initialised buffer of
+// SCAN_SP_MAX_TILES + 2 words; nullptr: three-kernel scans).  Set by the API entry points.
+#define SCAN_SP_MAX_TILES 4096
+void scan_set_state(u64* state);
 size_t scan_u32_temp_bytes(u64 n);
 
 // ---------------- KDE over open segments ([8], [36]; A6-A10) -----------------------------
@@ -64,7 +68,19 @@ struct SegDev {
   u64 lo, hi;   // value range [lo, hi] (global, replicated)
   double h, inv_h;
   double cq;    // (G - 1) / (hi - lo): cell estimate (made exact against the grid table)
+  double cm;    // margin in cell units: an estimate e = rn(rn(x - lo) * cq) with
+                // j + cm < e < j + 1 - cm (j < G - 1) proves g_j <= x < g_{j+1} (cell_fast)
 };
+// host: cm for segment [lo, hi] on a G-point grid (>= 1 disables the fast path).  With
+// E = (x - lo)(G - 1)/(hi - lo) exact, |e - E| <= G 2^-52 (two roundings) and every grid point
+// in cell units is within (hi + 1)(G - 1) 2^-51 / (hi - lo) of its index (A9: the product
+// (hi - lo) j rounded, one division, one addition), so e in (j + cm, j + 1 - cm) puts E strictly
+// between g_j and g_{j+1} (the grid is non-decreasing); cm doubles that bound.
+inline double cell_margin(u64 lo, u64 hi, u32 G) {
+  if (hi <= lo) return 2.0;
+  const double m = 2.0 * ((double)G * 0x1p-52 + ((double)hi + 1.0) * (double)(G - 1) * 0x1p-51 / (double)(hi - lo));
+  return m < 0.25 ? m : 2.0;
+}
 #define KDE_WC 7.54983443527075   // sqrt(57): |z| <= this <=> t <= 28.5 (in-window term count)
 #ifndef KDE_TJ
 #define KDE_TJ 32       // grid points per tile (32: one point per lane; 16: two value slices)
@@ -142,8 +158,10 @@ void launch_cell_group(const BucketChunk* chunks, u32 nchunks, const u64* src, c
 
 // ---------------- valleys and thresholds (A11-A13) ---------------------------------------------
 // T[s*tstride + q], nt[s], kind[s] (1 = valley, 2 = bisect)
-void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T,
-                    u32 tstride, u32* nt, u32* kind, cudaStream_t s);
+// D as the KDE leaves it (two u64 lanes per grid point: low-limb sum, rest); normalised to u128
+// in place when keep_D (debug read-back) or when G is too large to stage in shared memory
+void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, u64* D, u64* T,
+                    u32 tstride, u32* nt, u32* kind, bool keep_D, cudaStream_t s);
 
 // ---------------- part moments (A13 f) ----------------------------------------------------------
 // parts of segment s: q = 0..nt[s]; part_off[s] = first part index (exclusive scan of nt + 1, on
@@ -159,9 +177,10 @@ void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, 
 #define PART_REC (MOM_LANES + 4)
 #define PART_GUESS 16   // part slots per open segment before the exact count is known (a round
                         // with more parts redoes its part moments once with the exact count)
-// out[0] = parts, out[1 + p * PART_REC ..] = {lanes[9], min, max, ia, ib} (mapped host memory)
+// out[0] = parts, out[1 + p * PART_REC ..] = {lanes[9], min, max, ia, ib} (p < cap),
+// out[1 + cap * PART_REC + s] = nt[s] | kind[s] << 32 (ntk = [nt | kind]); mapped host memory
 void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, const u64* mm,
-                      const u64* ab, u64* out, cudaStream_t s);
+                      const u64* ab, const u32* ntk, u64* out, cudaStream_t s);
 // ---------------- pass B: assignment + per-(stratum, CTA) statistics -------------------
 struct KTab {      // per kernel
   u32 base;        // global id of its first stratum

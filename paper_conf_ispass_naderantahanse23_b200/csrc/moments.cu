@@ -30,6 +30,9 @@
 #define MOM_L2 6                              // limbs of x^2 (88 bits)
 #define MOM_WORDS (1 + MOM_L1 + MOM_L2)       // count + limbs, u32 each
 
+#ifndef MOM_MMTEST
+#define MOM_MMTEST 0
+#endif
 #ifndef MOM_AGG
 #define MOM_AGG 0                             // 1: warp-aggregate rows of equal kernels (A/B)
 #endif
@@ -39,7 +42,18 @@
 #endif
 
 int moments_kt(u32 K) { return (int)(K < MOM_KT ? K : MOM_KT); }
-static size_t moments_smem(u32 kt) { return (size_t)kt * (16 + 4 * MOM_WORDS); }
+// words between the two copies of the limb table: MOM_WORDS * kt rounded so that it is 16 mod 32
+// (the copies' words for one kernel sit in opposite halves of the 32 banks)
+__host__ __device__ inline u32 mom_copy_stride(u32 kt) {
+  const u32 w = MOM_WORDS * kt;
+  return w + ((16u - (w & 31u)) & 31u);
+}
+static size_t moments_smem(u32 kt, u32 nrep) { return (size_t)kt * 16 + (size_t)nrep * mom_copy_stride(kt) * 4; }
+#ifndef MOM_REP
+#define MOM_REP 2
+#endif
+#define MOM_SMEM_MAX (227 * 1024 - 2048)   // dynamic shared memory of one block (static part aside)
+static u32 moments_nrep(u32 kt) { return MOM_REP >= 2 && moments_smem(kt, 2) <= MOM_SMEM_MAX ? 2u : 1u; }
 
 __device__ __forceinline__ void atomic_min_u64_smem(u64* p, u64 v) {
   u64 cur = *(volatile u64*)p;
@@ -60,18 +74,23 @@ __device__ __forceinline__ void atomic_max_u64_smem(u64* p, u64 v) {
 
 __global__ void __launch_bounds__(MOM_THREADS, MOM_MINB)
 k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __restrict__ y,
-          u64 n, u32 K, u32 k0, u32 kt, KMomPartial* __restrict__ part,
+          u64 n, u32 K, u32 k0, u32 kt, u32 nrep, KMomPartial* __restrict__ part,
           u64* __restrict__ blk_tot, u64* errflags) {
   extern __shared__ __align__(16) unsigned char smem[];
   u64* s_mn = (u64*)smem;                 // [kt]
   u64* s_mx = s_mn + kt;                  // [kt]
-  u32* s_w = (u32*)(s_mx + kt);           // [MOM_WORDS][kt]: count, x limbs, x^2 limbs
+  u32* s_w = (u32*)(s_mx + kt);           // nrep x [MOM_WORDS][kt]: count, x limbs, x^2 limbs
+  // nrep = 2: lanes 16..31 add into a second copy of the limb table, half a bank row away, so a
+  // kernel that appears in both halves of a warp costs two parallel atomics, not two serial ones
+  // (same-address collisions of Zipf-hot kernels dominated the shared-atomic wavefronts)
+  const u32 cs = mom_copy_stride(kt);
   KMomPartial* rec = part + (u64)blockIdx.x * kt;
   for (u32 i = threadIdx.x; i < kt; i += blockDim.x) {
     s_mn[i] = ~0ull;
     s_mx[i] = 0;
+    for (u32 r = 0; r < nrep; r++)
 #pragma unroll
-    for (int w = 0; w < MOM_WORDS; w++) s_w[w * kt + i] = 0;
+      for (int w = 0; w < MOM_WORDS; w++) s_w[r * cs + w * kt + i] = 0;
     KMomPartial z = {0, 0, 0, 0, 0, 0, 0};
     rec[i] = z;
   }
@@ -120,11 +139,12 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
     return;
 #endif
     if (l >= kt || v == 0 || v >= SIEVE_X_LIMIT) return;
-    atomicAdd(&s_w[l], 1u);
+    u32* const sw = s_w + ((nrep == 2 && (lane_id() & 16u)) ? cs : 0u);
+    atomicAdd(&sw[l], 1u);
 #pragma unroll
     for (int i = 0; i < MOM_L1; i++) {
       u32 limb = (u32)(v >> (MOM_LB * i)) & MOM_LMASK;
-      if (limb) atomicAdd(&s_w[(1 + i) * kt + l], limb);
+      if (limb) atomicAdd(&sw[(1 + i) * kt + l], limb);
     }
     u64 sqlo = v * v, sqhi = __umul64hi(v, v);
 #pragma unroll
@@ -132,29 +152,38 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
       int sh = MOM_LB * i;
       u64 bits = sh < 64 ? ((sqlo >> sh) | (sh ? (sqhi << (64 - sh)) : 0ull)) : (sqhi >> (sh - 64));
       u32 limb = (u32)bits & MOM_LMASK;
-      if (limb) atomicAdd(&s_w[(1 + MOM_L1 + i) * kt + l], limb);
+      if (limb) atomicAdd(&sw[(1 + MOM_L1 + i) * kt + l], limb);
     }
+#if MOM_MMTEST  // timing probe only (wrong min / max): 32-bit fire-and-forget min / max of x >> 12
+    atomicMin((u32*)&s_mn[l], (u32)(v >> 12));
+    atomicMax((u32*)&s_mx[l], (u32)(v >> 12));
+#else
     atomic_min_u64_smem(&s_mn[l], v);
     atomic_max_u64_smem(&s_mx[l], v);
+#endif
   };
 
   auto flush = [&]() {
     __syncthreads();
     for (u32 i = threadIdx.x; i < kt; i += blockDim.x) {
-      u32 c = s_w[i];
+      u32 c = 0;
+      for (u32 r = 0; r < nrep; r++) c += s_w[r * cs + i];
       if (!c) continue;
       u128 s1 = 0, s2 = 0;
+      for (u32 r = 0; r < nrep; r++) {
+        u32* sw = s_w + r * cs;
 #pragma unroll
-      for (int j = 0; j < MOM_L1; j++) {
-        s1 += (u128)s_w[(1 + j) * kt + i] << (MOM_LB * j);
-        s_w[(1 + j) * kt + i] = 0;
-      }
+        for (int j = 0; j < MOM_L1; j++) {
+          s1 += (u128)sw[(1 + j) * kt + i] << (MOM_LB * j);
+          sw[(1 + j) * kt + i] = 0;
+        }
 #pragma unroll
-      for (int j = 0; j < MOM_L2; j++) {
-        s2 += (u128)s_w[(1 + MOM_L1 + j) * kt + i] << (MOM_LB * j);
-        s_w[(1 + MOM_L1 + j) * kt + i] = 0;
+        for (int j = 0; j < MOM_L2; j++) {
+          s2 += (u128)sw[(1 + MOM_L1 + j) * kt + i] << (MOM_LB * j);
+          sw[(1 + MOM_L1 + j) * kt + i] = 0;
+        }
+        sw[i] = 0;
       }
-      s_w[i] = 0;
       KMomPartial r = rec[i];
       u128 a1 = (((u128)r.s1hi << 64) | r.s1lo) + s1;
       u128 a2 = (((u128)r.s2hi << 64) | r.s2lo) + s2;
@@ -254,9 +283,9 @@ int moments_grid(u32 kt) {
   cudaGetDevice(&dev);
   int* e = cache[dev & 63];
   if (e[0] != (int)kt || e[1] < 1) {
-    sv_smem_attr(k_moments, (int)moments_smem(MOM_KT));
+    sv_smem_attr(k_moments, MOM_SMEM_MAX);
     int per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_moments, MOM_THREADS, moments_smem(kt));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_moments, MOM_THREADS, moments_smem(kt, moments_nrep(kt)));
     e[0] = (int)kt;
     e[1] = per_sm < 1 ? 1 : per_sm;
   }
@@ -265,8 +294,10 @@ int moments_grid(u32 kt) {
 
 void launch_moments(const u32* kid, const u64* x, const u64* y, u64 n, u32 K, u32 k0, u32 kt,
                     KMomPartial* part, u64* blk_tot, u64* errflags, int grid, cudaStream_t s) {
-  sv_smem_attr(k_moments, (int)moments_smem(MOM_KT));
-  SV_LAUNCH(k_moments, grid, MOM_THREADS, moments_smem(kt), s)(kid, x, y, n, K, k0, kt, part, blk_tot, errflags);
+  sv_smem_attr(k_moments, MOM_SMEM_MAX);
+  const u32 nrep = moments_nrep(kt);
+  SV_LAUNCH(k_moments, grid, MOM_THREADS, moments_smem(kt, nrep), s)(kid, x, y, n, K, k0, kt, nrep, part, blk_tot,
+                                                                     errflags);
 }
 
 // one warp per kernel: the lanes stride over the blocks' partials, exact u128 sums reduced by

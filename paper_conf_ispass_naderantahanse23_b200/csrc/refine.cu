@@ -143,20 +143,26 @@ __device__ u32 valley_warp(const u64* src, u32 G, u64 mx, u32 shift, const SegDe
 #define VAL_WARPS 4
 #define VAL_GMAX 2048   // segments with more grid points fall back to reading D from global memory
 __global__ void __launch_bounds__(32 * VAL_WARPS)
-k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, u32 tstride,
-          u32* nt, u32* kind) {
+k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, u64* D, u64* T, u32 tstride,
+          u32* nt, u32* kind, bool writeback) {
   extern __shared__ __align__(16) unsigned char vsm[];
   u32 w = threadIdx.x >> 5;
   u32 s = blockIdx.x * VAL_WARPS + w;
   if (s >= nseg) return;
-  const u64* d = D + 2 * (u64)s * G;
+  u64* d = D + 2 * (u64)s * G;
   const bool staged = G <= VAL_GMAX;
   u64* sd = (u64*)vsm + (u64)w * 2 * G;
-  // stage + max over the segment (warp reduction on u128 as (hi, lo))
+  // The KDE leaves D_j as two u64 lanes (sum of the low 32-bit limbs, sum of the rest), summed
+  // across ranks as they are: normalise to u128 here, stage, and reduce the maximum (warp
+  // reduction on u128 as (hi, lo)).  The normalised D goes back to global memory when it is read
+  // from there (large G) or read back (keep_debug).
   u128 mx = 0;
   for (u32 j = lane_id(); j < G; j += 32) {
-    u64 lo = d[2 * j], hi = d[2 * j + 1];
+    const u64 a = d[2 * j], b = d[2 * j + 1];
+    const u64 lo = a + (b << 32);
+    const u64 hi = (b >> 32) + (lo < a);
     if (staged) { sd[2 * j] = lo; sd[2 * j + 1] = hi; }
+    if (writeback) { d[2 * j] = lo; d[2 * j + 1] = hi; }
     u128 v = ((u128)hi << 64) | lo;
     mx = v > mx ? v : mx;
   }
@@ -185,11 +191,11 @@ k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T, 
   kind[s] = k;
 }
 
-void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, const u64* D, u64* T,
-                    u32 tstride, u32* nt, u32* kind, cudaStream_t s) {
+void launch_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, u64* D, u64* T,
+                    u32 tstride, u32* nt, u32* kind, bool keep_D, cudaStream_t s) {
   if (!nseg) return;
   size_t smem = G <= VAL_GMAX ? (size_t)VAL_WARPS * 2 * G * 8 : 0;
   sv_smem_attr(k_valleys, (int)((size_t)VAL_WARPS * 2 * VAL_GMAX * 8));
   SV_LAUNCH(k_valleys, div_up(nseg, VAL_WARPS), 32 * VAL_WARPS, smem, s)(segs, nseg, G, shift, D, T,
-                                                                  tstride, nt, kind);
+                                                                  tstride, nt, kind, keep_D || G > VAL_GMAX);
 }

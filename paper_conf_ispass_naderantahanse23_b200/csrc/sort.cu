@@ -147,11 +147,94 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_single(const u32* in, u64 n
 
 size_t scan_u32_temp_bytes(u64 n) { return ((n + SC_TILE - 1) / SC_TILE + 2) * sizeof(u32); }
 
+// look-back status words: GPU-scope relaxed accesses (served by L2; volatile would be
+// system scope).  Each word is written whole, so a reader sees either 0 or a complete value.
+__device__ __forceinline__ u64 ld_volatile_u64(const u64* p) {
+  u64 v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_volatile_u64(u64* p, u64 v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// ------------------------------------------------------------------------------------------
+// single-pass scan (one launch instead of three): tiles taken from a ticket counter, decoupled
+// look-back over 64-bit status words (2 flag bits + 62-bit sum).  The status words, the ticket
+// and the done counter live in a per-context persistent buffer that starts zeroed and is
+// re-zeroed by the last tile to finish, so no memset is launched.
+// ------------------------------------------------------------------------------------------
+#define SP_FLAG_AGG (1ull << 62)
+#define SP_FLAG_PRE (2ull << 62)
+#define SP_VAL ((1ull << 62) - 1)
+static thread_local u64* tl_scan_state = nullptr;   // [SCAN_SP_MAX_TILES + 2] on the device
+void scan_set_state(u64* state) { tl_scan_state = state; }
+
+__global__ void __launch_bounds__(SC_THREADS) k_scan_sp(const u32* in, u32* out, u64 n, u32 ntiles, u64* st,
+                                                        u32* total) {
+  __shared__ u32 s_tile;
+  __shared__ u64 s_excl;
+  __shared__ bool s_last;
+  unsigned int* ticket = (unsigned int*)(st + SCAN_SP_MAX_TILES);
+  unsigned int* done = ticket + 1;
+  if (threadIdx.x == 0) s_tile = atomicAdd(ticket, 1u);
+  __syncthreads();
+  const u32 tile = s_tile;
+  const u64 base = (u64)tile * SC_TILE + (u64)threadIdx.x * SC_IPT;
+  u32 v[SC_IPT];
+  u32 sum = 0;
+#pragma unroll
+  for (int j = 0; j < SC_IPT; j++) {
+    v[j] = base + j < n ? in[base + j] : 0;
+    sum += v[j];
+  }
+  __shared__ u32 tot;
+  u32 ex = block_excl_scan<u32, SC_THREADS>(sum, &tot);
+  if (threadIdx.x == 0) {
+    u64 excl = 0;
+    if (tile == 0) {
+      st_volatile_u64(st, SP_FLAG_PRE | tot);
+    } else {
+      st_volatile_u64(st + tile, SP_FLAG_AGG | tot);
+      for (int j = (int)tile - 1; j >= 0; j--) {
+        u64 w;
+        do { w = ld_volatile_u64(st + j); } while ((w >> 62) == 0);
+        excl += w & SP_VAL;
+        if (w & SP_FLAG_PRE) break;
+      }
+      st_volatile_u64(st + tile, SP_FLAG_PRE | (excl + tot));
+    }
+    s_excl = excl;
+    if (tile == ntiles - 1 && total) *total = (u32)(excl + tot);
+  }
+  __syncthreads();
+  u32 run = (u32)s_excl + ex;
+#pragma unroll
+  for (int j = 0; j < SC_IPT; j++) {
+    if (base + j < n) out[base + j] = run;
+    run += v[j];
+  }
+  // the last tile to finish (every look-back is over by then) re-zeroes the state
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(done, 1u) == ntiles - 1;
+  }
+  __syncthreads();
+  if (s_last) {
+    for (u32 j = threadIdx.x; j < ntiles; j += SC_THREADS) st[j] = 0;
+    if (threadIdx.x == 0) { *ticket = 0; *done = 0; }
+  }
+}
+
 // exclusive scan in -> out (may alias); total (device pointer, nullable) receives the sum
 void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream_t s) {
   u32 nb = div_up(n ? n : 1, SC_TILE);
   if (nb <= SC_SMALL) {
     SV_LAUNCH(k_scan_single, 1, SC_THREADS, 0, s)(in, n, out, total);
+    return;
+  }
+  if (tl_scan_state && nb <= SCAN_SP_MAX_TILES) {
+    SV_LAUNCH(k_scan_sp, nb, SC_THREADS, 0, s)(in, out, n, nb, tl_scan_state, total);
     return;
   }
   u32* bsum = (u32*)temp;
@@ -250,17 +333,6 @@ k_os_hist(const u64* __restrict__ keys, u64 n, int npass, u64 kmask, u32* __rest
     for (int t = 0; t < tables; t++) s += s_hist[t * npass * 256 + i];
     if (s) atomicAdd(&ghist[i], s);
   }
-}
-
-// look-back status words: GPU-scope relaxed accesses (served by L2; volatile would be
-// system scope).  Each word is written whole, so a reader sees either 0 or a complete value.
-__device__ __forceinline__ u64 ld_volatile_u64(const u64* p) {
-  u64 v;
-  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_volatile_u64(u64* p, u64 v) {
-  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
 template <bool V>  // V: a u32 payload travels with each key
