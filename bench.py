@@ -72,7 +72,9 @@ TRAFFIC_KERNELS = {
     "k_kde": None,
     "k_moments": 20,          # kid 4 + x 8 + y 8 (pass A)
     "k_assign": 20,           # kid 4 + x 8 + cta 4 in, sid 4 out (pass B)
-    "k_t3_compact": 12,       # kid 4 + x 8 in (+ 8 B per Tier-3 key out, reported separately)
+    "k_t3_scatter": None,     # kid 4 per invocation + x 8 in / 8 out per Tier-3 row (round-1 grouping)
+    "k_cell_hist": None,      # per open value and round: x 8 in, cell 2 out
+    "k_cell_scatter": None,   # per open value and round: x 8 + cell 2 in, x 8 out
 }
 
 

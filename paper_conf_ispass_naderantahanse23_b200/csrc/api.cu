@@ -522,46 +522,6 @@ extern "C" void sieve_trace_free(sieve_trace t) {
 // ------------------------------------------------------------------------------------------
 // exact host arithmetic for the replicated decisions
 // ------------------------------------------------------------------------------------------
-struct W256 { u64 w[4]; };  // little-endian words
-
-static W256 w256_mul(u128 a, u128 b) {
-  u64 A[2] = {(u64)a, (u64)(a >> 64)}, B[2] = {(u64)b, (u64)(b >> 64)};
-  W256 r = {{0, 0, 0, 0}};
-  for (int i = 0; i < 2; i++)
-    for (int j = 0; j < 2; j++) {
-      u128 p = (u128)A[i] * B[j];
-      // add p at word i+j with carry propagation
-      int k = i + j;
-      u128 add = p;
-      while (add && k < 4) {
-        u128 s = (u128)r.w[k] + (u64)add;
-        r.w[k] = (u64)s;
-        add = (add >> 64) + (s >> 64);
-        k++;
-      }
-    }
-  return r;
-}
-static W256 w256_mul_small(W256 a, u64 m) {
-  W256 r;
-  u128 c = 0;
-  for (int i = 0; i < 4; i++) { u128 p = (u128)a.w[i] * m + c; r.w[i] = (u64)p; c = p >> 64; }
-  return r;
-}
-static W256 w256_sub(W256 a, W256 b) {
-  W256 r;
-  u64 br = 0;
-  for (int i = 0; i < 4; i++) {
-    u128 d = (u128)a.w[i] - b.w[i] - br;
-    r.w[i] = (u64)d;
-    br = (u64)(d >> 127);  // borrow if negative
-  }
-  return r;
-}
-static bool w256_lt(W256 a, W256 b) {
-  for (int i = 3; i >= 0; i--) if (a.w[i] != b.w[i]) return a.w[i] < b.w[i];
-  return false;
-}
 // correctly rounded conversion to double (round to nearest even)
 static double w256_to_double(W256 a) {
   int top = 3;
@@ -578,11 +538,6 @@ static double w256_to_double(W256 a) {
   return ldexp((double)(hi64 | (sticky ? 1ull : 0ull)), sh);
 }
 
-// CoV < p/q  <=>  q^2 (n S2 - S1^2) < p^2 S1^2   (A1-A5)
-static bool cov_lt(u64 n, u128 s1, u128 s2, u32 p, u32 q) {
-  W256 var_n2 = w256_sub(w256_mul(n, s2), w256_mul(s1, s1));
-  return w256_lt(w256_mul_small(var_n2, (u64)q * q), w256_mul_small(w256_mul(s1, s1), (u64)p * p));
-}
 
 // Scott's normal-reference bandwidth ([36]; A8), rounded to 16 significant bits
 static double scott_h(u64 n, u128 s1, u128 s2, double bw_scale) {
@@ -1128,7 +1083,8 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         launch_complement(pm.get(), cap, 1, S);
       }
       SV_TRY(mapped_get(c, (1 + (size_t)cap * PART_REC + nseg) * 8, &hrec, &drec));
-      launch_part_pack(d_off.get(), nseg, cap, pl.get(), pm.get(), pab.get(), ntk.get(), drec, S);
+      launch_part_pack(d_off.get(), nseg, cap, pl.get(), pm.get(), pab.get(), ntk.get(), P->theta_num,
+                       P->theta_den, drec, S);
       hc.mark("p");
       SV_TRY(sync(c));
       hc.mark("ps");
@@ -1173,15 +1129,15 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         R->segs.push_back(std::move(sd));
       }
       for (u32 p = part_off[s]; p < part_off[s + 1]; p++) {
-        const u64* L = hrec + 1 + (size_t)p * PART_REC;  // {lanes[9], min, max, ia, ib}
+        const u64* L = hrec + 1 + (size_t)p * PART_REC;  // {lanes[9], min, max, ia, ib, final}
         u64 pn = L[0];
         if (!pn) continue;  // empty part: dropped (A13 f)
-        u128 s1 = limbs_u128(L + 1), s2 = limbs_u128(L + 5);
+        u128 s1 = limbs_u128(L + 1);
         u64 lo = L[MOM_LANES], hi = L[MOM_LANES + 1];
-        if (lo == hi || cov_lt(pn, s1, s2, P->theta_num, P->theta_den))
+        if (L[MOM_LANES + 4])  // lo == hi or CoV < theta, decided exactly by k_part_pack
           fin.push_back({op[s].kid, 3, lo, hi, pn, s1, hh[s], round});
-        else  // re-opened: its values are [ia, ib) of this batch's sorted keys (x << ib)
-          next.push_back({op[s].kid, op[s].t3rank, lo, hi, pn, s1, s2, L[MOM_LANES + 2],
+        else  // re-opened: its values are [ia, ib) of this batch's grouped values
+          next.push_back({op[s].kid, op[s].t3rank, lo, hi, pn, s1, limbs_u128(L + 5), L[MOM_LANES + 2],
                           L[MOM_LANES + 3], ck.get(), vsh});
       }
     }

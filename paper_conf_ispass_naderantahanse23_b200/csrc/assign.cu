@@ -29,8 +29,8 @@
 #define AS_FLUSH (3 * AS_HC / 4)      // flush to the L2 table when this full
 #define AS_MAXP 32          // probes before falling back to the global table
 #ifndef AS_CHECK
-#define AS_CHECK 32         // tiles between the block barriers that check the table's fill (A/B on C4:
-                            // every tile 0.73 ms, every 4 tiles 0.60, 16: 0.55, 32: 0.54, 128: 0.53)
+#define AS_CHECK 32         // at most this many tiles between the fill checks (A/B, C4 / C5:
+                            // every tile 0.73 / 10.7 ms, growth-paced up to 8: 0.59, 32: 0.57 / 10.0)
 #endif
 
 // One block per SM with a large table: a block's contiguous chunk sees nearly every (stratum,
@@ -91,7 +91,7 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
   const u64 tile = (u64)AS_THREADS * AS_IPT;
   u32 kk[AS_IPT], cc[AS_IPT];
   u64 vv[AS_IPT];
-  u32 tiles_done = 0;
+  u32 tiles_done = 0, next_check = 1, last_fill = 0, last_check = 0;
   auto load_tile = [&](u64 base, u32* k_, u64* v_, u32* c_) {
 #pragma unroll
     for (int j = 0; j < AS_IPT; j++) {
@@ -156,9 +156,11 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
     }
     bool last = base + tile >= b1;
     ++tiles_done;
-    // the fill check needs a block barrier: every AS_CHECK tiles (a full table only sends rows
-    // to the L2 table directly, it is never wrong)
-    if (tiles_done % AS_CHECK != 0 && !last) {
+    // the fill check needs block barriers, so it runs only as often as the table's growth needs:
+    // after half the tiles the last interval's growth rate would take to reach the flush level,
+    // at most AS_CHECK tiles apart (a full table only sends rows to the L2 table directly, it is
+    // never wrong)
+    if (tiles_done < next_check && !last) {
 #if AS_PIPE
 #pragma unroll
       for (int j = 0; j < AS_IPT; j++) { kk[j] = nk[j]; vv[j] = nv[j]; cc[j] = nc[j]; }
@@ -166,7 +168,17 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
       continue;
     }
     __syncthreads();
-    if (s_fill > AS_FLUSH || last) {  // rows that find no slot go to the L2 table directly
+    const u32 fill = s_fill;  // one snapshot for the whole block: nobody inserts until all read it
+    __syncthreads();
+    {
+      const u32 grow = (fill > last_fill ? fill - last_fill : 0u) / max(1u, tiles_done - last_check);
+      const u32 room = fill < AS_FLUSH ? AS_FLUSH - fill : 0u;
+      const u32 k = grow ? room / (2u * grow) : (u32)AS_CHECK;
+      next_check = tiles_done + max(1u, min(k, (u32)AS_CHECK));
+      last_fill = fill;
+      last_check = tiles_done;
+    }
+    if (fill > AS_FLUSH || last) {  // rows that find no slot go to the L2 table directly
       for (u32 e = threadIdx.x; e < AS_HC; e += AS_THREADS) {
         u64 key = hk[e];
         if (key != HASH_EMPTY) {
@@ -176,6 +188,7 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
       }
       __syncthreads();
       if (threadIdx.x == 0) s_fill = 0;
+      last_fill = 0;
       __syncthreads();
     }
 #if AS_PIPE

@@ -361,7 +361,7 @@ void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, 
 // host memory: out[0] = number of parts, then per part {lanes[9], min, max, ia, ib}
 __global__ void k_part_pack(const u32* __restrict__ part_off, u32 nseg, u32 cap, const u64* __restrict__ lanes,
                             const u64* __restrict__ mm, const u64* __restrict__ ab, const u32* __restrict__ ntk,
-                            u64* out) {
+                            u32 tp, u32 tq, u64* out) {
   const u32 nparts = part_off[nseg];
   u32 p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p == 0) out[0] = nparts;
@@ -375,12 +375,21 @@ __global__ void k_part_pack(const u32* __restrict__ part_off, u32 nseg, u32 cap,
   o[MOM_LANES + 1] = mm[cap + p];
   o[MOM_LANES + 2] = ab[4 * (u64)p + 2];
   o[MOM_LANES + 3] = ab[4 * (u64)p + 3];
+  // the part's fate (A13 f): final stratum iff lo == hi or its exact CoV < theta = tp / tq (the
+  // same u256 test as the tiering); the records are all-reduced already, so every rank agrees
+  const u64* L = lanes + (u64)p * MOM_LANES;
+  u64 s1lo, s1hi, s2lo, s2hi;
+  limbs_to_u128(L + 1, &s1lo, &s1hi);
+  limbs_to_u128(L + 5, &s2lo, &s2hi);
+  const bool fin = L[0] != 0 && (mm[p] == mm[cap + p] ||
+                                 cov_lt(L[0], ((u128)s1hi << 64) | s1lo, ((u128)s2hi << 64) | s2lo, tp, tq));
+  o[MOM_LANES + 4] = fin ? 1ull : 0ull;
 }
 
 void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, const u64* mm,
-                      const u64* ab, const u32* ntk, u64* out, cudaStream_t s) {
+                      const u64* ab, const u32* ntk, u32 tp, u32 tq, u64* out, cudaStream_t s) {
   SV_LAUNCH(k_part_pack, div_up(std::max<u32>(std::max(cap, nseg), 1), 128), 128, 0, s)(part_off, nseg, cap, lanes,
-                                                                                    mm, ab, ntk, out);
+                                                                                    mm, ab, ntk, tp, tq, out);
 }
 
 // ==========================================================================================

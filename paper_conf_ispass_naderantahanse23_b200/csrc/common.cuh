@@ -68,6 +68,57 @@ __device__ __forceinline__ void add128(u64& lo, u64& hi, u64 alo, u64 ahi) {
 __device__ __forceinline__ u32 lane_id() { return threadIdx.x & 31u; }
 
 // ------------------------------------------------------------------------------------------
+// exact 256-bit arithmetic for the replicated decisions (host: tiers, parts; device: the part
+// records' final / re-open flag), identical on both sides
+// ------------------------------------------------------------------------------------------
+struct W256 { u64 w[4]; };  // little-endian words
+
+__host__ __device__ inline W256 w256_mul(u128 a, u128 b) {
+  u64 A[2] = {(u64)a, (u64)(a >> 64)}, B[2] = {(u64)b, (u64)(b >> 64)};
+  W256 r = {{0, 0, 0, 0}};
+  for (int i = 0; i < 2; i++)
+    for (int j = 0; j < 2; j++) {
+      u128 p = (u128)A[i] * B[j];
+      // add p at word i+j with carry propagation
+      int k = i + j;
+      u128 add = p;
+      while (add && k < 4) {
+        u128 s = (u128)r.w[k] + (u64)add;
+        r.w[k] = (u64)s;
+        add = (add >> 64) + (s >> 64);
+        k++;
+      }
+    }
+  return r;
+}
+__host__ __device__ inline W256 w256_mul_small(W256 a, u64 m) {
+  W256 r;
+  u128 c = 0;
+  for (int i = 0; i < 4; i++) { u128 p = (u128)a.w[i] * m + c; r.w[i] = (u64)p; c = p >> 64; }
+  return r;
+}
+__host__ __device__ inline W256 w256_sub(W256 a, W256 b) {
+  W256 r;
+  u64 br = 0;
+  for (int i = 0; i < 4; i++) {
+    u128 d = (u128)a.w[i] - b.w[i] - br;
+    r.w[i] = (u64)d;
+    br = (u64)(d >> 127);  // borrow if negative
+  }
+  return r;
+}
+__host__ __device__ inline bool w256_lt(W256 a, W256 b) {
+  for (int i = 3; i >= 0; i--) if (a.w[i] != b.w[i]) return a.w[i] < b.w[i];
+  return false;
+}
+// CoV < p/q  <=>  q^2 (n S2 - S1^2) < p^2 S1^2   (A1-A5)
+__host__ __device__ inline bool cov_lt(u64 n, u128 s1, u128 s2, u32 p, u32 q) {
+  W256 var_n2 = w256_sub(w256_mul(n, s2), w256_mul(s1, s1));
+  return w256_lt(w256_mul_small(var_n2, (u64)q * q), w256_mul_small(w256_mul(s1, s1), (u64)p * p));
+}
+
+
+// ------------------------------------------------------------------------------------------
 // launch helpers
 // ------------------------------------------------------------------------------------------
 static inline unsigned div_up(u64 a, u64 b) { return (unsigned)((a + b - 1) / b); }

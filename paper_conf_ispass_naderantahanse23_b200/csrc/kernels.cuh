@@ -174,13 +174,14 @@ void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, 
                        const u64* T, u32 tstride, const u32* nt, const u32* part_off, u32 cap,
                        const u64* vals, u32 vshift, u32* items /* [cap + 1] */, void* scan_temp,
                        u64* lanes, u64* mm, u64* ab, cudaStream_t s);
-#define PART_REC (MOM_LANES + 4)
+#define PART_REC (MOM_LANES + 5)
 #define PART_GUESS 16   // part slots per open segment before the exact count is known (a round
                         // with more parts redoes its part moments once with the exact count)
-// out[0] = parts, out[1 + p * PART_REC ..] = {lanes[9], min, max, ia, ib} (p < cap),
+// out[0] = parts, out[1 + p * PART_REC ..] = {lanes[9], min, max, ia, ib, final} (p < cap; final =
+// lo == hi or CoV < tp / tq, exact),
 // out[1 + cap * PART_REC + s] = nt[s] | kind[s] << 32 (ntk = [nt | kind]); mapped host memory
 void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, const u64* mm,
-                      const u64* ab, const u32* ntk, u64* out, cudaStream_t s);
+                      const u64* ab, const u32* ntk, u32 tp, u32 tq, u64* out, cudaStream_t s);
 // ---------------- pass B: assignment + per-(stratum, CTA) statistics -------------------
 struct KTab {      // per kernel
   u32 base;        // global id of its first stratum

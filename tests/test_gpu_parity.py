@@ -68,6 +68,34 @@ def test_cell_radix_path(G, radix, monkeypatch):
     assert_segments_equal(g["segments"], o.segments())
 
 
+@pytest.mark.parametrize("G,step", [(1024, 997), (64, 15_999), (1000, 1)])
+def test_values_on_grid_boundaries(G, step):
+    """a Tier-3 kernel whose values sit on both sides of every round-1 grid point (ceil(g_j) and
+    ceil(g_j) - 1, A9 evaluated with IEEE doubles as in the oracle): every cell decision of the
+    grouping is a boundary case (the fast path must defer to the exact search), and step = 1
+    makes the grid finer than the integers (fast path disabled)"""
+    import math
+    lo = 1
+    hi = lo + (G - 1) * step + 3
+    g = [float(lo) + float((hi - lo) * j) / float(G - 1) for j in range(G)]
+    vals = sorted({v for j in range(G) for v in (math.ceil(g[j]), math.ceil(g[j]) - 1) if lo <= v <= hi} | {lo, hi})
+    rng = np.random.default_rng(G)
+    x = np.array(vals * 3, np.uint64)
+    kid = np.zeros(len(x), np.uint32)
+    filler = np.full(500, 777, np.uint64)  # a Tier-1 kernel
+    tr = {"kid": np.concatenate([kid, np.ones(500, np.uint32)]), "x": np.concatenate([x, filler]), "K": 2}
+    perm = rng.permutation(len(tr["kid"]))
+    tr["kid"], tr["x"] = tr["kid"][perm], tr["x"][perm]
+    tr["cta"] = rng.choice(np.array([64, 128], np.uint32), len(perm))
+    tr["y"] = (tr["x"] * np.uint64(3)).astype(np.uint64)
+    o = run_oracle(tr, G=G, keep_debug=True)
+    assert int(o.strata["tier"][0]) == 3
+    g_run = run_gpu(tr, G=G, keep_debug=True)
+    assert_tables_equal(g_run["table"], o.strata)
+    assert np.array_equal(g_run["sid"], o.sid)
+    assert_segments_equal(g_run["segments"], o.segments())
+
+
 @pytest.mark.parametrize("theta", [(1, 10), (1, 2), (1, 1), (3, 7)])
 def test_theta_values(theta):
     tr = gen.make_trace("C2", n=100_000)
