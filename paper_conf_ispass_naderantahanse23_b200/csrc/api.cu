@@ -999,6 +999,8 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     // the part count; a round with more parts than slots redoes its part moments with the exact
     // count, which every rank reads after the round's one synchronisation (so all ranks agree).
     u32 cap = (u32)std::min<u64>((u64)nseg * tstride, (u64)nseg * PART_GUESS + 64);
+    if (const char* e = getenv("SIEVE_PART_SLOTS"))  // test hook: force the exact-count redo
+      cap = std::max<u32>(1, std::min<u32>(cap, (u32)atoi(e)));
     DBuf<u64> pl(c), pm(c), pab(c);
     SV_TRY(pl.alloc((size_t)cap * MOM_LANES));
     SV_TRY(pm.alloc((size_t)cap * 2));

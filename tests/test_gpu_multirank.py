@@ -90,3 +90,21 @@ def test_nccl_path_single_rank():
     torch.cuda.synchronize()
     assert st.table.tobytes() == one["table"].tobytes()
     assert np.array_equal(sid.cpu().numpy().view(np.uint32), one["sid"])
+
+
+@pytest.mark.parametrize("world", [1, 3])
+def test_part_slot_overflow_redo(world, monkeypatch):
+    """SIEVE_PART_SLOTS=1 leaves one part slot per round, so every round with more parts redoes
+    its part moments (and their all-reduce) with the exact count; results unchanged"""
+    monkeypatch.setenv("SIEVE_PART_SLOTS", "1")
+    tr = gen.make_trace("C2", n=150_000)
+    o = run_oracle(tr)
+    if world == 1:
+        g = run_gpu(tr)
+        assert_tables_equal(g["table"], o.strata)
+        assert np.array_equal(g["sid"], o.sid)
+    else:
+        res = _run_group(tr, world)
+        for table, _, _ in res:
+            assert_tables_equal(table, o.strata)
+        assert np.array_equal(np.concatenate([r[1] for r in res]), o.sid)

@@ -1,0 +1,3 @@
+mkdir -p gpurun_out
+timeout 1800 python -m pytest tests -m gpu -x -q > gpurun_out/tests_r02p.log 2>&1; echo rc=$? >> gpurun_out/tests_r02p.log
+timeout 900 python bench.py > gpurun_out/bench_r02p.log 2> gpurun_out/bench_r02p.err
