@@ -99,6 +99,8 @@ struct Owner {
   sieve_free_fn ff = nullptr;  // nullptr: cudaMallocAsync / cudaFreeAsync
   void* user = nullptr;
 };
+// a read-back staged in pinned memory: copied into its host destination at the next sync
+struct CtxPend { void* dst; void* pinned; size_t bytes; };
 
 struct sieve_ctx_s {
   uint32_t magic = CTX_MAGIC;
@@ -126,8 +128,8 @@ struct sieve_ctx_s {
   char* pin = nullptr;
   size_t pin_cap = 0, pin_off = 0, pin_hw = 0;
   std::vector<void*> pin_overflow;
-  struct Pend { void* dst; void* pinned; size_t bytes; };
-  std::vector<Pend> pend;
+  std::vector<CtxPend> pend;
+  cudaEvent_t ev_moments = nullptr;   // pass A's deferred read-back
   // SIEVE_HOST_TIMING: host-side accounting of the synchronisations of a call
   int hs_n = 0;
   bool count_terms = true;  // in-window KDE term count (sieve_ctx_set_term_count)
@@ -450,6 +452,7 @@ extern "C" void sieve_ctx_destroy(sieve_ctx ctx) {
   if (ctx->pin) cudaFreeHost(ctx->pin);
   if (ctx->mapped) cudaFreeHost(ctx->mapped);
   if (ctx->scan_state) cudaFree(ctx->scan_state);
+  if (ctx->ev_moments) cudaEventDestroy(ctx->ev_moments);
   delete ctx->comm;
   ctx->magic = 0;
   delete ctx;
@@ -702,10 +705,18 @@ struct MomentsHost {
   const KMomPartial* part = nullptr;
   int part_grid = 0;
   u32 part_kt = 0;
+  // device copies of the reduced moments (valid in the call that computed them)
+  const u64 *d_lanes = nullptr, *d_mm = nullptr, *d_localn = nullptr;
+  // deferred read-back: the host copies land after `ready` completes (moments_finish)
+  cudaEvent_t ready = nullptr;
+  std::vector<CtxPend> pend;
 };
 
 // ---------------- pass A: per-kernel moments + totals -------------------
-static int moments_pass(sieve_trace t, MomentsHost* M) {
+static int moments_finish(sieve_ctx c, MomentsHost* M);
+// Pass A.  defer = true: the read-back is queued and an event recorded, but the host does not
+// wait (the caller queues more device work first and then calls moments_finish)
+static int moments_pass(sieve_trace t, MomentsHost* M, bool defer = false) {
   sieve_ctx c = t->ctx;
   cudaStream_t S = c->stream;
   const u32 K = t->K;
@@ -741,8 +752,6 @@ static int moments_pass(sieve_trace t, MomentsHost* M) {
   }
   SV_CUDA(cudaGetLastError());
   tA.stop();
-  // AR-1: sums, then min/max (mm is interleaved min,max per kernel: reduce via a [2][K] copy)
-  std::vector<u64> h_lanes, h_mm, h_tot, h_localn;
   if (c->comm) {
     // AR-1, one grouped step: SUM of the limb lanes and C_meas; MAX of (min, max) per kernel with
     // the mins complemented (min(a, b) = ~max(~a, ~b)), max x and the error lanes
@@ -751,22 +760,38 @@ static int moments_pass(sieve_trace t, MomentsHost* M) {
                                {mm.get(), (size_t)K * 2, RED_MAX}, {tot.get() + 4, 4, RED_MAX}}));
     launch_complement(mm.get(), K, 2, S);
   }
+  if (K <= kt) { M->part = part.get(); M->part_grid = gridA; M->part_kt = kt; }
+  M->d_lanes = lanes.get(); M->d_mm = mm.get(); M->d_localn = local_n.get();
   {
     CopyBatch cb(c);
-    SV_TRY(cb.add_d2h(h_lanes, lanes.get(), (size_t)K * MOM_LANES));
-    SV_TRY(cb.add_d2h(h_mm, mm.get(), (size_t)K * 2));
-    SV_TRY(cb.add_d2h(h_tot, tot.get(), 8));
-    SV_TRY(cb.add_d2h(h_localn, local_n.get(), K));
+    SV_TRY(cb.add_d2h(M->lanes, lanes.get(), (size_t)K * MOM_LANES));
+    SV_TRY(cb.add_d2h(M->mm, mm.get(), (size_t)K * 2));
+    SV_TRY(cb.add_d2h(M->tot, tot.get(), 8));
+    SV_TRY(cb.add_d2h(M->localn, local_n.get(), K));
     SV_TRY(cb.flush());
-    SV_TRY(sync(c));
   }
-  if (h_tot[5]) return sv_fail(SIEVE_EINVAL, "kernel id >= num_kernels in the trace");
-  if (h_tot[6]) return sv_fail(SIEVE_ERANGE, "instruction count 0 or >= 2^44 in the trace (A21)");
-  if (K <= kt) { M->part = part.get(); M->part_grid = gridA; M->part_kt = kt; }
-  M->lanes.swap(h_lanes);
-  M->mm.swap(h_mm);
-  M->tot.swap(h_tot);
-  M->localn.swap(h_localn);
+  if (defer) {
+    M->pend.swap(c->pend);   // these copies complete with the event, not at the next sync(c)
+    if (!c->ev_moments) SV_CUDA(cudaEventCreateWithFlags(&c->ev_moments, cudaEventDisableTiming));
+    M->ready = c->ev_moments;
+    SV_CUDA(cudaEventRecord(M->ready, S));
+    return SIEVE_OK;
+  }
+  SV_TRY(sync(c));
+  return moments_finish(c, M);
+}
+
+// wait for pass A's read-back (deferred: only for its event, later work keeps running) and
+// check the trace's validity flags (identical on every rank: they were all-reduced)
+static int moments_finish(sieve_ctx c, MomentsHost* M) {
+  if (M->ready) {
+    SV_CUDA(cudaEventSynchronize(M->ready));
+    for (auto& q : M->pend) memcpy(q.dst, q.pinned, q.bytes);
+    M->pend.clear();
+    M->ready = nullptr;
+  }
+  if (M->tot[5]) return sv_fail(SIEVE_EINVAL, "kernel id >= num_kernels in the trace");
+  if (M->tot[6]) return sv_fail(SIEVE_ERANGE, "instruction count 0 or >= 2^44 in the trace (A21)");
   return SIEVE_OK;
 }
 
@@ -781,8 +806,36 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   const u32 K = t->K, G = P->grid_points;
   const u64 n = t->n;
   MomentsHost own;
+  // grouped path (G <= GROUP_MAXG): the Tier-3 rows' x grouped by segment (t3rank) at the bases
+  // the local counts give; radix path: tagged keys (t3rank << bx) + x in row order
+  const bool grouped = G <= GROUP_MAXG && !getenv("SIEVE_CELL_RADIX");
+  DBuf<u64> keys(c);
+  DBuf<u32> d_t3rank(c);
+  bool pre = false;   // the round-1 grouping was queued right behind pass A
   if (!cached) {
-    SV_TRY(moments_pass(t, &own));
+    pre = grouped && n > 0 && K <= GROUP_T3_SMEM_MAX && !getenv("SIEVE_NO_DEVICE_TIERS");
+    SV_TRY(moments_pass(t, &own, pre));
+    if (pre) {
+      // tiers decided on the device (the same exact test the host repeats below) and the
+      // round-1 grouping queued behind pass A; the host waits only for pass A's read-back and
+      // takes its own decisions while the grouping runs.  The output holds at most n values.
+      DBuf<u32> tab(c), cur(c);
+      DBuf<char> gtmp(c);
+      SV_TRY(d_t3rank.alloc(K));
+      SV_TRY(tab.alloc(2 * (size_t)K + 2));   // [segment bases | kernel of each segment | counts]
+      SV_TRY(cur.alloc(K));
+      SV_TRY(gtmp.alloc(group_t3_temp_bytes(K)));
+      SV_TRY(keys.alloc(n));
+      u32* counts = tab.get() + 2 * (size_t)K;
+      launch_tiers(own.d_lanes, own.d_mm, own.d_localn, K, P->theta_num, P->theta_den, d_t3rank.get(),
+                   tab.get(), tab.get() + K, counts, S);
+      PhaseTimer tm(c, SIEVE_PHASE_COMPACT, n * 4);
+      launch_group_t3(t->kid, t->x, n, K, d_t3rank.get(), K, counts, tab.get(), cur.get(), keys.get(),
+                      gtmp.get(), own.part, own.part_grid, own.part_kt, tab.get() + K, S);
+      tm.stop();
+      SV_CUDA(cudaGetLastError());
+    }
+    SV_TRY(moments_finish(c, &own));
     cached = &own;
   }
   const std::vector<u64>& h_lanes = cached->lanes;
@@ -819,16 +872,11 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   }
   R->total_instr = I;
 
-  // ---------------- Tier-3 values: compaction ---------------------------------------------------
-  // grouped path (G <= GROUP_MAXG): the Tier-3 rows' x grouped by segment (t3rank) at the bases
-  // the local counts give; radix path: tagged keys (t3rank << bx) + x in row order
-  const bool grouped = G <= GROUP_MAXG && !getenv("SIEVE_CELL_RADIX");
+  // ---------------- Tier-3 values: compaction (unless queued behind pass A) --------------------
   const u32 bx = std::max<u32>(1, bitlen(max_x));
-  DBuf<u64> keys(c);
-  DBuf<u32> d_t3rank(c);
   DBuf<unsigned long long> counter(c);
   SV_TRY(counter.alloc(4));
-  if (n_t3 && n3_local) {
+  if (n_t3 && n3_local && !pre) {
     SV_TRY(d_t3rank.alloc(K));
     CopyBatch cb(c);
     SV_TRY(cb.add_h2d(d_t3rank.get(), t3rank));
@@ -849,8 +897,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       SV_TRY(cb.add_h2d(d_sb.get(), sb));
       SV_TRY(cb.flush());
       if (n_t3 > GROUP_T3_SMEM_MAX) SV_CUDA(cudaMemsetAsync(cur.get(), 0, (size_t)n_t3 * 4, S));  // global-cursor path
-      launch_group_t3(t->kid, t->x, n, d_t3rank.get(), n_t3, d_sb.get(), cur.get(), keys.get(), gtmp.get(),
-                      cached == &own ? own.part : nullptr, own.part_grid, own.part_kt, d_sb.get() + n_t3, S);
+      launch_group_t3(t->kid, t->x, n, K, d_t3rank.get(), n_t3, nullptr, d_sb.get(), cur.get(), keys.get(),
+                      gtmp.get(), cached == &own ? own.part : nullptr, own.part_grid, own.part_kt,
+                      d_sb.get() + n_t3, S);
     } else
     launch_t3_compact(t->kid, t->x, n, d_t3rank.get(), bx, keys.get(), counter.get(), S);
     SV_CUDA(cudaGetLastError());

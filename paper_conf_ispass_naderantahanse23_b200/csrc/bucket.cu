@@ -484,8 +484,10 @@ __device__ __forceinline__ void t3_range(u64 n, u32 nb, u32 b, u64* r0, u64* r1)
 }
 
 __global__ void __launch_bounds__(T3_THREADS)
-k_t3_count(const u32* __restrict__ kid, u64 n, const u32* __restrict__ t3rank, u32 n_t3, u32* __restrict__ cnt) {
+k_t3_count(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, u32 K, const u32* __restrict__ t3rank,
+           u32 n_t3, const u32* __restrict__ n_t3_dev, u32* __restrict__ cnt) {
   extern __shared__ u32 s_c[];   // [n_t3]
+  if (n_t3_dev) n_t3 = *n_t3_dev;
   for (u32 i = threadIdx.x; i < n_t3; i += T3_THREADS) s_c[i] = 0;
   __syncthreads();
   u64 r0, r1;
@@ -499,8 +501,10 @@ k_t3_count(const u32* __restrict__ kid, u64 n, const u32* __restrict__ t3rank, u
     }
 #pragma unroll
     for (int u = 0; u < T3_U; u++) {
-      const u32 t = k[u] != 0xFFFFFFFFu ? __ldg(t3rank + k[u]) : 0xFFFFFFFFu;
-      if (t != 0xFFFFFFFFu) atomicAdd(&s_c[t], 1u);
+      const u32 t = k[u] < K ? __ldg(t3rank + k[u]) : 0xFFFFFFFFu;
+      if (t == 0xFFFFFFFFu) continue;
+      const u64 v = __ldcs(x + i0 + (u64)u * T3_THREADS);
+      if (v != 0 && v < SIEVE_X_LIMIT) atomicAdd(&s_c[t], 1u);   // the rows pass A counts
     }
   }
   __syncthreads();
@@ -510,9 +514,11 @@ k_t3_count(const u32* __restrict__ kid, u64 n, const u32* __restrict__ t3rank, u
 // one warp per segment: exclusive scan of its per-block counts, offset by the segment's base;
 // part != nullptr: the counts are pass A's per-block kernel counts (part[b * kt + kernel].n, the
 // same row ranges), t3kern[t] = the kernel of segment t
-__global__ void k_t3_offsets(u32* __restrict__ cnt, u32 nb, u32 n_t3, const u32* __restrict__ seg_base,
-                             const KMomPartial* __restrict__ part, u32 kt, const u32* __restrict__ t3kern) {
+__global__ void k_t3_offsets(u32* __restrict__ cnt, u32 nb, u32 n_t3, const u32* __restrict__ n_t3_dev,
+                             const u32* __restrict__ seg_base, const KMomPartial* __restrict__ part, u32 kt,
+                             const u32* __restrict__ t3kern) {
   const u32 t = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (n_t3_dev) n_t3 = *n_t3_dev;
   if (t >= n_t3) return;
   u32 carry = seg_base[t];
   u32* row = cnt + (u64)t * nb;
@@ -532,8 +538,9 @@ __global__ void k_t3_offsets(u32* __restrict__ cnt, u32 nb, u32 n_t3, const u32*
 }
 
 __global__ void __launch_bounds__(T3_SC_THREADS)
-k_t3_scatter(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, const u32* __restrict__ t3rank,
-             u32 n_t3, const u32* __restrict__ off, u64* __restrict__ out) {
+k_t3_scatter(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, u32 K, const u32* __restrict__ t3rank,
+             u32 n_t3, const u32* __restrict__ n_t3_dev, const u32* __restrict__ off, u64* __restrict__ out) {
+  if (n_t3_dev) n_t3 = *n_t3_dev;
   extern __shared__ u32 s_cur[];   // [n_t3]: this block's next output position per segment
   for (u32 t = threadIdx.x; t < n_t3; t += T3_SC_THREADS) s_cur[t] = off[(u64)t * gridDim.x + blockIdx.x];
   __syncthreads();
@@ -548,21 +555,23 @@ k_t3_scatter(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, cons
       t[u] = i < r1 ? __ldcs(kid + i) : 0xFFFFFFFFu;
     }
 #pragma unroll
-    for (int u = 0; u < T3_U; u++) t[u] = t[u] != 0xFFFFFFFFu ? __ldg(t3rank + t[u]) : 0xFFFFFFFFu;
+    for (int u = 0; u < T3_U; u++) t[u] = t[u] < K ? __ldg(t3rank + t[u]) : 0xFFFFFFFFu;
     // x only for the Tier-3 rows: a 32-byte sector none of whose rows is Tier-3 is never read
 #pragma unroll
     for (int u = 0; u < T3_U; u++) v[u] = t[u] != 0xFFFFFFFFu ? __ldcs(x + i0 + (u64)u * T3_SC_THREADS) : 0ull;
+    // only the rows pass A counted (a trace with invalid rows fails after pass A, but these
+    // kernels may already run: they must stay inside their ranges)
 #pragma unroll
     for (int u = 0; u < T3_U; u++)
-      if (t[u] != 0xFFFFFFFFu) out[atomicAdd(&s_cur[t[u]], 1u)] = v[u];
+      if (t[u] != 0xFFFFFFFFu && v[u] != 0 && v[u] < SIEVE_X_LIMIT) out[atomicAdd(&s_cur[t[u]], 1u)] = v[u];
   }
 }
 
 size_t group_t3_temp_bytes(u32 n_t3) { return (size_t)n_t3 * sv_num_sms() * 4 * 4 + 256; }
 
-void launch_group_t3(const u32* kid, const u64* x, u64 n, const u32* t3rank, u32 n_t3, const u32* seg_base,
-                     u32* cursor, u64* out, void* temp, const KMomPartial* part, int part_grid, u32 part_kt,
-                     const u32* t3kern, cudaStream_t s) {
+void launch_group_t3(const u32* kid, const u64* x, u64 n, u32 K, const u32* t3rank, u32 n_t3,
+                     const u32* n_t3_dev, const u32* seg_base, u32* cursor, u64* out, void* temp,
+                     const KMomPartial* part, int part_grid, u32 part_kt, const u32* t3kern, cudaStream_t s) {
   if (!n || !n_t3) return;
   if (n_t3 <= GT_SMEM_MAX) {
     // pass A's per-block kernel counts over the same row ranges, when the caller has them
@@ -573,10 +582,10 @@ void launch_group_t3(const u32* kid, const u64* x, u64 n, const u32* t3rank, u32
     const size_t sm = (size_t)n_t3 * 4;
     sv_smem_attr(k_t3_count, GT_SMEM_MAX * 4);
     sv_smem_attr(k_t3_scatter, GT_SMEM_MAX * 4);
-    if (!reuse) SV_LAUNCH(k_t3_count, nb, T3_THREADS, sm, s)(kid, n, t3rank, n_t3, cnt);
-    SV_LAUNCH(k_t3_offsets, div_up((u64)n_t3 * 32, 256), 256, 0, s)(cnt, nb, n_t3, seg_base,
+    if (!reuse) SV_LAUNCH(k_t3_count, nb, T3_THREADS, sm, s)(kid, x, n, K, t3rank, n_t3, n_t3_dev, cnt);
+    SV_LAUNCH(k_t3_offsets, div_up((u64)n_t3 * 32, 256), 256, 0, s)(cnt, nb, n_t3, n_t3_dev, seg_base,
                                                                     reuse ? part : nullptr, part_kt, t3kern);
-    SV_LAUNCH(k_t3_scatter, nb, T3_SC_THREADS, sm, s)(kid, x, n, t3rank, n_t3, cnt, out);
+    SV_LAUNCH(k_t3_scatter, nb, T3_SC_THREADS, sm, s)(kid, x, n, K, t3rank, n_t3, n_t3_dev, cnt, out);
     return;
   }
   // many Tier-3 kernels: global cursors (k_group_t3's global-atomic branch)

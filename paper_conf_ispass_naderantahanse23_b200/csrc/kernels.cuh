@@ -144,9 +144,17 @@ size_t group_t3_temp_bytes(u32 n_t3);
 // part (nullable): pass A's per-block partials of this trace (part_grid blocks x part_kt kernels,
 // every kernel in one pass), whose per-block counts then give the output bases directly;
 // t3kern[t] = the kernel of segment t (read only with part)
-void launch_group_t3(const u32* kid, const u64* x, u64 n, const u32* t3rank, u32 n_t3, const u32* seg_base,
-                     u32* cursor, u64* out, void* temp /* group_t3_temp_bytes(n_t3) */,
-                     const KMomPartial* part, int part_grid, u32 part_kt, const u32* t3kern, cudaStream_t s);
+// n_t3: Tier-3 kernels (an upper bound when n_t3_dev != nullptr holds the live count on the
+// device: the kernels may then be queued before the host knows the tiers)
+void launch_group_t3(const u32* kid, const u64* x, u64 n, u32 K, const u32* t3rank, u32 n_t3,
+                     const u32* n_t3_dev, const u32* seg_base, u32* cursor, u64* out,
+                     void* temp /* group_t3_temp_bytes(n_t3) */, const KMomPartial* part, int part_grid,
+                     u32 part_kt, const u32* t3kern, cudaStream_t s);
+// tiers on the device (the same exact test as the host's): t3rank[k] (0xFFFFFFFF unless Tier-3),
+// seg_base[t] = exclusive prefix of the local counts of the Tier-3 kernels in kernel order,
+// t3kern[t] = kernel of segment t, counts[0] = Tier-3 kernels, counts[1] = their local rows
+void launch_tiers(const u64* lanes, const u64* mm, const u64* local_n, u32 K, u32 p, u32 q, u32* t3rank,
+                  u32* seg_base, u32* t3kern, u32* counts, cudaStream_t s);
 // chunks (<= GROUP_CH values of one segment's source range each, the chunks of segment s are
 // seg_chunk[s] .. seg_chunk[s + 1] - 1) -> out grouped by (segment, cell) with
 // off[s * G + c] = first position of cell c of segment s, off[nseg * G] = values grouped

@@ -366,3 +366,67 @@ void launch_moments_reduce(const KMomPartial* part, const u64* blk_tot, int grid
   SV_LAUNCH(k_moments_reduce, div_up((u64)kt * 32, 256), 256, 0, s)(part, grid, k0, kt, lanes, mm, local_n);
   if (do_totals) SV_LAUNCH(k_totals_reduce, 1, 32, 0, s)(blk_tot, grid, tot_lanes, tot_max);
 }
+
+// Tiers on the device (A1-A5), the host's exact test, so the round-1 grouping can be
+// queued right behind pass A while the host takes the same decisions from its copy of the
+// moments.  One block walks the kernels in order, 1024 at a time, carrying the Tier-3 rank and
+// the running sum of the Tier-3 kernels' local rows.
+__global__ void __launch_bounds__(1024) k_tiers(const u64* __restrict__ lanes, const u64* __restrict__ mm,
+                                                const u64* __restrict__ local_n, u32 K, u32 p, u32 q,
+                                                u32* __restrict__ t3rank, u32* __restrict__ seg_base,
+                                                u32* __restrict__ t3kern, u32* __restrict__ counts) {
+  __shared__ u32 s_w[32], s_r[32];
+  __shared__ u32 c_rank, c_rows;
+  if (threadIdx.x == 0) { c_rank = 0; c_rows = 0; }
+  __syncthreads();
+  for (u32 k0 = 0; k0 < K; k0 += 1024) {
+    const u32 k = k0 + threadIdx.x;
+    bool t3 = false;
+    u32 rows = 0;
+    if (k < K) {
+      const u64* L = lanes + (u64)k * MOM_LANES;
+      if (L[0] && mm[2 * (u64)k] != mm[2 * (u64)k + 1]) {
+        u64 a, b, c2, d;
+        limbs_to_u128(L + 1, &a, &b);
+        limbs_to_u128(L + 5, &c2, &d);
+        t3 = !cov_lt(L[0], ((u128)b << 64) | a, ((u128)d << 64) | c2, p, q);
+      }
+      rows = t3 ? (u32)local_n[k] : 0u;
+    }
+    // block-wide exclusive scans of (is Tier-3, its rows)
+    u32 f = t3 ? 1u : 0u, r = rows;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const u32 a = __shfl_up_sync(0xffffffffu, f, o), b = __shfl_up_sync(0xffffffffu, r, o);
+      if ((int)lane_id() >= o) { f += a; r += b; }
+    }
+    const u32 w = threadIdx.x >> 5;
+    if (lane_id() == 31) { s_w[w] = f; s_r[w] = r; }
+    __syncthreads();
+    if (w == 0) {
+      u32 a = s_w[lane_id()], b = s_r[lane_id()];
+      const u32 a0 = a, b0 = b;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const u32 x1 = __shfl_up_sync(0xffffffffu, a, o), x2 = __shfl_up_sync(0xffffffffu, b, o);
+        if ((int)lane_id() >= o) { a += x1; b += x2; }
+      }
+      s_w[lane_id()] = a - a0;
+      s_r[lane_id()] = b - b0;
+    }
+    __syncthreads();
+    const u32 rank = c_rank + s_w[w] + f - (t3 ? 1u : 0u);
+    const u32 base = c_rows + s_r[w] + r - rows;
+    if (k < K) t3rank[k] = t3 ? rank : 0xFFFFFFFFu;
+    if (t3) { seg_base[rank] = base; t3kern[rank] = k; }
+    __syncthreads();
+    if (threadIdx.x == 1023) { c_rank = rank + (t3 ? 1u : 0u); c_rows = base + rows; }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) { counts[0] = c_rank; counts[1] = c_rows; }
+}
+
+void launch_tiers(const u64* lanes, const u64* mm, const u64* local_n, u32 K, u32 p, u32 q, u32* t3rank,
+                  u32* seg_base, u32* t3kern, u32* counts, cudaStream_t s) {
+  SV_LAUNCH(k_tiers, 1, 1024, 0, s)(lanes, mm, local_n, K, p, q, t3rank, seg_base, t3kern, counts);
+}

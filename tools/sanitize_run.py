@@ -62,7 +62,28 @@ def group(tr, world=2):
     print(f"group world={world} ok", flush=True)
 
 
+def invalid_rows():
+    """rows with x = 0 and a kernel id >= K: the call fails after pass A, while the round-1
+    grouping queued behind it still runs over the same rows (it must stay in bounds)"""
+    tr = gen.make_trace("C2", n=100_000)
+    for bad in ("x", "kid"):
+        kid, x = tr["kid"].copy(), tr["x"].copy()
+        if bad == "x":
+            x[::997] = 0
+        else:
+            kid[::991] = tr["K"] + 5
+        ctx = sieve.Ctx(device=0)
+        t = sieve.load_trace(ctx, kid, x, num_kernels=tr["K"], cta=tr["cta"], cycles=tr["y"])
+        try:
+            sieve.stratify(t)
+            raise AssertionError("invalid rows accepted")
+        except sieve.SieveError as e:
+            print(f"invalid {bad}: status {e.code}", flush=True)
+        torch.cuda.synchronize()
+
+
 if __name__ == "__main__":
+    invalid_rows()
     one(gen.make_trace("C1"))
     one(gen.make_trace("C2"), n=200_000)
     if "--no-group" not in sys.argv:
