@@ -55,6 +55,9 @@ enum {
 #define SIEVE_MEM_DEVICE 1u /* columns are device pointers on the ctx's device: copied D2D */
 #define SIEVE_ADOPT 2u      /* with SIEVE_MEM_DEVICE: borrow the caller's buffers, no copy; the
                                caller keeps them alive and unchanged until sieve_trace_free */
+#define SIEVE_KID16 4u      /* kernel_id points to uint16_t values (K <= 65536): half the bytes
+                               to copy; widened on the device.  Not with SIEVE_ADOPT */
+#define SIEVE_CTA16 8u      /* cta points to uint16_t values (CTA sizes < 65536); as SIEVE_KID16 */
 
 typedef struct sieve_ctx_s* sieve_ctx;       /* device, stream, communicator, allocator */
 typedef struct sieve_trace_s* sieve_trace;   /* this rank's slice of the profile, on the device */
@@ -112,7 +115,8 @@ void sieve_ctx_destroy(sieve_ctx ctx);
      instr        [n_local] u64 dynamic instruction count, 1 <= x < 2^44 (A21)
      cta          [n_local] u32 CTA (thread-block) size, opaque key (A16); NULL = all equal
      cycles       [n_local] u64 measured cycles; NULL = no measured cycles
-     mem          SIEVE_MEM_HOST | SIEVE_MEM_DEVICE [| SIEVE_ADOPT]
+     mem          SIEVE_MEM_HOST | SIEVE_MEM_DEVICE [| SIEVE_ADOPT] [| SIEVE_KID16] [| SIEVE_CTA16]
+                  (the 16-bit forms change only what is copied: the trace holds u32 columns)
    Value validation (kernel id < K, 1 <= x < 2^44) happens on the device in the first pass of
    sieve_stratify, which returns SIEVE_EINVAL / SIEVE_ERANGE on a bad row. */
 int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_id, uint32_t num_kernels,

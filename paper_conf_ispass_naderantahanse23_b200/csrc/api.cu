@@ -481,9 +481,11 @@ extern "C" int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_
   if (K == 0 || K > SIEVE_MAX_K) return sv_fail(SIEVE_ERANGE, "num_kernels must be in [1, 65536]");
   if (n_local >= (1ull << 32)) return sv_fail(SIEVE_ERANGE, "n_local must be < 2^32");
   if (n_local && (!kernel_id || !instr)) return sv_fail(SIEVE_EINVAL, "kernel_id and instr are required");
-  if (mem & ~3u) return sv_fail(SIEVE_EINVAL, "bad mem flags");
+  if (mem & ~15u) return sv_fail(SIEVE_EINVAL, "bad mem flags");
   bool dev = mem & SIEVE_MEM_DEVICE, adopt = mem & SIEVE_ADOPT;
+  const bool kid16 = mem & SIEVE_KID16, cta16 = mem & SIEVE_CTA16;
   if (adopt && !dev) return sv_fail(SIEVE_EINVAL, "SIEVE_ADOPT needs SIEVE_MEM_DEVICE");
+  if (adopt && (kid16 || cta16)) return sv_fail(SIEVE_EINVAL, "16-bit columns cannot be adopted");
   SV_CUDA(cudaSetDevice(ctx->device));
   sieve_trace_s* t = new sieve_trace_s();
   t->ctx = ctx; t->n = n_local; t->first_id = first_id; t->K = K; t->owned = !adopt;
@@ -498,10 +500,24 @@ extern "C" int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_
       if (bytes) SV_CUDA(cudaMemcpyAsync(*dst, src, bytes, kind, ctx->stream));
       return SIEVE_OK;
     };
+    // a 16-bit column is copied as it is into a temporary, then widened into the u32 column
+    auto cp16 = [&](void** dst, const void* src) -> int {
+      if (!src) { *dst = nullptr; return SIEVE_OK; }
+      SV_TRY(dalloc(ctx, dst, n_local * 4));
+      if (!n_local) return SIEVE_OK;
+      void* tmp = nullptr;
+      SV_TRY(dalloc(ctx, &tmp, n_local * 2));
+      cudaError_t e = cudaMemcpyAsync(tmp, src, n_local * 2, kind, ctx->stream);
+      if (e == cudaSuccess) { launch_widen_u16(tmp, n_local, (u32*)*dst, ctx->stream); e = cudaGetLastError(); }
+      dfree(ctx, t->owner, tmp);
+      if (e != cudaSuccess) return sv_cuda(e, "16-bit column", __LINE__);
+      return SIEVE_OK;
+    };
     int st = SIEVE_OK;
-    if (st == SIEVE_OK) st = cp((void**)&t->kid, kernel_id ? kernel_id : (const uint32_t*)&t->n, n_local * 4);
+    if (kid16) st = cp16((void**)&t->kid, kernel_id);
+    else if (st == SIEVE_OK) st = cp((void**)&t->kid, kernel_id ? kernel_id : (const uint32_t*)&t->n, n_local * 4);
     if (st == SIEVE_OK) st = cp((void**)&t->x, instr ? instr : (const uint64_t*)&t->n, n_local * 8);
-    if (st == SIEVE_OK) st = cp((void**)&t->cta, cta, n_local * 4);
+    if (st == SIEVE_OK) st = cta16 ? cp16((void**)&t->cta, cta) : cp((void**)&t->cta, cta, n_local * 4);
     if (st == SIEVE_OK) st = cp((void**)&t->y, cycles, n_local * 8);
     if (st == SIEVE_OK) { cudaError_t e = cudaStreamSynchronize(ctx->stream); if (e) st = sv_cuda(e, "load sync", __LINE__); }
     if (st != SIEVE_OK) { t->magic = TRACE_MAGIC; sieve_trace_free(t); return st; }
@@ -1200,23 +1216,27 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   // the KDE term count is read back with the representatives at the end (no extra sync)
   std::vector<unsigned long long> h_terms;
   keys.release();
+  hc.mark("rend");
 
   // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
-  {  // counting sort by kernel, then by lo inside each kernel's (short) run: O(#strata + K)
-    std::vector<u32> cnt(K + 1, 0);
+  {  // counting sort by kernel, then by lo inside each kernel's (short) run: O(#strata + K).
+     // The scratch vectors are the thread's, reused across calls: a fresh 260 KB vector per call
+     // cost more (page faults, zero fill) than the sort itself.
+    static thread_local std::vector<u32> cnt, pos;
+    static thread_local std::vector<Fin> by;
+    cnt.assign(K + 1, 0);
     for (const Fin& f : fin) cnt[f.kid + 1]++;
     for (u32 k = 0; k < K; k++) cnt[k + 1] += cnt[k];
-    std::vector<Fin> by(fin.size());
-    {
-      std::vector<u32> pos(cnt.begin(), cnt.end() - 1);
-      for (const Fin& f : fin) by[pos[f.kid]++] = f;
-    }
+    if (by.size() < fin.size()) by.resize(fin.size());
+    pos.assign(cnt.begin(), cnt.end() - 1);
+    for (const Fin& f : fin) by[pos[f.kid]++] = f;
     for (u32 k = 0; k < K; k++)
       if (cnt[k + 1] - cnt[k] > 1)
         std::sort(by.begin() + cnt[k], by.begin() + cnt[k + 1],
                   [](const Fin& a, const Fin& b) { return a.lo < b.lo; });
-    fin.swap(by);
+    std::copy(by.begin(), by.begin() + fin.size(), fin.begin());
   }
+  hc.mark("tsort");
   const u32 ns = (u32)fin.size();
   std::vector<KTab> ktab(K, KTab{0, 0, 0, 0});
   std::vector<u64> lows;
@@ -1258,10 +1278,15 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     if (attempt > 6) return sv_fail(SIEVE_ENOMEM, "(stratum, CTA) table kept overflowing");
     DBuf<u64> gkeys(c), gcnt(c), gfirst(c), ent(c);
     SV_TRY(gkeys.alloc(cap)); SV_TRY(gcnt.alloc(cap)); SV_TRY(gfirst.alloc(cap));
-    launch_fill_u64(gkeys.get(), cap, HASH_EMPTY, S);
-    SV_CUDA(cudaMemsetAsync(gcnt.get(), 0, cap * 8, S));
-    launch_fill_u64(gfirst.get(), cap, ~0ull, S);
-    SV_CUDA(cudaMemsetAsync(errf.get(), 0, 32, S));
+    SV_TRY(ent.alloc(cap * 3));   // [keys | counts | firsts] of the compacted entries
+    {  // every initialisation of pass B in two launches (the table, then the entry arrays)
+      FillRegions f1{{gkeys.get(), gcnt.get(), gfirst.get(), errf.get()}, {cap, cap, cap, 4},
+                     {HASH_EMPTY, 0, ~0ull, 0}, 4};
+      launch_fill_multi(f1, S);
+      FillRegions f2{{ent.get(), ent.get() + cap, ent.get() + 2 * cap, (u64*)counter.get()}, {cap, cap, cap, 1},
+                     {~0ull, 0, ~0ull, 0}, 4};
+      launch_fill_multi(f2, S);
+    }
     GHash gh{gkeys.get(), gcnt.get(), gfirst.get(), cap};
     {
       PhaseTimer tb(c, SIEVE_PHASE_ASSIGN, n * (12 + (t->cta ? 4 : 0) + (sid_out ? 4 : 0)));
@@ -1269,12 +1294,6 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
                     (u32)lows.size(), sid_out, gh, errf.get(), assign_grid(), S);
     }
     SV_CUDA(cudaGetLastError());
-    // ent = [keys | counts | firsts], cap each
-    SV_TRY(ent.alloc(cap * 3));
-    launch_fill_u64(ent.get(), cap, ~0ull, S);
-    SV_CUDA(cudaMemsetAsync(ent.get() + cap, 0, cap * 8, S));
-    launch_fill_u64(ent.get() + 2 * cap, cap, ~0ull, S);
-    SV_CUDA(cudaMemsetAsync(counter.get(), 0, 8, S));
     launch_hash_compact(gh, ent.get(), ent.get() + cap, ent.get() + 2 * cap, counter.get(), S);
     u64 Etot = cap;
     const u64* ak = ent.get();

@@ -407,3 +407,12 @@ void launch_exchange_prep(const u64* flag, const unsigned long long* count, int 
                           cudaStream_t s) {
   SV_LAUNCH(k_exchange_prep, 1, ((world + 31) / 32) * 32, 0, s)(flag, count, rank, world, x);
 }
+
+// 16-bit trace columns (SIEVE_KID16 / SIEVE_CTA16) widened to the library's u32 columns
+__global__ void k_widen_u16(const unsigned short* __restrict__ src, u64 n, u32* __restrict__ dst) {
+  for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) dst[i] = src[i];
+}
+void launch_widen_u16(const void* src, u64 n, u32* dst, cudaStream_t s) {
+  if (n) SV_LAUNCH(k_widen_u16, (u32)std::min<u64>(div_up(n, 256), (u64)sv_num_sms() * 16), 256, 0, s)(
+      (const unsigned short*)src, n, dst);
+}

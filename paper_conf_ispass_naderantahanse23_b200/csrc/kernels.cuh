@@ -273,6 +273,8 @@ void launch_copy(void* dst, const void* src, u64 bytes, cudaStream_t s);
 #define COPY_MAX 8
 struct CopyRegions { void* dst[COPY_MAX]; const void* src[COPY_MAX]; u64 bytes[COPY_MAX]; int k; };
 void launch_copy_multi(const CopyRegions& r, cudaStream_t s);
+// dst[i] = src[i] for a u16 column (SIEVE_KID16 / SIEVE_CTA16 loads)
+void launch_widen_u16(const void* src, u64 n, u32* dst, cudaStream_t s);
 // cross-rank encoding of u128 pairs [n][2] <-> 4 limbs [n][4]
 void launch_u128_to_limbs(const u64* src, u64 n, u64* limbs, cudaStream_t s);
 void launch_limbs_to_u128(const u64* limbs, u64 n, u64* dst, cudaStream_t s);

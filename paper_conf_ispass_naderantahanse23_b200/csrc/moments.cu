@@ -30,12 +30,6 @@
 #define MOM_L2 6                              // limbs of x^2 (88 bits)
 #define MOM_WORDS (1 + MOM_L1 + MOM_L2)       // count + limbs, u32 each
 
-#ifndef MOM_MMTEST
-#define MOM_MMTEST 0
-#endif
-#ifndef MOM_AGG
-#define MOM_AGG 0                             // 1: warp-aggregate rows of equal kernels (A/B)
-#endif
 #ifndef MOM_MINB
 #define MOM_MINB 1                            // resident blocks per SM (A/B on C4: 2 x 1024 threads caps the
                                               // kernel at 32 registers and spills: 0.72 -> 3.0 ms)
@@ -110,34 +104,6 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
       u64 s = ylo + w; yhi += s < ylo; ylo = s;
     }
     u32 l = k - k0;
-#if MOM_AGG
-    // rows of equal kernels in a warp are summed first (one leader atomic per limb and group):
-    // a Zipf-hot kernel appears in several lanes of a warp, whose same-address atomics serialise
-    const bool ok = !(l >= kt || v == 0 || v >= SIEVE_X_LIMIT);
-    const u32 act = __activemask();
-    const u32 grp = __match_any_sync(act, ok ? l : 0xFFFFFFFFu);
-    if (!ok) return;
-    const bool lead = (grp & ((1u << lane_id()) - 1u)) == 0;
-    if (lead) atomicAdd(&s_w[l], (u32)__popc(grp));
-#pragma unroll
-    for (int i = 0; i < MOM_L1; i++) {
-      u32 limb = __reduce_add_sync(grp, (u32)(v >> (MOM_LB * i)) & MOM_LMASK);
-      if (lead && limb) atomicAdd(&s_w[(1 + i) * kt + l], limb);
-    }
-    {
-      u64 sqlo = v * v, sqhi = __umul64hi(v, v);
-#pragma unroll
-      for (int i = 0; i < MOM_L2; i++) {
-        int sh = MOM_LB * i;
-        u64 bits = sh < 64 ? ((sqlo >> sh) | (sh ? (sqhi << (64 - sh)) : 0ull)) : (sqhi >> (sh - 64));
-        u32 limb = __reduce_add_sync(grp, (u32)bits & MOM_LMASK);
-        if (lead && limb) atomicAdd(&s_w[(1 + MOM_L1 + i) * kt + l], limb);
-      }
-    }
-    atomic_min_u64_smem(&s_mn[l], v);
-    atomic_max_u64_smem(&s_mx[l], v);
-    return;
-#endif
     if (l >= kt || v == 0 || v >= SIEVE_X_LIMIT) return;
     u32* const sw = s_w + ((nrep == 2 && (lane_id() & 16u)) ? cs : 0u);
     atomicAdd(&sw[l], 1u);
@@ -154,13 +120,8 @@ k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __r
       u32 limb = (u32)bits & MOM_LMASK;
       if (limb) atomicAdd(&sw[(1 + MOM_L1 + i) * kt + l], limb);
     }
-#if MOM_MMTEST  // timing probe only (wrong min / max): 32-bit fire-and-forget min / max of x >> 12
-    atomicMin((u32*)&s_mn[l], (u32)(v >> 12));
-    atomicMax((u32*)&s_mx[l], (u32)(v >> 12));
-#else
     atomic_min_u64_smem(&s_mn[l], v);
     atomic_max_u64_smem(&s_mx[l], v);
-#endif
   };
 
   auto flush = [&]() {

@@ -21,7 +21,7 @@ LIB_PATH = os.environ.get("SIEVE_LIB_PATH") or os.path.join(_HERE, "libsieve.so"
 
 SIEVE_OK, SIEVE_EINVAL, SIEVE_ERANGE, SIEVE_ENOMEM = 0, -1, -2, -3
 SIEVE_ECUDA, SIEVE_ENCCL, SIEVE_EDOM, SIEVE_ELIMIT, SIEVE_ESTATE = -4, -5, -6, -7, -8
-MEM_HOST, MEM_DEVICE, ADOPT = 0, 1, 2
+MEM_HOST, MEM_DEVICE, ADOPT, KID16, CTA16 = 0, 1, 2, 4, 8
 
 STRATUM_DTYPE = np.dtype([
     ("kernel_id", "<u4"), ("tier", "<u4"), ("index_in_kernel", "<u4"), ("rep_cta", "<u4"),
@@ -275,6 +275,17 @@ def kernel_launches():
     return _L.sieve_kernel_launches()
 
 
+def _is16(a):
+    """a 16-bit column (numpy uint16 / torch uint16, int16): loaded with SIEVE_KID16 / CTA16"""
+    if isinstance(a, np.ndarray):
+        return a.dtype == np.uint16
+    try:
+        import torch
+        return isinstance(a, torch.Tensor) and a.dtype in (torch.uint16, torch.int16)
+    except ImportError:
+        return False
+
+
 def _col(a, dtype, device_ok=True):
     """(pointer, is_device, keepalive) for a numpy array or a CUDA tensor."""
     if a is None:
@@ -284,7 +295,8 @@ def _col(a, dtype, device_ok=True):
         return a.ctypes.data_as(ctypes.c_void_p), False, a
     import torch
     if isinstance(a, torch.Tensor):
-        want = {np.uint32: (torch.uint32, torch.int32), np.uint64: (torch.uint64, torch.int64)}[dtype]
+        want = {np.uint32: (torch.uint32, torch.int32), np.uint64: (torch.uint64, torch.int64),
+                np.uint16: (torch.uint16, torch.int16)}[dtype]
         if a.dtype not in want:
             raise TypeError(f"tensor dtype {a.dtype} does not match {np.dtype(dtype)}")
         if not a.is_contiguous():
@@ -310,14 +322,17 @@ class Trace:
 
 
 def load_trace(ctx, kernel_id, instr, num_kernels, cta=None, cycles=None, first_id=0, adopt=False):
-    """sieve_load_trace: columns as numpy arrays (host, copied H2D) or CUDA tensors (device)."""
-    cols = [_col(kernel_id, np.uint32), _col(instr, np.uint64), _col(cta, np.uint32),
-            _col(cycles, np.uint64)]
+    """sieve_load_trace: columns as numpy arrays (host, copied H2D) or CUDA tensors (device).
+    kernel_id / cta may be 16-bit (uint16): half the bytes copied, widened on the device."""
+    k16, c16 = _is16(kernel_id), cta is not None and _is16(cta)
+    cols = [_col(kernel_id, np.uint16 if k16 else np.uint32), _col(instr, np.uint64),
+            _col(cta, np.uint16 if c16 else np.uint32), _col(cycles, np.uint64)]
     kinds = {c[1] for c in cols if c[1] is not None}
     if len(kinds) > 1:
         raise ValueError("all columns must be on the same side (host or device)")
     on_dev = kinds == {True}
-    mem = (MEM_DEVICE if on_dev else MEM_HOST) | (ADOPT if adopt else 0)
+    mem = (MEM_DEVICE if on_dev else MEM_HOST) | (ADOPT if adopt else 0) | (KID16 if k16 else 0) | \
+        (CTA16 if c16 else 0)
     n = len(kernel_id)
     for name, c in zip(("instr", "cta", "cycles"), (instr, cta, cycles)):
         if c is not None and len(c) != n:  # the library reads n rows of every column

@@ -276,3 +276,34 @@ def test_kde_evaluation_modes_identical(monkeypatch, mode):
     assert_tables_equal(g["table"], o.strata)
     assert np.array_equal(g["sid"], o.sid)
     assert_segments_equal(g["segments"], o.segments())
+
+
+@pytest.mark.parametrize("device", [False, True])
+def test_16bit_columns(device):
+    """SIEVE_KID16 / SIEVE_CTA16: kernel ids and CTA sizes handed over as uint16 (host or device)
+    load the same trace as the 32-bit columns"""
+    import torch
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr = gen.make_trace("C2", n=80_000)
+    o = run_oracle(tr)
+    kid16, cta16 = tr["kid"].astype(np.uint16), tr["cta"].astype(np.uint16)
+    if device:
+        kid16 = torch.from_numpy(kid16.view(np.int16)).cuda()
+        cta16 = torch.from_numpy(cta16.view(np.int16)).cuda()
+        x = torch.from_numpy(tr["x"].view(np.int64)).cuda()
+        y = torch.from_numpy(tr["y"].view(np.int64)).cuda()
+    else:
+        x, y = tr["x"], tr["y"]
+    ctx = sieve.Ctx(device=0)
+    t = sieve.load_trace(ctx, kid16, x, num_kernels=tr["K"], cta=cta16, cycles=y)
+    kid_back, x_back, cta_back, _ = sieve.trace_columns(t)
+    assert np.array_equal(kid_back, tr["kid"]) and np.array_equal(cta_back, tr["cta"])
+    sid = torch.empty(len(tr["kid"]), dtype=torch.int32, device="cuda")
+    st = sieve.stratify(t, stratum_of_invocation=sid)
+    torch.cuda.synchronize()
+    assert_tables_equal(st.table, o.strata)
+    assert np.array_equal(sid.cpu().numpy().view(np.uint32), o.sid)
+    with pytest.raises(sieve.SieveError):
+        sieve.load_trace(ctx, kid16 if device else torch.from_numpy(tr["kid"].astype(np.int16)).cuda(),
+                         x if device else torch.from_numpy(tr["x"].view(np.int64)).cuda(),
+                         num_kernels=tr["K"], adopt=True)

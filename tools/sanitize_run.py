@@ -82,7 +82,35 @@ def invalid_rows():
         torch.cuda.synchronize()
 
 
+def other_entry_points():
+    """the rest of the C-ABI on C1-sized inputs: theta sweep, tier census, multi-architecture
+    prediction, cycle CoV, exact min-strata DP, CSV ingest, and the radix cell path"""
+    import os
+    tr = gen.make_trace("C2", n=60_000)
+    ctx = sieve.Ctx(device=0)
+    t = sieve.load_trace(ctx, tr["kid"], tr["x"], num_kernels=tr["K"], cta=tr["cta"], cycles=tr["y"])
+    sts = sieve.stratify_sweep(t, [(1, 10), (2, 5), (1, 1)])
+    sieve.tier_census(t, [(1, 10), (2, 5)])
+    st = sts[1]
+    rc = np.stack([st.table["rep_cycles"], st.table["rep_cycles"] * np.uint64(2)])
+    sieve.predict_multi(st, t, rc)
+    sid = torch.empty(len(tr["kid"]), dtype=torch.int32, device="cuda")
+    st2 = sieve.stratify(t, stratum_of_invocation=sid)
+    sieve.cycle_cov(st2, t, sid)
+    sieve.min_strata(t, theta=(2, 5))
+    lines = ["kernel,instr,cta,cycles"] + [f"k{k},{x},{c},{y}" for k, x, c, y in
+                                           zip(tr["kid"][:5000], tr["x"][:5000], tr["cta"][:5000], tr["y"][:5000])]
+    tc, names = sieve.load_csv(ctx, "\n".join(lines) + "\n", col_kernel=0, col_instr=1, col_cta=2, col_cycles=3)
+    sieve.stratify(tc)
+    os.environ["SIEVE_CELL_RADIX"] = "1"
+    sieve.stratify(t, grid_points=256)
+    del os.environ["SIEVE_CELL_RADIX"]
+    torch.cuda.synchronize()
+    print("other entry points ok", flush=True)
+
+
 if __name__ == "__main__":
+    other_entry_points()
     invalid_rows()
     one(gen.make_trace("C1"))
     one(gen.make_trace("C2"), n=200_000)
