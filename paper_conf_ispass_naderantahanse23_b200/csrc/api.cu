@@ -206,8 +206,10 @@ extern "C" int sieve_timing_get(sieve_ctx ctx, uint32_t phase, double* ms, uint6
   return SIEVE_OK;
 }
 
+static std::atomic<u64> g_trace_serial{0};
 struct sieve_trace_s {
   uint32_t magic = TRACE_MAGIC;
+  u64 serial = ++g_trace_serial;   // unique per trace handle (a freed handle's address may recur)
   sieve_ctx ctx = nullptr;
   u64 n = 0, first_id = 0;
   u32 K = 0;
@@ -236,6 +238,11 @@ struct sieve_strata_s {
   u64 kde_terms = 0, kde_evaluated = 0;
   u128 total_instr = 0, c_meas = 0;
   bool has_cycles = false;
+  // the prediction from the trace's own cycles, computed with the representatives (same kernel,
+  // same inputs as sieve_predict would use); valid for the trace it was stratified from
+  bool pred_ok = false;
+  u64 pred_serial = 0;
+  double pred_r[4] = {0, 0, 0, 0};
 };
 
 static bool ctx_ok(sieve_ctx c) { return c && c->magic == CTX_MAGIC; }
@@ -966,14 +973,22 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     std::vector<u32> seg_chunk;  // grouped path: first chunk of every segment
     u64 maxlen = 0;  // largest segment (local values)
     u64 nsup = 0;    // grouped path: values of the segments' source ranges
-    for (u32 s = 0; s < nseg; s++) {
+    // The bandwidths (a glibc pow each, A8) are needed first by the KDE: on the grouped path
+    // without the in-window count they are computed while the cell grouping runs (the grouping
+    // only reads lo, hi and the cell estimate) and uploaded with a second copy.
+    const bool late_h = grouped && !c->count_terms;
+    auto set_h = [&](u32 s) {
       const OpenSeg& o = op[s];
-      double h = scott_h(o.n, o.s1, o.s2, P->bw_scale);
+      const double h = scott_h(o.n, o.s1, o.s2, P->bw_scale);
       hh[s] = h;
-      hs[s].lo = o.lo;
-      hs[s].hi = o.hi;
       hs[s].h = h;
       hs[s].inv_h = 1.0 / h;
+    };
+    for (u32 s = 0; s < nseg; s++) {
+      const OpenSeg& o = op[s];
+      if (late_h) { hh[s] = hs[s].h = hs[s].inv_h = 0.0; } else { set_h(s); }
+      hs[s].lo = o.lo;
+      hs[s].hi = o.hi;
       hs[s].cq = (double)(G - 1) / (double)(o.hi - o.lo);
       hs[s].cm = cell_margin(o.lo, o.hi, G);
       u64 len = round == 1 ? h_localn[o.kid] : o.e - o.b;
@@ -1030,6 +1045,12 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
                         rel.get(), tot.get(), off.get(), stemp.get(), ck.get(),
                         c->count_terms ? terms.get() : nullptr, S);
       SV_CUDA(cudaGetLastError());
+      if (late_h) {  // the bandwidths, while the grouping runs; the KDE reads them from this copy
+        for (u32 s = 0; s < nseg; s++) set_h(s);
+        CopyBatch hcb(c);
+        SV_TRY(hcb.add_h2d(segs.get(), hs));
+        SV_TRY(hcb.flush());
+      }
     } else
     {
       DBuf<char> tmp(c);
@@ -1260,12 +1281,22 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   SV_TRY(d_ktab.alloc(K));
   SV_TRY(d_lows.alloc(lows.size()));
   SV_TRY(errf.alloc(4));
+  // the strata weights W_s = S1_s (u128) on the device for the prediction computed with the
+  // representatives (below), uploaded with the assignment tables
+  std::vector<u64> hW(2 * (size_t)ns);
+  for (u32 s = 0; s < ns; s++) { hW[2 * s] = (u64)fin[s].s1; hW[2 * s + 1] = (u64)(fin[s].s1 >> 64); }
+  DBuf<u64> dW(c);
+  DBuf<double> dpred(c);
+  SV_TRY(dW.alloc(std::max<size_t>(hW.size(), 2)));
+  SV_TRY(dpred.alloc(4));
   {
     CopyBatch cb(c);
     SV_TRY(cb.add_h2d(d_ktab.get(), ktab));
     SV_TRY(cb.add_h2d(d_lows.get(), lows));
+    SV_TRY(cb.add_h2d(dW.get(), hW));
     SV_TRY(cb.flush());
   }
+  std::vector<double> h_pred;
   u64 cap = 1;
   while (cap < std::max<u64>(1u << 16, 8ull * ns)) cap <<= 1;
   // One rank: the (stratum, CTA) entries go to the representatives without a host round trip --
@@ -1367,10 +1398,18 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     tr.stop();
     SV_CUDA(cudaGetLastError());
     SV_TRY(allreduce(c, repxy.get(), 2 * (size_t)ns, RED_SUM));   // AR-5: owner contributes
+    // the prediction from the trace's own cycles: the kernel and inputs
+    // sieve_predict uses, computed here so it costs no extra synchronisation
+    const bool pre_pred = t->y != nullptr && ns > 0;
+    if (pre_pred) {
+      PhaseTimer tpr(c, SIEVE_PHASE_PREDICT, 0);
+      launch_predict(dW.get(), repxy.get(), repxy.get() + ns, ns, 1, dpred.get(), S);
+    }
     {
       CopyBatch cb(c);
       SV_TRY(cb.add_d2h(h_rep, rep.get(), 2 * (size_t)ns));
       SV_TRY(cb.add_d2h(h_xy, repxy.get(), 2 * (size_t)ns));
+      if (pre_pred) SV_TRY(cb.add_d2h(h_pred, dpred.get(), 4));
       if (!c->comm) SV_TRY(cb.add_d2h(hflag, errf.get(), 4));
       if (h_terms.empty()) SV_TRY(cb.add_d2h(h_terms, terms.get(), 2));
       SV_TRY(cb.flush());
@@ -1380,6 +1419,11 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     break;
   }
   resolve_timing(c);
+  if (!h_pred.empty()) {
+    R->pred_ok = true;
+    R->pred_serial = t->serial;
+    for (int i = 0; i < 4; i++) R->pred_r[i] = h_pred[i];
+  }
   R->kde_terms = h_terms[0];
   R->kde_evaluated = h_terms[1];
   if (c->timing) c->acc[SIEVE_PHASE_KDE].work += h_terms[0];
@@ -1400,8 +1444,8 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     o.lo = f.lo; o.hi = f.hi; o.count = f.n;
     o.instr_sum_lo = (u64)f.s1; o.instr_sum_hi = (u64)(f.s1 >> 64);
     o.rep_id = h_rep[s];
-    o.rep_instr = h_xy[2 * (size_t)s];
-    o.rep_cycles = h_xy[2 * (size_t)s + 1];
+    o.rep_instr = h_xy[s];
+    o.rep_cycles = h_xy[ns + (size_t)s];
     o.bandwidth = f.h;
     o.split_round = f.round;
   }
@@ -1722,6 +1766,10 @@ static int predict_impl(sieve_strata s, sieve_trace t, u32 M, const uint64_t* re
   sieve_ctx c = t->ctx;
   SV_CUDA(cudaSetDevice(c->device));
   const u32 ns = (u32)s->st.size();
+  std::vector<double> r;
+  if (!rep_cycles && M == 1 && s->pred_ok && s->pred_serial == t->serial) {
+    r.assign(s->pred_r, s->pred_r + 4);   // computed with the representatives (sieve_stratify)
+  } else {
   SV_TRY(arena_reset(c));
   std::vector<u64> hW(2 * (size_t)ns), hx(ns), hy((size_t)M * ns);
   for (u32 i = 0; i < ns; i++) {
@@ -1745,10 +1793,10 @@ static int predict_impl(sieve_strata s, sieve_trace t, u32 M, const uint64_t* re
   launch_predict(dW.get(), dx.get(), dy.get(), ns, M, dout.get(), c->stream);
   tpr.stop();
   SV_CUDA(cudaGetLastError());
-  std::vector<double> r;
   SV_TRY(d2h(c, r, dout.get(), 4 * (size_t)M));
   SV_TRY(sync(c));
   resolve_timing(c);
+  }
   for (u32 m = 0; m < M; m++) {
     const double* rm = &r[4 * (size_t)m];
     sieve_prediction& o = out[m];

@@ -295,8 +295,8 @@ __global__ void k_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_loc
   if (s >= nstrata) return;
   u64 r = rep_id[s];
   bool mine = r >= first_id && r - first_id < n_local;
-  out[2 * (u64)s] = mine ? x[r - first_id] : 0;
-  out[2 * (u64)s + 1] = (mine && y) ? y[r - first_id] : 0;
+  out[s] = mine ? x[r - first_id] : 0;                          // [x of every stratum |
+  out[nstrata + (u64)s] = (mine && y) ? y[r - first_id] : 0;    //  y of every stratum]
 }
 
 void launch_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, const u64* x,

@@ -217,7 +217,7 @@ void launch_iota_u32(u32* p, u64 n, cudaStream_t s);
 // reduce duplicates of equal keys (sorted) and pick each stratum's representative
 void launch_reps(const u64* key, const u64* cnt, const u64* first, u64 E, const u32* tier,
                  u32 nstrata, u64* rep_id, u64* rep_cta, cudaStream_t s);
-// representative (x, y) from the owner rank: out[s*2] = x, out[s*2+1] = y (0 if not local)
+// representative (x, y) from the owner rank: out[s] = x, out[nstrata + s] = y (0 if not local)
 void launch_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, const u64* x,
                    const u64* y, u64* out, cudaStream_t s);
 
