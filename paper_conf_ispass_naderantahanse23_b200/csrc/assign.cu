@@ -69,6 +69,7 @@ __global__ void __launch_bounds__(AS_THREADS)
 k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __restrict__ cta,
          u64 n, u64 first_id, const KTab* __restrict__ g_ktab, const u64* __restrict__ g_lows,
          u32 K, u32 nlows, u32* __restrict__ sid_out, GHash gh, u64* errflags) {
+  pdl_begin();
   extern __shared__ __align__(16) unsigned char smem[];
   u64* hk = (u64*)smem;              // [AS_HC]
   u32* hc = (u32*)(hk + AS_HC);      // [AS_HC]
@@ -219,6 +220,7 @@ void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 firs
 
 __global__ void k_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst,
                                unsigned long long* count) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   bool occ = i < gh.cap && gh.keys[i] != HASH_EMPTY;
   u32 m = __ballot_sync(0xffffffffu, occ);
@@ -239,6 +241,7 @@ void launch_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst, unsigned l
 }
 
 __global__ void k_iota_u32(u32* p, u64 n) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) p[i] = (u32)i;
 }
@@ -248,6 +251,7 @@ void launch_iota_u32(u32* p, u64 n, cudaStream_t s) {
 
 // stratum id of every compacted (stratum, CTA) entry; neutral slots (key ~0) map to ns
 __global__ void k_entry_sids(const u64* key, u64 n, u32 ns, u64* out) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) { u64 s = key[i] >> 32; out[i] = s < ns ? s : ns; }
 }
@@ -256,6 +260,7 @@ void launch_entry_sids(const u64* key, u64 n, u32 ns, u64* out, cudaStream_t s) 
 }
 
 __global__ void k_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) dst[i] = src[idx[i]];
 }
@@ -266,6 +271,7 @@ void launch_gather_u64(const u64* src, const u32* idx, u64 n, u64* dst, cudaStre
 // one thread per stratum over its (sorted) entries; equal keys (from different ranks) merge
 __global__ void k_reps(const u64* key, const u64* cnt, const u64* first, u64 E, const u32* tier,
                        u32 nstrata, u64* rep_id, u64* rep_cta) {
+  pdl_begin();
   u32 s = blockIdx.x * blockDim.x + threadIdx.x;
   if (s >= nstrata) return;
   u64 lo = 0, hi = E;
@@ -291,6 +297,7 @@ void launch_reps(const u64* key, const u64* cnt, const u64* first, u64 E, const 
 
 __global__ void k_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, const u64* x,
                          const u64* y, u64* out) {
+  pdl_begin();
   u32 s = blockIdx.x * blockDim.x + threadIdx.x;
   if (s >= nstrata) return;
   u64 r = rep_id[s];
@@ -311,9 +318,11 @@ void launch_rep_xy(const u64* rep_id, u32 nstrata, u64 first_id, u64 n_local, co
 // trace) occupies the copy engines for tens of milliseconds; copy-engine work queued behind it
 // would stall every synchronisation of this call.
 __global__ void k_copy_words(u32* __restrict__ dst, const u32* __restrict__ src, u64 n) {
+  pdl_begin();
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) dst[i] = src[i];
 }
 __global__ void k_copy_bytes(unsigned char* __restrict__ dst, const unsigned char* __restrict__ src, u64 n) {
+  pdl_begin();
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) dst[i] = src[i];
 }
 void launch_copy(void* dst, const void* src, u64 bytes, cudaStream_t s) {
@@ -330,6 +339,7 @@ void launch_copy(void* dst, const void* src, u64 bytes, cudaStream_t s) {
 // several copies in ONE launch (blockIdx.y = region): the orchestrator's small host <-> device
 // tables of one step go together (each separate copy was a launch plus a PCIe round trip)
 __global__ void k_copy_multi(CopyRegions r) {
+  pdl_begin();
   const int q = blockIdx.y;
   if (q >= r.k) return;
   unsigned char* d = (unsigned char*)r.dst[q];
@@ -355,6 +365,7 @@ void launch_copy_multi(const CopyRegions& r, cudaStream_t s) {
 }
 
 __global__ void k_fill_u64(u64* p, u64 n, u64 v) {
+  pdl_begin();
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) p[i] = v;
 }
 void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s) {
@@ -362,6 +373,7 @@ void launch_fill_u64(u64* p, u64 n, u64 v, cudaStream_t s) {
 }
 // several fills in one launch (FILL_MAX regions): per-round buffer initialisation
 __global__ void k_fill_multi(FillRegions r) {
+  pdl_begin();
   for (int q = 0; q < r.k; q++)
     for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < r.n[q]; i += (u64)gridDim.x * blockDim.x)
       r.p[q][i] = r.v[q];
@@ -373,10 +385,12 @@ void launch_fill_multi(const FillRegions& r, cudaStream_t s) {
 }
 
 __global__ void k_u128_to_limbs(const u64* src, u64 n, u64* limbs) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) limbs_from_u128(src[2 * i], src[2 * i + 1], limbs + 4 * i);
 }
 __global__ void k_limbs_to_u128(const u64* limbs, u64 n, u64* dst) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) limbs_to_u128(limbs + 4 * i, dst + 2 * i, dst + 2 * i + 1);
 }
@@ -389,6 +403,7 @@ void launch_limbs_to_u128(const u64* limbs, u64 n, u64* dst, cudaStream_t s) {
 
 // MIN folded into MAX for the grouped cross-rank reductions: min(a, b) = ~max(~a, ~b)
 __global__ void k_complement(u64* p, u64 n, u64 stride) {
+  pdl_begin();
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x)
     p[i * stride] = ~p[i * stride];
 }
@@ -399,6 +414,7 @@ void launch_complement(u64* p, u64 n, u64 stride, cudaStream_t s) {
 // pass B's exchange word set (one SUM all-reduce of world + 1 lanes, no host round trip before
 // it): x[0] = this rank's table-overflow flag, x[1 + r] = rank r's entry count (0 elsewhere)
 __global__ void k_exchange_prep(const u64* flag, const unsigned long long* count, int rank, int world, u64* x) {
+  pdl_begin();
   int i = threadIdx.x;
   if (i == 0) x[0] = flag[0] ? 1ull : 0ull;
   if (i < world) x[1 + i] = i == rank ? (u64)count[0] : 0ull;
@@ -410,6 +426,7 @@ void launch_exchange_prep(const u64* flag, const unsigned long long* count, int 
 
 // 16-bit trace columns (SIEVE_KID16 / SIEVE_CTA16) widened to the library's u32 columns
 __global__ void k_widen_u16(const unsigned short* __restrict__ src, u64 n, u32* __restrict__ dst) {
+  pdl_begin();
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (u64)gridDim.x * blockDim.x) dst[i] = src[i];
 }
 void launch_widen_u16(const void* src, u64 n, u32* dst, cudaStream_t s) {

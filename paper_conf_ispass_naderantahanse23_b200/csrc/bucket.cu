@@ -40,6 +40,7 @@ __device__ __forceinline__ double grid_pt_b(u64 lo, u64 hi, u32 j, u32 G) {
 }
 
 __global__ void k_grid_tab(const SegDev* __restrict__ segs, u32 nseg, u32 G, double* __restrict__ gtab) {
+  pdl_begin();
   u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (id >= (u64)nseg * G) return;
   u32 s = (u32)(id / G), j = (u32)(id % G);
@@ -104,6 +105,7 @@ k_cellkey(const BucketChunk* __restrict__ chunks, u32 nchunks, const u64* __rest
           u32 bx, u32 in_shift, const SegDev* __restrict__ segs, u32 G, const double* __restrict__ gtab,
           u32 ib, u32 ncell, u32 seg0, u64* __restrict__ out, unsigned long long* inwin,
           u32* __restrict__ ghist) {
+  pdl_begin();
   // ghist != nullptr: the radix sort's digit histograms of the output keys over bits [0, ib)
   // (the cell index) are accumulated here, so the sort skips its own histogram read
   __shared__ u32 s_hist[3 * 256];
@@ -186,6 +188,7 @@ void launch_cellkey(const BucketChunk* chunks, const u64* in, u64 nin, u32 bx, u
 // off[c] = first position of the sorted keys with idx >= c, c = 0..ncell (position i writes the
 // cells (idx(i-1), idx(i)]; position n writes the cells after the last key)
 __global__ void k_cell_offsets(const u64* __restrict__ keys, u64 n, u32 ib, u32 ncell, u32* __restrict__ off) {
+  pdl_begin();
   const u64 imask = (1ull << ib) - 1;
   const u64 stride = (u64)gridDim.x * blockDim.x;
   for (u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x; i <= n; i += stride) {
@@ -215,6 +218,7 @@ void launch_cell_offsets(const u64* keys, u64 n, u32 ib, u32 ncell, u32* off, cu
 // part_off[nseg] = number of parts -- the host needs no copy of the cut counts before the part
 // moments are launched
 __global__ void __launch_bounds__(1024) k_part_offsets(const u32* __restrict__ nt, u32 nseg, u32* part_off) {
+  pdl_begin();
   __shared__ u32 carry;
   __shared__ u32 wsum[32];
   if (threadIdx.x == 0) carry = 0;
@@ -253,6 +257,7 @@ __global__ void k_part_ranges(const SegDev* __restrict__ segs, u32 nseg, u32 G,
                               const double* __restrict__ gtab, const u32* __restrict__ off,
                               const u64* __restrict__ T, u32 tstride, const u32* __restrict__ nt,
                               const u32* __restrict__ part_off, u32 cap, u64* ab, u32* items) {
+  pdl_begin();
   u32 p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p >= cap) return;
   if (p >= part_off[nseg]) { items[p] = 0; return; }
@@ -281,6 +286,7 @@ __global__ void k_part_ranges(const SegDev* __restrict__ segs, u32 nseg, u32 G,
 __global__ void __launch_bounds__(PS_THREADS)
 k_part_stats(const u64* __restrict__ ab, const u32* __restrict__ item_off, u32 cap,
              const u64* __restrict__ vals, u32 vshift, u64* lanes, u64* mm) {
+  pdl_begin();
   __shared__ u64 r[PS_THREADS / 32][7];
   const u32 total = item_off[cap];
   for (u32 item = blockIdx.x; item < total; item += gridDim.x) {
@@ -362,6 +368,7 @@ void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, 
 __global__ void k_part_pack(const u32* __restrict__ part_off, u32 nseg, u32 cap, const u64* __restrict__ lanes,
                             const u64* __restrict__ mm, const u64* __restrict__ ab, const u32* __restrict__ ntk,
                             u32 tp, u32 tq, u64* out) {
+  pdl_begin();
   const u32 nparts = part_off[nseg];
   u32 p = blockIdx.x * blockDim.x + threadIdx.x;
   if (p == 0) out[0] = nparts;
@@ -416,6 +423,7 @@ void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, 
 __global__ void __launch_bounds__(GR_THREADS)
 k_group_t3(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, const u32* __restrict__ t3rank,
            u32 n_t3, const u32* __restrict__ seg_base, u32* __restrict__ cursor, u64* __restrict__ out) {
+  pdl_begin();
   extern __shared__ u32 s_cnt[];      // [n_t3]: tile counts, then the tile's output bases
   __shared__ u32 s_list[GR_THREADS * GT_ROWS];
   __shared__ u32 s_nlist;
@@ -486,6 +494,7 @@ __device__ __forceinline__ void t3_range(u64 n, u32 nb, u32 b, u64* r0, u64* r1)
 __global__ void __launch_bounds__(T3_THREADS)
 k_t3_count(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, u32 K, const u32* __restrict__ t3rank,
            u32 n_t3, const u32* __restrict__ n_t3_dev, u32* __restrict__ cnt) {
+  pdl_begin();
   extern __shared__ u32 s_c[];   // [n_t3]
   if (n_t3_dev) n_t3 = *n_t3_dev;
   for (u32 i = threadIdx.x; i < n_t3; i += T3_THREADS) s_c[i] = 0;
@@ -517,6 +526,7 @@ k_t3_count(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, u32 K,
 __global__ void k_t3_offsets(u32* __restrict__ cnt, u32 nb, u32 n_t3, const u32* __restrict__ n_t3_dev,
                              const u32* __restrict__ seg_base, const KMomPartial* __restrict__ part, u32 kt,
                              const u32* __restrict__ t3kern) {
+  pdl_begin();
   const u32 t = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (n_t3_dev) n_t3 = *n_t3_dev;
   if (t >= n_t3) return;
@@ -540,6 +550,7 @@ __global__ void k_t3_offsets(u32* __restrict__ cnt, u32 nb, u32 n_t3, const u32*
 __global__ void __launch_bounds__(T3_SC_THREADS)
 k_t3_scatter(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n, u32 K, const u32* __restrict__ t3rank,
              u32 n_t3, const u32* __restrict__ n_t3_dev, const u32* __restrict__ off, u64* __restrict__ out) {
+  pdl_begin();
   if (n_t3_dev) n_t3 = *n_t3_dev;
   extern __shared__ u32 s_cur[];   // [n_t3]: this block's next output position per segment
   for (u32 t = threadIdx.x; t < n_t3; t += T3_SC_THREADS) s_cur[t] = off[(u64)t * gridDim.x + blockIdx.x];
@@ -599,6 +610,7 @@ void launch_group_t3(const u32* kid, const u64* x, u64 n, u32 K, const u32* t3ra
 __global__ void __launch_bounds__(GR_THREADS)
 k_cell_hist(const BucketChunk* __restrict__ chunks, const u64* __restrict__ src, const SegDev* __restrict__ segs,
             u32 G, unsigned short* __restrict__ cells, u32* __restrict__ hist, unsigned long long* inwin) {
+  pdl_begin();
   extern __shared__ u32 s_h2[];       // [ceil(G / 2)]
   const BucketChunk ch = chunks[blockIdx.x];
   const u32 gw = (G + 1) / 2;
@@ -648,6 +660,7 @@ k_cell_hist(const BucketChunk* __restrict__ chunks, const u64* __restrict__ src,
 // consecutive cells of a chunk)
 __global__ void k_cell_walk(const u32* __restrict__ seg_chunk, u32 nseg, u32 G, const u32* __restrict__ hist,
                             u32* __restrict__ rel, u32* __restrict__ tot) {
+  pdl_begin();
   const u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (id >= (u64)nseg * G) return;
   const u32 s = (u32)(id / G), c = (u32)(id % G);
@@ -696,6 +709,7 @@ __global__ void __launch_bounds__(GR_THREADS)
 k_cell_scatter(const BucketChunk* __restrict__ chunks, const u64* __restrict__ src,
                const unsigned short* __restrict__ cells, u32 G, const u32* __restrict__ hist,
                const u32* __restrict__ rel, const u32* __restrict__ off, u64* __restrict__ out) {
+  pdl_begin();
   extern __shared__ __align__(16) unsigned char smem[];
   u64* s_v = (u64*)smem;                          // [GR_CH]
   unsigned short* s_c = (unsigned short*)(s_v + GR_CH);   // [GR_CH]

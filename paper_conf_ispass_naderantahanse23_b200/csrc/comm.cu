@@ -145,6 +145,7 @@ struct sieve_group_s {
 struct PtrPack { const u64* p[GROUP_MAX]; };
 
 __global__ void k_group_reduce(PtrPack pk, int world, size_t n, int op, u64* out) {
+  pdl_begin();
   for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
     u64 v = pk.p[0][i];
     for (int r = 1; r < world; r++) {

@@ -126,7 +126,40 @@ int sv_num_sms();
 // every kernel launch of the library goes through SV_LAUNCH so the process-wide launch
 // count (sieve_kernel_launches) is exact
 void sv_count_launch();
-#define SV_LAUNCH(k, g, b, sm, st) sv_count_launch(), k<<<g, b, sm, st>>>
+
+// Programmatic dependent launch (sm_90+): every kernel of the library is launched with
+// programmatic stream serialisation and starts with pdl_begin(), which waits for the preceding
+// grid to complete (its memory visible) before touching global memory, then lets the next
+// kernel's blocks be scheduled as this grid's blocks retire.  The next kernel's launch and block
+// dispatch overlap this one's tail instead of following it: the per-round chains of short
+// kernels are launch-latency bound.
+__device__ __forceinline__ void pdl_begin() {
+  asm volatile("griddepcontrol.wait;\n\tgriddepcontrol.launch_dependents;" ::: "memory");
+}
+template <typename F>
+struct PdlLaunch {
+  F* k;
+  dim3 g, b;
+  size_t sm;
+  cudaStream_t st;
+  template <typename... A>
+  void operator()(A... args) const {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = g;
+    cfg.blockDim = b;
+    cfg.dynamicSmemBytes = sm;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaLaunchKernelEx(&cfg, k, args...);
+  }
+};
+template <typename F>
+inline PdlLaunch<F> sv_pdl(F* k, dim3 g, dim3 b, size_t sm, cudaStream_t st) { return PdlLaunch<F>{k, g, b, sm, st}; }
+#define SV_LAUNCH(k, g, b, sm, st) sv_count_launch(), sv_pdl(k, dim3(g), dim3(b), (size_t)(sm), st)
 
 // cudaFuncSetAttribute(MaxDynamicSharedMemorySize) once per (kernel, device, size): launchers
 // run on the host between synchronisations, where every driver call is GPU idle time

@@ -21,6 +21,7 @@ void scan_u32(const u32* in, u32* out, u64 n, void* temp, u32* total, cudaStream
 
 __global__ void __launch_bounds__(CSV_THREADS)
 k_csv_count(const unsigned char* __restrict__ buf, u64 nbytes, u32* __restrict__ tile_count) {
+  pdl_begin();
   u64 base = (u64)blockIdx.x * CSV_TILE + (u64)threadIdx.x * CSV_TB;
   u32 c = 0;
   for (u32 j = 0; j < CSV_TB; j++) {
@@ -42,6 +43,7 @@ k_csv_count(const unsigned char* __restrict__ buf, u64 nbytes, u32* __restrict__
 __global__ void __launch_bounds__(CSV_THREADS)
 k_csv_ends(const unsigned char* __restrict__ buf, u64 nbytes, const u32* __restrict__ tile_off,
            u64* __restrict__ ends) {
+  pdl_begin();
   u64 base = (u64)blockIdx.x * CSV_TILE + (u64)threadIdx.x * CSV_TB;
   u32 c = 0;
   for (u32 j = 0; j < CSV_TB; j++) {
@@ -92,6 +94,7 @@ __global__ void k_csv_parse(const unsigned char* __restrict__ buf, u64 nbytes,
                             CsvSpec spec, u64* __restrict__ hash, u32* __restrict__ row,
                             u64* __restrict__ name_pos, u64* __restrict__ x, u32* __restrict__ cta,
                             u64* __restrict__ y, u64* errflag) {
+  pdl_begin();
   u64 r = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= nrows) return;
   u64 line = first_line + r;
@@ -133,6 +136,7 @@ __global__ void k_csv_parse(const unsigned char* __restrict__ buf, u64 nbytes,
 
 // after sorting (hash, row) by hash (stable): flag[i] = 1 if i starts a new distinct hash
 __global__ void k_csv_heads(const u64* __restrict__ h, u64 n, u32* __restrict__ flag) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) flag[i] = (i == 0 || h[i] != h[i - 1]) ? 1u : 0u;
 }
@@ -141,6 +145,7 @@ __global__ void k_csv_heads(const u64* __restrict__ h, u64 n, u32* __restrict__ 
 __global__ void k_csv_firsts(const u32* __restrict__ flag, const u32* __restrict__ seg,
                              const u32* __restrict__ row, u64 n, u64* __restrict__ first_key,
                              u32* __restrict__ first_val) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n && flag[i]) {
     first_key[seg[i]] = row[i];
@@ -150,6 +155,7 @@ __global__ void k_csv_firsts(const u32* __restrict__ flag, const u32* __restrict
 
 // id of distinct hash d = rank of its first row; scatter to every row
 __global__ void k_csv_rank(const u32* __restrict__ order, u64 nd, u32* __restrict__ id_of) {
+  pdl_begin();
   u64 r = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (r < nd) id_of[order[r]] = (u32)r;
 }
@@ -157,11 +163,13 @@ __global__ void k_csv_rank(const u32* __restrict__ order, u64 nd, u32* __restric
 __global__ void k_csv_scatter(const u32* __restrict__ flag, const u32* __restrict__ seg,
                               const u32* __restrict__ row, const u32* __restrict__ id_of, u64 n,
                               u32* __restrict__ kid) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) kid[row[i]] = id_of[seg[i] + flag[i] - 1];
 }
 
 __global__ void k_gather_pairs(const u64* src, const u64* idx, u64 n, u64* dst) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) { dst[2 * i] = src[2 * idx[i]]; dst[2 * i + 1] = src[2 * idx[i] + 1]; }
 }

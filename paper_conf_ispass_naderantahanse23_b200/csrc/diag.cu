@@ -20,6 +20,7 @@ int group_moments_kt(u32 ns) { return (int)(ns < GM_KT ? ns : GM_KT); }
 __global__ void __launch_bounds__(GM_THREADS)
 k_group_moments(const u32* __restrict__ sid, const u64* __restrict__ y, u64 n, u32 k0, u32 kt,
                 GMomPartial* __restrict__ part, u64* errflag) {
+  pdl_begin();
   extern __shared__ __align__(16) u32 s_w[];  // [GM_WORDS][kt]
   GMomPartial* rec = part + (u64)blockIdx.x * kt;
   for (u32 i = threadIdx.x; i < kt; i += blockDim.x) {
@@ -85,6 +86,7 @@ k_group_moments(const u32* __restrict__ sid, const u64* __restrict__ y, u64 n, u
 // S2 (6 limbs: a cross-rank S2 can exceed 2^128)
 __global__ void k_group_moments_reduce(const GMomPartial* __restrict__ part, int grid, u32 k0,
                                        u32 kt, u64* lanes) {
+  pdl_begin();
   u32 l = blockIdx.x * blockDim.x + threadIdx.x;
   if (l >= kt) return;
   u64 n = 0;

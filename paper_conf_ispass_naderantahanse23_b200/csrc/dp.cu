@@ -100,6 +100,7 @@ k_min_strata(const u64* __restrict__ ukey, const u32* __restrict__ ustart, const
              u64 xmask, u32 p, u32 q, u32 max_distinct, u64* __restrict__ Pn, u128* __restrict__ P1,
              u128* __restrict__ P2, u32* __restrict__ f, u32* __restrict__ arg, u32* __restrict__ count,
              u64* __restrict__ cuts) {
+  pdl_begin();
   __shared__ u64 s_n[DP_THREADS];
   __shared__ u128 s_1[DP_THREADS], s_2[DP_THREADS];
   __shared__ u64 red[33];
@@ -185,6 +186,7 @@ k_min_strata(const u64* __restrict__ ukey, const u32* __restrict__ ustart, const
 __global__ void k_rle(const u64* __restrict__ keys, const u32* __restrict__ flag,
                       const u32* __restrict__ seg, u64 n, u32 bx, u64* __restrict__ ukey,
                       u32* __restrict__ ustart, u32* __restrict__ kstart) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n || !flag[i]) return;
   u32 d = seg[i];
@@ -197,6 +199,7 @@ __global__ void k_rle(const u64* __restrict__ keys, const u32* __restrict__ flag
 __global__ void k_dp_gather(const u32* __restrict__ kstart, const u32* __restrict__ count,
                             const u64* __restrict__ off, const u64* __restrict__ cuts,
                             u64* __restrict__ out) {
+  pdl_begin();
   const u32 r = blockIdx.x;
   const u32 c = count[r];
   if (c < 2 || c == 0xFFFFFFFFu) return;

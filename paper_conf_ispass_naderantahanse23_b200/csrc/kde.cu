@@ -59,6 +59,7 @@ __device__ __forceinline__ double grid_pt(u64 lo, u64 hi, u32 j, u32 G) {
 // too; their terms are exactly 0 (k > 10526).
 __global__ void k_kde_tiles(const SegDev* segs, u32 nseg, u32 G, u32 tps, const double* gtab,
                             const u32* off, u64* tile_range, u32* tile_items) {
+  pdl_begin();
   u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (id >= (u64)nseg * tps) return;
   u32 s = (u32)(id / tps), t = (u32)(id % tps);
@@ -108,6 +109,7 @@ static_assert(sizeof(KdeItem) == 48, "KdeItem is copied as three 16-byte pieces"
 __global__ void k_kde_items(const SegDev* __restrict__ segs, u32 G, u32 tps,
                             const u64* __restrict__ tile_range, const u32* __restrict__ tile_items,
                             u32 ntiles, KdeItem* __restrict__ desc) {
+  pdl_begin();
   const u32 items = tile_items[ntiles];  // device-side total (no host round trip)
   for (u32 it = blockIdx.x * blockDim.x + threadIdx.x; it < items; it += gridDim.x * blockDim.x) {
     u32 lo = 0, hi = ntiles - 1;
@@ -326,6 +328,7 @@ __global__ void __launch_bounds__(32 * KDE_WARPS, KDE_MINB)
 k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
       const u64* __restrict__ vals, u32 vshift, u64* D, unsigned long long* evaluated,
       bool allow_fast) {
+  pdl_begin();
   extern __shared__ __align__(16) unsigned char smem[];
   double* sS = (double*)smem;
 #if KDE_SPLIT
@@ -433,6 +436,7 @@ k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
 
 // D[2j] (sum of low 32-bit limbs), D[2j + 1] (sum of high parts) -> u128 D_j
 __global__ void k_kde_fix(u64* D, u64 n) {
+  pdl_begin();
   u64 i = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   u64 lo = D[2 * i], hi = D[2 * i + 1];

@@ -70,6 +70,7 @@ __global__ void __launch_bounds__(MOM_THREADS, MOM_MINB)
 k_moments(const u32* __restrict__ kid, const u64* __restrict__ x, const u64* __restrict__ y,
           u64 n, u32 K, u32 k0, u32 kt, u32 nrep, KMomPartial* __restrict__ part,
           u64* __restrict__ blk_tot, u64* errflags) {
+  pdl_begin();
   extern __shared__ __align__(16) unsigned char smem[];
   u64* s_mn = (u64*)smem;                 // [kt]
   u64* s_mx = s_mn + kt;                  // [kt]
@@ -269,6 +270,7 @@ __device__ __forceinline__ u128 shfl_xor_u128(u128 v, int o) {
 }
 __global__ void k_moments_reduce(const KMomPartial* __restrict__ part, int grid, u32 k0, u32 kt,
                                  u64* lanes, u64* mm, u64* local_n) {
+  pdl_begin();
   u32 l = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (l >= kt) return;  // warp-uniform
   u128 n = 0, s1 = 0, s2 = 0;
@@ -302,6 +304,7 @@ __global__ void k_moments_reduce(const KMomPartial* __restrict__ part, int grid,
 }
 
 __global__ void k_totals_reduce(const u64* blk_tot, int grid, u64* tot_lanes, u64* tot_max) {
+  pdl_begin();
   if (blockIdx.x != 0 || threadIdx.x >= 32) return;
   u128 c = 0;
   u64 mx = 0;
@@ -336,6 +339,7 @@ __global__ void __launch_bounds__(1024) k_tiers(const u64* __restrict__ lanes, c
                                                 const u64* __restrict__ local_n, u32 K, u32 p, u32 q,
                                                 u32* __restrict__ t3rank, u32* __restrict__ seg_base,
                                                 u32* __restrict__ t3kern, u32* __restrict__ counts) {
+  pdl_begin();
   __shared__ u32 s_w[32], s_r[32];
   __shared__ u32 c_rank, c_rows;
   if (threadIdx.x == 0) { c_rank = 0; c_rows = 0; }

@@ -33,6 +33,7 @@ __device__ __forceinline__ double u128_to_double(u64 lo, u64 hi) {
 
 __global__ void __launch_bounds__(PR_THREADS)
 k_predict(const u64* W, const u64* rx, const u64* ry, u32 nstrata, double* out) {
+  pdl_begin();
   __shared__ DD s_c[PR_THREADS], s_i[PR_THREADS];
   __shared__ DD s_y[PR_THREADS];
   // block m predicts for the m-th cycle vector (one architecture each)

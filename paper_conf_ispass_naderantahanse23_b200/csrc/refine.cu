@@ -145,6 +145,7 @@ __device__ u32 valley_warp(const u64* src, u32 G, u64 mx, u32 shift, const SegDe
 __global__ void __launch_bounds__(32 * VAL_WARPS)
 k_valleys(const SegDev* segs, u32 nseg, u32 G, u32 shift, u64* D, u64* T, u32 tstride,
           u32* nt, u32* kind, bool writeback) {
+  pdl_begin();
   extern __shared__ __align__(16) unsigned char vsm[];
   u32 w = threadIdx.x >> 5;
   u32 s = blockIdx.x * VAL_WARPS + w;

@@ -65,6 +65,7 @@ __device__ __forceinline__ T block_excl_scan(T v, T* total) {
 #define SC_TILE (SC_THREADS * SC_IPT)
 
 __global__ void __launch_bounds__(SC_THREADS) k_scan_reduce(const u32* in, u64 n, u32* bsum) {
+  pdl_begin();
   u64 base = (u64)blockIdx.x * SC_TILE;
   u32 s = 0;
 #pragma unroll
@@ -78,6 +79,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_reduce(const u32* in, u64 n
 }
 
 __global__ void __launch_bounds__(SC_THREADS) k_scan_blocks(u32* bsum, u32 nb, u32* total) {
+  pdl_begin();
   __shared__ u32 carry_s;
   if (threadIdx.x == 0) carry_s = 0;
   __syncthreads();
@@ -97,6 +99,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_blocks(u32* bsum, u32 nb, u
 
 __global__ void __launch_bounds__(SC_THREADS) k_scan_apply(const u32* in, u64 n, const u32* bsum,
                                                            u32* out) {
+  pdl_begin();
   u64 base = (u64)blockIdx.x * SC_TILE + (u64)threadIdx.x * SC_IPT;
   u32 v[SC_IPT];
   u32 s = 0;
@@ -119,6 +122,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_apply(const u32* in, u64 n,
 // synchronisations is GPU idle time)
 #define SC_SMALL 4
 __global__ void __launch_bounds__(SC_THREADS) k_scan_single(const u32* in, u64 n, u32* out, u32* total) {
+  pdl_begin();
   __shared__ u32 carry_s;
   if (threadIdx.x == 0) carry_s = 0;
   __syncthreads();
@@ -172,6 +176,7 @@ void scan_set_state(u64* state) { tl_scan_state = state; }
 
 __global__ void __launch_bounds__(SC_THREADS) k_scan_sp(const u32* in, u32* out, u64 n, u32 ntiles, u64* st,
                                                         u32* total) {
+  pdl_begin();
   __shared__ u32 s_tile;
   __shared__ u64 s_excl;
   __shared__ bool s_last;
@@ -253,6 +258,7 @@ __global__ void __launch_bounds__(CP_THREADS)
 k_t3_compact(const u32* __restrict__ kid, const u64* __restrict__ x, u64 n,
              const u32* __restrict__ t3rank, u32 bx, u64* __restrict__ keys,
              unsigned long long* counter) {
+  pdl_begin();
   const u64 tile = (u64)CP_THREADS * CP_IPT;
   for (u64 base = (u64)blockIdx.x * tile; base < n; base += (u64)gridDim.x * tile) {
     u64 key[CP_IPT];
@@ -318,6 +324,7 @@ void launch_t3_compact(const u32* kid, const u64* x, u64 n, const u32* t3rank, u
 
 __global__ void __launch_bounds__(RS_THREADS)
 k_os_hist(const u64* __restrict__ keys, u64 n, int npass, u64 kmask, u32* __restrict__ ghist) {
+  pdl_begin();
   extern __shared__ u32 s_hist[];  // [RS_WARPS/2][npass][256] (pairs of warps share a table)
   const int tables = RS_WARPS / 2;
   for (int i = threadIdx.x; i < tables * npass * 256; i += RS_THREADS) s_hist[i] = 0;
@@ -340,6 +347,7 @@ __global__ void __launch_bounds__(RS_THREADS, RS_MINB)
 k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int shift, u32 dmask,
           const u32* __restrict__ gbase, u64* status, u32* tile_counter, u64* __restrict__ kout,
           u32* __restrict__ vout) {
+  pdl_begin();
   extern __shared__ __align__(16) unsigned char smem[];
   const int dbits = __popc(dmask);
   u64* s_k = (u64*)smem;                        // [RS_TILE]
@@ -446,6 +454,7 @@ k_os_pass(const u64* __restrict__ kin, const u32* __restrict__ vin, u64 n, int s
 
 // exclusive scan of each pass's 256-bin histogram (one block of 256 threads per pass)
 __global__ void __launch_bounds__(RS_THREADS) k_os_scan(const u32* __restrict__ ghist, u32* __restrict__ gbase) {
+  pdl_begin();
   __shared__ u32 tot;
   u32 v = ghist[blockIdx.x * 256 + threadIdx.x];
   gbase[blockIdx.x * 256 + threadIdx.x] = block_excl_scan<u32, RS_THREADS>(v, &tot);

@@ -58,6 +58,14 @@ def main():
             busy += max(0.0, f - end)
             end = max(end, f)
     per = a.steps
+    # the largest single gaps with their neighbours (one step's worth)
+    singles = []
+    for p_, e in zip(ev[:-1], ev[1:]):
+        g = e.time_range.start - p_.time_range.end
+        if g > 0:
+            singles.append((g, p_.name.split("(")[0][:32], e.name.split("(")[0][:32]))
+    singles.sort(reverse=True)
+    print("largest gaps (us): " + "; ".join(f"{g:.1f} {a_} -> {b_}" for g, a_, b_ in singles[:3 * per + 6]))
     print(f"{len(ev)} device events over {per} steps: span {span / 1e3 / per:.3f} ms/step, busy "
           f"{busy / 1e3 / per:.3f} ms/step, idle {(span - busy) / 1e3 / per:.3f} ms/step "
           f"(between the first and the last kernel)")
