@@ -246,6 +246,11 @@ struct sieve_strata_s {
 };
 
 static bool ctx_ok(sieve_ctx c) { return c && c->magic == CTX_MAGIC; }
+// a stratum-table buffer kept per thread between results (a result's table is ~100 B per stratum)
+static std::vector<sieve_stratum>& spare_strata() {
+  static thread_local std::vector<sieve_stratum> v;
+  return v;
+}
 static bool trace_ok(sieve_trace t) { return t && t->magic == TRACE_MAGIC && ctx_ok(t->ctx); }
 static bool strata_ok(sieve_strata s) { return s && s->magic == STRATA_MAGIC; }
 
@@ -822,10 +827,17 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
                          const MomentsHost* cached) {
   sieve_ctx c = t->ctx;
   cudaStream_t S = c->stream;
+  const auto t_entry = std::chrono::steady_clock::now();
   SV_TRY(arena_reset(c));
   ScanScope scan_scope(c);
   HostClock hc;
   hc.c = c;
+  if (hc.on) {
+    char b[64];
+    snprintf(b, sizeof b, " reset=%.3f",
+             std::chrono::duration<double, std::milli>(hc.t0 - t_entry).count());
+    hc.out += b;
+  }
   const u32 K = t->K, G = P->grid_points;
   const u64 n = t->n;
   MomentsHost own;
@@ -967,6 +979,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     const OpenSeg* op = open.data() + s0;
     const u64 ncell = (u64)nseg * G;
     const u32 ib = std::max<u32>(1, bitlen(ncell));
+    hc.mark("r0");
     std::vector<SegDev> hs(nseg);
     std::vector<double> hh(nseg);
     std::vector<BucketChunk> chunks;
@@ -1017,6 +1030,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     DBuf<u64> ck(c);
     DBuf<BucketChunk> d_chunks(c);
     SV_TRY(segs.alloc(nseg));
+    hc.mark("segs");
     CopyBatch rcb(c);   // this round's tables: one upload
     SV_TRY(rcb.add_h2d(segs.get(), hs));
     SV_TRY(gtab.alloc(ncell));
@@ -1240,30 +1254,36 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   hc.mark("rend");
 
   // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
-  {  // counting sort by kernel, then by lo inside each kernel's (short) run: O(#strata + K).
-     // The scratch vectors are the thread's, reused across calls: a fresh 260 KB vector per call
-     // cost more (page faults, zero fill) than the sort itself.
-    static thread_local std::vector<u32> cnt, pos;
-    static thread_local std::vector<Fin> by;
+  // Stratum order (kernel, lo) as a permutation of fin: a counting sort by kernel, then the few
+  // entries of each Tier-3 kernel by lo.  Indices move, not the 80-byte entries, and the scratch
+  // is the thread's, reused across calls (fresh large vectors cost page faults every call).
+  static thread_local std::vector<u32> cnt, pos, order;
+  {
     cnt.assign(K + 1, 0);
     for (const Fin& f : fin) cnt[f.kid + 1]++;
     for (u32 k = 0; k < K; k++) cnt[k + 1] += cnt[k];
-    if (by.size() < fin.size()) by.resize(fin.size());
     pos.assign(cnt.begin(), cnt.end() - 1);
-    for (const Fin& f : fin) by[pos[f.kid]++] = f;
-    for (u32 k = 0; k < K; k++)
-      if (cnt[k + 1] - cnt[k] > 1)
-        std::sort(by.begin() + cnt[k], by.begin() + cnt[k + 1],
-                  [](const Fin& a, const Fin& b) { return a.lo < b.lo; });
-    std::copy(by.begin(), by.begin() + fin.size(), fin.begin());
+    order.resize(fin.size());
+    for (u32 i = 0; i < (u32)fin.size(); i++) order[pos[fin[i].kid]++] = i;
+    for (u32 k = 0; k < K; k++) {
+      u32* a = order.data() + cnt[k];
+      const u32 m = cnt[k + 1] - cnt[k];
+      for (u32 i = 1; i < m; i++) {   // insertion sort: a kernel has a handful of strata
+        const u32 v = a[i];
+        const u64 lo = fin[v].lo;
+        u32 j = i;
+        while (j > 0 && fin[a[j - 1]].lo > lo) { a[j] = a[j - 1]; j--; }
+        a[j] = v;
+      }
+    }
   }
-  hc.mark("tsort");
   const u32 ns = (u32)fin.size();
+  auto F = [&](u32 s) -> const Fin& { return fin[order[s]]; };
   std::vector<KTab> ktab(K, KTab{0, 0, 0, 0});
   std::vector<u64> lows;
   std::vector<u32> tiers(ns);
   for (u32 s = 0; s < ns; s++) {
-    const Fin& f = fin[s];
+    const Fin& f = F(s);
     tiers[s] = f.tier;
     KTab& e = ktab[f.kid];
     if (e.m == 0) { e.base = s; e.lows_off = (u32)lows.size(); }
@@ -1284,7 +1304,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   // the strata weights W_s = S1_s (u128) on the device for the prediction computed with the
   // representatives (below), uploaded with the assignment tables
   std::vector<u64> hW(2 * (size_t)ns);
-  for (u32 s = 0; s < ns; s++) { hW[2 * s] = (u64)fin[s].s1; hW[2 * s + 1] = (u64)(fin[s].s1 >> 64); }
+  for (u32 s = 0; s < ns; s++) { hW[2 * s] = (u64)F(s).s1; hW[2 * s + 1] = (u64)(F(s).s1 >> 64); }
   DBuf<u64> dW(c);
   DBuf<double> dpred(c);
   SV_TRY(dW.alloc(std::max<size_t>(hW.size(), 2)));
@@ -1428,14 +1448,16 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   R->kde_evaluated = h_terms[1];
   if (c->timing) c->acc[SIEVE_PHASE_KDE].work += h_terms[0];
   hc.mark("reps");
+  struct AssembleMark { HostClock& h; ~AssembleMark() { h.mark("assemble"); } } assemble_mark{hc};
 
   // ---------------- assemble --------------------------------------------------------------------
-  R->st.resize(ns);
-  std::vector<u32> first_of(K, 0xFFFFFFFFu);
+  R->st.swap(spare_strata());   // capacity from a freed result of this thread (no page faults)
+  R->st.resize(ns);               // value-initialised: every field below is set, the pad is zero
+  static thread_local std::vector<u32> first_of;
+  first_of.assign(K, 0xFFFFFFFFu);
   for (u32 s = 0; s < ns; s++) {
-    const Fin& f = fin[s];
+    const Fin& f = F(s);
     sieve_stratum& o = R->st[s];
-    memset(&o, 0, sizeof o);
     if (first_of[f.kid] == 0xFFFFFFFFu) first_of[f.kid] = s;
     o.kernel_id = f.kid;
     o.tier = f.tier;
@@ -1671,6 +1693,8 @@ extern "C" int sieve_strata_stats(sieve_strata s, uint32_t* rounds, uint64_t* te
 extern "C" void sieve_strata_free(sieve_strata s) {
   if (!strata_ok(s)) return;
   s->magic = 0;
+  std::vector<sieve_stratum>& sp = spare_strata();   // keep the larger buffer for the next result
+  if (s->st.capacity() > sp.capacity()) { s->st.clear(); sp.swap(s->st); }
   delete s;
 }
 extern "C" int sieve_segment_count(sieve_strata s, uint64_t* n) {

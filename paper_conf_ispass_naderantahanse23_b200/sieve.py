@@ -429,17 +429,26 @@ class Strata:
         self._h = h
         n = ctypes.c_uint64()
         _check(_L.sieve_strata_count(h, ctypes.byref(n)), "sieve_strata_count")
-        self.table = np.zeros(n.value, STRATUM_DTYPE)
-        if n.value:
-            _check(_L.sieve_strata_copy(h, self.table.ctypes.data_as(ctypes.c_void_p), n.value),
-                   "sieve_strata_copy")
+        self._n = n.value
+        self._table = None   # copied out on first use (sieve_strata_copy)
         r, t, ev = ctypes.c_uint32(), ctypes.c_uint64(), ctypes.c_uint64()
         _check(_L.sieve_strata_stats(h, ctypes.byref(r), ctypes.byref(t), ctypes.byref(ev)),
                "sieve_strata_stats")
         self.rounds, self.kde_terms, self.kde_evaluated = r.value, t.value, ev.value
 
+    @property
+    def table(self):
+        """the stratum table (numpy structured array, STRATUM_DTYPE), copied on first access"""
+        if self._table is None:
+            tab = np.zeros(self._n, STRATUM_DTYPE)
+            if self._n:
+                _check(_L.sieve_strata_copy(self._h, tab.ctypes.data_as(ctypes.c_void_p), self._n),
+                       "sieve_strata_copy")
+            self._table = tab
+        return self._table
+
     def __len__(self):
-        return len(self.table)
+        return self._n
 
     def segments(self, G):
         n = ctypes.c_uint64()
