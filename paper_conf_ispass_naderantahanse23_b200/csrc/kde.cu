@@ -226,7 +226,7 @@ __constant__ double KDE_EXP2_NEG[256] = {
 // coefficients without a short (upper-word) immediate form: the constant bank
 __constant__ double c_kde[3] = {C_LOG2E_128, C_LN2_128, C_P3};
 
-struct KdeRegs { double log2e, magic; };  // operands that must sit in registers (see below)
+struct KdeRegs { double log2e, magic; u32 lane8; };  // operands that must sit in registers (see below)
 
 // acc + Q: the term's final fma adds rint(P * S) straight into an integer-valued accumulator in
 // [2^52, 2^53) (ulp 1).  rn(acc + P*S) = acc + rint(P*S) exactly because P*S is never an exact
@@ -258,16 +258,19 @@ __device__ __forceinline__ double kde_acc(double gs, double xs, const double* sS
   // S = T'[k] = (2^{-(k mod 256)/256} 2^40) * 2^-(k div 256): the 256-entry table is replicated
   // once per lane (entry e of replica l at byte 256 e + 8 l, so the lanes of every 128-byte
   // wavefront hit distinct bank pairs: conflict-free for any pattern of k), and the power of
-  // two is applied exactly by subtracting (k div 256) from the exponent field.  The byte
-  // permutes give (k mod 256) << 8 and (k div 256) << 16 in one instruction each.  For
-  // 10526 < k <= KDE_KCLAMP, P * S <= 1.0014 * 2^(40 - 10527/256) < 0.47, so
+  // two is applied exactly in the exponent field.  Two integer instructions besides the load:
+  //   * one byte permute gives the replica address (k mod 256) << 8 | 8 l (the table sits at
+  //     the start of shared memory, so the load takes no base register);
+  //   * the replica stores entry e with e << 12 added to its upper word, so one multiply-add
+  //     hi - k * 2^12 = hi(2^{-e/256} 2^40) - (k div 256) * 2^20 (k = 256 (k div 256) + e; the
+  //     upper word never wraps: k < 2^16) applies the power of two.
+  // For 10526 < k <= KDE_KCLAMP, P * S <= 1.0014 * 2^(40 - 10527/256) < 0.47, so
   // fma(P, S, acc) = acc exactly: the term is 0 as A10 defines, with no select.
   u32 k = (u32)__double2loint(kb);
   if (MODE >= 1) k = min(k, (u32)KDE_KCLAMP);
   if (MODE == 2) k = (u32)__double2hiint(u) >= 0x40540000u ? (u32)KDE_KCLAMP : k;
-  double T = *(const double*)((const char*)sS + __byte_perm(k, 0u, 0x4404u));
-  double S = __hiloint2double(__double2hiint(T) - (int)(__byte_perm(k, 0u, 0x4144u) << 4),
-                              __double2loint(T));
+  double T = *(const double*)((const char*)sS + __byte_perm(k, R.lane8, 0x5504u));
+  double S = __hiloint2double(__double2hiint(T) - (int)(k << 12), __double2loint(T));
 #else
   // fma(p, 0, acc) = acc for the zero entry T'[KDE_KCUT]
   u32 k = min((u32)__double2loint(kb), (u32)KDE_KCUT);
@@ -332,10 +335,11 @@ k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
   extern __shared__ __align__(16) unsigned char smem[];
   double* sS = (double*)smem;
 #if KDE_SPLIT
-  // replica l of entry e at double index 32 e + l: 2^{-e/256} * 2^40 (exact scaling)
+  // replica l of entry e at double index 32 e + l: 2^{-e/256} * 2^40 (exact scaling), its upper
+  // word biased by e << 12 for kde_acc's exponent step
   for (u32 q = threadIdx.x; q < 256 * 32; q += blockDim.x) {
     double T = KDE_EXP2_NEG[q >> 5];
-    sS[q] = __hiloint2double(__double2hiint(T) + 40 * (1 << 20), __double2loint(T));
+    sS[q] = __hiloint2double(__double2hiint(T) + 40 * (1 << 20) + (int)((q >> 5) << 12), __double2loint(T));
   }
 #else
   // T'[k] = ldexp(2^{-(k mod 256)/256}, 40 - k div 256), T'[KCUT] = 0
@@ -355,12 +359,9 @@ k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
   unsigned char* wsm = smem + KDE_SMEM_TABLE + (threadIdx.x >> 5) * KDE_WARP_BYTES;
   double* const buf0 = (double*)wsm;   // value buffers buf0 + b * KDE_CH, b = 0, 1
   KdeItem* sd = (KdeItem*)(wsm + 2 * KDE_CH * 8);
-#if KDE_SPLIT
-  const double* sSb = sS + lane;   // this lane's table replica
-#else
-  const double* sSb = sS;
-#endif
+  const double* sSb = sS;   // KDE_SPLIT: the lane's replica is selected by R.lane8
   KdeRegs R;
+  R.lane8 = 8 * lane;
   // the fma that forms kb has two constant operands and a DFMA takes at most one constant:
   // load both into registers once (opaque to the compiler, so it cannot re-materialise them)
   asm volatile("mov.b64 %0, %1;" : "=d"(R.log2e) : "d"(c_kde[0]));
