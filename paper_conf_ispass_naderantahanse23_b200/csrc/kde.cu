@@ -44,8 +44,9 @@
 #define KDE_MINB 1           // resident blocks per SM: one 64 KB table shared by the block
 #endif
 #ifndef KDE_UNROLL
-#define KDE_UNROLL 16        // terms in flight per lane
-#endif
+#define KDE_UNROLL 14        // terms in flight per lane (A/B on C4 after the two-instruction table
+#endif                       // step: 14 -> 6.36 ms, 16 -> 6.61, 12 -> 6.45, 8 -> 6.46, 15 -> 6.85)
+static_assert(KDE_CH % 32 == 0, "each lane stages KDE_CH / 32 values of an item");
 #define KDE_V (32 / KDE_TJ)  // value slices per warp
 
 __device__ __forceinline__ double grid_pt(u64 lo, u64 hi, u32 j, u32 G) {

@@ -86,7 +86,9 @@ inline double cell_margin(u64 lo, u64 hi, u32 G) {
 #define KDE_TJ 32       // grid points per tile (32: one point per lane; 16: two value slices)
 #endif
 #ifndef KDE_CH
+#ifndef KDE_CH
 #define KDE_CH 512      // values per work item (A/B: 512 beats 256 by 2.5%; 16-point tiles lose)
+#endif
 #endif
 // per (segment, tile of KDE_TJ grid points): the range of bucketed values whose cells meet the
 // tile's window, chunked into work items; tile_items[nseg * tiles] receives the item total
