@@ -1342,7 +1342,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     {
       PhaseTimer tb(c, SIEVE_PHASE_ASSIGN, n * (12 + (t->cta ? 4 : 0) + (sid_out ? 4 : 0)));
       launch_assign(t->kid, t->x, t->cta, n, t->first_id, d_ktab.get(), d_lows.get(), K,
-                    (u32)lows.size(), sid_out, gh, errf.get(), assign_grid(), S);
+                    (u32)lows.size(), ns, sid_out, gh, errf.get(), assign_grid(), S);
     }
     SV_CUDA(cudaGetLastError());
     launch_hash_compact(gh, ent.get(), ent.get() + cap, ent.get() + 2 * cap, counter.get(), S);

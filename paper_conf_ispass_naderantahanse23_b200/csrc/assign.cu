@@ -7,14 +7,18 @@
 //
 // B200 design: one coalesced pass (kernel id, x, CTA in; stratum id out).  Stratum lookup is a
 // per-kernel table plus a branch-free binary search over the kernel's stratum lower bounds.
-// (stratum, CTA) statistics use a block-private open-addressing hash table in shared memory
-// (native 32-bit atomics for counts and first offsets; 64-bit CAS only on first insertion),
-// flushed into an L2-resident global table when half full and at the end of the block's range.
+// (stratum, CTA) statistics are block-private in shared memory: two fixed slots per stratum
+// (k_assign_slots; a third CTA size of a stratum goes to the global table directly) or, when
+// the slots do not fit, an open-addressing hash table (k_assign; 64-bit CAS only on first
+// insertion) flushed when three-quarters full; native 32-bit atomics for counts and first
+// offsets.  Both end in an L2-resident global table at the end of the block's range.
 // The global table's contents (not its slot order) are deterministic; entries are compacted,
 // gathered across ranks, radix-sorted by key and reduced, so the result is identical for any
 // number of ranks or blocks.
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
+#include <cstring>
 
 #include "kernels.cuh"
 
@@ -26,7 +30,6 @@
 #define AS_IPT (AS_PIPE ? 4 : 8)
 #endif
 #define AS_HC 8192          // shared hash capacity (entries): 128 KB, one block per SM
-#define AS_FLUSH (3 * AS_HC / 4)      // flush to the L2 table when this full
 #define AS_MAXP 32          // probes before falling back to the global table
 #ifndef AS_CHECK
 #define AS_CHECK 32         // at most this many tiles between the fill checks (A/B, C4 / C5:
@@ -63,66 +66,91 @@ __device__ void ghash_update(GHash gh, u64 key, u64 cnt, u64 first, u64* errflag
 // SMEM_TAB: the per-kernel table and the strata lower bounds are staged in shared memory next
 // to the hash (every row looks them up; from global memory the dependent loads of the binary
 // search and the LSU queue were the kernel's main stalls)
+//
+// W > 0: a slot front.  Every stratum owns W fixed slots {CTA size, count, first offset} in
+// shared memory; a row reads its stratum's W CTA sizes with one vector load and adds to the
+// matching slot, a CTA size seen for the first time claims a free slot with a 32-bit CAS, and
+// only rows whose CTA size finds no slot go to the (then small) hash table.  The slots need no
+// probing (the hash alone makes a warp wait for the longest probe sequence among its lanes) and
+// no flushing; a block's slots go to the L2 table once, at the end.  Every path adds the same
+// (key, count, first) contributions, so the L2 table's contents are identical.
 #define AS_TAB_BUDGET (96 * 1024)
-template <bool SMEM_TAB>
+#define AS_EMPTY32 0xFFFFFFFFu
+#define AS_SMEM_MAX (227 * 1024 - 1024)
+#ifndef AS_SLOT_IPT
+#define AS_SLOT_IPT 2       // rows per thread per tile with the slot front (A/B on C4: 1 0.56, 2 0.495,
+#endif                      // 3 0.50, 4 0.51, 6 0.72, 8 0.92 ms: rows in flight compete for L1 room)
+template <bool SMEM_TAB, int W>
 __global__ void __launch_bounds__(AS_THREADS)
 k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __restrict__ cta,
          u64 n, u64 first_id, const KTab* __restrict__ g_ktab, const u64* __restrict__ g_lows,
-         u32 K, u32 nlows, u32* __restrict__ sid_out, GHash gh, u64* errflags) {
+         u32 K, u32 nlows, u32 ns, u32 hcap, u32* __restrict__ sid_out, GHash gh, u64* errflags) {
+  constexpr int IPT = W > 0 ? AS_SLOT_IPT : AS_IPT;
   pdl_begin();
   extern __shared__ __align__(16) unsigned char smem[];
-  u64* hk = (u64*)smem;              // [AS_HC]
-  u32* hc = (u32*)(hk + AS_HC);      // [AS_HC]
-  u32* hf = hc + AS_HC;              // [AS_HC]
-  KTab* s_ktab = (KTab*)(hf + AS_HC);          // [K]       (SMEM_TAB)
-  u64* s_lows = (u64*)(s_ktab + K);             // [nlows]   (SMEM_TAB)
+  const u32 nslot = W > 0 ? ns * W : 0u;
+  // slots: CTA sizes stratum-major (one vector load reads a stratum's W sizes); counts and first
+  // offsets slot-major, so the atomics of distinct strata fall into distinct banks
+  u32* sc = (u32*)smem;                       // [ns][W] CTA sizes (AS_EMPTY32: free)
+  u32* sn = sc + nslot;                       // [W][ns] counts
+  u32* sf = sn + nslot;                       // [W][ns] first offsets in the block's range
+  u64* hk = (u64*)(smem + ((3ull * nslot * 4 + 15) & ~15ull));   // [hcap]
+  u32* hc = (u32*)(hk + hcap);                // [hcap]
+  u32* hf = hc + hcap;                        // [hcap]
+  KTab* s_ktab = (KTab*)(hf + hcap);          // [K]       (SMEM_TAB)
+  u64* s_lows = (u64*)(s_ktab + K);           // [nlows]   (SMEM_TAB)
   const KTab* ktab = SMEM_TAB ? s_ktab : g_ktab;
   const u64* lows = SMEM_TAB ? s_lows : g_lows;
+  const u32 hmask = hcap - 1, hflush = 3 * hcap / 4;   // flush to the L2 table when this full
   __shared__ u32 s_fill;
   if (SMEM_TAB) {
     for (u32 i = threadIdx.x; i < K; i += AS_THREADS) s_ktab[i] = g_ktab[i];
     for (u32 i = threadIdx.x; i < nlows; i += AS_THREADS) s_lows[i] = g_lows[i];
   }
-  for (u32 i = threadIdx.x; i < AS_HC; i += AS_THREADS) { hk[i] = HASH_EMPTY; hc[i] = 0; hf[i] = 0xFFFFFFFFu; }
+  if constexpr (W > 0)
+    for (u32 i = threadIdx.x; i < nslot; i += AS_THREADS) { sc[i] = AS_EMPTY32; sn[i] = 0; sf[i] = AS_EMPTY32; }
+  for (u32 i = threadIdx.x; i < hcap; i += AS_THREADS) { hk[i] = HASH_EMPTY; hc[i] = 0; hf[i] = 0xFFFFFFFFu; }
   if (threadIdx.x == 0) s_fill = 0;
   __syncthreads();
-  u64 chunk = (n + gridDim.x - 1) / gridDim.x;
-  u64 b0 = (u64)blockIdx.x * chunk;
-  u64 b1 = b0 + chunk < n ? b0 + chunk : n;
-  const u64 tile = (u64)AS_THREADS * AS_IPT;
-  u32 kk[AS_IPT], cc[AS_IPT];
-  u64 vv[AS_IPT];
+  // n < 2^32 (sieve_load_trace): every index of the pass is a 32-bit offset
+  const u32 n32 = (u32)n;
+  const u32 chunk = (u32)((n + gridDim.x - 1) / gridDim.x);
+  const u32 b0 = blockIdx.x * chunk;
+  const u32 b1 = (u64)b0 + chunk < n32 ? b0 + chunk : n32;
+  const u32 tile = AS_THREADS * IPT;
+  u32 kk[IPT], cc[IPT];
+  u64 vv[IPT];
   u32 tiles_done = 0, next_check = 1, last_fill = 0, last_check = 0;
-  auto load_tile = [&](u64 base, u32* k_, u64* v_, u32* c_) {
+  auto load_tile = [&](u32 base, u32* k_, u64* v_, u32* c_) {
 #pragma unroll
-    for (int j = 0; j < AS_IPT; j++) {
-      u64 i = base + (u64)j * AS_THREADS + threadIdx.x;
-      bool ok = i < b1;
+    for (int j = 0; j < IPT; j++) {
+      const u32 i = base + j * AS_THREADS + threadIdx.x;
+      const bool ok = i < b1;
       k_[j] = ok ? __ldcs(kid + i) : 0u;
       v_[j] = ok ? __ldcs(x + i) : 0ull;
       c_[j] = (ok && cta) ? __ldcs(cta + i) : 0u;
     }
   };
 #if AS_PIPE
-  load_tile(b0, kk, vv, cc);
+  if (b0 < b1) load_tile(b0, kk, vv, cc);
 #endif
-  for (u64 base = b0; base < b1; base += tile) {
+  for (u32 base = b0; base < b1; base += tile) {
 #if AS_PIPE
-    u32 nk[AS_IPT], nc[AS_IPT];
-    u64 nv[AS_IPT];
+    u32 nk[IPT], nc[IPT];
+    u64 nv[IPT];
     load_tile(base + tile, nk, nv, nc);   // in flight while this tile is processed
 #else
     load_tile(base, kk, vv, cc);          // the tile's loads first, then the atomics
 #endif
-    KTab kts[AS_IPT];  // per-kernel table rows (L1-resident), all requested before use
+    KTab kts[IPT];  // per-kernel table rows, all requested before use
 #pragma unroll
-    for (int j = 0; j < AS_IPT; j++) kts[j] = ktab[kk[j]];
+    for (int j = 0; j < IPT; j++) kts[j] = ktab[kk[j]];
 #pragma unroll
-    for (int j = 0; j < AS_IPT; j++) {
-      u64 i = base + (u64)j * AS_THREADS + threadIdx.x;
+    for (int j = 0; j < IPT; j++) {
+      const u32 i = base + j * AS_THREADS + threadIdx.x;
       if (i >= b1) continue;
-      u64 v = vv[j];
-      KTab kt = kts[j];
+      const u64 v = vv[j];
+      const KTab kt = kts[j];
       u32 sid = kt.base;
       if (kt.m > 1) {  // number of lower bounds lows[1..m) that are <= v
         const u64* L = lows + kt.lows_off;
@@ -134,10 +162,34 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
         sid += lo;
       }
       if (sid_out) sid_out[i] = sid;
-      u32 c = cc[j];
-      u64 key = ((u64)sid << 32) | c;
-      u32 rel = (u32)(i - b0);
-      u32 h = hash_key(key) & (AS_HC - 1);
+      const u32 c = cc[j];
+      const u32 rel = i - b0;
+      if constexpr (W > 0) {
+        const u32 b = sid * W;
+        int slot;
+        if constexpr (W == 4) {
+          const uint4 k4 = *(const uint4*)(sc + b);
+          slot = k4.x == c ? 0 : k4.y == c ? 1 : k4.z == c ? 2 : k4.w == c ? 3 : -1;
+        } else {
+          const uint2 k2 = *(const uint2*)(sc + b);
+          slot = k2.x == c ? 0 : k2.y == c ? 1 : -1;
+        }
+        if (slot < 0 && c != AS_EMPTY32) {  // first sight of this CTA size (in the read above)
+#pragma unroll
+          for (int q = 0; q < W; q++) {
+            const u32 cur = atomicCAS(sc + b + q, AS_EMPTY32, c);
+            if (cur == AS_EMPTY32 || cur == c) { slot = q; break; }
+          }
+        }
+        if (slot >= 0) {
+          const u32 e = slot * ns + sid;
+          atomicAdd(sn + e, 1u);
+          if (*(volatile u32*)(sf + e) > rel) atomicMin(sf + e, rel);  // rarely lowers it
+          continue;
+        }
+      }
+      const u64 key = ((u64)sid << 32) | c;
+      u32 h = hash_key(key) & hmask;
       bool done = false;
       for (int p = 0; p < AS_MAXP; p++) {
         u64 cur = hk[h];
@@ -151,11 +203,11 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
           done = true;
           break;
         }
-        h = (h + 1) & (AS_HC - 1);
+        h = (h + 1) & hmask;
       }
       if (!done) ghash_update(gh, key, 1, first_id + i, errflags);
     }
-    bool last = base + tile >= b1;
+    const bool last = base + tile >= b1;
     ++tiles_done;
     // the fill check needs block barriers, so it runs only as often as the table's growth needs:
     // after half the tiles the last interval's growth rate would take to reach the flush level,
@@ -164,7 +216,7 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
     if (tiles_done < next_check && !last) {
 #if AS_PIPE
 #pragma unroll
-      for (int j = 0; j < AS_IPT; j++) { kk[j] = nk[j]; vv[j] = nv[j]; cc[j] = nc[j]; }
+      for (int j = 0; j < IPT; j++) { kk[j] = nk[j]; vv[j] = nv[j]; cc[j] = nc[j]; }
 #endif
       continue;
     }
@@ -173,14 +225,14 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
     __syncthreads();
     {
       const u32 grow = (fill > last_fill ? fill - last_fill : 0u) / max(1u, tiles_done - last_check);
-      const u32 room = fill < AS_FLUSH ? AS_FLUSH - fill : 0u;
+      const u32 room = fill < hflush ? hflush - fill : 0u;
       const u32 k = grow ? room / (2u * grow) : (u32)AS_CHECK;
       next_check = tiles_done + max(1u, min(k, (u32)AS_CHECK));
       last_fill = fill;
       last_check = tiles_done;
     }
-    if (fill > AS_FLUSH || last) {  // rows that find no slot go to the L2 table directly
-      for (u32 e = threadIdx.x; e < AS_HC; e += AS_THREADS) {
+    if (fill > hflush || last) {  // rows that find no slot go to the L2 table directly
+      for (u32 e = threadIdx.x; e < hcap; e += AS_THREADS) {
         u64 key = hk[e];
         if (key != HASH_EMPTY) {
           ghash_update(gh, key, hc[e], first_id + b0 + hf[e], errflags);
@@ -194,28 +246,73 @@ k_assign(const u32* __restrict__ kid, const u64* __restrict__ x, const u32* __re
     }
 #if AS_PIPE
 #pragma unroll
-    for (int j = 0; j < AS_IPT; j++) { kk[j] = nk[j]; vv[j] = nv[j]; cc[j] = nc[j]; }
+    for (int j = 0; j < IPT; j++) { kk[j] = nk[j]; vv[j] = nv[j]; cc[j] = nc[j]; }
 #endif
+  }
+  if constexpr (W > 0) {  // the slots, once (every thread passed the last tile's barriers above)
+    for (u32 e = threadIdx.x; e < nslot; e += AS_THREADS) {
+      const u32 c = sc[e], sid = e / W, f = (e % W) * ns + sid;
+      if (c != AS_EMPTY32 && sn[f]) ghash_update(gh, ((u64)sid << 32) | c, sn[f], first_id + b0 + sf[f], errflags);
+    }
   }
 }
 
+static size_t assign_smem(u32 W, u32 ns, u32 hcap, bool smem_tab, u32 K, u32 nlows) {
+  return ((3ull * ns * W * 4 + 15) & ~15ull) + (size_t)hcap * 16 +
+         (smem_tab ? (size_t)K * sizeof(KTab) + (size_t)nlows * 8 : 0);
+}
+
+template <bool SMEM_TAB, int W>
+static void launch_assign_v(const u32* kid, const u64* x, const u32* cta, u64 n, u64 first_id,
+                            const KTab* ktab, const u64* lows, u32 K, u32 nlows, u32 ns, u32 hcap,
+                            u32* sid_out, GHash gh, u64* errflags, int grid, cudaStream_t s) {
+  const size_t sm = assign_smem(W, ns, hcap, SMEM_TAB, K, nlows);
+  sv_smem_attr(k_assign<SMEM_TAB, W>, (int)sm);
+  SV_LAUNCH((k_assign<SMEM_TAB, W>), grid, AS_THREADS, sm, s)(kid, x, cta, n, first_id, ktab, lows, K, nlows,
+                                                              ns, hcap, sid_out, gh, errflags);
+}
+
+// Variant choice: the slot front with a small hash behind it (2 slots per stratum, a 2,048-entry
+// hash) when it fits in AS_SLOT_BUDGET of shared memory, else the 8,192-entry hash alone (A/B
+// on C4: slots + 512 / 1,024 / 2,048 / 4,096 hash entries 0.49 ms each; four slots per stratum
+// 0.67 ms -- the 16-byte key reads and the stride-4 atomics conflict; the hash alone 0.57 ms, on
+// C5 9.35 ms).  Without the hash behind them, slots that overflow send rows to contended L2
+// atomics (C5, five CTA sizes per stratum: 87 ms).  Test hook SIEVE_ASSIGN: "hash" forces the
+// hash alone, "4" four slots per stratum.
+#ifndef AS_SLOT_BUDGET
+#define AS_SLOT_BUDGET (176 * 1024)
+#endif
+#ifndef AS_SLOT_HASH
+#define AS_SLOT_HASH 2048
+#endif
 void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 first_id,
-                   const KTab* ktab, const u64* lows, u32 K, u32 nlows, u32* sid_out, GHash gh,
+                   const KTab* ktab, const u64* lows, u32 K, u32 nlows, u32 ns, u32* sid_out, GHash gh,
                    u64* errflags, int grid, cudaStream_t s) {
   if (n == 0) return;
-  size_t smem = (size_t)AS_HC * (8 + 4 + 4);
-  size_t tab = (size_t)K * sizeof(KTab) + (size_t)nlows * 8;
-  u64 maxgrid = (n + (u64)AS_THREADS * AS_IPT - 1) / ((u64)AS_THREADS * AS_IPT);
+  u64 maxgrid = (n + (u64)AS_THREADS * AS_SLOT_IPT - 1) / ((u64)AS_THREADS * AS_SLOT_IPT);
   if ((u64)grid > maxgrid) grid = (int)maxgrid;
-  if (tab <= AS_TAB_BUDGET) {
-    sv_smem_attr(k_assign<true>, (int)(smem + tab));
-    SV_LAUNCH(k_assign<true>, grid, AS_THREADS, smem + tab, s)(kid, x, cta, n, first_id, ktab, lows, K,
-                                                                nlows, sid_out, gh, errflags);
-  } else {
-    sv_smem_attr(k_assign<false>, (int)smem);
-    SV_LAUNCH(k_assign<false>, grid, AS_THREADS, smem, s)(kid, x, cta, n, first_id, ktab, lows, K,
-                                                           nlows, sid_out, gh, errflags);
+  const char* force = getenv("SIEVE_ASSIGN");
+  const bool hash_only = force && !strcmp(force, "hash");
+  const bool w4 = force && !strcmp(force, "4");
+  const size_t tab = (size_t)K * sizeof(KTab) + (size_t)nlows * 8;
+  if (!hash_only && tab <= AS_TAB_BUDGET) {
+    if (w4 && assign_smem(4, ns, AS_SLOT_HASH, true, K, nlows) <= AS_SMEM_MAX) {
+      launch_assign_v<true, 4>(kid, x, cta, n, first_id, ktab, lows, K, nlows, ns, AS_SLOT_HASH, sid_out, gh,
+                               errflags, grid, s);
+      return;
+    }
+    if (!w4 && assign_smem(2, ns, AS_SLOT_HASH, true, K, nlows) <= AS_SLOT_BUDGET) {
+      launch_assign_v<true, 2>(kid, x, cta, n, first_id, ktab, lows, K, nlows, ns, AS_SLOT_HASH, sid_out, gh,
+                               errflags, grid, s);
+      return;
+    }
   }
+  if (tab <= AS_TAB_BUDGET)
+    launch_assign_v<true, 0>(kid, x, cta, n, first_id, ktab, lows, K, nlows, ns, AS_HC, sid_out, gh, errflags,
+                             grid, s);
+  else
+    launch_assign_v<false, 0>(kid, x, cta, n, first_id, ktab, lows, K, nlows, ns, AS_HC, sid_out, gh, errflags,
+                              grid, s);
 }
 
 __global__ void k_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst,

@@ -208,7 +208,7 @@ struct GHash {     // global (sid, cta) table
 #define HASH_EMPTY 0xFFFFFFFFFFFFFFFFull
 int assign_grid();
 void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 first_id,
-                   const KTab* ktab, const u64* lows, u32 K, u32 nlows, u32* sid_out, GHash gh,
+                   const KTab* ktab, const u64* lows, u32 K, u32 nlows, u32 ns, u32* sid_out, GHash gh,
                    u64* errflags, int grid, cudaStream_t s);
 // compact occupied entries into (key, cnt, first) arrays; *count (device) += entries
 void launch_hash_compact(GHash gh, u64* okey, u64* ocnt, u64* ofirst, unsigned long long* count,

@@ -307,3 +307,20 @@ def test_16bit_columns(device):
         sieve.load_trace(ctx, kid16 if device else torch.from_numpy(tr["kid"].astype(np.int16)).cuda(),
                          x if device else torch.from_numpy(tr["x"].view(np.int64)).cuda(),
                          num_kernels=tr["K"], adopt=True)
+
+
+@pytest.mark.parametrize("variant", ["slots2", "4", "hash"])
+def test_assign_variants(variant, monkeypatch):
+    """pass B's (stratum, CTA) statistics: W fixed slots per stratum (default 2, or 4) and the
+    hash-table variant give the oracle's representatives; kernel 0 has seven CTA sizes, so its
+    stratum overflows the slots into the L2 table"""
+    if variant != "slots2":
+        monkeypatch.setenv("SIEVE_ASSIGN", variant)
+    tr = gen.make_trace("C2", n=150_000)
+    rng = np.random.default_rng(7)
+    k0 = np.nonzero(tr["kid"] == 0)[0]
+    tr["cta"][k0] = rng.choice(np.array([32, 64, 96, 128, 256, 512, 1024], np.uint32), size=len(k0))
+    g = run_gpu(tr)
+    o = run_oracle(tr)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
