@@ -133,9 +133,10 @@ struct sieve_ctx_s {
   // SIEVE_HOST_TIMING: host-side accounting of the synchronisations of a call
   int hs_n = 0;
   bool count_terms = true;  // in-window KDE term count (sieve_ctx_set_term_count)
-  // mapped (zero-copy) pinned host memory: kernels write each round's part results here
-  u64* mapped = nullptr;
-  size_t mapped_cap = 0;
+  // mapped (zero-copy) pinned host memory: kernels write each round's part results here, in two
+  // buffers used alternately, so one batch's records stay readable while the next batch runs
+  u64* mapped[2] = {nullptr, nullptr};
+  size_t mapped_cap[2] = {0, 0};
   u64* scan_state = nullptr;   // single-pass scans (sort.cu), zero-initialised at creation
   double hs_wait = 0, hs_between = 0;
   std::string hs_list;
@@ -287,21 +288,21 @@ static int pin_alloc(sieve_ctx c, void** p, size_t bytes) {
 
 // a mapped pinned host buffer of at least `bytes` (grown, never shrunk; its contents are only
 // valid between a kernel that writes it and the host's read after the next stream sync)
-static int mapped_get(sieve_ctx c, size_t bytes, u64** host, u64** dev) {
-  if (bytes > c->mapped_cap) {
+static int mapped_get(sieve_ctx c, int slot, size_t bytes, u64** host, u64** dev) {
+  if (bytes > c->mapped_cap[slot]) {
     SV_CUDA(cudaStreamSynchronize(c->stream));  // the old buffer may still be written
-    if (c->mapped) cudaFreeHost(c->mapped);
-    c->mapped = nullptr;
-    c->mapped_cap = 0;
+    if (c->mapped[slot]) cudaFreeHost(c->mapped[slot]);
+    c->mapped[slot] = nullptr;
+    c->mapped_cap[slot] = 0;
     size_t want = bytes + bytes / 2 + 4096;
     void* p;
     SV_CUDA(cudaHostAlloc(&p, want, cudaHostAllocMapped | cudaHostAllocPortable));
-    c->mapped = (u64*)p;
-    c->mapped_cap = want;
+    c->mapped[slot] = (u64*)p;
+    c->mapped_cap[slot] = want;
   }
   void* d;
-  SV_CUDA(cudaHostGetDevicePointer(&d, c->mapped, 0));
-  *host = c->mapped;
+  SV_CUDA(cudaHostGetDevicePointer(&d, c->mapped[slot], 0));
+  *host = c->mapped[slot];
   *dev = (u64*)d;
   return SIEVE_OK;
 }
@@ -462,7 +463,8 @@ extern "C" void sieve_ctx_destroy(sieve_ctx ctx) {
   cudaStreamSynchronize(ctx->stream);
   for (void* p : ctx->pin_overflow) cudaFreeHost(p);
   if (ctx->pin) cudaFreeHost(ctx->pin);
-  if (ctx->mapped) cudaFreeHost(ctx->mapped);
+  for (u64* m : ctx->mapped)
+    if (m) cudaFreeHost(m);
   if (ctx->scan_state) cudaFree(ctx->scan_state);
   if (ctx->ev_moments) cudaEventDestroy(ctx->ev_moments);
   delete ctx->comm;
@@ -906,6 +908,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     }
   }
   R->total_instr = I;
+  const u32 n12 = (u32)fin.size();   // the Tier-1/2 strata, in kernel order
 
   // ---------------- Tier-3 values: compaction (unless queued behind pass A) --------------------
   const u32 bx = std::max<u32>(1, bitlen(max_x));
@@ -960,6 +963,32 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   if (!grouped && !open.empty() && max_cells < G)
     return sv_fail(SIEVE_ELIMIT, "instruction counts too wide for the cell sort key");
   for (auto& o : open) { o.src = keys.get(); o.src_shift = 0; }
+  // The final parts of a batch become strata on the host after the NEXT batch's kernels are
+  // queued (just before its synchronisation), so that bookkeeping overlaps device work instead of
+  // delaying the next round's first launch; the batch's records stay valid in their mapped
+  // buffer (the next batch writes the other one).
+  struct DeferredFin { const u64* rec; u32 round; std::vector<u32> part_off, kid; std::vector<double> h; };
+  std::vector<DeferredFin> dfin;
+  // The Tier-3 strata are also kept sorted by (kernel, lo) as they arrive -- key kid << 44 | lo
+  // (x < 2^44, K <= 2^16) with their index in fin -- so the stratum order costs one merge at
+  // the end.
+  std::vector<std::pair<u64, u32>> t3s;
+  auto take_finals = [&]() {
+    const size_t mid = t3s.size();
+    for (const DeferredFin& d : dfin)
+      for (size_t s = 0; s + 1 < d.part_off.size(); s++)
+        for (u32 p = d.part_off[s]; p < d.part_off[s + 1]; p++) {
+          const u64* L = d.rec + 1 + (size_t)p * PART_REC;  // {lanes[9], min, max, ia, ib, final}
+          if (L[0] && L[MOM_LANES + 4]) {  // non-empty, and lo == hi or CoV < theta (k_part_pack)
+            t3s.push_back({((u64)d.kid[s] << 44) | L[MOM_LANES], (u32)fin.size()});
+            fin.push_back({d.kid[s], 3, L[MOM_LANES], L[MOM_LANES + 1], L[0], limbs_u128(L + 1), d.h[s], d.round});
+          }
+        }
+    dfin.clear();
+    std::sort(t3s.begin() + mid, t3s.end());
+    std::inplace_merge(t3s.begin(), t3s.begin() + mid, t3s.end());
+  };
+  u32 nbatch = 0;
   while (!open.empty()) {
     round++;
     if (round > P->max_rounds) return sv_fail(SIEVE_ELIMIT, "Tier-3 refinement exceeded max_rounds");
@@ -1053,6 +1082,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       }
       SV_TRY(rcb.add_h2d(d_sc.get(), seg_chunk));
       SV_TRY(rcb.flush());
+      hc.mark("up");
       PhaseTimer tm(c, SIEVE_PHASE_SORT, nin * 36 + (u64)nch * G * 16);
       launch_grid_tab(segs.get(), nseg, G, gtab.get(), S);
       launch_cell_group(d_chunks.get(), nch, src, segs.get(), nseg, G, d_sc.get(), cells.get(), hist.get(),
@@ -1184,10 +1214,12 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         SV_TRY(allreduce_group(c, {{pl.get(), (size_t)cap * MOM_LANES, RED_SUM}, {pm.get(), (size_t)cap * 2, RED_MAX}}));
         launch_complement(pm.get(), cap, 1, S);
       }
-      SV_TRY(mapped_get(c, (1 + (size_t)cap * PART_REC + nseg) * 8, &hrec, &drec));
+      SV_TRY(mapped_get(c, (int)(nbatch & 1), (1 + (size_t)cap * PART_REC + nseg) * 8, &hrec, &drec));
       launch_part_pack(d_off.get(), nseg, cap, pl.get(), pm.get(), pab.get(), ntk.get(), P->theta_num,
                        P->theta_den, drec, S);
       hc.mark("p");
+      take_finals();   // the previous batch's, while this one runs
+      hc.mark("fin");
       SV_TRY(sync(c));
       hc.mark("ps");
       const u64 live = hrec[0];  // replicated: every rank computed the same cuts from the same D
@@ -1211,6 +1243,18 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     for (u32 s = 0; s < nseg; s++) { part_off[s] = nparts; nparts += h_ntk[s] + 1; }
     part_off[nseg] = nparts;
     if (hrec[0] != nparts) return sv_fail(SIEVE_ESTATE, "internal: part count mismatch");
+    hc.mark("rec");
+    nbatch++;
+    {
+      DeferredFin d;
+      d.rec = hrec;
+      d.round = round;
+      d.part_off = part_off;
+      d.kid.resize(nseg);
+      for (u32 q = 0; q < nseg; q++) d.kid[q] = op[q].kid;
+      d.h.assign(hh.begin(), hh.end());
+      dfin.push_back(std::move(d));
+    }
     for (u32 s = 0; s < nseg; s++) {
       if (R->keep_debug) {
         SegDebug sd;
@@ -1232,21 +1276,18 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       }
       for (u32 p = part_off[s]; p < part_off[s + 1]; p++) {
         const u64* L = hrec + 1 + (size_t)p * PART_REC;  // {lanes[9], min, max, ia, ib, final}
-        u64 pn = L[0];
-        if (!pn) continue;  // empty part: dropped (A13 f)
-        u128 s1 = limbs_u128(L + 1);
-        u64 lo = L[MOM_LANES], hi = L[MOM_LANES + 1];
-        if (L[MOM_LANES + 4])  // lo == hi or CoV < theta, decided exactly by k_part_pack
-          fin.push_back({op[s].kid, 3, lo, hi, pn, s1, hh[s], round});
-        else  // re-opened: its values are [ia, ib) of this batch's grouped values
-          next.push_back({op[s].kid, op[s].t3rank, lo, hi, pn, s1, limbs_u128(L + 5), L[MOM_LANES + 2],
-                          L[MOM_LANES + 3], ck.get(), vsh});
+        // empty parts are dropped (A13 f); final parts go to the strata later (take_finals);
+        // a re-opened part's values are [ia, ib) of this batch's grouped values
+        if (L[0] && !L[MOM_LANES + 4])
+          next.push_back({op[s].kid, op[s].t3rank, L[MOM_LANES], L[MOM_LANES + 1], L[0], limbs_u128(L + 1),
+                          limbs_u128(L + 5), L[MOM_LANES + 2], L[MOM_LANES + 3], ck.get(), vsh});
       }
     }
     }  // batches
     open.swap(next);
     hc.mark("round");
   }
+  take_finals();   // the last batch's
   R->rounds = round;
   // the KDE term count is read back with the representatives at the end (no extra sync)
   std::vector<unsigned long long> h_terms;
@@ -1254,44 +1295,36 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   hc.mark("rend");
 
   // ---------------- stratum table: order by (kernel, lo) (A23) --------------------------------
-  // Stratum order (kernel, lo) as a permutation of fin: a counting sort by kernel, then the few
-  // entries of each Tier-3 kernel by lo.  Indices move, not the 80-byte entries, and the scratch
-  // is the thread's, reused across calls (fresh large vectors cost page faults every call).
-  static thread_local std::vector<u32> cnt, pos, order;
-  {
-    cnt.assign(K + 1, 0);
-    for (const Fin& f : fin) cnt[f.kid + 1]++;
-    for (u32 k = 0; k < K; k++) cnt[k + 1] += cnt[k];
-    pos.assign(cnt.begin(), cnt.end() - 1);
-    order.resize(fin.size());
-    for (u32 i = 0; i < (u32)fin.size(); i++) order[pos[fin[i].kid]++] = i;
-    for (u32 k = 0; k < K; k++) {
-      u32* a = order.data() + cnt[k];
-      const u32 m = cnt[k + 1] - cnt[k];
-      for (u32 i = 1; i < m; i++) {   // insertion sort: a kernel has a handful of strata
-        const u32 v = a[i];
-        const u64 lo = fin[v].lo;
-        u32 j = i;
-        while (j > 0 && fin[a[j - 1]].lo > lo) { a[j] = a[j - 1]; j--; }
-        a[j] = v;
-      }
-    }
-  }
+  // One pass: the Tier-1/2 strata (one per kernel, in kernel order) merged with the sorted Tier-3
+  // strata (disjoint kernels), building the permutation, the per-kernel lookup table, the lower
+  // bounds, the tiers and the weights together.
   const u32 ns = (u32)fin.size();
+  static thread_local std::vector<u32> order_tl;
+  std::vector<u32>& order = order_tl;
+  order.resize(ns);
   auto F = [&](u32 s) -> const Fin& { return fin[order[s]]; };
   std::vector<KTab> ktab(K, KTab{0, 0, 0, 0});
   std::vector<u64> lows;
   std::vector<u32> tiers(ns);
-  for (u32 s = 0; s < ns; s++) {
-    const Fin& f = F(s);
-    tiers[s] = f.tier;
-    KTab& e = ktab[f.kid];
-    if (e.m == 0) { e.base = s; e.lows_off = (u32)lows.size(); }
-    else lows.push_back(f.lo);
-    e.m++;
+  std::vector<u64> hW(2 * (size_t)ns);
+  {
+    u32 i = 0, s = 0;
+    size_t j = 0;
+    while (i < n12 || j < t3s.size()) {
+      const u32 idx = (j == t3s.size() || (i < n12 && fin[i].kid < (u32)(t3s[j].first >> 44))) ? i++ : t3s[j++].second;
+      const Fin& f = fin[idx];
+      order[s] = idx;
+      tiers[s] = f.tier;
+      KTab& e = ktab[f.kid];
+      if (e.m == 0) { e.base = s; e.lows_off = (u32)lows.size(); }
+      else lows.push_back(f.lo);   // a kernel's strata 1..m-1 lower bounds, contiguous, ascending
+      e.m++;
+      hW[2 * (size_t)s] = (u64)f.s1;
+      hW[2 * (size_t)s + 1] = (u64)(f.s1 >> 64);
+      s++;
+    }
+    if (s != ns) return sv_fail(SIEVE_ESTATE, "internal: stratum order");
   }
-  // lows for a kernel with m strata are its strata 1..m-1 lower bounds, contiguous per kernel
-  // (pushed in order above because fin is sorted by (kid, lo))
   if (lows.empty()) lows.push_back(0);
 
   hc.mark("table");
@@ -1303,8 +1336,6 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   SV_TRY(errf.alloc(4));
   // the strata weights W_s = S1_s (u128) on the device for the prediction computed with the
   // representatives (below), uploaded with the assignment tables
-  std::vector<u64> hW(2 * (size_t)ns);
-  for (u32 s = 0; s < ns; s++) { hW[2 * s] = (u64)F(s).s1; hW[2 * s + 1] = (u64)(F(s).s1 >> 64); }
   DBuf<u64> dW(c);
   DBuf<double> dpred(c);
   SV_TRY(dW.alloc(std::max<size_t>(hW.size(), 2)));
@@ -1325,6 +1356,29 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   // representatives (one synchronisation) and an overflow redoes pass B with a bigger table.
   // Several ranks: the entry counts are exchanged first (AR-4 needs them on the host).
   std::vector<u64> h_rep, h_xy, hflag;
+  // the stratum table's fields that do not depend on the representatives, filled while pass B
+  // and the representatives run (the rest after the synchronisation)
+  bool table_pre = false;
+  auto assemble_pre = [&]() {
+    R->st.swap(spare_strata());   // capacity from a freed result of this thread (no page faults)
+    R->st.resize(ns);               // value-initialised: every field is set, the pad is zero
+    static thread_local std::vector<u32> first_of_tl;
+    std::vector<u32>& first_of = first_of_tl;
+    first_of.assign(K, 0xFFFFFFFFu);
+    for (u32 s = 0; s < ns; s++) {
+      const Fin& f = F(s);
+      sieve_stratum& o = R->st[s];
+      if (first_of[f.kid] == 0xFFFFFFFFu) first_of[f.kid] = s;
+      o.kernel_id = f.kid;
+      o.tier = f.tier;
+      o.index_in_kernel = s - first_of[f.kid];
+      o.lo = f.lo; o.hi = f.hi; o.count = f.n;
+      o.instr_sum_lo = (u64)f.s1; o.instr_sum_hi = (u64)(f.s1 >> 64);
+      o.bandwidth = f.h;
+      o.split_round = f.round;
+    }
+    table_pre = true;
+  };
   for (int attempt = 0;; attempt++) {
     if (attempt > 6) return sv_fail(SIEVE_ENOMEM, "(stratum, CTA) table kept overflowing");
     DBuf<u64> gkeys(c), gcnt(c), gfirst(c), ent(c);
@@ -1434,6 +1488,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       if (h_terms.empty()) SV_TRY(cb.add_d2h(h_terms, terms.get(), 2));
       SV_TRY(cb.flush());
     }
+    if (!table_pre) assemble_pre();
     SV_TRY(sync(c));
     if (!c->comm && hflag[2]) { cap <<= 2; continue; }
     break;
@@ -1450,26 +1505,13 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   hc.mark("reps");
   struct AssembleMark { HostClock& h; ~AssembleMark() { h.mark("assemble"); } } assemble_mark{hc};
 
-  // ---------------- assemble --------------------------------------------------------------------
-  R->st.swap(spare_strata());   // capacity from a freed result of this thread (no page faults)
-  R->st.resize(ns);               // value-initialised: every field below is set, the pad is zero
-  static thread_local std::vector<u32> first_of;
-  first_of.assign(K, 0xFFFFFFFFu);
+  // ---------------- assemble: the representatives' fields ---------------------------------------
   for (u32 s = 0; s < ns; s++) {
-    const Fin& f = F(s);
     sieve_stratum& o = R->st[s];
-    if (first_of[f.kid] == 0xFFFFFFFFu) first_of[f.kid] = s;
-    o.kernel_id = f.kid;
-    o.tier = f.tier;
-    o.index_in_kernel = s - first_of[f.kid];
     o.rep_cta = (u32)h_rep[ns + s];
-    o.lo = f.lo; o.hi = f.hi; o.count = f.n;
-    o.instr_sum_lo = (u64)f.s1; o.instr_sum_hi = (u64)(f.s1 >> 64);
     o.rep_id = h_rep[s];
     o.rep_instr = h_xy[s];
     o.rep_cycles = h_xy[ns + (size_t)s];
-    o.bandwidth = f.h;
-    o.split_round = f.round;
   }
   return SIEVE_OK;
 }

@@ -477,21 +477,37 @@ class Strata:
         self.close()
 
 
+_SID_OK = {}   # (id, data_ptr, numel, dtype, id(trace), n) of the last tensor that passed _check_sid
+
+
 def _check_sid(t, trace):
     """stratum ids are written / read by the kernels as a DEVICE uint32 array of n_local entries"""
     import torch
-    if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype in (torch.int32, torch.uint32)
-            and t.is_contiguous()):
+    if not isinstance(t, torch.Tensor):
+        raise TypeError("stratum_of_invocation must be a contiguous CUDA int32/uint32 tensor")
+    key = (id(t), t.data_ptr(), t.numel(), t.dtype, id(trace), trace.n)
+    if _SID_OK.get("key") == key:   # the same tensor as last call (a bench or training loop)
+        return
+    if not (t.is_cuda and t.dtype in (torch.int32, torch.uint32) and t.is_contiguous()):
         raise TypeError("stratum_of_invocation must be a contiguous CUDA int32/uint32 tensor")
     if t.numel() < trace.n:
         raise ValueError(f"stratum_of_invocation has {t.numel()} entries, the trace {trace.n}")
     if t.device.index != trace.ctx.device:
         raise ValueError(f"stratum_of_invocation must live on cuda:{trace.ctx.device}")
+    _SID_OK["key"] = key
+
+
+_DEFAULT_PARAMS = []   # one default sieve_params, built on first use (the library only reads it)
 
 
 def stratify(trace, params=None, stratum_of_invocation=None, **kw):
     """sieve_stratify; stratum_of_invocation: optional CUDA int32/uint32 tensor [n_local]."""
-    p = params if params is not None else default_params(**kw)
+    if params is None and not kw:
+        if not _DEFAULT_PARAMS:
+            _DEFAULT_PARAMS.append(default_params())
+        p = _DEFAULT_PARAMS[0]
+    else:
+        p = params if params is not None else default_params(**kw)
     sid_ptr = None
     if stratum_of_invocation is not None:
         _check_sid(stratum_of_invocation, trace)

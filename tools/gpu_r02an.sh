@@ -1,0 +1,5 @@
+mkdir -p gpurun_out
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_r02an.log 2>&1
+SIEVE_HOST_TIMING=1 timeout 300 python bench.py --steps 5 --warmup 3 --no-e2e --no-cpu-baseline --no-ncu-traffic > gpurun_out/ht_r02an2.log 2> gpurun_out/ht_r02an2.err
+timeout 300 python bench.py --steps 20 --warmup 5 --no-e2e --no-cpu-baseline --no-ncu-traffic > gpurun_out/bench_r02an.log 2>&1
+timeout 600 python tools/timeline.py --steps 3 > gpurun_out/timeline_r02an.log 2>&1
