@@ -163,7 +163,7 @@ def measured_peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 100 ms while running."""
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms while running (the recipe's rate)."""
     Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
@@ -175,9 +175,12 @@ class ClockSampler:
         self.marks = {}
 
     def start(self):
+        if os.environ.get("BENCH_NO_CLOCKS"):   # diagnosis only: the line then reports no clocks
+            return
         try:
             self.proc = subprocess.Popen(
-                ["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits", "-lms", "100",
+                ["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits", "-lms",
+                 os.environ.get("BENCH_CLOCK_MS", "200"),
                  "-i", str(self.device)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except OSError:
             self.proc = None
@@ -439,14 +442,23 @@ def main():
             up = {"kid": hn["kid"], "cta": hn["cta"]}
         row_bytes = (2 + 8 + 2 + 8) if narrow else 24
 
+        e2e_debug = os.environ.get("BENCH_E2E_DEBUG")
+
         def e2e_step(c):
+            t0 = time.perf_counter()
             with load_lock:
+                t1 = time.perf_counter()
                 tr_h = sieve.load_trace(c, up["kid"], hn["x"], num_kernels=cfg.K, cta=up["cta"],
                                         cycles=hn["y"], first_id=first)
+            t2 = time.perf_counter()
             st_h = sieve.stratify(tr_h)
             pr = sieve.predict(st_h, tr_h)
             out["strata"] = len(st_h.table)   # the stratum table, read by the caller
             del tr_h
+            if e2e_debug:
+                t3 = time.perf_counter()
+                print(f"[e2e] {threading.current_thread().name} lock wait {1e3 * (t1 - t0):.2f} load "
+                      f"{1e3 * (t2 - t1):.2f} stratify+predict+free {1e3 * (t3 - t2):.2f} ms", file=sys.stderr)
             return pr
 
         for c, _ in lanes:   # warm each context once

@@ -514,17 +514,22 @@ extern "C" int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_
       if (bytes) SV_CUDA(cudaMemcpyAsync(*dst, src, bytes, kind, ctx->stream));
       return SIEVE_OK;
     };
-    // a 16-bit column is copied as it is into a temporary, then widened into the u32 column
+    // A 16-bit column is copied as it is into a temporary and widened into the u32 column after
+    // ALL the copies are queued: the copy engine streams the columns back to back (a widening
+    // kernel between two copies would wait for free SMs -- behind another context's KDE, say --
+    // with the engine idle).  The call returns once the caller's arrays have been read (an event
+    // after the last copy); the widening completes in stream order before any later work.
+    struct Widen { void* tmp; u32* dst; };
+    Widen wd[2];
+    int nwd = 0;
     auto cp16 = [&](void** dst, const void* src) -> int {
       if (!src) { *dst = nullptr; return SIEVE_OK; }
       SV_TRY(dalloc(ctx, dst, n_local * 4));
       if (!n_local) return SIEVE_OK;
       void* tmp = nullptr;
       SV_TRY(dalloc(ctx, &tmp, n_local * 2));
-      cudaError_t e = cudaMemcpyAsync(tmp, src, n_local * 2, kind, ctx->stream);
-      if (e == cudaSuccess) { launch_widen_u16(tmp, n_local, (u32*)*dst, ctx->stream); e = cudaGetLastError(); }
-      dfree(ctx, t->owner, tmp);
-      if (e != cudaSuccess) return sv_cuda(e, "16-bit column", __LINE__);
+      wd[nwd++] = {tmp, (u32*)*dst};
+      SV_CUDA(cudaMemcpyAsync(tmp, src, n_local * 2, kind, ctx->stream));
       return SIEVE_OK;
     };
     int st = SIEVE_OK;
@@ -533,7 +538,25 @@ extern "C" int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_
     if (st == SIEVE_OK) st = cp((void**)&t->x, instr ? instr : (const uint64_t*)&t->n, n_local * 8);
     if (st == SIEVE_OK) st = cta16 ? cp16((void**)&t->cta, cta) : cp((void**)&t->cta, cta, n_local * 4);
     if (st == SIEVE_OK) st = cp((void**)&t->y, cycles, n_local * 8);
-    if (st == SIEVE_OK) { cudaError_t e = cudaStreamSynchronize(ctx->stream); if (e) st = sv_cuda(e, "load sync", __LINE__); }
+    cudaEvent_t copied = nullptr;
+    if (st == SIEVE_OK && !dev) {
+      cudaError_t e = cudaEventCreateWithFlags(&copied, cudaEventDisableTiming);
+      if (e == cudaSuccess) e = cudaEventRecord(copied, ctx->stream);
+      if (e != cudaSuccess) st = sv_cuda(e, "load event", __LINE__);
+    }
+    for (int i = 0; i < nwd; i++) {
+      if (st == SIEVE_OK) {
+        launch_widen_u16(wd[i].tmp, n_local, wd[i].dst, ctx->stream);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) st = sv_cuda(e, "16-bit column", __LINE__);
+      }
+      dfree(ctx, t->owner, wd[i].tmp);
+    }
+    if (st == SIEVE_OK) {
+      cudaError_t e = copied ? cudaEventSynchronize(copied) : cudaStreamSynchronize(ctx->stream);
+      if (e) st = sv_cuda(e, "load sync", __LINE__);
+    }
+    if (copied) cudaEventDestroy(copied);
     if (st != SIEVE_OK) { t->magic = TRACE_MAGIC; sieve_trace_free(t); return st; }
   }
   *out = t;
