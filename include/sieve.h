@@ -118,7 +118,9 @@ void sieve_ctx_destroy(sieve_ctx ctx);
      mem          SIEVE_MEM_HOST | SIEVE_MEM_DEVICE [| SIEVE_ADOPT] [| SIEVE_KID16] [| SIEVE_CTA16]
                   (the 16-bit forms change only what is copied: the trace holds u32 columns)
    Value validation (kernel id < K, 1 <= x < 2^44) happens on the device in the first pass of
-   sieve_stratify, which returns SIEVE_EINVAL / SIEVE_ERANGE on a bad row. */
+   sieve_stratify, which returns SIEVE_EINVAL / SIEVE_ERANGE on a bad row.
+   Return: the caller's arrays have been read in full (host or device) and may be reused; the
+   widening of 16-bit columns may still run on ctx's stream, ahead of any later call's work. */
 int sieve_load_trace(sieve_ctx ctx, uint64_t n_local, uint64_t first_id, uint32_t num_kernels,
                      const uint32_t* kernel_id, const uint64_t* instr, const uint32_t* cta,
                      const uint64_t* cycles, uint32_t mem, sieve_trace* out);
