@@ -1164,25 +1164,26 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       launch_fill_multi(fr, S);
     }
     if (nin) {
-      DBuf<u64> tile_range(c);
+      DBuf<char> regions(c);
       DBuf<u32> tile_items(c);
       DBuf<char> stemp(c);
-      SV_TRY(tile_range.alloc((size_t)nseg * tps * 2));
+      SV_TRY(regions.alloc(kde_region_bytes((u64)nseg * tps)));
       SV_TRY(tile_items.alloc((size_t)nseg * tps + 1));
       SV_TRY(stemp.alloc(scan_u32_temp_bytes((u64)nseg * tps)));
       // work items are counted on the device; size the item map by a host-side bound so no
-      // synchronisation is needed here: a tile has at most ceil(segment values / KDE_CH) items
+      // synchronisation is needed here: a tile has at most ceil(segment values / KDE_CH) + slack
+      // items (its regions are disjoint runs of the segment's values)
       u64 items_bound = 0, global_bound = 0;
       for (u32 s = 0; s < nseg; s++) {
         u64 len = round == 1 ? h_localn[op[s].kid] : op[s].e - op[s].b;
-        items_bound += (u64)tps * ((len + KDE_CH - 1) / KDE_CH);
-        global_bound += (u64)tps * ((op[s].n + KDE_CH - 1) / KDE_CH);  // replicated on every rank
+        items_bound += (u64)tps * ((len + KDE_CH - 1) / KDE_CH + kde_items_per_tile_slack());
+        global_bound += (u64)tps * ((op[s].n + KDE_CH - 1) / KDE_CH + kde_items_per_tile_slack());  // replicated
       }
       // the limit is decided on the segments' GLOBAL counts, identical on every rank, so no rank
       // returns while the others enter AR-2 (the local bound is at most the global one)
       if (global_bound >= (1ull << 32)) return sv_fail(SIEVE_ELIMIT, "too many KDE work items");
       u32 items = (u32)items_bound;
-      kde_plan(segs.get(), nseg, G, gtab.get(), off.get(), tile_range.get(), tile_items.get(), stemp.get(), S);
+      kde_plan(segs.get(), nseg, G, gtab.get(), off.get(), regions.get(), tile_items.get(), stemp.get(), S);
       DBuf<char> item_tile(c);
       SV_TRY(item_tile.alloc(kde_item_bytes(items)));
       PhaseTimer tm(c, SIEVE_PHASE_KDE, 0);
@@ -1191,10 +1192,18 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       bool guard = false;
       for (u32 s = 0; s < nseg; s++)
         if ((double)(hs[s].hi - hs[s].lo) / (double)(G - 1) >= 140.0 * hs[s].h) guard = true;
-      launch_kde(segs.get(), nseg, G, ck.get(), vsh, tile_range.get(), tile_items.get(),
+      launch_kde(segs.get(), nseg, G, ck.get(), vsh, regions.get(), tile_items.get(),
                  item_tile.get(), items, D.get(), terms.get() + 1, guard, false, S);
       tm.stop();
       SV_CUDA(cudaGetLastError());
+      if (getenv("SIEVE_KDE_STATS")) {  // diagnostic: work items of this round
+        const u64 nt = (u64)nseg * tps;
+        std::vector<u32> hi(nt + 1);
+        SV_CUDA(cudaStreamSynchronize(S));
+        SV_CUDA(cudaMemcpy(hi.data(), tile_items.get(), 4 * (nt + 1), cudaMemcpyDeviceToHost));
+        fprintf(stderr, "[kde stats] round=%u nseg=%u tiles=%llu items=%u\n", round, nseg,
+                (unsigned long long)nt, hi[nt]);
+      }
     }
     // AR-2: the densities' two u64 lanes per grid point (16 B), summed as the KDE left them;
     // k_valleys normalises them to u128

@@ -15,9 +15,11 @@
 // B200 mapping (the paper's scripts have no GPU design; this is new).  The KDE is a windowed
 // gather over the values of each segment grouped by grid cell (bucket.cu), bound by the FP64
 // pipe (no contraction, so no tensor cores).  Work item = (segment, tile of 32 grid points,
-// chunk of <= KDE_CH = 512 values inside the tile's window |g - x| <= 7.6 h); items are dealt to warps
-// round-robin and staged by a per-warp cp.async pipeline (see k_kde); each lane owns one grid
-// point and reads the staged values as shared-memory broadcasts.  The term is arranged to be
+// region of the tile's window |g - x| <= 7.6 h, chunk of <= KDE_CH = 512 values); a region is
+// evaluated by the lanes whose windows meet it (32, 16 or 8 lanes with 1, 2 or 4 value slices:
+// the staircase of k_kde_tiles); items are dealt to warps round-robin and staged by a per-warp
+// cp.async pipeline (see k_kde); each lane owns one grid point and reads the staged values as
+// shared-memory broadcasts.  The term is arranged to be
 // bit-identical to the oracle's while issuing 9 FP64-pipe instructions and ~6 others:
 //   * xs (per value, at staging) and gs (per lane, per item) are the A10 scaled coordinates,
 //     so z = gs - xs is one subtraction;
@@ -47,68 +49,153 @@
 #define KDE_UNROLL 14        // terms in flight per lane (A/B on C4 after the two-instruction table
 #endif                       // step: 14 -> 6.36 ms, 16 -> 6.61, 12 -> 6.45, 8 -> 6.46, 15 -> 6.85)
 static_assert(KDE_CH % 32 == 0, "each lane stages KDE_CH / 32 values of an item");
-#define KDE_V (32 / KDE_TJ)  // value slices per warp
+static_assert(KDE_TJ == 32, "a tile is one grid point per lane; narrower shapes are per region");
+#define KDE_MAXR 7           // regions per tile (at most 2 * 4 - 1 elementary cell intervals)
+#ifndef KDE_ITEM_OVH
+#define KDE_ITEM_OVH 64.f    // estimated cost of a work item beyond its terms, in terms per lane
+#endif
 
 __device__ __forceinline__ double grid_pt(u64 lo, u64 hi, u32 j, u32 G) {
   return __dadd_rn(__ull2double_rn(lo),
                    __ddiv_rn(__ull2double_rn((hi - lo) * (u64)j), __uint2double_rn(G - 1)));
 }
 
-// per (segment, tile of KDE_TJ grid points): the range of bucketed values in the cells that meet
-// the tile's window [g_j0 - 7.6 h, g_j1 + 7.6 h], and the number of KDE_CH-value chunks (work
-// items) it takes.  Values of the two boundary cells that lie outside the window are evaluated
-// too; their terms are exactly 0 (k > 10526).
+// A region of a tile: a run of whole cells [a, a + len) of the bucketed values and the lanes that
+// evaluate it, lanes o .. o + 2^lw - 1 of the tile (grid points j0 + o ...).
+struct KdeRegion { u32 a, len, shape; };   // shape = o | lw << 8
+static_assert(sizeof(KdeRegion) == 12, "");
+
+// per (segment, tile of 32 grid points): the tile's values split by which lanes need them.
+// Lane l needs the cells that meet its window [g_l - 7.6 h, g_l + 7.6 h] (beyond it every term
+// is exactly 0).  For each group of m lanes (m = 8, 16 or 32) the cells [L_q, R_q] meet the
+// window of some lane of the group; L and R are non-decreasing in q, so the cuts {L_q} U
+// {R_q + 1} split the tile's cells into at most 2 * 32/m - 1 intervals, each needed by a
+// contiguous run of groups: 8 lanes evaluate it with 4 value slices, 16 lanes with 2 slices,
+// 24 or 32 lanes as the whole warp.  Against one 32-lane range per tile the staircase of 8-lane
+// steps cuts the out-of-window evaluations at the two ends of the tile's window from
+// 2 x 31 x 32 / 2 lane-cells to 2 x 176.  Narrow regions cost extra work items, so the tile
+// takes the plan (m = 8, 16 or 32) with the least estimated per-lane cost: terms per lane plus
+// `ovh` per work item.  Values a region's lanes do not need (partial cells, the idle group of a
+// 3-group interval) are evaluated and add exactly 0, as before.
+struct KdePlan { KdeRegion r[KDE_MAXR]; u32 nr, items; float cost; };
+
+__device__ __forceinline__ void kde_tile_plan(const u32* L8, const u32* R8, u32 ng8, u32 m8,
+                                              const u32* of, float ovh, KdePlan& P) {
+  // groups of m8 eight-lane groups: L = first cell, R1 = one past the last cell
+  const u32 ng = (ng8 + m8 - 1) / m8;
+  u32 L[4], R1[4];
+  for (u32 q = 0; q < ng; q++) {
+    L[q] = L8[q * m8];
+    R1[q] = R8[min(ng8 - 1, q * m8 + m8 - 1)];
+  }
+  P.nr = 0; P.items = 0; P.cost = 0.f;
+  u32 il = 0, ir = 0, p = L[0];
+  int last = -1;
+  while (ir < ng) {   // walk the merged cuts (both lists are non-decreasing)
+    while (il < ng && L[il] <= p) il++;
+    while (ir < ng && R1[ir] <= p) ir++;
+    if (ir >= ng) break;
+    const u32 nxt = min(il < ng ? L[il] : 0xFFFFFFFFu, R1[ir]);
+    // groups needing cells [p, nxt): L_q <= p < R1_q  <=>  ir <= q < il
+    if (il > ir) {
+      const u32 lanes = (il - ir) * 8 * m8;
+      const u32 shape = lanes == 8 ? 8 * m8 * ir | 3u << 8 : lanes == 16 ? 8 * m8 * ir | 4u << 8 : 5u << 8;
+      const u32 a = of[p], z = of[nxt];
+      if (z > a) {
+        if ((int)shape == last && P.r[P.nr - 1].a + P.r[P.nr - 1].len == a) {
+          P.r[P.nr - 1].len += z - a;
+        } else {
+          P.r[P.nr].a = a; P.r[P.nr].len = z - a; P.r[P.nr].shape = shape;
+          P.nr++;
+        }
+        last = (int)shape;
+      }
+    }
+    p = nxt;
+  }
+  for (u32 r = 0; r < P.nr; r++) {
+    const u32 ni = (P.r[r].len + KDE_CH - 1) / KDE_CH;
+    P.items += ni;
+    P.cost += (float)P.r[r].len * (float)(1u << (P.r[r].shape >> 8)) * (1.f / 32.f) + ovh * (float)ni;
+  }
+}
+
 __global__ void k_kde_tiles(const SegDev* segs, u32 nseg, u32 G, u32 tps, const double* gtab,
-                            const u32* off, u64* tile_range, u32* tile_items) {
+                            const u32* off, KdeRegion* regions, u32* tile_items, float ovh) {
   pdl_begin();
   u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
   if (id >= (u64)nseg * tps) return;
   u32 s = (u32)(id / tps), t = (u32)(id % tps);
   SegDev g = segs[s];
   const double* gt = gtab + (u64)s * G;
-  u32 j0 = t * KDE_TJ;
-  u32 j1 = min(G - 1, j0 + KDE_TJ - 1);
-  double w = __dmul_rn(KDE_W, g.h);
-  double ga = __dsub_rn(gt[j0], w);
-  double gb = __dadd_rn(gt[j1], w);
-  u64 xa = ga <= (double)g.lo ? g.lo : (u64)floor(ga);
-  u64 xb = gb >= (double)g.hi ? g.hi : (u64)ceil(gb);
-  u32 ca = cell_of(gt, G, g.lo, g.cq, xa), cb = cell_of(gt, G, g.lo, g.cq, xb);
-  u64 a = off[(u64)s * G + ca];
-  u64 z = off[(u64)s * G + cb + 1];
-  tile_range[2 * id] = a;
-  tile_range[2 * id + 1] = z;
-  tile_items[id] = (u32)((z - a + KDE_CH - 1) / KDE_CH);
+  const u32* of = off + (u64)s * G;
+  const u32 j0 = t * KDE_TJ;
+  const u32 live = min(G - j0, (u32)KDE_TJ);
+  const u32 ng = (live + 7) / 8;
+  const double w = __dmul_rn(KDE_W, g.h);
+  u32 L[4], R1[4];   // per 8-lane group: first cell, one past the last cell it needs
+  for (u32 q = 0; q < ng; q++) {
+    const double ga = __dsub_rn(gt[j0 + 8 * q], w);
+    const double gb = __dadd_rn(gt[min(G - 1, j0 + 8 * q + 7)], w);
+    const u64 xa = ga <= (double)g.lo ? g.lo : (u64)floor(ga);
+    const u64 xb = gb >= (double)g.hi ? g.hi : (u64)ceil(gb);
+    L[q] = cell_of(gt, G, g.lo, g.cq, xa);
+    R1[q] = cell_of(gt, G, g.lo, g.cq, xb) + 1;
+  }
+  KdePlan best, P;
+  kde_tile_plan(L, R1, ng, 4, of, ovh, best);   // one 32-lane region
+  if (ovh < 1e30f) {
+    for (u32 m8 = 2; m8 >= 1; m8--) {
+      kde_tile_plan(L, R1, ng, m8, of, ovh, P);
+      if (P.cost < best.cost) best = P;
+    }
+  }
+  KdeRegion* rg = regions + id * KDE_MAXR;
+  for (u32 r = 0; r < KDE_MAXR; r++) {
+    if (r < best.nr) rg[r] = best.r[r];
+    else rg[r].len = 0;
+  }
+  tile_items[id] = best.items;
 }
 
-
 void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
-              u64* tile_range, u32* tile_items, void* scan_temp, cudaStream_t s) {
+              void* regions, u32* tile_items, void* scan_temp, cudaStream_t s) {
   u32 tps = div_up(G, KDE_TJ);
   u64 nt = (u64)nseg * tps;
-  SV_LAUNCH(k_kde_tiles, div_up(nt, 128), 128, 0, s)(segs, nseg, G, tps, gtab, off, tile_range, tile_items);
+  // SIEVE_KDE_OVH: the per-item cost the plan choice assumes, in terms per lane (A/B and test
+  // hook: 0 = always the finest staircase, "inf" = always one 32-lane region per tile)
+  const char* e = getenv("SIEVE_KDE_OVH");
+  float ovh = e ? (float)atof(e) : KDE_ITEM_OVH;
+  if (!(ovh >= 0.f)) ovh = KDE_ITEM_OVH;
+  SV_LAUNCH(k_kde_tiles, div_up(nt, 128), 128, 0, s)(segs, nseg, G, tps, gtab, off, (KdeRegion*)regions,
+                                                     tile_items, ovh);
   // exclusive scan in place; tile_items[nt] receives the total (read on the device by k_kde)
   scan_u32(tile_items, tile_items, nt, scan_temp, tile_items + nt, s);
 }
+
+size_t kde_region_bytes(u64 ntiles) { return (size_t)ntiles * KDE_MAXR * sizeof(KdeRegion); }
+u32 kde_items_per_tile_slack() { return KDE_MAXR - 1; }
 
 // one work item's descriptor, built on the device so a warp can prefetch it with one
 // asynchronous 48-byte copy: value range, first grid point and the segment's grid parameters
 struct __align__(16) KdeItem {
   u64 va;        // first value (index into the sorted cell keys)
   u32 len;       // values (<= KDE_CH)
-  u32 j0;        // first grid point of the tile
+  u32 j0;        // grid point of the item's lane 0 (tile start + region offset o)
   u64 lo, hi;    // segment range (grid g_j = rn(lo) + rn((hi - lo) j) / rn(G - 1))
   double inv_h;
   u32 s;         // segment
-  unsigned short live;    // grid points of the tile that exist (< KDE_TJ only in the last tile)
-  unsigned short fast;    // 1: every evaluated |z| < 18.8 (Delta / h < 0.33), so MODE 0 is exact
+  unsigned char live;   // lanes with an existing grid point (<= 2^lw)
+  unsigned char fast;   // 1: every evaluated |z| < 18.8 (Delta / h < 0.33), so MODE 0 is exact
+  unsigned char lw;     // log2 of the lanes per value slice: 5 (32 x 1), 4 (16 x 2), 3 (8 x 4)
+  unsigned char pad;
 };
 static_assert(sizeof(KdeItem) == 48, "KdeItem is copied as three 16-byte pieces");
 
 // item -> descriptor: one thread per item, binary search of the last tile whose first item is
-// <= it
+// <= it, then a walk over the tile's regions
 __global__ void k_kde_items(const SegDev* __restrict__ segs, u32 G, u32 tps,
-                            const u64* __restrict__ tile_range, const u32* __restrict__ tile_items,
+                            const KdeRegion* __restrict__ regions, const u32* __restrict__ tile_items,
                             u32 ntiles, KdeItem* __restrict__ desc) {
   pdl_begin();
   const u32 items = tile_items[ntiles];  // device-side total (no host round trip)
@@ -119,18 +206,28 @@ __global__ void k_kde_items(const SegDev* __restrict__ segs, u32 G, u32 tps,
       if (tile_items[m] <= it) lo = m; else hi = m - 1;
     }
     const u32 tile = lo, s = tile / tps, t = tile % tps;
+    const KdeRegion* rg = regions + (u64)tile * KDE_MAXR;
+    u32 rem = it - tile_items[tile], r = 0;
+    for (; r < KDE_MAXR - 1; r++) {
+      const u32 ni = (rg[r].len + KDE_CH - 1) / KDE_CH;
+      if (rem < ni) break;
+      rem -= ni;
+    }
+    const KdeRegion R = rg[r];
     const SegDev g = segs[s];
     KdeItem d;
-    d.va = tile_range[2 * (u64)tile] + (u64)(it - tile_items[tile]) * KDE_CH;
-    d.len = (u32)min((u64)KDE_CH, tile_range[2 * (u64)tile + 1] - d.va);
-    d.j0 = t * KDE_TJ;
+    d.va = (u64)R.a + (u64)rem * KDE_CH;
+    d.len = min((u32)KDE_CH, R.len - rem * KDE_CH);
+    d.j0 = t * KDE_TJ + (R.shape & 0xFF);
     d.lo = g.lo;
     d.hi = g.hi;
     d.inv_h = g.inv_h;
     d.s = s;
-    d.live = (unsigned short)min((u32)KDE_TJ, G - d.j0);
+    d.lw = (unsigned char)(R.shape >> 8);
+    d.live = (unsigned char)min(1u << d.lw, G - d.j0);
     // |z| <= 7.6 (window) + 33 grid steps (31 lanes + the two boundary cells) in units of h
     d.fast = (double)(g.hi - g.lo) < 0.33 * g.h * (double)(G - 1);
+    d.pad = 0;
     desc[it] = d;
   }
 }
@@ -292,19 +389,51 @@ __device__ __forceinline__ double kde_acc(double gs, double xs, const double* sS
 #endif
 // one lane's sum over the item's values: KDE_UNROLL independent accumulators, each an integer
 // in [2^52, 2^53) (a lane adds at most KDE_CH terms of <= 2^40 per item)
+// pair of staged values at a shared-memory byte address (a 128-bit shared load); volatile with a
+// memory clobber so the compiler keeps it behind the staging stores and __syncwarp
+#ifndef KDE_LDS
+#define KDE_LDS 1
+#endif
+__device__ __forceinline__ double2 lds_f64x2(u32 addr) {
+  double2 v;
+#if KDE_LDS == 1
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(addr) : "memory");
+#elif KDE_LDS == 2
+  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(addr));
+#else
+  v = *(const double2*)__cvta_shared_to_generic(addr);
+#endif
+  return v;
+}
+
+// one lane's run of len staged values starting at the shared-memory byte address sa (16-byte
+// aligned: runs start at even indices), read as 128-bit pairs with one induction variable
 template <int MODE>
-__device__ __forceinline__ u64 kde_item_sum(double gs, const double* sx, u32 i, u32 len,
-                                            const double* sSb, KdeRegs R) {
+__device__ __forceinline__ u64 kde_run_sum(double gs, u32 sa, u32 len, const double* sSb, KdeRegs R) {
+  static_assert(KDE_UNROLL % 2 == 0, "values are loaded in pairs");
   double ac[KDE_UNROLL];
 #pragma unroll
   for (int q = 0; q < KDE_UNROLL; q++) ac[q] = C_TWO52;
-  for (; i + (KDE_UNROLL - 1) * KDE_V < len; i += KDE_UNROLL * KDE_V) {
+  const u32 steps = len / KDE_UNROLL;   // full steps; the rest (< KDE_UNROLL values) one by one
+  const u32 ea = sa + steps * (KDE_UNROLL * 8);
+  u32 a = sa;
+  for (; a != ea; a += KDE_UNROLL * 8) {
 #pragma unroll
-    for (int q = 0; q < KDE_UNROLL; q++) ac[q] = kde_acc<MODE>(gs, sx[i + q * KDE_V], sSb, R, ac[q]);
+    for (int q = 0; q < KDE_UNROLL / 2; q++) {
+      const double2 v = lds_f64x2(a + 16 * q);
+      ac[2 * q] = kde_acc<MODE>(gs, v.x, sSb, R, ac[2 * q]);
+      ac[2 * q + 1] = kde_acc<MODE>(gs, v.y, sSb, R, ac[2 * q + 1]);
+    }
   }
+  const u32 rest = len - steps * KDE_UNROLL;   // < KDE_UNROLL
 #pragma unroll
-  for (int q = 0; q < KDE_UNROLL - 1; q++)
-    if (i + q * KDE_V < len) ac[q] = kde_acc<MODE>(gs, sx[i + q * KDE_V], sSb, R, ac[q]);
+  for (int q = 0; q < KDE_UNROLL - 1; q++) {
+    if ((u32)q < rest) {
+      double v;
+      asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a + 8 * q) : "memory");
+      ac[q] = kde_acc<MODE>(gs, v, sSb, R, ac[q]);
+    }
+  }
   u64 acc = 0;
 #pragma unroll
   for (int q = 0; q < KDE_UNROLL; q++) acc += (u64)__double_as_longlong(ac[q]) - 0x4330000000000000ull;
@@ -316,17 +445,11 @@ __device__ __forceinline__ u64 kde_item_sum(double gs, const double* sx, u32 i, 
 #define KDE_WARP_BYTES (2 * KDE_CH * 8 + 3 * 48)
 #define KDE_SMEM_BYTES (KDE_SMEM_TABLE + KDE_WARPS * KDE_WARP_BYTES)
 
-// A warp owns KDE_TJ grid points x KDE_V = 32 / KDE_TJ value slices: lane l evaluates grid
-// point j0 + l % KDE_TJ over the values i = l / KDE_TJ + m * KDE_V; slices are summed with
-// shuffles.  (Measured: 32 x 1 beats 8 x 4 -- the narrower value window of 8 x 4 saves ~10%
-// out-of-window terms but quadruples the per-item overhead at equal chunk size.)
+// A warp evaluates one item: its 2^lw lanes-per-slice own grid points j0 .. j0 + 2^lw - 1 (lane
+// l: j0 + l mod 2^lw) and the 32 / 2^lw value slices split the item's values into contiguous
+// runs (slice l div 2^lw); slices are summed with shuffles.  Whole-warp items (lw = 5) are the
+// tile's core, narrower ones the staircase at the ends of its window (k_kde_tiles).
 //
-// Items are dealt to warps round-robin (item w, w + W, w + 2W, ...; W warps in the grid; items
-// cost about the same) so every warp knows its future items, and a three-stage cp.async
-// pipeline keeps all global latency off the FP64 pipe: while item k is evaluated, the values of
-// item k + 1 and the descriptor of item k + 2 are in flight.  Densities are accumulated with
-// fire-and-forget reductions of two limbs (low 32 bits, the rest) into D[2j], D[2j + 1];
-// k_kde_fix turns them into the u128 D_j afterwards.
 template <bool GUARD>
 __global__ void __launch_bounds__(32 * KDE_WARPS, KDE_MINB)
 k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
@@ -413,14 +536,21 @@ k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
         sx[i] = __dmul_rn(__ull2double_rn(((u64)__double_as_longlong(sx[i]) >> vshift) - lo), inv_h);
     }
     __syncwarp();
-    const u32 slice = lane / KDE_TJ;
-    const u32 j = cd->j0 + lane % KDE_TJ;
+    const u32 lw = cd->lw;
+    const u32 slice = lane >> lw;
+    const u32 j = cd->j0 + (lane & ((1u << lw) - 1u));
+    // the slice's values: runs of an even length cs (16-byte aligned), cs != 0 mod 8 so the (up
+    // to four) slices' 128-bit loads fall in different banks
+    u32 cs = ((len >> (5 - lw)) + 2) & ~1u;
+    if ((cs & 7u) == 0) cs += 2;
+    const u32 sa = min(len, slice * cs);
+    const u32 sn = min(len - sa, cs);
     // gs = rn(rn(g_j - rn(lo)) * inv_h) (A10)
     const double gs = __dmul_rn(__dsub_rn(grid_pt(lo, cd->hi, j < G ? j : G - 1, G), __ull2double_rn(lo)), inv_h);
-    u64 acc = (!GUARD && allow_fast && cd->fast) ? kde_item_sum<0>(gs, sx, slice, len, sSb, R)
-                                   : kde_item_sum<GUARD ? 2 : 1>(gs, sx, slice, len, sSb, R);
-#pragma unroll
-    for (int o = KDE_TJ; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+    const bool fast = !GUARD && allow_fast && cd->fast;
+    const u32 ra = (u32)__cvta_generic_to_shared(sx + sa);
+    u64 acc = fast ? kde_run_sum<0>(gs, ra, sn, sSb, R) : kde_run_sum<GUARD ? 2 : 1>(gs, ra, sn, sSb, R);
+    for (u32 o = 1u << lw; o < 32; o <<= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
     // evaluated (lane, value) pairs of this item, wasted ones included
     if (evaluated && lane == 0) atomicAdd(evaluated, (unsigned long long)cd->live * len);
     if (j < G && slice == 0 && acc) {
@@ -449,7 +579,7 @@ __global__ void k_kde_fix(u64* D, u64 n) {
 
 size_t kde_item_bytes(u32 items) { return (size_t)items * sizeof(KdeItem) + 16; }
 
-void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const u64* tile_range,
+void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const void* regions,
                 const u32* tile_items, void* item_desc, u32 items, u64* D,
                 unsigned long long* evaluated, bool guard, bool fix, cudaStream_t s) {
   if (items == 0) {
@@ -461,7 +591,7 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift
   // `items` is a host-side upper bound: grids are sized by it, the kernels stop at the
   // device-side count tile_items[ntiles]
   KdeItem* desc = (KdeItem*)item_desc;
-  SV_LAUNCH(k_kde_items, min(div_up(items, 256), 4096u), 256, 0, s)(segs, G, tps, tile_range, tile_items,
+  SV_LAUNCH(k_kde_items, min(div_up(items, 256), 4096u), 256, 0, s)(segs, G, tps, (const KdeRegion*)regions, tile_items,
                                                                      ntiles, desc);
   // test hook SIEVE_KDE_FORCE: 1 = never the unclamped fast path, 2 = always the guarded
   // variant (all three evaluate identical terms; the parity tests run each)

@@ -90,15 +90,19 @@ inline double cell_margin(u64 lo, u64 hi, u32 G) {
 #define KDE_CH 512      // values per work item (A/B: 512 beats 256 by 2.5%; 16-point tiles lose)
 #endif
 #endif
-// per (segment, tile of KDE_TJ grid points): the range of bucketed values whose cells meet the
-// tile's window, chunked into work items; tile_items[nseg * tiles] receives the item total
+// per (segment, tile of KDE_TJ grid points): the bucketed values whose cells meet the tile's
+// window, split into regions by the lanes that need them (regions: kde_region_bytes(tiles)) and
+// chunked into work items; tile_items[nseg * tiles] receives the item total
 void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
-              u64* tile_range, u32* tile_items, void* scan_temp, cudaStream_t s);
+              void* regions, u32* tile_items, void* scan_temp, cudaStream_t s);
+size_t kde_region_bytes(u64 ntiles);
+// a tile has at most ceil(tile values / KDE_CH) + kde_items_per_tile_slack() work items
+u32 kde_items_per_tile_slack();
 size_t kde_item_bytes(u32 items);
 // D[2j] accumulates the low 32-bit limbs of the item sums, D[2j + 1] the rest (both are plain
 // u64 sums: several ranks may all-reduce them as they are); fix = true normalises them into the
 // u128 D_j right away (else call launch_kde_fix after the cross-rank sum)
-void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const u64* tile_range,
+void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift, const void* regions,
                 const u32* tile_items, void* item_desc /* kde_item_bytes(items) */, u32 items,
                 u64* D /* [nseg][G][2] */, unsigned long long* evaluated, bool guard, bool fix,
                 cudaStream_t s);

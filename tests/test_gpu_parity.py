@@ -278,6 +278,31 @@ def test_kde_evaluation_modes_identical(monkeypatch, mode):
     assert_segments_equal(g["segments"], o.segments())
 
 
+def test_kde_staircase_plans_identical(monkeypatch):
+    """k_kde_tiles splits each tile's values into regions evaluated by 8, 16 or 32 lanes (the
+    staircase at the ends of the tile's window) and picks a plan per tile by estimated cost.
+    The test hook SIEVE_KDE_OVH forces the finest staircase everywhere (0) or one 32-lane region
+    per tile (inf); both, and the default choice, must give every density, cut and stratum of
+    the oracle, and the staircase must evaluate fewer (lane, value) pairs, never fewer than the
+    in-window terms."""
+    tr = gen.make_trace("C3", n=400_000)
+    o = run_oracle(tr, keep_debug=True)
+    ev = {}
+    for ovh in ["0", "inf", None]:
+        if ovh is None:
+            monkeypatch.delenv("SIEVE_KDE_OVH", raising=False)
+        else:
+            monkeypatch.setenv("SIEVE_KDE_OVH", ovh)
+        g = run_gpu(tr, keep_debug=True)
+        assert_tables_equal(g["table"], o.strata)
+        assert np.array_equal(g["sid"], o.sid)
+        assert_segments_equal(g["segments"], o.segments())
+        ev[ovh] = (g["strata"].kde_evaluated, g["terms"])
+    assert ev["0"][1] == ev["inf"][1] == ev[None][1]
+    assert ev["0"][1] <= ev["0"][0] < ev["inf"][0]
+    assert ev["0"][0] <= ev[None][0] <= ev["inf"][0]
+
+
 @pytest.mark.parametrize("device", [False, True])
 def test_16bit_columns(device):
     """SIEVE_KID16 / SIEVE_CTA16: kernel ids and CTA sizes handed over as uint16 (host or device)
