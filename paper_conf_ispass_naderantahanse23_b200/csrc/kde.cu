@@ -77,85 +77,135 @@ static_assert(sizeof(KdeRegion) == 12, "");
 // takes the plan (m = 8, 16 or 32) with the least estimated per-lane cost: terms per lane plus
 // `ovh` per work item.  Values a region's lanes do not need (partial cells, the idle group of a
 // 3-group interval) are evaluated and add exactly 0, as before.
-struct KdePlan { KdeRegion r[KDE_MAXR]; u32 nr, items; float cost; };
-
-__device__ __forceinline__ void kde_tile_plan(const u32* L8, const u32* R8, u32 ng8, u32 m8,
-                                              const u32* of, float ovh, KdePlan& P) {
-  // groups of m8 eight-lane groups: L = first cell, R1 = one past the last cell
-  const u32 ng = (ng8 + m8 - 1) / m8;
-  u32 L[4], R1[4];
-  for (u32 q = 0; q < ng; q++) {
-    L[q] = L8[q * m8];
-    R1[q] = R8[min(ng8 - 1, q * m8 + m8 - 1)];
+// One plan (M8 = 4: one 32-lane region; 2: 16-lane steps; 1: 8-lane steps) over the tile's
+// per-group cells L[q] (first) and R1[q] (one past the last) and their value offsets LO / RO:
+// returns its estimated cost (terms per lane + ovh per work item) and item count, and with EMIT
+// writes its regions.  Everything stays in registers (static loops): the cut values are sorted
+// with their offsets by a static exchange sort, then each interval between distinct consecutive
+// cuts takes the lanes of the groups q with L_q <= p < R1_q (a contiguous run ir .. il - 1);
+// adjacent intervals of the same shape merge into one region.
+template <int M8, bool EMIT>
+__device__ __forceinline__ float kde_tile_plan(const u32 (&L)[4], const u32 (&R1)[4], const u32 (&LO)[4],
+                                               const u32 (&RO)[4], u32 ng8, float ovh, u32& items,
+                                               KdeRegion* rg) {
+  constexpr int NQ = 4 / M8;   // groups of this plan at most
+  const u32 ng = (ng8 + M8 - 1) / M8;
+  u32 Lm[NQ], Rm[NQ], c[2 * NQ], o[2 * NQ];
+#pragma unroll
+  for (int q = 0; q < NQ; q++) {
+    const bool live = (u32)q < ng;
+    const u32 qr = min(ng8 - 1, (u32)(q * M8 + M8 - 1));
+    u32 rv = 0, ro = 0;   // R1[qr], RO[qr] by a static select (a dynamic index would spill)
+#pragma unroll
+    for (int k = 0; k < 4; k++)
+      if ((u32)k == qr) { rv = R1[k]; ro = RO[k]; }
+    Lm[q] = live ? L[q * M8] : 0xFFFFFFFFu;
+    Rm[q] = live ? rv : 0xFFFFFFFFu;
+    c[q] = Lm[q]; o[q] = live ? LO[q * M8] : 0u;
+    c[NQ + q] = Rm[q]; o[NQ + q] = live ? ro : 0u;
   }
-  P.nr = 0; P.items = 0; P.cost = 0.f;
-  u32 il = 0, ir = 0, p = L[0];
-  int last = -1;
-  while (ir < ng) {   // walk the merged cuts (both lists are non-decreasing)
-    while (il < ng && L[il] <= p) il++;
-    while (ir < ng && R1[ir] <= p) ir++;
-    if (ir >= ng) break;
-    const u32 nxt = min(il < ng ? L[il] : 0xFFFFFFFFu, R1[ir]);
-    // groups needing cells [p, nxt): L_q <= p < R1_q  <=>  ir <= q < il
-    if (il > ir) {
-      const u32 lanes = (il - ir) * 8 * m8;
-      const u32 shape = lanes == 8 ? 8 * m8 * ir | 3u << 8 : lanes == 16 ? 8 * m8 * ir | 4u << 8 : 5u << 8;
-      const u32 a = of[p], z = of[nxt];
-      if (z > a) {
-        if ((int)shape == last && P.r[P.nr - 1].a + P.r[P.nr - 1].len == a) {
-          P.r[P.nr - 1].len += z - a;
-        } else {
-          P.r[P.nr].a = a; P.r[P.nr].len = z - a; P.r[P.nr].shape = shape;
-          P.nr++;
-        }
-        last = (int)shape;
+#pragma unroll
+  for (int i = 0; i < 2 * NQ; i++)
+#pragma unroll
+    for (int j = i + 1; j < 2 * NQ; j++)
+      if (c[j] < c[i]) {
+        const u32 tc = c[i], to = o[i];
+        c[i] = c[j]; o[i] = o[j]; c[j] = tc; o[j] = to;
       }
+  float cost = 0.f;
+  items = 0;
+  u32 pa = 0, plen = 0, pshape = 0xFFFFFFFFu, nr = 0;   // the pending region
+  auto close = [&]() {
+    if (pshape == 0xFFFFFFFFu) return;
+    const u32 ni = (plen + KDE_CH - 1) / KDE_CH;
+    items += ni;
+    cost += (float)plen * (float)(1u << (pshape >> 8)) * (1.f / 32.f) + ovh * (float)ni;
+    if (EMIT) { rg[nr].a = pa; rg[nr].len = plen; rg[nr].shape = pshape; }
+    nr++;
+  };
+#pragma unroll
+  for (int i = 0; i + 1 < 2 * NQ; i++) {
+    const u32 p = c[i], nx = c[i + 1];
+    if (nx == 0xFFFFFFFFu || nx == p) continue;
+    u32 il = 0, ir = 0;   // groups with L <= p, groups with R1 <= p (both lists non-decreasing)
+#pragma unroll
+    for (int q = 0; q < NQ; q++) {
+      il += Lm[q] <= p;
+      ir += Rm[q] <= p;
     }
-    p = nxt;
+    if (il <= ir) continue;   // no group needs cells [p, nx)
+    const u32 lanes = (il - ir) * 8 * M8;
+    const u32 shape = lanes == 8 ? 8 * M8 * ir | 3u << 8 : lanes == 16 ? 8 * M8 * ir | 4u << 8 : 5u << 8;
+    const u32 a = o[i], z = o[i + 1];
+    if (z <= a) continue;
+    if (shape == pshape && pa + plen == a) {
+      plen += z - a;
+    } else {
+      close();
+      pa = a; plen = z - a; pshape = shape;
+    }
   }
-  for (u32 r = 0; r < P.nr; r++) {
-    const u32 ni = (P.r[r].len + KDE_CH - 1) / KDE_CH;
-    P.items += ni;
-    P.cost += (float)P.r[r].len * (float)(1u << (P.r[r].shape >> 8)) * (1.f / 32.f) + ovh * (float)ni;
-  }
+  close();
+  if (EMIT)
+    for (u32 r = nr; r < KDE_MAXR; r++) rg[r].len = 0;
+  return cost;
 }
 
+// eight threads per tile: thread (side, q) finds group q's first cell (side 0) or one past its
+// last cell (side 1) and that cell's value offset, in parallel (each a short chain of dependent
+// loads); the tile's first thread gathers them by shuffles and plans in registers
 __global__ void k_kde_tiles(const SegDev* segs, u32 nseg, u32 G, u32 tps, const double* gtab,
                             const u32* off, KdeRegion* regions, u32* tile_items, float ovh) {
   pdl_begin();
-  u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
-  if (id >= (u64)nseg * tps) return;
-  u32 s = (u32)(id / tps), t = (u32)(id % tps);
-  SegDev g = segs[s];
-  const double* gt = gtab + (u64)s * G;
-  const u32* of = off + (u64)s * G;
-  const u32 j0 = t * KDE_TJ;
-  const u32 live = min(G - j0, (u32)KDE_TJ);
-  const u32 ng = (live + 7) / 8;
-  const double w = __dmul_rn(KDE_W, g.h);
-  u32 L[4], R1[4];   // per 8-lane group: first cell, one past the last cell it needs
-  for (u32 q = 0; q < ng; q++) {
-    const double ga = __dsub_rn(gt[j0 + 8 * q], w);
-    const double gb = __dadd_rn(gt[min(G - 1, j0 + 8 * q + 7)], w);
-    const u64 xa = ga <= (double)g.lo ? g.lo : (u64)floor(ga);
-    const u64 xb = gb >= (double)g.hi ? g.hi : (u64)ceil(gb);
-    L[q] = cell_of(gt, G, g.lo, g.cq, xa);
-    R1[q] = cell_of(gt, G, g.lo, g.cq, xb) + 1;
-  }
-  KdePlan best, P;
-  kde_tile_plan(L, R1, ng, 4, of, ovh, best);   // one 32-lane region
-  if (ovh < 1e30f) {
-    for (u32 m8 = 2; m8 >= 1; m8--) {
-      kde_tile_plan(L, R1, ng, m8, of, ovh, P);
-      if (P.cost < best.cost) best = P;
+  const u64 nt = (u64)nseg * tps;
+  const u64 id = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 3;
+  const u32 t8 = threadIdx.x & 7, q = t8 & 3, side = t8 >> 2;
+  const bool valid = id < nt;
+  u32 s = 0, j0 = 0, ng = 0, cell = 0, coff = 0;
+  if (valid) {
+    s = (u32)(id / tps);
+    j0 = (u32)(id % tps) * KDE_TJ;
+    ng = (min(G - j0, (u32)KDE_TJ) + 7) / 8;
+    if (q < ng) {
+      const SegDev g = segs[s];
+      const double* gt = gtab + (u64)s * G;
+      const double w = __dmul_rn(KDE_W, g.h);
+      if (side == 0) {
+        const double ga = __dsub_rn(gt[j0 + 8 * q], w);
+        const u64 xa = ga <= (double)g.lo ? g.lo : (u64)floor(ga);
+        cell = cell_of(gt, G, g.lo, g.cq, xa);
+      } else {
+        const double gb = __dadd_rn(gt[min(G - 1, j0 + 8 * q + 7)], w);
+        const u64 xb = gb >= (double)g.hi ? g.hi : (u64)ceil(gb);
+        cell = cell_of(gt, G, g.lo, g.cq, xb) + 1;
+      }
+      coff = off[(u64)s * G + cell];
     }
   }
-  KdeRegion* rg = regions + id * KDE_MAXR;
-  for (u32 r = 0; r < KDE_MAXR; r++) {
-    if (r < best.nr) rg[r] = best.r[r];
-    else rg[r].len = 0;
+  u32 L[4], R1[4], LO[4], RO[4];
+  const u32 base = lane_id() & ~7u;
+#pragma unroll
+  for (int i = 0; i < 4; i++) {
+    L[i] = __shfl_sync(0xffffffffu, cell, base + i);
+    LO[i] = __shfl_sync(0xffffffffu, coff, base + i);
+    R1[i] = __shfl_sync(0xffffffffu, cell, base + 4 + i);
+    RO[i] = __shfl_sync(0xffffffffu, coff, base + 4 + i);
   }
-  tile_items[id] = best.items;
+  if (!valid || t8 != 0) return;
+  KdeRegion* rg = regions + id * KDE_MAXR;
+  u32 items = 0, it2 = 0, it1 = 0;
+  if (!(ovh < 1e30f)) {   // test hook "inf": one 32-lane region per tile
+    kde_tile_plan<4, true>(L, R1, LO, RO, ng, 0.f, items, rg);
+    tile_items[id] = items;
+    return;
+  }
+  const float c4 = kde_tile_plan<4, false>(L, R1, LO, RO, ng, ovh, items, rg);
+  const float c2 = kde_tile_plan<2, false>(L, R1, LO, RO, ng, ovh, it2, rg);
+  const float c1 = kde_tile_plan<1, false>(L, R1, LO, RO, ng, ovh, it1, rg);
+  if (c1 < c2 && c1 < c4) kde_tile_plan<1, true>(L, R1, LO, RO, ng, ovh, items, rg);
+  else if (c2 < c4) kde_tile_plan<2, true>(L, R1, LO, RO, ng, ovh, items, rg);
+  else kde_tile_plan<4, true>(L, R1, LO, RO, ng, ovh, items, rg);
+  tile_items[id] = items;
 }
 
 void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
@@ -167,8 +217,8 @@ void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32
   const char* e = getenv("SIEVE_KDE_OVH");
   float ovh = e ? (float)atof(e) : KDE_ITEM_OVH;
   if (!(ovh >= 0.f)) ovh = KDE_ITEM_OVH;
-  SV_LAUNCH(k_kde_tiles, div_up(nt, 128), 128, 0, s)(segs, nseg, G, tps, gtab, off, (KdeRegion*)regions,
-                                                     tile_items, ovh);
+  SV_LAUNCH(k_kde_tiles, div_up(nt * 8, 256), 256, 0, s)(segs, nseg, G, tps, gtab, off, (KdeRegion*)regions,
+                                                         tile_items, ovh);
   // exclusive scan in place; tile_items[nt] receives the total (read on the device by k_kde)
   scan_u32(tile_items, tile_items, nt, scan_temp, tile_items + nt, s);
 }
@@ -192,43 +242,54 @@ struct __align__(16) KdeItem {
 };
 static_assert(sizeof(KdeItem) == 48, "KdeItem is copied as three 16-byte pieces");
 
-// item -> descriptor: one thread per item, binary search of the last tile whose first item is
-// <= it, then a walk over the tile's regions
+// tile -> its items' descriptors: one warp per tile (no search: the tile's first item is its
+// scanned item count); lane i writes items i, i + 32, ... of the tile, finding each one's region
+// from the regions' item counts (at most KDE_MAXR, read once per lane)
 __global__ void k_kde_items(const SegDev* __restrict__ segs, u32 G, u32 tps,
                             const KdeRegion* __restrict__ regions, const u32* __restrict__ tile_items,
                             u32 ntiles, KdeItem* __restrict__ desc) {
   pdl_begin();
-  const u32 items = tile_items[ntiles];  // device-side total (no host round trip)
-  for (u32 it = blockIdx.x * blockDim.x + threadIdx.x; it < items; it += gridDim.x * blockDim.x) {
-    u32 lo = 0, hi = ntiles - 1;
-    while (lo < hi) {
-      u32 m = (lo + hi + 1) >> 1;
-      if (tile_items[m] <= it) lo = m; else hi = m - 1;
-    }
-    const u32 tile = lo, s = tile / tps, t = tile % tps;
+  const u32 lane = lane_id();
+  const u32 warps = gridDim.x * (blockDim.x >> 5);
+  for (u32 tile = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); tile < ntiles; tile += warps) {
+    const u32 first = tile_items[tile], n = tile_items[tile + 1] - first;
+    if (n == 0) continue;
+    const u32 s = tile / tps, t = tile % tps;
     const KdeRegion* rg = regions + (u64)tile * KDE_MAXR;
-    u32 rem = it - tile_items[tile], r = 0;
-    for (; r < KDE_MAXR - 1; r++) {
-      const u32 ni = (rg[r].len + KDE_CH - 1) / KDE_CH;
-      if (rem < ni) break;
-      rem -= ni;
+    KdeRegion R[KDE_MAXR];
+    u32 ni[KDE_MAXR];
+#pragma unroll
+    for (int r = 0; r < KDE_MAXR; r++) {
+      R[r] = rg[r];
+      ni[r] = (R[r].len + KDE_CH - 1) / KDE_CH;
     }
-    const KdeRegion R = rg[r];
     const SegDev g = segs[s];
-    KdeItem d;
-    d.va = (u64)R.a + (u64)rem * KDE_CH;
-    d.len = min((u32)KDE_CH, R.len - rem * KDE_CH);
-    d.j0 = t * KDE_TJ + (R.shape & 0xFF);
-    d.lo = g.lo;
-    d.hi = g.hi;
-    d.inv_h = g.inv_h;
-    d.s = s;
-    d.lw = (unsigned char)(R.shape >> 8);
-    d.live = (unsigned char)min(1u << d.lw, G - d.j0);
     // |z| <= 7.6 (window) + 33 grid steps (31 lanes + the two boundary cells) in units of h
-    d.fast = (double)(g.hi - g.lo) < 0.33 * g.h * (double)(G - 1);
-    d.pad = 0;
-    desc[it] = d;
+    const unsigned char fast = (double)(g.hi - g.lo) < 0.33 * g.h * (double)(G - 1);
+    for (u32 k = lane; k < n; k += 32) {
+      u32 q = k, a = 0, len = 0, shape = 0;   // q: the item's chunk inside its region
+      bool found = false;
+#pragma unroll
+      for (int r = 0; r < KDE_MAXR; r++) {      // static selects (no local memory)
+        if (!found) {
+          if (q < ni[r]) { found = true; a = R[r].a; len = R[r].len; shape = R[r].shape; }
+          else q -= ni[r];
+        }
+      }
+      KdeItem d;
+      d.va = (u64)a + (u64)q * KDE_CH;
+      d.len = min((u32)KDE_CH, len - q * KDE_CH);
+      d.j0 = t * KDE_TJ + (shape & 0xFF);
+      d.lo = g.lo;
+      d.hi = g.hi;
+      d.inv_h = g.inv_h;
+      d.s = s;
+      d.lw = (unsigned char)(shape >> 8);
+      d.live = (unsigned char)min(1u << d.lw, G - d.j0);
+      d.fast = fast;
+      d.pad = 0;
+      desc[first + k] = d;
+    }
   }
 }
 
@@ -591,7 +652,7 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift
   // `items` is a host-side upper bound: grids are sized by it, the kernels stop at the
   // device-side count tile_items[ntiles]
   KdeItem* desc = (KdeItem*)item_desc;
-  SV_LAUNCH(k_kde_items, min(div_up(items, 256), 4096u), 256, 0, s)(segs, G, tps, (const KdeRegion*)regions, tile_items,
+  SV_LAUNCH(k_kde_items, min(div_up(ntiles, 8), 4096u), 256, 0, s)(segs, G, tps, (const KdeRegion*)regions, tile_items,
                                                                      ntiles, desc);
   // test hook SIEVE_KDE_FORCE: 1 = never the unclamped fast path, 2 = always the guarded
   // variant (all three evaluate identical terms; the parity tests run each)

@@ -44,8 +44,14 @@ def test_c3_parity():
     assert_predictions_close(sieve.predict(g["strata"], g["trace"]), o.predict())
 
 
-@pytest.mark.parametrize("G", [3, 64, 1000, 4096])
-def test_grid_sizes(G):
+@pytest.mark.parametrize("G,ovh", [(3, None), (64, None), (1000, None), (4096, None), (3, "0"), (21, "0"),
+                                   (50, "0"), (1000, "0"), (10000, "0")])
+def test_grid_sizes(G, ovh, monkeypatch):
+    """grid sizes from 3 to 10000, with the default KDE tile plans and with the finest staircase
+    forced (ovh "0"): tiles with fewer than 32 live grid points, partial 8-lane groups, and the
+    radix cell path (G > 8192)"""
+    if ovh is not None:
+        monkeypatch.setenv("SIEVE_KDE_OVH", ovh)
     tr = gen.make_trace("C2", n=120_000)
     g = run_gpu(tr, G=G, keep_debug=True)
     o = run_oracle(tr, G=G, keep_debug=True)

@@ -15,14 +15,22 @@ template <int V>
 __device__ __forceinline__ double term(double gs, double xs, double L, double M, double acc) {
   double z = __dsub_rn(gs, xs);
   double u = __dmul_rn(z, z);
-  double kb = __fma_rn(u, L, M);
+  double Lu = L;
+  if (V == 4) asm volatile("ld.const.f64 %0, [c_k];" : "=d"(Lu));
+  double kb = __fma_rn(u, Lu, M);
   double kf;
   if (V == 0) kf = __dsub_rn(kb, C_MAGIC);
   else if (V == 1) kf = __int2double_rn(__double2loint(kb));
   else if (V == 2) kf = __uint2double_rn((u32)__double2loint(kb));
-  else kf = (double)__int2float_rn(__double2loint(kb));
-  double r = __fma_rn(-kf, c_k[1], u);
-  double p = __fma_rn(c_k[2], r, 0.125);
+  else if (V == 3) kf = (double)__int2float_rn(__double2loint(kb));
+  else kf = __dsub_rn(kb, C_MAGIC);
+  double c1 = c_k[1], c2 = c_k[2];
+  if (V == 4) {   // constants through uniform registers: ld.const at the use, hoisted by ptxas
+    asm volatile("ld.const.f64 %0, [c_k+8];" : "=d"(c1));
+    asm volatile("ld.const.f64 %0, [c_k+16];" : "=d"(c2));
+  }
+  double r = __fma_rn(-kf, c1, u);
+  double p = __fma_rn(c2, r, 0.125);
   p = __fma_rn(p, r, -0.5);
   p = __fma_rn(p, r, 1.0);
   return __fma_rn(p, z, acc);
@@ -69,8 +77,9 @@ int main() {
     run<1, 14, 512>("kf = I2F.F64.S32(lo(kb))", d, it);
     run<2, 14, 512>("kf = I2F.F64.U32(lo(kb))", d, it);
     run<3, 14, 512>("kf = F2F.F64(I2F.F32)", d, it);
-    run<0, 8, 512>("kf = kb - magic (DADD)", d, it);
-    run<1, 8, 512>("kf = I2F.F64.S32(lo(kb))", d, it);
+    run<4, 14, 512>("constants in uniform regs", d, it);
+    run<4, 16, 512>("constants in uniform regs", d, it);
+    run<4, 12, 512>("constants in uniform regs", d, it);
   }
   return 0;
 }

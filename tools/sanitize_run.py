@@ -1,6 +1,7 @@
 """Workload for compute-sanitizer (memcheck / racecheck / synccheck): C1 and a 200k-invocation
 slice of C2 through sieve_stratify + sieve_predict (keep_debug on, so every KDE segment is read
-back; the C2 slice also with pass B's hash and four-slot variants), plus C1 over an in-process
+back; the C2 slice also with pass B's hash and four-slot variants and the KDE's finest and
+coarsest tile plans), plus C1 over an in-process
 2-rank group (the multi-rank reduction kernels).
 
     compute-sanitizer --tool racecheck python tools/sanitize_run.py [--no-group]
@@ -118,7 +119,11 @@ if __name__ == "__main__":
     for v in ("hash", "4"):   # pass B's other variants (two slots per stratum is the default)
         os.environ["SIEVE_ASSIGN"] = v
         one(gen.make_trace("C2"), n=200_000)
-    del os.environ["SIEVE_ASSIGN"]
+    os.environ.pop("SIEVE_ASSIGN", None)
+    for v in ("0", "inf"):    # the KDE plans: finest staircase everywhere, one region per tile
+        os.environ["SIEVE_KDE_OVH"] = v
+        one(gen.make_trace("C2"), n=200_000)
+    os.environ.pop("SIEVE_KDE_OVH", None)
     if "--no-group" not in sys.argv:
         group(gen.make_trace("C1"))
     print("sanitize workload done")
