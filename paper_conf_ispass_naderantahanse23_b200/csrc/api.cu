@@ -1942,19 +1942,16 @@ extern "C" int sieve_load_csv(sieve_ctx ctx, const char* data, uint64_t bytes, u
   cudaStream_t S = c->stream;
   SV_CUDA(cudaSetDevice(c->device));
   SV_TRY(arena_reset(c));
-  // the bytes on the device, and on the host (for the names)
+  // the bytes on the device (host text: one upload; the names are read from the host text, or,
+  // for device-resident text, gathered on the device and only they come back)
+  const bool dev_text = (mem & SIEVE_MEM_DEVICE) != 0;
   const unsigned char* dbuf = (const unsigned char*)data;
-  std::vector<char> hostcopy;
-  const char* hbuf = data;
-  if (!(mem & SIEVE_MEM_DEVICE)) {
+  const char* hbuf = dev_text ? nullptr : data;
+  if (!dev_text) {
     DBuf<unsigned char> db(c);
     SV_TRY(db.alloc(bytes ? bytes : 1));
     if (bytes) SV_CUDA(cudaMemcpyAsync(db.get(), data, bytes, cudaMemcpyHostToDevice, S));
     dbuf = db.get();
-  } else {
-    hostcopy.resize(bytes);
-    if (bytes) SV_CUDA(cudaMemcpyAsync(hostcopy.data(), data, bytes, cudaMemcpyDeviceToHost, S));
-    hbuf = hostcopy.data();
   }
   // 1. line ends
   const u64 nt = csv_tiles(bytes);
@@ -1966,12 +1963,14 @@ extern "C" int sieve_load_csv(sieve_ctx ctx, const char* data, uint64_t bytes, u
   launch_csv_count(dbuf, bytes, tiles.get(), stemp.get(), S);
   std::vector<u32> h_nl;
   SV_TRY(d2h(c, h_nl, tiles.get() + nt, 1));
+  char last = 0;   // the text's last byte (device-resident text: read with the line count)
+  if (bytes && dev_text) SV_TRY(d2h_raw(c, &last, dbuf + bytes - 1, 1));
   SV_TRY(sync(c));
   const u64 nends = h_nl[0];
   DBuf<u64> ends(c);
   SV_TRY(ends.alloc(nends + 1));
   launch_csv_ends(dbuf, bytes, tiles.get(), ends.get(), S);
-  bool trailing = bytes > 0 && hbuf[bytes - 1] == '\n';
+  const bool trailing = bytes > 0 && (dev_text ? last : hbuf[bytes - 1]) == '\n';
   const u64 nlines = nends + (bytes > 0 && !trailing ? 1 : 0);
   const u64 nrows = nlines > spec->header_lines ? nlines - spec->header_lines : 0;
   if (nrows >= (1ull << 32)) return sv_fail(SIEVE_ERANGE, "more than 2^32 - 1 rows");
@@ -2032,11 +2031,24 @@ extern "C" int sieve_load_csv(sieve_ctx ctx, const char* data, uint64_t bytes, u
     if ((st = sync(c)) != SIEVE_OK) return fail(st);
     { cudaError_t ce = cudaGetLastError(); if (ce) return fail(sv_cuda(ce, "csv kernels", __LINE__)); }
   }
+  std::vector<unsigned char> h_text;   // device-resident text: the distinct names' bytes only
+  std::vector<u64> name_off(nd + 1, 0);
+  if (dev_text && nd) {
+    for (u64 d = 0; d < nd; d++) name_off[d + 1] = name_off[d] + h_names[2 * d + 1];
+    DBuf<u64> d_pos(c), d_off(c);
+    DBuf<unsigned char> d_txt(c);
+    CSV_TRY(d_pos.alloc(2 * nd)); CSV_TRY(d_off.alloc(nd + 1)); CSV_TRY(d_txt.alloc(name_off[nd] + 1));
+    CSV_TRY(h2d(c, d_pos.get(), h_names));
+    CSV_TRY(h2d(c, d_off.get(), name_off));
+    launch_csv_names(dbuf, d_pos.get(), d_off.get(), nd, d_txt.get(), S);
+    CSV_TRY(d2h(c, h_text, d_txt.get(), name_off[nd]));
+    if ((st = sync(c)) != SIEVE_OK) return fail(st);
+  }
   t->K = nd ? (u32)nd : 1;
   t->names.resize(nd);
   for (u64 d = 0; d < nd; d++) {
     std::string s;
-    const char* q = hbuf + h_names[2 * d];
+    const char* q = dev_text ? (const char*)h_text.data() + name_off[d] : hbuf + h_names[2 * d];
     for (u64 i = 0; i < h_names[2 * d + 1]; i++) if (q[i] != '"') s.push_back(q[i]);
     t->names[d] = s;
   }

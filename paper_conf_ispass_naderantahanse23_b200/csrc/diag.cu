@@ -7,7 +7,7 @@
 #include "kernels.cuh"
 
 #define GM_THREADS 1024
-#define GM_KT 2048
+#define GM_KT 4608   // strata per shared-memory pass: 48 B each, 216 KB (C4's 3240 strata in one pass)
 #define GM_LB 15
 #define GM_LMASK ((1u << GM_LB) - 1u)
 #define GM_FLUSH ((1u << (32 - GM_LB)) - 1u)
@@ -36,9 +36,16 @@ k_group_moments(const u32* __restrict__ sid, const u64* __restrict__ y, u64 n, u
   bool bad = false;
   for (u64 c0 = b; c0 < e; c0 += GM_FLUSH) {
     u64 c1 = c0 + GM_FLUSH < e ? c0 + GM_FLUSH : e;
-    for (u64 i = c0 + threadIdx.x; i < c1; i += blockDim.x) {
-      u32 l = __ldcs(sid + i) - k0;
-      u64 v = __ldcs(y + i);
+    // software pipelined: the next row's (stratum, cycles) load while this row is added
+    u64 i = c0 + threadIdx.x;
+    u32 nl = i < c1 ? __ldcs(sid + i) : 0u;
+    u64 nv = i < c1 ? __ldcs(y + i) : 0ull;
+    for (; i < c1; i += blockDim.x) {
+      const u32 l = nl - k0;
+      const u64 v = nv;
+      const u64 i2 = i + blockDim.x;
+      nl = i2 < c1 ? __ldcs(sid + i2) : 0u;
+      nv = i2 < c1 ? __ldcs(y + i2) : 0ull;
       if (v >> 48) { bad = true; continue; }
       if (l >= kt) continue;
       atomicAdd(&s_w[l], 1u);

@@ -259,6 +259,9 @@ void launch_csv_firsts(const u32* flag, const u32* seg, const u32* row, u64 n, u
 void launch_csv_ids(const u32* order, u64 nd, u32* id_of, const u32* flag, const u32* seg,
                     const u32* row, u64 n, u32* kid, cudaStream_t s);
 void launch_gather_pairs(const u64* src, const u64* idx, u64 n, u64* dst, cudaStream_t s);
+// names of the distinct kernels: text[pos[2d], +pos[2d+1]) -> out[off[d] ...]
+void launch_csv_names(const unsigned char* buf, const u64* pos, const u64* off, u64 nd, unsigned char* out,
+                      cudaStream_t s);
 
 // ---------------- exact min-strata DP (NEXT-3) --------------------------------------------------
 void launch_rle(const u64* keys, const u32* flag, const u32* seg, u64 n, u32 bx, u64* ukey,

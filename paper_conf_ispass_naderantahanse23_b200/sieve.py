@@ -358,9 +358,13 @@ def load_csv(ctx, data, col_kernel, col_instr, col_cta=-1, col_cycles=-1, header
     keep = None
     if isinstance(data, str):
         data = data.encode()
-    if isinstance(data, (bytes, bytearray)):
-        keep = ctypes.create_string_buffer(bytes(data), len(data))
-        ptr, nbytes, mem = ctypes.cast(keep, ctypes.c_void_p), len(data), MEM_HOST
+    if isinstance(data, bytes):   # the bytes object's own buffer (no copy); kept alive below
+        keep = data
+        ptr, nbytes, mem = ctypes.cast(ctypes.c_char_p(data), ctypes.c_void_p), len(data), MEM_HOST
+    elif isinstance(data, bytearray):
+        keep = (ctypes.c_char * len(data)).from_buffer(data) if len(data) else None
+        ptr = ctypes.cast(keep, ctypes.c_void_p) if keep is not None else ctypes.c_void_p(None)
+        nbytes, mem = len(data), MEM_HOST
     else:
         import torch
         if not (isinstance(data, torch.Tensor) and data.is_cuda and data.dtype == torch.uint8):
