@@ -716,7 +716,21 @@ static int sync(sieve_ctx c) {
 // an open Tier-3 segment: global value range / moments (replicated) and this rank's index
 // range [b, e) in the sorted keys (local)
 // rounds > 1: its values are [b, e) of `src` (sorted cell keys, x = key >> src_shift)
-struct OpenSeg { u32 kid, t3rank; u64 lo, hi, n; u128 s1, s2; u64 b, e; const u64* src; u32 src_shift; };
+struct OpenSeg { u32 kid, t3rank; u64 lo, hi, n; u128 s1, s2; u64 b, e; const u64* src; u32 src_shift;
+                 int node = -1; };
+
+// The refinement tree of a theta sweep (sieve_stratify_sweep): every segment refined at the
+// smallest theta of the sweep, with its parts.  Whether a part is final depends on theta only
+// through its exact CoV test (lo == hi or CoV < theta), and a segment's KDE, cuts and parts
+// depend only on its values, so for theta >= theta_min the strata are the frontier of this tree
+// where the CoV test first holds: the refinement runs once, not once per theta.
+struct SweepTree {
+  struct Seg { u32 kid, round; u64 lo, hi, n; u128 s1, s2; double h; u32 p0, p1; };
+  struct Part { u64 lo, hi, n; u128 s1, s2; int child; };   // child: segment index, -1 if final
+  std::vector<Seg> segs;
+  std::vector<Part> parts;
+  std::vector<int> root;   // per kernel: its Tier-3 root segment, -1
+};
 
 // host-side wall-clock marks (SIEVE_HOST_TIMING=1 prints them to stderr): where the host
 // orchestration, not the device, spends time
@@ -849,7 +863,8 @@ static int moments_finish(sieve_ctx c, MomentsHost* M) {
 }
 
 static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out, sieve_strata_s* R,
-                         const MomentsHost* cached) {
+                         const MomentsHost* cached, SweepTree* rec = nullptr,
+                         const SweepTree* use = nullptr) {
   sieve_ctx c = t->ctx;
   cudaStream_t S = c->stream;
   const auto t_entry = std::chrono::steady_clock::now();
@@ -923,15 +938,52 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       fin.push_back({k, 1, lo, hi, nk, s1, 0.0, 0});
     } else if (cov_lt(nk, s1, s2, P->theta_num, P->theta_den)) { // Tier-2
       fin.push_back({k, 2, lo, hi, nk, s1, 0.0, 0});
+    } else if (use) {                                            // Tier-3: the sweep's tree
+      if (use->root[k] < 0) return sv_fail(SIEVE_ESTATE, "internal: sweep tree lacks a kernel");
     } else {                                                     // Tier-3 -> refinement
       t3rank[k] = n_t3++;
       // the sorted keys are grouped by t3rank: this kernel's local range follows the previous
       open.push_back({k, t3rank[k], lo, hi, nk, s1, s2, n3_local, n3_local + h_localn[k], nullptr, 0});
       n3_local += h_localn[k];
+      if (rec) {
+        open.back().node = (int)rec->segs.size();
+        rec->root[k] = open.back().node;
+        rec->segs.push_back({k, 1, lo, hi, nk, s1, s2, 0.0, 0, 0});
+      }
     }
   }
   R->total_instr = I;
   const u32 n12 = (u32)fin.size();   // the Tier-1/2 strata, in kernel order
+  std::vector<std::pair<u64, u32>> t3s;   // Tier-3 strata keys kid << 44 | lo, index in fin
+  u32 use_rounds = 0;
+  if (use) {
+    // the frontier of the tree at this theta: a part whose CoV test holds (or lo == hi) is a
+    // stratum, any other part was re-opened at theta_min too and its children are visited
+    std::vector<int> stack;
+    for (u32 k = 0; k < K; k++) {
+      const u64* L = &h_lanes[(size_t)k * MOM_LANES];
+      if (!L[0] || h_mm[2 * k] == h_mm[2 * k + 1]) continue;
+      if (cov_lt(L[0], limbs_u128(L + 1), limbs_u128(L + 5), P->theta_num, P->theta_den)) continue;
+      stack.assign(1, use->root[k]);
+      while (!stack.empty()) {
+        const SweepTree::Seg& g = use->segs[stack.back()];
+        stack.pop_back();
+        use_rounds = std::max(use_rounds, g.round);
+        // parts in descending order on the stack so they are visited by ascending lo
+        for (u32 q = g.p1; q-- > g.p0;) {
+          const SweepTree::Part& pt = use->parts[q];
+          if (pt.lo == pt.hi || cov_lt(pt.n, pt.s1, pt.s2, P->theta_num, P->theta_den)) {
+            t3s.push_back({((u64)k << 44) | pt.lo, (u32)fin.size()});
+            fin.push_back({k, 3, pt.lo, pt.hi, pt.n, pt.s1, g.h, g.round});
+          } else {
+            if (pt.child < 0) return sv_fail(SIEVE_ESTATE, "internal: sweep tree part not refined");
+            stack.push_back(pt.child);
+          }
+        }
+      }
+    }
+    std::sort(t3s.begin(), t3s.end());
+  }
 
   // ---------------- Tier-3 values: compaction (unless queued behind pass A) --------------------
   const u32 bx = std::max<u32>(1, bitlen(max_x));
@@ -995,7 +1047,6 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   // The Tier-3 strata are also kept sorted by (kernel, lo) as they arrive -- key kid << 44 | lo
   // (x < 2^44, K <= 2^16) with their index in fin -- so the stratum order costs one merge at
   // the end.
-  std::vector<std::pair<u64, u32>> t3s;
   auto take_finals = [&]() {
     const size_t mid = t3s.size();
     for (const DeferredFin& d : dfin)
@@ -1277,6 +1328,19 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     if (hrec[0] != nparts) return sv_fail(SIEVE_ESTATE, "internal: part count mismatch");
     hc.mark("rec");
     nbatch++;
+    if (rec) {   // the sweep's tree: this batch's segments' bandwidths, parts and re-opened children
+      for (u32 q = 0; q < nseg; q++) {
+        SweepTree::Seg& g = rec->segs[op[q].node];
+        g.h = hh[q];
+        g.p0 = (u32)rec->parts.size();
+        for (u32 p = part_off[q]; p < part_off[q + 1]; p++) {
+          const u64* L = hrec + 1 + (size_t)p * PART_REC;
+          if (!L[0]) continue;
+          rec->parts.push_back({L[MOM_LANES], L[MOM_LANES + 1], L[0], limbs_u128(L + 1), limbs_u128(L + 5), -1});
+        }
+        g.p1 = (u32)rec->parts.size();
+      }
+    }
     {
       DeferredFin d;
       d.rec = hrec;
@@ -1310,9 +1374,19 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         const u64* L = hrec + 1 + (size_t)p * PART_REC;  // {lanes[9], min, max, ia, ib, final}
         // empty parts are dropped (A13 f); final parts go to the strata later (take_finals);
         // a re-opened part's values are [ia, ib) of this batch's grouped values
-        if (L[0] && !L[MOM_LANES + 4])
+        if (L[0] && !L[MOM_LANES + 4]) {
           next.push_back({op[s].kid, op[s].t3rank, L[MOM_LANES], L[MOM_LANES + 1], L[0], limbs_u128(L + 1),
                           limbs_u128(L + 5), L[MOM_LANES + 2], L[MOM_LANES + 3], ck.get(), vsh});
+          if (rec) {   // the re-opened part's segment node (its part record is the p-th non-empty)
+            const int node = (int)rec->segs.size();
+            next.back().node = node;
+            rec->segs.push_back({op[s].kid, round + 1, L[MOM_LANES], L[MOM_LANES + 1], L[0], limbs_u128(L + 1),
+                                 limbs_u128(L + 5), 0.0, 0, 0});
+            u32 pi = rec->segs[op[s].node].p0;
+            for (u32 p2 = part_off[s]; p2 < p; p2++) pi += hrec[1 + (size_t)p2 * PART_REC] != 0;
+            rec->parts[pi].child = node;
+          }
+        }
       }
     }
     }  // batches
@@ -1320,7 +1394,7 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     hc.mark("round");
   }
   take_finals();   // the last batch's
-  R->rounds = round;
+  R->rounds = use ? use_rounds : round;
   // the KDE term count is read back with the representatives at the end (no extra sync)
   std::vector<unsigned long long> h_terms;
   keys.release();
@@ -1559,14 +1633,14 @@ static int check_params(const sieve_params* p, sieve_params* P) {
 }
 
 static int stratify_one(sieve_trace t, const sieve_params* P, uint32_t* sid_out, sieve_strata* out,
-                        const MomentsHost* cached) {
+                        const MomentsHost* cached, SweepTree* rec = nullptr, const SweepTree* use = nullptr) {
   sieve_ctx c = t->ctx;
   sieve_strata_s* R = new sieve_strata_s();
   R->ctx = c;
   R->G = P->grid_points;
   R->keep_debug = P->keep_debug != 0;
   R->has_cycles = t->y != nullptr;
-  int st = stratify_impl(t, P, sid_out, R, cached);
+  int st = stratify_impl(t, P, sid_out, R, cached, rec, use);
   if (st != SIEVE_OK) {
     cudaStreamSynchronize(c->stream);
     delete R;
@@ -1601,14 +1675,33 @@ extern "C" int sieve_stratify_sweep(sieve_trace t, const sieve_params* p, uint32
   SV_TRY(arena_reset(c));
   MomentsHost M;
   SV_TRY(moments_pass(t, &M));  // pass A once for every theta
-  for (uint32_t i = 0; i < count; i++) {
+  // The refinement runs once, at the smallest theta, recording its tree; every other theta takes
+  // the tree's frontier (SweepTree) and runs only the tiers, the table and pass B.  keep_debug
+  // (every KDE segment of each theta's own refinement) and the SIEVE_SWEEP_SEPARATE test hook
+  // refine every theta separately.
+  const bool tree = count > 1 && !P.keep_debug && !getenv("SIEVE_SWEEP_SEPARATE");
+  uint32_t imin = 0;
+  for (uint32_t i = 1; i < count; i++)   // theta_i < theta_min, exactly
+    if ((u64)theta_num[i] * theta_den[imin] < (u64)theta_num[imin] * theta_den[i]) imin = i;
+  SweepTree T;
+  T.root.assign(t->K, -1);
+  auto run = [&](uint32_t i, SweepTree* rec, const SweepTree* use) {
     P.theta_num = theta_num[i];
     P.theta_den = theta_den[i];
-    int st = stratify_one(t, &P, nullptr, &outs[i], &M);
-    if (st != SIEVE_OK) {
-      for (uint32_t j = 0; j < i; j++) { sieve_strata_free(outs[j]); outs[j] = nullptr; }
-      return st;
-    }
+    return stratify_one(t, &P, nullptr, &outs[i], &M, rec, use);
+  };
+  auto fail = [&](int st) {
+    for (uint32_t j = 0; j < count; j++) { if (outs[j]) sieve_strata_free(outs[j]); outs[j] = nullptr; }
+    return st;
+  };
+  if (tree) {
+    int st = run(imin, &T, nullptr);
+    if (st != SIEVE_OK) return fail(st);
+  }
+  for (uint32_t i = 0; i < count; i++) {
+    if (tree && i == imin) continue;
+    int st = run(i, nullptr, tree ? &T : nullptr);
+    if (st != SIEVE_OK) return fail(st);
   }
   return SIEVE_OK;
 }

@@ -1,5 +1,6 @@
 """NEXT-1: theta studies.  sieve_stratify_sweep must equal independent
-sieve_stratify / oracle runs for every theta (it only shares pass A), and sieve_tier_census must
+sieve_stratify / oracle runs for every theta (it shares pass A, and the refinement tree of the
+smallest theta, whose frontier gives every larger theta's strata), and sieve_tier_census must
 equal the oracle's tiers (Fig. 2 shape)."""
 import numpy as np
 import pytest
@@ -32,6 +33,27 @@ def test_sweep_equals_oracle_per_theta(name):
         p = sieve.predict(st, trace)
         q = o.predict()
         assert abs(p["predicted_cycles"] - q["predicted_cycles"]) <= 1e-9 * q["predicted_cycles"]
+
+
+@pytest.mark.parametrize("G", [64, 1024])
+def test_sweep_tree_equals_separate_refinements(G, monkeypatch):
+    """The sweep refines once, at the smallest theta, and takes each larger theta's strata from
+    that refinement tree; with the thetas unsorted and repeated, every table (and the per-theta
+    round counts) must equal what a separate refinement per theta gives (SIEVE_SWEEP_SEPARATE),
+    and the tree's results must equal separate sieve_stratify calls."""
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr, ctx, trace = _trace("C3", n=600_000)
+    thetas = [(1, 2), (1, 10), (3, 10), (1, 10), (2, 5), (1, 1), (7, 10), (1, 20)]
+    tree = sieve.stratify_sweep(trace, thetas, grid_points=G)
+    monkeypatch.setenv("SIEVE_SWEEP_SEPARATE", "1")
+    sep = sieve.stratify_sweep(trace, thetas, grid_points=G)
+    monkeypatch.delenv("SIEVE_SWEEP_SEPARATE")
+    for th, a, b in zip(thetas, tree, sep):
+        assert_tables_equal(a.table, b.table)
+        assert a.rounds == b.rounds, th
+    for th in [(1, 10), (1, 1)]:
+        one = sieve.stratify(trace, theta=th, grid_points=G)
+        assert_tables_equal(tree[thetas.index(th)].table, one.table)
 
 
 def test_census_matches_oracle_tiers():
