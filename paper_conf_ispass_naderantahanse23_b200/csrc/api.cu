@@ -1813,8 +1813,27 @@ extern "C" int sieve_min_strata(sieve_trace t, uint32_t theta_num, uint32_t thet
     SV_TRY(h2d(c, kstart.get() + nk, kend));
     launch_rle(keys.get(), flag.get(), seg.get(), n3, bx, ukey.get(), ustart.get(), kstart.get(), S);
     const u32 cap = max_distinct ? max_distinct : 16384u;
-    launch_min_strata(ukey.get(), ustart.get(), kstart.get(), nk, xmask, theta_num, theta_den, cap,
-                      Pn.get(), P1.get(), P2.get(), f.get(), arg.get(), dcount.get(), dcuts.get(), S);
+    // the DP by layers (dp.cu): layer k assigns f(j) = k; one synchronisation per layer reads how
+    // many kernels still lack f(m) (the layers number the largest optimum, not the values)
+    DBuf<u32> la(c), lb(c), ca(c), cb(c), dstate(c), rem(c);
+    SV_TRY(la.alloc(nu + nk)); SV_TRY(lb.alloc(nu + nk)); SV_TRY(ca.alloc(nk)); SV_TRY(cb.alloc(nk));
+    SV_TRY(dstate.alloc(nk)); SV_TRY(rem.alloc(1));
+    launch_dp_prefix(ukey.get(), ustart.get(), kstart.get(), nk, xmask, theta_num, theta_den, cap, Pn.get(),
+                     P1.get(), P2.get(), f.get(), dcount.get(), la.get(), ca.get(), dstate.get(), S);
+    u32* lst[2] = {la.get(), lb.get()};
+    u32* lct[2] = {ca.get(), cb.get()};
+    for (u32 k = 1;; k++) {
+      if (k > nu + 1) return sv_fail(SIEVE_ESTATE, "internal: min-strata layers did not converge");
+      SV_CUDA(cudaMemsetAsync(rem.get(), 0, 4, S));
+      launch_dp_layer(kstart.get(), nk, (u32)nu, k, theta_num, theta_den, Pn.get(), P1.get(), P2.get(), f.get(),
+                      arg.get(), lst[(k - 1) & 1], lct[(k - 1) & 1], dstate.get(), S);
+      launch_dp_compact(kstart.get(), nk, k, f.get(), arg.get(), ukey.get(), xmask, lst[k & 1], lct[k & 1],
+                        dstate.get(), dcount.get(), dcuts.get(), rem.get(), S);
+      std::vector<u32> h_rem;
+      SV_TRY(d2h(c, h_rem, rem.get(), 1));
+      SV_TRY(sync(c));
+      if (h_rem[0] == 0) break;
+    }
     std::vector<u32> h_count;
     SV_TRY(d2h(c, h_count, dcount.get(), nk));
     SV_TRY(sync(c));

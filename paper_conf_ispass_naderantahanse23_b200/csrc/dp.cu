@@ -3,12 +3,18 @@
 //
 // Per Tier-3 kernel, over its distinct instruction counts (run-length encoded from the sorted
 // Tier-3 keys): f(0) = 0, f(j) = min { f(i) + 1 : CoV(values i+1..j) < theta }, ties -> the
-// smallest i; the backtrack from m gives the canonical optimal cuts.  One 1024-thread block per
-// kernel: block-wide u128 prefix sums of (count, count*v, count*v^2), then the O(m^2) DP with
-// the threads spread over i for every j (one block-wide min per j).  Each (i, j) test is the
-// exact u256 comparison q^2 (n S2 - S1^2) < p^2 S1^2, decided in fp64 when the ratio is
-// further than 1e-12 (relative) from the boundary -- far beyond the fp64 error of the ratio
-// (< 8 ulp), so the decision is always the exact one.
+// smallest i; the backtrack from m gives the canonical optimal cuts.  Each (i, j) test is the
+// exact u256 comparison q^2 (n S2 - S1^2) < p^2 S1^2 on prefix sums of (count, count*v,
+// count*v^2), decided in fp64 when the ratio is further than 1e-12 (relative) from the boundary
+// -- far beyond the fp64 error of the ratio (< 8 ulp), so the decision is always the exact one.
+//
+// B200 mapping: the DP is evaluated by layers, not by j.  Layer k assigns f(j) = k to every j
+// not yet assigned that has a valid run (i, j] from some i of layer k-1 (L_{k-1}), with arg(j) =
+// the smallest such i: by induction exactly the DP's values and tie rule.  A layer is one launch
+// over every kernel's j at once (one thread per j scanning L_{k-1} in ascending order, the
+// lanes of a warp sharing the list), then one block per kernel compacts L_k; the layers stop
+// when every kernel's f(m) is known.  (Round 1 ran the DP by j in one block per kernel, a
+// block-wide minimum per j: 2.0 s for C3's largest kernels against all of the GPU here.)
 #include "kernels.cuh"
 
 #define DP_THREADS 1024
@@ -73,42 +79,23 @@ __device__ __forceinline__ bool run_ok(u64 n, u128 s1, u128 s2, u32 p, u32 q, do
   return lt256(lhs, rhs);
 }
 
-__device__ __forceinline__ u64 block_min_u64(u64 v, u64* red) {
-  for (int o = 16; o > 0; o >>= 1) {
-    u64 w = __shfl_xor_sync(0xffffffffu, v, o);
-    v = w < v ? w : v;
-  }
-  if (lane_id() == 0) red[threadIdx.x >> 5] = v;
-  __syncthreads();
-  if (threadIdx.x < 32) {
-    v = threadIdx.x < (DP_THREADS / 32) ? red[threadIdx.x] : ~0ull;
-    for (int o = 16; o > 0; o >>= 1) {
-      u64 w = __shfl_xor_sync(0xffffffffu, v, o);
-      v = w < v ? w : v;
-    }
-    if (threadIdx.x == 0) red[32] = v;
-  }
-  __syncthreads();
-  u64 r = red[32];
-  return r;
-}
+#define DP_INF 0xFFFFFFFFu
 
 // per Tier-3 rank r: distinct values ukey[kstart[r] .. kstart[r+1]), run starts ustart[] (with
-// ustart[nu] = nkeys).  Scratch at offset kstart[r] + r: prefix arrays of m + 1 entries.
+// ustart[nu] = nkeys).  Arrays indexed at off = kstart[r] + r hold m + 1 entries per kernel:
+// prefix sums, f, arg and the layer lists.  state[r] = 1 while the kernel's f(m) is unknown.
 __global__ void __launch_bounds__(DP_THREADS)
-k_min_strata(const u64* __restrict__ ukey, const u32* __restrict__ ustart, const u32* __restrict__ kstart,
-             u64 xmask, u32 p, u32 q, u32 max_distinct, u64* __restrict__ Pn, u128* __restrict__ P1,
-             u128* __restrict__ P2, u32* __restrict__ f, u32* __restrict__ arg, u32* __restrict__ count,
-             u64* __restrict__ cuts) {
+k_dp_prefix(const u64* __restrict__ ukey, const u32* __restrict__ ustart, const u32* __restrict__ kstart,
+            u64 xmask, u32 p, u32 q, u32 max_distinct, u64* __restrict__ Pn, u128* __restrict__ P1,
+            u128* __restrict__ P2, u32* __restrict__ f, u32* __restrict__ count, u32* __restrict__ list,
+            u32* __restrict__ lcnt, u32* __restrict__ state) {
   pdl_begin();
   __shared__ u64 s_n[DP_THREADS];
   __shared__ u128 s_1[DP_THREADS], s_2[DP_THREADS];
-  __shared__ u64 red[33];
   const u32 r = blockIdx.x;
   const u32 b = kstart[r], m = kstart[r + 1] - b;
   const u64 off = (u64)b + r;
   const double bound = 1.0 + ((double)p * p) / ((double)q * q);
-  // whole kernel valid?  (never for a Tier-3 kernel, but cheap and keeps the kernel general)
   // prefix sums: thread t owns a contiguous chunk
   const u32 T = DP_THREADS, t = threadIdx.x;
   const u32 chunk = (m + T - 1) / T;
@@ -142,43 +129,96 @@ k_min_strata(const u64* __restrict__ ukey, const u32* __restrict__ ustart, const
     l2 += (u128)c * ((u128)v * v);
   }
   if (c1 == m && (c0 < c1 || t == 0)) { Pn[off + m] = ln; P1[off + m] = l1; P2[off + m] = l2; }
-  if (t == 0) f[off] = 0;
+  for (u32 j = t; j <= m; j += T) f[off + j] = j == 0 ? 0u : DP_INF;
   __syncthreads();
-  if (run_ok(Pn[off + m], P1[off + m], P2[off + m], p, q, bound)) {
-    if (t == 0) count[r] = 1;
-    return;
+  if (t != 0) return;
+  if (run_ok(Pn[off + m], P1[off + m], P2[off + m], p, q, bound)) {   // one stratum
+    count[r] = 1;
+    state[r] = 0;
+  } else if (m > max_distinct) {
+    count[r] = 0xFFFFFFFFu;
+    state[r] = 0;
+  } else {
+    list[off] = 0;   // L_0 = {0}
+    lcnt[r] = 1;
+    state[r] = 1;
   }
-  if (m > max_distinct) {
-    if (t == 0) count[r] = 0xFFFFFFFFu;
-    return;
-  }
-  for (u32 j = 1; j <= m; j++) {
+}
+
+// layer k: every unassigned j of a live kernel scans L_{k-1} (ascending) for its first valid run
+__global__ void k_dp_layer(const u32* __restrict__ kstart, u32 nk, u32 nu, u32 k, u32 p, u32 q,
+                           const u64* __restrict__ Pn, const u128* __restrict__ P1,
+                           const u128* __restrict__ P2, u32* __restrict__ f, u32* __restrict__ arg,
+                           const u32* __restrict__ lprev, const u32* __restrict__ lcnt,
+                           const u32* __restrict__ state) {
+  pdl_begin();
+  const double bound = 1.0 + ((double)p * p) / ((double)q * q);
+  for (u32 e = blockIdx.x * blockDim.x + threadIdx.x; e < nu; e += gridDim.x * blockDim.x) {
+    u32 lo = 0, hi = nk - 1;   // kernel of distinct value e: last r with kstart[r] <= e
+    while (lo < hi) {
+      const u32 mid = (lo + hi + 1) >> 1;
+      if (kstart[mid] <= e) lo = mid; else hi = mid - 1;
+    }
+    const u32 r = lo;
+    if (!state[r]) continue;
+    const u64 off = (u64)kstart[r] + r;
+    const u32 j = e - kstart[r] + 1;
+    if (f[off + j] != DP_INF) continue;
     const u64 nj = Pn[off + j];
     const u128 sj1 = P1[off + j], sj2 = P2[off + j];
-    // candidate i = j - 1 (one distinct value) is always valid: an upper bound for pruning
-    const u32 ub = f[off + j - 1] + 1;
-    u64 best = ((u64)ub << 32) | (j - 1);
-    for (u32 i = t; i + 1 < j; i += T) {
-      u32 fi = f[off + i];
-      if (fi + 1 > ub) continue;          // cannot beat (or tie) i = j - 1 with a smaller i
-      u64 key = ((u64)(fi + 1) << 32) | i;
-      if (key >= best) continue;
-      if (run_ok(nj - Pn[off + i], sj1 - P1[off + i], sj2 - P2[off + i], p, q, bound)) best = key;
+    const u32 cnt = lcnt[r];
+    for (u32 x = 0; x < cnt; x++) {
+      const u32 i = lprev[off + x];
+      if (i >= j) break;
+      if (run_ok(nj - Pn[off + i], sj1 - P1[off + i], sj2 - P2[off + i], p, q, bound)) {
+        f[off + j] = k;
+        arg[off + j] = i;
+        break;
+      }
     }
-    best = block_min_u64(best, red);
-    if (t == 0) { f[off + j] = (u32)(best >> 32); arg[off + j] = (u32)best; }
-    __syncthreads();
   }
+}
+
+// one block per live kernel: L_k = { j : f(j) = k } in ascending order; a kernel whose f(m) is
+// known is done (its count and canonical cuts written), else it counts into *remaining
+__global__ void __launch_bounds__(DP_THREADS)
+k_dp_compact(const u32* __restrict__ kstart, u32 k, const u32* __restrict__ f, const u32* __restrict__ arg,
+             const u64* __restrict__ ukey, u64 xmask, u32* __restrict__ lnext, u32* __restrict__ lcnt,
+             u32* __restrict__ state, u32* __restrict__ count, u64* __restrict__ cuts,
+             u32* __restrict__ remaining) {
+  pdl_begin();
+  __shared__ u32 s_c[DP_THREADS];
+  const u32 r = blockIdx.x;
+  if (!state[r]) return;
+  const u32 b = kstart[r], m = kstart[r + 1] - b;
+  const u64 off = (u64)b + r;
+  const u32 T = DP_THREADS, t = threadIdx.x;
+  const u32 chunk = (m + 1 + T - 1) / T;
+  const u32 c0 = min(m + 1, t * chunk), c1 = min(m + 1, c0 + chunk);
+  u32 c = 0;
+  for (u32 j = c0; j < c1; j++) c += f[off + j] == k;
+  s_c[t] = c;
+  __syncthreads();
   if (t == 0) {
-    u32 fm = f[off + m];
-    count[r] = fm;
-    // cuts (lowest value of every stratum but the first), ascending, at cuts[b .. b + fm - 1)
-    u32 j = m, w = fm - 1;
-    while (j > 0) {
-      u32 i = arg[off + j];
-      if (i > 0) cuts[b + (--w)] = ukey[b + i] & xmask;
-      j = i;
-    }
+    u32 a = 0;
+    for (u32 w = 0; w < T; w++) { const u32 x = s_c[w]; s_c[w] = a; a += x; }
+    lcnt[r] = a;
+  }
+  __syncthreads();
+  u32 o = s_c[t];
+  for (u32 j = c0; j < c1; j++)
+    if (f[off + j] == k) lnext[off + o++] = j;
+  if (t != 0) return;
+  const u32 fm = f[off + m];
+  if (fm == DP_INF) { atomicAdd(remaining, 1u); return; }
+  state[r] = 0;
+  count[r] = fm;
+  // cuts (lowest value of every stratum but the first), ascending, at cuts[b .. b + fm - 1)
+  u32 j = m, w = fm - 1;
+  while (j > 0) {
+    const u32 i = arg[off + j];
+    if (i > 0) cuts[b + (--w)] = ukey[b + i] & xmask;
+    j = i;
   }
 }
 
@@ -211,12 +251,26 @@ void launch_rle(const u64* keys, const u32* flag, const u32* seg, u64 n, u32 bx,
   if (n) SV_LAUNCH(k_rle, div_up(n, 256), 256, 0, s)(keys, flag, seg, n, bx, ukey, ustart, kstart);
 }
 
-void launch_min_strata(const u64* ukey, const u32* ustart, const u32* kstart, u32 nk, u64 xmask,
-                       u32 p, u32 q, u32 max_distinct, u64* Pn, u128* P1, u128* P2, u32* f, u32* arg,
-                       u32* count, u64* cuts, cudaStream_t s) {
+void launch_dp_prefix(const u64* ukey, const u32* ustart, const u32* kstart, u32 nk, u64 xmask, u32 p, u32 q,
+                      u32 max_distinct, u64* Pn, u128* P1, u128* P2, u32* f, u32* count, u32* list,
+                      u32* lcnt, u32* state, cudaStream_t s) {
   if (nk)
-    SV_LAUNCH(k_min_strata, nk, DP_THREADS, 0, s)(ukey, ustart, kstart, xmask, p, q, max_distinct,
-                                                  Pn, P1, P2, f, arg, count, cuts);
+    SV_LAUNCH(k_dp_prefix, nk, DP_THREADS, 0, s)(ukey, ustart, kstart, xmask, p, q, max_distinct, Pn, P1, P2,
+                                                 f, count, list, lcnt, state);
+}
+void launch_dp_layer(const u32* kstart, u32 nk, u32 nu, u32 k, u32 p, u32 q, const u64* Pn, const u128* P1,
+                     const u128* P2, u32* f, u32* arg, const u32* lprev, const u32* lcnt, const u32* state,
+                     cudaStream_t s) {
+  if (nk && nu)
+    SV_LAUNCH(k_dp_layer, min(div_up(nu, 256), (u32)sv_num_sms() * 8), 256, 0, s)(
+        kstart, nk, nu, k, p, q, Pn, P1, P2, f, arg, lprev, lcnt, state);
+}
+void launch_dp_compact(const u32* kstart, u32 nk, u32 k, const u32* f, const u32* arg, const u64* ukey,
+                       u64 xmask, u32* lnext, u32* lcnt, u32* state, u32* count, u64* cuts, u32* remaining,
+                       cudaStream_t s) {
+  if (nk)
+    SV_LAUNCH(k_dp_compact, nk, DP_THREADS, 0, s)(kstart, k, f, arg, ukey, xmask, lnext, lcnt, state, count,
+                                                  cuts, remaining);
 }
 
 void launch_dp_gather(const u32* kstart, const u32* count, const u64* off, const u64* cuts, u32 nk,

@@ -266,9 +266,17 @@ void launch_csv_names(const unsigned char* buf, const u64* pos, const u64* off, 
 // ---------------- exact min-strata DP (NEXT-3) --------------------------------------------------
 void launch_rle(const u64* keys, const u32* flag, const u32* seg, u64 n, u32 bx, u64* ukey,
                 u32* ustart, u32* kstart, cudaStream_t s);
-void launch_min_strata(const u64* ukey, const u32* ustart, const u32* kstart, u32 nk, u64 xmask,
-                       u32 p, u32 q, u32 max_distinct, u64* Pn, u128* P1, u128* P2, u32* f, u32* arg,
-                       u32* count, u64* cuts, cudaStream_t s);
+// the min-strata DP by layers (dp.cu): prefix sums and L_0, then per layer k one k_dp_layer and one
+// k_dp_compact (lists ping-pong; *remaining = kernels still without f(m))
+void launch_dp_prefix(const u64* ukey, const u32* ustart, const u32* kstart, u32 nk, u64 xmask, u32 p, u32 q,
+                      u32 max_distinct, u64* Pn, u128* P1, u128* P2, u32* f, u32* count, u32* list,
+                      u32* lcnt, u32* state, cudaStream_t s);
+void launch_dp_layer(const u32* kstart, u32 nk, u32 nu, u32 k, u32 p, u32 q, const u64* Pn, const u128* P1,
+                     const u128* P2, u32* f, u32* arg, const u32* lprev, const u32* lcnt, const u32* state,
+                     cudaStream_t s);
+void launch_dp_compact(const u32* kstart, u32 nk, u32 k, const u32* f, const u32* arg, const u64* ukey,
+                       u64 xmask, u32* lnext, u32* lcnt, u32* state, u32* count, u64* cuts, u32* remaining,
+                       cudaStream_t s);
 void launch_dp_gather(const u32* kstart, const u32* count, const u64* off, const u64* cuts, u32 nk,
                       u64* out, cudaStream_t s);
 
