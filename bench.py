@@ -545,7 +545,7 @@ def main():
     phase_out = {}
     for name, (pms, calls, work) in phases.items():
         e = {"ms_per_step": pms / phase_steps, "calls": calls}
-        if name in ("moments", "compact", "sort", "prefix", "assign") and pms > 0:
+        if name in ("moments", "compact", "sort", "assign") and pms > 0:
             e["GB/s"] = work / (pms / 1000.0) / 1e9
             e["hbm_frac"] = e["GB/s"] / hbm
         phase_out[name] = e

@@ -263,8 +263,8 @@ enum {
   SIEVE_PHASE_MOMENTS = 0, /* pass A: per-kernel moments */
   SIEVE_PHASE_COMPACT = 1, /* Tier-3 key compaction */
   SIEVE_PHASE_SORT = 2,    /* per round: sort of the open segments' values by (segment, grid cell) */
-  SIEVE_PHASE_PREFIX = 3,  /* reserved (0): the former u128 prefix sums */
-  SIEVE_PHASE_KDE = 4,     /* fixed-point KDE (all rounds) */
+  SIEVE_PHASE_KDE_PLAN = 3, /* KDE planning: tile regions, item scan, work-item descriptors */
+  SIEVE_PHASE_KDE = 4,     /* fixed-point KDE kernel (all rounds) */
   SIEVE_PHASE_REFINE = 5,  /* valleys + part moments (all rounds) */
   SIEVE_PHASE_ASSIGN = 6,  /* pass B: assignment + (stratum, CTA) statistics */
   SIEVE_PHASE_REPS = 7,    /* entry compaction, sort, representatives */

@@ -1234,9 +1234,13 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
       // returns while the others enter AR-2 (the local bound is at most the global one)
       if (global_bound >= (1ull << 32)) return sv_fail(SIEVE_ELIMIT, "too many KDE work items");
       u32 items = (u32)items_bound;
-      kde_plan(segs.get(), nseg, G, gtab.get(), off.get(), regions.get(), tile_items.get(), stemp.get(), S);
       DBuf<char> item_tile(c);
       SV_TRY(item_tile.alloc(kde_item_bytes(items)));
+      {
+        PhaseTimer tp(c, SIEVE_PHASE_KDE_PLAN, 0);
+        kde_plan(segs.get(), nseg, G, gtab.get(), off.get(), regions.get(), tile_items.get(), stemp.get(),
+                 item_tile.get(), S);
+      }
       PhaseTimer tm(c, SIEVE_PHASE_KDE, 0);
       // the unguarded KDE variant needs |z| < 4800 for every evaluated pair: window 7.6 h plus
       // KDE_TJ - 1 grid steps plus two boundary cells, so max Delta / h < 140 suffices

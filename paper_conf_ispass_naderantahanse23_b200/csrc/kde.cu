@@ -208,21 +208,6 @@ __global__ void k_kde_tiles(const SegDev* segs, u32 nseg, u32 G, u32 tps, const 
   tile_items[id] = items;
 }
 
-void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
-              void* regions, u32* tile_items, void* scan_temp, cudaStream_t s) {
-  u32 tps = div_up(G, KDE_TJ);
-  u64 nt = (u64)nseg * tps;
-  // SIEVE_KDE_OVH: the per-item cost the plan choice assumes, in terms per lane (A/B and test
-  // hook: 0 = always the finest staircase, "inf" = always one 32-lane region per tile)
-  const char* e = getenv("SIEVE_KDE_OVH");
-  float ovh = e ? (float)atof(e) : KDE_ITEM_OVH;
-  if (!(ovh >= 0.f)) ovh = KDE_ITEM_OVH;
-  SV_LAUNCH(k_kde_tiles, div_up(nt * 8, 256), 256, 0, s)(segs, nseg, G, tps, gtab, off, (KdeRegion*)regions,
-                                                         tile_items, ovh);
-  // exclusive scan in place; tile_items[nt] receives the total (read on the device by k_kde)
-  scan_u32(tile_items, tile_items, nt, scan_temp, tile_items + nt, s);
-}
-
 size_t kde_region_bytes(u64 ntiles) { return (size_t)ntiles * KDE_MAXR * sizeof(KdeRegion); }
 u32 kde_items_per_tile_slack() { return KDE_MAXR - 1; }
 
@@ -291,6 +276,24 @@ __global__ void k_kde_items(const SegDev* __restrict__ segs, u32 G, u32 tps,
       desc[first + k] = d;
     }
   }
+}
+
+void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
+              void* regions, u32* tile_items, void* scan_temp, void* item_desc, cudaStream_t s) {
+  u32 tps = div_up(G, KDE_TJ);
+  u64 nt = (u64)nseg * tps;
+  // SIEVE_KDE_OVH: the per-item cost the plan choice assumes, in terms per lane (A/B and test
+  // hook: 0 = always the finest staircase, "inf" = always one 32-lane region per tile)
+  const char* e = getenv("SIEVE_KDE_OVH");
+  float ovh = e ? (float)atof(e) : KDE_ITEM_OVH;
+  if (!(ovh >= 0.f)) ovh = KDE_ITEM_OVH;
+  SV_LAUNCH(k_kde_tiles, div_up(nt * 8, 256), 256, 0, s)(segs, nseg, G, tps, gtab, off, (KdeRegion*)regions,
+                                                         tile_items, ovh);
+  // exclusive scan in place; tile_items[nt] receives the total (read on the device by k_kde)
+  scan_u32(tile_items, tile_items, nt, scan_temp, tile_items + nt, s);
+  // the work items' descriptors (grids sized by the tiles; the device-side total bounds them)
+  SV_LAUNCH(k_kde_items, (u32)std::min<u64>(div_up(nt, 8), 4096), 256, 0, s)(segs, G, tps, (const KdeRegion*)regions,
+                                                                 tile_items, (u32)nt, (KdeItem*)item_desc);
 }
 
 __device__ __forceinline__ void cp_async8(void* sdst, const void* gsrc) {
@@ -651,9 +654,7 @@ void launch_kde(const SegDev* segs, u32 nseg, u32 G, const u64* vals, u32 vshift
   u32 ntiles = nseg * tps;
   // `items` is a host-side upper bound: grids are sized by it, the kernels stop at the
   // device-side count tile_items[ntiles]
-  KdeItem* desc = (KdeItem*)item_desc;
-  SV_LAUNCH(k_kde_items, min(div_up(ntiles, 8), 4096u), 256, 0, s)(segs, G, tps, (const KdeRegion*)regions, tile_items,
-                                                                     ntiles, desc);
+  KdeItem* desc = (KdeItem*)item_desc;   // written by kde_plan
   // test hook SIEVE_KDE_FORCE: 1 = never the unclamped fast path, 2 = always the guarded
   // variant (all three evaluate identical terms; the parity tests run each)
   const char* force = getenv("SIEVE_KDE_FORCE");

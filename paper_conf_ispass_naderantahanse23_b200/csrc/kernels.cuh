@@ -92,9 +92,11 @@ inline double cell_margin(u64 lo, u64 hi, u32 G) {
 #endif
 // per (segment, tile of KDE_TJ grid points): the bucketed values whose cells meet the tile's
 // window, split into regions by the lanes that need them (regions: kde_region_bytes(tiles)) and
-// chunked into work items; tile_items[nseg * tiles] receives the item total
+// chunked into work items whose descriptors go to item_desc; tile_items[nseg * tiles] receives
+// the item total
 void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32* off,
-              void* regions, u32* tile_items, void* scan_temp, cudaStream_t s);
+              void* regions, u32* tile_items, void* scan_temp, void* item_desc /* kde_item_bytes */,
+              cudaStream_t s);
 size_t kde_region_bytes(u64 ntiles);
 // a tile has at most ceil(tile values / KDE_CH) + kde_items_per_tile_slack() work items
 u32 kde_items_per_tile_slack();

@@ -41,7 +41,7 @@ EXPORTED = [
     "sieve_predict_multi", "sieve_cycle_cov", "sieve_load_csv", "sieve_trace_copy",
     "sieve_trace_kernel_names", "sieve_min_strata",
 ]
-PHASES = ["moments", "compact", "sort", "prefix", "kde", "refine", "assign", "reps", "predict"]
+PHASES = ["moments", "compact", "sort", "kde_plan", "kde", "refine", "assign", "reps", "predict"]
 
 
 class Params(ctypes.Structure):

@@ -16,6 +16,7 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--config", default="C4")
     ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--dump", action="store_true", help="list the last step's kernels and gaps in order")
     a = ap.parse_args()
     import numpy as np
     import torch
@@ -69,6 +70,15 @@ def main():
     print(f"{len(ev)} device events over {per} steps: span {span / 1e3 / per:.3f} ms/step, busy "
           f"{busy / 1e3 / per:.3f} ms/step, idle {(span - busy) / 1e3 / per:.3f} ms/step "
           f"(between the first and the last kernel)")
+    if a.dump:   # the last step: every device event with its start (us from the step's first) and the gap
+        starts = [i for i, e in enumerate(ev) if e.name.startswith("k_moments") and "reduce" not in e.name]
+        first = starts[-1] if starts else 0
+        t0 = ev[first].time_range.start
+        prev_end = ev[first - 1].time_range.end if first else t0
+        for e in ev[first:]:
+            s_, f_ = e.time_range.start, e.time_range.end
+            print(f"{(s_ - t0):9.1f} {(f_ - s_):8.1f} gap {max(0.0, s_ - prev_end):6.1f}  {e.name.split('(')[0][:48]}")
+            prev_end = max(prev_end, f_)
     print("| idle before kernel | us/step | gaps/step |\n|---|---|---|")
     for k, v in sorted(gaps.items(), key=lambda x: -x[1])[:25]:
         print(f"| {k} | {v / per:.1f} | {gap_count[k] / per:.1f} |")
