@@ -43,7 +43,7 @@ def parse():
     ap.add_argument("--impl", default="sieve", choices=["sieve", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-sample", type=int, default=1_000_000)
+    ap.add_argument("--cpu-sample", type=int, default=3_000_000)   # ~14 s of single-threaded oracle
     ap.add_argument("--no-ncu-traffic", action="store_true",
                     help="skip the ncu DRAM-traffic capture that runs before the timed steps")
     ap.add_argument("--ncu-child", action="store_true", help=argparse.SUPPRESS)
