@@ -66,6 +66,45 @@ def test_group_ranks_identical(name, world):
     assert all(p == preds[0] for p in preds)
 
 
+def test_group_sweep_tree_identical():
+    """The theta sweep's refinement tree on a 3-rank group: every rank records the same tree from
+    the replicated part records, so each theta's table equals the single-rank sweep's."""
+    import torch
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr = gen.make_trace("C2", n=300_000)
+    thetas = [(2, 5), (1, 10), (1, 1), (3, 10)]
+    ctx1 = sieve.Ctx(device=0)
+    t1 = sieve.load_trace(ctx1, tr["kid"], tr["x"], num_kernels=tr["K"], cta=tr["cta"], cycles=tr["y"])
+    ref = [s.table.copy() for s in sieve.stratify_sweep(t1, thetas)]
+    world, n = 3, len(tr["kid"])
+    grp = sieve.Group(world)
+    res, errs = [None] * world, []
+
+    def rank_main(r):
+        try:
+            torch.cuda.set_device(0)
+            s = torch.cuda.Stream()
+            ctx = sieve.Ctx(device=0, stream=s, rank=r, group=grp)
+            first, cnt = shard_bounds(n, world, r)
+            sl = slice(first, first + cnt)
+            trace = sieve.load_trace(ctx, tr["kid"][sl], tr["x"][sl], num_kernels=tr["K"],
+                                     cta=tr["cta"][sl], cycles=tr["y"][sl], first_id=first)
+            res[r] = [st.table.copy() for st in sieve.stratify_sweep(trace, thetas)]
+            s.synchronize()
+        except Exception as e:  # pragma: no cover - reported below
+            errs.append((r, repr(e)))
+
+    th = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=600)
+    assert not errs, errs
+    for tables in res:
+        for a, b in zip(tables, ref):
+            assert a.tobytes() == b.tobytes()
+
+
 def test_group_rank_with_empty_slice():
     tr = gen.make_trace("C1")
     tr = {k: (v[:3] if isinstance(v, np.ndarray) else v) for k, v in tr.items()}
