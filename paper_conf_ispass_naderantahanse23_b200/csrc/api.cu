@@ -953,6 +953,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     }
   }
   R->total_instr = I;
+  // the round-1 grouping queued behind pass A was counted as its kernel-id reads (4 B/row); its
+  // Tier-3 rows' x reads and grouped writes (16 B each) are known now
+  if (pre && c->timing) c->acc[SIEVE_PHASE_COMPACT].work += n3_local * 16;
   const u32 n12 = (u32)fin.size();   // the Tier-1/2 strata, in kernel order
   std::vector<std::pair<u64, u32>> t3s;   // Tier-3 strata keys kid << 44 | lo, index in fin
   u32 use_rounds = 0;
