@@ -455,18 +455,9 @@ __device__ __forceinline__ double kde_acc(double gs, double xs, const double* sS
 // in [2^52, 2^53) (a lane adds at most KDE_CH terms of <= 2^40 per item)
 // pair of staged values at a shared-memory byte address (a 128-bit shared load); volatile with a
 // memory clobber so the compiler keeps it behind the staging stores and __syncwarp
-#ifndef KDE_LDS
-#define KDE_LDS 1
-#endif
 __device__ __forceinline__ double2 lds_f64x2(u32 addr) {
   double2 v;
-#if KDE_LDS == 1
   asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(addr) : "memory");
-#elif KDE_LDS == 2
-  asm volatile("ld.shared.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "r"(addr));
-#else
-  v = *(const double2*)__cvta_shared_to_generic(addr);
-#endif
   return v;
 }
 
