@@ -113,30 +113,22 @@ k_csv_ends(const unsigned char* __restrict__ buf, u64 nbytes, const u32* __restr
   }
 }
 
-template <typename Src>
-__device__ __forceinline__ bool parse_u64(Src at, u64 p, u32 len, u64* out) {
-  u64 v = 0;
-  bool any = false;
-  for (u32 i = 0; i < len; i++) {
-    unsigned char ch = at(p + i);
-    if (ch >= '0' && ch <= '9') {
-      const u64 q = ~0ull / 10;  // 1844674407370955161: v * 10 + d fits iff v < q or v == q, d <= 5
-      if (v > q || (v == q && (u32)(ch - '0') > (u32)(~0ull % 10))) return false;
-      v = v * 10 + (ch - '0');
-      any = true;
-    } else if (ch == ',' || ch == '"' || ch == ' ' || ch == '_' || ch == '\r' || ch == '\t') {
-      continue;  // thousands separators, quotes, padding
-    } else {
-      return false;
-    }
-  }
-  *out = v;
-  return any;
+// 64-bit finaliser (murmur3 fmix64): the kernel-name hash mixes eight name bytes at a time
+__device__ __forceinline__ u64 fmix64(u64 k) {
+  k ^= k >> 33;
+  k *= 0xff51afd7ed558ccdull;
+  k ^= k >> 33;
+  k *= 0xc4ceb9fe1a85ec53ull;
+  k ^= k >> 33;
+  return k;
 }
 
-// one thread per data line: fields by a quote-aware walk (ncu: instruction-bound, ALU pipe 71%,
-// issue 86%; staging each block's lines in shared memory first was slower: 0.73 against 0.66 ms
-// for 2M lines)
+// One thread per data line, one pass over its bytes: a quote-aware walk that splits the fields,
+// hashes the kernel-name field (its unquoted bytes, eight at a time) and accumulates the numeric
+// fields as it goes (digits; thousands separators, quotes and padding skipped; anything else, an
+// empty field or a value past 2^64 - 1 is an error).  Bytes come from 4-byte word loads (byte
+// loads near the buffer's end).  Round 1 read every byte with its own load and re-read each
+// numeric field to parse it: 0.66 ms for 2M lines, instruction-bound (ALU 71%, issue 86%).
 #define CSV_PT 128                 // lines (threads) per block
 __global__ void __launch_bounds__(CSV_PT)
 k_csv_parse(const unsigned char* __restrict__ buf, u64 nbytes,
@@ -145,36 +137,66 @@ k_csv_parse(const unsigned char* __restrict__ buf, u64 nbytes,
             u64* __restrict__ name_pos, u64* __restrict__ x, u32* __restrict__ cta,
             u64* __restrict__ y, u64* errflag) {
   pdl_begin();
-  const u64 r0 = (u64)blockIdx.x * CSV_PT;
-  const u64 r = r0 + threadIdx.x;
+  const u64 r = (u64)blockIdx.x * CSV_PT + threadIdx.x;
   if (r >= nrows) return;
-  auto at = [&](u64 i) -> unsigned char { return buf[i]; };
-  u64 line = first_line + r;
-  u64 b = line == 0 ? 0 : ends[line - 1] + 1;
+  const bool words = (((uintptr_t)buf) & 3) == 0;
+  u64 wa = ~0ull;   // address of the cached word
+  u32 w = 0;
+  auto at = [&](u64 i) -> u32 {
+    const u64 a = i & ~3ull;
+    if (words && a + 4 <= nbytes) {
+      if (a != wa) { w = __ldg((const unsigned int*)(buf + a)); wa = a; }
+      return (w >> (8 * (u32)(i & 3))) & 0xFFu;
+    }
+    return buf[i];
+  };
+  const u64 line = first_line + r;
+  const u64 b = line == 0 ? 0 : ends[line - 1] + 1;
   u64 e = line < nends ? ends[line] : nbytes;
   if (e > b && at(e - 1) == '\r') e--;
-  int field = 0;
+  enum { SKIP = 0, NAME = 1, NX = 2, NC = 3, NY = 4 };
+  auto role_of = [&](int f) -> int {
+    return f == spec.col_kernel ? NAME : f == spec.col_instr ? NX : f == spec.col_cta ? NC
+         : f == spec.col_cycles ? NY : SKIP;
+  };
+  int field = 0, role = role_of(0);
   bool inq = false;
-  u64 fs = b;
-  u64 h = 0xcbf29ce484222325ull;
+  u64 h = 0x9e3779b97f4a7c15ull, acc = 0;   // name hash state, pending name bytes
+  u32 nb = 0;                               // name bytes
+  u64 npos = 0, nlen = 0;
+  u64 v = 0;                                // the numeric field being read
+  bool any = false, bad = false;
   u64 vx = 0, vy = 0, vc = 0;
   bool okx = spec.col_instr < 0, oky = spec.col_cycles < 0, okc = spec.col_cta < 0, okn = false;
-  u64 npos = 0, nlen = 0;
+  const u64 q10 = ~0ull / 10;   // v * 10 + d fits iff v < q10, or v == q10 and d <= 5
   for (u64 i = b; i <= e; i++) {
-    unsigned char ch = i < e ? at(i) : (unsigned char)spec.delim;
+    const u32 ch = i < e ? at(i) : (u32)spec.delim;
     if (i < e && ch == '"') { inq = !inq; continue; }
-    if (i < e && (inq || ch != (unsigned char)spec.delim)) {
-      if (field == spec.col_kernel) { h = (h ^ ch) * 0x100000001b3ull; if (!nlen) npos = i; nlen = i - npos + 1; }
+    if (i < e && (inq || ch != (u32)spec.delim)) {
+      if (role == NAME) {
+        acc |= (u64)ch << (8 * (nb & 7));
+        if ((++nb & 7) == 0) { h = fmix64(h ^ acc); acc = 0; }
+        if (!nlen) npos = i;
+        nlen = i - npos + 1;
+      } else if (role != SKIP) {
+        if (ch >= '0' && ch <= '9') {
+          const u32 d = ch - '0';
+          if (v > q10 || (v == q10 && d > (u32)(~0ull % 10))) bad = true;
+          v = v * 10 + d;
+          any = true;
+        } else if (!(ch == ',' || ch == ' ' || ch == '_' || ch == '\r' || ch == '\t')) {
+          bad = true;
+        }
+      }
       continue;
     }
-    // end of field [fs, i)
-    u32 len = (u32)(i - fs);
-    if (field == spec.col_kernel) okn = true;
-    if (field == spec.col_instr) okx = parse_u64(at, fs, len, &vx);
-    if (field == spec.col_cycles) oky = parse_u64(at, fs, len, &vy);
-    if (field == spec.col_cta) { okc = parse_u64(at, fs, len, &vc) && vc <= 0xFFFFFFFFull; }
-    field++;
-    fs = i + 1;
+    // end of field
+    if (role == NAME) { okn = true; h = fmix64(h ^ acc ^ ((u64)nb << 56)); }
+    else if (role == NX) { okx = any && !bad; vx = v; }
+    else if (role == NY) { oky = any && !bad; vy = v; }
+    else if (role == NC) { okc = any && !bad && v <= 0xFFFFFFFFull; vc = v; }
+    role = role_of(++field);
+    v = 0; any = false; bad = false;
   }
   if (!(okx && oky && okc && okn)) atomicMax((unsigned long long*)errflag, 1ull);
   hash[r] = h;
