@@ -273,18 +273,19 @@ static void launch_assign_v(const u32* kid, const u64* x, const u32* cta, u64 n,
 }
 
 // Variant choice: the slot front with a small hash behind it (2 slots per stratum, a 2,048-entry
-// hash) when it fits in AS_SLOT_BUDGET of shared memory, else the 8,192-entry hash alone (A/B
+// hash, or 1,024 / 512 entries when that is what fits) in AS_SLOT_BUDGET of shared memory, else
+// the 8,192-entry hash alone (A/B
 // on C4: slots + 512 / 1,024 / 2,048 / 4,096 hash entries 0.49 ms each; four slots per stratum
 // 0.67 ms -- the 16-byte key reads and the stride-4 atomics conflict; the hash alone 0.57 ms, on
 // C5 9.35 ms).  Without the hash behind them, slots that overflow send rows to contended L2
 // atomics (C5, five CTA sizes per stratum: 87 ms).  Test hook SIEVE_ASSIGN: "hash" forces the
 // hash alone, "4" four slots per stratum.
 #ifndef AS_SLOT_BUDGET
-#define AS_SLOT_BUDGET (176 * 1024)
+#define AS_SLOT_BUDGET (220 * 1024)
 #endif
 #ifndef AS_SLOT_HASH
-#define AS_SLOT_HASH 2048
-#endif
+#define AS_SLOT_HASH 2048   // the hash behind the slots: this size, or the largest of 1,024 / 512
+#endif                      // that fits the budget (C5's 5,566 strata: 1,024 entries, 9.37 -> 6.95 ms)
 void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 first_id,
                    const KTab* ktab, const u64* lows, u32 K, u32 nlows, u32 ns, u32* sid_out, GHash gh,
                    u64* errflags, int grid, cudaStream_t s) {
@@ -301,11 +302,13 @@ void launch_assign(const u32* kid, const u64* x, const u32* cta, u64 n, u64 firs
                                errflags, grid, s);
       return;
     }
-    if (!w4 && assign_smem(2, ns, AS_SLOT_HASH, true, K, nlows) <= AS_SLOT_BUDGET) {
-      launch_assign_v<true, 2>(kid, x, cta, n, first_id, ktab, lows, K, nlows, ns, AS_SLOT_HASH, sid_out, gh,
-                               errflags, grid, s);
-      return;
-    }
+    if (!w4)
+      for (u32 hc = AS_SLOT_HASH; hc >= 512; hc >>= 1)
+        if (assign_smem(2, ns, hc, true, K, nlows) <= AS_SLOT_BUDGET) {
+          launch_assign_v<true, 2>(kid, x, cta, n, first_id, ktab, lows, K, nlows, ns, hc, sid_out, gh,
+                                   errflags, grid, s);
+          return;
+        }
   }
   if (tab <= AS_TAB_BUDGET)
     launch_assign_v<true, 0>(kid, x, cta, n, first_id, ktab, lows, K, nlows, ns, AS_HC, sid_out, gh, errflags,
