@@ -227,53 +227,87 @@ struct __align__(16) KdeItem {
 };
 static_assert(sizeof(KdeItem) == 48, "KdeItem is copied as three 16-byte pieces");
 
-// tile -> its items' descriptors: one warp per tile (no search: the tile's first item is its
-// scanned item count); lane i writes items i, i + 32, ... of the tile, finding each one's region
-// from the regions' item counts (at most KDE_MAXR, read once per lane)
+// item -> descriptor.  Each warp takes a run of consecutive items of the global item space
+// (about one run per warp, at most KDE_IT_RUN items, so a large tile's items spread over many
+// warps: C5 has tiles of ~1e5 items, which one warp per tile wrote in ~1 ms), finds the tile of
+// its first item by a binary search over the scanned counts and walks forward per lane; a lane
+// reloads its tile's regions only when its tile changes.  The warp's 32 descriptors of a step
+// are staged in shared memory and written as contiguous 16-byte chunks.
+#define KDE_IT_RUN 1024
 __global__ void k_kde_items(const SegDev* __restrict__ segs, u32 G, u32 tps,
                             const KdeRegion* __restrict__ regions, const u32* __restrict__ tile_items,
                             u32 ntiles, KdeItem* __restrict__ desc) {
   pdl_begin();
+  __shared__ __align__(16) KdeItem s_it[8][32];   // blockDim.x = 256
   const u32 lane = lane_id();
-  const u32 warps = gridDim.x * (blockDim.x >> 5);
-  for (u32 tile = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); tile < ntiles; tile += warps) {
-    const u32 first = tile_items[tile], n = tile_items[tile + 1] - first;
-    if (n == 0) continue;
-    const u32 s = tile / tps, t = tile % tps;
-    const KdeRegion* rg = regions + (u64)tile * KDE_MAXR;
+  const u32 nwarp = gridDim.x * (blockDim.x >> 5);
+  KdeItem* const st = s_it[threadIdx.x >> 5];
+  const u32 total = tile_items[ntiles];
+  // runs of a multiple of 32 items, about one per warp (at most KDE_IT_RUN: a larger count
+  // takes several passes)
+  const u32 run = min((u32)KDE_IT_RUN, max(32u, ((total + nwarp - 1) / nwarp + 31) & ~31u));
+  for (u64 base = (u64)(blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * run; base < total;
+       base += (u64)nwarp * run) {
+    const u32 end = (u32)min((u64)total, base + run);
+    // the tile of item `base`: the last tile whose first item is <= base
+    u32 lo = 0, hi = ntiles - 1;
+    while (lo < hi) {
+      const u32 m = (lo + hi + 1) >> 1;
+      if (tile_items[m] <= (u32)base) lo = m; else hi = m - 1;
+    }
+    u32 tile = lo, loaded = 0xFFFFFFFFu, first = 0, s = 0, t = 0;
     KdeRegion R[KDE_MAXR];
     u32 ni[KDE_MAXR];
+    SegDev g;
+    unsigned char fast = 0;
+    for (u32 k0 = (u32)base; k0 < end; k0 += 32) {
+      const u32 k = k0 + lane;
+      if (k < end) {
+        while (tile_items[tile + 1] <= k) tile++;   // tiles are contiguous in the item space
+        if (tile != loaded) {
+          loaded = tile;
+          first = tile_items[tile];
+          s = tile / tps;
+          t = tile % tps;
+          const KdeRegion* rg = regions + (u64)tile * KDE_MAXR;
 #pragma unroll
-    for (int r = 0; r < KDE_MAXR; r++) {
-      R[r] = rg[r];
-      ni[r] = (R[r].len + KDE_CH - 1) / KDE_CH;
-    }
-    const SegDev g = segs[s];
-    // |z| <= 7.6 (window) + 33 grid steps (31 lanes + the two boundary cells) in units of h
-    const unsigned char fast = (double)(g.hi - g.lo) < 0.33 * g.h * (double)(G - 1);
-    for (u32 k = lane; k < n; k += 32) {
-      u32 q = k, a = 0, len = 0, shape = 0;   // q: the item's chunk inside its region
-      bool found = false;
-#pragma unroll
-      for (int r = 0; r < KDE_MAXR; r++) {      // static selects (no local memory)
-        if (!found) {
-          if (q < ni[r]) { found = true; a = R[r].a; len = R[r].len; shape = R[r].shape; }
-          else q -= ni[r];
+          for (int r = 0; r < KDE_MAXR; r++) {
+            R[r] = rg[r];
+            ni[r] = (R[r].len + KDE_CH - 1) / KDE_CH;
+          }
+          g = segs[s];
+          // |z| <= 7.6 (window) + 33 grid steps (31 lanes + the two boundary cells) in units of h
+          fast = (double)(g.hi - g.lo) < 0.33 * g.h * (double)(G - 1);
         }
+        u32 q = k - first, a = 0, len = 0, shape = 0;   // q: the item's chunk inside its region
+        bool found = false;
+#pragma unroll
+        for (int r = 0; r < KDE_MAXR; r++) {      // static selects (no local memory)
+          if (!found) {
+            if (q < ni[r]) { found = true; a = R[r].a; len = R[r].len; shape = R[r].shape; }
+            else q -= ni[r];
+          }
+        }
+        KdeItem d;
+        d.va = (u64)a + (u64)q * KDE_CH;
+        d.len = min((u32)KDE_CH, len - q * KDE_CH);
+        d.j0 = t * KDE_TJ + (shape & 0xFF);
+        d.lo = g.lo;
+        d.hi = g.hi;
+        d.inv_h = g.inv_h;
+        d.s = s;
+        d.lw = (unsigned char)(shape >> 8);
+        d.live = (unsigned char)min(1u << d.lw, G - d.j0);
+        d.fast = fast;
+        d.pad = 0;
+        st[lane] = d;
       }
-      KdeItem d;
-      d.va = (u64)a + (u64)q * KDE_CH;
-      d.len = min((u32)KDE_CH, len - q * KDE_CH);
-      d.j0 = t * KDE_TJ + (shape & 0xFF);
-      d.lo = g.lo;
-      d.hi = g.hi;
-      d.inv_h = g.inv_h;
-      d.s = s;
-      d.lw = (unsigned char)(shape >> 8);
-      d.live = (unsigned char)min(1u << d.lw, G - d.j0);
-      d.fast = fast;
-      d.pad = 0;
-      desc[first + k] = d;
+      __syncwarp();
+      const u32 nv = min(32u, end - k0) * 3;   // 16-byte chunks of this step
+      const uint4* src = (const uint4*)st;
+      uint4* dst = (uint4*)(desc + k0);
+      for (u32 c = lane; c < nv; c += 32) dst[c] = src[c];
+      __syncwarp();
     }
   }
 }
@@ -292,7 +326,7 @@ void kde_plan(const SegDev* segs, u32 nseg, u32 G, const double* gtab, const u32
   // exclusive scan in place; tile_items[nt] receives the total (read on the device by k_kde)
   scan_u32(tile_items, tile_items, nt, scan_temp, tile_items + nt, s);
   // the work items' descriptors (grids sized by the tiles; the device-side total bounds them)
-  SV_LAUNCH(k_kde_items, (u32)std::min<u64>(div_up(nt, 8), 4096), 256, 0, s)(segs, G, tps, (const KdeRegion*)regions,
+  SV_LAUNCH(k_kde_items, (u32)sv_num_sms() * 8, 256, 0, s)(segs, G, tps, (const KdeRegion*)regions,
                                                                  tile_items, (u32)nt, (KdeItem*)item_desc);
 }
 
