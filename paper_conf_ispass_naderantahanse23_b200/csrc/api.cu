@@ -1158,13 +1158,41 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
         SV_TRY(rcb.add_h2d(d_chunks.get(), chunks));
       }
       SV_TRY(rcb.add_h2d(d_sc.get(), seg_chunk));
+      // a segment of more than WALK_MIN_CHUNKS chunks: the per-cell walk in groups of WALK_GROUP
+      // (parallel over groups; one thread per (segment, cell) would walk thousands of chunks at
+      // C5: 7.5 -> 5.0 ms; C4's largest segments, 76 chunks, keep the single walk)
+      u32 max_sc = 0, wgsz = WALK_GROUP, wmin = WALK_MIN_CHUNKS;
+      if (const char* e = getenv("SIEVE_WALK_GROUP")) {   // test hook: smaller groups, always
+        wgsz = std::max(1, atoi(e));
+        wmin = wgsz;
+      }
+      for (u32 q = 0; q < nseg; q++) max_sc = std::max(max_sc, seg_chunk[q + 1] - seg_chunk[q]);
+      DBuf<uint2> d_grp(c);
+      DBuf<u32> d_sg(c), d_gs(c);
+      WalkGroups wg{nullptr, nullptr, 0, nullptr};
+      if (max_sc > wmin) {
+        std::vector<uint2> grp;
+        std::vector<u32> sg(nseg + 1);
+        for (u32 q = 0; q < nseg; q++) {
+          sg[q] = (u32)grp.size();
+          for (u32 k = seg_chunk[q]; k < seg_chunk[q + 1]; k += wgsz)
+            grp.push_back(make_uint2(k, std::min<u32>(k + wgsz, seg_chunk[q + 1])));
+        }
+        sg[nseg] = (u32)grp.size();
+        SV_TRY(d_grp.alloc(std::max<size_t>(grp.size(), 1)));
+        SV_TRY(d_sg.alloc(nseg + 1));
+        SV_TRY(d_gs.alloc(std::max<size_t>(grp.size(), 1) * G));
+        if (!grp.empty()) SV_TRY(rcb.add_h2d(d_grp.get(), grp));
+        SV_TRY(rcb.add_h2d(d_sg.get(), sg));
+        wg = WalkGroups{d_grp.get(), d_sg.get(), (u32)grp.size(), d_gs.get()};
+      }
       SV_TRY(rcb.flush());
       hc.mark("up");
       PhaseTimer tm(c, SIEVE_PHASE_SORT, nin * 36 + (u64)nch * G * 16);
       launch_grid_tab(segs.get(), nseg, G, gtab.get(), S);
       launch_cell_group(d_chunks.get(), nch, src, segs.get(), nseg, G, d_sc.get(), cells.get(), hist.get(),
                         rel.get(), tot.get(), off.get(), stemp.get(), ck.get(),
-                        c->count_terms ? terms.get() : nullptr, S);
+                        c->count_terms ? terms.get() : nullptr, S, wg.ngrp ? &wg : nullptr);
       SV_CUDA(cudaGetLastError());
       if (late_h) {  // the bandwidths, while the grouping runs; the KDE reads them from this copy
         for (u32 s = 0; s < nseg; s++) set_h(s);

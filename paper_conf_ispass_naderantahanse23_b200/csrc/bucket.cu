@@ -682,6 +682,63 @@ __global__ void k_cell_walk(const u32* __restrict__ seg_chunk, u32 nseg, u32 G, 
   tot[id] = run;
 }
 
+// The walk for segments of many chunks, in three parallel steps over groups of <= WALK_GROUP
+// chunks (grp[g] = {first chunk, end chunk}, segment s owns groups seg_grp[s] .. seg_grp[s+1]):
+// per (group, cell) the group's count; per (segment, cell) the groups' exclusive prefix (in
+// place) and the cell total; per (group, cell) the chunks' offsets from the group's prefix.
+__global__ void k_walk_gsum(const uint2* __restrict__ grp, u32 ngrp, u32 G, const u32* __restrict__ hist,
+                            u32* __restrict__ gs) {
+  pdl_begin();
+  const u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (id >= (u64)ngrp * G) return;
+  const u32 g = (u32)(id / G), c = (u32)(id % G);
+  const uint2 r = grp[g];
+  u32 sum = 0, k = r.x;
+  for (; k + 8 <= r.y; k += 8) {
+    u32 h[8];
+#pragma unroll
+    for (int j = 0; j < 8; j++) h[j] = hist[(u64)(k + j) * G + c];
+#pragma unroll
+    for (int j = 0; j < 8; j++) sum += h[j];
+  }
+  for (; k < r.y; k++) sum += hist[(u64)k * G + c];
+  gs[id] = sum;
+}
+__global__ void k_walk_gscan(const u32* __restrict__ seg_grp, u32 nseg, u32 G, u32* __restrict__ gs,
+                             u32* __restrict__ tot) {
+  pdl_begin();
+  const u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (id >= (u64)nseg * G) return;
+  const u32 s = (u32)(id / G), c = (u32)(id % G);
+  u32 run = 0;
+  for (u32 g = seg_grp[s]; g < seg_grp[s + 1]; g++) {
+    const u32 v = gs[(u64)g * G + c];
+    gs[(u64)g * G + c] = run;
+    run += v;
+  }
+  tot[id] = run;
+}
+__global__ void k_walk_rel(const uint2* __restrict__ grp, u32 ngrp, u32 G, const u32* __restrict__ hist,
+                           const u32* __restrict__ gs, u32* __restrict__ rel) {
+  pdl_begin();
+  const u64 id = (u64)blockIdx.x * blockDim.x + threadIdx.x;
+  if (id >= (u64)ngrp * G) return;
+  const u32 g = (u32)(id / G), c = (u32)(id % G);
+  const uint2 r = grp[g];
+  u32 run = gs[id], k = r.x;
+  for (; k + 8 <= r.y; k += 8) {
+    u32 h[8];
+#pragma unroll
+    for (int j = 0; j < 8; j++) h[j] = hist[(u64)(k + j) * G + c];
+#pragma unroll
+    for (int j = 0; j < 8; j++) { rel[(u64)(k + j) * G + c] = run; run += h[j]; }
+  }
+  for (; k < r.y; k++) {
+    rel[(u64)k * G + c] = run;
+    run += hist[(u64)k * G + c];
+  }
+}
+
 // exclusive prefix of v over a GR_THREADS block; *total receives the block sum
 __device__ __forceinline__ u32 block_excl_scan_u32(u32 v, u32* total) {
   __shared__ u32 s_w[GR_THREADS / 32];
@@ -772,14 +829,22 @@ size_t cell_scatter_smem(u32 G) { return (size_t)GR_CH * 10 + (size_t)G * 12; }
 
 void launch_cell_group(const BucketChunk* chunks, u32 nchunks, const u64* src, const SegDev* segs, u32 nseg,
                        u32 G, const u32* seg_chunk, unsigned short* cells, u32* hist, u32* rel, u32* tot,
-                       u32* off, void* scan_temp, u64* out, unsigned long long* inwin, cudaStream_t s) {
+                       u32* off, void* scan_temp, u64* out, unsigned long long* inwin, cudaStream_t s,
+                       const WalkGroups* wg) {
   const u64 ncell = (u64)nseg * G;
   if (nchunks) {
     const size_t hs = (size_t)(G + 1) / 2 * 4;
     sv_smem_attr(k_cell_hist, (int)hs);
     SV_LAUNCH(k_cell_hist, nchunks, GR_THREADS, hs, s)(chunks, src, segs, G, cells, hist, inwin);
   }
-  SV_LAUNCH(k_cell_walk, div_up(ncell, 256), 256, 0, s)(seg_chunk, nseg, G, hist, rel, tot);
+  if (wg && wg->ngrp) {
+    const u64 ng = (u64)wg->ngrp * G;
+    SV_LAUNCH(k_walk_gsum, div_up(ng, 256), 256, 0, s)(wg->grp, wg->ngrp, G, hist, wg->gs);
+    SV_LAUNCH(k_walk_gscan, div_up(ncell, 256), 256, 0, s)(wg->seg_grp, nseg, G, wg->gs, tot);
+    SV_LAUNCH(k_walk_rel, div_up(ng, 256), 256, 0, s)(wg->grp, wg->ngrp, G, hist, wg->gs, rel);
+  } else {
+    SV_LAUNCH(k_cell_walk, div_up(ncell, 256), 256, 0, s)(seg_chunk, nseg, G, hist, rel, tot);
+  }
   scan_u32(tot, off, ncell, scan_temp, off + ncell, s);
   if (nchunks) {
     const size_t ss = cell_scatter_smem(G);

@@ -168,9 +168,16 @@ void launch_tiers(const u64* lanes, const u64* mm, const u64* local_n, u32 K, u3
 // off[s * G + c] = first position of cell c of segment s, off[nseg * G] = values grouped
 // (values outside their segment's [lo, hi] are dropped); cells [nchunks * GROUP_CH], hist / rel
 // [nchunks * G], tot [nseg * G] scratch; *inwin += in-window KDE terms (nullable)
+// segments of many chunks walk in groups of <= WALK_GROUP chunks (nullable: one thread per
+// (segment, cell) walks all its chunks): grp[g] = {first, end chunk}, seg_grp[nseg + 1] the
+// segments' group ranges, gs [ngrp * G] scratch
+#define WALK_GROUP 64
+#define WALK_MIN_CHUNKS 256   // the groups only when some segment has more chunks than this
+struct WalkGroups { const uint2* grp; const u32* seg_grp; u32 ngrp; u32* gs; };
 void launch_cell_group(const BucketChunk* chunks, u32 nchunks, const u64* src, const SegDev* segs, u32 nseg,
                        u32 G, const u32* seg_chunk, unsigned short* cells, u32* hist, u32* rel, u32* tot,
-                       u32* off, void* scan_temp, u64* out, unsigned long long* inwin, cudaStream_t s);
+                       u32* off, void* scan_temp, u64* out, unsigned long long* inwin, cudaStream_t s,
+                       const WalkGroups* wg = nullptr);
 
 // ---------------- valleys and thresholds (A11-A13) ---------------------------------------------
 // T[s*tstride + q], nt[s], kind[s] (1 = valley, 2 = bisect)

@@ -60,6 +60,21 @@ def test_grid_sizes(G, ovh, monkeypatch):
     assert_segments_equal(g["segments"], o.segments())
 
 
+@pytest.mark.parametrize("group", ["1", "2", "5"])
+def test_cell_walk_in_groups(group, monkeypatch):
+    """Segments of many value chunks run the cell grouping's per-cell walk in groups of chunks
+    (per-group counts, their prefix per segment, then the offsets inside each group); the test
+    hook SIEVE_WALK_GROUP forces tiny groups on a C3 slice, whose densities, cuts and strata must
+    equal the oracle's."""
+    monkeypatch.setenv("SIEVE_WALK_GROUP", group)
+    tr = gen.make_trace("C3", n=300_000)
+    g = run_gpu(tr, keep_debug=True)
+    o = run_oracle(tr, keep_debug=True)
+    assert_tables_equal(g["table"], o.strata)
+    assert np.array_equal(g["sid"], o.sid)
+    assert_segments_equal(g["segments"], o.segments())
+
+
 @pytest.mark.parametrize("G,radix", [(1024, True), (10000, False)])
 def test_cell_radix_path(G, radix, monkeypatch):
     """the onesweep cell-key path (forced by SIEVE_CELL_RADIX, and taken for G > GROUP_MAXG) gives
