@@ -365,18 +365,9 @@ void launch_part_stats(const SegDev* segs, u32 nseg, u32 G, const double* gtab, 
 
 // the round's results in one record per live part, written straight into mapped (zero-copy)
 // host memory: out[0] = number of parts, then per part {lanes[9], min, max, ia, ib}
-__global__ void k_part_pack(const u32* __restrict__ part_off, u32 nseg, u32 cap, const u64* __restrict__ lanes,
-                            const u64* __restrict__ mm, const u64* __restrict__ ab, const u32* __restrict__ ntk,
-                            u32 tp, u32 tq, u64* out) {
-  pdl_begin();
-  const u32 nparts = part_off[nseg];
-  u32 p = blockIdx.x * blockDim.x + threadIdx.x;
-  if (p == 0) out[0] = nparts;
-  // per segment: cut count and split kind (after the cap part slots)
-  for (u32 q = p; q < nseg; q += gridDim.x * blockDim.x)
-    out[1 + (u64)cap * PART_REC + q] = (u64)ntk[q] | ((u64)ntk[nseg + q] << 32);
-  if (p >= nparts || p >= cap) return;
-  u64* o = out + 1 + (u64)p * PART_REC;
+__device__ __forceinline__ void fill_part_record(u64* o, u32 p, u32 cap, const u64* __restrict__ lanes,
+                                                      const u64* __restrict__ mm, const u64* __restrict__ ab,
+                                                      u32 tp, u32 tq) {
   for (int k = 0; k < MOM_LANES; k++) o[k] = lanes[(u64)p * MOM_LANES + k];
   o[MOM_LANES] = mm[p];
   o[MOM_LANES + 1] = mm[cap + p];
@@ -392,6 +383,34 @@ __global__ void k_part_pack(const u32* __restrict__ part_off, u32 nseg, u32 cap,
                                  cov_lt(L[0], ((u128)s1hi << 64) | s1lo, ((u128)s2hi << 64) | s2lo, tp, tq));
   o[MOM_LANES + 4] = fin ? 1ull : 0ull;
 }
+
+__global__ void k_part_pack(const u32* __restrict__ part_off, u32 nseg, u32 cap, const u64* __restrict__ lanes,
+                            const u64* __restrict__ mm, const u64* __restrict__ ab, const u32* __restrict__ ntk,
+                            u32 tp, u32 tq, u64* out) {
+  pdl_begin();
+  // the block's records are built in shared memory and written to the mapped host buffer as one
+  // contiguous run of 8-byte words (consecutive threads, consecutive words: the PCIe writes
+  // combine; a thread writing its own 112-byte record sent 8-byte writes 112 bytes apart)
+  __shared__ u64 s_rec[128 * PART_REC];   // blockDim.x = 128
+  const u32 nparts = part_off[nseg];
+  const u32 p0 = blockIdx.x * blockDim.x;
+  u32 p = p0 + threadIdx.x;
+  if (p == 0) out[0] = nparts;
+  // per segment: cut count and split kind (after the cap part slots)
+  for (u32 q = p; q < nseg; q += gridDim.x * blockDim.x)
+    out[1 + (u64)cap * PART_REC + q] = (u64)ntk[q] | ((u64)ntk[nseg + q] << 32);
+  const u32 pend = min(nparts, cap);
+  if (p0 >= pend) return;   // block-uniform
+  if (p < pend) {
+    u64* o = s_rec + threadIdx.x * PART_REC;
+    fill_part_record(o, p, cap, lanes, mm, ab, tp, tq);
+  }
+  __syncthreads();
+  const u32 nw = (min(pend, p0 + blockDim.x) - p0) * PART_REC;
+  u64* dst = out + 1 + (u64)p0 * PART_REC;
+  for (u32 w = threadIdx.x; w < nw; w += blockDim.x) dst[w] = s_rec[w];
+}
+
 
 void launch_part_pack(const u32* part_off, u32 nseg, u32 cap, const u64* lanes, const u64* mm,
                       const u64* ab, const u32* ntk, u32 tp, u32 tq, u64* out, cudaStream_t s) {
