@@ -1069,7 +1069,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   while (!open.empty()) {
     round++;
     if (round > P->max_rounds) return sv_fail(SIEVE_ELIMIT, "Tier-3 refinement exceeded max_rounds");
-    std::vector<OpenSeg> next;
+    static thread_local std::vector<OpenSeg> next_tl;   // capacity kept across rounds and calls
+    std::vector<OpenSeg>& next = next_tl;
+    next.clear();
     const u32 nopen = (u32)open.size();
     u32 batch = grouped ? nopen : (u32)std::min<u64>(nopen, std::min<u64>(max_cells / G, 0xFFFFFFFEull / G));
     if (const char* e = getenv("SIEVE_SEG_BATCH"))  // test hook: force small batches
@@ -1088,8 +1090,12 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
     hc.mark("r0");
     std::vector<SegDev> hs(nseg);
     std::vector<double> hh(nseg);
-    std::vector<BucketChunk> chunks;
-    std::vector<u32> seg_chunk;  // grouped path: first chunk of every segment
+    static thread_local std::vector<BucketChunk> chunks_tl;   // capacity kept across rounds
+    static thread_local std::vector<u32> seg_chunk_tl;
+    std::vector<BucketChunk>& chunks = chunks_tl;
+    std::vector<u32>& seg_chunk = seg_chunk_tl;   // grouped path: first chunk of every segment
+    chunks.clear();
+    seg_chunk.clear();
     u64 maxlen = 0;  // largest segment (local values)
     u64 nsup = 0;    // grouped path: values of the segments' source ranges
     // The bandwidths (a glibc pow each, A8) are needed first by the KDE: on the grouped path
