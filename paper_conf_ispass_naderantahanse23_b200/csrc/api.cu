@@ -921,7 +921,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
 
   hc.mark("passA");
   // ---------------- tiers ---------------------------------------------------------
-  std::vector<Fin> fin;
+  static thread_local std::vector<Fin> fin_tl;
+  std::vector<Fin>& fin = fin_tl;
+  fin.clear();
   std::vector<OpenSeg> open;
   std::vector<u32> t3rank(K, 0xFFFFFFFFu);
   u32 n_t3 = 0;
@@ -957,7 +959,9 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   // Tier-3 rows' x reads and grouped writes (16 B each) are known now
   if (pre && c->timing) c->acc[SIEVE_PHASE_COMPACT].work += n3_local * 16;
   const u32 n12 = (u32)fin.size();   // the Tier-1/2 strata, in kernel order
-  std::vector<std::pair<u64, u32>> t3s;   // Tier-3 strata keys kid << 44 | lo, index in fin
+  static thread_local std::vector<std::pair<u64, u32>> t3s_tl;
+  std::vector<std::pair<u64, u32>>& t3s = t3s_tl;   // Tier-3 strata keys kid << 44 | lo, index in fin
+  t3s.clear();
   u32 use_rounds = 0;
   if (use) {
     // the frontier of the tree at this theta: a part whose CoV test holds (or lo == hi) is a
@@ -1450,10 +1454,19 @@ static int stratify_impl(sieve_trace t, const sieve_params* P, uint32_t* sid_out
   std::vector<u32>& order = order_tl;
   order.resize(ns);
   auto F = [&](u32 s) -> const Fin& { return fin[order[s]]; };
-  std::vector<KTab> ktab(K, KTab{0, 0, 0, 0});
-  std::vector<u64> lows;
-  std::vector<u32> tiers(ns);
-  std::vector<u64> hW(2 * (size_t)ns);
+  // the call's host tables keep their capacity across calls (no allocation or first-touch page
+  // faults between the last round's synchronisation and pass B's launch)
+  static thread_local std::vector<KTab> ktab_tl;
+  static thread_local std::vector<u64> lows_tl, hW_tl;
+  static thread_local std::vector<u32> tiers_tl;
+  std::vector<KTab>& ktab = ktab_tl;
+  std::vector<u64>& lows = lows_tl;
+  std::vector<u32>& tiers = tiers_tl;
+  std::vector<u64>& hW = hW_tl;
+  ktab.assign(K, KTab{0, 0, 0, 0});
+  lows.clear();
+  tiers.resize(ns);
+  hW.resize(2 * (size_t)ns);
   {
     u32 i = 0, s = 0;
     size_t j = 0;
