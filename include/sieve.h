@@ -203,10 +203,16 @@ void sieve_strata_free(sieve_strata s);
 /* ---- theta studies (Fig. 2, Fig. 10) -------------------- */
 
 /* Stratify for `count` thresholds theta_i = theta_num[i] / theta_den[i] (host arrays) in one
-   call: the per-kernel moments (pass A and its reduction) are computed once and reused; each
-   theta then runs tiering, the Tier-3 refinement and the assignment.  outs[i] receives the
-   strata for theta_i (free each with sieve_strata_free); on error none is returned.
-   Other fields of *p (grid, valley shift, ...) apply to every theta.  Collective if world > 1. */
+   call: the per-kernel moments (pass A and its reduction) are computed once and reused; the
+   Tier-3 refinement runs once, at the smallest theta, recording its tree of segments and parts,
+   and every other theta takes the tree's frontier (a part is a stratum at theta where lo == hi
+   or its exact CoV < theta first holds: a segment's KDE, cuts and parts depend only on its
+   values), then runs tiering and the assignment.  Every table equals a separate
+   sieve_stratify at that theta; kde_terms / kde_evaluated (sieve_strata_stats) are counted on
+   the smallest theta's result only (the others run no KDE).  With keep_debug each theta refines
+   separately.  outs[i] receives the strata for theta_i (free each with sieve_strata_free); on
+   error none is returned.  Other fields of *p (grid, valley shift, ...) apply to every theta.
+   Collective if world > 1. */
 int sieve_stratify_sweep(sieve_trace t, const sieve_params* p, uint32_t count,
                          const uint32_t* theta_num, const uint32_t* theta_den, sieve_strata* outs);
 
