@@ -95,12 +95,13 @@ def test_predict_multi_architecture():
     assert preds[0]["predicted_cycles"] == single["predicted_cycles"]
 
 
-@pytest.mark.parametrize("name", ["C1", "C2"])
+@pytest.mark.parametrize("name", ["C1", "C2", "manyK"])
 def test_cycle_cov_matches_oracle(name):
-    """Fig. 4 diagnostic: per-stratum cycle CoV bit-identical to the oracle."""
+    """Fig. 4 diagnostic: per-stratum cycle CoV bit-identical to the oracle.  manyK:
+    9,000 kernels, 8,742 strata: two shared-memory passes of the per-stratum table (4,608 each)."""
     import paper_conf_ispass_naderantahanse23_b200 as sieve
     from tests.gpu_helpers import run_gpu
-    tr = gen.make_trace(name)
+    tr = gen.make_trace("C2", K=9000, n=800_000) if name == "manyK" else gen.make_trace(name)
     g = run_gpu(tr)
     import torch
     sid = torch.from_numpy(g["sid"].view(np.int32)).cuda()
