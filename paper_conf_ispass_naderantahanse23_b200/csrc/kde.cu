@@ -243,6 +243,9 @@ __global__ void k_kde_items(const SegDev* __restrict__ segs, u32 G, u32 tps,
   const u32 nwarp = gridDim.x * (blockDim.x >> 5);
   KdeItem* const st = s_it[threadIdx.x >> 5];
   const u32 total = tile_items[ntiles];
+  // the KDE's tail-item counter sits right after the last descriptor (the buffer has 16 spare
+  // bytes: kde_item_bytes)
+  if (blockIdx.x == 0 && threadIdx.x == 0) *(u32*)(desc + total) = 0;
   // runs of a multiple of 32 items, about one per warp (at most KDE_IT_RUN: a larger count
   // takes several passes)
   const u32 run = min((u32)KDE_IT_RUN, max(32u, ((total + nwarp - 1) / nwarp + 31) & ~31u));
@@ -429,6 +432,9 @@ struct KdeRegs { double log2e, magic; u32 lane8; };  // operands that must sit i
 // half-integer: with p, s the odd significands of P and S, P*S = p*s*2^(a+b) has fraction 1/2
 // only if a + b = -1, which needs >= 12 trailing zero bits in T_j' (A10 sets T_0 = 1 - 2^-53; the
 // other entries have <= 6, pinned in tests), so the sum is exact in any order.
+#ifndef KDE_TAIL
+#define KDE_TAIL 8           // the last items / KDE_TAIL are claimed dynamically (A/B on C4: 4 / 8 / 16: 6.185 / 6.181 / 6.186 ms against 6.30 all round-robin; 0 = off)
+#endif
 #ifndef KDE_SPLIT
 #define KDE_SPLIT 1          // 1: lane-replicated 256-entry table + exponent arithmetic (below)
 #endif
@@ -539,6 +545,18 @@ __device__ __forceinline__ u64 kde_run_sum(double gs, u32 sa, u32 len, const dou
 // runs (slice l div 2^lw); slices are summed with shuffles.  Whole-warp items (lw = 5) are the
 // tile's core, narrower ones the staircase at the ends of its window (k_kde_tiles).
 //
+#if KDE_TAIL
+// the warp's next item from the tail counter (lane 0 claims, the warp shares it); kept out of line
+// so the claim does not enter the register allocation of the term loop
+__device__ __noinline__ u32 kde_claim_tail(const KdeItem* desc, u32 items) {
+  const u32 S = items - items / KDE_TAIL;
+  u32 c = 0;
+  if (lane_id() == 0) c = atomicAdd((u32*)(desc + items), 1u);
+  c = __shfl_sync(0xffffffffu, c, 0);
+  return S + c < items ? S + c : items;
+}
+#endif
+
 template <bool GUARD>
 __global__ void __launch_bounds__(32 * KDE_WARPS, KDE_MINB)
 k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
@@ -569,6 +587,14 @@ k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
   const u32 W = gridDim.x * KDE_WARPS;
   u32 it = blockIdx.x * KDE_WARPS + (threadIdx.x >> 5);
   if (it >= items) return;
+#if KDE_TAIL
+  // a warp whose first round-robin item lies in the claimed tail claims its first item instead
+  // (every tail item is handed out exactly once, by the counter)
+  if (it >= items - items / KDE_TAIL) {
+    it = kde_claim_tail(desc, items);
+    if (it >= items) return;
+  }
+#endif
   unsigned char* wsm = smem + KDE_SMEM_TABLE + (threadIdx.x >> 5) * KDE_WARP_BYTES;
   double* const buf0 = (double*)wsm;   // value buffers buf0 + b * KDE_CH, b = 0, 1
   KdeItem* sd = (KdeItem*)(wsm + 2 * KDE_CH * 8);
@@ -598,7 +624,20 @@ k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
   cp_async_wait_all();
   __syncwarp();
   fetch_vals(sd, buf0);
+#if KDE_TAIL
+  // Items below S = items - items / KDE_TAIL are dealt round-robin; the last items / KDE_TAIL are
+  // claimed from a counter (desc + items, zeroed by k_kde_items), so the SMs that drew cheaper
+  // items take more of the tail and finish with the others.
+  auto next_of = [&](u32 cur_it) -> u32 {   // the item after cur_it for this warp
+    if (cur_it >= items) return items;
+    if (cur_it + W < items - items / KDE_TAIL) return cur_it + W;
+    return kde_claim_tail(desc, items);
+  };
+  u32 nx1 = next_of(it);
+  if (nx1 < items) fetch_desc(nx1, sd + 1);
+#else
   if (it + W < items) fetch_desc(it + W, sd + 1);
+#endif
   cp_async_commit();
   u32 cur = 0, b = 0;   // ring slot of the current descriptor, current value buffer
   for (;;) {
@@ -606,11 +645,21 @@ k_kde(const KdeItem* __restrict__ desc, const u32* __restrict__ n_items, u32 G,
     __syncwarp();
     const KdeItem* cd = sd + cur;
     const u32 nxt = cur == 2 ? 0 : cur + 1, nn = nxt == 2 ? 0 : nxt + 1;
+#if KDE_TAIL
+    const u32 it1 = nx1;
+    const u32 it2 = next_of(it1);
+    if (it1 < items) {
+      fetch_vals(sd + nxt, buf0 + (b ^ 1) * KDE_CH);
+      if (it2 < items) fetch_desc(it2, sd + nn);
+    }
+    nx1 = it2;
+#else
     const u32 it1 = it + W;
     if (it1 < items) {
       fetch_vals(sd + nxt, buf0 + (b ^ 1) * KDE_CH);
       if (it1 + W < items) fetch_desc(it1 + W, sd + nn);
     }
+#endif
     cp_async_commit();
     double* sx = buf0 + b * KDE_CH;
     const u32 len = cd->len;
