@@ -17,8 +17,8 @@
 // pipe (no contraction, so no tensor cores).  Work item = (segment, tile of 32 grid points,
 // region of the tile's window |g - x| <= 7.6 h, chunk of <= KDE_CH = 512 values); a region is
 // evaluated by the lanes whose windows meet it (32, 16 or 8 lanes with 1, 2 or 4 value slices:
-// the staircase of k_kde_tiles); items are dealt to warps round-robin and staged by a per-warp
-// cp.async pipeline (see k_kde); each lane owns one grid point and reads the staged values as
+// the staircase of k_kde_tiles); items are dealt to warps round-robin, the last 1/8 claimed from
+// a counter as warps finish, and staged by a per-warp cp.async pipeline (see k_kde); each lane owns one grid point and reads the staged values as
 // shared-memory broadcasts.  The term is arranged to be
 // bit-identical to the oracle's while issuing 9 FP64-pipe instructions and ~6 others:
 //   * xs (per value, at staging) and gs (per lane, per item) are the A10 scaled coordinates,
