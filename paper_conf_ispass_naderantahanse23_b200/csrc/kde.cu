@@ -545,6 +545,13 @@ __device__ __forceinline__ u64 kde_run_sum(double gs, u32 sa, u32 len, const dou
 // runs (slice l div 2^lw); slices are summed with shuffles.  Whole-warp items (lw = 5) are the
 // tile's core, narrower ones the staircase at the ends of its window (k_kde_tiles).
 //
+// Items are dealt to warps round-robin (item w, w + W, w + 2W, ...; W warps in the grid) up to the
+// last items / KDE_TAIL, which warps claim from a counter as they run out (so the SMs finish
+// together); every warp knows its next two items, and a three-stage cp.async pipeline keeps all
+// global latency off the FP64 pipe: while item k is evaluated, the values of item k + 1 and the
+// descriptor of item k + 2 are in flight.  Densities are accumulated with fire-and-forget
+// reductions of two limbs (low 32 bits, the rest) into D[2j], D[2j + 1]; k_valleys turns them
+// into the u128 D_j.
 #if KDE_TAIL
 // the warp's next item from the tail counter (lane 0 claims, the warp shares it); kept out of line
 // so the claim does not enter the register allocation of the term loop
