@@ -46,8 +46,10 @@
 #define KDE_MINB 1           // resident blocks per SM: one 64 KB table shared by the block
 #endif
 #ifndef KDE_UNROLL
-#define KDE_UNROLL 14        // terms in flight per lane (A/B on C4 after the two-instruction table
-#endif                       // step: 14 -> 6.36 ms, 16 -> 6.61, 12 -> 6.45, 8 -> 6.46, 15 -> 6.85)
+#define KDE_UNROLL 10         // terms in flight per lane (A/B on C4 with the claimed tail: 10 / 12 / 14 / 8
+                             // -> 6.01 / 6.11 / 6.19 / 6.22 ms: at 10 and 12 ptxas keeps the accumulators
+                             // in place, at 14 it adds five register moves per step; C5 74.0 -> 71.9)
+#endif
 static_assert(KDE_CH % 32 == 0, "each lane stages KDE_CH / 32 values of an item");
 static_assert(KDE_TJ == 32, "a tile is one grid point per lane; narrower shapes are per region");
 #define KDE_MAXR 7           // regions per tile (at most 2 * 4 - 1 elementary cell intervals)
