@@ -300,8 +300,8 @@ k_part_stats(const u64* __restrict__ ab, const u32* __restrict__ item_off, u32 c
     const u64 i0 = ab[4 * (u64)p + 2] + (u64)(item - item_off[p]) * PS_CH;
     const u64 i1 = min(i0 + PS_CH, ab[4 * (u64)p + 3]);
     u64 n = 0, s1lo = 0, s1hi = 0, s2lo = 0, s2hi = 0, mn = ~0ull, mx = 0;
-    for (u64 i = i0 + threadIdx.x; i < i1; i += PS_THREADS) {
-      u64 x = vals[i] >> vshift;
+    auto take = [&](u64 x) {
+      x >>= vshift;
       if (x >= a && x < b) {
         n++;
         add128(s1lo, s1hi, x, 0);
@@ -309,7 +309,17 @@ k_part_stats(const u64* __restrict__ ab, const u32* __restrict__ item_off, u32 c
         mn = x < mn ? x : mn;
         mx = x > mx ? x : mx;
       }
+    };
+    // eight values per thread loaded before they are added (one memory latency per eight)
+    u64 i = i0 + threadIdx.x;
+    for (; i + 7 * PS_THREADS < i1; i += 8 * PS_THREADS) {
+      u64 v[8];
+#pragma unroll
+      for (int k = 0; k < 8; k++) v[k] = vals[i + (u64)k * PS_THREADS];
+#pragma unroll
+      for (int k = 0; k < 8; k++) take(v[k]);
     }
+    for (; i < i1; i += PS_THREADS) take(vals[i]);
     for (int o = 16; o > 0; o >>= 1) {
       n += __shfl_down_sync(0xffffffffu, n, o);
       u64 al = __shfl_down_sync(0xffffffffu, s1lo, o), ah = __shfl_down_sync(0xffffffffu, s1hi, o);
