@@ -56,6 +56,20 @@ def test_sweep_tree_equals_separate_refinements(G, monkeypatch):
         assert_tables_equal(tree[thetas.index(th)].table, one.table)
 
 
+def test_sweep_degenerate_theta_lists():
+    """A sweep of one theta (no tree), of one theta repeated (the tree and its own root), and of
+    an empty list."""
+    import paper_conf_ispass_naderantahanse23_b200 as sieve
+    tr, ctx, trace = _trace("C2", n=200_000)
+    one = sieve.stratify(trace, theta=(2, 5))
+    for thetas in ([(2, 5)], [(2, 5), (2, 5), (4, 10)]):
+        outs = sieve.stratify_sweep(trace, thetas)
+        assert len(outs) == len(thetas)
+        for st in outs:
+            assert_tables_equal(st.table, one.table)
+    assert sieve.stratify_sweep(trace, []) == []
+
+
 def test_census_matches_oracle_tiers():
     import paper_conf_ispass_naderantahanse23_b200 as sieve
     tr, ctx, trace = _trace("C2")
